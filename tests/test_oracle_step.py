@@ -1,0 +1,298 @@
+"""Pins for the oracle's DGI step (Eqs. 1-6; readings c5-c11, c13-c15).
+
+Fixed by closed forms, special cases reducing to textbook linear algebra,
+central finite differences, an independent PyTorch float64 autograd
+formulation, and a hand-derived worked example (tests/golden/dgi_2node.json).
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth import graphs as SG
+from tests.util import scaled_err, split_params
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+LN2 = math.log(2.0)
+
+
+def _sig(x):
+    return 1.0 / (1.0 + math.exp(-x))
+
+
+def _softplus(x):
+    return max(x, 0.0) + math.log1p(math.exp(-abs(x)))
+
+
+def _tiny_batch(idx=0, G=1):
+    return oracle.Batch([SG.tiny(idx + g) for g in range(G)])
+
+
+def _brute_anorm(N, indptr, indices):
+    A = np.eye(N)
+    for u in range(N):
+        for e in range(indptr[u], indptr[u + 1]):
+            v = int(indices[e])
+            if u != v:
+                A[u, v] = A[v, u] = 1.0
+    d = A.sum(1)
+    return A / np.sqrt(np.outer(d, d))
+
+
+def test_golden_two_node_example():
+    with open(os.path.join(GOLDEN, "dgi_2node.json")) as f:
+        gold = json.load(f)
+
+    class Gr:
+        num_nodes = gold["N"]
+        indptr = np.array(gold["indptr"], np.int64)
+        indices = np.array(gold["indices"], np.int32)
+        features = np.array(gold["X"], np.float32)
+    b = oracle.Batch([Gr()])
+    pp = gold["params"]
+    params = np.array(pp["W1"] + pp["W2"] + pp["W3"] + pp["M"] + pp["alpha"], np.float64)
+    loss, grads, s, acts = oracle.step_grads(b, 1, params, np.array(gold["perm"], np.int32))
+    sg = _sig(0.5)
+    l = sg / 2
+    assert np.allclose(acts["Z3"], 0.5, rtol=0, atol=1e-15)
+    assert abs(s[0, 0] - sg) < 1e-15
+    assert abs(loss - 0.5 * (_softplus(-l) + _softplus(l))) < 1e-15
+    dv = (2 * _sig(l) - 1) / 4
+    assert abs(grads[3] - dv * sg) < 1e-15          # dM (H = 1: params [W1 W2 W3 M a1 a2 a3])
+
+
+def test_csr_mode_equals_dense_mode():
+    g = SG.tiny(0)
+    b = oracle.Batch([g])
+    F, H = 16, 32
+    params = oracle.xavier(7, F, H).astype(np.float64)
+    perm = oracle.perm(7, 0, 0, g.num_nodes)
+    loss, grads, _, acts = oracle.step_grads(b, H, params, perm)
+    adj = oracle.dense_adjacency(g.num_nodes, g.indptr, g.indices)
+    dloss, dgrads, demb = oracle.dense_step(adj, g.features, perm, params, H)
+    assert abs(loss - dloss) < 1e-13
+    assert scaled_err(grads, dgrads) < 1e-12
+    H3 = np.where(acts["Z3"] > 0, acts["Z3"], params[-1] * acts["Z3"])[: g.num_nodes]
+    assert scaled_err(H3, demb) < 1e-13
+    assert scaled_err(oracle.encode(b, H, params), demb) < 1e-13
+
+
+def test_linear_network_closed_form():
+    """alpha = 1 makes PReLU the identity: H3 = Â_n^3 X W1 W2 W3 (textbook product)."""
+    g = SG.tiny(3)
+    F, H = 16, 32
+    p = oracle.xavier(3, F, H).astype(np.float64)
+    p[-3:] = 1.0
+    P = split_params(p, F, H)
+    An = _brute_anorm(g.num_nodes, g.indptr, g.indices)
+    X = g.features.astype(np.float64)
+    want = An @ An @ An @ X @ P["W1"].reshape(F, H) @ P["W2"].reshape(H, H) @ P["W3"].reshape(H, H)
+    got = oracle.encode(oracle.Batch([g]), H, p)
+    assert scaled_err(got, want) < 1e-13
+
+
+def test_zero_weights_give_zero_embeddings_and_ln2():
+    b = _tiny_batch()
+    F, H = 16, 32
+    p = oracle.xavier(1, F, H).astype(np.float64)
+    n = F * H + 2 * H * H
+    p[:n] = 0.0                                     # all W_l = 0, any M
+    loss, grads, s, acts = oracle.step_grads(b, H, p, b.perms(1, 0, 0))
+    assert np.all(acts["Z3"] == 0.0)
+    assert abs(loss - LN2) < 1e-15
+    assert np.all(grads == 0.0)                     # a saddle: every gradient vanishes
+    assert np.allclose(s, 0.5)
+
+
+def test_M_zero_gives_ln2_and_closed_form_dM():
+    """M = 0: v = 0, every score is 0, L = ln 2, dW = dalpha = 0 and
+    dM = 1/4 (mean H~3 - mean H3) s^T."""
+    b = _tiny_batch()
+    F, H = 16, 32
+    p = oracle.xavier(2, F, H).astype(np.float64)
+    P = split_params(p, F, H)
+    P["M"][:] = 0.0
+    loss, grads, s, acts = oracle.step_grads(b, H, p, b.perms(2, 0, 0))
+    assert abs(loss - LN2) < 1e-15
+    G = split_params(grads, F, H)
+    for k in ("W1", "W2", "W3", "alpha"):
+        assert np.all(G[k] == 0.0)
+    a3 = p[-1]
+    H3 = np.where(acts["Z3"] > 0, acts["Z3"], a3 * acts["Z3"])
+    N = b.Nt
+    dv = 0.25 * (H3[N:].mean(0) - H3[:N].mean(0))
+    assert scaled_err(G["M"].reshape(H, H), np.outer(dv, s[0])) < 1e-13
+
+
+def test_identity_permutation_loss_at_least_ln2():
+    b = _tiny_batch()
+    F, H = 16, 32
+    p = oracle.xavier(5, F, H).astype(np.float64)
+    loss, *_ = oracle.step_grads(b, H, p, np.arange(b.Nt, dtype=np.int32))
+    assert loss >= LN2 - 1e-15
+
+
+def _kink_free_params(b, F, H, perm):
+    for seed in range(100):
+        p = oracle.xavier(seed, F, H).astype(np.float64)
+        acts = oracle.forward(b, H, p, perm)
+        if min(np.abs(acts[k]).min() for k in ("Z1", "Z2", "Z3")) > 2e-6:
+            return p
+    pytest.skip("no kink-free init found")
+
+
+def test_finite_differences_all_parameters():
+    """Central differences of the double loss w.r.t. every parameter (h = 1e-7; inits with |Z| <= 2e-6 are rejected so no step crosses a PReLU kink)."""
+    g = SG.tiny(0)
+    b = oracle.Batch([g])
+    F, H = 16, 32
+    perm = oracle.perm(11, 0, 0, g.num_nodes)
+    p = _kink_free_params(b, F, H, perm)
+    p[-3:] = [0.25, 0.1, 0.4]
+    loss, grads, *_ = oracle.step_grads(b, H, p, perm)
+    h = 1e-7
+    fd = np.zeros_like(p)
+    for i in range(p.size):
+        q = p.copy(); q[i] += h
+        lp = oracle.step_grads(b, H, q, perm)[0]
+        q[i] -= 2 * h
+        lm = oracle.step_grads(b, H, q, perm)[0]
+        fd[i] = (lp - lm) / (2 * h)
+    assert scaled_err(grads, fd) < 1e-6
+    roundoff = 50 * np.finfo(np.float64).eps * abs(loss) / h      # FD cancellation floor
+    for name, blk in split_params(grads - fd, F, H).items():
+        ref = split_params(fd, F, H)[name]
+        assert np.max(np.abs(blk)) <= 1e-6 * np.max(np.abs(ref)) + roundoff, name
+
+
+def _torch_dgi(g_list, perms, params, F, H):
+    """Independent formulation: dense Â_n per graph built with torch, PReLU via
+    torch.nn.functional.prelu, BCE via binary_cross_entropy_with_logits; the
+    gradient comes from autograd."""
+    p = torch.tensor(params, dtype=torch.float64, requires_grad=True)
+    o = 0
+    W1 = p[o:o + F * H].view(F, H); o += F * H
+    W2 = p[o:o + H * H].view(H, H); o += H * H
+    W3 = p[o:o + H * H].view(H, H); o += H * H
+    M = p[o:o + H * H].view(H, H); o += H * H
+    al = p[o:o + 3]
+    total = 0.0
+    off = 0
+    for g in g_list:
+        N = g.num_nodes
+        A = torch.zeros(N, N, dtype=torch.float64)
+        for u in range(N):
+            for e in range(g.indptr[u], g.indptr[u + 1]):
+                v = int(g.indices[e])
+                if u != v:
+                    A[u, v] = 1.0; A[v, u] = 1.0
+        A = A + torch.eye(N, dtype=torch.float64)
+        dm = A.sum(1).rsqrt()
+        An = dm[:, None] * A * dm[None, :]
+        X = torch.tensor(g.features, dtype=torch.float64)
+        pi = torch.tensor(perms[off:off + N].astype(np.int64))
+        off += N
+
+        def enc(h):
+            for l, W in enumerate((W1, W2, W3)):
+                h = torch.nn.functional.prelu(An @ h @ W, al[l:l + 1])
+            return h
+        Hp, Hn = enc(X), enc(X[pi])
+        s = torch.sigmoid(Hp.mean(0))
+        lp = Hp @ (M @ s)
+        ln = Hn @ (M @ s)
+        logits = torch.cat([lp, ln])
+        lab = torch.cat([torch.ones(N), torch.zeros(N)]).double()
+        total = total + torch.nn.functional.binary_cross_entropy_with_logits(logits, lab)
+    loss = total / len(g_list)
+    loss.backward()
+    return float(loss), p.grad.numpy()
+
+
+def test_torch_autograd_agrees():
+    gl = [SG.tiny(0), SG.tiny(1)]
+    b = oracle.Batch(gl)
+    F, H = 16, 32
+    p = oracle.xavier(9, F, H).astype(np.float64)
+    perms = b.perms(9, 3, 10)
+    loss, grads, *_ = oracle.step_grads(b, H, p, perms)
+    tl, tg = _torch_dgi(gl, perms, p, F, H)
+    assert abs(loss - tl) < 1e-13
+    assert scaled_err(grads, tg) < 1e-12
+
+
+def test_batch_is_mean_of_separate_runs():
+    gl = [SG.tiny(i) for i in range(3)]
+    F, H = 16, 32
+    p = oracle.xavier(4, F, H).astype(np.float64)
+    b = oracle.Batch(gl)
+    loss, grads, *_ = oracle.step_grads(b, H, p, b.perms(4, 1, 20))
+    ls, gs = [], []
+    for i, g in enumerate(gl):
+        bi = oracle.Batch([g])
+        l_, g_, *_ = oracle.step_grads(bi, H, p, bi.perms(4, 1, 20 + i))
+        ls.append(l_); gs.append(g_)
+    assert abs(loss - np.mean(ls)) < 1e-14
+    assert scaled_err(grads, np.mean(gs, 0)) < 1e-13
+
+
+def test_encode_permutation_equivariance():
+    g = SG.tiny(4)
+    N, F, H = g.num_nodes, 16, 32
+    p = oracle.xavier(6, F, H).astype(np.float64)
+    sig = np.random.default_rng(0).permutation(N)
+    src = np.repeat(np.arange(N), np.diff(g.indptr))
+    s2, d2 = sig[src], sig[g.indices]
+    o = np.argsort(s2, kind="stable")
+    indptr = np.zeros(N + 1, np.int64)
+    np.add.at(indptr, s2 + 1, 1)
+
+    class G2:
+        num_nodes = N
+    G2.indptr = np.cumsum(indptr)
+    G2.indices = d2[o].astype(np.int32)
+    X2 = np.zeros_like(g.features); X2[sig] = g.features
+    G2.features = X2
+    e1 = oracle.encode(oracle.Batch([g]), H, p)
+    e2 = oracle.encode(oracle.Batch([G2]), H, p)
+    assert scaled_err(e2[sig], e1) < 1e-13
+
+
+def test_adam_first_step_closed_form():
+    rng = np.random.default_rng(0)
+    p0 = rng.standard_normal(1000); g = rng.standard_normal(1000)
+    p1, m, v = oracle.adam(p0, np.zeros(1000), np.zeros(1000), g, 1, lr=1e-3)
+    np.testing.assert_allclose(p1, p0 - 1e-3 * g / (np.abs(g) + 1e-8), rtol=0, atol=1e-15)
+
+
+@pytest.mark.parametrize("clip", [0.0, 0.5])
+def test_adam_matches_torch(clip):
+    rng = np.random.default_rng(1)
+    P = 300
+    p = rng.standard_normal(P)
+    tp = torch.tensor(p.copy(), requires_grad=True)
+    opt = torch.optim.Adam([tp], lr=3e-3, betas=(0.9, 0.999), eps=1e-8)
+    m = np.zeros(P); v = np.zeros(P)
+    for t in range(1, 6):
+        g = rng.standard_normal(P)
+        tp.grad = torch.tensor(g.copy())
+        if clip > 0:
+            torch.nn.utils.clip_grad_norm_([tp], clip)
+        opt.step()
+        p, m, v = oracle.adam(p, m, v, g, t, lr=3e-3, clip=clip)
+    assert scaled_err(p, tp.detach().numpy()) < 1e-14
+
+
+def test_xavier_bounds_and_alpha():
+    F, H = 64, 256
+    p = oracle.xavier(0, F, H)
+    P = split_params(p, F, H)
+    b1 = np.float32(math.sqrt(6 / (F + H)))
+    b2 = np.float32(math.sqrt(6 / (2 * H)))
+    assert np.all(np.abs(P["W1"]) <= b1) and np.all(np.abs(P["W2"]) <= b2)
+    assert abs(P["W1"].mean()) < 0.01 and abs(P["M"].std() - b2 / math.sqrt(3)) < 0.005
+    assert np.all(P["alpha"] == np.float32(0.25))
