@@ -1,0 +1,354 @@
+#!/usr/bin/env python
+"""bench.py -- DGI contrastive pre-training throughput on GNMT-shaped op graphs.
+
+Metric (BASELINE.json): "DGI contrastive steps/s on GNMT-shaped op graph; SpMM
+GB/s vs HBM peak".  One bench step = one full pass of the hot path (corruption,
+3 GCN layers on both branches, readout / discriminator / BCE, full backward,
+NCCL gradient allreduce when N > 1, Adam) over a batch of 16 GNMT-shaped op
+graphs per GPU (one (graph, sample) pair each, weak scaling).  `value` counts
+per-graph DGI steps per second over the whole job (N x 16 x K / time).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU, NCCL)
+
+Device time: CUDA events on the stream the library launches on (torch's
+current stream, handed to libmars), barrier + synchronize on both sides, max
+over ranks.  The per-step working set (~2.8 GB of activations) exceeds the
+126 MB L2, so no explicit flush is needed between steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "DGI contrastive steps/s on GNMT-shaped op graph; SpMM GB/s vs HBM peak"
+UNIT = "graph-steps/s"
+F, H = 64, 256
+FFMA_TFLOPS_NOTE = "148 SM x 128 FP32 lanes x 2 flop x 1.965 GHz (B200_PROFILING.md counts)"
+
+
+def peaks():
+    p = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "source": "fallback (B200_PROFILING.md)"}
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            m = json.load(f)
+        p.update(hbm_gbs=float(m["hbm_gbs"]), bf16_tflops=float(m["bf16_tflops"]),
+                 bf16_tflops_sustained=float(m.get("bf16_tflops_sustained", m["bf16_tflops"])),
+                 sm_max_mhz=float(m.get("sm_max_mhz", 1965.0)), source="measured")
+    except Exception:
+        pass
+    p["ffma_tflops"] = 148 * 128 * 2 * p.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+    return p
+
+
+# ------------------------------------------------------------------ clocks sampler
+class Clocks:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as fh:
+            for ln in fh:
+                parts = [x.strip() for x in ln.split(",")]
+                if len(parts) < 9 or not parts[0].isdigit() or int(parts[0]) != self.idx:
+                    continue
+                rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        sm = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        reasons = set()
+        for r in rows:
+            for name, col in (("hw_slowdown", 5), ("hw_thermal_slowdown", 6),
+                              ("sw_thermal_slowdown", 7), ("sw_power_cap", 8)):
+                if r[col].lower().startswith("active"):
+                    reasons.add(name)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": float(rows[0][2]) if rows[0][2].replace(".", "").isdigit() else None,
+                "reasons": sorted(reasons), "samples": len(rows)}
+
+
+# ------------------------------------------------------------------ algorithmic bytes / flops
+def spmm_bytes(N, Z, C, layer1=False, bwd=False, s=4):
+    """Per SpMM launch over the stacked [pos; neg] rows:
+    rowptr + (colind, val) + input rows + output rows (+ perm for layer 1,
+    + Z read for the backward epilogue)."""
+    b = 4 * (N + 1) + 8 * Z + 2 * N * C * s + 2 * N * C * s
+    if layer1:
+        b += 4 * N
+    if bwd:
+        b += 2 * N * C * s
+    return b
+
+
+def step_accounting(N, Z):
+    """Per-step launches of each phase with algorithmic bytes / flops."""
+    R = 2 * N
+    sp = [("spmm_fwd", spmm_bytes(N, Z, F, layer1=True)), ("spmm_fwd", spmm_bytes(N, Z, H)),
+          ("spmm_fwd", spmm_bytes(N, Z, H)), ("spmm_bwd", spmm_bytes(N, Z, H, bwd=True)),
+          ("spmm_bwd", spmm_bytes(N, Z, H, bwd=True))]
+    gemm = {"gemm_fwd": 2 * R * H * (F + H + H), "gemm_dw": 2 * R * H * (F + H + H),
+            "gemm_dy": 2 * R * H * (H + H)}
+    gemm_bytes = {"gemm_fwd": 4 * R * ((F + H) + (H + H) + (H + H)),
+                  "gemm_dw": 4 * R * ((F + H) + (H + H) + (H + H)),
+                  "gemm_dy": 4 * R * ((H + H) + (H + H))}
+    return sp, gemm, gemm_bytes
+
+
+# ------------------------------------------------------------------ arms
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def run_reference(args):
+    """The oracle (fp64, single thread) on the host cores, as it stands."""
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    import oracle
+    from synth import graphs as SG
+    graphs = [SG.cached("gnmt", i) for i in range(args.graphs_per_gpu)]
+    small = min(graphs, key=lambda g: g.num_nodes)
+    tiny = SG.tiny(0)
+    for w in range(args.warmup):                      # untimed (CPU has nothing to warm up)
+        b = oracle.Batch([tiny])
+        oracle.step_grads(b, 32, oracle.xavier(0, 16, 32).astype(np.float64), b.perms(0, w, 0))
+    b = oracle.Batch([small])
+    p = oracle.xavier(0, F, H).astype(np.float64)
+    m = np.zeros_like(p); v = np.zeros_like(p)
+    t0 = time.perf_counter()
+    for k in range(args.steps):
+        loss, grads, _, _ = oracle.step_grads(b, H, p, b.perms(0, k, 0))
+        p, m, v = oracle.adam(p, m, v, grads, k + 1)
+    dt = time.perf_counter() - t0
+    val = args.steps / dt
+    sample = (f"1 GNMT-shaped graph per step (the smallest of the workload's "
+              f"{args.graphs_per_gpu}, N={small.num_nodes}), full DGI step + Adam in fp64")
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * dt / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": f"gnmt x{args.graphs_per_gpu} per GPU (sampled: 1 graph/step)",
+                       "F": F, "H": H},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_mine(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icpp_lancl21_b200 as mars
+    from paper_conf_icpp_lancl21_b200 import dp
+    from synth import graphs as SG
+
+    rank, world, local = dp.env()
+    if world != args.gpus:
+        args.gpus = world
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    b = args.graphs_per_gpu
+    graphs = [SG.cached("gnmt", i) for i in dp.graph_indices(rank, world, b)]
+    uid = dp.broadcast_unique_id(mars.nccl_get_unique_id)
+    g = mars.graph_load(graphs, device=local)
+    info = g.info()
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local, world_size=world,
+                        rank=rank, nccl_unique_id=uid)
+    # a dedicated (non-legacy) stream: libmars launches and captures on it and
+    # torch's CUDA events are recorded on it
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
+    m.set_stream(stream.cuda_stream)
+    base, B = dp.pair_range(rank, world, b)
+    for w in range(args.warmup):
+        m.step(g, w, base, B)
+    torch.cuda.synchronize()
+    phys = local
+    cvd = os.environ.get("CUDA_VISIBLE_DEVICES")
+    if cvd:
+        try:
+            phys = int(cvd.split(",")[local])
+        except Exception:
+            pass
+    clk = Clocks(phys)
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for k in range(args.steps):
+        m.step(g, args.warmup + k, base, B)
+    ev1.record(stream)
+    ev1.synchronize()
+    ms = ev0.elapsed_time(ev1)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = clk.stop()
+    launches = m.last_launches() * args.steps
+    if world > 1:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = world * b * args.steps / (ms / 1000.0)
+
+    # per-phase device time, CUDA events on the launching stream (same kernels, eager)
+    nprof = max(1, min(args.steps, args.profile_steps))
+    acc = {}
+    prof_total = 0.0
+    for k in range(nprof):
+        ph = m.profile_step(g, args.warmup + args.steps + k, base, B)
+        for name, t in ph:
+            acc.setdefault(name, []).append(t)
+        prof_total += sum(t for _, t in ph)
+    per_step = {k: sum(v) / nprof for k, v in acc.items()}
+    N, Z = info["total_nodes"], info["nnz"]
+    sp, gflops, gbytes = step_accounting(N, Z)
+    pk = peaks()
+    spmm_ms = per_step.get("spmm_fwd", 0) + per_step.get("spmm_bwd", 0)
+    spmm_algo = sum(bb for _, bb in sp)
+    spmm_gbs = spmm_algo / (spmm_ms / 1e3) / 1e9 if spmm_ms else None
+    shares = {k: v / sum(per_step.values()) for k, v in per_step.items()}
+    kinds = {"gemm": sum(per_step.get(k, 0) for k in ("gemm_fwd", "gemm_dw", "gemm_dy")),
+             "spmm": spmm_ms}
+    if kinds["gemm"] >= kinds["spmm"]:
+        fl = sum(gflops.values())
+        ach = fl / (kinds["gemm"] / 1e3) / 1e12
+        roof = {"kernel": "gemm (fp32 FFMA: fwd Y·W, dY = dZ·Wᵀ, dW = Yᵀ·dZ)", "bound": "alu",
+                "achieved": ach, "peak": pk["ffma_tflops"], "unit": "TFLOP/s",
+                "frac": ach / pk["ffma_tflops"], "traffic": None,
+                "peak_source": FFMA_TFLOPS_NOTE, "share_of_step": kinds["gemm"] / sum(per_step.values())}
+    else:
+        roof = {"kernel": "spmm (fwd x3 + bwd x2)", "bound": "hbm", "achieved": spmm_gbs,
+                "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": spmm_gbs / pk["hbm_gbs"],
+                "traffic": None, "peak_source": pk["source"],
+                "share_of_step": spmm_ms / sum(per_step.values())}
+    spmm_obj = {"achieved_gbs": spmm_gbs, "peak_gbs": pk["hbm_gbs"],
+                "frac": (spmm_gbs / pk["hbm_gbs"]) if spmm_gbs else None,
+                "algorithmic_bytes_per_step": spmm_algo, "ms_per_step": spmm_ms,
+                "peak_source": pk["source"]}
+
+    # e2e through the public API: H2D of the step's graph batch from host memory,
+    # CSR build, the step, D2H of the loss -- every step
+    e2e = None
+    if not args.no_e2e:
+        h2d = sum(gr.indptr.nbytes + gr.indices.nbytes + gr.features.nbytes for gr in graphs)
+        ke = max(1, min(args.steps, args.e2e_steps))
+        m2 = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local,
+                             world_size=1, rank=0)
+        m2.set_stream(stream.cuda_stream)
+        gg = mars.graph_load(graphs, device=local)          # warm allocator / staging
+        m2.step(gg, 0, base, B, want_loss=True)
+        gg.free()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for k in range(ke):
+            gg = mars.graph_load(graphs, device=local)
+            m2.step(gg, 1 + k, base, B, want_loss=True)
+            gg.free()
+        torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        m2.free()
+        e2e = {"value": b * ke / dt, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": 4, "steps": ke,
+               "note": "per step: mars_graph_load (H2D + CSR build) + mars_dgi_step + loss D2H, "
+                       "wall clock, rank-local (no allreduce)"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        gr0 = graphs[0]
+        bo = oracle.Batch([gr0])
+        p0 = oracle.xavier(args.seed, F, H).astype(np.float64)
+        t0 = time.perf_counter()
+        loss, grads, _, _ = oracle.step_grads(bo, H, p0, bo.perms(args.seed, 0, 0))
+        oracle.adam(p0, np.zeros_like(p0), np.zeros_like(p0), grads, 1)
+        dt = time.perf_counter() - t0
+        cpu = {"value": 1.0 / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"1 of the {b} GNMT-shaped graphs of a step (graph 0, N={gr0.num_nodes}), "
+                         f"full fp64 DGI step + Adam, single thread, {dt:.1f} s"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+                "data": "synthetic",
+                "config": {"workload": f"gnmt x{b} per GPU (GNMT-4 shaped training op graphs, "
+                                       f"T~U[20,50])", "graphs_per_gpu": b, "F": F, "H": H,
+                           "nodes_per_gpu": N, "nnz_per_gpu": Z, "global_batch": B,
+                           "parallelism": f"dp{world}",
+                           "l2": "inputs larger than L2 (activations ~%.1f GB/step)"
+                                 % (2 * N * 4 * (F + 7 * H) / 1e9)},
+                "roofline": roof, "spmm": spmm_obj,
+                "phases_ms_per_step": per_step, "phase_share": shares,
+                "profiled_step_ms": prof_total / nprof,
+                "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches}
+        print(json.dumps(line), flush=True)
+    m.free()
+    g.free()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="mine", choices=["mine", "reference"])
+    ap.add_argument("--graphs-per-gpu", type=int, default=16)
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--profile-steps", type=int, default=5)
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_mine(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,200 @@
+/*
+ * include/mars.h -- C ABI of libmars.so, the B200 (sm_100a) implementation of
+ * the data-parallel hot path of Mars (Lan, Chen & Li, "Accelerated Device
+ * Placement Optimization with Contrastive Learning", ICPP'21): one Deep Graph
+ * Infomax (DGI) pre-training step of the 3-layer GCN operation encoder over a
+ * DNN op graph (§3.1-§3.2, Eqs. 1-6), its backward pass and Adam.
+ *
+ * Citations "P:Lnnn" are lines of the paper text; "c<k>" are the readings of
+ * silent / garbled passages listed in DESIGN.md §3.
+ *
+ * Conventions (all calls):
+ *  - Every call returns mars_status; nothing throws across the ABI.  On a
+ *    non-OK status mars_last_error() returns a thread-local message.
+ *  - Inputs are BORROWED: host arrays are copied during the call and may be
+ *    freed on return.  Output arrays are allocated by the caller (host memory
+ *    unless stated).  Handles belong to the caller until mars_free().
+ *  - Handles are not thread-safe; distinct handles are independent.
+ *  - There is no CPU fallback: with no usable CUDA device every compute call
+ *    returns MARS_ECUDA.
+ *  - Flat parameter layout (H = hidden_dim, F = in_dim, P = F*H + 3*H*H + 3):
+ *      [ W1 (F×H row-major) | W2 (H×H) | W3 (H×H) | M (H×H) | a1 a2 a3 ]
+ *    Z_l = Y_l · W_l, so W_l is C_in×H (Eq. 1's Θ); M is the bilinear matrix of
+ *    Eq. 5 (the paper's "W"); a_l is the PReLU slope of layer l (c6).
+ */
+#ifndef MARS_H_
+#define MARS_H_
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define MARS_API __attribute__((visibility("default")))
+#else
+#define MARS_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  MARS_OK = 0,
+  MARS_EINVAL = 1,      /* invalid argument / malformed graph                    */
+  MARS_ENOMEM = 2,      /* device or host allocation failed                      */
+  MARS_ECUDA = 3,       /* CUDA runtime / driver error, or no device             */
+  MARS_ENCCL = 4,       /* NCCL error (multi-GPU data parallelism)               */
+  MARS_ENUMERIC = 5,    /* non-finite loss detected                              */
+  MARS_ESTATE = 6       /* wrong / freed handle, or call out of order            */
+} mars_status;
+
+typedef enum { MARS_FP32 = 0, MARS_BF16 = 1 } mars_precision;
+
+/* Thread-local text for the last non-OK status of this thread ("" if none). */
+MARS_API const char* mars_last_error(void);
+/* Library version string, e.g. "mars-b200 0.1 sm_100a". */
+MARS_API const char* mars_version(void);
+/* P = F*H + 3*H*H + 3 (the flat layout above). */
+MARS_API int64_t mars_num_params(int32_t in_dim, int32_t hidden_dim);
+
+typedef struct mars_graph mars_graph;   /* device-resident Â_n of 1..G op graphs */
+typedef struct mars_dgi mars_dgi;       /* params, Adam state, workspaces, stream */
+
+/* ------------------------------------------------------------------------ */
+/* a1-a3: ingest op graphs and build Â_n = D̂^-1/2 (A ∨ Aᵀ + I) D̂^-1/2.        */
+/* ------------------------------------------------------------------------ */
+/* One op graph in host memory: N ops, directed data-flow edges
+ * u->v ("v requires the output of u") as a CSR whose row u lists the
+ * consumers v of u, and the per-op feature matrix X (one-hot op type +
+ * normalised input/output shapes).  Duplicate edges and self-loops are
+ * allowed (collapsed / dropped, c2). */
+typedef struct {
+  int32_t num_nodes;          /* N >= 1                                        */
+  const int64_t* indptr;      /* [N+1], indptr[0] = 0, non-decreasing          */
+  const int32_t* indices;     /* [indptr[N]], each in [0, N)                   */
+  int32_t feat_dim;           /* F, identical for every graph of a set         */
+  const float* features;      /* [N*F] row-major fp32                          */
+} mars_graph_desc;
+
+/* Loads G >= 1 graphs as ONE block-diagonal set on `device` and builds, in
+ * device kernels, the symmetrised CSR of Â (colind ascending per row, the
+ * diagonal included), integer degrees d_i = |row i| (c3), dinv_i = f32(1/√d_i)
+ * and vals_ij = f32(1/√(d_i d_j)) computed in double and rounded once (c4).
+ * EINVAL: G < 1, N < 1, malformed indptr, index out of range, F mismatch,
+ * F not in {16, 32, 64, 128, 256}, or ΣN + 2·ΣE >= 2^31.  Immutable. */
+MARS_API mars_status mars_graph_load(const mars_graph_desc* graphs, int32_t num_graphs, int32_t device,
+                            mars_graph** out);
+
+/* Shape queries.  Any output pointer may be NULL. */
+MARS_API mars_status mars_graph_info(const mars_graph* g, int32_t* num_graphs, int64_t* total_nodes,
+                            int64_t* total_nnz, int32_t* feat_dim);
+/* Node count and nnz(Â) of graph `graph_idx` of the set. */
+MARS_API mars_status mars_graph_size(const mars_graph* g, int32_t graph_idx, int32_t* num_nodes,
+                            int64_t* nnz);
+/* Test hook (parity P1): copies graph `graph_idx`'s CSR with LOCAL indices to
+ * host arrays rowptr[N+1], colind[nnz], deg[N], dinv[N], vals[nnz] (any may be
+ * NULL). */
+MARS_API mars_status mars_graph_export_csr(const mars_graph* g, int32_t graph_idx, int32_t* rowptr,
+                                  int32_t* colind, int32_t* deg, float* dinv, float* vals);
+
+/* ------------------------------------------------------------------------ */
+/* The pre-training model: 3 GCN layers with PReLU (Eq. 1),     */
+/* sigmoid-mean readout (Eq. 4), bilinear discriminator (Eq. 5), BCE (Eq. 6), */
+/* Adam (c13).                                                               */
+/* ------------------------------------------------------------------------ */
+typedef struct {
+  int32_t in_dim;             /* F in {16, 32, 64, 128, 256}                    */
+  int32_t hidden_dim;         /* H in {32, 64, 128, 256} (paper: 256)  */
+  int32_t num_layers;         /* L: must be 3 (c10)                     */
+  int32_t precision;          /* mars_precision: MARS_FP32 (reference, c18)     */
+  double lr, beta1, beta2, eps; /* Adam (c13): defaults 1e-3, 0.9, 0.999, 1e-8  */
+  double clip_norm;           /* <= 0: no clipping (default)                    */
+  uint64_t seed;              /* Xavier init (c14) and corruption keys (c12)    */
+  const float* init_params;   /* optional [P] host; NULL => Xavier-uniform(seed) */
+  int32_t device;             /* CUDA device ordinal                           */
+  int32_t world_size, rank;   /* data parallelism; 1, 0 for a single GPU       */
+  const void* nccl_unique_id; /* 128-byte ncclUniqueId when world_size > 1     */
+} mars_dgi_config;
+
+/* Fills cfg with the defaults above (F = 64, H = 256, L = 3, FP32, seed 0,
+ * device 0, world 1). */
+MARS_API void mars_dgi_config_default(mars_dgi_config* cfg);
+/* Allocates params (init per c14 unless init_params), Adam state (m = v = 0,
+ * t = 0) and a library stream on cfg->device; with world_size > 1 joins the
+ * NCCL communicator (ncclCommInitRank; every rank must call collectively). */
+MARS_API mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** out);
+/* Rank 0 only: writes a fresh 128-byte ncclUniqueId to out128. */
+MARS_API mars_status mars_nccl_get_unique_id(void* out128);
+/* Use `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream()) instead
+ * of the library stream.  NULL restores the library stream. */
+MARS_API mars_status mars_dgi_set_stream(mars_dgi* m, void* cuda_stream);
+/* Enables (1) / disables (0) CUDA-Graph capture of the step (default 1). */
+MARS_API mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable);
+
+/* Optional outputs of a step (host pointers; NULL = not requested). */
+typedef struct {
+  float* loss;                /* [1]  L averaged over the GLOBAL batch (c15)    */
+  float* grads;               /* [P]  global-batch mean gradient BEFORE Adam    */
+  int32_t* perms;             /* [ΣN] corruption permutations, LOCAL indices    */
+} mars_step_out;
+
+/* One DGI step over every graph of `g` (each graph = one (graph, sample) pair,
+ * pair index = global_pair_base + graph index, c15):
+ *   a4  pi = argsort_(key,i) sm64 keys (c12), X~ = X[pi] (Eq. 2)
+ *   a5-a7 Y_l = Â_n·act(T_{l-1}), Z_l = Y_l·W_l, both branches (Eqs. 1, 3)
+ *   a8-a10 s = sig(mean H3), scores h_iᵀ M s, BCE loss (Eqs. 4-6)
+ *   a11-a12 full backward; a13 NCCL allreduce(sum) when world_size > 1;
+ *   a14 Adam.
+ * global_batch = B, the number of pairs over all ranks the loss is averaged
+ * over.  Asynchronous on the library stream unless an output is requested. */
+MARS_API mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
+                          int64_t global_pair_base, int64_t global_batch, mars_step_out* out);
+
+/* a15: node embeddings H3 = encoder(X, A) of the positive branch (P:L132,
+ * L153) for every node of the set, [ΣN × H] fp32 row-major HOST array.
+ * Synchronous.  Overwrites the activations kept for the export hook. */
+MARS_API mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* embeddings);
+
+/* Test hook (parity P3): the last step's saved activations of layer
+ * `layer` in 1..3, stacked [pos; neg]: Y [2ΣN × C_in], Z [2ΣN × H] (host,
+ * fp32; either may be NULL). */
+MARS_API mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t layer, float* Y, float* Z);
+
+/* Checkpoint / resume: params, Adam m and v ([P] each) and step count t. */
+MARS_API mars_status mars_dgi_get_state(const mars_dgi* m, float* params, float* adam_m, float* adam_v,
+                               int64_t* t);
+MARS_API mars_status mars_dgi_set_state(mars_dgi* m, const float* params, const float* adam_m,
+                               const float* adam_v, int64_t t);
+
+/* Reporting hook: phases of the step schedule. */
+typedef enum {
+  MARS_PH_PERM = 0,       /* a4 corruption permutation                       */
+  MARS_PH_SPMM_FWD = 1,   /* a5 Y_l = Â_n act(T_{l-1}) (3 per step)          */
+  MARS_PH_GEMM_FWD = 2,   /* a6 Z_l = Y_l W_l (3 per step)                    */
+  MARS_PH_HEAD = 3,       /* a8-a11 readout, scores, loss, head backward, dZ3 */
+  MARS_PH_GEMM_DW = 4,    /* a12 dW_l = Y_lᵀ dZ_l (3 per step)                */
+  MARS_PH_GEMM_DY = 5,    /* a12 dY_l = dZ_l W_lᵀ (2 per step)                */
+  MARS_PH_SPMM_BWD = 6,   /* a12 dZ_{l-1} = (Â_n dY_l) ⊙ PReLU' (2 per step)  */
+  MARS_PH_ALLREDUCE = 7,  /* a13 NCCL gradient allreduce                      */
+  MARS_PH_ADAM = 8,       /* a14                                              */
+  MARS_PH_REDUCE = 9      /* dalpha partial reductions                        */
+} mars_phase;
+
+/* Reporting hook: runs one step exactly like mars_dgi_step (same kernels,
+ * same state update) but eagerly, with a CUDA event recorded on the launching
+ * stream after every kernel group; writes up to max_phases (phase id, device
+ * milliseconds) pairs in schedule order.  Synchronous. */
+MARS_API mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
+                                           int64_t global_pair_base, int64_t global_batch,
+                                           int32_t* phase_ids, float* phase_ms,
+                                           int32_t max_phases, int32_t* n_phases);
+
+/* Kernel launches enqueued by the most recent mars_dgi_step (for reporting). */
+MARS_API int64_t mars_dgi_last_launches(const mars_dgi* m);
+
+/* Frees a mars_graph* or mars_dgi* (tag-checked; NULL is a no-op). */
+MARS_API void mars_free(void* handle);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MARS_H_ */

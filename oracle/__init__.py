@@ -70,6 +70,12 @@ def lib():
             L.oracle_adam.argtypes = [ctypes.c_int64, f64p, f64p, f64p, f64p, ctypes.c_int64,
                                       ctypes.c_double, ctypes.c_double, ctypes.c_double,
                                       ctypes.c_double, ctypes.c_double]
+            L.oracle_head.restype = ctypes.c_double
+            L.oracle_head.argtypes = [ctypes.c_int32, i32p, ctypes.c_int32, ctypes.c_double, f64p,
+                                      ctypes.c_double, f64p, f64p, f64p, f64p, f64p]
+            L.oracle_spmm_rows.restype = None
+            L.oracle_spmm_rows.argtypes = [ctypes.c_int32, i32p, i32p, ctypes.c_int32, f64p,
+                                           ctypes.c_double, ctypes.c_int64, i64p, f64p]
             L.oracle_dense_anorm.restype = None
             L.oracle_dense_anorm.argtypes = [ctypes.c_int32, i32p, f64p]
             L.oracle_dense_step.restype = ctypes.c_double
@@ -194,6 +200,38 @@ def step_grads(batch: Batch, H: int, params, perms, B: float | None = None):
     acts = forward(batch, H, params, perms)
     loss, grads, s = backward(batch, H, params, acts, B)
     return loss, grads, s, acts
+
+
+def head(batch: Batch, H: int, params, Z3, B: float | None = None):
+    """Head only (a8-a11) at the given Z3: loss, s [G×H], dM [H×H], dZ3, dalpha3."""
+    F = batch.F
+    p = np.ascontiguousarray(params, np.float64)
+    M = np.ascontiguousarray(p[F * H + 2 * H * H:F * H + 3 * H * H])
+    a3 = float(p[-1])
+    Z3 = np.ascontiguousarray(Z3, np.float64)
+    s = np.zeros((batch.G, H)); dM = np.zeros((H, H)); dZ3 = np.zeros_like(Z3)
+    da = np.zeros(1)
+    loss = lib().oracle_head(batch.G, batch.node_off, H, float(batch.G if B is None else B), M, a3,
+                             Z3, s, dM, dZ3, da)
+    return loss, s, dM, dZ3, float(da[0])
+
+
+def layer1_input(batch: Batch, perms) -> np.ndarray:
+    """T0 = [X; X~] with X~[i] = X[off_g + pi[i]] (Eq. 2), stacked as the GPU does."""
+    perms = np.asarray(perms, np.int64)
+    gid = np.repeat(np.arange(batch.G), np.diff(batch.node_off))
+    src = batch.node_off[gid].astype(np.int64) + perms
+    return np.ascontiguousarray(np.concatenate([batch.X, batch.X[src]], 0))
+
+
+def spmm_rows(batch: Batch, T, rows, alpha=None) -> np.ndarray:
+    """Rows `rows` (stacked ids) of Â_n · act(T), act = PReLU_alpha or identity."""
+    T = np.ascontiguousarray(T, np.float64)
+    rows = np.ascontiguousarray(rows, np.int64)
+    out = np.zeros((rows.size, T.shape[1]))
+    lib().oracle_spmm_rows(batch.Nt, batch.rowptr, batch.colind, T.shape[1], T,
+                           float("nan") if alpha is None else float(alpha), rows.size, rows, out)
+    return out
 
 
 def encode(batch: Batch, H: int, params) -> np.ndarray:

@@ -1,0 +1,9 @@
+"""B200-native (sm_100a) DGI pre-training hot path of Mars (ICPP'21).
+
+The product is ``libmars.so`` (CUDA kernels + C ABI, ``include/mars.h``); this
+package holds it and a thin ctypes binding (``mars.py``) with the ABI's names.
+It never imports ``oracle/`` and has no CPU fallback.
+"""
+from .mars import (DGI, Graph, MarsError, MARS_BF16, MARS_FP32, config_default, dgi_create,  # noqa: F401
+                   dgi_export_activations, dgi_step, encode, free, graph_export_csr, graph_load,
+                   lib, nccl_get_unique_id, num_params, version, LIB_PATH, SIGNATURES)

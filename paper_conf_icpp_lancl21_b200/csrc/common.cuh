@@ -1,0 +1,42 @@
+// Device helpers shared by the libmars.so kernels.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace mars {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// splitmix64 mixer (DESIGN.md c12, c14): z += golden; two xor-shift-multiply rounds.
+__host__ __device__ __forceinline__ uint64_t sm64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ULL;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+  return v;
+}
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+  return v;
+}
+
+__device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
+
+// PReLU (c6): slope 1 for z > 0, a otherwise.
+__device__ __forceinline__ float prelu(float z, float a) { return z > 0.f ? z : a * z; }
+
+// Launch counter bump used by every launcher (mars_dgi_last_launches).
+__host__ inline void count_launch(int* launches, int n = 1) {
+  if (launches) *launches += n;
+}
+
+inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b); }
+
+}  // namespace mars

@@ -1,0 +1,277 @@
+// a8-a11 and the layer-3 part of a12: readout (Eq. 4), bilinear
+// discriminator (Eq. 5), BCE/JSD loss (Eq. 6 as read in c8,
+// P:L143-L145) and their backward, for every (graph, sample) pair of the set.
+//
+//   H3 = PReLU_{a3}(Z3)                     (recomputed on load, never stored)
+//   m_g = (1/N_g) Σ_{i∈g, pos} H3[i]; s_g = sig(m_g); v_g = M s_g
+//   l_i = H3[i]·v_g, l~_i = H3~[i]·v_g
+//   L = (1/B) Σ_g (1/(2N_g)) Σ_i [softplus(-l_i) + softplus(l~_i)]
+//   dl_i = (sig(l_i)-1)/(2 N_g B), dl~_i = sig(l~_i)/(2 N_g B)
+//   dv_g = Σ dl_i H3[i] + Σ dl~_i H3~[i]; dM = Σ_g dv_g s_gᵀ; ds = Mᵀ dv;
+//   dm = ds ⊙ s(1-s); dH3 = dl v_g + [pos] dm_g / N_g; dZ3 = dH3 ⊙ PReLU'(Z3)
+// Every cross-row reduction is two-stage with fixed-order fp64 combination
+// over row chunks that never straddle a graph (deterministic, no float atomics).
+#include "common.cuh"
+#include "internal.cuh"
+
+namespace mars {
+namespace {
+
+constexpr int kWarps = 8;
+
+// Stage 1 of m_g: per-chunk column sums of H3 over positive rows (fp64).
+// Block = H threads (one column each), one block per chunk.
+__global__ void k_colsum(const float* __restrict__ Z3, const float* __restrict__ alpha,
+                         const int32_t* __restrict__ chunk_row, int H,
+                         double* __restrict__ part) {
+  int c = threadIdx.x;
+  int ch = blockIdx.x;
+  float a = alpha[2];
+  double acc = 0.0;
+  for (int32_t r = chunk_row[ch]; r < chunk_row[ch + 1]; ++r)
+    acc += (double)prelu(Z3[(int64_t)r * H + c], a);
+  part[(int64_t)ch * H + c] = acc;
+}
+
+// Per graph: m, s = sig(m) (Eq. 4), v = M s (Eq. 5).  Block = H threads.
+__global__ void k_readout(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
+                          const int32_t* __restrict__ node_off, const float* __restrict__ M,
+                          int H, double* __restrict__ sd, float* __restrict__ sf,
+                          float* __restrict__ vf) {
+  extern __shared__ double sh_s[];
+  int g = blockIdx.x, c = threadIdx.x;
+  double acc = 0.0;
+  for (int ch = graph_chunk[g]; ch < graph_chunk[g + 1]; ++ch) acc += part[(int64_t)ch * H + c];
+  double Ng = (double)(node_off[g + 1] - node_off[g]);
+  double s = 1.0 / (1.0 + exp(-(acc / Ng)));
+  sh_s[c] = s;
+  sd[(int64_t)g * H + c] = s;
+  sf[(int64_t)g * H + c] = (float)s;
+  __syncthreads();
+  int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = H / 32;
+  for (int r = w; r < H; r += nw) {                  // v[r] = Σ_c M[r][c] s[c]
+    double t = 0.0;
+    for (int cc = lane; cc < H; cc += 32) t += (double)M[(int64_t)r * H + cc] * sh_s[cc];
+    t = warp_sum(t);
+    if (lane == 0) vf[(int64_t)g * H + r] = (float)t;
+  }
+}
+
+__device__ __forceinline__ double softplus_d(double x) {
+  return (x > 0.0 ? x : 0.0) + log1p(exp(-fabs(x)));
+}
+
+// Scores, loss partials, dl, and dv partials.  One block (8 warps) per chunk;
+// each warp takes rows i of the chunk, both the positive row i and the
+// corrupted row Nt+i; lanes own H/32 columns.
+template <int NC>
+__global__ void __launch_bounds__(kWarps * 32)
+k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
+        const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
+        const int32_t* __restrict__ node_off, const float* __restrict__ vf,
+        const StepParams* __restrict__ sp, int32_t Nt, float* __restrict__ dl,
+        double* __restrict__ dv_part, double* __restrict__ loss_part) {
+  constexpr int H = NC * 32;
+  __shared__ double sh_dv[kWarps][H];
+  __shared__ double sh_loss[kWarps];
+  int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  int g = chunk_graph[ch];
+  float a = alpha[2];
+  double Ng = (double)(node_off[g + 1] - node_off[g]);
+  double coef = (double)sp->inv_batch / (2.0 * Ng);
+  float v[NC];
+#pragma unroll
+  for (int q = 0; q < NC; ++q) v[q] = vf[(int64_t)g * H + lane + 32 * q];
+  double dv[NC];
+#pragma unroll
+  for (int q = 0; q < NC; ++q) dv[q] = 0.0;
+  double loss = 0.0;
+  for (int32_t i = chunk_row[ch] + w; i < chunk_row[ch + 1]; i += kWarps) {
+    float hp[NC], hn[NC];
+    float lp = 0.f, ln = 0.f;
+#pragma unroll
+    for (int q = 0; q < NC; ++q) {
+      hp[q] = prelu(Z3[(int64_t)i * H + lane + 32 * q], a);
+      hn[q] = prelu(Z3[((int64_t)Nt + i) * H + lane + 32 * q], a);
+      lp = fmaf(hp[q], v[q], lp);
+      ln = fmaf(hn[q], v[q], ln);
+    }
+    lp = warp_sum(lp);
+    ln = warp_sum(ln);
+    double sp_ = 1.0 / (1.0 + exp(-(double)lp));
+    double sn_ = 1.0 / (1.0 + exp(-(double)ln));
+    float dlp = (float)((sp_ - 1.0) * coef);
+    float dln = (float)(sn_ * coef);
+    if (lane == 0) {
+      dl[i] = dlp;
+      dl[Nt + i] = dln;
+      loss += softplus_d(-(double)lp) + softplus_d((double)ln);
+    }
+#pragma unroll
+    for (int q = 0; q < NC; ++q) dv[q] += (double)dlp * hp[q] + (double)dln * hn[q];
+  }
+#pragma unroll
+  for (int q = 0; q < NC; ++q) sh_dv[w][lane + 32 * q] = dv[q];
+  if (lane == 0) sh_loss[w] = loss;
+  __syncthreads();
+  for (int c = threadIdx.x; c < H; c += kWarps * 32) {
+    double t = 0.0;
+    for (int k = 0; k < kWarps; ++k) t += sh_dv[k][c];
+    dv_part[(int64_t)ch * H + c] = t;
+  }
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int k = 0; k < kWarps; ++k) t += sh_loss[k];
+    loss_part[ch] = t * coef;      // (1/B) (1/(2 N_g)) Σ softplus terms of this chunk
+  }
+}
+
+// Per graph: dv_g (fixed-order fp64 sum of chunks), ds = Mᵀ dv, dm = ds s(1-s)/N_g.
+__global__ void k_head_bwd(const double* __restrict__ dv_part,
+                           const int32_t* __restrict__ graph_chunk,
+                           const int32_t* __restrict__ node_off, const float* __restrict__ M,
+                           const double* __restrict__ sd, int H, double* __restrict__ dvd,
+                           float* __restrict__ dvf, float* __restrict__ dmf) {
+  extern __shared__ double sh_dv[];
+  int g = blockIdx.x, c = threadIdx.x;
+  double acc = 0.0;
+  for (int ch = graph_chunk[g]; ch < graph_chunk[g + 1]; ++ch) acc += dv_part[(int64_t)ch * H + c];
+  sh_dv[c] = acc;
+  dvd[(int64_t)g * H + c] = acc;
+  dvf[(int64_t)g * H + c] = (float)acc;
+  __syncthreads();
+  double ds = 0.0;
+  for (int r = 0; r < H; ++r) ds += (double)M[(int64_t)r * H + c] * sh_dv[r];
+  double s = sd[(int64_t)g * H + c];
+  double Ng = (double)(node_off[g + 1] - node_off[g]);
+  dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / Ng);
+}
+
+// dM[r][c] = Σ_g dv_g[r] s_g[c] (fixed order); block 0 also writes the loss.
+__global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ sd, int G, int H,
+                     const double* __restrict__ loss_part, int nchunks,
+                     float* __restrict__ gM, float* __restrict__ loss_out) {
+  int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e < (int64_t)H * H) {
+    int r = (int)(e / H), c = (int)(e % H);
+    double t = 0.0;
+    for (int g = 0; g < G; ++g) t += dvd[(int64_t)g * H + r] * sd[(int64_t)g * H + c];
+    gM[e] = (float)t;
+  }
+  if (e == 0) {
+    double t = 0.0;
+    for (int k = 0; k < nchunks; ++k) t += loss_part[k];
+    *loss_out = (float)t;
+  }
+}
+
+// dZ3 = (dl v_g + [pos] dm_g) ⊙ PReLU'(Z3), dalpha3 partials.  Warp per row.
+template <int NC>
+__global__ void __launch_bounds__(kWarps * 32)
+k_dz3(const float* __restrict__ Z3, const float* __restrict__ alpha,
+      const int32_t* __restrict__ node_graph, const float* __restrict__ dl,
+      const float* __restrict__ vf, const float* __restrict__ dmf, int32_t Nt,
+      float* __restrict__ dZ, double* __restrict__ slots) {
+  constexpr int H = NC * 32;
+  __shared__ double wpart[kWarps];
+  int lane = threadIdx.x & 31;
+  int64_t r = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
+  float da = 0.f;
+  if (r < 2LL * Nt) {
+    int32_t i = (int32_t)(r < Nt ? r : r - Nt);
+    bool pos = r < Nt;
+    int g = node_graph[i];
+    float a = alpha[2];
+    float d = dl[r];
+#pragma unroll
+    for (int q = 0; q < NC; ++q) {
+      int c = lane + 32 * q;
+      float dh = d * vf[(int64_t)g * H + c] + (pos ? dmf[(int64_t)g * H + c] : 0.f);
+      float z = Z3[r * H + c];
+      dZ[r * H + c] = z > 0.f ? dh : a * dh;
+      da += z > 0.f ? 0.f : dh * z;
+    }
+  }
+  double t = warp_sum((double)da);
+  if (lane == 0) wpart[threadIdx.x >> 5] = t;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double s = 0.0;
+    for (int k = 0; k < kWarps; ++k) s += wpart[k];
+    slots[blockIdx.x] = s;
+  }
+}
+
+__global__ void k_reduce_slots(const double* __restrict__ slots, int n, float* __restrict__ out) {
+  __shared__ double sh[256];
+  double t = 0.0;
+  for (int k = threadIdx.x; k < n; k += 256) t += slots[k];
+  sh[threadIdx.x] = t;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (threadIdx.x < o) sh[threadIdx.x] += sh[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *out = (float)sh[0];
+}
+
+__global__ void k_prelu(const float* __restrict__ Z, const float* __restrict__ alpha, int layer,
+                        float* __restrict__ out, int64_t n) {
+  int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e < n) out[e] = prelu(Z[e], alpha[layer]);
+}
+
+template <int NC>
+cudaError_t head_nc(const GraphDev& g, const float* Z3, const float* M, const float* alpha,
+                    const StepParams* sp, const HeadWork& w, float* dZ, float* gM,
+                    float* loss_out, int* nslots, cudaStream_t s) {
+  constexpr int H = NC * 32;
+  k_colsum<<<g.nchunks, H, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
+  k_readout<<<g.G, H, H * sizeof(double), s>>>(w.colsum_part, g.graph_chunk, g.node_off, M, H,
+                                                w.sd, w.s, w.v);
+  k_score<NC><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph, g.node_off,
+                                                w.v, sp, g.Nt, w.dl, w.dv_part, w.loss_part);
+  k_head_bwd<<<g.G, H, H * sizeof(double), s>>>(w.dv_part, g.graph_chunk, g.node_off, M, w.sd, H,
+                                                 w.dvd, w.dv, w.dm);
+  k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_part, g.nchunks, gM,
+                                                 loss_out);
+  unsigned nb = cdiv(2LL * g.Nt, kWarps);
+  k_dz3<NC><<<nb, kWarps * 32, 0, s>>>(Z3, alpha, g.node_graph, w.dl, w.v, w.dm, g.Nt, dZ,
+                                       w.slots);
+  *nslots = (int)nb;
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+int head_slots(const GraphDev& g) { return (int)cdiv(2LL * g.Nt, kWarps) + 1; }
+
+cudaError_t launch_head(const GraphDev& g, int H, const float* Z3, const float* params_M,
+                        const float* alpha_dev, const StepParams* sp, const HeadWork& w,
+                        float* dZ, float* grad_M, float* loss_out, int* nslots, cudaStream_t s,
+                        int* launches) {
+  count_launch(launches, 6);
+  switch (H) {
+    case 32: return head_nc<1>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
+    case 64: return head_nc<2>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
+    case 128: return head_nc<4>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
+    case 256: return head_nc<8>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
+                                int* launches) {
+  count_launch(launches);
+  k_reduce_slots<<<1, 256, 0, s>>>(slots, n, grad);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_prelu(const float* Z, const float* alpha_dev, int layer, float* out, int64_t n,
+                         cudaStream_t s, int* launches) {
+  count_launch(launches);
+  k_prelu<<<cdiv(n, 256), 256, 0, s>>>(Z, alpha_dev, layer, out, n);
+  return cudaGetLastError();
+}
+
+}  // namespace mars

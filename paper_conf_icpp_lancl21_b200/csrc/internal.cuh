@@ -1,0 +1,152 @@
+// Internal declarations shared by the libmars.so translation units (kernels +
+// runtime).  Nothing here is part of the ABI; include/mars.h is.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace mars {
+
+constexpr int kLayers = 3;
+
+// Per-step scalars the captured step graph reads from device memory (written
+// by one H2D copy before each replay, so a replay never bakes them in).
+struct StepParams {
+  uint64_t step_index;
+  int64_t pair_base;
+  float inv_batch;      // 1 / global batch B
+  float adam_step_size; // lr / (1 - beta1^t)
+  float adam_bc2_sqrt;  // sqrt(1 - beta2^t)
+  float pad;
+};
+
+// Device view of a loaded graph set (block-diagonal, global node ids).
+struct GraphDev {
+  int32_t G;            // graphs
+  int32_t Nt;           // total nodes
+  int64_t nnz;          // nnz(Â) total
+  int32_t F;
+  const int32_t* node_off;   // [G+1]
+  const int32_t* node_graph; // [Nt] graph id of each node
+  const int32_t* rowptr;     // [Nt+1]
+  const int32_t* colind;     // [nnz] global ids
+  const float* vals;         // [nnz]
+  const float* X;            // [Nt*F]
+  // deterministic reduction chunks: rows [chunk_row[c], chunk_row[c+1]) all in graph chunk_graph[c]
+  int32_t nchunks;
+  const int32_t* chunk_row;  // [nchunks+1]
+  const int32_t* chunk_graph;// [nchunks]
+  const int32_t* graph_chunk;// [G+1] first chunk of each graph
+  // permutation buckets
+  int32_t nbuckets;
+  const int32_t* bucket_off; // [G+1]
+  const int32_t* bucket_log2;// [G]
+};
+
+// ---------------------------------------------------------------- builder.cu
+// Builds the CSR of Â for the packed set.  d_indptr: [Nt + G] int64 concatenated
+// per-graph indptr arrays; d_indices: [Et] local indices; node_off/edge_off
+// per graph.  Outputs rowptr [Nt+1], colind (allocated by caller with the
+// returned capacity), deg, dinv, vals.  err_flag: set nonzero on malformed input.
+struct BuilderIO {
+  int32_t G, Nt;
+  int64_t Et;
+  const int64_t* indptr;     // [Nt+G]
+  const int32_t* indices;    // [Et]
+  const int32_t* node_off;   // [G+1]
+  const int64_t* edge_off;   // [G+1]
+  const int32_t* node_graph; // [Nt]
+  int32_t* cnt;              // [Nt+1] scratch
+  int32_t* off_dup;          // [Nt+1] scratch
+  int32_t* cursor;           // [Nt] scratch
+  int32_t* buf;              // [Nt+2Et] scratch
+  int32_t* buf2;             // [Nt+2Et] scratch
+  int32_t* ucnt;             // [Nt+1] scratch
+  int32_t* rowptr;           // [Nt+1] out
+  int32_t* deg;              // [Nt] out
+  float* dinv;               // [Nt] out
+  int32_t* err;              // [1]
+  void* scan_tmp;            // scratch for scans
+  size_t scan_tmp_bytes;
+};
+size_t scan_tmp_bytes(int64_t n);
+cudaError_t scan_exclusive_i32(const int32_t* in, int32_t* out, int64_t n, void* tmp,
+                               cudaStream_t s, int* launches);
+cudaError_t build_csr_phase1(const BuilderIO& io, cudaStream_t s);  // -> rowptr (host reads nnz)
+cudaError_t build_csr_phase2(const BuilderIO& io, int32_t* colind, float* vals,
+                             cudaStream_t s);
+
+// ---------------------------------------------------------------- perm.cu
+// Corruption permutation (Eq. 2, c12) for every graph of the set; writes
+// perm_global[Nt] (global node id of X~ row i).
+struct PermWork {
+  uint64_t* keys;     // [Nt]
+  int32_t* bucket;    // [Nt]
+  int32_t* bcnt;      // [nbuckets+1]
+  int32_t* bstart;    // [nbuckets+1]
+  int32_t* bcur;      // [nbuckets]
+  int32_t* members;   // [Nt]
+  void* scan_tmp;
+};
+cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
+                        const PermWork& w, int32_t* perm_global, cudaStream_t s, int* launches);
+
+// ---------------------------------------------------------------- spmm.cu
+// Forward aggregate of both branches: Y[i] = Σ_j a_ij act(T[j]), Y[Nt+i] = Σ_j a_ij
+// act(T[Nt+j]).  layer1: T = X (pos) and X[perm[j]] (neg), act = identity.
+// Otherwise act = PReLU(alpha[act_layer]).  neg_rows = 0 aggregates only the
+// positive branch (encode).
+cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const float* T, const int32_t* perm,
+                            const float* alpha_dev, int act_layer, float* Y, int both,
+                            cudaStream_t s, int* launches);
+// Backward aggregate dH = Â_n dY (Â_n symmetric) with the PReLU'(Z) epilogue:
+// dZ = dH ⊙ (Z > 0 ? 1 : a), dalpha partials Σ dH·min(Z,0) -> slots[gridDim].
+cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const float* dY, const float* Z,
+                            const float* alpha_dev, int layer, float* dZ, double* slots,
+                            int* nslots, cudaStream_t s, int* launches);
+int spmm_bwd_slots(const GraphDev& g);
+
+// ---------------------------------------------------------------- gemm_simt.cu
+// fp32 SIMT GEMMs (parity path).
+cudaError_t gemm_nn(const float* A, const float* B, float* C, int64_t M, int N, int K,
+                    cudaStream_t s, int* launches);       // C[M×N] = A[M×K] B[K×N]
+cudaError_t gemm_nt(const float* A, const float* B, float* C, int64_t M, int N, int K,
+                    cudaStream_t s, int* launches);       // C[M×N] = A[M×K] B[N×K]ᵀ
+size_t gemm_tn_partial_floats(int64_t R, int M, int N);
+cudaError_t gemm_tn(const float* A, const float* B, float* out, int64_t R, int M, int N,
+                    double* partial, cudaStream_t s, int* launches);  // out[M×N] = Aᵀ B, A[R×M], B[R×N]
+
+// ---------------------------------------------------------------- head.cu
+struct HeadWork {
+  double* colsum_part;  // [nchunks*H]
+  double* dv_part;      // [nchunks*H]
+  double* loss_part;    // [nchunks]
+  float* s;             // [G*H]
+  float* v;             // [G*H]
+  float* dm;            // [G*H] (already divided by N_g)
+  float* dv;            // [G*H]
+  double* dvd;          // [G*H]
+  double* sd;           // [G*H]
+  float* dl;            // [2*Nt]
+  double* slots;        // [nslots] dalpha3 partials
+};
+// Forward head + head backward: writes grads of M (dM) and the loss slot,
+// dZ3 into dZ, dalpha3 partials into w.slots.
+cudaError_t launch_head(const GraphDev& g, int H, const float* Z3, const float* params_M,
+                        const float* alpha_dev, const StepParams* sp, const HeadWork& w,
+                        float* dZ, float* grad_M, float* loss_out, int* nslots,
+                        cudaStream_t s, int* launches);
+int head_slots(const GraphDev& g);
+// grad[0] = Σ slots (fixed order, double)
+cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
+                                int* launches);
+// H3 = PReLU(Z3) for the first `rows` rows (encode)
+cudaError_t launch_prelu(const float* Z, const float* alpha_dev, int layer, float* out,
+                         int64_t n, cudaStream_t s, int* launches);
+
+// ---------------------------------------------------------------- adam.cu
+cudaError_t launch_adam(float* params, float* m, float* v, const float* grads, int64_t P,
+                        double beta1, double beta2, double eps, double clip_norm, double* norm_part,
+                        const StepParams* sp, cudaStream_t s, int* launches);
+cudaError_t launch_check_finite(const float* loss, int32_t* flag, cudaStream_t s, int* launches);
+
+}  // namespace mars

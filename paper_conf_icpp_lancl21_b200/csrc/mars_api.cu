@@ -1,0 +1,941 @@
+// libmars.so runtime and C ABI (include/mars.h): handle management, graph-set
+// ingest, workspaces, the per-step kernel schedule captured once
+// into a CUDA Graph and replayed, NCCL data parallelism, test hooks.
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/mars.h"
+#include "common.cuh"
+#include "internal.cuh"
+
+using namespace mars;
+
+namespace {
+
+constexpr uint64_t kTagGraph = 0x4D41525347524150ULL;  // "MARSGRAP"
+constexpr uint64_t kTagDgi = 0x4D41525344474931ULL;    // "MARSDGI1"
+constexpr uint64_t kTagDead = 0xDEADDEADDEADDEADULL;
+constexpr int kChunkRows = 64;
+
+thread_local std::string g_err;
+
+mars_status fail(mars_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+#define CK(call)                                                                   \
+  do {                                                                             \
+    cudaError_t e_ = (call);                                                       \
+    if (e_ != cudaSuccess) {                                                       \
+      cudaGetLastError();                                                          \
+      return fail(e_ == cudaErrorMemoryAllocation ? MARS_ENOMEM : MARS_ECUDA,       \
+                  "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    }                                                                              \
+  } while (0)
+
+bool valid_F(int F) { return F == 16 || F == 32 || F == 64 || F == 128 || F == 256; }
+bool valid_H(int H) { return H == 32 || H == 64 || H == 128 || H == 256; }
+
+template <typename T>
+cudaError_t dalloc(T** p, size_t n) {
+  return cudaMalloc(reinterpret_cast<void**>(p), sizeof(T) * (n ? n : 1));
+}
+
+// ---------------------------------------------------------------- NCCL (dlopen)
+struct NcclApi {
+  bool tried = false, ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+NcclApi g_nccl;
+std::mutex g_nccl_mu;
+
+bool nccl_load() {
+  std::lock_guard<std::mutex> lk(g_nccl_mu);
+  if (g_nccl.tried) return g_nccl.ok;
+  g_nccl.tried = true;
+  void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+  if (!h) return false;
+  g_nccl.GetUniqueId = reinterpret_cast<decltype(g_nccl.GetUniqueId)>(dlsym(h, "ncclGetUniqueId"));
+  g_nccl.CommInitRank = reinterpret_cast<decltype(g_nccl.CommInitRank)>(dlsym(h, "ncclCommInitRank"));
+  g_nccl.AllReduce = reinterpret_cast<decltype(g_nccl.AllReduce)>(dlsym(h, "ncclAllReduce"));
+  g_nccl.CommDestroy = reinterpret_cast<decltype(g_nccl.CommDestroy)>(dlsym(h, "ncclCommDestroy"));
+  g_nccl.GetErrorString =
+      reinterpret_cast<decltype(g_nccl.GetErrorString)>(dlsym(h, "ncclGetErrorString"));
+  g_nccl.ok = g_nccl.GetUniqueId && g_nccl.CommInitRank && g_nccl.AllReduce && g_nccl.CommDestroy;
+  return g_nccl.ok;
+}
+
+// ---------------------------------------------------------------- pinned staging
+struct Pinned {
+  std::mutex mu;
+  void* p = nullptr;
+  size_t cap = 0;
+  void* get(size_t n) {
+    if (n > cap) {
+      if (p) cudaFreeHost(p);
+      p = nullptr;
+      cap = 0;
+      size_t want = n + n / 4 + 4096;
+      if (cudaMallocHost(&p, want) != cudaSuccess) return nullptr;
+      cap = want;
+    }
+    return p;
+  }
+};
+Pinned g_stage;
+
+// ---------------------------------------------------------------- kernels local to the runtime
+__global__ void k_node_graph(const int32_t* __restrict__ node_off, int G, int32_t Nt,
+                             int32_t* __restrict__ node_graph) {
+  int32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= Nt) return;
+  int lo = 0, hi = G - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (node_off[mid] <= i) lo = mid; else hi = mid - 1;
+  }
+  node_graph[i] = lo;
+}
+
+// Xavier-uniform init (c14): w = f32((2u-1) b), u = (sm64(sm64(seed^tag)^idx) >> 40) 2^-24.
+__global__ void k_xavier(float* __restrict__ p, int64_t n, uint64_t seed, uint64_t tag, float b) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint64_t base = sm64(seed ^ tag);
+  double u = (double)(sm64(base ^ (uint64_t)i) >> 40) * (1.0 / 16777216.0);
+  p[i] = __double2float_rn(__dmul_rn(__dsub_rn(__dmul_rn(2.0, u), 1.0), (double)b));
+}
+
+__global__ void k_fill(float* __restrict__ p, int64_t n, float v) {
+  int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = v;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------- handles
+std::atomic<uint64_t> g_graph_uid{1};
+
+struct mars_graph {
+  uint64_t tag = kTagGraph;
+  uint64_t uid = g_graph_uid.fetch_add(1);
+  int device = 0;
+  int G = 0, F = 0;
+  int32_t Nt = 0;
+  int64_t Et = 0, nnz = 0;
+  std::vector<int32_t> h_node_off;
+  std::vector<int64_t> h_nnz_off;
+  int32_t *node_off = nullptr, *node_graph = nullptr, *rowptr = nullptr, *colind = nullptr;
+  int32_t *deg = nullptr, *chunk_row = nullptr, *chunk_graph = nullptr, *graph_chunk = nullptr;
+  int32_t *bucket_off = nullptr, *bucket_log2 = nullptr;
+  float *vals = nullptr, *dinv = nullptr, *X = nullptr;
+  GraphDev dev{};
+  ~mars_graph() {
+    for (void* p : {(void*)node_off, (void*)node_graph, (void*)rowptr, (void*)colind, (void*)deg,
+                    (void*)chunk_row, (void*)chunk_graph, (void*)graph_chunk, (void*)bucket_off,
+                    (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X})
+      if (p) cudaFree(p);
+  }
+};
+
+struct Workspace {
+  int32_t Nt = 0, G = 0, nchunks = 0, nbuckets = 0, F = 0, H = 0;
+  float *Y1 = nullptr, *Z[3] = {nullptr, nullptr, nullptr}, *Y23[2] = {nullptr, nullptr};
+  float *dZ = nullptr, *dY = nullptr;
+  int32_t* perm = nullptr;
+  PermWork pw{};
+  HeadWork hw{};
+  double *slots[3] = {nullptr, nullptr, nullptr};
+  double* tn_part = nullptr;
+  size_t tn_part_n = 0;
+  std::vector<void*> owned;
+  void release() {
+    for (void* p : owned) cudaFree(p);
+    owned.clear();
+    *this = Workspace();
+  }
+};
+
+struct mars_dgi {
+  uint64_t tag = kTagDgi;
+  mars_dgi_config cfg{};
+  int F = 0, H = 0;
+  int64_t P = 0;
+  int64_t t = 0;
+  cudaStream_t own_stream = nullptr, stream = nullptr;
+  float *params = nullptr, *adam_m = nullptr, *adam_v = nullptr, *grads = nullptr;
+  double* norm_part = nullptr;
+  int32_t* finite_flag = nullptr;
+  StepParams* d_sp = nullptr;
+  StepParams* h_sp = nullptr;       // pinned ring
+  cudaEvent_t* sp_ev = nullptr;
+  int sp_ring = 32, sp_next = 0;
+  Workspace ws;
+  const mars_graph* ws_graph = nullptr;
+  bool capture = true;
+  cudaGraphExec_t exec = nullptr;
+  uint64_t exec_graph = 0;          // uid of the graph set the exec was captured for
+  uint64_t prev_graph = 0;          // uid of the graph set of the previous step
+  cudaStream_t exec_stream = nullptr;
+  int64_t last_launches = 0, exec_launches = 0;
+  int32_t last_Nt = 0;              // node count of the last step's graph set (export hook)
+  ncclComm_t comm = nullptr;
+  ~mars_dgi() {
+    if (exec) cudaGraphExecDestroy(exec);
+    ws.release();
+    for (void* p : {(void*)params, (void*)adam_m, (void*)adam_v, (void*)grads, (void*)norm_part,
+                    (void*)finite_flag, (void*)d_sp})
+      if (p) cudaFree(p);
+    if (sp_ev) {
+      for (int i = 0; i < sp_ring; ++i) cudaEventDestroy(sp_ev[i]);
+      delete[] sp_ev;
+    }
+    if (h_sp) cudaFreeHost(h_sp);
+    if (comm && g_nccl.CommDestroy) g_nccl.CommDestroy(comm);
+    if (own_stream) cudaStreamDestroy(own_stream);
+  }
+};
+
+// ---------------------------------------------------------------- misc ABI
+extern "C" const char* mars_last_error(void) { return g_err.c_str(); }
+extern "C" const char* mars_version(void) { return "mars-b200 0.1 sm_100a"; }
+extern "C" int64_t mars_num_params(int32_t F, int32_t H) {
+  return (int64_t)F * H + 3LL * H * H + 3;
+}
+
+extern "C" void mars_dgi_config_default(mars_dgi_config* c) {
+  if (!c) return;
+  memset(c, 0, sizeof *c);
+  c->in_dim = 64;
+  c->hidden_dim = 256;
+  c->num_layers = 3;
+  c->precision = MARS_FP32;
+  c->lr = 1e-3;
+  c->beta1 = 0.9;
+  c->beta2 = 0.999;
+  c->eps = 1e-8;
+  c->clip_norm = 0.0;
+  c->seed = 0;
+  c->init_params = nullptr;
+  c->device = 0;
+  c->world_size = 1;
+  c->rank = 0;
+  c->nccl_unique_id = nullptr;
+}
+
+static mars_status check_graph(const mars_graph* g) {
+  if (!g || g->tag != kTagGraph) return fail(MARS_ESTATE, "invalid or freed mars_graph handle");
+  return MARS_OK;
+}
+static mars_status check_dgi(const mars_dgi* m) {
+  if (!m || m->tag != kTagDgi) return fail(MARS_ESTATE, "invalid or freed mars_dgi handle");
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- graph load (a1-a3)
+extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, int32_t device,
+                                       mars_graph** out) {
+  if (!out) return fail(MARS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!descs || G < 1) return fail(MARS_EINVAL, "need at least one graph");
+  int F = descs[0].feat_dim;
+  if (!valid_F(F)) return fail(MARS_EINVAL, "feat_dim %d not in {16,32,64,128,256}", F);
+  int64_t Nt = 0, Et = 0;
+  for (int g = 0; g < G; ++g) {
+    const mars_graph_desc& d = descs[g];
+    if (d.num_nodes < 1) return fail(MARS_EINVAL, "graph %d: num_nodes < 1", g);
+    if (!d.indptr || !d.features || (!d.indices && d.indptr[d.num_nodes] > 0))
+      return fail(MARS_EINVAL, "graph %d: NULL array", g);
+    if (d.feat_dim != F) return fail(MARS_EINVAL, "graph %d: feat_dim mismatch", g);
+    if (d.indptr[0] != 0 || d.indptr[d.num_nodes] < 0)
+      return fail(MARS_EINVAL, "graph %d: malformed indptr", g);
+    Nt += d.num_nodes;
+    Et += d.indptr[d.num_nodes];
+  }
+  if (Nt + 2 * Et >= (int64_t)INT32_MAX - 1) return fail(MARS_EINVAL, "graph set too large");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "no CUDA device (libmars has no CPU fallback)");
+  }
+  if (device < 0 || device >= ndev) return fail(MARS_EINVAL, "bad device %d", device);
+  CK(cudaSetDevice(device));
+
+  auto* gr = new mars_graph();
+  std::unique_ptr<mars_graph> guard(gr);
+  gr->device = device;
+  gr->G = G;
+  gr->F = F;
+  gr->Nt = (int32_t)Nt;
+  gr->Et = Et;
+  // host-side small tables: node/edge offsets, reduction chunks, permutation buckets
+  gr->h_node_off.resize(G + 1);
+  std::vector<int64_t> edge_off(G + 1);
+  std::vector<int32_t> chunk_row, chunk_graph, graph_chunk(G + 1), bucket_off(G + 1),
+      bucket_log2(G);
+  gr->h_node_off[0] = 0;
+  edge_off[0] = 0;
+  for (int g = 0; g < G; ++g) {
+    int32_t N = descs[g].num_nodes;
+    gr->h_node_off[g + 1] = gr->h_node_off[g] + N;
+    edge_off[g + 1] = edge_off[g] + descs[g].indptr[N];
+    graph_chunk[g] = (int32_t)chunk_graph.size();
+    for (int32_t r = 0; r < N; r += kChunkRows) {
+      chunk_row.push_back(gr->h_node_off[g] + r);
+      chunk_graph.push_back(g);
+    }
+    int lb = 0;
+    while ((1LL << lb) < N) ++lb;
+    lb = lb > 2 ? lb - 2 : 0;
+    bucket_log2[g] = lb;
+    bucket_off[g + 1] = bucket_off[g] + (1 << lb);
+  }
+  bucket_off[0] = 0;
+  graph_chunk[G] = (int32_t)chunk_graph.size();
+  chunk_row.push_back((int32_t)Nt);
+  int nchunks = (int)chunk_graph.size();
+
+  // pack inputs into pinned staging and copy once
+  size_t b_indptr = sizeof(int64_t) * (size_t)(Nt + G);
+  size_t b_idx = sizeof(int32_t) * (size_t)Et;
+  size_t b_X = sizeof(float) * (size_t)Nt * F;
+  std::lock_guard<std::mutex> lk(g_stage.mu);
+  char* stage = static_cast<char*>(g_stage.get(b_indptr + b_idx + b_X + 64));
+  if (!stage) return fail(MARS_ENOMEM, "pinned staging allocation failed");
+  int64_t* s_indptr = reinterpret_cast<int64_t*>(stage);
+  int32_t* s_idx = reinterpret_cast<int32_t*>(stage + b_indptr);
+  float* s_X = reinterpret_cast<float*>(stage + b_indptr + b_idx);
+  for (int g = 0; g < G; ++g) {
+    const mars_graph_desc& d = descs[g];
+    int32_t N = d.num_nodes;
+    memcpy(s_indptr + gr->h_node_off[g] + g, d.indptr, sizeof(int64_t) * (size_t)(N + 1));
+    if (d.indptr[N] > 0) memcpy(s_idx + edge_off[g], d.indices, sizeof(int32_t) * (size_t)d.indptr[N]);
+    memcpy(s_X + (int64_t)gr->h_node_off[g] * F, d.features, sizeof(float) * (size_t)N * F);
+  }
+  cudaStream_t s = nullptr;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+
+  int64_t* d_indptr;
+  int32_t* d_idx;
+  int64_t* d_edge_off;
+  CK(dalloc(&d_indptr, (size_t)(Nt + G)));
+  struct F1 { void* p; ~F1() { cudaFree(p); } } f1{d_indptr};
+  CK(dalloc(&d_idx, (size_t)Et));
+  F1 f2{d_idx};
+  CK(dalloc(&d_edge_off, (size_t)G + 1));
+  F1 f3{d_edge_off};
+  CK(dalloc(&gr->X, (size_t)Nt * F));
+  CK(dalloc(&gr->node_off, (size_t)G + 1));
+  CK(dalloc(&gr->node_graph, (size_t)Nt));
+  CK(dalloc(&gr->rowptr, (size_t)Nt + 1));
+  CK(dalloc(&gr->deg, (size_t)Nt));
+  CK(dalloc(&gr->dinv, (size_t)Nt));
+  CK(dalloc(&gr->chunk_row, (size_t)nchunks + 1));
+  CK(dalloc(&gr->chunk_graph, (size_t)nchunks));
+  CK(dalloc(&gr->graph_chunk, (size_t)G + 1));
+  CK(dalloc(&gr->bucket_off, (size_t)G + 1));
+  CK(dalloc(&gr->bucket_log2, (size_t)G));
+  CK(cudaMemcpyAsync(d_indptr, s_indptr, b_indptr, cudaMemcpyHostToDevice, s));
+  if (Et) CK(cudaMemcpyAsync(d_idx, s_idx, b_idx, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->X, s_X, b_X, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(d_edge_off, edge_off.data(), sizeof(int64_t) * (G + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->node_off, gr->h_node_off.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->chunk_row, chunk_row.data(), sizeof(int32_t) * (nchunks + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->chunk_graph, chunk_graph.data(), sizeof(int32_t) * nchunks, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->graph_chunk, graph_chunk.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->bucket_off, bucket_off.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(gr->bucket_log2, bucket_log2.data(), sizeof(int32_t) * G, cudaMemcpyHostToDevice, s));
+  k_node_graph<<<cdiv(Nt, 256), 256, 0, s>>>(gr->node_off, G, (int32_t)Nt, gr->node_graph);
+  CK(cudaGetLastError());
+
+  // builder scratch
+  BuilderIO io{};
+  io.G = G;
+  io.Nt = (int32_t)Nt;
+  io.Et = Et;
+  io.indptr = d_indptr;
+  io.indices = d_idx;
+  io.node_off = gr->node_off;
+  io.edge_off = d_edge_off;
+  io.node_graph = gr->node_graph;
+  int64_t cap = Nt + 2 * Et;
+  std::vector<void*> scratch;
+  struct SF { std::vector<void*>* v; ~SF() { for (void* p : *v) cudaFree(p); } } sf{&scratch};
+  auto salloc = [&](void** p, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMalloc(p, bytes ? bytes : 4);
+    if (e == cudaSuccess) scratch.push_back(*p);
+    return e;
+  };
+  CK(salloc((void**)&io.cnt, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.off_dup, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.cursor, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.buf, sizeof(int32_t) * cap));
+  CK(salloc((void**)&io.buf2, sizeof(int32_t) * cap));
+  CK(salloc((void**)&io.ucnt, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.err, sizeof(int32_t) * 2));
+  io.scan_tmp_bytes = scan_tmp_bytes(Nt + 1);
+  CK(salloc(&io.scan_tmp, io.scan_tmp_bytes));
+  io.rowptr = gr->rowptr;
+  io.deg = gr->deg;
+  io.dinv = gr->dinv;
+  CK(build_csr_phase1(io, s));
+  int32_t herr[2] = {0, 0};
+  CK(cudaMemcpyAsync(herr, io.err, sizeof herr, cudaMemcpyDeviceToHost, s));
+  std::vector<int32_t> h_rowptr((size_t)Nt + 1);
+  CK(cudaMemcpyAsync(h_rowptr.data(), gr->rowptr, sizeof(int32_t) * (Nt + 1), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (herr[0]) return fail(MARS_EINVAL, "malformed graph input (code %d): %s", herr[0],
+                           (herr[0] & 2) ? "edge index out of range" : "indptr inconsistent");
+  gr->nnz = h_rowptr[Nt];
+  gr->h_nnz_off.resize(G + 1);
+  for (int g = 0; g <= G; ++g) gr->h_nnz_off[g] = h_rowptr[gr->h_node_off[g]];
+  CK(dalloc(&gr->colind, (size_t)gr->nnz));
+  CK(dalloc(&gr->vals, (size_t)gr->nnz));
+  CK(build_csr_phase2(io, gr->colind, gr->vals, s));
+  CK(cudaStreamSynchronize(s));
+
+  GraphDev& v = gr->dev;
+  v.G = G;
+  v.Nt = (int32_t)Nt;
+  v.nnz = gr->nnz;
+  v.F = F;
+  v.node_off = gr->node_off;
+  v.node_graph = gr->node_graph;
+  v.rowptr = gr->rowptr;
+  v.colind = gr->colind;
+  v.vals = gr->vals;
+  v.X = gr->X;
+  v.nchunks = nchunks;
+  v.chunk_row = gr->chunk_row;
+  v.chunk_graph = gr->chunk_graph;
+  v.graph_chunk = gr->graph_chunk;
+  v.nbuckets = bucket_off[G];
+  v.bucket_off = gr->bucket_off;
+  v.bucket_log2 = gr->bucket_log2;
+  *out = guard.release();
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_graph_info(const mars_graph* g, int32_t* G, int64_t* Nt, int64_t* nnz,
+                                       int32_t* F) {
+  if (mars_status st = check_graph(g)) return st;
+  if (G) *G = g->G;
+  if (Nt) *Nt = g->Nt;
+  if (nnz) *nnz = g->nnz;
+  if (F) *F = g->F;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_graph_size(const mars_graph* g, int32_t idx, int32_t* N, int64_t* nnz) {
+  if (mars_status st = check_graph(g)) return st;
+  if (idx < 0 || idx >= g->G) return fail(MARS_EINVAL, "graph index out of range");
+  if (N) *N = g->h_node_off[idx + 1] - g->h_node_off[idx];
+  if (nnz) *nnz = g->h_nnz_off[idx + 1] - g->h_nnz_off[idx];
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_graph_export_csr(const mars_graph* g, int32_t idx, int32_t* rowptr,
+                                             int32_t* colind, int32_t* deg, float* dinv,
+                                             float* vals) {
+  if (mars_status st = check_graph(g)) return st;
+  if (idx < 0 || idx >= g->G) return fail(MARS_EINVAL, "graph index out of range");
+  CK(cudaSetDevice(g->device));
+  int32_t n0 = g->h_node_off[idx], N = g->h_node_off[idx + 1] - n0;
+  int64_t z0 = g->h_nnz_off[idx], Z = g->h_nnz_off[idx + 1] - z0;
+  if (rowptr) {
+    CK(cudaMemcpy(rowptr, g->rowptr + n0, sizeof(int32_t) * (N + 1), cudaMemcpyDeviceToHost));
+    for (int32_t i = 0; i <= N; ++i) rowptr[i] -= (int32_t)z0;
+  }
+  if (colind) {
+    CK(cudaMemcpy(colind, g->colind + z0, sizeof(int32_t) * Z, cudaMemcpyDeviceToHost));
+    for (int64_t k = 0; k < Z; ++k) colind[k] -= n0;
+  }
+  if (deg) CK(cudaMemcpy(deg, g->deg + n0, sizeof(int32_t) * N, cudaMemcpyDeviceToHost));
+  if (dinv) CK(cudaMemcpy(dinv, g->dinv + n0, sizeof(float) * N, cudaMemcpyDeviceToHost));
+  if (vals) CK(cudaMemcpy(vals, g->vals + z0, sizeof(float) * Z, cudaMemcpyDeviceToHost));
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- model create
+extern "C" mars_status mars_nccl_get_unique_id(void* out128) {
+  if (!out128) return fail(MARS_EINVAL, "out is NULL");
+  if (!nccl_load()) return fail(MARS_ENCCL, "libnccl.so.2 not loadable");
+  ncclUniqueId id;
+  ncclResult_t r = g_nccl.GetUniqueId(&id);
+  if (r != ncclSuccess) return fail(MARS_ENCCL, "ncclGetUniqueId failed (%d)", (int)r);
+  memcpy(out128, &id, sizeof id);
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** out) {
+  if (!cfg || !out) return fail(MARS_EINVAL, "NULL argument");
+  *out = nullptr;
+  if (!valid_F(cfg->in_dim)) return fail(MARS_EINVAL, "in_dim %d unsupported", cfg->in_dim);
+  if (!valid_H(cfg->hidden_dim)) return fail(MARS_EINVAL, "hidden_dim %d unsupported", cfg->hidden_dim);
+  if (cfg->num_layers != 3) return fail(MARS_EINVAL, "num_layers must be 3 (P:L101, c10)");
+  if (cfg->precision != MARS_FP32) return fail(MARS_EINVAL, "precision %d not built", cfg->precision);
+  if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
+    return fail(MARS_EINVAL, "bad world_size/rank");
+  if (cfg->world_size > 1 && !cfg->nccl_unique_id)
+    return fail(MARS_EINVAL, "world_size > 1 needs nccl_unique_id");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "no CUDA device (libmars has no CPU fallback)");
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) return fail(MARS_EINVAL, "bad device");
+  CK(cudaSetDevice(cfg->device));
+  auto* m = new mars_dgi();
+  std::unique_ptr<mars_dgi> guard(m);
+  m->cfg = *cfg;
+  m->cfg.init_params = nullptr;
+  m->cfg.nccl_unique_id = nullptr;
+  m->F = cfg->in_dim;
+  m->H = cfg->hidden_dim;
+  m->P = mars_num_params(m->F, m->H);
+  CK(cudaStreamCreateWithFlags(&m->own_stream, cudaStreamNonBlocking));
+  m->stream = m->own_stream;
+  CK(dalloc(&m->params, m->P));
+  CK(dalloc(&m->adam_m, m->P));
+  CK(dalloc(&m->adam_v, m->P));
+  CK(dalloc(&m->grads, m->P + 1));
+  CK(dalloc(&m->norm_part, 160));
+  CK(dalloc(&m->finite_flag, 1));
+  CK(dalloc(&m->d_sp, 1));
+  CK(cudaMallocHost(&m->h_sp, sizeof(StepParams) * m->sp_ring));
+  m->sp_ev = new cudaEvent_t[m->sp_ring];
+  for (int i = 0; i < m->sp_ring; ++i) {
+    CK(cudaEventCreateWithFlags(&m->sp_ev[i], cudaEventDisableTiming));
+    CK(cudaEventRecord(m->sp_ev[i], m->stream));
+  }
+  cudaStream_t s = m->stream;
+  CK(cudaMemsetAsync(m->adam_m, 0, sizeof(float) * m->P, s));
+  CK(cudaMemsetAsync(m->adam_v, 0, sizeof(float) * m->P, s));
+  CK(cudaMemsetAsync(m->grads, 0, sizeof(float) * (m->P + 1), s));
+  if (cfg->init_params) {
+    CK(cudaMemcpyAsync(m->params, cfg->init_params, sizeof(float) * m->P, cudaMemcpyHostToDevice, s));
+  } else {
+    int64_t off = 0;
+    for (int t = 1; t <= 4; ++t) {
+      int fin = t == 1 ? m->F : m->H;
+      int64_t n = (int64_t)fin * m->H;
+      float b = (float)std::sqrt(6.0 / (double)(fin + m->H));
+      k_xavier<<<cdiv(n, 256), 256, 0, s>>>(m->params + off, n, cfg->seed, (uint64_t)t, b);
+      off += n;
+    }
+    k_fill<<<1, 32, 0, s>>>(m->params + off, 3, 0.25f);
+    CK(cudaGetLastError());
+  }
+  CK(cudaStreamSynchronize(s));
+  if (cfg->world_size > 1) {
+    if (!nccl_load()) return fail(MARS_ENCCL, "libnccl.so.2 not loadable");
+    ncclUniqueId id;
+    memcpy(&id, cfg->nccl_unique_id, sizeof id);
+    ncclResult_t r = g_nccl.CommInitRank(&m->comm, cfg->world_size, id, cfg->rank);
+    if (r != ncclSuccess)
+      return fail(MARS_ENCCL, "ncclCommInitRank: %s",
+                  g_nccl.GetErrorString ? g_nccl.GetErrorString(r) : "error");
+  }
+  *out = guard.release();
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_set_stream(mars_dgi* m, void* stream) {
+  if (mars_status st = check_dgi(m)) return st;
+  m->stream = stream ? static_cast<cudaStream_t>(stream) : m->own_stream;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable) {
+  if (mars_status st = check_dgi(m)) return st;
+  m->capture = enable != 0;
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- workspaces
+static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
+  Workspace& w = m->ws;
+  if (w.Nt >= g->Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks && w.nbuckets >= g->dev.nbuckets &&
+      w.F == m->F && w.H == m->H)
+    return MARS_OK;
+  if (m->exec) {
+    cudaGraphExecDestroy(m->exec);
+    m->exec = nullptr;
+    m->exec_graph = 0;
+  }
+  CK(cudaStreamSynchronize(m->stream));
+  w.release();
+  int64_t Nt = g->Nt, R = 2 * Nt;
+  int F = m->F, H = m->H, G = g->G, nch = g->dev.nchunks, nb = g->dev.nbuckets;
+  auto al = [&](void** p, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMalloc(p, bytes ? bytes : 8);
+    if (e == cudaSuccess) w.owned.push_back(*p);
+    return e;
+  };
+  CK(al((void**)&w.Y1, sizeof(float) * R * F));
+  for (int l = 0; l < 3; ++l) CK(al((void**)&w.Z[l], sizeof(float) * R * H));
+  for (int l = 0; l < 2; ++l) CK(al((void**)&w.Y23[l], sizeof(float) * R * H));
+  CK(al((void**)&w.dZ, sizeof(float) * R * H));
+  CK(al((void**)&w.dY, sizeof(float) * R * H));
+  CK(al((void**)&w.perm, sizeof(int32_t) * Nt));
+  CK(al((void**)&w.pw.keys, sizeof(uint64_t) * Nt));
+  CK(al((void**)&w.pw.bucket, sizeof(int32_t) * Nt));
+  CK(al((void**)&w.pw.bcnt, sizeof(int32_t) * (nb + 1)));
+  CK(al((void**)&w.pw.bstart, sizeof(int32_t) * (nb + 1)));
+  CK(al((void**)&w.pw.bcur, sizeof(int32_t) * (nb + 1)));
+  CK(al((void**)&w.pw.members, sizeof(int32_t) * Nt));
+  CK(al(&w.pw.scan_tmp, scan_tmp_bytes(nb + 1)));
+  HeadWork& h = w.hw;
+  CK(al((void**)&h.colsum_part, sizeof(double) * nch * H));
+  CK(al((void**)&h.dv_part, sizeof(double) * nch * H));
+  CK(al((void**)&h.loss_part, sizeof(double) * nch));
+  CK(al((void**)&h.s, sizeof(float) * G * H));
+  CK(al((void**)&h.v, sizeof(float) * G * H));
+  CK(al((void**)&h.dm, sizeof(float) * G * H));
+  CK(al((void**)&h.dv, sizeof(float) * G * H));
+  CK(al((void**)&h.dvd, sizeof(double) * G * H));
+  CK(al((void**)&h.sd, sizeof(double) * G * H));
+  CK(al((void**)&h.dl, sizeof(float) * R));
+  int nsl = std::max(head_slots(g->dev), spmm_bwd_slots(g->dev));
+  for (int l = 0; l < 3; ++l) CK(al((void**)&w.slots[l], sizeof(double) * nsl));
+  h.slots = w.slots[2];
+  size_t tn = std::max(gemm_tn_partial_floats(R, F, H), gemm_tn_partial_floats(R, H, H));
+  CK(al((void**)&w.tn_part, sizeof(double) * tn));
+  w.tn_part_n = tn;
+  w.Nt = (int32_t)Nt;
+  w.G = G;
+  w.nchunks = nch;
+  w.nbuckets = nb;
+  w.F = F;
+  w.H = H;
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- the step schedule
+// Optional per-phase event profiler (mars_dgi_profile_step): an event is
+// recorded on the launching stream after every kernel group.
+struct Profiler {
+  std::vector<cudaEvent_t> ev;
+  std::vector<int32_t> phase;
+  cudaError_t mark(int ph, cudaStream_t s) {
+    cudaEvent_t e;
+    cudaError_t r = cudaEventCreate(&e);
+    if (r != cudaSuccess) return r;
+    ev.push_back(e);
+    phase.push_back(ph);
+    return cudaEventRecord(e, s);
+  }
+  ~Profiler() {
+    for (cudaEvent_t e : ev) cudaEventDestroy(e);
+  }
+};
+
+// Enqueues one full DGI step (a4-a14) on stream s.  Reads step scalars from m->d_sp.
+static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl,
+                                Profiler* prof = nullptr) {
+  const GraphDev& g = gr->dev;
+  Workspace& w = m->ws;
+  const int F = m->F, H = m->H;
+  const int64_t R = 2LL * g.Nt;
+  float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
+  float* Mp = m->params + (int64_t)F * H + 2LL * H * H;
+  float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
+  float* gW[3] = {m->grads, m->grads + (int64_t)F * H, m->grads + (int64_t)F * H + (int64_t)H * H};
+  float* gM = m->grads + (int64_t)F * H + 2LL * H * H;
+  float* galpha = m->grads + (int64_t)F * H + 3LL * H * H;
+  float* gloss = m->grads + m->P;
+  float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
+  cudaError_t e;
+#define RET(x) if ((e = (x)) != cudaSuccess) return e
+#define MARK(ph) if (prof) RET(prof->mark(ph, s))
+  MARK(-1);
+  // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM)
+  RET(launch_perm(g, m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
+  MARK(MARS_PH_PERM);
+  // a5-a7: forward, l = 1..3
+  for (int l = 0; l < 3; ++l) {
+    int Cin = l == 0 ? F : H;
+    const float* T = l == 0 ? g.X : w.Z[l - 1];
+    RET(launch_spmm_fwd(g, Cin, T, w.perm, alpha, l - 1, Ys[l], 1, s, nl));
+    MARK(MARS_PH_SPMM_FWD);
+    RET(gemm_nn(Ys[l], W[l], w.Z[l], R, H, Cin, s, nl));
+    MARK(MARS_PH_GEMM_FWD);
+  }
+  // a8-a11 + dZ3
+  int ns = 0;
+  RET(launch_head(g, H, w.Z[2], Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl));
+  RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
+  MARK(MARS_PH_HEAD);
+  // a12: backward, l = 3..1
+  for (int l = 2; l >= 0; --l) {
+    int Cin = l == 0 ? F : H;
+    RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
+    MARK(MARS_PH_GEMM_DW);
+    if (l > 0) {
+      RET(gemm_nt(w.dZ, W[l], w.dY, R, Cin, H, s, nl));
+      MARK(MARS_PH_GEMM_DY);
+      RET(launch_spmm_bwd(g, Cin, w.dY, w.Z[l - 1], alpha, l - 1, w.dZ, w.slots[l - 1], &ns, s, nl));
+      MARK(MARS_PH_SPMM_BWD);
+      RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
+      MARK(MARS_PH_REDUCE);
+    }
+  }
+  // a13: data-parallel gradient allreduce (grads + loss, pre-scaled by 1/B)
+  if (m->comm) {
+    ncclResult_t r = g_nccl.AllReduce(m->grads, m->grads, (size_t)(m->P + 1), ncclFloat32, ncclSum,
+                                      m->comm, s);
+    if (r != ncclSuccess) return cudaErrorUnknown;
+    MARK(MARS_PH_ALLREDUCE);
+  }
+  // a14: Adam
+  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads, m->P, m->cfg.beta1, m->cfg.beta2,
+                  m->cfg.eps, m->cfg.clip_norm, m->norm_part, m->d_sp, s, nl));
+  MARK(MARS_PH_ADAM);
+#undef MARK
+#undef RET
+  return cudaSuccess;
+}
+
+// Writes the step scalars for the next step into a pinned ring slot and
+// enqueues their copy to the device (the captured graph reads them there).
+static mars_status push_step_params(mars_dgi* m, uint64_t step_index, int64_t pair_base,
+                                    int64_t global_batch) {
+  cudaStream_t s = m->stream;
+  m->t += 1;
+  int slot = m->sp_next;
+  m->sp_next = (m->sp_next + 1) % m->sp_ring;
+  CK(cudaEventSynchronize(m->sp_ev[slot]));
+  StepParams& sp = m->h_sp[slot];
+  sp.step_index = step_index;
+  sp.pair_base = pair_base;
+  sp.inv_batch = (float)(1.0 / (double)global_batch);
+  double bc1 = 1.0 - std::pow((double)m->cfg.beta1, (double)m->t);
+  double bc2 = 1.0 - std::pow((double)m->cfg.beta2, (double)m->t);
+  sp.adam_step_size = (float)((double)m->cfg.lr / bc1);
+  sp.adam_bc2_sqrt = (float)std::sqrt(bc2);
+  CK(cudaMemcpyAsync(m->d_sp, &sp, sizeof sp, cudaMemcpyHostToDevice, s));
+  CK(cudaEventRecord(m->sp_ev[slot], s));
+  return MARS_OK;
+}
+
+static mars_status check_step_args(mars_dgi* m, const mars_graph* g, int64_t global_batch) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (mars_status st = check_graph(g)) return st;
+  if (g->F != m->F) return fail(MARS_EINVAL, "graph feat_dim %d != model in_dim %d", g->F, m->F);
+  if (g->device != m->cfg.device) return fail(MARS_EINVAL, "graph and model on different devices");
+  if (global_batch < g->G) return fail(MARS_EINVAL, "global_batch < graphs in this set");
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
+                                             int64_t pair_base, int64_t global_batch,
+                                             int32_t* phase_ids, float* phase_ms,
+                                             int32_t max_phases, int32_t* n_phases) {
+  if (mars_status st = check_step_args(m, g, global_batch)) return st;
+  if (!phase_ids || !phase_ms || !n_phases) return fail(MARS_EINVAL, "NULL output");
+  CK(cudaSetDevice(m->cfg.device));
+  if (mars_status st = ensure_ws(m, g)) return st;
+  if (mars_status st = push_step_params(m, step_index, pair_base, global_batch)) return st;
+  Profiler prof;
+  int nl = 0;
+  cudaError_t e = enqueue_step(m, g, m->stream, &nl, &prof);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "profile step: %s", cudaGetErrorString(e));
+  }
+  CK(cudaStreamSynchronize(m->stream));
+  int n = 0;
+  for (size_t k = 1; k < prof.ev.size() && n < max_phases; ++k, ++n) {
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, prof.ev[k - 1], prof.ev[k]));
+    phase_ids[n] = prof.phase[k];
+    phase_ms[n] = ms;
+  }
+  *n_phases = n;
+  m->last_launches = nl;
+  m->last_Nt = g->Nt;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
+                                     int64_t pair_base, int64_t global_batch, mars_step_out* out) {
+  if (mars_status st = check_step_args(m, g, global_batch)) return st;
+  CK(cudaSetDevice(m->cfg.device));
+  if (mars_status st = ensure_ws(m, g)) return st;
+  cudaStream_t s = m->stream;
+  if (mars_status st = push_step_params(m, step_index, pair_base, global_batch)) return st;
+
+  int nl = 0;
+  // Capture once a graph set is stepped twice in a row (pre-training reuses one
+  // set for many steps); a set seen once (streamed batches) runs eagerly.
+  bool replay = m->capture && ((m->exec && m->exec_graph == g->uid && m->exec_stream == s) ||
+                               m->prev_graph == g->uid);
+  m->prev_graph = g->uid;
+  if (replay) {
+    if (!m->exec || m->exec_graph != g->uid || m->exec_stream != s) {
+      if (m->exec) {
+        cudaGraphExecDestroy(m->exec);
+        m->exec = nullptr;
+      }
+      cudaGraph_t graph;
+      CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+      cudaError_t e = enqueue_step(m, g, s, &nl);
+      cudaError_t e2 = cudaStreamEndCapture(s, &graph);
+      if (e != cudaSuccess || e2 != cudaSuccess) {
+        if (e2 == cudaSuccess) cudaGraphDestroy(graph);
+        cudaGetLastError();
+        return fail(MARS_ECUDA, "step capture failed: %s",
+                    cudaGetErrorString(e != cudaSuccess ? e : e2));
+      }
+      cudaError_t e3 = cudaGraphInstantiate(&m->exec, graph, 0);
+      cudaGraphDestroy(graph);
+      CK(e3);
+      m->exec_graph = g->uid;
+      m->exec_stream = s;
+      m->exec_launches = nl;
+    }
+    CK(cudaGraphLaunch(m->exec, s));
+    nl = (int)m->exec_launches;
+  } else {
+    cudaError_t e = enqueue_step(m, g, s, &nl);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(m->comm && e == cudaErrorUnknown ? MARS_ENCCL : MARS_ECUDA, "step: %s",
+                  cudaGetErrorString(e));
+    }
+  }
+  m->last_launches = nl;
+  m->last_Nt = g->Nt;
+  if (out && (out->loss || out->grads || out->perms)) {
+    float loss = 0.f;
+    CK(cudaMemcpyAsync(&loss, m->grads + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+    if (out->grads)
+      CK(cudaMemcpyAsync(out->grads, m->grads, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
+    if (out->perms)
+      CK(cudaMemcpyAsync(out->perms, m->ws.perm, sizeof(int32_t) * g->Nt, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (out->perms)
+      for (int gi = 0; gi < g->G; ++gi)
+        for (int32_t i = g->h_node_off[gi]; i < g->h_node_off[gi + 1]; ++i)
+          out->perms[i] -= g->h_node_off[gi];
+    if (out->loss) *out->loss = loss;
+    if (!std::isfinite(loss)) return fail(MARS_ENUMERIC, "non-finite loss");
+  }
+  return MARS_OK;
+}
+
+extern "C" int64_t mars_dgi_last_launches(const mars_dgi* m) {
+  return (m && m->tag == kTagDgi) ? m->last_launches : -1;
+}
+
+// ---------------------------------------------------------------- encode (a15)
+extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (mars_status st = check_graph(g)) return st;
+  if (!emb) return fail(MARS_EINVAL, "embeddings is NULL");
+  if (g->F != m->F) return fail(MARS_EINVAL, "feat_dim mismatch");
+  CK(cudaSetDevice(m->cfg.device));
+  if (mars_status st = ensure_ws(m, g)) return st;
+  const GraphDev& gd = g->dev;
+  Workspace& w = m->ws;
+  cudaStream_t s = m->stream;
+  const int F = m->F, H = m->H;
+  float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
+  float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
+  float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
+  int nl = 0;
+  for (int l = 0; l < 3; ++l) {
+    int Cin = l == 0 ? F : H;
+    const float* T = l == 0 ? gd.X : w.Z[l - 1];
+    CK(launch_spmm_fwd(gd, Cin, T, nullptr, alpha, l - 1, Ys[l], 0, s, &nl));
+    CK(gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
+  }
+  CK(launch_prelu(w.Z[2], alpha, 2, w.dY, (int64_t)gd.Nt * H, s, &nl));
+  CK(cudaMemcpyAsync(emb, w.dY, sizeof(float) * (size_t)gd.Nt * H, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  m->last_Nt = 0;
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- hooks / state
+extern "C" mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t layer, float* Y,
+                                                   float* Z) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (layer < 1 || layer > 3) return fail(MARS_EINVAL, "layer must be 1..3");
+  if (!m->ws.Y1 || !m->last_Nt) return fail(MARS_ESTATE, "no step has run since the last encode");
+  CK(cudaSetDevice(m->cfg.device));
+  CK(cudaStreamSynchronize(m->stream));
+  int64_t R = 2LL * m->last_Nt;
+  const float* Ys[3] = {m->ws.Y1, m->ws.Y23[0], m->ws.Y23[1]};
+  int Cin = layer == 1 ? m->F : m->H;
+  if (Y) CK(cudaMemcpy(Y, Ys[layer - 1], sizeof(float) * R * Cin, cudaMemcpyDeviceToHost));
+  if (Z) CK(cudaMemcpy(Z, m->ws.Z[layer - 1], sizeof(float) * R * m->H, cudaMemcpyDeviceToHost));
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_get_state(const mars_dgi* m, float* params, float* am, float* av,
+                                          int64_t* t) {
+  if (mars_status st = check_dgi(m)) return st;
+  CK(cudaSetDevice(m->cfg.device));
+  CK(cudaStreamSynchronize(m->stream));
+  if (params) CK(cudaMemcpy(params, m->params, sizeof(float) * m->P, cudaMemcpyDeviceToHost));
+  if (am) CK(cudaMemcpy(am, m->adam_m, sizeof(float) * m->P, cudaMemcpyDeviceToHost));
+  if (av) CK(cudaMemcpy(av, m->adam_v, sizeof(float) * m->P, cudaMemcpyDeviceToHost));
+  if (t) *t = m->t;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_set_state(mars_dgi* m, const float* params, const float* am,
+                                          const float* av, int64_t t) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (t < 0) return fail(MARS_EINVAL, "t < 0");
+  CK(cudaSetDevice(m->cfg.device));
+  CK(cudaStreamSynchronize(m->stream));
+  if (params) CK(cudaMemcpy(m->params, params, sizeof(float) * m->P, cudaMemcpyHostToDevice));
+  if (am) CK(cudaMemcpy(m->adam_m, am, sizeof(float) * m->P, cudaMemcpyHostToDevice));
+  if (av) CK(cudaMemcpy(m->adam_v, av, sizeof(float) * m->P, cudaMemcpyHostToDevice));
+  m->t = t;
+  return MARS_OK;
+}
+
+extern "C" void mars_free(void* h) {
+  if (!h) return;
+  uint64_t tag = *static_cast<uint64_t*>(h);
+  if (tag == kTagGraph) {
+    auto* g = static_cast<mars_graph*>(h);
+    cudaSetDevice(g->device);
+    cudaDeviceSynchronize();
+    g->tag = kTagDead;
+    delete g;
+  } else if (tag == kTagDgi) {
+    auto* m = static_cast<mars_dgi*>(h);
+    cudaSetDevice(m->cfg.device);
+    cudaStreamSynchronize(m->stream);
+    m->tag = kTagDead;
+    delete m;
+  }
+}

@@ -1,0 +1,333 @@
+"""Thin ctypes binding of libmars.so (include/mars.h) -- argument marshalling only.
+
+Every step of the hot path runs in the library's sm_100a kernels; there is no
+CPU fallback.  If libmars.so is missing this module raises on import-time use
+(``lib()``), and every compute call raises ``MarsError`` with the library's
+status when no CUDA device is usable.
+
+Names follow the C ABI: ``graph_load``, ``dgi_create``, ``dgi_step``,
+``encode``, ``free`` (+ the test hooks ``graph_export_csr`` and
+``dgi_export_activations``).  ``Graph`` / ``DGI`` wrap the handles.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libmars.so")
+
+MARS_OK, MARS_EINVAL, MARS_ENOMEM, MARS_ECUDA, MARS_ENCCL, MARS_ENUMERIC, MARS_ESTATE = range(7)
+MARS_FP32, MARS_BF16 = 0, 1
+_STATUS = {0: "OK", 1: "EINVAL", 2: "ENOMEM", 3: "ECUDA", 4: "ENCCL", 5: "ENUMERIC", 6: "ESTATE"}
+PHASES = ["perm", "spmm_fwd", "gemm_fwd", "head", "gemm_dw", "gemm_dy", "spmm_bwd", "allreduce",
+          "adam", "reduce"]
+
+
+class MarsError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"MARS_{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class GraphDesc(ctypes.Structure):
+    _fields_ = [("num_nodes", ctypes.c_int32), ("indptr", ctypes.c_void_p),
+                ("indices", ctypes.c_void_p), ("feat_dim", ctypes.c_int32),
+                ("features", ctypes.c_void_p)]
+
+
+class DgiConfig(ctypes.Structure):
+    _fields_ = [("in_dim", ctypes.c_int32), ("hidden_dim", ctypes.c_int32),
+                ("num_layers", ctypes.c_int32), ("precision", ctypes.c_int32),
+                ("lr", ctypes.c_double), ("beta1", ctypes.c_double), ("beta2", ctypes.c_double),
+                ("eps", ctypes.c_double), ("clip_norm", ctypes.c_double),
+                ("seed", ctypes.c_uint64), ("init_params", ctypes.c_void_p),
+                ("device", ctypes.c_int32), ("world_size", ctypes.c_int32),
+                ("rank", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
+
+
+class StepOut(ctypes.Structure):
+    _fields_ = [("loss", ctypes.c_void_p), ("grads", ctypes.c_void_p), ("perms", ctypes.c_void_p)]
+
+
+# symbol -> (restype, argtypes); every symbol include/mars.h declares
+SIGNATURES = {
+    "mars_last_error": (ctypes.c_char_p, []),
+    "mars_version": (ctypes.c_char_p, []),
+    "mars_num_params": (ctypes.c_int64, [ctypes.c_int32, ctypes.c_int32]),
+    "mars_graph_load": (ctypes.c_int, [ctypes.POINTER(GraphDesc), ctypes.c_int32, ctypes.c_int32,
+                                       ctypes.POINTER(ctypes.c_void_p)]),
+    "mars_graph_info": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                       ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_graph_size": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p,
+                                       ctypes.c_void_p]),
+    "mars_graph_export_csr": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32] + [ctypes.c_void_p] * 5),
+    "mars_dgi_config_default": (None, [ctypes.POINTER(DgiConfig)]),
+    "mars_dgi_create": (ctypes.c_int, [ctypes.POINTER(DgiConfig), ctypes.POINTER(ctypes.c_void_p)]),
+    "mars_nccl_get_unique_id": (ctypes.c_int, [ctypes.c_void_p]),
+    "mars_dgi_set_stream": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_set_graph_capture": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mars_dgi_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                     ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(StepOut)]),
+    "mars_encode": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_export_activations": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32,
+                                                   ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_get_state": (ctypes.c_int, [ctypes.c_void_p] * 4 + [ctypes.c_void_p]),
+    "mars_dgi_set_state": (ctypes.c_int, [ctypes.c_void_p] * 4 + [ctypes.c_int64]),
+    "mars_dgi_profile_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                             ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p,
+                                             ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
+    "mars_dgi_last_launches": (ctypes.c_int64, [ctypes.c_void_p]),
+    "mars_free": (None, [ctypes.c_void_p]),
+}
+
+_lib = None
+_lock = threading.Lock()
+
+
+def lib():
+    """Load libmars.so (fails loudly when the CUDA extension was not built)."""
+    global _lib
+    with _lock:
+        if _lib is None:
+            if not os.path.exists(LIB_PATH):
+                raise ImportError(f"{LIB_PATH} not built (run `make` or __graft_entry__.build())")
+            L = ctypes.CDLL(LIB_PATH)
+            for name, (res, args) in SIGNATURES.items():
+                fn = getattr(L, name)
+                fn.restype = res
+                fn.argtypes = args
+            _lib = L
+    return _lib
+
+
+def _check(st: int):
+    if st != MARS_OK:
+        raise MarsError(st, lib().mars_last_error().decode(errors="replace"))
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def version() -> str:
+    return lib().mars_version().decode()
+
+
+def num_params(F: int, H: int) -> int:
+    return int(lib().mars_num_params(F, H))
+
+
+# ------------------------------------------------------------------ graph sets
+class Graph:
+    """A device-resident set of op graphs (mars_graph*)."""
+
+    def __init__(self, handle, sizes, F):
+        self.handle = handle
+        self.sizes = list(sizes)
+        self.F = F
+
+    @property
+    def num_graphs(self):
+        return len(self.sizes)
+
+    @property
+    def total_nodes(self):
+        return int(sum(self.sizes))
+
+    def info(self):
+        G = ctypes.c_int32(); Nt = ctypes.c_int64(); Z = ctypes.c_int64(); F = ctypes.c_int32()
+        _check(lib().mars_graph_info(self.handle, ctypes.byref(G), ctypes.byref(Nt),
+                                     ctypes.byref(Z), ctypes.byref(F)))
+        return dict(num_graphs=G.value, total_nodes=Nt.value, nnz=Z.value, feat_dim=F.value)
+
+    def size(self, idx):
+        N = ctypes.c_int32(); Z = ctypes.c_int64()
+        _check(lib().mars_graph_size(self.handle, idx, ctypes.byref(N), ctypes.byref(Z)))
+        return N.value, Z.value
+
+    def export_csr(self, idx):
+        return graph_export_csr(self, idx)
+
+    def free(self):
+        if self.handle:
+            lib().mars_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def graph_load(graphs, device: int = 0) -> Graph:
+    """mars_graph_load: graphs = iterable of objects with num_nodes, indptr (int64
+    [N+1]), indices (int32), features (float32 [N, F])."""
+    graphs = list(graphs)
+    keep = []
+    descs = (GraphDesc * len(graphs))()
+    F = None
+    for i, g in enumerate(graphs):
+        ip = np.ascontiguousarray(g.indptr, np.int64)
+        ix = np.ascontiguousarray(g.indices, np.int32)
+        X = np.ascontiguousarray(g.features, np.float32)
+        keep += [ip, ix, X]
+        F = X.shape[1] if X.ndim == 2 else int(getattr(g, "feat_dim"))
+        descs[i] = GraphDesc(int(g.num_nodes), ip.ctypes.data, ix.ctypes.data if ix.size else None,
+                             int(F), X.ctypes.data)
+    h = ctypes.c_void_p()
+    _check(lib().mars_graph_load(descs, len(graphs), device, ctypes.byref(h)))
+    return Graph(h, [int(g.num_nodes) for g in graphs], F)
+
+
+def graph_export_csr(g: Graph, idx: int):
+    N, Z = g.size(idx)
+    rowptr = np.zeros(N + 1, np.int32); colind = np.zeros(max(Z, 1), np.int32)
+    deg = np.zeros(N, np.int32); dinv = np.zeros(N, np.float32); vals = np.zeros(max(Z, 1), np.float32)
+    _check(lib().mars_graph_export_csr(g.handle, idx, _ptr(rowptr), _ptr(colind), _ptr(deg),
+                                       _ptr(dinv), _ptr(vals)))
+    return dict(rowptr=rowptr, colind=colind[:Z], deg=deg, dinv=dinv, vals=vals[:Z])
+
+
+# ------------------------------------------------------------------ model
+def config_default() -> DgiConfig:
+    c = DgiConfig()
+    lib().mars_dgi_config_default(ctypes.byref(c))
+    return c
+
+
+def nccl_get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().mars_nccl_get_unique_id(buf))
+    return buf.raw
+
+
+class DGI:
+    """A DGI pre-training model instance (mars_dgi*)."""
+
+    def __init__(self, handle, F, H):
+        self.handle = handle
+        self.F, self.H = F, H
+        self.P = num_params(F, H)
+
+    def step(self, g: Graph, step_index: int, pair_base: int = 0, global_batch: int | None = None,
+             want_loss=False, want_grads=False, want_perms=False):
+        return dgi_step(self, g, step_index, pair_base, global_batch, want_loss, want_grads,
+                        want_perms)
+
+    def encode(self, g: Graph):
+        return encode(self, g)
+
+    def export_activations(self, layer: int):
+        return dgi_export_activations(self, layer)
+
+    def get_state(self):
+        p = np.zeros(self.P, np.float32); m = np.zeros(self.P, np.float32)
+        v = np.zeros(self.P, np.float32); t = ctypes.c_int64()
+        _check(lib().mars_dgi_get_state(self.handle, _ptr(p), _ptr(m), _ptr(v), ctypes.byref(t)))
+        return p, m, v, t.value
+
+    def set_state(self, params=None, m=None, v=None, t=0):
+        arrs = [None if a is None else np.ascontiguousarray(a, np.float32) for a in (params, m, v)]
+        _check(lib().mars_dgi_set_state(self.handle, *[None if a is None else _ptr(a) for a in arrs],
+                                        int(t)))
+
+    def set_stream(self, stream_ptr):
+        _check(lib().mars_dgi_set_stream(self.handle, stream_ptr))
+
+    def set_graph_capture(self, enable: bool):
+        _check(lib().mars_dgi_set_graph_capture(self.handle, 1 if enable else 0))
+
+    def profile_step(self, g: Graph, step_index: int, pair_base: int = 0,
+                     global_batch: int | None = None):
+        """mars_dgi_profile_step: [(phase name, device ms)] in schedule order."""
+        B = g.num_graphs if global_batch is None else int(global_batch)
+        ids = np.zeros(256, np.int32); ms = np.zeros(256, np.float32); n = ctypes.c_int32()
+        _check(lib().mars_dgi_profile_step(self.handle, g.handle, step_index & (2 ** 64 - 1),
+                                           int(pair_base), B, _ptr(ids), _ptr(ms), 256,
+                                           ctypes.byref(n)))
+        self._last_nt = g.total_nodes
+        return [(PHASES[int(i)], float(t)) for i, t in zip(ids[:n.value], ms[:n.value])]
+
+    def last_launches(self) -> int:
+        return int(lib().mars_dgi_last_launches(self.handle))
+
+    def free(self):
+        if self.handle:
+            lib().mars_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def dgi_create(in_dim=64, hidden_dim=256, precision=MARS_FP32, lr=1e-3, beta1=0.9, beta2=0.999,
+               eps=1e-8, clip_norm=0.0, seed=0, init_params=None, device=0, world_size=1, rank=0,
+               nccl_unique_id: bytes | None = None) -> DGI:
+    c = config_default()
+    c.in_dim, c.hidden_dim, c.num_layers, c.precision = in_dim, hidden_dim, 3, precision
+    c.lr, c.beta1, c.beta2, c.eps, c.clip_norm = lr, beta1, beta2, eps, clip_norm
+    c.seed = seed & (2 ** 64 - 1)
+    keep = None
+    if init_params is not None:
+        keep = np.ascontiguousarray(init_params, np.float32)
+        c.init_params = keep.ctypes.data
+    c.device, c.world_size, c.rank = device, world_size, rank
+    uid = None
+    if nccl_unique_id is not None:
+        uid = ctypes.create_string_buffer(nccl_unique_id, 128)
+        c.nccl_unique_id = ctypes.cast(uid, ctypes.c_void_p)
+    h = ctypes.c_void_p()
+    _check(lib().mars_dgi_create(ctypes.byref(c), ctypes.byref(h)))
+    del keep, uid
+    return DGI(h, in_dim, hidden_dim)
+
+
+def dgi_step(m: DGI, g: Graph, step_index: int, pair_base: int = 0, global_batch: int | None = None,
+             want_loss=False, want_grads=False, want_perms=False):
+    """mars_dgi_step.  Returns dict with the requested host outputs."""
+    B = g.num_graphs if global_batch is None else int(global_batch)
+    res = {}
+    out = StepOut()
+    if want_loss:
+        res["loss"] = np.zeros(1, np.float32); out.loss = res["loss"].ctypes.data
+    if want_grads:
+        res["grads"] = np.zeros(m.P, np.float32); out.grads = res["grads"].ctypes.data
+    if want_perms:
+        res["perms"] = np.zeros(g.total_nodes, np.int32); out.perms = res["perms"].ctypes.data
+    _check(lib().mars_dgi_step(m.handle, g.handle, step_index & (2 ** 64 - 1), int(pair_base), B,
+                               ctypes.byref(out)))
+    m._last_nt = g.total_nodes
+    if want_loss:
+        res["loss"] = float(res["loss"][0])
+    return res
+
+
+def encode(m: DGI, g: Graph) -> np.ndarray:
+    out = np.zeros((g.total_nodes, m.H), np.float32)
+    _check(lib().mars_encode(m.handle, g.handle, _ptr(out)))
+    m._last_nt = None          # encode overwrote the saved activations
+    return out
+
+
+def dgi_export_activations(m: DGI, layer: int):
+    """Test hook: the last step's (Y_l, Z_l), stacked [pos; neg], as fp32 arrays."""
+    if getattr(m, "_last_nt", None) is None:
+        raise MarsError(MARS_ESTATE, "no step has run")
+    R = 2 * m._last_nt
+    cin = m.F if layer == 1 else m.H
+    Y = np.zeros((R, cin), np.float32)
+    Z = np.zeros((R, m.H), np.float32)
+    _check(lib().mars_dgi_export_activations(m.handle, layer, _ptr(Y), _ptr(Z)))
+    return Y, Z
+
+
+def free(handle_obj):
+    handle_obj.free()
