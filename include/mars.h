@@ -127,6 +127,11 @@ MARS_API mars_status mars_nccl_get_unique_id(void* out128);
 /* Use `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream()) instead
  * of the library stream.  NULL restores the library stream. */
 MARS_API mars_status mars_dgi_set_stream(mars_dgi* m, void* cuda_stream);
+/* Dense-transform implementation (a6/a12).  MARS_GEMM_AUTO (default): tcgen05
+ * tensor cores with 3xTF32 splitting (fp32-accurate) when H == 256 and
+ * C_in in {64, 128, 256}, FFMA otherwise; MARS_GEMM_SIMT: always FFMA. */
+enum { MARS_GEMM_AUTO = 0, MARS_GEMM_SIMT = 1 };
+MARS_API mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl);
 /* Enables (1) / disables (0) CUDA-Graph capture of the step (default 1). */
 MARS_API mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable);
 
@@ -187,6 +192,17 @@ MARS_API mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, uin
                                            int64_t global_pair_base, int64_t global_batch,
                                            int32_t* phase_ids, float* phase_ms,
                                            int32_t max_phases, int32_t* n_phases);
+
+/* Test / micro-benchmark hook for the dense-transform kernels (a6, a12) in
+ * isolation, host buffers in and out, on `device`:
+ *   op 0 ("rows"): C[M×N] = A[M×K] · Bᵀ with B [N×K]   (forward / dY shape)
+ *   op 1 ("dw")  : C[K×N] = Aᵀ · B with A [M×K], B [M×N] (weight gradient;
+ *                  M = R rows reduced over, N must be 256)
+ * impl = MARS_GEMM_AUTO or MARS_GEMM_SIMT.  Runs `iters` timed launches after
+ * one warm-up and writes the mean device milliseconds per launch to *ms. */
+MARS_API mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl, const float* A,
+                                     const float* B, float* C, int64_t M, int32_t N, int32_t K,
+                                     int32_t iters, float* ms);
 
 /* Kernel launches enqueued by the most recent mars_dgi_step (for reporting). */
 MARS_API int64_t mars_dgi_last_launches(const mars_dgi* m);

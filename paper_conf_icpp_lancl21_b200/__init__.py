@@ -4,6 +4,7 @@ The product is ``libmars.so`` (CUDA kernels + C ABI, ``include/mars.h``); this
 package holds it and a thin ctypes binding (``mars.py``) with the ABI's names.
 It never imports ``oracle/`` and has no CPU fallback.
 """
-from .mars import (DGI, Graph, MarsError, MARS_BF16, MARS_FP32, config_default, dgi_create,  # noqa: F401
-                   dgi_export_activations, dgi_step, encode, free, graph_export_csr, graph_load,
-                   lib, nccl_get_unique_id, num_params, version, LIB_PATH, SIGNATURES)
+from .mars import (DGI, Graph, MarsError, MARS_BF16, MARS_FP32, PHASES, config_default,  # noqa: F401
+                   debug_gemm, dgi_create, dgi_export_activations, dgi_step, encode, free,
+                   graph_export_csr, graph_load, lib, nccl_get_unique_id, num_params, version,
+                   LIB_PATH, SIGNATURES)

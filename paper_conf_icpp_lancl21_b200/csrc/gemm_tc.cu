@@ -1,0 +1,537 @@
+// a6 / a12 on the 5th-generation tensor cores: the dense transforms of Eq. 1
+// -- Z_l = Y_l·W_l, dY_l = dZ_l·W_lᵀ, dW_l = Y_lᵀ·dZ_l -- at fp32
+// accuracy with 3xTF32 (reading c18: the fp32 reference precision).
+//
+// Each fp32 operand is split a = hi + lo with hi = tf32_rn(a) and lo = a - hi
+// (exact in fp32); D += A_hi·B_hi + A_hi·B_lo + A_lo·B_hi on tcgen05.mma
+// kind::tf32 with fp32 accumulation in TMEM.  The dropped lo·lo term and the
+// tf32 rounding of lo are ~2^-22 relative.
+//
+// Operands arrive by TMA with 128-byte swizzle.  For a 4-byte type the
+// swizzle atom "8 rows x 128 B" is the same bytes whether the 32 contiguous
+// elements are read as the K dimension (K-major) or the M/N dimension
+// (MN-major), so row-major activations feed both the forward (K-major A) and
+// the weight-gradient (MN-major A and B, reduction over rows) without
+// transposes -- only the UMMA descriptors differ.  The lo parts are written by
+// converter warps in place of / beside the TMA tile (position-preserving, so
+// the swizzle needs no remapping), then fence.proxy.async hands them to MMA.
+//
+// k_tc_rows  : C[M×N] = A[M×K]·Bᵀ, B [N×K] = weights pre-split (hi/lo arrays).
+//              Persistent over 128-row tiles; warp 0 TMA, warp 1 MMA issuer,
+//              warps 2-3 split A, warps 4-7 epilogue (TMEM -> registers ->
+//              global); double-buffered TMEM accumulators so the epilogue of
+//              tile i overlaps the main loop of tile i+1.
+// k_tc_dw    : per CTA one chunk of the R = 2ΣN rows, D = dZ_chunkᵀ·Y_chunk
+//              [256 × Cin] in two TMEM accumulators (M = 128 halves of H),
+//              written as an fp32 partial; k_dw_reduce sums the partials in a
+//              fixed order in fp64 and transposes into dW [Cin × H].
+#include <cudaTypedefs.h>
+
+#include <cstdlib>
+#include <mutex>
+
+#include "common.cuh"
+#include "internal.cuh"
+#include "tc_ptx.cuh"
+
+namespace mars {
+namespace {
+
+using namespace tc;
+
+constexpr int kBM = 128;        // tile rows (UMMA M)
+constexpr int kBK = 32;         // fp32 elements per 128-byte swizzle row
+constexpr int kThreads = 256;
+
+// ---------------------------------------------------------------- k_tc_rows
+template <int N>
+struct RowsCfg {
+  static constexpr int kStages = N > 128 ? 2 : 3;
+  static constexpr int A_BYTES = kBM * kBK * 4;       // 16 KB
+  static constexpr int B_BYTES = N * kBK * 4;
+  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int SMEM = kStages * STAGE + 1024 + 256;
+  static constexpr uint32_t TMEM_COLS = (2 * N) <= 32 ? 32 : (2 * N) <= 64 ? 64 : (2 * N) <= 128 ? 128
+                                        : (2 * N) <= 256 ? 256 : 512;
+};
+
+template <int N>
+__global__ void __launch_bounds__(kThreads, 1)
+k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBhi,
+          const __grid_constant__ CUtensorMap tmBlo, float* __restrict__ C, int32_t M, int32_t K) {
+  using Cfg = RowsCfg<N>;
+  constexpr int S = Cfg::kStages;
+  extern __shared__ uint8_t smem_raw[];
+  // 1024-byte alignment for the 128-byte swizzle atoms, by pointer arithmetic on
+  // the shared array itself so every access stays in the shared window (LDS/STS).
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;            // TMA landed            (count 1 + tx)
+  uint64_t* conv = bars + S;        // A split done          (count 2 warps)
+  uint64_t* empty = bars + 2 * S;   // MMA done with stage   (commit)
+  uint64_t* tfull = bars + 3 * S;   // accumulator ready     (commit)   [2]
+  uint64_t* tempty = bars + 3 * S + 2;  // accumulator drained (4 warps) [2]
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 4);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ntiles = (M + kBM - 1) / kBM;
+  const int nk = K / kBK;
+  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stAlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto stB = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
+  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 2);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 4);
+    }
+    fence_mbar_init();
+    tma_prefetch(&tmA);
+    tma_prefetch(&tmBhi);
+    tma_prefetch(&tmBlo);
+  }
+  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer
+      int s = 0;
+      uint32_t ph = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x)
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&empty[s], ph ^ 1);
+          mbar_expect_tx(&full[s], Cfg::A_BYTES + 2 * Cfg::B_BYTES);
+          tma_load_2d(stA(s), &tmA, kb * kBK, t * kBM, &full[s]);
+          tma_load_2d(stB(s), &tmBhi, kb * kBK, 0, &full[s]);
+          tma_load_2d(stBlo(s), &tmBlo, kb * kBK, 0, &full[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {                                         // ---- MMA issuer
+      constexpr uint32_t idesc = idesc_tf32(kBM, N, false, false);
+      int s = 0;
+      uint32_t ph = 0;
+      int acc = 0;
+      uint32_t aph = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        mbar_wait(&tempty[acc], aph ^ 1);
+        tc_fence_after();
+        const uint32_t d = tbase + acc * N;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&conv[s], ph);
+          tc_fence_after();
+          const uint32_t a = smem_u32(stA(s)), al = smem_u32(stAlo(s));
+          const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
+#pragma unroll
+          for (int k = 0; k < kBK / 8; ++k) {
+            const uint64_t ah = sdesc_sw128(a + 32 * k, 16, 1024);
+            const uint64_t alo = sdesc_sw128(al + 32 * k, 16, 1024);
+            const uint64_t bh = sdesc_sw128(b + 32 * k, 16, 1024);
+            const uint64_t blo = sdesc_sw128(bl + 32 * k, 16, 1024);
+            mma_tf32(d, ah, bh, idesc, (kb | k) != 0);
+            mma_tf32(d, ah, blo, idesc, 1);
+            mma_tf32(d, alo, bh, idesc, 1);
+          }
+          mma_commit(&empty[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+        mma_commit(&tfull[acc]);
+        acc ^= 1;
+        if (acc == 0) aph ^= 1;
+      }
+    }
+  } else if (warp < 4) {                                     // ---- split A = hi + lo
+    const int ct = threadIdx.x - 64;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x)
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&full[s], ph);
+        float4* a = reinterpret_cast<float4*>(stA(s));
+        float4* al = reinterpret_cast<float4*>(stAlo(s));
+#pragma unroll 4
+        for (int i = ct; i < Cfg::A_BYTES / 16; i += 64) {
+          float4 v = a[i];
+          float4 h = make_float4(to_tf32(v.x), to_tf32(v.y), to_tf32(v.z), to_tf32(v.w));
+          a[i] = h;
+          al[i] = make_float4(v.x - h.x, v.y - h.y, v.z - h.z, v.w - h.w);
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&conv[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+  } else {                                                   // ---- epilogue
+    const int q = warp & 3;
+    int acc = 0;
+    uint32_t aph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      mbar_wait(&tfull[acc], aph);
+      tc_fence_after();
+      const int64_t row = (int64_t)t * kBM + q * 32 + lane;
+#pragma unroll 1
+      for (int c0 = 0; c0 < N; c0 += 32) {
+        uint32_t r[32];
+        tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
+        tmem_wait_ld();
+        if (row < M) {
+          float4* dst = reinterpret_cast<float4*>(C + row * N + c0);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);
+      acc ^= 1;
+      if (acc == 0) aph ^= 1;
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tbase, Cfg::TMEM_COLS);
+  }
+}
+
+// ---------------------------------------------------------------- k_tc_dw
+constexpr int kDwBK = 16;        // rows of R per stage
+constexpr int kDwStages = 3;
+
+template <int CIN>
+struct DwCfg {
+  static constexpr int A_BYTES = 256 * kDwBK * 4;     // dZ: 8 boxes of 32 cols x 16 rows (16 KB)
+  static constexpr int B_BYTES = CIN * kDwBK * 4;     // Y : CIN/32 boxes
+  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int SMEM = kDwStages * STAGE + 1024 + 256;
+  static constexpr uint32_t TMEM_COLS = (2 * CIN) <= 32 ? 32 : (2 * CIN) <= 64 ? 64
+                                        : (2 * CIN) <= 128 ? 128 : (2 * CIN) <= 256 ? 256 : 512;
+  static constexpr int BOX = 32 * kDwBK * 4;          // bytes of one 32-col box (2 KB)
+};
+
+template <int CIN>
+__global__ void __launch_bounds__(kThreads, 1)
+k_tc_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
+        float* __restrict__ part, int32_t R, int32_t rows_per_chunk) {
+  using Cfg = DwCfg<CIN>;
+  constexpr int S = kDwStages;
+  constexpr int NCONV = 6;                                   // warps 2..7 split both operands
+  extern __shared__ uint8_t smem_raw[];
+  // 1024-byte alignment for the 128-byte swizzle atoms, by pointer arithmetic on
+  // the shared array itself so every access stays in the shared window (LDS/STS).
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;
+  uint64_t* conv = bars + S;
+  uint64_t* empty = bars + 2 * S;
+  uint64_t* tfull = bars + 3 * S;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int32_t r0 = blockIdx.x * rows_per_chunk;
+  const int32_t r1 = min(R, r0 + rows_per_chunk);
+  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
+  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stAlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto stB = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
+  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], NCONV);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(tfull, 1);
+    fence_mbar_init();
+    tma_prefetch(&tmDZ);
+    tma_prefetch(&tmY);
+  }
+  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer
+      int s = 0;
+      uint32_t ph = 0;
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
+        const int32_t row = r0 + kb * kDwBK;
+#pragma unroll
+        for (int bx = 0; bx < 8; ++bx) tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 32, row, &full[s]);
+#pragma unroll
+        for (int bx = 0; bx < CIN / 32; ++bx) tma_load_2d(stB(s) + bx * Cfg::BOX, &tmY, bx * 32, row, &full[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {                                         // ---- MMA issuer
+      constexpr uint32_t idesc = idesc_tf32(kBM, CIN, true, true);
+      int s = 0;
+      uint32_t ph = 0;
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&conv[s], ph);
+        tc_fence_after();
+        const uint32_t a = smem_u32(stA(s)), al = smem_u32(stAlo(s));
+        const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
+#pragma unroll
+        for (int k = 0; k < kDwBK / 8; ++k) {
+          // MN-major tf32: atoms of 4 K-rows x 128 B (512 B, SBO) ; 32-element
+          // MN blocks one box apart (LBO); one MMA (K = 8) spans two atoms.
+          const uint64_t bh = sdesc_sw128_b32(b + 1024 * k, Cfg::BOX, 512);
+          const uint64_t blo = sdesc_sw128_b32(bl + 1024 * k, Cfg::BOX, 512);
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {                      // two 128-row halves of H
+            const uint64_t ah = sdesc_sw128_b32(a + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
+            const uint64_t alo = sdesc_sw128_b32(al + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
+            const uint32_t d = tbase + h * CIN;
+            mma_tf32(d, ah, bh, idesc, (kb | k) != 0);
+            mma_tf32(d, ah, blo, idesc, 1);
+            mma_tf32(d, alo, bh, idesc, 1);
+          }
+        }
+        mma_commit(&empty[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+      mma_commit(tfull);
+    }
+  } else {                                                   // ---- split (warps 2..7)
+    const int ct = threadIdx.x - 64;
+    constexpr int NT = NCONV * 32;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int kb = 0; kb < nk; ++kb) {
+      mbar_wait(&full[s], ph);
+      float4* a = reinterpret_cast<float4*>(stA(s));
+      float4* al = reinterpret_cast<float4*>(stAlo(s));
+      for (int i = ct; i < (Cfg::A_BYTES + Cfg::B_BYTES) / 16; i += NT) {
+        float4* src = i < Cfg::A_BYTES / 16 ? a + i : reinterpret_cast<float4*>(stB(s)) + (i - Cfg::A_BYTES / 16);
+        float4* dlo = i < Cfg::A_BYTES / 16 ? al + i : reinterpret_cast<float4*>(stBlo(s)) + (i - Cfg::A_BYTES / 16);
+        float4 v = *src;
+        float4 hv = make_float4(to_tf32(v.x), to_tf32(v.y), to_tf32(v.z), to_tf32(v.w));
+        *src = hv;
+        *dlo = make_float4(v.x - hv.x, v.y - hv.y, v.z - hv.z, v.w - hv.w);
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&conv[s]);
+      if (++s == S) { s = 0; ph ^= 1; }
+    }
+    if (warp >= 4) {                                         // ---- epilogue (warps 4..7)
+      const int q = warp & 3;
+      float* out = part + (int64_t)blockIdx.x * 256 * CIN;
+      if (nk > 0) {
+        mbar_wait(tfull, 0);
+        tc_fence_after();
+      }
+#pragma unroll 1
+      for (int h = 0; h < 2; ++h) {
+        const int hrow = h * 128 + q * 32 + lane;
+#pragma unroll 1
+        for (int c0 = 0; c0 < CIN; c0 += 32) {
+          uint32_t r[32];
+          if (nk > 0) {
+            tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + h * CIN + c0, r);
+            tmem_wait_ld();
+          } else {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) r[j] = 0u;
+          }
+          float4* dst = reinterpret_cast<float4*>(out + (int64_t)hrow * CIN + c0);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tbase, Cfg::TMEM_COLS);
+  }
+}
+
+// dW[c][h] = Σ_chunk part[chunk][h][c], fixed order, fp64.
+__global__ void k_dw_reduce(const float* __restrict__ part, int nchunk, int CIN,
+                            float* __restrict__ dW) {
+  int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;   // e = h * CIN + c
+  if (e >= 256LL * CIN) return;
+  double t = 0.0;
+  for (int k = 0; k < nchunk; ++k) t += (double)part[(int64_t)k * 256 * CIN + e];
+  int h = (int)(e / CIN), c = (int)(e % CIN);
+  dW[(int64_t)c * 256 + h] = (float)t;
+}
+
+// hi / lo split of the weights for the B operand: Bt = Wᵀ [H × Cin] (forward)
+// and B = W [Cin × H] (dY), written once per step from the current params.
+__global__ void k_split_w(const float* __restrict__ W, int CIN, int H, float* __restrict__ Bt_hi,
+                          float* __restrict__ Bt_lo, float* __restrict__ B_hi,
+                          float* __restrict__ B_lo) {
+  int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;   // e = c * H + h
+  if (e >= (int64_t)CIN * H) return;
+  int c = (int)(e / H), h = (int)(e % H);
+  float w = W[e];
+  float hi = to_tf32(w), lo = w - hi;
+  B_hi[e] = hi;
+  B_lo[e] = lo;
+  Bt_hi[(int64_t)h * CIN + c] = hi;
+  Bt_lo[(int64_t)h * CIN + c] = lo;
+}
+
+// ---------------------------------------------------------------- host side
+PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+std::once_flag g_encode_once;
+
+bool encode_fn() {
+  std::call_once(g_encode_once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  });
+  return g_encode != nullptr;
+}
+
+// Row-major fp32 [rows × cols] with a {box_cols (= 32), box_rows} box and a
+// 128-byte swizzle: 16-byte atoms for K-major operands, 32-byte atoms for
+// MN-major tf32 operands (mn_major).
+bool tmap_2d(CUtensorMap* m, const float* base, int64_t rows, int64_t cols, int box_rows,
+             bool mn_major = false) {
+  if (!encode_fn()) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
+  cuuint32_t box[2] = {32, (cuuint32_t)box_rows};
+  cuuint32_t es[2] = {1, 1};
+  return g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides,
+                  box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  mn_major ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+int g_sms = 0;
+int num_sms() {
+  if (!g_sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (!g_sms) g_sms = 148;
+  }
+  return g_sms;
+}
+
+template <int N>
+cudaError_t rows_n(const float* A, const float* Bhi, const float* Blo, float* C, int64_t M, int K,
+                   cudaStream_t s) {
+  using Cfg = RowsCfg<N>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_tc_rows<N>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap ta, tbh, tbl;
+  if (!tmap_2d(&ta, A, M, K, kBM) || !tmap_2d(&tbh, Bhi, N, K, N) || !tmap_2d(&tbl, Blo, N, K, N))
+    return cudaErrorInvalidValue;
+  int ntiles = (int)((M + kBM - 1) / kBM);
+  int grid = std::min(ntiles, num_sms());
+  k_tc_rows<N><<<grid, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, C, (int32_t)M, K);
+  return cudaGetLastError();
+}
+
+template <int CIN>
+cudaError_t dw_c(const float* Y, const float* dZ, float* part, int nchunk, int64_t R, int rows,
+                 cudaStream_t s) {
+  using Cfg = DwCfg<CIN>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_tc_dw<CIN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap tdz, ty;
+  if (!tmap_2d(&tdz, dZ, R, 256, kDwBK, true) || !tmap_2d(&ty, Y, R, CIN, kDwBK, true))
+    return cudaErrorInvalidValue;
+  k_tc_dw<CIN><<<nchunk, kThreads, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+bool tc_supported(int K_or_cin, int N_or_h) {
+  return N_or_h == 256 && (K_or_cin == 64 || K_or_cin == 128 || K_or_cin == 256);
+}
+
+cudaError_t tc_split_weights(const float* W, int CIN, int H, float* Bt_hi, float* Bt_lo,
+                             float* B_hi, float* B_lo, cudaStream_t s, int* launches) {
+  count_launch(launches);
+  k_split_w<<<cdiv((int64_t)CIN * H, 256), 256, 0, s>>>(W, CIN, H, Bt_hi, Bt_lo, B_hi, B_lo);
+  return cudaGetLastError();
+}
+
+// C[M×N] = A[M×K] · Bᵀ with B = (B_hi + B_lo) [N×K].
+cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, float* C,
+                         int64_t M, int N, int K, cudaStream_t s, int* launches) {
+  count_launch(launches);
+  if (K % kBK) return cudaErrorInvalidValue;
+  switch (N) {
+    case 64: return rows_n<64>(A, B_hi, B_lo, C, M, K, s);
+    case 128: return rows_n<128>(A, B_hi, B_lo, C, M, K, s);
+    case 256: return rows_n<256>(A, B_hi, B_lo, C, M, K, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+int tc_dw_chunks(int64_t R) {
+  int64_t want = num_sms();
+  int64_t maxc = std::max<int64_t>(1, R / 256);
+  return (int)std::min(want, maxc);
+}
+
+size_t tc_dw_partial_floats(int64_t R, int CIN) { return (size_t)tc_dw_chunks(R) * 256 * CIN; }
+
+// dW [CIN × 256] = Yᵀ dZ with Y [R × CIN], dZ [R × 256].
+cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN,
+                       float* part, cudaStream_t s, int* launches) {
+  count_launch(launches, 2);
+  int nchunk = tc_dw_chunks(R);
+  int rows = (int)((R + nchunk - 1) / nchunk);
+  rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
+  nchunk = (int)((R + rows - 1) / rows);
+  cudaError_t e;
+  switch (CIN) {
+    case 64: e = dw_c<64>(Y, dZ, part, nchunk, R, rows, s); break;
+    case 128: e = dw_c<128>(Y, dZ, part, nchunk, R, rows, s); break;
+    case 256: e = dw_c<256>(Y, dZ, part, nchunk, R, rows, s); break;
+    default: return cudaErrorInvalidValue;
+  }
+  if (e != cudaSuccess) return e;
+  k_dw_reduce<<<cdiv(256LL * CIN, 256), 256, 0, s>>>(part, nchunk, CIN, dW);
+  return cudaGetLastError();
+}
+
+}  // namespace mars

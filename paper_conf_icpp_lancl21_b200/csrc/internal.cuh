@@ -115,6 +115,18 @@ size_t gemm_tn_partial_floats(int64_t R, int M, int N);
 cudaError_t gemm_tn(const float* A, const float* B, float* out, int64_t R, int M, int N,
                     double* partial, cudaStream_t s, int* launches);  // out[M×N] = Aᵀ B, A[R×M], B[R×N]
 
+// ---------------------------------------------------------------- gemm_tc.cu
+// 3xTF32 tcgen05 GEMMs (fp32-accurate).  Supported when H == 256 and
+// C_in in {64, 128, 256}.
+bool tc_supported(int cin, int h);
+cudaError_t tc_split_weights(const float* W, int CIN, int H, float* Bt_hi, float* Bt_lo,
+                             float* B_hi, float* B_lo, cudaStream_t s, int* launches);
+cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, float* C,
+                         int64_t M, int N, int K, cudaStream_t s, int* launches);
+size_t tc_dw_partial_floats(int64_t R, int CIN);
+cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN,
+                       float* part, cudaStream_t s, int* launches);
+
 // ---------------------------------------------------------------- head.cu
 struct HeadWork {
   double* colsum_part;  // [nchunks*H]

@@ -171,6 +171,9 @@ struct Workspace {
   double *slots[3] = {nullptr, nullptr, nullptr};
   double* tn_part = nullptr;
   size_t tn_part_n = 0;
+  // tcgen05 path: per-layer hi/lo weight splits (Wᵀ for the forward, W for dY)
+  float *wt_hi[3] = {}, *wt_lo[3] = {}, *w_hi[3] = {}, *w_lo[3] = {};
+  float* dw_part = nullptr;
   std::vector<void*> owned;
   void release() {
     for (void* p : owned) cudaFree(p);
@@ -196,6 +199,7 @@ struct mars_dgi {
   Workspace ws;
   const mars_graph* ws_graph = nullptr;
   bool capture = true;
+  int gemm_impl = 0;                // 0 auto (tcgen05 3xTF32 when supported), 1 SIMT FFMA
   cudaGraphExec_t exec = nullptr;
   uint64_t exec_graph = 0;          // uid of the graph set the exec was captured for
   uint64_t prev_graph = 0;          // uid of the graph set of the previous step
@@ -570,6 +574,18 @@ extern "C" mars_status mars_dgi_set_stream(mars_dgi* m, void* stream) {
   return MARS_OK;
 }
 
+extern "C" mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (impl != MARS_GEMM_AUTO && impl != MARS_GEMM_SIMT) return fail(MARS_EINVAL, "bad gemm impl");
+  if (impl != m->gemm_impl && m->exec) {
+    cudaGraphExecDestroy(m->exec);
+    m->exec = nullptr;
+    m->exec_graph = 0;
+  }
+  m->gemm_impl = impl;
+  return MARS_OK;
+}
+
 extern "C" mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable) {
   if (mars_status st = check_dgi(m)) return st;
   m->capture = enable != 0;
@@ -626,6 +642,15 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   size_t tn = std::max(gemm_tn_partial_floats(R, F, H), gemm_tn_partial_floats(R, H, H));
   CK(al((void**)&w.tn_part, sizeof(double) * tn));
   w.tn_part_n = tn;
+  for (int l = 0; l < 3; ++l) {
+    int64_t n = (int64_t)(l == 0 ? F : H) * H;
+    CK(al((void**)&w.wt_hi[l], sizeof(float) * n));
+    CK(al((void**)&w.wt_lo[l], sizeof(float) * n));
+    CK(al((void**)&w.w_hi[l], sizeof(float) * n));
+    CK(al((void**)&w.w_lo[l], sizeof(float) * n));
+  }
+  CK(al((void**)&w.dw_part, sizeof(float) * std::max(tc_dw_partial_floats(R, F),
+                                                      tc_dw_partial_floats(R, H))));
   w.Nt = (int32_t)Nt;
   w.G = G;
   w.nchunks = nch;
@@ -670,19 +695,33 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   float* gloss = m->grads + m->P;
   float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
   cudaError_t e;
-#define RET(x) if ((e = (x)) != cudaSuccess) return e
-#define MARK(ph) if (prof) RET(prof->mark(ph, s))
+#define RET(x)                                  \
+  do {                                          \
+    if ((e = (x)) != cudaSuccess) return e;     \
+  } while (0)
+#define MARK(ph)                                \
+  do {                                          \
+    if (prof) RET(prof->mark(ph, s));           \
+  } while (0)
   MARK(-1);
   // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM)
   RET(launch_perm(g, m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
   MARK(MARS_PH_PERM);
+  bool tc[3];
+  for (int l = 0; l < 3; ++l) {
+    int Cin = l == 0 ? F : H;
+    tc[l] = m->gemm_impl == 0 && tc_supported(Cin, H);
+    if (tc[l]) RET(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, nl));
+  }
+  MARK(MARS_PH_GEMM_FWD);
   // a5-a7: forward, l = 1..3
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     const float* T = l == 0 ? g.X : w.Z[l - 1];
     RET(launch_spmm_fwd(g, Cin, T, w.perm, alpha, l - 1, Ys[l], 1, s, nl));
     MARK(MARS_PH_SPMM_FWD);
-    RET(gemm_nn(Ys[l], W[l], w.Z[l], R, H, Cin, s, nl));
+    if (tc[l]) RET(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], R, H, Cin, s, nl));
+    else RET(gemm_nn(Ys[l], W[l], w.Z[l], R, H, Cin, s, nl));
     MARK(MARS_PH_GEMM_FWD);
   }
   // a8-a11 + dZ3
@@ -693,10 +732,12 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   // a12: backward, l = 3..1
   for (int l = 2; l >= 0; --l) {
     int Cin = l == 0 ? F : H;
-    RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
+    if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, w.dw_part, s, nl));
+    else RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
     MARK(MARS_PH_GEMM_DW);
     if (l > 0) {
-      RET(gemm_nt(w.dZ, W[l], w.dY, R, Cin, H, s, nl));
+      if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], w.dY, R, Cin, H, s, nl));
+      else RET(gemm_nt(w.dZ, W[l], w.dY, R, Cin, H, s, nl));
       MARK(MARS_PH_GEMM_DY);
       RET(launch_spmm_bwd(g, Cin, w.dY, w.Z[l - 1], alpha, l - 1, w.dZ, w.slots[l - 1], &ns, s, nl));
       MARK(MARS_PH_SPMM_BWD);
@@ -872,7 +913,12 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
     int Cin = l == 0 ? F : H;
     const float* T = l == 0 ? gd.X : w.Z[l - 1];
     CK(launch_spmm_fwd(gd, Cin, T, nullptr, alpha, l - 1, Ys[l], 0, s, &nl));
-    CK(gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
+    if (m->gemm_impl == 0 && tc_supported(Cin, H)) {
+      CK(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, &nl));
+      CK(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
+    } else {
+      CK(gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
+    }
   }
   CK(launch_prelu(w.Z[2], alpha, 2, w.dY, (int64_t)gd.Nt * H, s, &nl));
   CK(cudaMemcpyAsync(emb, w.dY, sizeof(float) * (size_t)gd.Nt * H, cudaMemcpyDeviceToHost, s));
@@ -919,6 +965,70 @@ extern "C" mars_status mars_dgi_set_state(mars_dgi* m, const float* params, cons
   if (am) CK(cudaMemcpy(m->adam_m, am, sizeof(float) * m->P, cudaMemcpyHostToDevice));
   if (av) CK(cudaMemcpy(m->adam_v, av, sizeof(float) * m->P, cudaMemcpyHostToDevice));
   m->t = t;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl, const float* A,
+                                       const float* B, float* C, int64_t M, int32_t N, int32_t K,
+                                       int32_t iters, float* ms) {
+  if (!A || !B || !C || M < 1 || N < 1 || K < 1 || (op != 0 && op != 1))
+    return fail(MARS_EINVAL, "bad debug_gemm arguments");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "no CUDA device");
+  }
+  CK(cudaSetDevice(device));
+  const bool tcp = impl == MARS_GEMM_AUTO && (op == 0 ? tc_supported(K, N) || tc_supported(N, K)
+                                                     : tc_supported(K, N));
+  size_t nA = (size_t)M * K, nB = op == 0 ? (size_t)N * K : (size_t)M * N;
+  size_t nC = op == 0 ? (size_t)M * N : (size_t)K * N;
+  float *dA, *dB, *dC, *bh, *bl, *bth, *btl, *part;
+  double* tpart;
+  CK(dalloc(&dA, nA));
+  CK(dalloc(&dB, nB));
+  CK(dalloc(&dC, nC));
+  CK(dalloc(&bh, (size_t)N * K));
+  CK(dalloc(&bl, (size_t)N * K));
+  CK(dalloc(&bth, (size_t)N * K));
+  CK(dalloc(&btl, (size_t)N * K));
+  size_t np = std::max(tc_dw_partial_floats(M, K), (size_t)1);
+  CK(dalloc(&part, np));
+  CK(dalloc(&tpart, gemm_tn_partial_floats(M, K, N)));
+  CK(cudaMemcpy(dA, A, sizeof(float) * nA, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(dB, B, sizeof(float) * nB, cudaMemcpyHostToDevice));
+  cudaStream_t s = nullptr;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  auto run = [&]() -> cudaError_t {
+    if (op == 0) {
+      if (tcp) {
+        cudaError_t e = tc_split_weights(dB, N, K, bth, btl, bh, bl, s, nullptr);
+        if (e != cudaSuccess) return e;
+        return tc_gemm_rows(dA, bh, bl, dC, M, N, K, s, nullptr);
+      }
+      return gemm_nt(dA, dB, dC, M, N, K, s, nullptr);
+    }
+    if (tcp) return tc_gemm_dw(dA, dB, dC, M, K, part, s, nullptr);
+    return gemm_tn(dA, dB, dC, M, K, N, tpart, s, nullptr);
+  };
+  cudaEvent_t e0, e1;
+  CK(cudaEventCreate(&e0));
+  CK(cudaEventCreate(&e1));
+  CK(run());
+  CK(cudaEventRecord(e0, s));
+  for (int i = 0; i < iters; ++i) CK(run());
+  CK(cudaEventRecord(e1, s));
+  CK(cudaStreamSynchronize(s));
+  float t = 0.f;
+  CK(cudaEventElapsedTime(&t, e0, e1));
+  if (ms) *ms = iters > 0 ? t / iters : 0.f;
+  CK(cudaMemcpy(C, dC, sizeof(float) * nC, cudaMemcpyDeviceToHost));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaStreamDestroy(s);
+  for (void* p : {(void*)dA, (void*)dB, (void*)dC, (void*)bh, (void*)bl, (void*)bth, (void*)btl,
+                  (void*)part, (void*)tpart})
+    cudaFree(p);
   return MARS_OK;
 }
 

@@ -70,6 +70,7 @@ SIGNATURES = {
     "mars_nccl_get_unique_id": (ctypes.c_int, [ctypes.c_void_p]),
     "mars_dgi_set_stream": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dgi_set_graph_capture": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mars_dgi_set_gemm_impl": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
     "mars_dgi_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                      ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(StepOut)]),
     "mars_encode": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
@@ -81,6 +82,10 @@ SIGNATURES = {
                                              ctypes.c_int64, ctypes.c_int64, ctypes.c_void_p,
                                              ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p]),
     "mars_dgi_last_launches": (ctypes.c_int64, [ctypes.c_void_p]),
+    "mars_debug_gemm": (ctypes.c_int, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
+                                       ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                       ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                       ctypes.c_int32, ctypes.c_void_p]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -239,6 +244,10 @@ class DGI:
     def set_stream(self, stream_ptr):
         _check(lib().mars_dgi_set_stream(self.handle, stream_ptr))
 
+    def set_gemm_impl(self, impl: str):
+        """'auto' (tcgen05 3xTF32 where supported) or 'simt' (FFMA everywhere)."""
+        _check(lib().mars_dgi_set_gemm_impl(self.handle, {"auto": 0, "simt": 1}[impl]))
+
     def set_graph_capture(self, enable: bool):
         _check(lib().mars_dgi_set_graph_capture(self.handle, 1 if enable else 0))
 
@@ -327,6 +336,24 @@ def dgi_export_activations(m: DGI, layer: int):
     Z = np.zeros((R, m.H), np.float32)
     _check(lib().mars_dgi_export_activations(m.handle, layer, _ptr(Y), _ptr(Z)))
     return Y, Z
+
+
+def debug_gemm(op: str, A, B, impl: str = "auto", iters: int = 0, device: int = 0):
+    """mars_debug_gemm: op 'rows' -> A[M×K]·Bᵀ (B [N×K]); op 'dw' -> Aᵀ·B (A [M×K],
+    B [M×N]).  Returns (C, mean ms per launch)."""
+    A = np.ascontiguousarray(A, np.float32)
+    B = np.ascontiguousarray(B, np.float32)
+    M, K = A.shape
+    if op == "rows":
+        N = B.shape[0]
+        C = np.zeros((M, N), np.float32)
+    else:
+        N = B.shape[1]
+        C = np.zeros((K, N), np.float32)
+    ms = ctypes.c_float()
+    _check(lib().mars_debug_gemm(device, 0 if op == "rows" else 1, {"auto": 0, "simt": 1}[impl],
+                                 _ptr(A), _ptr(B), _ptr(C), M, N, K, iters, ctypes.byref(ms)))
+    return C, ms.value
 
 
 def free(handle_obj):

@@ -1,0 +1,49 @@
+"""Dense-transform kernels in isolation (mars_debug_gemm) vs fp64 numpy:
+tcgen05 3xTF32 and FFMA paths, ragged row counts, both operand majors."""
+import numpy as np
+import pytest
+
+import paper_conf_icpp_lancl21_b200 as mars
+from tests.util import scaled_err
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("impl", ["auto", "simt"])
+@pytest.mark.parametrize("M,N,K", [(128, 256, 64), (1000, 256, 256), (4133, 256, 64),
+                                   (777, 64, 256), (300, 128, 256)])
+def test_rows(impl, M, N, K):
+    rng = np.random.default_rng(M + N + K)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    B = rng.standard_normal((N, K)).astype(np.float32)
+    C, _ = mars.debug_gemm("rows", A, B, impl)
+    ref = A.astype(np.float64) @ B.astype(np.float64).T
+    e = scaled_err(C, ref)
+    print(impl, M, N, K, e)
+    assert e < 5e-6
+
+
+@pytest.mark.parametrize("impl", ["auto", "simt"])
+@pytest.mark.parametrize("M,K", [(16, 64), (5000, 256), (40001, 64), (123457, 256)])
+def test_dw(impl, M, K):
+    rng = np.random.default_rng(M + K)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    B = rng.standard_normal((M, 256)).astype(np.float32)
+    C, _ = mars.debug_gemm("dw", A, B, impl)
+    ref = A.astype(np.float64).T @ B.astype(np.float64)
+    e = scaled_err(C, ref)
+    print(impl, M, K, e)
+    assert e < 5e-6
+
+
+def test_timing_report():
+    rng = np.random.default_rng(0)
+    R = 419232
+    for K in (64, 256):
+        A = rng.standard_normal((R, K)).astype(np.float32)
+        W = rng.standard_normal((256, K)).astype(np.float32)
+        D = rng.standard_normal((R, 256)).astype(np.float32)
+        for impl in ("auto", "simt"):
+            _, t1 = mars.debug_gemm("rows", A, W, impl, iters=5)
+            _, t2 = mars.debug_gemm("dw", A, D, impl, iters=5)
+            print(f"TIMING K={K} {impl}: rows {t1:.3f} ms  dw {t2:.3f} ms")

@@ -197,6 +197,12 @@ def test_bench_config_sampled():
     G = split_params(out["grads"], F, H)
     assert scaled_err(G["M"].reshape(H, H), dM) <= TOL
     assert abs(G["alpha"][2] - da3) <= TOL * max(abs(da3), 1e-12) * 10
+    # dW3 = Y3ᵀ dZ3 over all 2ΣN = 419k rows (the longest reduction of the step),
+    # stage-wise from the GPU's Y3 and the oracle's dZ3
+    Y3, _ = m.export_activations(3)
+    e = scaled_err(G["W3"].reshape(H, H), Y3.astype(np.float64).T @ dZ3)
+    print("bench-config dW3 stage-wise err", e)
+    assert e <= TOL
 
 
 def test_capture_replay_matches_eager():
