@@ -191,6 +191,7 @@ def run_mine(args):
     info = g.info()
     m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local, world_size=world,
                         rank=rank, nccl_unique_id=uid)
+    m.set_gemm_impl(args.gemm)
     # a dedicated (non-legacy) stream: libmars launches and captures on it and
     # torch's CUDA events are recorded on it
     stream = torch.cuda.Stream()
@@ -248,20 +249,36 @@ def run_mine(args):
     spmm_algo = sum(bb for _, bb in sp)
     spmm_gbs = spmm_algo / (spmm_ms / 1e3) / 1e9 if spmm_ms else None
     shares = {k: v / sum(per_step.values()) for k, v in per_step.items()}
-    kinds = {"gemm": sum(per_step.get(k, 0) for k in ("gemm_fwd", "gemm_dw", "gemm_dy")),
-             "spmm": spmm_ms}
-    if kinds["gemm"] >= kinds["spmm"]:
-        fl = sum(gflops.values())
-        ach = fl / (kinds["gemm"] / 1e3) / 1e12
-        roof = {"kernel": "gemm (fp32 FFMA: fwd Y·W, dY = dZ·Wᵀ, dW = Yᵀ·dZ)", "bound": "alu",
-                "achieved": ach, "peak": pk["ffma_tflops"], "unit": "TFLOP/s",
-                "frac": ach / pk["ffma_tflops"], "traffic": None,
-                "peak_source": FFMA_TFLOPS_NOTE, "share_of_step": kinds["gemm"] / sum(per_step.values())}
-    else:
-        roof = {"kernel": "spmm (fwd x3 + bwd x2)", "bound": "hbm", "achieved": spmm_gbs,
-                "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": spmm_gbs / pk["hbm_gbs"],
-                "traffic": None, "peak_source": pk["source"],
-                "share_of_step": spmm_ms / sum(per_step.values())}
+    step_total = sum(per_step.values())
+    gemm_ms = sum(per_step.get(k, 0) for k in ("gemm_fwd", "gemm_dw", "gemm_dy"))
+    head_ms = per_step.get("head", 0)
+    fl = sum(gflops.values())
+    # 3xTF32: three tf32 MMAs per fp32 product, so the fp32-equivalent tensor
+    # peak is the tf32 peak / 3; tf32 = bf16 x (1.1 / 2.25) nominal ratio.
+    tf32_peak = pk["bf16_tflops"] * (1.1 / 2.25)
+    gemm_peak = tf32_peak / 3.0 if args.gemm == "auto" else pk["ffma_tflops"]
+    gemm_ach = fl / (gemm_ms / 1e3) / 1e12 if gemm_ms else None
+    head_bytes = 16 * N * H                     # Z3 in, dZ3 out (stacked pos/neg)
+    head_gbs = head_bytes / (head_ms / 1e3) / 1e9 if head_ms else None
+    rooflines = {
+        "gemm": {"kernel": "dense transforms (Z = Y·W, dY = dZ·Wᵀ, dW = Yᵀ·dZ), "
+                           + ("tcgen05 3xTF32" if args.gemm == "auto" else "FFMA"),
+                 "bound": "tensor" if args.gemm == "auto" else "alu", "achieved": gemm_ach,
+                 "peak": gemm_peak, "unit": "TFLOP/s",
+                 "frac": gemm_ach / gemm_peak if gemm_ach else None, "traffic": None,
+                 "peak_source": ("measured bf16 x 1.1/2.25 (tf32) / 3 (3xTF32), fp32-equivalent"
+                                 if args.gemm == "auto" else FFMA_TFLOPS_NOTE),
+                 "algorithmic_flops_per_step": fl, "share_of_step": gemm_ms / step_total},
+        "spmm": {"kernel": "spmm (fwd x3 + bwd x2)", "bound": "hbm", "achieved": spmm_gbs,
+                 "peak": pk["hbm_gbs"], "unit": "GB/s",
+                 "frac": spmm_gbs / pk["hbm_gbs"] if spmm_gbs else None, "traffic": None,
+                 "peak_source": pk["source"], "share_of_step": spmm_ms / step_total},
+        "head": {"kernel": "head (readout, scores, BCE, head backward, dZ3)", "bound": "hbm",
+                 "achieved": head_gbs, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                 "frac": head_gbs / pk["hbm_gbs"] if head_gbs else None, "traffic": None,
+                 "peak_source": pk["source"], "share_of_step": head_ms / step_total},
+    }
+    roof = max(rooflines.values(), key=lambda r: r["share_of_step"])
     spmm_obj = {"achieved_gbs": spmm_gbs, "peak_gbs": pk["hbm_gbs"],
                 "frac": (spmm_gbs / pk["hbm_gbs"]) if spmm_gbs else None,
                 "algorithmic_bytes_per_step": spmm_algo, "ms_per_step": spmm_ms,
@@ -318,7 +335,7 @@ def run_mine(args):
                            "parallelism": f"dp{world}",
                            "l2": "inputs larger than L2 (activations ~%.1f GB/step)"
                                  % (2 * N * 4 * (F + 7 * H) / 1e9)},
-                "roofline": roof, "spmm": spmm_obj,
+                "roofline": roof, "rooflines": rooflines, "spmm": spmm_obj,
                 "phases_ms_per_step": per_step, "phase_share": shares,
                 "profiled_step_ms": prof_total / nprof,
                 "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches}
@@ -338,6 +355,8 @@ def main():
     ap.add_argument("--impl", default="mine", choices=["mine", "reference"])
     ap.add_argument("--graphs-per-gpu", type=int, default=16)
     ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--gemm", default="auto", choices=["auto", "simt"],
+                    help="dense-transform kernels: tcgen05 3xTF32 (auto) or FFMA (simt)")
     ap.add_argument("--profile-steps", type=int, default=5)
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-e2e", action="store_true")

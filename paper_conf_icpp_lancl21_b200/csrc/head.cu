@@ -10,7 +10,9 @@
 //   dv_g = Σ dl_i H3[i] + Σ dl~_i H3~[i]; dM = Σ_g dv_g s_gᵀ; ds = Mᵀ dv;
 //   dm = ds ⊙ s(1-s); dH3 = dl v_g + [pos] dm_g / N_g; dZ3 = dH3 ⊙ PReLU'(Z3)
 // Every cross-row reduction is two-stage with fixed-order fp64 combination
-// over row chunks that never straddle a graph (deterministic, no float atomics).
+// over row chunks (<= kChunkRows rows, never straddling a graph): deterministic,
+// no float atomics.  The per-graph second stages are small and latency-bound;
+// they are spread over G x 8 warps with independent accumulators.
 #include "common.cuh"
 #include "internal.cuh"
 
@@ -20,36 +22,58 @@ namespace {
 constexpr int kWarps = 8;
 
 // Stage 1 of m_g: per-chunk column sums of H3 over positive rows (fp64).
-// Block = H threads (one column each), one block per chunk.
+// Block = 256 threads: threads own columns c = tid % H, rows split across
+// 256 / H row-groups, combined in fixed order through shared memory.
 __global__ void k_colsum(const float* __restrict__ Z3, const float* __restrict__ alpha,
                          const int32_t* __restrict__ chunk_row, int H,
                          double* __restrict__ part) {
-  int c = threadIdx.x;
-  int ch = blockIdx.x;
-  float a = alpha[2];
-  double acc = 0.0;
-  for (int32_t r = chunk_row[ch]; r < chunk_row[ch + 1]; ++r)
-    acc += (double)prelu(Z3[(int64_t)r * H + c], a);
-  part[(int64_t)ch * H + c] = acc;
+  __shared__ double sh[256];
+  const int groups = 256 / H;
+  const int c = threadIdx.x % H, gr = threadIdx.x / H;
+  const int ch = blockIdx.x;
+  const float a = alpha[2];
+  double acc0 = 0.0, acc1 = 0.0;
+  const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
+  int32_t r = r0 + gr;
+  for (; r + groups < r1; r += 2 * groups) {
+    acc0 += (double)prelu(Z3[(int64_t)r * H + c], a);
+    acc1 += (double)prelu(Z3[(int64_t)(r + groups) * H + c], a);
+  }
+  if (r < r1) acc0 += (double)prelu(Z3[(int64_t)r * H + c], a);
+  sh[threadIdx.x] = acc0 + acc1;
+  __syncthreads();
+  if (gr == 0) {
+    double t = 0.0;
+    for (int k = 0; k < groups; ++k) t += sh[k * H + c];
+    part[(int64_t)ch * H + c] = t;
+  }
 }
 
-// Per graph: m, s = sig(m) (Eq. 4), v = M s (Eq. 5).  Block = H threads.
+// Per graph: m, s = sig(m) (Eq. 4), v = M s (Eq. 5).  Block = 256 threads.
 __global__ void k_readout(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
                           const int32_t* __restrict__ node_off, const float* __restrict__ M,
                           int H, double* __restrict__ sd, float* __restrict__ sf,
                           float* __restrict__ vf) {
-  extern __shared__ double sh_s[];
-  int g = blockIdx.x, c = threadIdx.x;
-  double acc = 0.0;
-  for (int ch = graph_chunk[g]; ch < graph_chunk[g + 1]; ++ch) acc += part[(int64_t)ch * H + c];
-  double Ng = (double)(node_off[g + 1] - node_off[g]);
-  double s = 1.0 / (1.0 + exp(-(acc / Ng)));
-  sh_s[c] = s;
-  sd[(int64_t)g * H + c] = s;
-  sf[(int64_t)g * H + c] = (float)s;
+  __shared__ double sh_s[256];
+  const int g = blockIdx.x;
+  const double Ng = (double)(node_off[g + 1] - node_off[g]);
+  for (int c = threadIdx.x; c < H; c += blockDim.x) {
+    double a0 = 0.0, a1 = 0.0;
+    int ch = graph_chunk[g];
+    const int ce = graph_chunk[g + 1];
+    for (; ch + 1 < ce; ch += 2) {
+      a0 += part[(int64_t)ch * H + c];
+      a1 += part[(int64_t)(ch + 1) * H + c];
+    }
+    if (ch < ce) a0 += part[(int64_t)ch * H + c];
+    const double s = 1.0 / (1.0 + exp(-((a0 + a1) / Ng)));
+    sh_s[c] = s;
+    sd[(int64_t)g * H + c] = s;
+    sf[(int64_t)g * H + c] = (float)s;
+  }
   __syncthreads();
-  int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = H / 32;
-  for (int r = w; r < H; r += nw) {                  // v[r] = Σ_c M[r][c] s[c]
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int r = w; r < H; r += nw) {                    // v[r] = Σ_c M[r][c] s[c]
     double t = 0.0;
     for (int cc = lane; cc < H; cc += 32) t += (double)M[(int64_t)r * H + cc] * sh_s[cc];
     t = warp_sum(t);
@@ -74,18 +98,22 @@ k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
   constexpr int H = NC * 32;
   __shared__ double sh_dv[kWarps][H];
   __shared__ double sh_loss[kWarps];
-  int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  int g = chunk_graph[ch];
-  float a = alpha[2];
-  double Ng = (double)(node_off[g + 1] - node_off[g]);
-  double coef = (double)sp->inv_batch / (2.0 * Ng);
+  const int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int g = chunk_graph[ch];
+  const float a = alpha[2];
+  const double Ng = (double)(node_off[g + 1] - node_off[g]);
+  const double coef = (double)sp->inv_batch / (2.0 * Ng);
   float v[NC];
 #pragma unroll
   for (int q = 0; q < NC; ++q) v[q] = vf[(int64_t)g * H + lane + 32 * q];
+  float dvp[NC];
+#pragma unroll
+  for (int q = 0; q < NC; ++q) dvp[q] = 0.f;
   double dv[NC];
 #pragma unroll
   for (int q = 0; q < NC; ++q) dv[q] = 0.0;
   double loss = 0.0;
+  int cnt = 0;
   for (int32_t i = chunk_row[ch] + w; i < chunk_row[ch + 1]; i += kWarps) {
     float hp[NC], hn[NC];
     float lp = 0.f, ln = 0.f;
@@ -98,20 +126,26 @@ k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
     }
     lp = warp_sum(lp);
     ln = warp_sum(ln);
-    double sp_ = 1.0 / (1.0 + exp(-(double)lp));
-    double sn_ = 1.0 / (1.0 + exp(-(double)ln));
-    float dlp = (float)((sp_ - 1.0) * coef);
-    float dln = (float)(sn_ * coef);
+    const double sp_ = 1.0 / (1.0 + exp(-(double)lp));
+    const double sn_ = 1.0 / (1.0 + exp(-(double)ln));
+    const float dlp = (float)((sp_ - 1.0) * coef);
+    const float dln = (float)(sn_ * coef);
     if (lane == 0) {
       dl[i] = dlp;
       dl[Nt + i] = dln;
       loss += softplus_d(-(double)lp) + softplus_d((double)ln);
     }
+    // fp32 partials over <= 8 rows, then folded into fp64
 #pragma unroll
-    for (int q = 0; q < NC; ++q) dv[q] += (double)dlp * hp[q] + (double)dln * hn[q];
+    for (int q = 0; q < NC; ++q) dvp[q] = fmaf(dlp, hp[q], fmaf(dln, hn[q], dvp[q]));
+    if (++cnt == 8) {
+#pragma unroll
+      for (int q = 0; q < NC; ++q) { dv[q] += (double)dvp[q]; dvp[q] = 0.f; }
+      cnt = 0;
+    }
   }
 #pragma unroll
-  for (int q = 0; q < NC; ++q) sh_dv[w][lane + 32 * q] = dv[q];
+  for (int q = 0; q < NC; ++q) sh_dv[w][lane + 32 * q] = dv[q] + (double)dvp[q];
   if (lane == 0) sh_loss[w] = loss;
   __syncthreads();
   for (int c = threadIdx.x; c < H; c += kWarps * 32) {
@@ -126,31 +160,59 @@ k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
   }
 }
 
-// Per graph: dv_g (fixed-order fp64 sum of chunks), ds = Mᵀ dv, dm = ds s(1-s)/N_g.
-__global__ void k_head_bwd(const double* __restrict__ dv_part,
+// Per graph: dv_g (fixed-order fp64 sum of chunks), ds = Mᵀ dv, dm = ds s(1-s)/N_g,
+// and the graph's loss.  Block = 256 threads; the Mᵀ dv product is split over
+// 256/H row groups with four independent accumulators each (fixed order).
+__global__ void k_head_bwd(const double* __restrict__ dv_part, const double* __restrict__ loss_part,
                            const int32_t* __restrict__ graph_chunk,
                            const int32_t* __restrict__ node_off, const float* __restrict__ M,
                            const double* __restrict__ sd, int H, double* __restrict__ dvd,
-                           float* __restrict__ dvf, float* __restrict__ dmf) {
-  extern __shared__ double sh_dv[];
-  int g = blockIdx.x, c = threadIdx.x;
-  double acc = 0.0;
-  for (int ch = graph_chunk[g]; ch < graph_chunk[g + 1]; ++ch) acc += dv_part[(int64_t)ch * H + c];
-  sh_dv[c] = acc;
-  dvd[(int64_t)g * H + c] = acc;
-  dvf[(int64_t)g * H + c] = (float)acc;
+                           float* __restrict__ dvf, float* __restrict__ dmf,
+                           double* __restrict__ loss_g) {
+  __shared__ double sh_dv[256];
+  __shared__ double sh_ds[256];
+  const int g = blockIdx.x;
+  const int cb = graph_chunk[g], ce = graph_chunk[g + 1];
+  for (int c = threadIdx.x; c < H; c += blockDim.x) {
+    double a0 = 0.0, a1 = 0.0;
+    int ch = cb;
+    for (; ch + 1 < ce; ch += 2) {
+      a0 += dv_part[(int64_t)ch * H + c];
+      a1 += dv_part[(int64_t)(ch + 1) * H + c];
+    }
+    if (ch < ce) a0 += dv_part[(int64_t)ch * H + c];
+    sh_dv[c] = a0 + a1;
+    dvd[(int64_t)g * H + c] = a0 + a1;
+    dvf[(int64_t)g * H + c] = (float)(a0 + a1);
+  }
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int ch = cb; ch < ce; ++ch) t += loss_part[ch];
+    loss_g[g] = t;
+  }
   __syncthreads();
-  double ds = 0.0;
-  for (int r = 0; r < H; ++r) ds += (double)M[(int64_t)r * H + c] * sh_dv[r];
-  double s = sd[(int64_t)g * H + c];
-  double Ng = (double)(node_off[g + 1] - node_off[g]);
-  dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / Ng);
+  const int groups = blockDim.x / H;                  // 256/H row groups
+  const int c = threadIdx.x % H, gr = threadIdx.x / H;
+  const int rows = H / groups;
+  double a[4] = {0.0, 0.0, 0.0, 0.0};
+  for (int r = gr * rows; r < (gr + 1) * rows; r += 4)
+#pragma unroll
+    for (int k = 0; k < 4; ++k) a[k] += (double)M[(int64_t)(r + k) * H + c] * sh_dv[r + k];
+  sh_ds[threadIdx.x] = (a[0] + a[1]) + (a[2] + a[3]);
+  __syncthreads();
+  if (gr == 0) {
+    double ds = 0.0;
+    for (int k = 0; k < groups; ++k) ds += sh_ds[k * H + c];
+    const double s = sd[(int64_t)g * H + c];
+    const double Ng = (double)(node_off[g + 1] - node_off[g]);
+    dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / Ng);
+  }
 }
 
 // dM[r][c] = Σ_g dv_g[r] s_g[c] (fixed order); block 0 also writes the loss.
 __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ sd, int G, int H,
-                     const double* __restrict__ loss_part, int nchunks,
-                     float* __restrict__ gM, float* __restrict__ loss_out) {
+                     const double* __restrict__ loss_g, float* __restrict__ gM,
+                     float* __restrict__ loss_out) {
   int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (e < (int64_t)H * H) {
     int r = (int)(e / H), c = (int)(e % H);
@@ -160,12 +222,13 @@ __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ 
   }
   if (e == 0) {
     double t = 0.0;
-    for (int k = 0; k < nchunks; ++k) t += loss_part[k];
+    for (int g = 0; g < G; ++g) t += loss_g[g];
     *loss_out = (float)t;
   }
 }
 
-// dZ3 = (dl v_g + [pos] dm_g) ⊙ PReLU'(Z3), dalpha3 partials.  Warp per row.
+// dZ3 = (dl v_g + [pos] dm_g) ⊙ PReLU'(Z3), dalpha3 partials.  Warp per row,
+// float4 columns.
 template <int NC>
 __global__ void __launch_bounds__(kWarps * 32)
 k_dz3(const float* __restrict__ Z3, const float* __restrict__ alpha,
@@ -173,26 +236,42 @@ k_dz3(const float* __restrict__ Z3, const float* __restrict__ alpha,
       const float* __restrict__ vf, const float* __restrict__ dmf, int32_t Nt,
       float* __restrict__ dZ, double* __restrict__ slots) {
   constexpr int H = NC * 32;
+  constexpr int V = H / 4;                           // float4 per row
+  constexpr int PER = (V + 31) / 32;
   __shared__ double wpart[kWarps];
-  int lane = threadIdx.x & 31;
-  int64_t r = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
+  const int lane = threadIdx.x & 31;
+  const int64_t r = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   float da = 0.f;
   if (r < 2LL * Nt) {
-    int32_t i = (int32_t)(r < Nt ? r : r - Nt);
-    bool pos = r < Nt;
-    int g = node_graph[i];
-    float a = alpha[2];
-    float d = dl[r];
+    const int32_t i = (int32_t)(r < Nt ? r : r - Nt);
+    const bool pos = r < Nt;
+    const int g = node_graph[i];
+    const float a = alpha[2];
+    const float d = dl[r];
+    const float4* Z4 = reinterpret_cast<const float4*>(Z3 + r * H);
+    const float4* v4 = reinterpret_cast<const float4*>(vf + (int64_t)g * H);
+    const float4* m4 = reinterpret_cast<const float4*>(dmf + (int64_t)g * H);
+    float4* o4 = reinterpret_cast<float4*>(dZ + r * H);
 #pragma unroll
-    for (int q = 0; q < NC; ++q) {
-      int c = lane + 32 * q;
-      float dh = d * vf[(int64_t)g * H + c] + (pos ? dmf[(int64_t)g * H + c] : 0.f);
-      float z = Z3[r * H + c];
-      dZ[r * H + c] = z > 0.f ? dh : a * dh;
-      da += z > 0.f ? 0.f : dh * z;
+    for (int q = 0; q < PER; ++q) {
+      const int c4 = lane + 32 * q;
+      if (c4 < V) {
+        const float4 z = Z4[c4], vv = v4[c4];
+        float4 dh = make_float4(d * vv.x, d * vv.y, d * vv.z, d * vv.w);
+        if (pos) {
+          const float4 mm = m4[c4];
+          dh.x += mm.x; dh.y += mm.y; dh.z += mm.z; dh.w += mm.w;
+        }
+        float4 o;
+        o.x = z.x > 0.f ? dh.x : a * dh.x;  da += z.x > 0.f ? 0.f : dh.x * z.x;
+        o.y = z.y > 0.f ? dh.y : a * dh.y;  da += z.y > 0.f ? 0.f : dh.y * z.y;
+        o.z = z.z > 0.f ? dh.z : a * dh.z;  da += z.z > 0.f ? 0.f : dh.z * z.z;
+        o.w = z.w > 0.f ? dh.w : a * dh.w;  da += z.w > 0.f ? 0.f : dh.w * z.w;
+        o4[c4] = o;
+      }
     }
   }
-  double t = warp_sum((double)da);
+  const double t = warp_sum((double)da);
   if (lane == 0) wpart[threadIdx.x >> 5] = t;
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -226,15 +305,13 @@ cudaError_t head_nc(const GraphDev& g, const float* Z3, const float* M, const fl
                     const StepParams* sp, const HeadWork& w, float* dZ, float* gM,
                     float* loss_out, int* nslots, cudaStream_t s) {
   constexpr int H = NC * 32;
-  k_colsum<<<g.nchunks, H, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
-  k_readout<<<g.G, H, H * sizeof(double), s>>>(w.colsum_part, g.graph_chunk, g.node_off, M, H,
-                                                w.sd, w.s, w.v);
+  k_colsum<<<g.nchunks, 256, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
+  k_readout<<<g.G, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.node_off, M, H, w.sd, w.s, w.v);
   k_score<NC><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph, g.node_off,
                                                 w.v, sp, g.Nt, w.dl, w.dv_part, w.loss_part);
-  k_head_bwd<<<g.G, H, H * sizeof(double), s>>>(w.dv_part, g.graph_chunk, g.node_off, M, w.sd, H,
-                                                 w.dvd, w.dv, w.dm);
-  k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_part, g.nchunks, gM,
-                                                 loss_out);
+  k_head_bwd<<<g.G, 256, 0, s>>>(w.dv_part, w.loss_part, g.graph_chunk, g.node_off, M, w.sd, H,
+                                 w.dvd, w.dv, w.dm, w.loss_g);
+  k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
   unsigned nb = cdiv(2LL * g.Nt, kWarps);
   k_dz3<NC><<<nb, kWarps * 32, 0, s>>>(Z3, alpha, g.node_graph, w.dl, w.v, w.dm, g.Nt, dZ,
                                        w.slots);

@@ -139,6 +139,7 @@ struct HeadWork {
   double* dvd;          // [G*H]
   double* sd;           // [G*H]
   float* dl;            // [2*Nt]
+  double* loss_g;       // [G] per-graph loss (already / (2 N_g B))
   double* slots;        // [nslots] dalpha3 partials
 };
 // Forward head + head backward: writes grads of M (dM) and the loss slot,

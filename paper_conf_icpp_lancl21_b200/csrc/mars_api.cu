@@ -26,7 +26,7 @@ namespace {
 constexpr uint64_t kTagGraph = 0x4D41525347524150ULL;  // "MARSGRAP"
 constexpr uint64_t kTagDgi = 0x4D41525344474931ULL;    // "MARSDGI1"
 constexpr uint64_t kTagDead = 0xDEADDEADDEADDEADULL;
-constexpr int kChunkRows = 64;
+constexpr int kChunkRows = 256;   // deterministic reduction chunk (rows, within one graph)
 
 thread_local std::string g_err;
 
@@ -636,6 +636,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   CK(al((void**)&h.dvd, sizeof(double) * G * H));
   CK(al((void**)&h.sd, sizeof(double) * G * H));
   CK(al((void**)&h.dl, sizeof(float) * R));
+  CK(al((void**)&h.loss_g, sizeof(double) * G));
   int nsl = std::max(head_slots(g->dev), spmm_bwd_slots(g->dev));
   for (int l = 0; l < 3; ++l) CK(al((void**)&w.slots[l], sizeof(double) * nsl));
   h.slots = w.slots[2];
