@@ -40,17 +40,22 @@ namespace {
 using namespace tc;
 
 constexpr int kBM = 128;        // tile rows (UMMA M)
-constexpr int kBK = 32;         // fp32 elements per 128-byte swizzle row
+constexpr int kBK = 16;         // fp32 elements per K-block = one 64-byte swizzle row
 constexpr int kThreads = 256;
 
 // ---------------------------------------------------------------- k_tc_rows
 template <int N>
 struct RowsCfg {
-  static constexpr int kStages = N > 128 ? 2 : 3;
-  static constexpr int A_BYTES = kBM * kBK * 4;       // 16 KB
+  // 64-byte K-blocks keep a stage at 48 KB (N = 256) so four stages are in
+  // flight: enough to cover TMA latency + the A split ahead of the MMAs.
+  static constexpr int kStages = N > 128 ? 4 : 6;
+  static constexpr int A_BYTES = kBM * kBK * 4;       // 8 KB
   static constexpr int B_BYTES = N * kBK * 4;
   static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int SMEM = kStages * STAGE + 1024 + 256;
+  // epilogue staging: per epilogue warp two 32 x 32 fp32 slabs (128-byte swizzle)
+  static constexpr int SLAB = 32 * 32 * 4;
+  static constexpr int STAGING = 4 * 2 * SLAB;
+  static constexpr int SMEM = kStages * STAGE + STAGING + 1024 + 256;
   static constexpr uint32_t TMEM_COLS = (2 * N) <= 32 ? 32 : (2 * N) <= 64 ? 64 : (2 * N) <= 128 ? 128
                                         : (2 * N) <= 256 ? 256 : 512;
 };
@@ -58,14 +63,16 @@ struct RowsCfg {
 template <int N>
 __global__ void __launch_bounds__(kThreads, 1)
 k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBhi,
-          const __grid_constant__ CUtensorMap tmBlo, float* __restrict__ C, int32_t M, int32_t K) {
+          const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmC,
+          int32_t M, int32_t K) {
   using Cfg = RowsCfg<N>;
   constexpr int S = Cfg::kStages;
   extern __shared__ uint8_t smem_raw[];
   // 1024-byte alignment for the 128-byte swizzle atoms, by pointer arithmetic on
   // the shared array itself so every access stays in the shared window (LDS/STS).
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
+  uint8_t* staging = smem + S * Cfg::STAGE;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE + Cfg::STAGING);
   uint64_t* full = bars;            // TMA landed            (count 1 + tx)
   uint64_t* conv = bars + S;        // A split done          (count 2 warps)
   uint64_t* empty = bars + 2 * S;   // MMA done with stage   (commit)
@@ -95,6 +102,7 @@ k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUten
     tma_prefetch(&tmA);
     tma_prefetch(&tmBhi);
     tma_prefetch(&tmBlo);
+    tma_prefetch(&tmC);
   }
   if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
   tc_fence_before();
@@ -134,10 +142,11 @@ k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUten
           const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
 #pragma unroll
           for (int k = 0; k < kBK / 8; ++k) {
-            const uint64_t ah = sdesc_sw128(a + 32 * k, 16, 1024);
-            const uint64_t alo = sdesc_sw128(al + 32 * k, 16, 1024);
-            const uint64_t bh = sdesc_sw128(b + 32 * k, 16, 1024);
-            const uint64_t blo = sdesc_sw128(bl + 32 * k, 16, 1024);
+            // K-major, 64-byte swizzle: rows 64 B apart, 8-row groups 512 B (SBO)
+            const uint64_t ah = sdesc_sw64(a + 32 * k, 16, 512);
+            const uint64_t alo = sdesc_sw64(al + 32 * k, 16, 512);
+            const uint64_t bh = sdesc_sw64(b + 32 * k, 16, 512);
+            const uint64_t blo = sdesc_sw64(bl + 32 * k, 16, 512);
             mma_tf32(d, ah, bh, idesc, (kb | k) != 0);
             mma_tf32(d, ah, blo, idesc, 1);
             mma_tf32(d, alo, bh, idesc, 1);
@@ -175,21 +184,32 @@ k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUten
     const int q = warp & 3;
     int acc = 0;
     uint32_t aph = 0;
+    // TMEM -> registers -> 128B-swizzled smem slab (conflict-free row-per-lane
+    // writes) -> TMA tile store: coalesced full-line writes, tail rows clipped
+    uint8_t* slab0 = staging + q * 2 * Cfg::SLAB;
+    int nslab = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
-      const int64_t row = (int64_t)t * kBM + q * 32 + lane;
 #pragma unroll 1
-      for (int c0 = 0; c0 < N; c0 += 32) {
+      for (int c0 = 0; c0 < N; c0 += 32, ++nslab) {
         uint32_t r[32];
         tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
+        uint8_t* slab = slab0 + (nslab & 1) * Cfg::SLAB;
+        if (lane == 0) bulk_wait_read<1>();                // the store issued 2 slabs ago is done
+        __syncwarp();
         tmem_wait_ld();
-        if (row < M) {
-          float4* dst = reinterpret_cast<float4*>(C + row * N + c0);
 #pragma unroll
-          for (int j = 0; j < 8; ++j)
-            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
-                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+        for (int j = 0; j < 8; ++j) {
+          float4* dst = reinterpret_cast<float4*>(slab + lane * 128 + ((j ^ (lane & 7)) << 4));
+          *dst = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
+                             __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_2d(&tmC, slab, c0, t * kBM + q * 32);
+          bulk_commit();
         }
       }
       tc_fence_before();
@@ -198,6 +218,7 @@ k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUten
       acc ^= 1;
       if (acc == 0) aph ^= 1;
     }
+    if (lane == 0) bulk_wait<0>();
   }
   tc_fence_before();
   __syncthreads();
@@ -624,19 +645,32 @@ bool encode_fn() {
   return g_encode != nullptr;
 }
 
-// Row-major fp32 [rows × cols] with a {box_cols (= 32), box_rows} box and a
-// 128-byte swizzle: 16-byte atoms for K-major operands, 32-byte atoms for
-// MN-major tf32 operands (mn_major).
+// Row-major fp32 [rows × cols] boxes for the UMMA operand layouts:
+//  mn_major: {32 cols, box_rows}, 128-byte swizzle with 32-byte atoms (MN-major tf32)
+//  else    : {kBK = 16 cols, box_rows}, 64-byte swizzle (K-major, 64-byte rows)
 bool tmap_2d(CUtensorMap* m, const float* base, int64_t rows, int64_t cols, int box_rows,
              bool mn_major = false) {
   if (!encode_fn()) return false;
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
   cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
-  cuuint32_t box[2] = {32, (cuuint32_t)box_rows};
+  cuuint32_t box[2] = {mn_major ? 32u : (cuuint32_t)kBK, (cuuint32_t)box_rows};
   cuuint32_t es[2] = {1, 1};
   return g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides,
                   box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                  mn_major ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_128B,
+                  mn_major ? CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B : CU_TENSOR_MAP_SWIZZLE_64B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// Output [rows × cols] fp32 for the epilogue's TMA stores: {32, 32} boxes, 128B swizzle.
+bool tmap_store(CUtensorMap* m, const float* base, int64_t rows, int64_t cols) {
+  if (!encode_fn()) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
+  cuuint32_t box[2] = {32, 32};
+  cuuint32_t es[2] = {1, 1};
+  return g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides,
+                  box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
@@ -663,12 +697,13 @@ cudaError_t rows_n(const float* A, const float* Bhi, const float* Blo, float* C,
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  CUtensorMap ta, tbh, tbl;
-  if (!tmap_2d(&ta, A, M, K, kBM) || !tmap_2d(&tbh, Bhi, N, K, N) || !tmap_2d(&tbl, Blo, N, K, N))
+  CUtensorMap ta, tbh, tbl, tc;
+  if (!tmap_2d(&ta, A, M, K, kBM) || !tmap_2d(&tbh, Bhi, N, K, N) ||
+      !tmap_2d(&tbl, Blo, N, K, N) || !tmap_store(&tc, C, M, N))
     return cudaErrorInvalidValue;
   int ntiles = (int)((M + kBM - 1) / kBM);
   int grid = std::min(ntiles, num_sms());
-  k_tc_rows<N><<<grid, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, C, (int32_t)M, K);
+  k_tc_rows<N><<<grid, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, tc, (int32_t)M, K);
   return cudaGetLastError();
 }
 
@@ -720,7 +755,8 @@ cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, f
 
 // Row chunks so that chunks x C_in tiles ~ one CTA per SM.
 int tc_dw_chunks(int64_t R, int CIN) {
-  int64_t want = std::max<int64_t>(1, num_sms() / (CIN / dw_tile(CIN)));
+  const int ntile = std::max(1, CIN / dw_tile(CIN));
+  int64_t want = std::max<int64_t>(1, num_sms() / ntile);
   int64_t maxc = std::max<int64_t>(1, R / 256);
   return (int)std::min(want, maxc);
 }

@@ -58,6 +58,37 @@ cudaError_t dalloc(T** p, size_t n) {
   return cudaMalloc(reinterpret_cast<void**>(p), sizeof(T) * (n ? n : 1));
 }
 
+// Stream-ordered allocation from the device's default pool (graph sets are
+// loaded and freed per batch when op graphs are streamed; the pool keeps the
+// memory instead of returning it to the driver).
+template <typename T>
+cudaError_t palloc(T** p, size_t n, cudaStream_t s) {
+  return cudaMallocAsync(reinterpret_cast<void**>(p), sizeof(T) * (n ? n : 1), s);
+}
+
+void pool_init(int device) {
+  static std::mutex mu;
+  static bool done[64] = {};
+  std::lock_guard<std::mutex> lk(mu);
+  if (device < 0 || device >= 64 || done[device]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t thr = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  cudaGetLastError();
+  done[device] = true;
+}
+
+bool is_pinned(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost;
+}
+
 // ---------------------------------------------------------------- NCCL (dlopen)
 struct NcclApi {
   bool tried = false, ok = false;
@@ -129,6 +160,13 @@ __global__ void k_xavier(float* __restrict__ p, int64_t n, uint64_t seed, uint64
   p[i] = __double2float_rn(__dmul_rn(__dsub_rn(__dmul_rn(2.0, u), 1.0), (double)b));
 }
 
+__global__ void k_gather_rowptr(const int32_t* __restrict__ rowptr,
+                                const int32_t* __restrict__ node_off, int G,
+                                int32_t* __restrict__ out) {
+  int g = blockIdx.x * blockDim.x + threadIdx.x;
+  if (g <= G) out[g] = rowptr[node_off[g]];
+}
+
 __global__ void k_fill(float* __restrict__ p, int64_t n, float v) {
   int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i < n) p[i] = v;
@@ -153,11 +191,11 @@ struct mars_graph {
   int32_t *bucket_off = nullptr, *bucket_log2 = nullptr;
   float *vals = nullptr, *dinv = nullptr, *X = nullptr;
   GraphDev dev{};
-  ~mars_graph() {
+  ~mars_graph() {   // pool memory; mars_free synchronises the device first
     for (void* p : {(void*)node_off, (void*)node_graph, (void*)rowptr, (void*)colind, (void*)deg,
                     (void*)chunk_row, (void*)chunk_graph, (void*)graph_chunk, (void*)bucket_off,
                     (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X})
-      if (p) cudaFree(p);
+      if (p) cudaFreeAsync(p, nullptr);
   }
 };
 
@@ -322,50 +360,74 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   chunk_row.push_back((int32_t)Nt);
   int nchunks = (int)chunk_graph.size();
 
-  // pack inputs into pinned staging and copy once
-  size_t b_indptr = sizeof(int64_t) * (size_t)(Nt + G);
-  size_t b_idx = sizeof(int32_t) * (size_t)Et;
-  size_t b_X = sizeof(float) * (size_t)Nt * F;
-  std::lock_guard<std::mutex> lk(g_stage.mu);
-  char* stage = static_cast<char*>(g_stage.get(b_indptr + b_idx + b_X + 64));
-  if (!stage) return fail(MARS_ENOMEM, "pinned staging allocation failed");
-  int64_t* s_indptr = reinterpret_cast<int64_t*>(stage);
-  int32_t* s_idx = reinterpret_cast<int32_t*>(stage + b_indptr);
-  float* s_X = reinterpret_cast<float*>(stage + b_indptr + b_idx);
-  for (int g = 0; g < G; ++g) {
-    const mars_graph_desc& d = descs[g];
-    int32_t N = d.num_nodes;
-    memcpy(s_indptr + gr->h_node_off[g] + g, d.indptr, sizeof(int64_t) * (size_t)(N + 1));
-    if (d.indptr[N] > 0) memcpy(s_idx + edge_off[g], d.indices, sizeof(int32_t) * (size_t)d.indptr[N]);
-    memcpy(s_X + (int64_t)gr->h_node_off[g] * F, d.features, sizeof(float) * (size_t)N * F);
-  }
   cudaStream_t s = nullptr;
   CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+  pool_init(device);
 
+  size_t b_indptr = sizeof(int64_t) * (size_t)(Nt + G);
+  size_t b_idx = sizeof(int32_t) * (size_t)Et;
+  size_t b_X = sizeof(float) * (size_t)Nt * F;
   int64_t* d_indptr;
   int32_t* d_idx;
   int64_t* d_edge_off;
-  CK(dalloc(&d_indptr, (size_t)(Nt + G)));
-  struct F1 { void* p; ~F1() { cudaFree(p); } } f1{d_indptr};
-  CK(dalloc(&d_idx, (size_t)Et));
+  struct F1 { void* p; ~F1() { if (p) cudaFreeAsync(p, nullptr); } };
+  CK(palloc(&d_indptr, (size_t)(Nt + G), s));
+  F1 f1{d_indptr};
+  CK(palloc(&d_idx, (size_t)Et, s));
   F1 f2{d_idx};
-  CK(dalloc(&d_edge_off, (size_t)G + 1));
+  CK(palloc(&d_edge_off, (size_t)G + 1, s));
   F1 f3{d_edge_off};
-  CK(dalloc(&gr->X, (size_t)Nt * F));
-  CK(dalloc(&gr->node_off, (size_t)G + 1));
-  CK(dalloc(&gr->node_graph, (size_t)Nt));
-  CK(dalloc(&gr->rowptr, (size_t)Nt + 1));
-  CK(dalloc(&gr->deg, (size_t)Nt));
-  CK(dalloc(&gr->dinv, (size_t)Nt));
-  CK(dalloc(&gr->chunk_row, (size_t)nchunks + 1));
-  CK(dalloc(&gr->chunk_graph, (size_t)nchunks));
-  CK(dalloc(&gr->graph_chunk, (size_t)G + 1));
-  CK(dalloc(&gr->bucket_off, (size_t)G + 1));
-  CK(dalloc(&gr->bucket_log2, (size_t)G));
-  CK(cudaMemcpyAsync(d_indptr, s_indptr, b_indptr, cudaMemcpyHostToDevice, s));
-  if (Et) CK(cudaMemcpyAsync(d_idx, s_idx, b_idx, cudaMemcpyHostToDevice, s));
-  CK(cudaMemcpyAsync(gr->X, s_X, b_X, cudaMemcpyHostToDevice, s));
+  CK(palloc(&gr->X, (size_t)Nt * F, s));
+  CK(palloc(&gr->node_off, (size_t)G + 1, s));
+  CK(palloc(&gr->node_graph, (size_t)Nt, s));
+  CK(palloc(&gr->rowptr, (size_t)Nt + 1, s));
+  CK(palloc(&gr->deg, (size_t)Nt, s));
+  CK(palloc(&gr->dinv, (size_t)Nt, s));
+  CK(palloc(&gr->chunk_row, (size_t)nchunks + 1, s));
+  CK(palloc(&gr->chunk_graph, (size_t)nchunks, s));
+  CK(palloc(&gr->graph_chunk, (size_t)G + 1, s));
+  CK(palloc(&gr->bucket_off, (size_t)G + 1, s));
+  CK(palloc(&gr->bucket_log2, (size_t)G, s));
+
+  // Inputs in page-locked host memory are copied straight to the device;
+  // otherwise they are packed into a pinned staging buffer first.
+  bool pinned = true;
+  for (int g = 0; g < G && pinned; ++g)
+    pinned = is_pinned(descs[g].indptr) && is_pinned(descs[g].features) &&
+             (descs[g].indptr[descs[g].num_nodes] == 0 || is_pinned(descs[g].indices));
+  std::unique_lock<std::mutex> lk(g_stage.mu, std::defer_lock);
+  if (pinned) {
+    for (int g = 0; g < G; ++g) {
+      const mars_graph_desc& d = descs[g];
+      int32_t N = d.num_nodes;
+      CK(cudaMemcpyAsync(d_indptr + gr->h_node_off[g] + g, d.indptr, sizeof(int64_t) * (N + 1),
+                         cudaMemcpyHostToDevice, s));
+      if (d.indptr[N] > 0)
+        CK(cudaMemcpyAsync(d_idx + edge_off[g], d.indices, sizeof(int32_t) * d.indptr[N],
+                           cudaMemcpyHostToDevice, s));
+      CK(cudaMemcpyAsync(gr->X + (int64_t)gr->h_node_off[g] * F, d.features,
+                         sizeof(float) * (size_t)N * F, cudaMemcpyHostToDevice, s));
+    }
+  } else {
+    lk.lock();
+    char* stage = static_cast<char*>(g_stage.get(b_indptr + b_idx + b_X + 64));
+    if (!stage) return fail(MARS_ENOMEM, "pinned staging allocation failed");
+    int64_t* s_indptr = reinterpret_cast<int64_t*>(stage);
+    int32_t* s_idx = reinterpret_cast<int32_t*>(stage + b_indptr);
+    float* s_X = reinterpret_cast<float*>(stage + b_indptr + b_idx);
+    for (int g = 0; g < G; ++g) {
+      const mars_graph_desc& d = descs[g];
+      int32_t N = d.num_nodes;
+      memcpy(s_indptr + gr->h_node_off[g] + g, d.indptr, sizeof(int64_t) * (size_t)(N + 1));
+      if (d.indptr[N] > 0)
+        memcpy(s_idx + edge_off[g], d.indices, sizeof(int32_t) * (size_t)d.indptr[N]);
+      memcpy(s_X + (int64_t)gr->h_node_off[g] * F, d.features, sizeof(float) * (size_t)N * F);
+    }
+    CK(cudaMemcpyAsync(d_indptr, s_indptr, b_indptr, cudaMemcpyHostToDevice, s));
+    if (Et) CK(cudaMemcpyAsync(d_idx, s_idx, b_idx, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(gr->X, s_X, b_X, cudaMemcpyHostToDevice, s));
+  }
   CK(cudaMemcpyAsync(d_edge_off, edge_off.data(), sizeof(int64_t) * (G + 1), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(gr->node_off, gr->h_node_off.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(gr->chunk_row, chunk_row.data(), sizeof(int32_t) * (nchunks + 1), cudaMemcpyHostToDevice, s));
@@ -388,9 +450,13 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   io.node_graph = gr->node_graph;
   int64_t cap = Nt + 2 * Et;
   std::vector<void*> scratch;
-  struct SF { std::vector<void*>* v; ~SF() { for (void* p : *v) cudaFree(p); } } sf{&scratch};
+  struct SF {
+    std::vector<void*>* v;
+    cudaStream_t s;
+    ~SF() { for (void* p : *v) cudaFreeAsync(p, s); }
+  } sf{&scratch, s};
   auto salloc = [&](void** p, size_t bytes) -> cudaError_t {
-    cudaError_t e = cudaMalloc(p, bytes ? bytes : 4);
+    cudaError_t e = cudaMallocAsync(p, bytes ? bytes : 4, s);
     if (e == cudaSuccess) scratch.push_back(*p);
     return e;
   };
@@ -407,18 +473,22 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   io.deg = gr->deg;
   io.dinv = gr->dinv;
   CK(build_csr_phase1(io, s));
-  int32_t herr[2] = {0, 0};
-  CK(cudaMemcpyAsync(herr, io.err, sizeof herr, cudaMemcpyDeviceToHost, s));
-  std::vector<int32_t> h_rowptr((size_t)Nt + 1);
-  CK(cudaMemcpyAsync(h_rowptr.data(), gr->rowptr, sizeof(int32_t) * (Nt + 1), cudaMemcpyDeviceToHost, s));
+  // per-graph nnz offsets rowptr[node_off[g]] (+ the error flags) in one small D2H
+  std::vector<int32_t> hbuf((size_t)G + 3);
+  int32_t* d_nnzoff = io.ucnt;                         // ucnt is free after the scan
+  k_gather_rowptr<<<cdiv(G + 1, 256), 256, 0, s>>>(gr->rowptr, gr->node_off, G, d_nnzoff);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(hbuf.data(), d_nnzoff, sizeof(int32_t) * (G + 1), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(hbuf.data() + G + 1, io.err, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
-  if (herr[0]) return fail(MARS_EINVAL, "malformed graph input (code %d): %s", herr[0],
-                           (herr[0] & 2) ? "edge index out of range" : "indptr inconsistent");
-  gr->nnz = h_rowptr[Nt];
+  const int32_t herr = hbuf[G + 1];
+  if (herr) return fail(MARS_EINVAL, "malformed graph input (code %d): %s", herr,
+                        (herr & 2) ? "edge index out of range" : "indptr inconsistent");
   gr->h_nnz_off.resize(G + 1);
-  for (int g = 0; g <= G; ++g) gr->h_nnz_off[g] = h_rowptr[gr->h_node_off[g]];
-  CK(dalloc(&gr->colind, (size_t)gr->nnz));
-  CK(dalloc(&gr->vals, (size_t)gr->nnz));
+  for (int g = 0; g <= G; ++g) gr->h_nnz_off[g] = hbuf[g];
+  gr->nnz = gr->h_nnz_off[G];
+  CK(palloc(&gr->colind, (size_t)gr->nnz, s));
+  CK(palloc(&gr->vals, (size_t)gr->nnz, s));
   CK(build_csr_phase2(io, gr->colind, gr->vals, s));
   CK(cudaStreamSynchronize(s));
 

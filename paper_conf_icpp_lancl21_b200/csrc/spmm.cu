@@ -19,6 +19,7 @@ namespace mars {
 namespace {
 
 constexpr int kSpmmThreads = 256;
+constexpr int kU = 4;           // neighbours whose gathers are in flight together
 
 // C in {16, 32, 64, 128, 256} (mars.h restricts F and H to these widths).
 template <int C>
@@ -68,8 +69,36 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
       myv = vals[k0 + sl];
       if (BOTH) myjn = (MODE == 0) ? perm[myj] : Nt + myj;
     }
-#pragma unroll 4
-    for (int t = 0; t < cnt; ++t) {
+    // groups of kU neighbours: every gather of the group is issued before the
+    // first FMA (memory-level parallelism); FMAs stay in ascending colind order
+    int t = 0;
+    for (; t + kU <= cnt; t += kU) {
+      int32_t j[kU], jn[kU];
+      float w[kU];
+      float4 xp[kU][S::NT], xn[kU][S::NT];
+#pragma unroll
+      for (int u = 0; u < kU; ++u) {
+        j[u] = __shfl_sync(gmask, myj, t + u, S::L);
+        w[u] = __shfl_sync(gmask, myv, t + u, S::L);
+        jn[u] = BOTH ? __shfl_sync(gmask, myjn, t + u, S::L) : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < kU; ++u)
+#pragma unroll
+        for (int q = 0; q < S::NT; ++q) {
+          const int c4 = sl + q * S::L;
+          xp[u][q] = __ldg(T4 + (int64_t)j[u] * (C / 4) + c4);
+          if (BOTH) xn[u][q] = __ldg(T4 + (int64_t)jn[u] * (C / 4) + c4);
+        }
+#pragma unroll
+      for (int u = 0; u < kU; ++u)
+#pragma unroll
+        for (int q = 0; q < S::NT; ++q) {
+          f4_fma(accp[q], w[u], MODE == 1 ? f4_prelu(xp[u][q], a) : xp[u][q]);
+          if (BOTH) f4_fma(accn[q], w[u], MODE == 1 ? f4_prelu(xn[u][q], a) : xn[u][q]);
+        }
+    }
+    for (; t < cnt; ++t) {
       int32_t j = __shfl_sync(gmask, myj, t, S::L);
       float w = __shfl_sync(gmask, myv, t, S::L);
       int32_t jn = BOTH ? __shfl_sync(gmask, myjn, t, S::L) : 0;
@@ -124,8 +153,33 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
         myj = colind[k0 + sl];
         myv = vals[k0 + sl];
       }
-#pragma unroll 4
-      for (int t = 0; t < cnt; ++t) {
+      int t = 0;
+      for (; t + kU <= cnt; t += kU) {
+        int32_t j[kU];
+        float w[kU];
+        float4 xp[kU][S::NT], xn[kU][S::NT];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+          j[u] = __shfl_sync(gmask, myj, t + u, S::L);
+          w[u] = __shfl_sync(gmask, myv, t + u, S::L);
+        }
+#pragma unroll
+        for (int u = 0; u < kU; ++u)
+#pragma unroll
+          for (int q = 0; q < S::NT; ++q) {
+            const int c4 = sl + q * S::L;
+            xp[u][q] = __ldg(D4 + (int64_t)j[u] * (C / 4) + c4);
+            xn[u][q] = __ldg(D4 + ((int64_t)Nt + j[u]) * (C / 4) + c4);
+          }
+#pragma unroll
+        for (int u = 0; u < kU; ++u)
+#pragma unroll
+          for (int q = 0; q < S::NT; ++q) {
+            f4_fma(accp[q], w[u], xp[u][q]);
+            f4_fma(accn[q], w[u], xn[u][q]);
+          }
+      }
+      for (; t < cnt; ++t) {
         int32_t j = __shfl_sync(gmask, myj, t, S::L);
         float w = __shfl_sync(gmask, myv, t, S::L);
 #pragma unroll
