@@ -436,6 +436,205 @@ k_tc_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtens
   }
 }
 
+// ---------------------------------------------------------------- k_tc_dw2
+// Same tiling as k_tc_dw, but the fp32 master accumulator lives in the
+// registers of eight epilogue warps (quadrant q = warp & 3 owns TMEM lanes
+// 32q.., column half ch = (warp-4)/4 owns half of the tile's columns), so the
+// two TMEM work accumulators can be double-buffered: the tensor cores fill
+// one 128-row run while the epilogue folds the previous one (IEEE adds).
+// 12 warps: 0 TMA, 1 MMA, 2-3 split, 4-11 fold / write.
+template <int CINT>
+struct Dw2Cfg {
+  static constexpr int A_BYTES = 256 * kDwBK * 4;
+  static constexpr int B_BYTES = CINT * kDwBK * 4;
+  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int SMEM = kDwStages * STAGE + 1024 + 256;
+  static constexpr uint32_t TMEM_COLS = 4 * CINT;     // 2 work buffers x 2 halves of H
+  static constexpr int BOX = 32 * kDwBK * 4;
+  static constexpr int MCOLS = CINT / 2;              // columns per epilogue thread per half
+};
+
+template <int CINT>
+__global__ void __launch_bounds__(384, 1)
+k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
+         float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN) {
+  using Cfg = Dw2Cfg<CINT>;
+  constexpr int S = kDwStages;
+  constexpr int MC = Cfg::MCOLS;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;
+  uint64_t* conv = bars + S;
+  uint64_t* empty = bars + 2 * S;
+  uint64_t* tfull = bars + 3 * S;        // [2]
+  uint64_t* tempty = bars + 3 * S + 2;   // [2]
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 4);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ntile = CIN / CINT;
+  const int chunk = blockIdx.x / ntile, c_off = (blockIdx.x % ntile) * CINT;
+  const int32_t r0 = chunk * rows_per_chunk;
+  const int32_t r1 = min(R, r0 + rows_per_chunk);
+  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
+  const int nsub = (nk + kSubKb - 1) / kSubKb;
+  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stAlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto stB = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
+  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 10);                               // split warps 2..11
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 8);
+    }
+    fence_mbar_init();
+    tma_prefetch(&tmDZ);
+    tma_prefetch(&tmY);
+  }
+  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer
+      int s = 0;
+      uint32_t ph = 0;
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
+        const int32_t row = r0 + kb * kDwBK;
+#pragma unroll
+        for (int bx = 0; bx < 8; ++bx)
+          tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 32, row, &full[s]);
+#pragma unroll
+        for (int bx = 0; bx < CINT / 32; ++bx)
+          tma_load_2d(stB(s) + bx * Cfg::BOX, &tmY, c_off + bx * 32, row, &full[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {                                         // ---- MMA issuer
+      constexpr uint32_t idesc = idesc_tf32(kBM, CINT, true, true);
+      int s = 0;
+      uint32_t ph = 0;
+      for (int sub = 0; sub < nsub; ++sub) {
+        const int buf = sub & 1;
+        mbar_wait(&tempty[buf], ((sub >> 1) & 1) ^ 1);      // previous use of this buffer folded
+        tc_fence_after();
+        const uint32_t twork = tbase + buf * 2 * CINT;
+        const int kb1 = min(nk, (sub + 1) * kSubKb);
+        for (int kb = sub * kSubKb; kb < kb1; ++kb) {
+          mbar_wait(&conv[s], ph);
+          tc_fence_after();
+          const uint32_t a = smem_u32(stA(s)), al = smem_u32(stAlo(s));
+          const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
+#pragma unroll
+          for (int k = 0; k < kDwBK / 8; ++k) {
+            const uint64_t bh = sdesc_sw128_b32(b + 1024 * k, Cfg::BOX, 512);
+            const uint64_t blo = sdesc_sw128_b32(bl + 1024 * k, Cfg::BOX, 512);
+            const uint32_t first = (kb == sub * kSubKb && k == 0) ? 0u : 1u;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const uint64_t ah = sdesc_sw128_b32(a + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
+              const uint64_t alo = sdesc_sw128_b32(al + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
+              const uint32_t d = twork + h * CINT;
+              mma_tf32(d, ah, bh, idesc, first);
+              mma_tf32(d, ah, blo, idesc, 1);
+              mma_tf32(d, alo, bh, idesc, 1);
+            }
+          }
+          mma_commit(&empty[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+        mma_commit(&tfull[buf]);
+      }
+    }
+  } else {                         // ---- split (warps 2..11); warps 4..11 also fold
+    const bool folder = warp >= 4;
+    const int ct = (warp - 2) * 32 + lane;
+    constexpr int NT = 10 * 32;
+    const int q = warp & 3, ch = (warp - 4) >> 2;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    float master[2][MC];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int j = 0; j < MC; ++j) master[h][j] = 0.f;
+    int folded = 0;
+    // fold work run `sub` (double-buffered in TMEM) into the register master
+    auto fold = [&](int sub) {
+      const int buf = sub & 1;
+      mbar_wait(&tfull[buf], (sub >> 1) & 1);
+      tc_fence_after();
+      const uint32_t twork = tbase + buf * 2 * CINT + ch * MC;
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int c0 = 0; c0 < MC; c0 += 32) {
+          uint32_t w[32];
+          tmem_ld32(twork + lane_off + h * CINT + c0, w);
+          tmem_wait_ld();
+#pragma unroll
+          for (int j = 0; j < 32; ++j) master[h][c0 + j] += __uint_as_float(w[j]);
+        }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[buf]);
+    };
+    int s = 0;
+    uint32_t ph = 0;
+    for (int kb = 0; kb < nk; ++kb) {
+      mbar_wait(&full[s], ph);
+      float4* a = reinterpret_cast<float4*>(stA(s));
+      float4* al = reinterpret_cast<float4*>(stAlo(s));
+      float4* bb = reinterpret_cast<float4*>(stB(s));
+      float4* bl = reinterpret_cast<float4*>(stBlo(s));
+      for (int i = ct; i < (Cfg::A_BYTES + Cfg::B_BYTES) / 16; i += NT) {
+        const bool isA = i < Cfg::A_BYTES / 16;
+        float4* src = isA ? a + i : bb + (i - Cfg::A_BYTES / 16);
+        float4* dlo = isA ? al + i : bl + (i - Cfg::A_BYTES / 16);
+        const float4 v = *src;
+        const float4 hv = make_float4(to_tf32(v.x), to_tf32(v.y), to_tf32(v.z), to_tf32(v.w));
+        *src = hv;
+        *dlo = make_float4(v.x - hv.x, v.y - hv.y, v.z - hv.z, v.w - hv.w);
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&conv[s]);
+      if (++s == S) { s = 0; ph ^= 1; }
+      // mid-way through run sub+1 the MMAs of run sub are done: fold it, well
+      // before run sub+2 needs its TMEM buffer back
+      if (folder && (kb % kSubKb) == kSubKb / 2 && kb / kSubKb >= 1) fold(folded++);
+    }
+    if (folder) {
+      while (folded < nsub) fold(folded++);
+      float* out = part + (int64_t)chunk * 256 * CIN + c_off + ch * MC;   // chunk partial
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        float4* dst = reinterpret_cast<float4*>(out + (int64_t)(h * 128 + q * 32 + lane) * CIN);
+#pragma unroll
+        for (int j = 0; j < MC / 4; ++j)
+          dst[j] = make_float4(master[h][4 * j], master[h][4 * j + 1], master[h][4 * j + 2],
+                               master[h][4 * j + 3]);
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tbase, Cfg::TMEM_COLS);
+  }
+}
+
 #if 0  // superseded single-accumulator version (kept out of the build)
 constexpr int kDwBK_old = 16;        // rows of R per stage
 constexpr int kDwStages = 3;
@@ -710,10 +909,10 @@ cudaError_t rows_n(const float* A, const float* Bhi, const float* Blo, float* C,
 template <int CINT>
 cudaError_t dw_c(const float* Y, const float* dZ, float* part, int nchunk, int64_t R, int rows,
                  int CIN, cudaStream_t s) {
-  using Cfg = DwCfg<CINT>;
+  using Cfg = Dw2Cfg<CINT>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_tc_dw<CINT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(k_tc_dw2<CINT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          Cfg::SMEM);
     if (e != cudaSuccess) return e;
     attr = true;
@@ -721,7 +920,7 @@ cudaError_t dw_c(const float* Y, const float* dZ, float* part, int nchunk, int64
   CUtensorMap tdz, ty;
   if (!tmap_2d(&tdz, dZ, R, 256, kDwBK, true) || !tmap_2d(&ty, Y, R, CIN, kDwBK, true))
     return cudaErrorInvalidValue;
-  k_tc_dw<CINT><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows, CIN);
+  k_tc_dw2<CINT><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows, CIN);
   return cudaGetLastError();
 }
 

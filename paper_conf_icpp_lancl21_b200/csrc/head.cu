@@ -49,6 +49,78 @@ __global__ void k_colsum(const float* __restrict__ Z3, const float* __restrict__
   }
 }
 
+// Second stage of a per-graph column reduction over the graph's chunks, for 32
+// columns per block: grid (G, H/32), 8 warps; warp w sums chunks w, w+8, ...
+// (lanes = columns), the 8 warp sums are combined in fixed order.
+//   mode 0 (readout, Eq. 4): s = sig(Σ / N_g) -> outd (fp64), outf (fp32)
+//   mode 1 (dv):             Σ -> outd, outf; block (g, 0) also sums the
+//                            graph's loss partials -> loss_g[g]
+__global__ void k_chunk_sum(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
+                            const int32_t* __restrict__ node_off, int H, int mode,
+                            double* __restrict__ outd, float* __restrict__ outf,
+                            const double* __restrict__ loss_part, double* __restrict__ loss_g) {
+  __shared__ double sh[kWarps][32];
+  const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int c = blockIdx.y * 32 + lane;
+  const int cb = graph_chunk[g], ce = graph_chunk[g + 1];
+  double acc = 0.0;
+  for (int ch = cb + w; ch < ce; ch += kWarps) acc += part[(int64_t)ch * H + c];
+  sh[w][lane] = acc;
+  __syncthreads();
+  if (w == 0) {
+    double t = 0.0;
+#pragma unroll
+    for (int k = 0; k < kWarps; ++k) t += sh[k][lane];
+    if (mode == 0) t = 1.0 / (1.0 + exp(-(t / (double)(node_off[g + 1] - node_off[g]))));
+    outd[(int64_t)g * H + c] = t;
+    outf[(int64_t)g * H + c] = (float)t;
+  }
+  if (mode == 1 && blockIdx.y == 0 && w == 1) {          // graph loss: lanes stride, fixed tree
+    double t = 0.0;
+    for (int ch = cb + lane; ch < ce; ch += 32) t += loss_part[ch];
+    t = warp_sum(t);
+    if (lane == 0) loss_g[g] = t;
+  }
+}
+
+// v_g = M s_g (Eq. 5): grid (G, H/32); warp w computes rows r0 + 4w .. +3,
+// lanes stride the columns (coalesced rows of M), fixed-order warp reduction.
+__global__ void k_Mv(const float* __restrict__ M, const double* __restrict__ sd, int H,
+                     float* __restrict__ vf) {
+  const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const double* s = sd + (int64_t)g * H;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int r = blockIdx.y * 32 + w * 4 + i;
+    double t = 0.0;
+    for (int c = lane; c < H; c += 32) t += (double)M[(int64_t)r * H + c] * s[c];
+    t = warp_sum(t);
+    if (lane == 0) vf[(int64_t)g * H + r] = (float)t;
+  }
+}
+
+// ds = Mᵀ dv_g and dm = ds s (1 - s) / N_g: grid (G, H/32); lanes own 32
+// columns, warp w sums rows w, w+8, ... (coalesced), fixed-order combine.
+__global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dvd,
+                      const double* __restrict__ sd, const int32_t* __restrict__ node_off, int H,
+                      float* __restrict__ dmf) {
+  __shared__ double sh[kWarps][32];
+  const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int c = blockIdx.y * 32 + lane;
+  const double* dv = dvd + (int64_t)g * H;
+  double acc = 0.0;
+  for (int r = w; r < H; r += kWarps) acc += (double)M[(int64_t)r * H + c] * dv[r];
+  sh[w][lane] = acc;
+  __syncthreads();
+  if (w == 0) {
+    double ds = 0.0;
+#pragma unroll
+    for (int k = 0; k < kWarps; ++k) ds += sh[k][lane];
+    const double s = sd[(int64_t)g * H + c];
+    dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / (double)(node_off[g + 1] - node_off[g]));
+  }
+}
+
 // Per graph: m, s = sig(m) (Eq. 4), v = M s (Eq. 5).  Block = 256 threads.
 __global__ void k_readout(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
                           const int32_t* __restrict__ node_off, const float* __restrict__ M,
@@ -305,12 +377,16 @@ cudaError_t head_nc(const GraphDev& g, const float* Z3, const float* M, const fl
                     const StepParams* sp, const HeadWork& w, float* dZ, float* gM,
                     float* loss_out, int* nslots, cudaStream_t s) {
   constexpr int H = NC * 32;
+  const dim3 gh(g.G, H / 32);
   k_colsum<<<g.nchunks, 256, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
-  k_readout<<<g.G, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.node_off, M, H, w.sd, w.s, w.v);
+  k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.node_off, H, 0, w.sd, w.s,
+                                 nullptr, nullptr);
+  k_Mv<<<gh, 256, 0, s>>>(M, w.sd, H, w.v);
   k_score<NC><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph, g.node_off,
                                                 w.v, sp, g.Nt, w.dl, w.dv_part, w.loss_part);
-  k_head_bwd<<<g.G, 256, 0, s>>>(w.dv_part, w.loss_part, g.graph_chunk, g.node_off, M, w.sd, H,
-                                 w.dvd, w.dv, w.dm, w.loss_g);
+  k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.node_off, H, 1, w.dvd, w.dv,
+                                 w.loss_part, w.loss_g);
+  k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.node_off, H, w.dm);
   k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
   unsigned nb = cdiv(2LL * g.Nt, kWarps);
   k_dz3<NC><<<nb, kWarps * 32, 0, s>>>(Z3, alpha, g.node_graph, w.dl, w.v, w.dm, g.Nt, dZ,
@@ -327,7 +403,7 @@ cudaError_t launch_head(const GraphDev& g, int H, const float* Z3, const float* 
                         const float* alpha_dev, const StepParams* sp, const HeadWork& w,
                         float* dZ, float* grad_M, float* loss_out, int* nslots, cudaStream_t s,
                         int* launches) {
-  count_launch(launches, 6);
+  count_launch(launches, 8);
   switch (H) {
     case 32: return head_nc<1>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
     case 64: return head_nc<2>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
