@@ -100,11 +100,13 @@ class Clocks:
 
 
 # ------------------------------------------------------------------ algorithmic bytes / flops
-def spmm_bytes(N, Z, C, layer1=False, bwd=False, s=4):
+def spmm_bytes(N, Z, C, layer1=False, bwd=False, s=4, s_in=None):
     """Per SpMM launch over the stacked [pos; neg] rows:
     rowptr + (colind, val) + input rows + output rows (+ perm for layer 1,
-    + Z read for the backward epilogue)."""
-    b = 4 * (N + 1) + 8 * Z + 2 * N * C * s + 2 * N * C * s
+    + Z read for the backward epilogue).  s = storage bytes per element,
+    s_in = input element bytes when it differs (layer 1 reads fp32 X)."""
+    s_in = s if s_in is None else s_in
+    b = 4 * (N + 1) + 8 * Z + 2 * N * C * s_in + 2 * N * C * s
     if layer1:
         b += 4 * N
     if bwd:
@@ -112,17 +114,18 @@ def spmm_bytes(N, Z, C, layer1=False, bwd=False, s=4):
     return b
 
 
-def step_accounting(N, Z):
+def step_accounting(N, Z, s=4):
     """Per-step launches of each phase with algorithmic bytes / flops."""
     R = 2 * N
-    sp = [("spmm_fwd", spmm_bytes(N, Z, F, layer1=True)), ("spmm_fwd", spmm_bytes(N, Z, H)),
-          ("spmm_fwd", spmm_bytes(N, Z, H)), ("spmm_bwd", spmm_bytes(N, Z, H, bwd=True)),
-          ("spmm_bwd", spmm_bytes(N, Z, H, bwd=True))]
+    sp = [("spmm_fwd", spmm_bytes(N, Z, F, layer1=True, s=s, s_in=4)),
+          ("spmm_fwd", spmm_bytes(N, Z, H, s=s)), ("spmm_fwd", spmm_bytes(N, Z, H, s=s)),
+          ("spmm_bwd", spmm_bytes(N, Z, H, bwd=True, s=s)),
+          ("spmm_bwd", spmm_bytes(N, Z, H, bwd=True, s=s))]
     gemm = {"gemm_fwd": 2 * R * H * (F + H + H), "gemm_dw": 2 * R * H * (F + H + H),
             "gemm_dy": 2 * R * H * (H + H)}
-    gemm_bytes = {"gemm_fwd": 4 * R * ((F + H) + (H + H) + (H + H)),
-                  "gemm_dw": 4 * R * ((F + H) + (H + H) + (H + H)),
-                  "gemm_dy": 4 * R * ((H + H) + (H + H))}
+    gemm_bytes = {"gemm_fwd": s * R * ((F + H) + (H + H) + (H + H)),
+                  "gemm_dw": s * R * ((F + H) + (H + H) + (H + H)),
+                  "gemm_dy": s * R * ((H + H) + (H + H))}
     return sp, gemm, gemm_bytes
 
 
@@ -323,6 +326,38 @@ def run_mine(args):
                "note": "per step: mars_graph_load (H2D + CSR build) + mars_dgi_step + loss D2H, "
                        "wall clock, rank-local (no allreduce)"}
 
+    # the bf16 path (MARS_BF16, 2e-2 parity bar) on the same workload, same timing
+    b16 = None
+    if not args.no_bf16:
+        m16 = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local,
+                              world_size=world, rank=rank, nccl_unique_id=uid,
+                              precision=mars.MARS_BF16) if world == 1 else None
+        if m16 is not None:
+            m16.set_stream(stream.cuda_stream)
+            for w in range(args.warmup):
+                m16.step(g, w, base, B)
+            torch.cuda.synchronize()
+            ev0.record(stream)
+            for k in range(args.steps):
+                m16.step(g, args.warmup + k, base, B)
+            ev1.record(stream)
+            ev1.synchronize()
+            ms16 = ev0.elapsed_time(ev1)
+            acc16 = {}
+            for k in range(nprof):
+                for name, t in m16.profile_step(g, 10**6 + k, base, B):
+                    acc16.setdefault(name, []).append(t)
+            ps16 = {k: sum(v) / nprof for k, v in acc16.items()}
+            sp16 = ps16.get("spmm_fwd", 0) + ps16.get("spmm_bwd", 0)
+            sp16_bytes = sum(bb for _, bb in step_accounting(N, Z, s=2)[0])
+            b16 = {"value": world * b * args.steps / (ms16 / 1000.0), "unit": UNIT,
+                   "ms_per_step": ms16 / args.steps, "dtype": "bf16",
+                   "phases_ms_per_step": ps16,
+                   "spmm_gbs": sp16_bytes / (sp16 / 1e3) / 1e9 if sp16 else None,
+                   "note": "bf16 activations + bf16 tcgen05 MMAs, fp32 accumulation and "
+                           "master params; parity bar 2e-2 (tests/test_gpu_bf16.py)"}
+            m16.free()
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         import oracle
@@ -351,7 +386,8 @@ def run_mine(args):
                 "roofline": roof, "rooflines": rooflines, "spmm": spmm_obj,
                 "phases_ms_per_step": per_step, "phase_share": shares,
                 "profiled_step_ms": prof_total / nprof,
-                "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches}
+                "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
+                "bf16": b16}
         print(json.dumps(line), flush=True)
     m.free()
     g.free()
@@ -374,6 +410,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-bf16", action="store_true", help="skip the bf16-path measurement")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -928,6 +928,21 @@ int dw_tile(int CIN) { return CIN >= 128 ? 128 : 64; }
 
 }  // namespace
 
+// Shared with gemm_tc16.cu.
+bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base, int64_t rows,
+             int64_t cols, int box_cols, int box_rows, CUtensorMapSwizzle swz) {
+  if (!encode_fn()) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)cols * (cuuint64_t)elem_bytes};
+  cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
+  cuuint32_t es[2] = {1, 1};
+  return g_encode(m, dt, 2, const_cast<void*>(base), dims, strides, box, es,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+int tc_num_sms() { return num_sms(); }
+
 bool tc_supported(int K_or_cin, int N_or_h) {
   return N_or_h == 256 && (K_or_cin == 64 || K_or_cin == 128 || K_or_cin == 256);
 }

@@ -10,11 +10,13 @@
 //   dv_g = Σ dl_i H3[i] + Σ dl~_i H3~[i]; dM = Σ_g dv_g s_gᵀ; ds = Mᵀ dv;
 //   dm = ds ⊙ s(1-s); dH3 = dl v_g + [pos] dm_g / N_g; dZ3 = dH3 ⊙ PReLU'(Z3)
 // Every cross-row reduction is two-stage with fixed-order fp64 combination
-// over row chunks (<= kChunkRows rows, never straddling a graph): deterministic,
-// no float atomics.  The per-graph second stages are small and latency-bound;
-// they are spread over G x 8 warps with independent accumulators.
+// over row chunks (<= 256 rows, never straddling a graph): deterministic, no
+// float atomics.  The per-graph second stages are small and latency-bound; they
+// are spread over G x H/32 blocks.  Z3 / dZ3 are stored fp32 or bf16 (the
+// storage type of the path); arithmetic is fp32 / fp64.
 #include "common.cuh"
 #include "internal.cuh"
+#include "vec.cuh"
 
 namespace mars {
 namespace {
@@ -24,7 +26,8 @@ constexpr int kWarps = 8;
 // Stage 1 of m_g: per-chunk column sums of H3 over positive rows (fp64).
 // Block = 256 threads: threads own columns c = tid % H, rows split across
 // 256 / H row-groups, combined in fixed order through shared memory.
-__global__ void k_colsum(const float* __restrict__ Z3, const float* __restrict__ alpha,
+template <typename T>
+__global__ void k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
                          const int32_t* __restrict__ chunk_row, int H,
                          double* __restrict__ part) {
   __shared__ double sh[256];
@@ -36,10 +39,10 @@ __global__ void k_colsum(const float* __restrict__ Z3, const float* __restrict__
   const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
   int32_t r = r0 + gr;
   for (; r + groups < r1; r += 2 * groups) {
-    acc0 += (double)prelu(Z3[(int64_t)r * H + c], a);
-    acc1 += (double)prelu(Z3[(int64_t)(r + groups) * H + c], a);
+    acc0 += (double)prelu(to_f(Z3[(int64_t)r * H + c]), a);
+    acc1 += (double)prelu(to_f(Z3[(int64_t)(r + groups) * H + c]), a);
   }
-  if (r < r1) acc0 += (double)prelu(Z3[(int64_t)r * H + c], a);
+  if (r < r1) acc0 += (double)prelu(to_f(Z3[(int64_t)r * H + c]), a);
   sh[threadIdx.x] = acc0 + acc1;
   __syncthreads();
   if (gr == 0) {
@@ -121,38 +124,6 @@ __global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dv
   }
 }
 
-// Per graph: m, s = sig(m) (Eq. 4), v = M s (Eq. 5).  Block = 256 threads.
-__global__ void k_readout(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
-                          const int32_t* __restrict__ node_off, const float* __restrict__ M,
-                          int H, double* __restrict__ sd, float* __restrict__ sf,
-                          float* __restrict__ vf) {
-  __shared__ double sh_s[256];
-  const int g = blockIdx.x;
-  const double Ng = (double)(node_off[g + 1] - node_off[g]);
-  for (int c = threadIdx.x; c < H; c += blockDim.x) {
-    double a0 = 0.0, a1 = 0.0;
-    int ch = graph_chunk[g];
-    const int ce = graph_chunk[g + 1];
-    for (; ch + 1 < ce; ch += 2) {
-      a0 += part[(int64_t)ch * H + c];
-      a1 += part[(int64_t)(ch + 1) * H + c];
-    }
-    if (ch < ce) a0 += part[(int64_t)ch * H + c];
-    const double s = 1.0 / (1.0 + exp(-((a0 + a1) / Ng)));
-    sh_s[c] = s;
-    sd[(int64_t)g * H + c] = s;
-    sf[(int64_t)g * H + c] = (float)s;
-  }
-  __syncthreads();
-  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-  for (int r = w; r < H; r += nw) {                    // v[r] = Σ_c M[r][c] s[c]
-    double t = 0.0;
-    for (int cc = lane; cc < H; cc += 32) t += (double)M[(int64_t)r * H + cc] * sh_s[cc];
-    t = warp_sum(t);
-    if (lane == 0) vf[(int64_t)g * H + r] = (float)t;
-  }
-}
-
 __device__ __forceinline__ double softplus_d(double x) {
   return (x > 0.0 ? x : 0.0) + log1p(exp(-fabs(x)));
 }
@@ -160,9 +131,9 @@ __device__ __forceinline__ double softplus_d(double x) {
 // Scores, loss partials, dl, and dv partials.  One block (8 warps) per chunk;
 // each warp takes rows i of the chunk, both the positive row i and the
 // corrupted row Nt+i; lanes own H/32 columns.
-template <int NC>
+template <int NC, typename T>
 __global__ void __launch_bounds__(kWarps * 32)
-k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
+k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
         const int32_t* __restrict__ node_off, const float* __restrict__ vf,
         const StepParams* __restrict__ sp, int32_t Nt, float* __restrict__ dl,
@@ -179,11 +150,9 @@ k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
 #pragma unroll
   for (int q = 0; q < NC; ++q) v[q] = vf[(int64_t)g * H + lane + 32 * q];
   float dvp[NC];
-#pragma unroll
-  for (int q = 0; q < NC; ++q) dvp[q] = 0.f;
   double dv[NC];
 #pragma unroll
-  for (int q = 0; q < NC; ++q) dv[q] = 0.0;
+  for (int q = 0; q < NC; ++q) { dvp[q] = 0.f; dv[q] = 0.0; }
   double loss = 0.0;
   int cnt = 0;
   for (int32_t i = chunk_row[ch] + w; i < chunk_row[ch + 1]; i += kWarps) {
@@ -191,8 +160,8 @@ k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
     float lp = 0.f, ln = 0.f;
 #pragma unroll
     for (int q = 0; q < NC; ++q) {
-      hp[q] = prelu(Z3[(int64_t)i * H + lane + 32 * q], a);
-      hn[q] = prelu(Z3[((int64_t)Nt + i) * H + lane + 32 * q], a);
+      hp[q] = prelu(to_f(Z3[(int64_t)i * H + lane + 32 * q]), a);
+      hn[q] = prelu(to_f(Z3[((int64_t)Nt + i) * H + lane + 32 * q]), a);
       lp = fmaf(hp[q], v[q], lp);
       ln = fmaf(hn[q], v[q], ln);
     }
@@ -232,55 +201,6 @@ k_score(const float* __restrict__ Z3, const float* __restrict__ alpha,
   }
 }
 
-// Per graph: dv_g (fixed-order fp64 sum of chunks), ds = Mᵀ dv, dm = ds s(1-s)/N_g,
-// and the graph's loss.  Block = 256 threads; the Mᵀ dv product is split over
-// 256/H row groups with four independent accumulators each (fixed order).
-__global__ void k_head_bwd(const double* __restrict__ dv_part, const double* __restrict__ loss_part,
-                           const int32_t* __restrict__ graph_chunk,
-                           const int32_t* __restrict__ node_off, const float* __restrict__ M,
-                           const double* __restrict__ sd, int H, double* __restrict__ dvd,
-                           float* __restrict__ dvf, float* __restrict__ dmf,
-                           double* __restrict__ loss_g) {
-  __shared__ double sh_dv[256];
-  __shared__ double sh_ds[256];
-  const int g = blockIdx.x;
-  const int cb = graph_chunk[g], ce = graph_chunk[g + 1];
-  for (int c = threadIdx.x; c < H; c += blockDim.x) {
-    double a0 = 0.0, a1 = 0.0;
-    int ch = cb;
-    for (; ch + 1 < ce; ch += 2) {
-      a0 += dv_part[(int64_t)ch * H + c];
-      a1 += dv_part[(int64_t)(ch + 1) * H + c];
-    }
-    if (ch < ce) a0 += dv_part[(int64_t)ch * H + c];
-    sh_dv[c] = a0 + a1;
-    dvd[(int64_t)g * H + c] = a0 + a1;
-    dvf[(int64_t)g * H + c] = (float)(a0 + a1);
-  }
-  if (threadIdx.x == 0) {
-    double t = 0.0;
-    for (int ch = cb; ch < ce; ++ch) t += loss_part[ch];
-    loss_g[g] = t;
-  }
-  __syncthreads();
-  const int groups = blockDim.x / H;                  // 256/H row groups
-  const int c = threadIdx.x % H, gr = threadIdx.x / H;
-  const int rows = H / groups;
-  double a[4] = {0.0, 0.0, 0.0, 0.0};
-  for (int r = gr * rows; r < (gr + 1) * rows; r += 4)
-#pragma unroll
-    for (int k = 0; k < 4; ++k) a[k] += (double)M[(int64_t)(r + k) * H + c] * sh_dv[r + k];
-  sh_ds[threadIdx.x] = (a[0] + a[1]) + (a[2] + a[3]);
-  __syncthreads();
-  if (gr == 0) {
-    double ds = 0.0;
-    for (int k = 0; k < groups; ++k) ds += sh_ds[k * H + c];
-    const double s = sd[(int64_t)g * H + c];
-    const double Ng = (double)(node_off[g + 1] - node_off[g]);
-    dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / Ng);
-  }
-}
-
 // dM[r][c] = Σ_g dv_g[r] s_g[c] (fixed order); block 0 also writes the loss.
 __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ sd, int G, int H,
                      const double* __restrict__ loss_g, float* __restrict__ gM,
@@ -300,16 +220,17 @@ __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ 
 }
 
 // dZ3 = (dl v_g + [pos] dm_g) ⊙ PReLU'(Z3), dalpha3 partials.  Warp per row,
-// float4 columns.
-template <int NC>
+// 16-byte vectors of T.
+template <int NC, typename T>
 __global__ void __launch_bounds__(kWarps * 32)
-k_dz3(const float* __restrict__ Z3, const float* __restrict__ alpha,
+k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
       const int32_t* __restrict__ node_graph, const float* __restrict__ dl,
       const float* __restrict__ vf, const float* __restrict__ dmf, int32_t Nt,
-      float* __restrict__ dZ, double* __restrict__ slots) {
+      T* __restrict__ dZ, double* __restrict__ slots) {
   constexpr int H = NC * 32;
-  constexpr int V = H / 4;                           // float4 per row
-  constexpr int PER = (V + 31) / 32;
+  constexpr int V = Vec<T>::N;
+  constexpr int NV = H / V;                          // vectors per row
+  constexpr int PER = (NV + 31) / 32;
   __shared__ double wpart[kWarps];
   const int lane = threadIdx.x & 31;
   const int64_t r = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
@@ -320,26 +241,22 @@ k_dz3(const float* __restrict__ Z3, const float* __restrict__ alpha,
     const int g = node_graph[i];
     const float a = alpha[2];
     const float d = dl[r];
-    const float4* Z4 = reinterpret_cast<const float4*>(Z3 + r * H);
-    const float4* v4 = reinterpret_cast<const float4*>(vf + (int64_t)g * H);
-    const float4* m4 = reinterpret_cast<const float4*>(dmf + (int64_t)g * H);
-    float4* o4 = reinterpret_cast<float4*>(dZ + r * H);
+    const float* vg = vf + (int64_t)g * H;
+    const float* mg = dmf + (int64_t)g * H;
 #pragma unroll
     for (int q = 0; q < PER; ++q) {
-      const int c4 = lane + 32 * q;
-      if (c4 < V) {
-        const float4 z = Z4[c4], vv = v4[c4];
-        float4 dh = make_float4(d * vv.x, d * vv.y, d * vv.z, d * vv.w);
-        if (pos) {
-          const float4 mm = m4[c4];
-          dh.x += mm.x; dh.y += mm.y; dh.z += mm.z; dh.w += mm.w;
+      const int cv = lane + 32 * q;
+      if (cv < NV) {
+        const int c = cv * V;
+        float z[V], o[V];
+        Vec<T>::load(Z3 + r * H + c, z);
+#pragma unroll
+        for (int e = 0; e < V; ++e) {
+          const float dh = d * vg[c + e] + (pos ? mg[c + e] : 0.f);
+          o[e] = z[e] > 0.f ? dh : a * dh;
+          da += z[e] > 0.f ? 0.f : dh * z[e];
         }
-        float4 o;
-        o.x = z.x > 0.f ? dh.x : a * dh.x;  da += z.x > 0.f ? 0.f : dh.x * z.x;
-        o.y = z.y > 0.f ? dh.y : a * dh.y;  da += z.y > 0.f ? 0.f : dh.y * z.y;
-        o.z = z.z > 0.f ? dh.z : a * dh.z;  da += z.z > 0.f ? 0.f : dh.z * z.z;
-        o.w = z.w > 0.f ? dh.w : a * dh.w;  da += z.w > 0.f ? 0.f : dh.w * z.w;
-        o4[c4] = o;
+        StoreN<T, V>::store(dZ + r * H + c, o);
       }
     }
   }
@@ -366,51 +283,69 @@ __global__ void k_reduce_slots(const double* __restrict__ slots, int n, float* _
   if (threadIdx.x == 0) *out = (float)sh[0];
 }
 
-__global__ void k_prelu(const float* __restrict__ Z, const float* __restrict__ alpha, int layer,
+template <typename T>
+__global__ void k_prelu(const T* __restrict__ Z, const float* __restrict__ alpha, int layer,
                         float* __restrict__ out, int64_t n) {
   int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (e < n) out[e] = prelu(Z[e], alpha[layer]);
+  if (e < n) out[e] = prelu(to_f(Z[e]), alpha[layer]);
 }
 
-template <int NC>
-cudaError_t head_nc(const GraphDev& g, const float* Z3, const float* M, const float* alpha,
-                    const StepParams* sp, const HeadWork& w, float* dZ, float* gM,
-                    float* loss_out, int* nslots, cudaStream_t s) {
+__global__ void k_upcast(const bf16* __restrict__ in, float* __restrict__ out, int64_t n) {
+  int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e < n) out[e] = __bfloat162float(in[e]);
+}
+
+template <int NC, typename T>
+cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float* alpha,
+                    const StepParams* sp, const HeadWork& w, T* dZ, float* gM, float* loss_out,
+                    int* nslots, cudaStream_t s) {
   constexpr int H = NC * 32;
   const dim3 gh(g.G, H / 32);
-  k_colsum<<<g.nchunks, 256, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
+  k_colsum<T><<<g.nchunks, 256, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
   k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.node_off, H, 0, w.sd, w.s,
                                  nullptr, nullptr);
   k_Mv<<<gh, 256, 0, s>>>(M, w.sd, H, w.v);
-  k_score<NC><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph, g.node_off,
-                                                w.v, sp, g.Nt, w.dl, w.dv_part, w.loss_part);
+  k_score<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
+                                                   g.node_off, w.v, sp, g.Nt, w.dl, w.dv_part,
+                                                   w.loss_part);
   k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.node_off, H, 1, w.dvd, w.dv,
                                  w.loss_part, w.loss_g);
   k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.node_off, H, w.dm);
   k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
-  unsigned nb = cdiv(2LL * g.Nt, kWarps);
-  k_dz3<NC><<<nb, kWarps * 32, 0, s>>>(Z3, alpha, g.node_graph, w.dl, w.v, w.dm, g.Nt, dZ,
-                                       w.slots);
+  const unsigned nb = cdiv(2LL * g.Nt, kWarps);
+  k_dz3<NC, T><<<nb, kWarps * 32, 0, s>>>(Z3, alpha, g.node_graph, w.dl, w.v, w.dm, g.Nt, dZ,
+                                          w.slots);
   *nslots = (int)nb;
   return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t head_t(const GraphDev& g, int H, const void* Z3, const float* M, const float* alpha,
+                   const StepParams* sp, const HeadWork& w, void* dZ, float* gM, float* loss,
+                   int* nslots, cudaStream_t s) {
+  const T* z = static_cast<const T*>(Z3);
+  T* d = static_cast<T*>(dZ);
+  switch (H) {
+    case 32: return head_nc<1, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
+    case 64: return head_nc<2, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
+    case 128: return head_nc<4, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
+    case 256: return head_nc<8, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
+    default: return cudaErrorInvalidValue;
+  }
 }
 
 }  // namespace
 
 int head_slots(const GraphDev& g) { return (int)cdiv(2LL * g.Nt, kWarps) + 1; }
 
-cudaError_t launch_head(const GraphDev& g, int H, const float* Z3, const float* params_M,
-                        const float* alpha_dev, const StepParams* sp, const HeadWork& w,
-                        float* dZ, float* grad_M, float* loss_out, int* nslots, cudaStream_t s,
+cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, const float* params_M,
+                        const float* alpha_dev, const StepParams* sp, const HeadWork& w, void* dZ,
+                        float* grad_M, float* loss_out, int* nslots, cudaStream_t s,
                         int* launches) {
   count_launch(launches, 8);
-  switch (H) {
-    case 32: return head_nc<1>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
-    case 64: return head_nc<2>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
-    case 128: return head_nc<4>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
-    case 256: return head_nc<8>(g, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
-    default: return cudaErrorInvalidValue;
-  }
+  if (bf16_)
+    return head_t<bf16>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
+  return head_t<float>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
 }
 
 cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
@@ -420,10 +355,18 @@ cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStr
   return cudaGetLastError();
 }
 
-cudaError_t launch_prelu(const float* Z, const float* alpha_dev, int layer, float* out, int64_t n,
-                         cudaStream_t s, int* launches) {
+cudaError_t launch_prelu(const void* Z, int bf16_, const float* alpha_dev, int layer, float* out,
+                         int64_t n, cudaStream_t s, int* launches) {
   count_launch(launches);
-  k_prelu<<<cdiv(n, 256), 256, 0, s>>>(Z, alpha_dev, layer, out, n);
+  if (bf16_)
+    k_prelu<bf16><<<cdiv(n, 256), 256, 0, s>>>(static_cast<const bf16*>(Z), alpha_dev, layer, out, n);
+  else
+    k_prelu<float><<<cdiv(n, 256), 256, 0, s>>>(static_cast<const float*>(Z), alpha_dev, layer, out, n);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_upcast(const void* in, float* out, int64_t n, cudaStream_t s) {
+  k_upcast<<<cdiv(n, 256), 256, 0, s>>>(static_cast<const bf16*>(in), out, n);
   return cudaGetLastError();
 }
 

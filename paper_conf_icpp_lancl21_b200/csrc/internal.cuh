@@ -1,6 +1,7 @@
 // Internal declarations shared by the libmars.so translation units (kernels +
 // runtime).  Nothing here is part of the ABI; include/mars.h is.
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -95,13 +96,15 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
 // act(T[Nt+j]).  layer1: T = X (pos) and X[perm[j]] (neg), act = identity.
 // Otherwise act = PReLU(alpha[act_layer]).  neg_rows = 0 aggregates only the
 // positive branch (encode).
-cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const float* T, const int32_t* perm,
-                            const float* alpha_dev, int act_layer, float* Y, int both,
-                            cudaStream_t s, int* launches);
+// in_bf16 / out_bf16: storage type of T / Y (fp32 or bf16); fp32 accumulation.
+cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16,
+                            const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
+                            int out_bf16, int both, cudaStream_t s, int* launches);
 // Backward aggregate dH = Â_n dY (Â_n symmetric) with the PReLU'(Z) epilogue:
 // dZ = dH ⊙ (Z > 0 ? 1 : a), dalpha partials Σ dH·min(Z,0) -> slots[gridDim].
-cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const float* dY, const float* Z,
-                            const float* alpha_dev, int layer, float* dZ, double* slots,
+// dY, Z, dZ share one storage type (bf16 != 0: bf16).
+cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16,
+                            const float* alpha_dev, int layer, void* dZ, double* slots,
                             int* nslots, cudaStream_t s, int* launches);
 int spmm_bwd_slots(const GraphDev& g);
 
@@ -126,6 +129,20 @@ cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, f
 size_t tc_dw_partial_floats(int64_t R, int CIN);
 cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN,
                        float* part, cudaStream_t s, int* launches);
+bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,
+             int64_t rows, int64_t cols, int box_cols, int box_rows, CUtensorMapSwizzle swz);
+int tc_num_sms();
+
+// ---------------------------------------------------------------- gemm_tc16.cu
+// bf16 path (MARS_BF16): one kind::f16 MMA per k-step, bf16 operands, fp32
+// accumulation in TMEM.  Same support condition as tc_supported.
+cudaError_t tc16_weights(const float* W, int CIN, int H, void* Bt16, void* B16, cudaStream_t s,
+                         int* launches);   // Bt16 = bf16(Wᵀ) [H×Cin], B16 = bf16(W) [Cin×H]
+cudaError_t tc16_gemm_rows(const void* A, const void* B, void* C, int64_t M, int N, int K,
+                           cudaStream_t s, int* launches);   // C = A·Bᵀ, all bf16
+size_t tc16_dw_partial_floats(int64_t R, int CIN);
+cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, int CIN,
+                         float* part, cudaStream_t s, int* launches);
 
 // ---------------------------------------------------------------- head.cu
 struct HeadWork {
@@ -144,17 +161,20 @@ struct HeadWork {
 };
 // Forward head + head backward: writes grads of M (dM) and the loss slot,
 // dZ3 into dZ, dalpha3 partials into w.slots.
-cudaError_t launch_head(const GraphDev& g, int H, const float* Z3, const float* params_M,
-                        const float* alpha_dev, const StepParams* sp, const HeadWork& w,
-                        float* dZ, float* grad_M, float* loss_out, int* nslots,
+// Z3 / dZ storage: fp32 or bf16 (bf16 != 0).
+cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16,
+                        const float* params_M, const float* alpha_dev, const StepParams* sp,
+                        const HeadWork& w, void* dZ, float* grad_M, float* loss_out, int* nslots,
                         cudaStream_t s, int* launches);
 int head_slots(const GraphDev& g);
 // grad[0] = Σ slots (fixed order, double)
 cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
                                 int* launches);
-// H3 = PReLU(Z3) for the first `rows` rows (encode)
-cudaError_t launch_prelu(const float* Z, const float* alpha_dev, int layer, float* out,
+// H3 = PReLU(Z3) for the first `rows` rows (encode); Z fp32 or bf16, out fp32
+cudaError_t launch_prelu(const void* Z, int bf16, const float* alpha_dev, int layer, float* out,
                          int64_t n, cudaStream_t s, int* launches);
+// fp32 copy of a bf16 array (export hooks)
+cudaError_t launch_upcast(const void* in, float* out, int64_t n, cudaStream_t s);
 
 // ---------------------------------------------------------------- adam.cu
 cudaError_t launch_adam(float* params, float* m, float* v, const float* grads, int64_t P,

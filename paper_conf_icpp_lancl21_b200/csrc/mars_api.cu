@@ -212,6 +212,10 @@ struct Workspace {
   // tcgen05 path: per-layer hi/lo weight splits (Wᵀ for the forward, W for dY)
   float *wt_hi[3] = {}, *wt_lo[3] = {}, *w_hi[3] = {}, *w_lo[3] = {};
   float* dw_part = nullptr;
+  // bf16 path: bf16 weight copies (Wᵀ for the forward, W for dY), dW partials.
+  // (Activation buffers are sized for fp32 and hold bf16 in that mode.)
+  void *w16t[3] = {}, *w16[3] = {};
+  float* dw16_part = nullptr;
   std::vector<void*> owned;
   void release() {
     for (void* p : owned) cudaFree(p);
@@ -571,7 +575,11 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   if (!valid_F(cfg->in_dim)) return fail(MARS_EINVAL, "in_dim %d unsupported", cfg->in_dim);
   if (!valid_H(cfg->hidden_dim)) return fail(MARS_EINVAL, "hidden_dim %d unsupported", cfg->hidden_dim);
   if (cfg->num_layers != 3) return fail(MARS_EINVAL, "num_layers must be 3 (P:L101, c10)");
-  if (cfg->precision != MARS_FP32) return fail(MARS_EINVAL, "precision %d not built", cfg->precision);
+  if (cfg->precision != MARS_FP32 && cfg->precision != MARS_BF16)
+    return fail(MARS_EINVAL, "unknown precision %d", cfg->precision);
+  if (cfg->precision == MARS_BF16 &&
+      !(tc_supported(cfg->in_dim, cfg->hidden_dim) && tc_supported(cfg->hidden_dim, cfg->hidden_dim)))
+    return fail(MARS_EINVAL, "MARS_BF16 needs hidden_dim 256 and in_dim in {64, 128, 256}");
   if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
     return fail(MARS_EINVAL, "bad world_size/rank");
   if (cfg->world_size > 1 && !cfg->nccl_unique_id)
@@ -722,6 +730,15 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   }
   CK(al((void**)&w.dw_part, sizeof(float) * std::max(tc_dw_partial_floats(R, F),
                                                       tc_dw_partial_floats(R, H))));
+  if (m->cfg.precision == MARS_BF16) {
+    for (int l = 0; l < 3; ++l) {
+      const int64_t n = (int64_t)(l == 0 ? F : H) * H;
+      CK(al(&w.w16t[l], 2 * n));
+      CK(al(&w.w16[l], 2 * n));
+    }
+    CK(al((void**)&w.dw16_part, sizeof(float) * std::max(tc16_dw_partial_floats(R, F),
+                                                          tc16_dw_partial_floats(R, H))));
+  }
   w.Nt = (int32_t)Nt;
   w.G = G;
   w.nchunks = nch;
@@ -778,39 +795,46 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM)
   RET(launch_perm(g, m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
   MARK(MARS_PH_PERM);
+  const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     tc[l] = m->gemm_impl == 0 && tc_supported(Cin, H);
-    if (tc[l]) RET(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, nl));
+    if (b16) RET(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl));
+    else if (tc[l])
+      RET(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, nl));
   }
   MARK(MARS_PH_GEMM_FWD);
   // a5-a7: forward, l = 1..3
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
-    const float* T = l == 0 ? g.X : w.Z[l - 1];
-    RET(launch_spmm_fwd(g, Cin, T, w.perm, alpha, l - 1, Ys[l], 1, s, nl));
+    const void* T = l == 0 ? (const void*)g.X : (const void*)w.Z[l - 1];
+    RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.perm, alpha, l - 1, Ys[l], b16, 1, s, nl));
     MARK(MARS_PH_SPMM_FWD);
-    if (tc[l]) RET(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], R, H, Cin, s, nl));
+    if (b16) RET(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], R, H, Cin, s, nl));
+    else if (tc[l]) RET(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], R, H, Cin, s, nl));
     else RET(gemm_nn(Ys[l], W[l], w.Z[l], R, H, Cin, s, nl));
     MARK(MARS_PH_GEMM_FWD);
   }
   // a8-a11 + dZ3
   int ns = 0;
-  RET(launch_head(g, H, w.Z[2], Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl));
+  RET(launch_head(g, H, w.Z[2], b16, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl));
   RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
   MARK(MARS_PH_HEAD);
   // a12: backward, l = 3..1
   for (int l = 2; l >= 0; --l) {
     int Cin = l == 0 ? F : H;
-    if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, w.dw_part, s, nl));
+    if (b16) RET(tc16_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, w.dw16_part, s, nl));
+    else if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, w.dw_part, s, nl));
     else RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
     MARK(MARS_PH_GEMM_DW);
     if (l > 0) {
-      if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], w.dY, R, Cin, H, s, nl));
+      if (b16) RET(tc16_gemm_rows(w.dZ, w.w16[l], w.dY, R, Cin, H, s, nl));
+      else if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], w.dY, R, Cin, H, s, nl));
       else RET(gemm_nt(w.dZ, W[l], w.dY, R, Cin, H, s, nl));
       MARK(MARS_PH_GEMM_DY);
-      RET(launch_spmm_bwd(g, Cin, w.dY, w.Z[l - 1], alpha, l - 1, w.dZ, w.slots[l - 1], &ns, s, nl));
+      RET(launch_spmm_bwd(g, Cin, w.dY, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
+                          s, nl));
       MARK(MARS_PH_SPMM_BWD);
       RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
       MARK(MARS_PH_REDUCE);
@@ -980,18 +1004,22 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
   float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
   float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
   int nl = 0;
+  const bool b16 = m->cfg.precision == MARS_BF16;
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
-    const float* T = l == 0 ? gd.X : w.Z[l - 1];
-    CK(launch_spmm_fwd(gd, Cin, T, nullptr, alpha, l - 1, Ys[l], 0, s, &nl));
-    if (m->gemm_impl == 0 && tc_supported(Cin, H)) {
+    const void* T = l == 0 ? (const void*)gd.X : (const void*)w.Z[l - 1];
+    CK(launch_spmm_fwd(gd, Cin, T, b16 && l > 0, nullptr, alpha, l - 1, Ys[l], b16, 0, s, &nl));
+    if (b16) {
+      CK(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, &nl));
+      CK(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
+    } else if (m->gemm_impl == 0 && tc_supported(Cin, H)) {
       CK(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, &nl));
       CK(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
     } else {
       CK(gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
     }
   }
-  CK(launch_prelu(w.Z[2], alpha, 2, w.dY, (int64_t)gd.Nt * H, s, &nl));
+  CK(launch_prelu(w.Z[2], b16, alpha, 2, w.dY, (int64_t)gd.Nt * H, s, &nl));
   CK(cudaMemcpyAsync(emb, w.dY, sizeof(float) * (size_t)gd.Nt * H, cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   m->last_Nt = 0;
@@ -1009,6 +1037,20 @@ extern "C" mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t la
   int64_t R = 2LL * m->last_Nt;
   const float* Ys[3] = {m->ws.Y1, m->ws.Y23[0], m->ws.Y23[1]};
   int Cin = layer == 1 ? m->F : m->H;
+  if (m->cfg.precision == MARS_BF16) {     // upcast bf16 storage through a scratch buffer
+    float* tmp = nullptr;
+    CK(cudaMalloc(&tmp, sizeof(float) * R * std::max(Cin, m->H)));
+    struct FT { float* p; ~FT() { cudaFree(p); } } ft{tmp};
+    if (Y) {
+      CK(launch_upcast(Ys[layer - 1], tmp, R * Cin, nullptr));
+      CK(cudaMemcpy(Y, tmp, sizeof(float) * R * Cin, cudaMemcpyDeviceToHost));
+    }
+    if (Z) {
+      CK(launch_upcast(m->ws.Z[layer - 1], tmp, R * m->H, nullptr));
+      CK(cudaMemcpy(Z, tmp, sizeof(float) * R * m->H, cudaMemcpyDeviceToHost));
+    }
+    return MARS_OK;
+  }
   if (Y) CK(cudaMemcpy(Y, Ys[layer - 1], sizeof(float) * R * Cin, cudaMemcpyDeviceToHost));
   if (Z) CK(cudaMemcpy(Z, m->ws.Z[layer - 1], sizeof(float) * R * m->H, cudaMemcpyDeviceToHost));
   return MARS_OK;
