@@ -154,6 +154,20 @@ typedef struct {
 MARS_API mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
                           int64_t global_pair_base, int64_t global_batch, mars_step_out* out);
 
+/* NEXT-1, the pre-training schedule ("pre-train the graph encoder ...
+ * for 1000 iterations and save the parameters corresponding to the lowest
+ * loss"): n_steps consecutive mars_dgi_step calls (step indices step0 ..
+ * step0 + n_steps - 1) on `g`, tracking on the device, without host syncs,
+ * the lowest loss and the parameters that produced it (those before that
+ * step's Adam update; ties: the earliest step wins, c17).  Outputs (host,
+ * optional): losses [n_steps], best_params [P], best_loss, best_step (0-based
+ * within the run).  Synchronous.  The model's live parameters are the final
+ * ones (after n_steps updates). */
+MARS_API mars_status mars_dgi_pretrain(mars_dgi* m, const mars_graph* g, uint64_t step0,
+                                       int32_t n_steps, int64_t global_pair_base,
+                                       int64_t global_batch, float* losses, float* best_params,
+                                       float* best_loss, int64_t* best_step);
+
 /* a15: node embeddings H3 = encoder(X, A) of the positive branch (P:L132,
  * L153) for every node of the set, [ΣN × H] fp32 row-major HOST array.
  * Synchronous.  Overwrites the activations kept for the export hook. */

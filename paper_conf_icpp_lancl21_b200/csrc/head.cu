@@ -23,31 +23,74 @@ namespace {
 
 constexpr int kWarps = 8;
 
-// Stage 1 of m_g: per-chunk column sums of H3 over positive rows (fp64).
-// Block = 256 threads: threads own columns c = tid % H, rows split across
-// 256 / H row-groups, combined in fixed order through shared memory.
-template <typename T>
-__global__ void k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
-                         const int32_t* __restrict__ chunk_row, int H,
-                         double* __restrict__ part) {
-  __shared__ double sh[256];
-  const int groups = 256 / H;
-  const int c = threadIdx.x % H, gr = threadIdx.x / H;
+// Row tiling shared by the three streaming kernels: lanes cover a row with
+// 16-byte vectors of T (LPR lanes, PER vectors each); a warp keeps RU
+// consecutive rows in flight per iteration so every SM has >= 32 KB of loads
+// outstanding (Little's law at ~7 TB/s).
+template <int NC, typename T>
+struct RowTile {
+  static constexpr int H = NC * 32;
+  static constexpr int V = Vec<T>::N;
+  static constexpr int LPR = (H / V) < 32 ? (H / V) : 32;
+  static constexpr int PER = H / (V * LPR);
+  static constexpr int RU = PER >= 8 ? 1 : 8 / PER;
+};
+
+// Stage 1 of m_g: per-chunk column sums of H3 over positive rows.  Block = 8
+// warps; warp w takes RU consecutive rows per iteration, fp32 sums over the RU
+// rows folded into fp64, warp partials combined in fixed order through shared
+// memory.
+template <int NC, typename T>
+__global__ void __launch_bounds__(kWarps * 32)
+k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
+         const int32_t* __restrict__ chunk_row, double* __restrict__ part) {
+  using RT = RowTile<NC, T>;
+  constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER, RU = RT::RU;
+  __shared__ double sh[kWarps][H];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ch = blockIdx.x;
   const float a = alpha[2];
-  double acc0 = 0.0, acc1 = 0.0;
   const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
-  int32_t r = r0 + gr;
-  for (; r + groups < r1; r += 2 * groups) {
-    acc0 += (double)prelu(to_f(Z3[(int64_t)r * H + c]), a);
-    acc1 += (double)prelu(to_f(Z3[(int64_t)(r + groups) * H + c]), a);
+  const bool act = lane < LPR;
+  double d[PER][V];
+#pragma unroll
+  for (int q = 0; q < PER; ++q)
+#pragma unroll
+    for (int e = 0; e < V; ++e) d[q][e] = 0.0;
+  for (int32_t r = r0 + w * RU; r < r1; r += kWarps * RU) {
+    float x[RU][PER][V];
+#pragma unroll
+    for (int u = 0; u < RU; ++u)
+#pragma unroll
+      for (int q = 0; q < PER; ++q) {
+        if (act && r + u < r1) {
+          Vec<T>::load(Z3 + (int64_t)(r + u) * H + (lane + q * LPR) * V, x[u][q]);
+        } else {
+#pragma unroll
+          for (int e = 0; e < V; ++e) x[u][q][e] = 0.f;
+        }
+      }
+#pragma unroll
+    for (int q = 0; q < PER; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) {
+        float f = 0.f;
+#pragma unroll
+        for (int u = 0; u < RU; ++u) f += prelu(x[u][q][e], a);
+        d[q][e] += (double)f;
+      }
   }
-  if (r < r1) acc0 += (double)prelu(to_f(Z3[(int64_t)r * H + c]), a);
-  sh[threadIdx.x] = acc0 + acc1;
+  if (act) {
+#pragma unroll
+    for (int q = 0; q < PER; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) sh[w][(lane + q * LPR) * V + e] = d[q][e];
+  }
   __syncthreads();
-  if (gr == 0) {
+  for (int c = threadIdx.x; c < H; c += kWarps * 32) {
     double t = 0.0;
-    for (int k = 0; k < groups; ++k) t += sh[k * H + c];
+#pragma unroll
+    for (int k = 0; k < kWarps; ++k) t += sh[k][c];
     part[(int64_t)ch * H + c] = t;
   }
 }
@@ -129,8 +172,11 @@ __device__ __forceinline__ double softplus_d(double x) {
 }
 
 // Scores, loss partials, dl, and dv partials.  One block (8 warps) per chunk;
-// each warp takes rows i of the chunk, both the positive row i and the
-// corrupted row Nt+i; lanes own H/32 columns.
+// warp w takes NU consecutive nodes i per iteration, each with its positive
+// row i and corrupted row Nt+i (2 NU rows in flight); lanes own H/32 columns.
+// The 2 NU logits are reduced across the warp, then lane j < 2 NU evaluates
+// the sigmoid / softplus of logit j in fp64 (parallel over lanes) and the
+// dl values are broadcast back.
 template <int NC, typename T>
 __global__ void __launch_bounds__(kWarps * 32)
 k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
@@ -138,59 +184,98 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         const int32_t* __restrict__ node_off, const float* __restrict__ vf,
         const StepParams* __restrict__ sp, int32_t Nt, float* __restrict__ dl,
         double* __restrict__ dv_part, double* __restrict__ loss_part) {
-  constexpr int H = NC * 32;
+  using RT = RowTile<NC, T>;
+  constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER;
+  constexpr int NU = RT::RU >= 2 ? RT::RU / 2 : 1;
   __shared__ double sh_dv[kWarps][H];
   __shared__ double sh_loss[kWarps];
   const int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool act = lane < LPR;
   const int g = chunk_graph[ch];
   const float a = alpha[2];
   const double Ng = (double)(node_off[g + 1] - node_off[g]);
   const double coef = (double)sp->inv_batch / (2.0 * Ng);
-  float v[NC];
+  const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
+  float v[PER][V];
+  double dv[PER][V];
 #pragma unroll
-  for (int q = 0; q < NC; ++q) v[q] = vf[(int64_t)g * H + lane + 32 * q];
-  float dvp[NC];
-  double dv[NC];
+  for (int q = 0; q < PER; ++q)
 #pragma unroll
-  for (int q = 0; q < NC; ++q) { dvp[q] = 0.f; dv[q] = 0.0; }
+    for (int e = 0; e < V; ++e) {
+      v[q][e] = act ? vf[(int64_t)g * H + (lane + q * LPR) * V + e] : 0.f;
+      dv[q][e] = 0.0;
+    }
   double loss = 0.0;
-  int cnt = 0;
-  for (int32_t i = chunk_row[ch] + w; i < chunk_row[ch + 1]; i += kWarps) {
-    float hp[NC], hn[NC];
-    float lp = 0.f, ln = 0.f;
+  for (int32_t i = r0 + w * NU; i < r1; i += kWarps * NU) {
+    float h[2 * NU][PER][V];
 #pragma unroll
-    for (int q = 0; q < NC; ++q) {
-      hp[q] = prelu(to_f(Z3[(int64_t)i * H + lane + 32 * q]), a);
-      hn[q] = prelu(to_f(Z3[((int64_t)Nt + i) * H + lane + 32 * q]), a);
-      lp = fmaf(hp[q], v[q], lp);
-      ln = fmaf(hn[q], v[q], ln);
-    }
-    lp = warp_sum(lp);
-    ln = warp_sum(ln);
-    const double sp_ = 1.0 / (1.0 + exp(-(double)lp));
-    const double sn_ = 1.0 / (1.0 + exp(-(double)ln));
-    const float dlp = (float)((sp_ - 1.0) * coef);
-    const float dln = (float)(sn_ * coef);
-    if (lane == 0) {
-      dl[i] = dlp;
-      dl[Nt + i] = dln;
-      loss += softplus_d(-(double)lp) + softplus_d((double)ln);
-    }
-    // fp32 partials over <= 8 rows, then folded into fp64
+    for (int u = 0; u < NU; ++u)
 #pragma unroll
-    for (int q = 0; q < NC; ++q) dvp[q] = fmaf(dlp, hp[q], fmaf(dln, hn[q], dvp[q]));
-    if (++cnt == 8) {
+      for (int q = 0; q < PER; ++q) {
+        const int c = (lane + q * LPR) * V;
+        if (act && i + u < r1) {
+          Vec<T>::load(Z3 + (int64_t)(i + u) * H + c, h[2 * u][q]);
+          Vec<T>::load(Z3 + ((int64_t)Nt + i + u) * H + c, h[2 * u + 1][q]);
+        } else {
 #pragma unroll
-      for (int q = 0; q < NC; ++q) { dv[q] += (double)dvp[q]; dvp[q] = 0.f; }
-      cnt = 0;
+          for (int e = 0; e < V; ++e) h[2 * u][q][e] = h[2 * u + 1][q][e] = 0.f;
+        }
+      }
+    float l[2 * NU];
+#pragma unroll
+    for (int j = 0; j < 2 * NU; ++j) {
+      float t = 0.f;
+#pragma unroll
+      for (int q = 0; q < PER; ++q)
+#pragma unroll
+        for (int e = 0; e < V; ++e) {
+          h[j][q][e] = prelu(h[j][q][e], a);
+          t = fmaf(h[j][q][e], v[q][e], t);
+        }
+      l[j] = warp_sum(t);
     }
+    float mine = l[0];
+#pragma unroll
+    for (int j = 1; j < 2 * NU; ++j) mine = lane == j ? l[j] : mine;
+    float dmine = 0.f;
+    if (lane < 2 * NU && i + (lane >> 1) < r1) {
+      const double x = (double)mine;
+      const double sg = 1.0 / (1.0 + exp(-x));
+      const bool neg = lane & 1;
+      dmine = (float)((neg ? sg : sg - 1.0) * coef);
+      dl[(neg ? (int64_t)Nt : 0) + i + (lane >> 1)] = dmine;
+      loss += neg ? softplus_d(x) : softplus_d(-x);
+    }
+    float dvp[PER][V];
+#pragma unroll
+    for (int q = 0; q < PER; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) dvp[q][e] = 0.f;
+#pragma unroll
+    for (int j = 0; j < 2 * NU; ++j) {
+      const float dj = __shfl_sync(kFull, dmine, j);
+#pragma unroll
+      for (int q = 0; q < PER; ++q)
+#pragma unroll
+        for (int e = 0; e < V; ++e) dvp[q][e] = fmaf(dj, h[j][q][e], dvp[q][e]);
+    }
+#pragma unroll
+    for (int q = 0; q < PER; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) dv[q][e] += (double)dvp[q][e];
   }
+  if (act) {
 #pragma unroll
-  for (int q = 0; q < NC; ++q) sh_dv[w][lane + 32 * q] = dv[q] + (double)dvp[q];
+    for (int q = 0; q < PER; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) sh_dv[w][(lane + q * LPR) * V + e] = dv[q][e];
+  }
+  loss = warp_sum(loss);
   if (lane == 0) sh_loss[w] = loss;
   __syncthreads();
   for (int c = threadIdx.x; c < H; c += kWarps * 32) {
     double t = 0.0;
+#pragma unroll
     for (int k = 0; k < kWarps; ++k) t += sh_dv[k][c];
     dv_part[(int64_t)ch * H + c] = t;
   }
@@ -219,54 +304,76 @@ __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ 
   }
 }
 
-// dZ3 = (dl v_g + [pos] dm_g) ⊙ PReLU'(Z3), dalpha3 partials.  Warp per row,
-// 16-byte vectors of T.
+// dZ3 = (dl v_g + [pos] dm_g) ⊙ PReLU'(Z3), dalpha3 partials.  Grid (chunk,
+// half): block (ch, 0) covers the chunk's positive rows, (ch, 1) the matching
+// corrupted rows Nt + i.  v_g and dm_g are loaded once per block into
+// registers; warp w streams RU consecutive rows per iteration.  One dalpha
+// slot per block, folded in fixed order.
 template <int NC, typename T>
 __global__ void __launch_bounds__(kWarps * 32)
 k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
-      const int32_t* __restrict__ node_graph, const float* __restrict__ dl,
-      const float* __restrict__ vf, const float* __restrict__ dmf, int32_t Nt,
-      T* __restrict__ dZ, double* __restrict__ slots) {
-  constexpr int H = NC * 32;
-  constexpr int V = Vec<T>::N;
-  constexpr int NV = H / V;                          // vectors per row
-  constexpr int PER = (NV + 31) / 32;
+      const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
+      const float* __restrict__ dl, const float* __restrict__ vf, const float* __restrict__ dmf,
+      int32_t Nt, T* __restrict__ dZ, double* __restrict__ slots) {
+  using RT = RowTile<NC, T>;
+  constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER, RU = RT::RU;
   __shared__ double wpart[kWarps];
-  const int lane = threadIdx.x & 31;
-  const int64_t r = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
-  float da = 0.f;
-  if (r < 2LL * Nt) {
-    const int32_t i = (int32_t)(r < Nt ? r : r - Nt);
-    const bool pos = r < Nt;
-    const int g = node_graph[i];
-    const float a = alpha[2];
-    const float d = dl[r];
-    const float* vg = vf + (int64_t)g * H;
-    const float* mg = dmf + (int64_t)g * H;
+  const int ch = blockIdx.x, half = blockIdx.y;
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool act = lane < LPR;
+  const int g = chunk_graph[ch];
+  const float a = alpha[2];
+  const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
+  const int64_t base = half ? (int64_t)Nt : 0;
+  float vg[PER][V], mg[PER][V];
 #pragma unroll
-    for (int q = 0; q < PER; ++q) {
-      const int cv = lane + 32 * q;
-      if (cv < NV) {
-        const int c = cv * V;
-        float z[V], o[V];
-        Vec<T>::load(Z3 + r * H + c, z);
+  for (int q = 0; q < PER; ++q)
 #pragma unroll
-        for (int e = 0; e < V; ++e) {
-          const float dh = d * vg[c + e] + (pos ? mg[c + e] : 0.f);
-          o[e] = z[e] > 0.f ? dh : a * dh;
-          da += z[e] > 0.f ? 0.f : dh * z[e];
+    for (int e = 0; e < V; ++e) {
+      const int64_t c = (int64_t)g * H + (lane + q * LPR) * V + e;
+      vg[q][e] = act ? vf[c] : 0.f;
+      mg[q][e] = (act && !half) ? dmf[c] : 0.f;
+    }
+  double da = 0.0;
+  for (int32_t r = r0 + w * RU; r < r1; r += kWarps * RU) {
+    float z[RU][PER][V], d[RU];
+#pragma unroll
+    for (int u = 0; u < RU; ++u) {
+      const bool ok = r + u < r1;
+      d[u] = ok ? dl[base + r + u] : 0.f;
+#pragma unroll
+      for (int q = 0; q < PER; ++q) {
+        if (act && ok) {
+          Vec<T>::load(Z3 + (base + r + u) * H + (lane + q * LPR) * V, z[u][q]);
+        } else {
+#pragma unroll
+          for (int e = 0; e < V; ++e) z[u][q][e] = 0.f;
         }
-        StoreN<T, V>::store(dZ + r * H + c, o);
       }
     }
+    float daf = 0.f;
+#pragma unroll
+    for (int u = 0; u < RU; ++u)
+#pragma unroll
+      for (int q = 0; q < PER; ++q) {
+        float o[V];
+#pragma unroll
+        for (int e = 0; e < V; ++e) {
+          const float dh = fmaf(d[u], vg[q][e], mg[q][e]);
+          o[e] = z[u][q][e] > 0.f ? dh : a * dh;
+          daf += z[u][q][e] > 0.f ? 0.f : dh * z[u][q][e];
+        }
+        if (act && r + u < r1) StoreN<T, V>::store(dZ + (base + r + u) * H + (lane + q * LPR) * V, o);
+      }
+    da += (double)daf;
   }
-  const double t = warp_sum((double)da);
-  if (lane == 0) wpart[threadIdx.x >> 5] = t;
+  da = warp_sum(da);
+  if (lane == 0) wpart[w] = da;
   __syncthreads();
   if (threadIdx.x == 0) {
     double s = 0.0;
     for (int k = 0; k < kWarps; ++k) s += wpart[k];
-    slots[blockIdx.x] = s;
+    slots[(int64_t)ch * 2 + half] = s;
   }
 }
 
@@ -301,7 +408,7 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
                     int* nslots, cudaStream_t s) {
   constexpr int H = NC * 32;
   const dim3 gh(g.G, H / 32);
-  k_colsum<T><<<g.nchunks, 256, 0, s>>>(Z3, alpha, g.chunk_row, H, w.colsum_part);
+  k_colsum<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, w.colsum_part);
   k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.node_off, H, 0, w.sd, w.s,
                                  nullptr, nullptr);
   k_Mv<<<gh, 256, 0, s>>>(M, w.sd, H, w.v);
@@ -312,10 +419,9 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
                                  w.loss_part, w.loss_g);
   k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.node_off, H, w.dm);
   k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
-  const unsigned nb = cdiv(2LL * g.Nt, kWarps);
-  k_dz3<NC, T><<<nb, kWarps * 32, 0, s>>>(Z3, alpha, g.node_graph, w.dl, w.v, w.dm, g.Nt, dZ,
-                                          w.slots);
-  *nslots = (int)nb;
+  k_dz3<NC, T><<<dim3(g.nchunks, 2), kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
+                                                          w.dl, w.v, w.dm, g.Nt, dZ, w.slots);
+  *nslots = 2 * g.nchunks;
   return cudaGetLastError();
 }
 
@@ -336,7 +442,7 @@ cudaError_t head_t(const GraphDev& g, int H, const void* Z3, const float* M, con
 
 }  // namespace
 
-int head_slots(const GraphDev& g) { return (int)cdiv(2LL * g.Nt, kWarps) + 1; }
+int head_slots(const GraphDev& g) { return 2 * g.nchunks + 1; }
 
 cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, const float* params_M,
                         const float* alpha_dev, const StepParams* sp, const HeadWork& w, void* dZ,

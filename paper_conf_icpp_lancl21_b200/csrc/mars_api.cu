@@ -917,11 +917,107 @@ extern "C" mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, u
   return MARS_OK;
 }
 
+static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
+                            int64_t pair_base, int64_t global_batch);
+
 extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
                                      int64_t pair_base, int64_t global_batch, mars_step_out* out) {
   if (mars_status st = check_step_args(m, g, global_batch)) return st;
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
+  if (mars_status st = run_step(m, g, step_index, pair_base, global_batch)) return st;
+  cudaStream_t s = m->stream;
+  if (out && (out->loss || out->grads || out->perms)) {
+    float loss = 0.f;
+    CK(cudaMemcpyAsync(&loss, m->grads + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+    if (out->grads)
+      CK(cudaMemcpyAsync(out->grads, m->grads, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
+    if (out->perms)
+      CK(cudaMemcpyAsync(out->perms, m->ws.perm, sizeof(int32_t) * g->Nt, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (out->perms)
+      for (int gi = 0; gi < g->G; ++gi)
+        for (int32_t i = g->h_node_off[gi]; i < g->h_node_off[gi + 1]; ++i)
+          out->perms[i] -= g->h_node_off[gi];
+    if (out->loss) *out->loss = loss;
+    if (!std::isfinite(loss)) return fail(MARS_ENUMERIC, "non-finite loss");
+  }
+  return MARS_OK;
+}
+
+namespace {
+// NEXT-1 best-loss tracking (c17): strict < keeps the earliest minimum.
+__global__ void k_track_decide(const float* __restrict__ loss, int64_t t, float* __restrict__ losses,
+                               float* __restrict__ best_loss, int64_t* __restrict__ best_step,
+                               int32_t* __restrict__ flag) {
+  const float l = *loss;
+  losses[t] = l;
+  const bool better = l < *best_loss;
+  *flag = better ? 1 : 0;
+  if (better) {
+    *best_loss = l;
+    *best_step = t;
+  }
+}
+__global__ void k_track_copy(const int32_t* __restrict__ flag, const float* __restrict__ prev,
+                             float* __restrict__ best, int64_t P) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < P && *flag) best[i] = prev[i];
+}
+__global__ void k_init_best(float* best_loss, int64_t* best_step) {
+  *best_loss = INFINITY;
+  *best_step = -1;
+}
+}  // namespace
+
+extern "C" mars_status mars_dgi_pretrain(mars_dgi* m, const mars_graph* g, uint64_t step0,
+                                         int32_t n_steps, int64_t pair_base, int64_t global_batch,
+                                         float* losses, float* best_params, float* best_loss,
+                                         int64_t* best_step) {
+  if (mars_status st = check_step_args(m, g, global_batch)) return st;
+  if (n_steps < 1) return fail(MARS_EINVAL, "n_steps < 1");
+  CK(cudaSetDevice(m->cfg.device));
+  if (mars_status st = ensure_ws(m, g)) return st;
+  cudaStream_t s = m->stream;
+  float *prev = nullptr, *best = nullptr, *d_losses = nullptr, *d_bl = nullptr;
+  int64_t* d_bs = nullptr;
+  int32_t* d_flag = nullptr;
+  struct FreeAll {
+    std::vector<void*> v;
+    ~FreeAll() { for (void* p : v) cudaFree(p); }
+  } fa;
+  CK(dalloc(&prev, m->P)); fa.v.push_back(prev);
+  CK(dalloc(&best, m->P)); fa.v.push_back(best);
+  CK(dalloc(&d_losses, (size_t)n_steps)); fa.v.push_back(d_losses);
+  CK(dalloc(&d_bl, 1)); fa.v.push_back(d_bl);
+  CK(dalloc(&d_bs, 1)); fa.v.push_back(d_bs);
+  CK(dalloc(&d_flag, 1)); fa.v.push_back(d_flag);
+  k_init_best<<<1, 1, 0, s>>>(d_bl, d_bs);
+  CK(cudaMemcpyAsync(best, m->params, sizeof(float) * m->P, cudaMemcpyDeviceToDevice, s));
+  for (int32_t t = 0; t < n_steps; ++t) {
+    // the parameters a step's loss is computed with are the ones before its Adam update
+    CK(cudaMemcpyAsync(prev, m->params, sizeof(float) * m->P, cudaMemcpyDeviceToDevice, s));
+    if (mars_status st = run_step(m, g, step0 + (uint64_t)t, pair_base, global_batch)) return st;
+    k_track_decide<<<1, 1, 0, s>>>(m->grads + m->P, t, d_losses, d_bl, d_bs, d_flag);
+    k_track_copy<<<cdiv(m->P, 256), 256, 0, s>>>(d_flag, prev, best, m->P);
+    CK(cudaGetLastError());
+  }
+  int64_t bs = -1;
+  float bl = 0.f;
+  if (losses) CK(cudaMemcpyAsync(losses, d_losses, sizeof(float) * n_steps, cudaMemcpyDeviceToHost, s));
+  if (best_params) CK(cudaMemcpyAsync(best_params, best, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&bl, d_bl, sizeof(float), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&bs, d_bs, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (best_loss) *best_loss = bl;
+  if (best_step) *best_step = bs;
+  if (bs < 0) return fail(MARS_ENUMERIC, "no finite loss during pre-training");
+  return MARS_OK;
+}
+
+// Enqueues one step (graph replay or eager) after the step scalars.
+static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
+                            int64_t pair_base, int64_t global_batch) {
   cudaStream_t s = m->stream;
   if (mars_status st = push_step_params(m, step_index, pair_base, global_batch)) return st;
 
@@ -966,21 +1062,6 @@ extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t 
   }
   m->last_launches = nl;
   m->last_Nt = g->Nt;
-  if (out && (out->loss || out->grads || out->perms)) {
-    float loss = 0.f;
-    CK(cudaMemcpyAsync(&loss, m->grads + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
-    if (out->grads)
-      CK(cudaMemcpyAsync(out->grads, m->grads, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
-    if (out->perms)
-      CK(cudaMemcpyAsync(out->perms, m->ws.perm, sizeof(int32_t) * g->Nt, cudaMemcpyDeviceToHost, s));
-    CK(cudaStreamSynchronize(s));
-    if (out->perms)
-      for (int gi = 0; gi < g->G; ++gi)
-        for (int32_t i = g->h_node_off[gi]; i < g->h_node_off[gi + 1]; ++i)
-          out->perms[i] -= g->h_node_off[gi];
-    if (out->loss) *out->loss = loss;
-    if (!std::isfinite(loss)) return fail(MARS_ENUMERIC, "non-finite loss");
-  }
   return MARS_OK;
 }
 

@@ -74,6 +74,10 @@ SIGNATURES = {
     "mars_dgi_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                      ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(StepOut)]),
     "mars_encode": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_pretrain": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
+                                         ctypes.c_int32, ctypes.c_int64, ctypes.c_int64,
+                                         ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                         ctypes.c_void_p]),
     "mars_dgi_export_activations": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32,
                                                    ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dgi_get_state": (ctypes.c_int, [ctypes.c_void_p] * 4 + [ctypes.c_void_p]),
@@ -226,6 +230,20 @@ class DGI:
 
     def encode(self, g: Graph):
         return encode(self, g)
+
+    def pretrain(self, g: Graph, n_steps: int, step0: int = 0, pair_base: int = 0,
+                 global_batch: int | None = None):
+        """mars_dgi_pretrain: returns dict(losses, best_params, best_loss,
+        best_step)."""
+        B = g.num_graphs if global_batch is None else int(global_batch)
+        losses = np.zeros(n_steps, np.float32)
+        best = np.zeros(self.P, np.float32)
+        bl = ctypes.c_float(); bs = ctypes.c_int64()
+        _check(lib().mars_dgi_pretrain(self.handle, g.handle, step0 & (2 ** 64 - 1), int(n_steps),
+                                       int(pair_base), B, _ptr(losses), _ptr(best),
+                                       ctypes.byref(bl), ctypes.byref(bs)))
+        self._last_nt = g.total_nodes
+        return dict(losses=losses, best_params=best, best_loss=bl.value, best_step=bs.value)
 
     def export_activations(self, layer: int):
         return dgi_export_activations(self, layer)

@@ -242,3 +242,25 @@ def test_training_decreases_loss():
         m.step(g, s, 0)
     last = m.step(g, 200, 0, want_loss=True)["loss"]
     assert last < first and last < np.log(2)
+
+
+def test_pretrain_best_loss_snapshot():
+    """NEXT-1: mars_dgi_pretrain equals a manual step loop, and the
+    snapshot is the parameter vector that produced the lowest loss (earliest
+    minimum, c17)."""
+    gs = [SG.tiny(0), SG.tiny(1)]
+    n = 30
+    g = mars.graph_load(gs)
+    ma = mars.dgi_create(in_dim=16, hidden_dim=32, seed=21, lr=3e-3)
+    res = ma.pretrain(g, n, step0=5)
+    mb = mars.dgi_create(in_dim=16, hidden_dim=32, seed=21, lr=3e-3)
+    losses, before = [], []
+    for t in range(n):
+        before.append(mb.get_state()[0])
+        losses.append(mb.step(g, 5 + t, 0, want_loss=True)["loss"])
+    losses = np.array(losses, np.float32)
+    assert np.array_equal(res["losses"], losses)
+    k = int(np.argmin(losses))
+    assert res["best_step"] == k and res["best_loss"] == losses[k]
+    assert np.array_equal(res["best_params"], before[k])
+    assert np.array_equal(ma.get_state()[0], mb.get_state()[0])
