@@ -326,12 +326,7 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 // dW[c][h] = Σ_chunk part[chunk][h][c], fixed order, fp64.
 __global__ void k_dw16_reduce(const float* __restrict__ part, int nchunk, int CIN,
                               float* __restrict__ dW) {
-  int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (e >= 256LL * CIN) return;
-  double t = 0.0;
-  for (int k = 0; k < nchunk; ++k) t += (double)part[(int64_t)k * 256 * CIN + e];
-  int h = (int)(e / CIN), c = (int)(e % CIN);
-  dW[(int64_t)c * 256 + h] = (float)t;
+  dw_reduce_body(part, nchunk, CIN, dW);
 }
 
 __global__ void k_w16(const float* __restrict__ W, int CIN, int H, bf16* __restrict__ Bt,
@@ -439,7 +434,7 @@ cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, in
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
-  k_dw16_reduce<<<cdiv(256LL * CIN, 256), 256, 0, s>>>(part, nchunk, CIN, dW);
+  k_dw16_reduce<<<cdiv(256LL * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, dW);
   return cudaGetLastError();
 }
 

@@ -41,7 +41,7 @@ struct RowTile {
 // rows folded into fp64, warp partials combined in fixed order through shared
 // memory.
 template <int NC, typename T>
-__global__ void __launch_bounds__(kWarps * 32)
+__global__ void __launch_bounds__(kWarps * 32, 3)
 k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
          const int32_t* __restrict__ chunk_row, double* __restrict__ part) {
   using RT = RowTile<NC, T>;
@@ -58,27 +58,29 @@ k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
 #pragma unroll
     for (int e = 0; e < V; ++e) d[q][e] = 0.0;
   for (int32_t r = r0 + w * RU; r < r1; r += kWarps * RU) {
-    float x[RU][PER][V];
+    typename Vec<T>::Raw xr[RU][PER];
 #pragma unroll
     for (int u = 0; u < RU; ++u)
 #pragma unroll
-      for (int q = 0; q < PER; ++q) {
-        if (act && r + u < r1) {
-          Vec<T>::load(Z3 + (int64_t)(r + u) * H + (lane + q * LPR) * V, x[u][q]);
-        } else {
+      for (int q = 0; q < PER; ++q)
+        xr[u][q] = (act && r + u < r1)
+                       ? Vec<T>::ld(Z3 + (int64_t)(r + u) * H + (lane + q * LPR) * V)
+                       : typename Vec<T>::Raw{};
 #pragma unroll
-          for (int e = 0; e < V; ++e) x[u][q][e] = 0.f;
-        }
+    for (int q = 0; q < PER; ++q) {
+      float f[V];
+#pragma unroll
+      for (int e = 0; e < V; ++e) f[e] = 0.f;
+#pragma unroll
+      for (int u = 0; u < RU; ++u) {
+        float x[V];
+        Vec<T>::cvt(xr[u][q], x);
+#pragma unroll
+        for (int e = 0; e < V; ++e) f[e] += prelu(x[e], a);
       }
 #pragma unroll
-    for (int q = 0; q < PER; ++q)
-#pragma unroll
-      for (int e = 0; e < V; ++e) {
-        float f = 0.f;
-#pragma unroll
-        for (int u = 0; u < RU; ++u) f += prelu(x[u][q][e], a);
-        d[q][e] += (double)f;
-      }
+      for (int e = 0; e < V; ++e) d[q][e] += (double)f[e];
+    }
   }
   if (act) {
 #pragma unroll
@@ -178,7 +180,10 @@ __device__ __forceinline__ double softplus_d(double x) {
 // the sigmoid / softplus of logit j in fp64 (parallel over lanes) and the
 // dl values are broadcast back.
 template <int NC, typename T>
-__global__ void __launch_bounds__(kWarps * 32)
+#ifndef MARS_SCORE_MINB
+#define MARS_SCORE_MINB 3
+#endif
+__global__ void __launch_bounds__(kWarps * 32, MARS_SCORE_MINB)
 k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
         const int32_t* __restrict__ node_off, const float* __restrict__ vf,
@@ -186,7 +191,7 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         double* __restrict__ dv_part, double* __restrict__ loss_part) {
   using RT = RowTile<NC, T>;
   constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER;
-  constexpr int NU = RT::RU >= 2 ? RT::RU / 2 : 1;
+  constexpr int NU = RT::RU >= 4 ? 2 : 1;          // nodes per iteration (2 NU rows)
   __shared__ double sh_dv[kWarps][H];
   __shared__ double sh_loss[kWarps];
   const int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -207,18 +212,18 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
     }
   double loss = 0.0;
   for (int32_t i = r0 + w * NU; i < r1; i += kWarps * NU) {
-    float h[2 * NU][PER][V];
+    // rows kept as raw 16-byte vectors (4 registers each) and converted on use
+    typename Vec<T>::Raw h[2 * NU][PER];
 #pragma unroll
     for (int u = 0; u < NU; ++u)
 #pragma unroll
       for (int q = 0; q < PER; ++q) {
         const int c = (lane + q * LPR) * V;
         if (act && i + u < r1) {
-          Vec<T>::load(Z3 + (int64_t)(i + u) * H + c, h[2 * u][q]);
-          Vec<T>::load(Z3 + ((int64_t)Nt + i + u) * H + c, h[2 * u + 1][q]);
+          h[2 * u][q] = Vec<T>::ld(Z3 + (int64_t)(i + u) * H + c);
+          h[2 * u + 1][q] = Vec<T>::ld(Z3 + ((int64_t)Nt + i + u) * H + c);
         } else {
-#pragma unroll
-          for (int e = 0; e < V; ++e) h[2 * u][q][e] = h[2 * u + 1][q][e] = 0.f;
+          h[2 * u][q] = h[2 * u + 1][q] = typename Vec<T>::Raw{};
         }
       }
     float l[2 * NU];
@@ -226,12 +231,12 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
     for (int j = 0; j < 2 * NU; ++j) {
       float t = 0.f;
 #pragma unroll
-      for (int q = 0; q < PER; ++q)
+      for (int q = 0; q < PER; ++q) {
+        float x[V];
+        Vec<T>::cvt(h[j][q], x);
 #pragma unroll
-        for (int e = 0; e < V; ++e) {
-          h[j][q][e] = prelu(h[j][q][e], a);
-          t = fmaf(h[j][q][e], v[q][e], t);
-        }
+        for (int e = 0; e < V; ++e) t = fmaf(prelu(x[e], a), v[q][e], t);
+      }
       l[j] = warp_sum(t);
     }
     float mine = l[0];
@@ -255,9 +260,12 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
     for (int j = 0; j < 2 * NU; ++j) {
       const float dj = __shfl_sync(kFull, dmine, j);
 #pragma unroll
-      for (int q = 0; q < PER; ++q)
+      for (int q = 0; q < PER; ++q) {
+        float x[V];
+        Vec<T>::cvt(h[j][q], x);
 #pragma unroll
-        for (int e = 0; e < V; ++e) dvp[q][e] = fmaf(dj, h[j][q][e], dvp[q][e]);
+        for (int e = 0; e < V; ++e) dvp[q][e] = fmaf(dj, prelu(x[e], a), dvp[q][e]);
+      }
     }
 #pragma unroll
     for (int q = 0; q < PER; ++q)
@@ -310,7 +318,7 @@ __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ 
 // registers; warp w streams RU consecutive rows per iteration.  One dalpha
 // slot per block, folded in fixed order.
 template <int NC, typename T>
-__global__ void __launch_bounds__(kWarps * 32)
+__global__ void __launch_bounds__(kWarps * 32, 3)
 k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
       const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
       const float* __restrict__ dl, const float* __restrict__ vf, const float* __restrict__ dmf,
@@ -336,32 +344,29 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
     }
   double da = 0.0;
   for (int32_t r = r0 + w * RU; r < r1; r += kWarps * RU) {
-    float z[RU][PER][V], d[RU];
+    typename Vec<T>::Raw zr[RU][PER];
+    float d[RU];
 #pragma unroll
     for (int u = 0; u < RU; ++u) {
       const bool ok = r + u < r1;
       d[u] = ok ? dl[base + r + u] : 0.f;
 #pragma unroll
-      for (int q = 0; q < PER; ++q) {
-        if (act && ok) {
-          Vec<T>::load(Z3 + (base + r + u) * H + (lane + q * LPR) * V, z[u][q]);
-        } else {
-#pragma unroll
-          for (int e = 0; e < V; ++e) z[u][q][e] = 0.f;
-        }
-      }
+      for (int q = 0; q < PER; ++q)
+        zr[u][q] = (act && ok) ? Vec<T>::ld(Z3 + (base + r + u) * H + (lane + q * LPR) * V)
+                               : typename Vec<T>::Raw{};
     }
     float daf = 0.f;
 #pragma unroll
     for (int u = 0; u < RU; ++u)
 #pragma unroll
       for (int q = 0; q < PER; ++q) {
-        float o[V];
+        float o[V], z[V];
+        Vec<T>::cvt(zr[u][q], z);
 #pragma unroll
         for (int e = 0; e < V; ++e) {
           const float dh = fmaf(d[u], vg[q][e], mg[q][e]);
-          o[e] = z[u][q][e] > 0.f ? dh : a * dh;
-          daf += z[u][q][e] > 0.f ? 0.f : dh * z[u][q][e];
+          o[e] = z[e] > 0.f ? dh : a * dh;
+          daf += z[e] > 0.f ? 0.f : dh * z[e];
         }
         if (act && r + u < r1) StoreN<T, V>::store(dZ + (base + r + u) * H + (lane + q * LPR) * V, o);
       }
@@ -377,13 +382,23 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
   }
 }
 
-__global__ void k_reduce_slots(const double* __restrict__ slots, int n, float* __restrict__ out) {
-  __shared__ double sh[256];
-  double t = 0.0;
-  for (int k = threadIdx.x; k < n; k += 256) t += slots[k];
-  sh[threadIdx.x] = t;
+// Sum of n fp64 partials -> fp32, one block of 1024 threads: thread t keeps
+// four accumulators (k = t + 4096 i + 1024 q), then a fixed-shape tree.
+__global__ void __launch_bounds__(1024) k_reduce_slots(const double* __restrict__ slots, int n,
+                                                       float* __restrict__ out) {
+  __shared__ double sh[1024];
+  double t0 = 0.0, t1 = 0.0, t2 = 0.0, t3 = 0.0;
+  int k = threadIdx.x;
+  for (; k + 3072 < n; k += 4096) {
+    t0 += slots[k];
+    t1 += slots[k + 1024];
+    t2 += slots[k + 2048];
+    t3 += slots[k + 3072];
+  }
+  for (; k < n; k += 1024) t0 += slots[k];
+  sh[threadIdx.x] = (t0 + t1) + (t2 + t3);
   __syncthreads();
-  for (int o = 128; o > 0; o >>= 1) {
+  for (int o = 512; o > 0; o >>= 1) {
     if (threadIdx.x < o) sh[threadIdx.x] += sh[threadIdx.x + o];
     __syncthreads();
   }
@@ -457,7 +472,7 @@ cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, con
 cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
                                 int* launches) {
   count_launch(launches);
-  k_reduce_slots<<<1, 256, 0, s>>>(slots, n, grad);
+  k_reduce_slots<<<1, 1024, 0, s>>>(slots, n, grad);
   return cudaGetLastError();
 }
 

@@ -16,7 +16,14 @@ template <>
 struct Vec<float> {
   static constexpr int N = 4;  // elements per 16 bytes
   __device__ __forceinline__ static void load(const float* p, float (&x)[4]) {
-    const float4 v = __ldg(reinterpret_cast<const float4*>(p));
+    cvt(ld(p), x);
+  }
+  // raw 16-byte form: a load kept in flight costs 4 registers whatever T is
+  typedef float4 Raw;
+  __device__ __forceinline__ static Raw ld(const float* p) {
+    return __ldg(reinterpret_cast<const float4*>(p));
+  }
+  __device__ __forceinline__ static void cvt(const Raw& v, float (&x)[4]) {
     x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
   }
 };
@@ -25,7 +32,13 @@ template <>
 struct Vec<bf16> {
   static constexpr int N = 8;
   __device__ __forceinline__ static void load(const bf16* p, float (&x)[8]) {
-    const uint4 v = __ldg(reinterpret_cast<const uint4*>(p));
+    cvt(ld(p), x);
+  }
+  typedef uint4 Raw;
+  __device__ __forceinline__ static Raw ld(const bf16* p) {
+    return __ldg(reinterpret_cast<const uint4*>(p));
+  }
+  __device__ __forceinline__ static void cvt(const Raw& v, float (&x)[8]) {
     const uint32_t w[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
