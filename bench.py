@@ -99,6 +99,22 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(rows)}
 
 
+def ncu_traffic(prec: str, group: str):
+    """DRAM bytes per step of a kernel group from the committed one-step
+    `ncu --set full` capture (profiles/<tag>_traffic.json, written by
+    tools/traffic_from_ncu.py); None when absent."""
+    import glob
+    files = sorted(glob.glob(os.path.join(ROOT, "profiles", "*_traffic.json")))
+    if not files:
+        return None
+    try:
+        with open(files[-1]) as f:
+            g = json.load(f)[prec][group]
+        return float(g["dram_bytes_per_step"]), os.path.relpath(files[-1], ROOT)
+    except Exception:
+        return None
+
+
 # ------------------------------------------------------------------ algorithmic bytes / flops
 def spmm_bytes(N, Z, C, layer1=False, bwd=False, s=4, s_in=None):
     """Per SpMM launch over the stacked [pos; neg] rows:
@@ -281,6 +297,13 @@ def run_mine(args):
                  "frac": head_gbs / pk["hbm_gbs"] if head_gbs else None, "traffic": None,
                  "peak_source": pk["source"], "share_of_step": head_ms / step_total},
     }
+    algo_bytes = {"gemm": sum(gbytes.values()), "spmm": spmm_algo, "head": head_bytes}
+    for grp, r in rooflines.items():
+        t = ncu_traffic("fp32", grp)
+        if t is not None:
+            r["traffic"] = t[0]
+            r["traffic_note"] = (f"DRAM read+write bytes per step of the group, ncu --set full ({t[1]}); "
+                                 f"algorithmic bytes per step {algo_bytes[grp]:.4g}")
     roof = max(rooflines.values(), key=lambda r: r["share_of_step"])
     spmm_obj = {"achieved_gbs": spmm_gbs, "peak_gbs": pk["hbm_gbs"],
                 "frac": (spmm_gbs / pk["hbm_gbs"]) if spmm_gbs else None,
@@ -354,6 +377,9 @@ def run_mine(args):
                    "ms_per_step": ms16 / args.steps, "dtype": "bf16",
                    "phases_ms_per_step": ps16,
                    "spmm_gbs": sp16_bytes / (sp16 / 1e3) / 1e9 if sp16 else None,
+                   "spmm_frac": (sp16_bytes / (sp16 / 1e3) / 1e9 / pk["hbm_gbs"]) if sp16 else None,
+                   "spmm_traffic": (ncu_traffic("bf16", "spmm") or (None,))[0],
+                   "spmm_algorithmic_bytes_per_step": sp16_bytes,
                    "note": "bf16 activations + bf16 tcgen05 MMAs, fp32 accumulation and "
                            "master params; parity bar 2e-2 (tests/test_gpu_bf16.py)"}
             m16.free()

@@ -7,24 +7,21 @@
 // kind::tf32 with fp32 accumulation in TMEM.  The dropped lo·lo term and the
 // tf32 rounding of lo are ~2^-22 relative.
 //
-// Operands arrive by TMA with 128-byte swizzle.  For a 4-byte type the
-// swizzle atom "8 rows x 128 B" is the same bytes whether the 32 contiguous
-// elements are read as the K dimension (K-major) or the M/N dimension
-// (MN-major), so row-major activations feed both the forward (K-major A) and
-// the weight-gradient (MN-major A and B, reduction over rows) without
-// transposes -- only the UMMA descriptors differ.  The lo parts are written by
-// converter warps in place of / beside the TMA tile (position-preserving, so
-// the swizzle needs no remapping), then fence.proxy.async hands them to MMA.
+// Row-major activations feed both the forward (K-major A) and the weight
+// gradient (MN-major A and B, reduction over rows) without transposes: only
+// the TMA swizzle mode and the UMMA descriptors differ.  The lo parts are
+// written by converter warps beside the TMA tile (position-preserving, so the
+// swizzle needs no remapping), then fence.proxy.async hands them to the MMA.
 //
-// k_tc_rows  : C[M×N] = A[M×K]·Bᵀ, B [N×K] = weights pre-split (hi/lo arrays).
-//              Persistent over 128-row tiles; warp 0 TMA, warp 1 MMA issuer,
-//              warps 2-3 split A, warps 4-7 epilogue (TMEM -> registers ->
-//              global); double-buffered TMEM accumulators so the epilogue of
-//              tile i overlaps the main loop of tile i+1.
-// k_tc_dw    : per CTA one chunk of the R = 2ΣN rows, D = dZ_chunkᵀ·Y_chunk
-//              [256 × Cin] in two TMEM accumulators (M = 128 halves of H),
-//              written as an fp32 partial; k_dw_reduce sums the partials in a
-//              fixed order in fp64 and transposes into dW [Cin × H].
+// k_tc_rows  : C[M×N] = A[M×K]·Bᵀ, B [N×K] = weights pre-split (hi/lo arrays,
+//              k_split_w).  K-blocks of 16 fp32 (64-byte rows, 64B swizzle)
+//              so 4 (N = 256) / 6 stages fit; persistent over 128-row tiles;
+//              warp 0 TMA, warp 1 MMA issuer, warps 2-3 split A, warps 4-7
+//              epilogue (tcgen05.ld -> 128B-swizzled smem slabs -> TMA store);
+//              double-buffered TMEM accumulators so the epilogue of tile i
+//              overlaps the main loop of tile i+1.
+// k_tc_dw2   : dW partials per row chunk (below), MN-major operands with the
+//              128B swizzle in 32-byte atoms (layout type SW128_BASE32B).
 #include <cudaTypedefs.h>
 
 #include <cstdlib>
@@ -228,221 +225,24 @@ k_tc_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUten
   }
 }
 
-// ---------------------------------------------------------------- k_tc_dw
-// Per CTA: one chunk of rows x one CINT-wide tile of C_in.  D = dZᵀ·Y for the
-// tile is accumulated by the tensor cores in a TMEM "work" accumulator for
-// kSubRows rows at a time; epilogue warps then fold it into a TMEM "master"
-// accumulator with IEEE fp32 adds (tcgen05.ld / add / tcgen05.st), so the
-// tensor core's own fp32 accumulation never runs over more than kSubRows
-// rows (its truncating accumulation error grows with the run length), and the
-// chunk result is written as an fp32 partial for the fixed-order fp64 reduce.
+// ---------------------------------------------------------------- k_tc_dw2 tiling
 constexpr int kDwBK = 16;        // rows of R per stage
 constexpr int kDwStages = 4;
 constexpr int kSubKb = 8;        // k-blocks per work accumulation (128 rows)
 
-template <int CINT>
-struct DwCfg {
-  static constexpr int A_BYTES = 256 * kDwBK * 4;     // dZ: 8 boxes of 32 cols x 16 rows (16 KB)
-  static constexpr int B_BYTES = CINT * kDwBK * 4;    // Y : CINT/32 boxes
-  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int SMEM = kDwStages * STAGE + 1024 + 256;
-  static constexpr uint32_t TMEM_COLS = 4 * CINT;     // work [2 halves] + master [2 halves]
-  static constexpr int BOX = 32 * kDwBK * 4;          // bytes of one 32-col box (2 KB)
-};
-
-template <int CINT>
-__global__ void __launch_bounds__(384, 1)
-k_tc_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
-        float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN) {
-  using Cfg = DwCfg<CINT>;
-  constexpr int S = kDwStages;
-  constexpr int NCONV = 6;                                   // warps 2, 3, 8..11
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
-  uint64_t* full = bars;
-  uint64_t* conv = bars + S;
-  uint64_t* empty = bars + 2 * S;
-  uint64_t* tfull = bars + 3 * S;
-  uint64_t* tempty = bars + 3 * S + 1;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 2);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int ntile = CIN / CINT;
-  const int chunk = blockIdx.x / ntile, c_off = (blockIdx.x % ntile) * CINT;
-  const int32_t r0 = chunk * rows_per_chunk;
-  const int32_t r1 = min(R, r0 + rows_per_chunk);
-  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
-  const int nsub = (nk + kSubKb - 1) / kSubKb;
-  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
-  auto stAlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
-  auto stB = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
-  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
-
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&conv[s], NCONV);
-      mbar_init(&empty[s], 1);
-    }
-    mbar_init(tfull, 1);
-    mbar_init(tempty, 4);
-    fence_mbar_init();
-    tma_prefetch(&tmDZ);
-    tma_prefetch(&tmY);
-  }
-  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tbase = *tslot;
-  const uint32_t twork = tbase, tmaster = tbase + 2 * CINT;
-
-  if (warp == 0) {
-    if (lane == 0) {                                         // ---- TMA producer
-      int s = 0;
-      uint32_t ph = 0;
-      for (int kb = 0; kb < nk; ++kb) {
-        mbar_wait(&empty[s], ph ^ 1);
-        mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
-        const int32_t row = r0 + kb * kDwBK;
-#pragma unroll
-        for (int bx = 0; bx < 8; ++bx)
-          tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 32, row, &full[s]);
-#pragma unroll
-        for (int bx = 0; bx < CINT / 32; ++bx)
-          tma_load_2d(stB(s) + bx * Cfg::BOX, &tmY, c_off + bx * 32, row, &full[s]);
-        if (++s == S) { s = 0; ph ^= 1; }
-      }
-    }
-  } else if (warp == 1) {
-    if (lane == 0) {                                         // ---- MMA issuer
-      constexpr uint32_t idesc = idesc_tf32(kBM, CINT, true, true);
-      int s = 0;
-      uint32_t ph = 0;
-      for (int sub = 0; sub < nsub; ++sub) {
-        mbar_wait(tempty, (sub & 1) ^ 1);                    // epilogue drained the work acc
-        tc_fence_after();
-        const int kb1 = min(nk, (sub + 1) * kSubKb);
-        for (int kb = sub * kSubKb; kb < kb1; ++kb) {
-          mbar_wait(&conv[s], ph);
-          tc_fence_after();
-          const uint32_t a = smem_u32(stA(s)), al = smem_u32(stAlo(s));
-          const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
-#pragma unroll
-          for (int k = 0; k < kDwBK / 8; ++k) {
-            // MN-major tf32: atoms of 4 K-rows x 128 B (512 B, SBO); 32-element
-            // MN blocks one box apart (LBO); one MMA (K = 8) spans two atoms.
-            const uint64_t bh = sdesc_sw128_b32(b + 1024 * k, Cfg::BOX, 512);
-            const uint64_t blo = sdesc_sw128_b32(bl + 1024 * k, Cfg::BOX, 512);
-            const uint32_t first = (kb == sub * kSubKb && k == 0) ? 0u : 1u;
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {                    // two 128-row halves of H
-              const uint64_t ah = sdesc_sw128_b32(a + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
-              const uint64_t alo = sdesc_sw128_b32(al + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
-              const uint32_t d = twork + h * CINT;
-              mma_tf32(d, ah, bh, idesc, first);
-              mma_tf32(d, ah, blo, idesc, 1);
-              mma_tf32(d, alo, bh, idesc, 1);
-            }
-          }
-          mma_commit(&empty[s]);
-          if (++s == S) { s = 0; ph ^= 1; }
-        }
-        mma_commit(tfull);
-      }
-    }
-  } else if (warp >= 4 && warp < 8) {                       // ---- fold work -> master, write
-    const int q = warp & 3;
-    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
-    for (int sub = 0; sub < nsub; ++sub) {
-      mbar_wait(tfull, sub & 1);
-      tc_fence_after();
-#pragma unroll 1
-      for (int h = 0; h < 2; ++h)
-#pragma unroll 1
-        for (int c0 = 0; c0 < CINT; c0 += 32) {
-          uint32_t w[32];
-          tmem_ld32(twork + lane_off + h * CINT + c0, w);
-          if (sub > 0) {
-            uint32_t m[32];
-            tmem_ld32(tmaster + lane_off + h * CINT + c0, m);
-            tmem_wait_ld();
-#pragma unroll
-            for (int j = 0; j < 32; ++j)
-              w[j] = __float_as_uint(__uint_as_float(w[j]) + __uint_as_float(m[j]));
-          } else {
-            tmem_wait_ld();
-          }
-          tmem_st32(tmaster + lane_off + h * CINT + c0, w);
-        }
-      tmem_wait_st();
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(tempty);
-    }
-    float* out = part + (int64_t)chunk * 256 * CIN + c_off;
-#pragma unroll 1
-    for (int h = 0; h < 2; ++h) {
-      const int hrow = h * 128 + q * 32 + lane;
-#pragma unroll 1
-      for (int c0 = 0; c0 < CINT; c0 += 32) {
-        uint32_t r[32];
-        if (nsub > 0) {
-          tmem_ld32(tmaster + lane_off + h * CINT + c0, r);
-          tmem_wait_ld();
-        } else {
-#pragma unroll
-          for (int j = 0; j < 32; ++j) r[j] = 0u;
-        }
-        float4* dst = reinterpret_cast<float4*>(out + (int64_t)hrow * CIN + c0);
-#pragma unroll
-        for (int j = 0; j < 8; ++j)
-          dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
-                               __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
-      }
-    }
-  } else {                                                   // ---- split (warps 2, 3, 8..11)
-    const int ct = (warp < 4 ? warp - 2 : warp - 6) * 32 + lane;
-    constexpr int NT = NCONV * 32;
-    int s = 0;
-    uint32_t ph = 0;
-    for (int kb = 0; kb < nk; ++kb) {
-      mbar_wait(&full[s], ph);
-      float4* a = reinterpret_cast<float4*>(stA(s));
-      float4* al = reinterpret_cast<float4*>(stAlo(s));
-      float4* bb = reinterpret_cast<float4*>(stB(s));
-      float4* bl = reinterpret_cast<float4*>(stBlo(s));
-      for (int i = ct; i < (Cfg::A_BYTES + Cfg::B_BYTES) / 16; i += NT) {
-        const bool isA = i < Cfg::A_BYTES / 16;
-        float4* src = isA ? a + i : bb + (i - Cfg::A_BYTES / 16);
-        float4* dlo = isA ? al + i : bl + (i - Cfg::A_BYTES / 16);
-        const float4 v = *src;
-        const float4 hv = make_float4(to_tf32(v.x), to_tf32(v.y), to_tf32(v.z), to_tf32(v.w));
-        *src = hv;
-        *dlo = make_float4(v.x - hv.x, v.y - hv.y, v.z - hv.z, v.w - hv.w);
-      }
-      fence_proxy_async_smem();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&conv[s]);
-      if (++s == S) { s = 0; ph ^= 1; }
-    }
-  }
-  tc_fence_before();
-  __syncthreads();
-  if (warp == 1) {
-    tc_fence_after();
-    tmem_dealloc(tbase, Cfg::TMEM_COLS);
-  }
-}
-
 // ---------------------------------------------------------------- k_tc_dw2
-// Same tiling as k_tc_dw, but the fp32 master accumulator lives in the
-// registers of eight epilogue warps (quadrant q = warp & 3 owns TMEM lanes
-// 32q.., column half ch = (warp-4)/4 owns half of the tile's columns), so the
-// two TMEM work accumulators can be double-buffered: the tensor cores fill
-// one 128-row run while the epilogue folds the previous one (IEEE adds).
-// 12 warps: 0 TMA, 1 MMA, 2-3 split, 4-11 fold / write.
+// Per CTA: one chunk of rows x one CINT-wide tile of C_in.  D = dZᵀ·Y for the
+// tile is accumulated by the tensor cores in a TMEM "work" accumulator for
+// 128 rows (kSubKb k-blocks) at a time; epilogue warps then fold each run into
+// an fp32 master held in their registers with IEEE adds, so the tensor core's
+// own fp32 accumulation never runs over more than 128 rows (its truncating
+// accumulation error grows with the run length; folding keeps dW at ~1e-6 of
+// scale on the bench graphs).  Quadrant q = warp & 3 owns TMEM lanes 32q..,
+// column half ch = (warp-4)/4 owns half of the tile's columns; the two TMEM
+// work accumulators are double-buffered so the tensor cores fill one run
+// while the epilogue folds the previous one.  The chunk result is written as
+// an fp32 partial for the fixed-order fp64 reduce (k_dw_reduce).
+// 12 warps: 0 TMA, 1 MMA issuer, 2-11 split the tf32 lo parts and fold.
 template <int CINT>
 struct Dw2Cfg {
   static constexpr int A_BYTES = 256 * kDwBK * 4;
@@ -635,171 +435,6 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
   }
 }
 
-#if 0  // superseded single-accumulator version (kept out of the build)
-constexpr int kDwBK_old = 16;        // rows of R per stage
-constexpr int kDwStages = 3;
-
-template <int CIN>
-struct DwCfg {
-  static constexpr int A_BYTES = 256 * kDwBK * 4;     // dZ: 8 boxes of 32 cols x 16 rows (16 KB)
-  static constexpr int B_BYTES = CIN * kDwBK * 4;     // Y : CIN/32 boxes
-  static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int SMEM = kDwStages * STAGE + 1024 + 256;
-  static constexpr uint32_t TMEM_COLS = (2 * CIN) <= 32 ? 32 : (2 * CIN) <= 64 ? 64
-                                        : (2 * CIN) <= 128 ? 128 : (2 * CIN) <= 256 ? 256 : 512;
-  static constexpr int BOX = 32 * kDwBK * 4;          // bytes of one 32-col box (2 KB)
-};
-
-template <int CIN>
-__global__ void __launch_bounds__(kThreads, 1)
-k_tc_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
-        float* __restrict__ part, int32_t R, int32_t rows_per_chunk) {
-  using Cfg = DwCfg<CIN>;
-  constexpr int S = kDwStages;
-  constexpr int NCONV = 6;                                   // warps 2..7 split both operands
-  extern __shared__ uint8_t smem_raw[];
-  // 1024-byte alignment for the 128-byte swizzle atoms, by pointer arithmetic on
-  // the shared array itself so every access stays in the shared window (LDS/STS).
-  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
-  uint64_t* full = bars;
-  uint64_t* conv = bars + S;
-  uint64_t* empty = bars + 2 * S;
-  uint64_t* tfull = bars + 3 * S;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 1);
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int32_t r0 = blockIdx.x * rows_per_chunk;
-  const int32_t r1 = min(R, r0 + rows_per_chunk);
-  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
-  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
-  auto stAlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
-  auto stB = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES; };
-  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + 2 * Cfg::A_BYTES + Cfg::B_BYTES; };
-
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&conv[s], NCONV);
-      mbar_init(&empty[s], 1);
-    }
-    mbar_init(tfull, 1);
-    fence_mbar_init();
-    tma_prefetch(&tmDZ);
-    tma_prefetch(&tmY);
-  }
-  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tbase = *tslot;
-
-  if (warp == 0) {
-    if (lane == 0) {                                         // ---- TMA producer
-      int s = 0;
-      uint32_t ph = 0;
-      for (int kb = 0; kb < nk; ++kb) {
-        mbar_wait(&empty[s], ph ^ 1);
-        mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
-        const int32_t row = r0 + kb * kDwBK;
-#pragma unroll
-        for (int bx = 0; bx < 8; ++bx) tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 32, row, &full[s]);
-#pragma unroll
-        for (int bx = 0; bx < CIN / 32; ++bx) tma_load_2d(stB(s) + bx * Cfg::BOX, &tmY, bx * 32, row, &full[s]);
-        if (++s == S) { s = 0; ph ^= 1; }
-      }
-    }
-  } else if (warp == 1) {
-    if (lane == 0) {                                         // ---- MMA issuer
-      constexpr uint32_t idesc = idesc_tf32(kBM, CIN, true, true);
-      int s = 0;
-      uint32_t ph = 0;
-      for (int kb = 0; kb < nk; ++kb) {
-        mbar_wait(&conv[s], ph);
-        tc_fence_after();
-        const uint32_t a = smem_u32(stA(s)), al = smem_u32(stAlo(s));
-        const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
-#pragma unroll
-        for (int k = 0; k < kDwBK / 8; ++k) {
-          // MN-major tf32: atoms of 4 K-rows x 128 B (512 B, SBO) ; 32-element
-          // MN blocks one box apart (LBO); one MMA (K = 8) spans two atoms.
-          const uint64_t bh = sdesc_sw128_b32(b + 1024 * k, Cfg::BOX, 512);
-          const uint64_t blo = sdesc_sw128_b32(bl + 1024 * k, Cfg::BOX, 512);
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {                      // two 128-row halves of H
-            const uint64_t ah = sdesc_sw128_b32(a + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
-            const uint64_t alo = sdesc_sw128_b32(al + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
-            const uint32_t d = tbase + h * CIN;
-            mma_tf32(d, ah, bh, idesc, (kb | k) != 0);
-            mma_tf32(d, ah, blo, idesc, 1);
-            mma_tf32(d, alo, bh, idesc, 1);
-          }
-        }
-        mma_commit(&empty[s]);
-        if (++s == S) { s = 0; ph ^= 1; }
-      }
-      mma_commit(tfull);
-    }
-  } else {                                                   // ---- split (warps 2..7)
-    const int ct = threadIdx.x - 64;
-    constexpr int NT = NCONV * 32;
-    int s = 0;
-    uint32_t ph = 0;
-    for (int kb = 0; kb < nk; ++kb) {
-      mbar_wait(&full[s], ph);
-      float4* a = reinterpret_cast<float4*>(stA(s));
-      float4* al = reinterpret_cast<float4*>(stAlo(s));
-      for (int i = ct; i < (Cfg::A_BYTES + Cfg::B_BYTES) / 16; i += NT) {
-        float4* src = i < Cfg::A_BYTES / 16 ? a + i : reinterpret_cast<float4*>(stB(s)) + (i - Cfg::A_BYTES / 16);
-        float4* dlo = i < Cfg::A_BYTES / 16 ? al + i : reinterpret_cast<float4*>(stBlo(s)) + (i - Cfg::A_BYTES / 16);
-        float4 v = *src;
-        float4 hv = make_float4(to_tf32(v.x), to_tf32(v.y), to_tf32(v.z), to_tf32(v.w));
-        *src = hv;
-        *dlo = make_float4(v.x - hv.x, v.y - hv.y, v.z - hv.z, v.w - hv.w);
-      }
-      fence_proxy_async_smem();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&conv[s]);
-      if (++s == S) { s = 0; ph ^= 1; }
-    }
-    if (warp >= 4) {                                         // ---- epilogue (warps 4..7)
-      const int q = warp & 3;
-      float* out = part + (int64_t)blockIdx.x * 256 * CIN;
-      if (nk > 0) {
-        mbar_wait(tfull, 0);
-        tc_fence_after();
-      }
-#pragma unroll 1
-      for (int h = 0; h < 2; ++h) {
-        const int hrow = h * 128 + q * 32 + lane;
-#pragma unroll 1
-        for (int c0 = 0; c0 < CIN; c0 += 32) {
-          uint32_t r[32];
-          if (nk > 0) {
-            tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + h * CIN + c0, r);
-            tmem_wait_ld();
-          } else {
-#pragma unroll
-            for (int j = 0; j < 32; ++j) r[j] = 0u;
-          }
-          float4* dst = reinterpret_cast<float4*>(out + (int64_t)hrow * CIN + c0);
-#pragma unroll
-          for (int j = 0; j < 8; ++j)
-            dst[j] = make_float4(__uint_as_float(r[4 * j]), __uint_as_float(r[4 * j + 1]),
-                                 __uint_as_float(r[4 * j + 2]), __uint_as_float(r[4 * j + 3]));
-        }
-      }
-    }
-  }
-  tc_fence_before();
-  __syncthreads();
-  if (warp == 1) {
-    tc_fence_after();
-    tmem_dealloc(tbase, Cfg::TMEM_COLS);
-  }
-}
-
-#endif
 
 // dW[c][h] = Σ_chunk part[chunk][h][c], fixed order, fp64.
 __global__ void k_dw_reduce(const float* __restrict__ part, int nchunk, int CIN,
