@@ -112,7 +112,7 @@ typedef struct {
   const float* init_params;   /* optional [P] host; NULL => Xavier-uniform(seed) */
   int32_t device;             /* CUDA device ordinal                           */
   int32_t world_size, rank;   /* data parallelism; 1, 0 for a single GPU       */
-  const void* nccl_unique_id; /* 128-byte ncclUniqueId when world_size > 1     */
+  const void* nccl_unique_id; /* 128-byte ncclUniqueId; required when world_size > 1, optional with 1 (1-rank communicator) */
 } mars_dgi_config;
 
 /* Fills cfg with the defaults above (F = 64, H = 256, L = 3, FP32, seed 0,

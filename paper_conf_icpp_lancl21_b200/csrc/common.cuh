@@ -43,12 +43,12 @@ inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b);
 // Split-K combination of the weight-gradient partials, deterministic:
 // dW[c][h] = Σ_k part[k][h·CIN + c] in fp64.  Block = 32 consecutive outputs ×
 // 8 k-groups (group j sums k = j, j+8, ...), the 8 group sums combined in order
-// j = 0..7; grid = ceil(256·CIN / 32) blocks of 256 threads.
+// j = 0..7; grid = ceil(H·CIN / 32) blocks of 256 threads.
 __device__ __forceinline__ void dw_reduce_body(const float* __restrict__ part, int nchunk, int CIN,
-                                               float* __restrict__ dW) {
+                                               int H, float* __restrict__ dW) {
   __shared__ double sh[8][32];
   const int lane = threadIdx.x & 31, j = threadIdx.x >> 5;
-  const int64_t n = 256LL * CIN;
+  const int64_t n = (int64_t)H * CIN;
   const int64_t e = (int64_t)blockIdx.x * 32 + lane;     // e = h * CIN + c
   double t = 0.0;
   if (e < n)
@@ -60,7 +60,7 @@ __device__ __forceinline__ void dw_reduce_body(const float* __restrict__ part, i
 #pragma unroll
     for (int q = 0; q < 8; ++q) s += sh[q][lane];
     const int h = (int)(e / CIN), c = (int)(e % CIN);
-    dW[(int64_t)c * 256 + h] = (float)s;
+    dW[(int64_t)c * H + h] = (float)s;
   }
 }
 

@@ -243,22 +243,24 @@ constexpr int kSubKb = 8;        // k-blocks per work accumulation (128 rows)
 // while the epilogue folds the previous one.  The chunk result is written as
 // an fp32 partial for the fixed-order fp64 reduce (k_dw_reduce).
 // 12 warps: 0 TMA, 1 MMA issuer, 2-11 split the tf32 lo parts and fold.
-template <int CINT>
+template <int CINT, int HH>
 struct Dw2Cfg {
-  static constexpr int A_BYTES = 256 * kDwBK * 4;
+  static constexpr int NH = HH / 128;                 // 128-row halves of H (UMMA M)
+  static constexpr int A_BYTES = HH * kDwBK * 4;
   static constexpr int B_BYTES = CINT * kDwBK * 4;
   static constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
   static constexpr int SMEM = kDwStages * STAGE + 1024 + 256;
-  static constexpr uint32_t TMEM_COLS = 4 * CINT;     // 2 work buffers x 2 halves of H
+  static constexpr uint32_t TMEM_COLS = 2 * NH * CINT;  // 2 work buffers x NH halves of H
   static constexpr int BOX = 32 * kDwBK * 4;
   static constexpr int MCOLS = CINT / 2;              // columns per epilogue thread per half
 };
 
-template <int CINT>
+template <int CINT, int HH>
 __global__ void __launch_bounds__(384, 1)
 k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
          float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN) {
-  using Cfg = Dw2Cfg<CINT>;
+  using Cfg = Dw2Cfg<CINT, HH>;
+  constexpr int NH = Cfg::NH;
   constexpr int S = kDwStages;
   constexpr int MC = Cfg::MCOLS;
   extern __shared__ uint8_t smem_raw[];
@@ -312,7 +314,7 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
         mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
         const int32_t row = r0 + kb * kDwBK;
 #pragma unroll
-        for (int bx = 0; bx < 8; ++bx)
+        for (int bx = 0; bx < HH / 32; ++bx)
           tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 32, row, &full[s]);
 #pragma unroll
         for (int bx = 0; bx < CINT / 32; ++bx)
@@ -329,7 +331,7 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
         const int buf = sub & 1;
         mbar_wait(&tempty[buf], ((sub >> 1) & 1) ^ 1);      // previous use of this buffer folded
         tc_fence_after();
-        const uint32_t twork = tbase + buf * 2 * CINT;
+        const uint32_t twork = tbase + buf * NH * CINT;
         const int kb1 = min(nk, (sub + 1) * kSubKb);
         for (int kb = sub * kSubKb; kb < kb1; ++kb) {
           mbar_wait(&conv[s], ph);
@@ -342,7 +344,7 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
             const uint64_t blo = sdesc_sw128_b32(bl + 1024 * k, Cfg::BOX, 512);
             const uint32_t first = (kb == sub * kSubKb && k == 0) ? 0u : 1u;
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
+            for (int h = 0; h < NH; ++h) {
               const uint64_t ah = sdesc_sw128_b32(a + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
               const uint64_t alo = sdesc_sw128_b32(al + h * 4 * Cfg::BOX + 1024 * k, Cfg::BOX, 512);
               const uint32_t d = twork + h * CINT;
@@ -363,9 +365,9 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
     constexpr int NT = 10 * 32;
     const int q = warp & 3, ch = (warp - 4) >> 2;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
-    float master[2][MC];
+    float master[NH][MC];
 #pragma unroll
-    for (int h = 0; h < 2; ++h)
+    for (int h = 0; h < NH; ++h)
 #pragma unroll
       for (int j = 0; j < MC; ++j) master[h][j] = 0.f;
     int folded = 0;
@@ -374,9 +376,9 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
       const int buf = sub & 1;
       mbar_wait(&tfull[buf], (sub >> 1) & 1);
       tc_fence_after();
-      const uint32_t twork = tbase + buf * 2 * CINT + ch * MC;
+      const uint32_t twork = tbase + buf * NH * CINT + ch * MC;
 #pragma unroll
-      for (int h = 0; h < 2; ++h)
+      for (int h = 0; h < NH; ++h)
 #pragma unroll
         for (int c0 = 0; c0 < MC; c0 += 32) {
           uint32_t w[32];
@@ -416,9 +418,9 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
     }
     if (folder) {
       while (folded < nsub) fold(folded++);
-      float* out = part + (int64_t)chunk * 256 * CIN + c_off + ch * MC;   // chunk partial
+      float* out = part + (int64_t)chunk * HH * CIN + c_off + ch * MC;   // chunk partial
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
+      for (int h = 0; h < NH; ++h) {
         float4* dst = reinterpret_cast<float4*>(out + (int64_t)(h * 128 + q * 32 + lane) * CIN);
 #pragma unroll
         for (int j = 0; j < MC / 4; ++j)
@@ -437,9 +439,9 @@ k_tc_dw2(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUten
 
 
 // dW[c][h] = Σ_chunk part[chunk][h][c], fixed order, fp64.
-__global__ void k_dw_reduce(const float* __restrict__ part, int nchunk, int CIN,
+__global__ void k_dw_reduce(const float* __restrict__ part, int nchunk, int CIN, int H,
                             float* __restrict__ dW) {
-  dw_reduce_body(part, nchunk, CIN, dW);
+  dw_reduce_body(part, nchunk, CIN, H, dW);
 }
 
 // hi / lo split of the weights for the B operand: Bt = Wᵀ [H × Cin] (forward)
@@ -536,21 +538,21 @@ cudaError_t rows_n(const float* A, const float* Bhi, const float* Blo, float* C,
   return cudaGetLastError();
 }
 
-template <int CINT>
+template <int CINT, int HH>
 cudaError_t dw_c(const float* Y, const float* dZ, float* part, int nchunk, int64_t R, int rows,
                  int CIN, cudaStream_t s) {
-  using Cfg = Dw2Cfg<CINT>;
+  using Cfg = Dw2Cfg<CINT, HH>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_tc_dw2<CINT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(k_tc_dw2<CINT, HH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          Cfg::SMEM);
     if (e != cudaSuccess) return e;
     attr = true;
   }
   CUtensorMap tdz, ty;
-  if (!tmap_2d(&tdz, dZ, R, 256, kDwBK, true) || !tmap_2d(&ty, Y, R, CIN, kDwBK, true))
+  if (!tmap_2d(&tdz, dZ, R, HH, kDwBK, true) || !tmap_2d(&ty, Y, R, CIN, kDwBK, true))
     return cudaErrorInvalidValue;
-  k_tc_dw2<CINT><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows, CIN);
+  k_tc_dw2<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows, CIN);
   return cudaGetLastError();
 }
 
@@ -574,7 +576,7 @@ bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void*
 int tc_num_sms() { return num_sms(); }
 
 bool tc_supported(int K_or_cin, int N_or_h) {
-  return N_or_h == 256 && (K_or_cin == 64 || K_or_cin == 128 || K_or_cin == 256);
+  return (N_or_h == 128 || N_or_h == 256) && (K_or_cin == 64 || K_or_cin == 128 || K_or_cin == 256);
 }
 
 cudaError_t tc_split_weights(const float* W, int CIN, int H, float* Bt_hi, float* Bt_lo,
@@ -609,8 +611,8 @@ size_t tc_dw_partial_floats(int64_t R, int CIN) {
   return (size_t)tc_dw_chunks(R, CIN) * 256 * CIN;
 }
 
-// dW [CIN × 256] = Yᵀ dZ with Y [R × CIN], dZ [R × 256].
-cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN,
+// dW [CIN × H] = Yᵀ dZ with Y [R × CIN], dZ [R × H], H in {128, 256}.
+cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN, int H,
                        float* part, cudaStream_t s, int* launches) {
   count_launch(launches, 2);
   int nchunk = tc_dw_chunks(R, CIN);
@@ -618,14 +620,17 @@ cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, in
   rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
   nchunk = (int)((R + rows - 1) / rows);
   cudaError_t e;
+  if (H != 128 && H != 256) return cudaErrorInvalidValue;
   switch (CIN) {
-    case 64: e = dw_c<64>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
-    case 128: e = dw_c<128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
-    case 256: e = dw_c<128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
+    case 64: e = H == 256 ? dw_c<64, 256>(Y, dZ, part, nchunk, R, rows, CIN, s)
+                          : dw_c<64, 128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
+    case 128:
+    case 256: e = H == 256 ? dw_c<128, 256>(Y, dZ, part, nchunk, R, rows, CIN, s)
+                           : dw_c<128, 128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
-  k_dw_reduce<<<cdiv(256LL * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, dW);
+  k_dw_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
   return cudaGetLastError();
 }
 

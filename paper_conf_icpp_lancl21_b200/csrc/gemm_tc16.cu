@@ -176,22 +176,24 @@ constexpr int kDwBK = 16;        // rows per stage (one K = 16 MMA)
 constexpr int kDwStages = 8;
 constexpr int kSubKb = 8;        // stages per TMEM work run (128 rows)
 
-template <int CINT>
+template <int CINT, int HH>
 struct D16Cfg {
+  static constexpr int NH = HH / 128;                 // 128-row halves of H (UMMA M)
   static constexpr int BOX = 64 * kDwBK * 2;          // 64 bf16 cols x 16 rows = 2 KB
-  static constexpr int A_BYTES = 4 * BOX;             // dZ: 256 cols
+  static constexpr int A_BYTES = (HH / 64) * BOX;     // dZ: HH cols
   static constexpr int B_BYTES = (CINT / 64) * BOX;   // Y : CINT cols
   static constexpr int STAGE = A_BYTES + B_BYTES;
   static constexpr int SMEM = kDwStages * STAGE + 1024 + 256;
-  static constexpr uint32_t TMEM_COLS = 4 * CINT;
+  static constexpr uint32_t TMEM_COLS = 2 * NH * CINT;
   static constexpr int MCOLS = CINT / 2;
 };
 
-template <int CINT>
+template <int CINT, int HH>
 __global__ void __launch_bounds__(384, 1)
 k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
           float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN) {
-  using Cfg = D16Cfg<CINT>;
+  using Cfg = D16Cfg<CINT, HH>;
+  constexpr int NH = Cfg::NH;
   constexpr int S = kDwStages;
   constexpr int MC = Cfg::MCOLS;
   extern __shared__ uint8_t smem_raw[];
@@ -241,7 +243,7 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
         mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
         const int32_t row = r0 + kb * kDwBK;
 #pragma unroll
-        for (int bx = 0; bx < 4; ++bx)
+        for (int bx = 0; bx < HH / 64; ++bx)
           tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 64, row, &full[s]);
 #pragma unroll
         for (int bx = 0; bx < CINT / 64; ++bx)
@@ -258,7 +260,7 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
         const int buf = sub & 1;
         mbar_wait(&tempty[buf], ((sub >> 1) & 1) ^ 1);
         tc_fence_after();
-        const uint32_t twork = tbase + buf * 2 * CINT;
+        const uint32_t twork = tbase + buf * NH * CINT;
         const int kb1 = min(nk, (sub + 1) * kSubKb);
         for (int kb = sub * kSubKb; kb < kb1; ++kb) {
           mbar_wait(&full[s], ph);
@@ -269,7 +271,7 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
           const uint64_t bd = sdesc_sw128(b, Cfg::BOX, 1024);
           const uint32_t first = kb == sub * kSubKb ? 0u : 1u;
 #pragma unroll
-          for (int h = 0; h < 2; ++h)
+          for (int h = 0; h < NH; ++h)
             mma_f16(twork + h * CINT, sdesc_sw128(a + h * 2 * Cfg::BOX, Cfg::BOX, 1024), bd, idesc,
                     first);
           mma_commit(&empty[s]);
@@ -281,18 +283,18 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
   } else if (warp >= 4) {                                    // ---- fold (warps 4..11)
     const int q = warp & 3, ch = (warp - 4) >> 2;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
-    float master[2][MC];
+    float master[NH][MC];
 #pragma unroll
-    for (int h = 0; h < 2; ++h)
+    for (int h = 0; h < NH; ++h)
 #pragma unroll
       for (int j = 0; j < MC; ++j) master[h][j] = 0.f;
     for (int sub = 0; sub < nsub; ++sub) {
       const int buf = sub & 1;
       mbar_wait(&tfull[buf], (sub >> 1) & 1);
       tc_fence_after();
-      const uint32_t twork = tbase + buf * 2 * CINT + ch * MC;
+      const uint32_t twork = tbase + buf * NH * CINT + ch * MC;
 #pragma unroll
-      for (int h = 0; h < 2; ++h)
+      for (int h = 0; h < NH; ++h)
 #pragma unroll
         for (int c0 = 0; c0 < MC; c0 += 32) {
           uint32_t w[32];
@@ -305,9 +307,9 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[buf]);
     }
-    float* out = part + (int64_t)chunk * 256 * CIN + c_off + ch * MC;
+    float* out = part + (int64_t)chunk * HH * CIN + c_off + ch * MC;
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
+    for (int h = 0; h < NH; ++h) {
       float4* dst = reinterpret_cast<float4*>(out + (int64_t)(h * 128 + q * 32 + lane) * CIN);
 #pragma unroll
       for (int j = 0; j < MC / 4; ++j)
@@ -324,9 +326,9 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 }
 
 // dW[c][h] = Σ_chunk part[chunk][h][c], fixed order, fp64.
-__global__ void k_dw16_reduce(const float* __restrict__ part, int nchunk, int CIN,
+__global__ void k_dw16_reduce(const float* __restrict__ part, int nchunk, int CIN, int H,
                               float* __restrict__ dW) {
-  dw_reduce_body(part, nchunk, CIN, dW);
+  dw_reduce_body(part, nchunk, CIN, H, dW);
 }
 
 __global__ void k_w16(const float* __restrict__ W, int CIN, int H, bf16* __restrict__ Bt,
@@ -374,21 +376,21 @@ int dw16_chunks(int64_t R, int CIN) {
   return (int)std::min(want, maxc);
 }
 
-template <int CINT>
+template <int CINT, int HH>
 cudaError_t dw16_c(const void* Y, const void* dZ, float* part, int nchunk, int64_t R, int rows,
                    int CIN, cudaStream_t s) {
-  using Cfg = D16Cfg<CINT>;
+  using Cfg = D16Cfg<CINT, HH>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_tc16_dw<CINT>,
+    cudaError_t e = cudaFuncSetAttribute(k_tc16_dw<CINT, HH>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
     if (e != cudaSuccess) return e;
     attr = true;
   }
   CUtensorMap tdz, ty;
-  if (!tmap16(&tdz, dZ, R, 256, 64, kDwBK) || !tmap16(&ty, Y, R, CIN, 64, kDwBK))
+  if (!tmap16(&tdz, dZ, R, HH, 64, kDwBK) || !tmap16(&ty, Y, R, CIN, 64, kDwBK))
     return cudaErrorInvalidValue;
-  k_tc16_dw<CINT><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows,
+  k_tc16_dw<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows,
                                                                CIN);
   return cudaGetLastError();
 }
@@ -419,7 +421,7 @@ size_t tc16_dw_partial_floats(int64_t R, int CIN) {
   return (size_t)dw16_chunks(R, CIN) * 256 * CIN;
 }
 
-cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, int CIN,
+cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, int CIN, int H,
                          float* part, cudaStream_t s, int* launches) {
   count_launch(launches, 2);
   int nchunk = dw16_chunks(R, CIN);
@@ -427,14 +429,17 @@ cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, in
   rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
   nchunk = (int)((R + rows - 1) / rows);
   cudaError_t e;
+  if (H != 128 && H != 256) return cudaErrorInvalidValue;
   switch (CIN) {
-    case 64: e = dw16_c<64>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
-    case 128: e = dw16_c<128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
-    case 256: e = dw16_c<128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
+    case 64: e = H == 256 ? dw16_c<64, 256>(Y, dZ, part, nchunk, R, rows, CIN, s)
+                          : dw16_c<64, 128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
+    case 128:
+    case 256: e = H == 256 ? dw16_c<128, 256>(Y, dZ, part, nchunk, R, rows, CIN, s)
+                           : dw16_c<128, 128>(Y, dZ, part, nchunk, R, rows, CIN, s); break;
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
-  k_dw16_reduce<<<cdiv(256LL * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, dW);
+  k_dw16_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
   return cudaGetLastError();
 }
 

@@ -127,7 +127,7 @@ cudaError_t tc_split_weights(const float* W, int CIN, int H, float* Bt_hi, float
 cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, float* C,
                          int64_t M, int N, int K, cudaStream_t s, int* launches);
 size_t tc_dw_partial_floats(int64_t R, int CIN);
-cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN,
+cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN, int H,
                        float* part, cudaStream_t s, int* launches);
 bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,
              int64_t rows, int64_t cols, int box_cols, int box_rows, CUtensorMapSwizzle swz);
@@ -141,7 +141,7 @@ cudaError_t tc16_weights(const float* W, int CIN, int H, void* Bt16, void* B16, 
 cudaError_t tc16_gemm_rows(const void* A, const void* B, void* C, int64_t M, int N, int K,
                            cudaStream_t s, int* launches);   // C = A·Bᵀ, all bf16
 size_t tc16_dw_partial_floats(int64_t R, int CIN);
-cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, int CIN,
+cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, int CIN, int H,
                          float* part, cudaStream_t s, int* launches);
 
 // ---------------------------------------------------------------- head.cu

@@ -579,7 +579,7 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
     return fail(MARS_EINVAL, "unknown precision %d", cfg->precision);
   if (cfg->precision == MARS_BF16 &&
       !(tc_supported(cfg->in_dim, cfg->hidden_dim) && tc_supported(cfg->hidden_dim, cfg->hidden_dim)))
-    return fail(MARS_EINVAL, "MARS_BF16 needs hidden_dim 256 and in_dim in {64, 128, 256}");
+    return fail(MARS_EINVAL, "MARS_BF16 needs hidden_dim in {128, 256} and in_dim in {64, 128, 256}");
   if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
     return fail(MARS_EINVAL, "bad world_size/rank");
   if (cfg->world_size > 1 && !cfg->nccl_unique_id)
@@ -633,7 +633,9 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
     CK(cudaGetLastError());
   }
   CK(cudaStreamSynchronize(s));
-  if (cfg->world_size > 1) {
+  // world_size > 1 needs a communicator; with world_size == 1 an id may still
+  // be passed to run the (identity) allreduce path, which the tests use.
+  if (cfg->world_size > 1 || cfg->nccl_unique_id) {
     if (!nccl_load()) return fail(MARS_ENCCL, "libnccl.so.2 not loadable");
     ncclUniqueId id;
     memcpy(&id, cfg->nccl_unique_id, sizeof id);
@@ -824,8 +826,8 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   // a12: backward, l = 3..1
   for (int l = 2; l >= 0; --l) {
     int Cin = l == 0 ? F : H;
-    if (b16) RET(tc16_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, w.dw16_part, s, nl));
-    else if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, w.dw_part, s, nl));
+    if (b16) RET(tc16_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, H, w.dw16_part, s, nl));
+    else if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, H, w.dw_part, s, nl));
     else RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
     MARK(MARS_PH_GEMM_DW);
     if (l > 0) {
@@ -1202,7 +1204,7 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
       }
       return gemm_nt(dA, dB, dC, M, N, K, s, nullptr);
     }
-    if (tcp) return tc_gemm_dw(dA, dB, dC, M, K, part, s, nullptr);
+    if (tcp) return tc_gemm_dw(dA, dB, dC, M, K, N, part, s, nullptr);
     return gemm_tn(dA, dB, dC, M, K, N, tpart, s, nullptr);
   };
   cudaEvent_t e0, e1;

@@ -32,10 +32,10 @@ def test_bf16_config_validation():
         mars.dgi_create(in_dim=16, hidden_dim=32, precision=mars.MARS_BF16)
 
 
-@pytest.mark.parametrize("name", ["gnmt", "bert"])
-def test_bf16_step(name):
+@pytest.mark.parametrize("name,H", [("gnmt", 256), ("bert", 256), ("inception", 128)])
+def test_bf16_step(name, H):
     gs = [SG.cached(name, 0)]
-    F, H = 64, 256
+    F = 64
     g, m, b, p0, out = _run(gs, F, H, 2)
     perms = b.perms(2, 0, 0)
     assert np.array_equal(out["perms"], perms)

@@ -24,11 +24,12 @@ def test_rows(impl, M, N, K):
 
 
 @pytest.mark.parametrize("impl", ["auto", "simt"])
-@pytest.mark.parametrize("M,K", [(16, 64), (5000, 256), (40001, 64), (123457, 256)])
-def test_dw(impl, M, K):
-    rng = np.random.default_rng(M + K)
+@pytest.mark.parametrize("H", [256, 128])
+@pytest.mark.parametrize("M,K", [(16, 64), (5000, 256), (40001, 64), (123457, 256), (3001, 128)])
+def test_dw(impl, H, M, K):
+    rng = np.random.default_rng(M + K + H)
     A = rng.standard_normal((M, K)).astype(np.float32)
-    B = rng.standard_normal((M, 256)).astype(np.float32)
+    B = rng.standard_normal((M, H)).astype(np.float32)
     C, _ = mars.debug_gemm("dw", A, B, impl)
     ref = A.astype(np.float64).T @ B.astype(np.float64)
     e = scaled_err(C, ref)

@@ -264,3 +264,22 @@ def test_pretrain_best_loss_snapshot():
     assert res["best_step"] == k and res["best_loss"] == losses[k]
     assert np.array_equal(res["best_params"], before[k])
     assert np.array_equal(ma.get_state()[0], mb.get_state()[0])
+
+
+def test_nccl_allreduce_path_one_rank():
+    """a13 plumbing on one GPU: a 1-rank NCCL communicator runs the captured
+    allreduce of grads + loss; the sum over one rank is the identity, so the
+    trajectory must equal the communicator-free run bitwise."""
+    gs = [SG.tiny(0), SG.tiny(1)]
+    g = mars.graph_load(gs)
+    try:
+        uid = mars.nccl_get_unique_id()
+    except mars.MarsError as e:
+        pytest.skip(f"NCCL not loadable: {e}")
+    ma = mars.dgi_create(in_dim=16, hidden_dim=32, seed=4, nccl_unique_id=uid)
+    mb = mars.dgi_create(in_dim=16, hidden_dim=32, seed=4)
+    for t in range(4):                       # steps 2+ replay the captured graph
+        la = ma.step(g, t, 0, want_loss=True)["loss"]
+        lb = mb.step(g, t, 0, want_loss=True)["loss"]
+        assert la == lb
+    assert np.array_equal(ma.get_state()[0], mb.get_state()[0])
