@@ -195,7 +195,8 @@ typedef enum {
   MARS_PH_SPMM_BWD = 6,   /* a12 dZ_{l-1} = (Â_n dY_l) ⊙ PReLU' (2 per step)  */
   MARS_PH_ALLREDUCE = 7,  /* a13 NCCL gradient allreduce                      */
   MARS_PH_ADAM = 8,       /* a14                                              */
-  MARS_PH_REDUCE = 9      /* dalpha partial reductions                        */
+  MARS_PH_REDUCE = 9,     /* dalpha partial reductions                        */
+  MARS_PH_EXCHANGE = 10   /* row-sharded graph: barriers, head / grad exchange */
 } mars_phase;
 
 /* Reporting hook: runs one step exactly like mars_dgi_step (same kernels,
@@ -217,6 +218,72 @@ MARS_API mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, uin
 MARS_API mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl, const float* A,
                                      const float* B, float* C, int64_t M, int32_t N, int32_t K,
                                      int32_t iters, float* ms);
+
+/* Copies the most recent step's loss and global-mean gradient (the values
+ * Adam consumed) to host memory (either may be NULL).  Synchronous.  For a
+ * row-sharded model, ECUDA if a cross-shard barrier timed out. */
+MARS_API mars_status mars_dgi_read_step(mars_dgi* m, float* loss, float* grads);
+
+/* ------------------------------------------------------------------------ */
+/* Row-sharded single graph: one op graph too large for   */
+/* one GPU (config 5: ~1M ops) split into P <= 8 contiguous row blocks, one   */
+/* per GPU.  Eq. 1's aggregation Â_n·act(T) on shard p needs the     */
+/* rows of T owned by other shards wherever its rows have columns outside the */
+/* block (the halo).  Every shard's activation buffers are mapped into every  */
+/* other shard's address space (CUDA IPC across processes, or peer access in  */
+/* one process) and the SpMM kernels gather halo rows directly by global      */
+/* column id over NVLink -- the exchange is fused into the aggregation.       */
+/* Device-side barriers order the reads; the readout sum (Eq. 4) and dv/loss  */
+/* (Eqs. 5-6) are exchanged after the shard-local reductions; W / alpha       */
+/* gradients are summed over shards in rank order, so every shard holds       */
+/* identical parameters.  One step of the P shards equals one step of the     */
+/* unsharded graph (one (graph, sample) pair, global_batch 1) up to fp32      */
+/* reduction order.  Every shard computes the whole corruption permutation   */
+/* and keeps the whole X (a few hundred MB at 1M ops).                        */
+/* Protocol: every shard (one process per GPU, or all in one process):       */
+/*   mars_graph_load_shard -> mars_dgi_create (same seed) -> mars_shard_attach */
+/*   -> mars_shard_export (blob, mars_shard_blob_bytes() bytes) -> all-gather */
+/*   the P blobs in rank order (e.g. torch.distributed) -> mars_shard_connect */
+/*   (or mars_shard_connect_local for models of one process) -> mars_dgi_step */
+/*   on every shard with the same step index.  A shard's step waits on device */
+/*   for its peers, so steps of the P shards must be enqueued without waiting */
+/*   for each other (out = NULL, then mars_dgi_read_step).  The graph must     */
+/*   outlive the model.  Needs hidden_dim in {128, 256}, the tcgen05 GEMMs and */
+/*   world_size 1 (no data parallelism on top).                               */
+/* ------------------------------------------------------------------------ */
+/* Loads shard `shard` of `num_shards` (<= 8) of one op graph: builds Â_n of
+ * the whole graph on `device` (as mars_graph_load), splits the rows into
+ * contiguous blocks balanced by nnz (start_p = first row whose rowptr >=
+ * p·nnz/P, each block >= 1 row).  EINVAL as mars_graph_load, or bad shard
+ * indices, or fewer nodes than shards. */
+MARS_API mars_status mars_graph_load_shard(const mars_graph_desc* graph, int32_t num_shards,
+                                           int32_t shard, int32_t device, mars_graph** out);
+/* Host-only (no device needed): the row split mars_graph_load_shard uses.
+ * rowptr [N+1] of Â (nnz offsets); writes starts[P+1]: start_0 = 0,
+ * start_p = max(start_{p-1} + 1, min(N - (P - p), first row r with
+ * rowptr[r] >= floor(p·nnz / P))), start_P = N. */
+MARS_API mars_status mars_shard_partition(const int32_t* rowptr, int32_t num_nodes,
+                                          int32_t num_shards, int32_t* starts);
+/* Shard geometry (any pointer may be NULL): shard count, index, the owned
+ * global rows [row_begin, row_end), their nnz, and the halo (distinct
+ * columns of the owned rows owned by other shards).  Unsharded graphs report
+ * 1, 0, [0, N), nnz, 0. */
+MARS_API mars_status mars_graph_shard_info(const mars_graph* g, int32_t* num_shards, int32_t* shard,
+                                           int32_t* row_begin, int32_t* row_end,
+                                           int64_t* local_nnz, int64_t* halo_rows);
+/* Binds model m to shard graph g for its lifetime: allocates the fixed
+ * workspace and the peer-visible exchange buffers. */
+MARS_API mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g);
+/* Size of the blob mars_shard_export writes. */
+MARS_API int64_t mars_shard_blob_bytes(void);
+/* Writes this shard's CUDA IPC handles (+ geometry check) into blob. */
+MARS_API mars_status mars_shard_export(const mars_dgi* m, void* blob);
+/* blobs: the P shards' blobs concatenated in rank order.  Opens the peers'
+ * buffers; after this, mars_dgi_step(m, g, ...) runs the sharded step. */
+MARS_API mars_status mars_shard_connect(mars_dgi* m, const void* blobs);
+/* Same for P models of this process (models[q] attached to shard q); enables
+ * peer access between distinct devices. */
+MARS_API mars_status mars_shard_connect_local(mars_dgi* const* models, int32_t num_shards);
 
 /* Kernel launches enqueued by the most recent mars_dgi_step (for reporting). */
 MARS_API int64_t mars_dgi_last_launches(const mars_dgi* m);

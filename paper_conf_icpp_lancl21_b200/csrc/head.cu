@@ -103,8 +103,10 @@ k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
 //   mode 0 (readout, Eq. 4): s = sig(Σ / N_g) -> outd (fp64), outf (fp32)
 //   mode 1 (dv):             Σ -> outd, outf; block (g, 0) also sums the
 //                            graph's loss partials -> loss_g[g]
+//   outf == nullptr (row-sharded graph): the raw shard-local Σ -> outd only
+//                            (summed over shards and finished in k_head_xsum)
 __global__ void k_chunk_sum(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
-                            const int32_t* __restrict__ node_off, int H, int mode,
+                            const int32_t* __restrict__ gsize, int H, int mode,
                             double* __restrict__ outd, float* __restrict__ outf,
                             const double* __restrict__ loss_part, double* __restrict__ loss_g) {
   __shared__ double sh[kWarps][32];
@@ -119,9 +121,9 @@ __global__ void k_chunk_sum(const double* __restrict__ part, const int32_t* __re
     double t = 0.0;
 #pragma unroll
     for (int k = 0; k < kWarps; ++k) t += sh[k][lane];
-    if (mode == 0) t = 1.0 / (1.0 + exp(-(t / (double)(node_off[g + 1] - node_off[g]))));
+    if (mode == 0 && outf) t = 1.0 / (1.0 + exp(-(t / (double)gsize[g])));
     outd[(int64_t)g * H + c] = t;
-    outf[(int64_t)g * H + c] = (float)t;
+    if (outf) outf[(int64_t)g * H + c] = (float)t;
   }
   if (mode == 1 && blockIdx.y == 0 && w == 1) {          // graph loss: lanes stride, fixed tree
     double t = 0.0;
@@ -150,7 +152,7 @@ __global__ void k_Mv(const float* __restrict__ M, const double* __restrict__ sd,
 // ds = Mᵀ dv_g and dm = ds s (1 - s) / N_g: grid (G, H/32); lanes own 32
 // columns, warp w sums rows w, w+8, ... (coalesced), fixed-order combine.
 __global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dvd,
-                      const double* __restrict__ sd, const int32_t* __restrict__ node_off, int H,
+                      const double* __restrict__ sd, const int32_t* __restrict__ gsize, int H,
                       float* __restrict__ dmf) {
   __shared__ double sh[kWarps][32];
   const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -165,7 +167,7 @@ __global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dv
 #pragma unroll
     for (int k = 0; k < kWarps; ++k) ds += sh[k][lane];
     const double s = sd[(int64_t)g * H + c];
-    dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / (double)(node_off[g + 1] - node_off[g]));
+    dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / (double)gsize[g]);
   }
 }
 
@@ -186,7 +188,7 @@ template <int NC, typename T>
 __global__ void __launch_bounds__(kWarps * 32, MARS_SCORE_MINB)
 k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
-        const int32_t* __restrict__ node_off, const float* __restrict__ vf,
+        const int32_t* __restrict__ gsize, const float* __restrict__ vf,
         const StepParams* __restrict__ sp, int32_t Nt, float* __restrict__ dl,
         double* __restrict__ dv_part, double* __restrict__ loss_part) {
   using RT = RowTile<NC, T>;
@@ -198,7 +200,7 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
   const bool act = lane < LPR;
   const int g = chunk_graph[ch];
   const float a = alpha[2];
-  const double Ng = (double)(node_off[g + 1] - node_off[g]);
+  const double Ng = (double)gsize[g];
   const double coef = (double)sp->inv_batch / (2.0 * Ng);
   const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
   float v[PER][V];
@@ -420,19 +422,38 @@ __global__ void k_upcast(const bf16* __restrict__ in, float* __restrict__ out, i
 template <int NC, typename T>
 cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float* alpha,
                     const StepParams* sp, const HeadWork& w, T* dZ, float* gM, float* loss_out,
-                    int* nslots, cudaStream_t s) {
+                    int* nslots, cudaStream_t s, const HeadShard* hs) {
   constexpr int H = NC * 32;
   const dim3 gh(g.G, H / 32);
+  cudaError_t e;
   k_colsum<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, w.colsum_part);
-  k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.node_off, H, 0, w.sd, w.s,
-                                 nullptr, nullptr);
+  if (!hs) {
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.gsize, H, 0, w.sd, w.s,
+                                   nullptr, nullptr);
+  } else {      // shard-local sums -> own exchange buffer; barrier; sum over shards
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.gsize, H, 0, hs->x_own[0],
+                                   nullptr, nullptr, nullptr);
+    if ((e = launch_shard_barrier(*hs->sync, s, nullptr)) != cudaSuccess) return e;
+    if ((e = launch_head_xsum(hs->x_peers[0], hs->sync->P, H, 0, g.gsize, w.sd, w.s, nullptr, s,
+                              nullptr)) != cudaSuccess)
+      return e;
+  }
   k_Mv<<<gh, 256, 0, s>>>(M, w.sd, H, w.v);
   k_score<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
-                                                   g.node_off, w.v, sp, g.Nt, w.dl, w.dv_part,
+                                                   g.gsize, w.v, sp, g.Nt, w.dl, w.dv_part,
                                                    w.loss_part);
-  k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.node_off, H, 1, w.dvd, w.dv,
-                                 w.loss_part, w.loss_g);
-  k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.node_off, H, w.dm);
+  if (!hs) {
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, w.dvd, w.dv,
+                                   w.loss_part, w.loss_g);
+  } else {
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, hs->x_own[1], nullptr,
+                                   w.loss_part, hs->x_own[1] + H);
+    if ((e = launch_shard_barrier(*hs->sync, s, nullptr)) != cudaSuccess) return e;
+    if ((e = launch_head_xsum(hs->x_peers[1], hs->sync->P, H, 1, g.gsize, w.dvd, w.dv, w.loss_g,
+                              s, nullptr)) != cudaSuccess)
+      return e;
+  }
+  k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.gsize, H, w.dm);
   k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
   k_dz3<NC, T><<<dim3(g.nchunks, 2), kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
                                                           w.dl, w.v, w.dm, g.Nt, dZ, w.slots);
@@ -443,14 +464,14 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
 template <typename T>
 cudaError_t head_t(const GraphDev& g, int H, const void* Z3, const float* M, const float* alpha,
                    const StepParams* sp, const HeadWork& w, void* dZ, float* gM, float* loss,
-                   int* nslots, cudaStream_t s) {
+                   int* nslots, cudaStream_t s, const HeadShard* hs) {
   const T* z = static_cast<const T*>(Z3);
   T* d = static_cast<T*>(dZ);
   switch (H) {
-    case 32: return head_nc<1, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
-    case 64: return head_nc<2, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
-    case 128: return head_nc<4, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
-    case 256: return head_nc<8, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s);
+    case 32: return head_nc<1, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s, hs);
+    case 64: return head_nc<2, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s, hs);
+    case 128: return head_nc<4, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s, hs);
+    case 256: return head_nc<8, T>(g, z, M, alpha, sp, w, d, gM, loss, nslots, s, hs);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -462,11 +483,11 @@ int head_slots(const GraphDev& g) { return 2 * g.nchunks + 1; }
 cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, const float* params_M,
                         const float* alpha_dev, const StepParams* sp, const HeadWork& w, void* dZ,
                         float* grad_M, float* loss_out, int* nslots, cudaStream_t s,
-                        int* launches) {
-  count_launch(launches, 8);
+                        int* launches, const HeadShard* hs) {
+  count_launch(launches, hs ? 12 : 8);
   if (bf16_)
-    return head_t<bf16>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
-  return head_t<float>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s);
+    return head_t<bf16>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s, hs);
+  return head_t<float>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s, hs);
 }
 
 cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,

@@ -8,6 +8,7 @@
 namespace mars {
 
 constexpr int kLayers = 3;
+constexpr int kMaxShards = 8;     // row shards of one graph (one per GPU of a node)
 
 // Per-step scalars the captured step graph reads from device memory (written
 // by one H2D copy before each replay, so a replay never bakes them in).
@@ -41,7 +42,44 @@ struct GraphDev {
   int32_t nbuckets;
   const int32_t* bucket_off; // [G+1]
   const int32_t* bucket_log2;// [G]
+  const int32_t* gsize;      // [G] node count N_g of each graph (all shards of a row-sharded graph)
 };
+
+// ---------------------------------------------------------------- row sharding
+// A row-sharded activation buffer as seen by every shard: shard p holds global
+// rows [start[p], start[p+1]) stacked [pos; neg] (2 n_p rows of C) at base[p],
+// which is device memory of shard p's GPU (peer-mapped; CUDA IPC across
+// processes).  start[q] = INT32_MAX for q > P, so owner(j) = #{q >= 1 : start[q] <= j}.
+struct PeerRows {
+  const void* base[kMaxShards];
+  int32_t start[kMaxShards + 1];
+};
+// Cross-shard device barrier: shard `me` stores its epoch into slot `me` of
+// every shard's arrival array (flags[q], peer-mapped) with release semantics at
+// system scope, then spins (acquire) until every slot of its own array reaches
+// the epoch.  epoch is a local device counter, so captured replays advance it.
+// A wait longer than ~20 s sets *err and returns (no hang).
+struct ShardSync {
+  int32_t P, me;
+  unsigned long long* flags[kMaxShards];
+  unsigned long long* epoch;
+  int32_t* err;
+};
+// Peer-visible small buffers read after a barrier (head exchange, gradients).
+struct PeerPtrs {
+  const void* p[kMaxShards];
+};
+cudaError_t launch_shard_barrier(const ShardSync& s, cudaStream_t st, int* launches);
+// Head exchange: t[c] = Σ_p x_p[c] over shards in rank order (fp64), c < H; the
+// loss slot x_p[H] is summed into *loss_g.  mode 0: outd = sig(t / N), outf =
+// (float) outd (readout s);  mode 1: outd = t, outf = (float) t (dv).
+cudaError_t launch_head_xsum(const PeerPtrs& x, int P, int H, int mode, const int32_t* gsize,
+                             double* outd, float* outf, double* loss_g, cudaStream_t st,
+                             int* launches);
+// out[k] = Σ_p g_p[k] (fp64, rank order) for k outside [keep_b, keep_e) and
+// k != n - 1; inside (dM, loss: already global on every shard) out[k] = g_me[k].
+cudaError_t launch_grad_sum(const PeerPtrs& g, int P, int me, int64_t n, int64_t keep_b,
+                            int64_t keep_e, float* out, cudaStream_t st, int* launches);
 
 // ---------------------------------------------------------------- builder.cu
 // Builds the CSR of Â for the packed set.  d_indptr: [Nt + G] int64 concatenated
@@ -97,15 +135,19 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
 // Otherwise act = PReLU(alpha[act_layer]).  neg_rows = 0 aggregates only the
 // positive branch (encode).
 // in_bf16 / out_bf16: storage type of T / Y (fp32 or bf16); fp32 accumulation.
+// peers != nullptr (row-sharded graph, layers 2-3 only): T is gathered from the
+// shards' buffers by global column id (C in {128, 256}, in_bf16 == out_bf16).
 cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16,
                             const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
-                            int out_bf16, int both, cudaStream_t s, int* launches);
+                            int out_bf16, int both, cudaStream_t s, int* launches,
+                            const PeerRows* peers = nullptr);
 // Backward aggregate dH = Â_n dY (Â_n symmetric) with the PReLU'(Z) epilogue:
 // dZ = dH ⊙ (Z > 0 ? 1 : a), dalpha partials Σ dH·min(Z,0) -> slots[gridDim].
 // dY, Z, dZ share one storage type (bf16 != 0: bf16).
 cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16,
                             const float* alpha_dev, int layer, void* dZ, double* slots,
-                            int* nslots, cudaStream_t s, int* launches);
+                            int* nslots, cudaStream_t s, int* launches,
+                            const PeerRows* peers = nullptr);
 int spmm_bwd_slots(const GraphDev& g);
 
 // ---------------------------------------------------------------- gemm_simt.cu
@@ -162,10 +204,17 @@ struct HeadWork {
 // Forward head + head backward: writes grads of M (dM) and the loss slot,
 // dZ3 into dZ, dalpha3 partials into w.slots.
 // Z3 / dZ storage: fp32 or bf16 (bf16 != 0).
+// Row-sharded graph: the two per-graph reductions (readout sum, dv + loss) are
+// exchanged between shards: chunk sums -> own x buffer, barrier, rank-ordered sum.
+struct HeadShard {
+  const ShardSync* sync;
+  double* x_own[2];          // [H + 1] each, peer-visible
+  PeerPtrs x_peers[2];
+};
 cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16,
                         const float* params_M, const float* alpha_dev, const StepParams* sp,
                         const HeadWork& w, void* dZ, float* grad_M, float* loss_out, int* nslots,
-                        cudaStream_t s, int* launches);
+                        cudaStream_t s, int* launches, const HeadShard* hs = nullptr);
 int head_slots(const GraphDev& g);
 // grad[0] = Σ slots (fixed order, double)
 cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,

@@ -190,17 +190,32 @@ struct mars_graph {
   int32_t *deg = nullptr, *chunk_row = nullptr, *chunk_graph = nullptr, *graph_chunk = nullptr;
   int32_t *bucket_off = nullptr, *bucket_log2 = nullptr;
   float *vals = nullptr, *dinv = nullptr, *X = nullptr;
+  int32_t* gsize = nullptr;
   GraphDev dev{};
+  // Row-sharded graph (mars_graph_load_shard): dev is the
+  // view of this shard's rows [row_begin, row_end) (local row ids, global
+  // column ids, the whole X); dev_full the whole graph (corruption permutation).
+  bool sharded = false;
+  int32_t P = 1, me = 0, row_begin = 0, row_end = 0;
+  int64_t halo_rows = 0, local_nnz = 0;
+  std::vector<int32_t> starts;
+  GraphDev dev_full{};
+  int32_t *l_node_off = nullptr, *l_node_graph = nullptr, *l_chunk_row = nullptr,
+          *l_chunk_graph = nullptr, *l_graph_chunk = nullptr;
   ~mars_graph() {   // pool memory; mars_free synchronises the device first
     for (void* p : {(void*)node_off, (void*)node_graph, (void*)rowptr, (void*)colind, (void*)deg,
                     (void*)chunk_row, (void*)chunk_graph, (void*)graph_chunk, (void*)bucket_off,
-                    (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X})
+                    (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X, (void*)gsize,
+                    (void*)l_node_off, (void*)l_node_graph, (void*)l_chunk_row,
+                    (void*)l_chunk_graph, (void*)l_graph_chunk})
       if (p) cudaFreeAsync(p, nullptr);
   }
+  const GraphDev& perm_view() const { return sharded ? dev_full : dev; }
 };
 
 struct Workspace {
   int32_t Nt = 0, G = 0, nchunks = 0, nbuckets = 0, F = 0, H = 0;
+  int32_t Nperm = 0;      // rows of the permutation (the whole graph when row-sharded)
   float *Y1 = nullptr, *Z[3] = {nullptr, nullptr, nullptr}, *Y23[2] = {nullptr, nullptr};
   float *dZ = nullptr, *dY = nullptr;
   int32_t* perm = nullptr;
@@ -249,8 +264,29 @@ struct mars_dgi {
   int64_t last_launches = 0, exec_launches = 0;
   int32_t last_Nt = 0;              // node count of the last step's graph set (export hook)
   ncclComm_t comm = nullptr;
+  // Row-sharded graph: the shard this model is attached to,
+  // its peer-visible buffers, and the peers' buffers once connected.
+  struct Shard {
+    const mars_graph* g = nullptr;
+    uint64_t guid = 0;
+    bool connected = false;
+    unsigned long long* flags = nullptr;   // [kMaxShards] arrival slots (peer-visible)
+    unsigned long long* epoch = nullptr;   // barrier counter (local)
+    int32_t* err = nullptr;                // barrier timeout flag (local)
+    double* xbuf = nullptr;                // [2][H+1] head exchange (peer-visible)
+    void* dY2 = nullptr;                   // layer-2 dY (layer 3 uses ws.dY), peer-visible
+    float* gsum = nullptr;                 // [P+1] gradients summed over shards
+    ShardSync sync{};
+    PeerRows z[2]{}, dy[2]{};
+    PeerPtrs x[2]{}, grads{};
+    std::vector<void*> ipc;                // pointers opened with cudaIpcOpenMemHandle
+    std::vector<void*> owned;
+  } sh;
+  float* grads_final() const { return sh.connected ? sh.gsum : grads; }
   ~mars_dgi() {
     if (exec) cudaGraphExecDestroy(exec);
+    for (void* p : sh.ipc) cudaIpcCloseMemHandle(p);
+    for (void* p : sh.owned) cudaFree(p);
     ws.release();
     for (void* p : {(void*)params, (void*)adam_m, (void*)adam_v, (void*)grads, (void*)norm_part,
                     (void*)finite_flag, (void*)d_sp})
@@ -393,6 +429,7 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   CK(palloc(&gr->graph_chunk, (size_t)G + 1, s));
   CK(palloc(&gr->bucket_off, (size_t)G + 1, s));
   CK(palloc(&gr->bucket_log2, (size_t)G, s));
+  CK(palloc(&gr->gsize, (size_t)G, s));
 
   // Inputs in page-locked host memory are copied straight to the device;
   // otherwise they are packed into a pinned staging buffer first.
@@ -439,6 +476,9 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   CK(cudaMemcpyAsync(gr->graph_chunk, graph_chunk.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(gr->bucket_off, bucket_off.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, s));
   CK(cudaMemcpyAsync(gr->bucket_log2, bucket_log2.data(), sizeof(int32_t) * G, cudaMemcpyHostToDevice, s));
+  std::vector<int32_t> gsize(G);
+  for (int g = 0; g < G; ++g) gsize[g] = descs[g].num_nodes;
+  CK(cudaMemcpyAsync(gr->gsize, gsize.data(), sizeof(int32_t) * G, cudaMemcpyHostToDevice, s));
   k_node_graph<<<cdiv(Nt, 256), 256, 0, s>>>(gr->node_off, G, (int32_t)Nt, gr->node_graph);
   CK(cudaGetLastError());
 
@@ -514,6 +554,7 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   v.nbuckets = bucket_off[G];
   v.bucket_off = gr->bucket_off;
   v.bucket_log2 = gr->bucket_log2;
+  v.gsize = gr->gsize;
   *out = guard.release();
   return MARS_OK;
 }
@@ -675,9 +716,11 @@ extern "C" mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable) {
 // ---------------------------------------------------------------- workspaces
 static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   Workspace& w = m->ws;
-  if (w.Nt >= g->Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks && w.nbuckets >= g->dev.nbuckets &&
-      w.F == m->F && w.H == m->H)
+  const GraphDev& pv = g->perm_view();
+  if (w.Nt >= g->dev.Nt && w.Nperm >= pv.Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks &&
+      w.nbuckets >= pv.nbuckets && w.F == m->F && w.H == m->H)
     return MARS_OK;
+  if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
   if (m->exec) {
     cudaGraphExecDestroy(m->exec);
     m->exec = nullptr;
@@ -685,8 +728,8 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   }
   CK(cudaStreamSynchronize(m->stream));
   w.release();
-  int64_t Nt = g->Nt, R = 2 * Nt;
-  int F = m->F, H = m->H, G = g->G, nch = g->dev.nchunks, nb = g->dev.nbuckets;
+  int64_t Nt = g->dev.Nt, R = 2 * Nt, Np = pv.Nt;
+  int F = m->F, H = m->H, G = g->G, nch = g->dev.nchunks, nb = pv.nbuckets;
   auto al = [&](void** p, size_t bytes) -> cudaError_t {
     cudaError_t e = cudaMalloc(p, bytes ? bytes : 8);
     if (e == cudaSuccess) w.owned.push_back(*p);
@@ -697,13 +740,13 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   for (int l = 0; l < 2; ++l) CK(al((void**)&w.Y23[l], sizeof(float) * R * H));
   CK(al((void**)&w.dZ, sizeof(float) * R * H));
   CK(al((void**)&w.dY, sizeof(float) * R * H));
-  CK(al((void**)&w.perm, sizeof(int32_t) * Nt));
-  CK(al((void**)&w.pw.keys, sizeof(uint64_t) * Nt));
-  CK(al((void**)&w.pw.bucket, sizeof(int32_t) * Nt));
+  CK(al((void**)&w.perm, sizeof(int32_t) * Np));
+  CK(al((void**)&w.pw.keys, sizeof(uint64_t) * Np));
+  CK(al((void**)&w.pw.bucket, sizeof(int32_t) * Np));
   CK(al((void**)&w.pw.bcnt, sizeof(int32_t) * (nb + 1)));
   CK(al((void**)&w.pw.bstart, sizeof(int32_t) * (nb + 1)));
   CK(al((void**)&w.pw.bcur, sizeof(int32_t) * (nb + 1)));
-  CK(al((void**)&w.pw.members, sizeof(int32_t) * Nt));
+  CK(al((void**)&w.pw.members, sizeof(int32_t) * Np));
   CK(al(&w.pw.scan_tmp, scan_tmp_bytes(nb + 1)));
   HeadWork& h = w.hw;
   CK(al((void**)&h.colsum_part, sizeof(double) * nch * H));
@@ -742,6 +785,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
                                                           tc16_dw_partial_floats(R, H))));
   }
   w.Nt = (int32_t)Nt;
+  w.Nperm = (int32_t)Np;
   w.G = G;
   w.nchunks = nch;
   w.nbuckets = nb;
@@ -794,8 +838,12 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     if (prof) RET(prof->mark(ph, s));           \
   } while (0)
   MARK(-1);
-  // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM)
-  RET(launch_perm(g, m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
+  // Row-sharded graph: exchange steps between the shards (shard.cu).  A
+  // barrier precedes every read of buffers the peers wrote in this step.
+  const bool shard = m->sh.connected && gr->uid == m->sh.guid;
+  // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM);
+  // a row-sharded graph permutes the whole graph on every shard
+  RET(launch_perm(gr->perm_view(), m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
   MARK(MARS_PH_PERM);
   const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
@@ -811,7 +859,12 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     const void* T = l == 0 ? (const void*)g.X : (const void*)w.Z[l - 1];
-    RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.perm, alpha, l - 1, Ys[l], b16, 1, s, nl));
+    if (shard && l > 0) {
+      RET(launch_shard_barrier(m->sh.sync, s, nl));   // peers' Z_{l-1} complete
+      MARK(MARS_PH_EXCHANGE);
+    }
+    RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.perm, alpha, l - 1, Ys[l], b16, 1, s, nl,
+                        shard && l > 0 ? &m->sh.z[l - 1] : nullptr));
     MARK(MARS_PH_SPMM_FWD);
     if (b16) RET(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], R, H, Cin, s, nl));
     else if (tc[l]) RET(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], R, H, Cin, s, nl));
@@ -820,7 +873,16 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   }
   // a8-a11 + dZ3
   int ns = 0;
-  RET(launch_head(g, H, w.Z[2], b16, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl));
+  HeadShard hs{};
+  if (shard) {
+    hs.sync = &m->sh.sync;
+    hs.x_own[0] = m->sh.xbuf;
+    hs.x_own[1] = m->sh.xbuf + H + 1;
+    hs.x_peers[0] = m->sh.x[0];
+    hs.x_peers[1] = m->sh.x[1];
+  }
+  RET(launch_head(g, H, w.Z[2], b16, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl,
+                  shard ? &hs : nullptr));
   RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
   MARK(MARS_PH_HEAD);
   // a12: backward, l = 3..1
@@ -831,12 +893,18 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     else RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
     MARK(MARS_PH_GEMM_DW);
     if (l > 0) {
-      if (b16) RET(tc16_gemm_rows(w.dZ, w.w16[l], w.dY, R, Cin, H, s, nl));
-      else if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], w.dY, R, Cin, H, s, nl));
-      else RET(gemm_nt(w.dZ, W[l], w.dY, R, Cin, H, s, nl));
+      // sharded: the two backward aggregations use separate peer-visible dY buffers
+      float* dYl = (shard && l == 1) ? static_cast<float*>(m->sh.dY2) : w.dY;
+      if (b16) RET(tc16_gemm_rows(w.dZ, w.w16[l], dYl, R, Cin, H, s, nl));
+      else if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], dYl, R, Cin, H, s, nl));
+      else RET(gemm_nt(w.dZ, W[l], dYl, R, Cin, H, s, nl));
       MARK(MARS_PH_GEMM_DY);
-      RET(launch_spmm_bwd(g, Cin, w.dY, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
-                          s, nl));
+      if (shard) {
+        RET(launch_shard_barrier(m->sh.sync, s, nl));  // peers' dY_l complete
+        MARK(MARS_PH_EXCHANGE);
+      }
+      RET(launch_spmm_bwd(g, Cin, dYl, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
+                          s, nl, shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr));
       MARK(MARS_PH_SPMM_BWD);
       RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
       MARK(MARS_PH_REDUCE);
@@ -849,9 +917,18 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     if (r != ncclSuccess) return cudaErrorUnknown;
     MARK(MARS_PH_ALLREDUCE);
   }
+  // row-sharded: sum the shards' W / alpha partials in rank order (dM and the
+  // loss are already global on every shard after the head exchange)
+  if (shard) {
+    RET(launch_shard_barrier(m->sh.sync, s, nl));
+    const int64_t mb = (int64_t)F * H + 2LL * H * H;
+    RET(launch_grad_sum(m->sh.grads, m->sh.sync.P, m->sh.sync.me, m->P + 1, mb, mb + (int64_t)H * H,
+                        m->sh.gsum, s, nl));
+    MARK(MARS_PH_EXCHANGE);
+  }
   // a14: Adam
-  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads, m->P, m->cfg.beta1, m->cfg.beta2,
-                  m->cfg.eps, m->cfg.clip_norm, m->norm_part, m->d_sp, s, nl));
+  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads_final(), m->P, m->cfg.beta1,
+                  m->cfg.beta2, m->cfg.eps, m->cfg.clip_norm, m->norm_part, m->d_sp, s, nl));
   MARK(MARS_PH_ADAM);
 #undef MARK
 #undef RET
@@ -915,7 +992,7 @@ extern "C" mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, u
   }
   *n_phases = n;
   m->last_launches = nl;
-  m->last_Nt = g->Nt;
+  m->last_Nt = g->dev.Nt;
   return MARS_OK;
 }
 
@@ -931,9 +1008,10 @@ extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t 
   cudaStream_t s = m->stream;
   if (out && (out->loss || out->grads || out->perms)) {
     float loss = 0.f;
-    CK(cudaMemcpyAsync(&loss, m->grads + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&loss, m->grads_final() + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
     if (out->grads)
-      CK(cudaMemcpyAsync(out->grads, m->grads, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
+      CK(cudaMemcpyAsync(out->grads, m->grads_final(), sizeof(float) * m->P,
+                         cudaMemcpyDeviceToHost, s));
     if (out->perms)
       CK(cudaMemcpyAsync(out->perms, m->ws.perm, sizeof(int32_t) * g->Nt, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
@@ -1000,7 +1078,7 @@ extern "C" mars_status mars_dgi_pretrain(mars_dgi* m, const mars_graph* g, uint6
     // the parameters a step's loss is computed with are the ones before its Adam update
     CK(cudaMemcpyAsync(prev, m->params, sizeof(float) * m->P, cudaMemcpyDeviceToDevice, s));
     if (mars_status st = run_step(m, g, step0 + (uint64_t)t, pair_base, global_batch)) return st;
-    k_track_decide<<<1, 1, 0, s>>>(m->grads + m->P, t, d_losses, d_bl, d_bs, d_flag);
+    k_track_decide<<<1, 1, 0, s>>>(m->grads_final() + m->P, t, d_losses, d_bl, d_bs, d_flag);
     k_track_copy<<<cdiv(m->P, 256), 256, 0, s>>>(d_flag, prev, best, m->P);
     CK(cudaGetLastError());
   }
@@ -1063,7 +1141,7 @@ static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_inde
     }
   }
   m->last_launches = nl;
-  m->last_Nt = g->Nt;
+  m->last_Nt = g->dev.Nt;
   return MARS_OK;
 }
 
@@ -1076,6 +1154,7 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
   if (mars_status st = check_dgi(m)) return st;
   if (mars_status st = check_graph(g)) return st;
   if (!emb) return fail(MARS_EINVAL, "embeddings is NULL");
+  if (g->sharded) return fail(MARS_EINVAL, "mars_encode runs on an unsharded graph");
   if (g->F != m->F) return fail(MARS_EINVAL, "feat_dim mismatch");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
@@ -1225,6 +1304,343 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   for (void* p : {(void*)dA, (void*)dB, (void*)dC, (void*)bh, (void*)bl, (void*)bth, (void*)btl,
                   (void*)part, (void*)tpart})
     cudaFree(p);
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- row-sharded graph (§8(e)(ii))
+namespace {
+constexpr uint64_t kShardBlobMagic = 0x4D41525353484431ULL;   // "MARSSHD1"
+constexpr int kShardBufs = 7;     // Z1, Z2, dY (layer 3), dY2 (layer 2), xbuf, flags, grads
+struct ShardBlob {
+  uint64_t magic;
+  int32_t P, me, device, H;
+  uint64_t graph_key;               // N, nnz and the row split must agree across shards
+  cudaIpcMemHandle_t h[kShardBufs];
+};
+
+uint64_t shard_key(const mars_graph* g) {
+  uint64_t k = sm64((uint64_t)g->Nt) ^ sm64((uint64_t)g->nnz + 0x51ULL);
+  for (int32_t v : g->starts) k = sm64(k ^ (uint64_t)(uint32_t)v);
+  return k;
+}
+
+void* shard_buf(const mars_dgi* m, int k) {
+  switch (k) {
+    case 0: return m->ws.Z[0];
+    case 1: return m->ws.Z[1];
+    case 2: return m->ws.dY;
+    case 3: return m->sh.dY2;
+    case 4: return m->sh.xbuf;
+    case 5: return m->sh.flags;
+    default: return m->grads;
+  }
+}
+
+// Fills the peer tables of m from the P shards' buffer pointers bufs[q][k].
+void shard_wire(mars_dgi* m, void* const (*bufs)[kShardBufs]) {
+  mars_dgi::Shard& sh = m->sh;
+  const mars_graph* g = sh.g;
+  PeerRows rows{};
+  for (int q = 0; q <= kMaxShards; ++q)
+    rows.start[q] = q < g->P ? g->starts[q] : (q == g->P ? g->Nt : INT32_MAX);
+  sh.z[0] = sh.z[1] = sh.dy[0] = sh.dy[1] = rows;
+  sh.sync.P = g->P;
+  sh.sync.me = g->me;
+  sh.sync.epoch = sh.epoch;
+  sh.sync.err = sh.err;
+  for (int q = 0; q < g->P; ++q) {
+    sh.z[0].base[q] = bufs[q][0];
+    sh.z[1].base[q] = bufs[q][1];
+    sh.dy[0].base[q] = bufs[q][2];
+    sh.dy[1].base[q] = bufs[q][3];
+    sh.x[0].p[q] = bufs[q][4];
+    sh.x[1].p[q] = static_cast<double*>(bufs[q][4]) + (m->H + 1);
+    sh.sync.flags[q] = static_cast<unsigned long long*>(bufs[q][5]);
+    sh.grads.p[q] = bufs[q][6];
+  }
+  sh.connected = true;
+  if (m->exec) {          // a captured step of this graph predates the wiring
+    cudaGraphExecDestroy(m->exec);
+    m->exec = nullptr;
+    m->exec_graph = 0;
+  }
+}
+
+// Captures the sharded step once at connect time and forces every kernel it
+// launches to load (cudaFuncGetAttributes).  With CUDA's lazy module loading a
+// kernel's first launch may wait for the whole context to go idle; inside a
+// sharded step that would wait on a barrier kernel spinning for a peer whose
+// launches are queued behind it (several shards in one process).  The
+// instantiated graph is kept, so the first step already replays it.
+mars_status shard_prepare(mars_dgi* m) {
+  const mars_graph* g = m->sh.g;
+  cudaStream_t s = m->stream;
+  int nl = 0;
+  cudaGraph_t graph;
+  CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+  cudaError_t e = enqueue_step(m, g, s, &nl);
+  cudaError_t e2 = cudaStreamEndCapture(s, &graph);
+  if (e != cudaSuccess || e2 != cudaSuccess) {
+    if (e2 == cudaSuccess) cudaGraphDestroy(graph);
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "sharded step capture failed: %s",
+                cudaGetErrorString(e != cudaSuccess ? e : e2));
+  }
+  struct GD { cudaGraph_t g; ~GD() { cudaGraphDestroy(g); } } gd{graph};
+  size_t n = 0;
+  CK(cudaGraphGetNodes(graph, nullptr, &n));
+  std::vector<cudaGraphNode_t> nodes(n);
+  CK(cudaGraphGetNodes(graph, nodes.data(), &n));
+  for (cudaGraphNode_t node : nodes) {
+    cudaGraphNodeType t;
+    CK(cudaGraphNodeGetType(node, &t));
+    if (t != cudaGraphNodeTypeKernel) continue;
+    cudaKernelNodeParams kp;
+    CK(cudaGraphKernelNodeGetParams(node, &kp));
+    cudaFuncAttributes fa;
+    CK(cudaFuncGetAttributes(&fa, kp.func));
+  }
+  if (m->exec) cudaGraphExecDestroy(m->exec);
+  m->exec = nullptr;
+  CK(cudaGraphInstantiate(&m->exec, graph, 0));
+  m->exec_graph = g->uid;
+  m->exec_stream = s;
+  m->exec_launches = nl;
+  return MARS_OK;
+}
+}  // namespace
+
+extern "C" mars_status mars_shard_partition(const int32_t* rowptr, int32_t N, int32_t P,
+                                            int32_t* starts) {
+  if (!rowptr || !starts || N < 1 || P < 1 || P > kMaxShards || N < P)
+    return fail(MARS_EINVAL, "bad partition arguments");
+  const int64_t nnz = rowptr[N];
+  starts[0] = 0;
+  for (int p = 1; p < P; ++p) {
+    const int64_t target = nnz * p / P;
+    int32_t r = (int32_t)(std::lower_bound(rowptr, rowptr + N + 1, (int32_t)target) - rowptr);
+    r = std::max(r, starts[p - 1] + 1);          // every shard owns >= 1 row
+    r = std::min(r, N - (P - p));
+    starts[p] = r;
+  }
+  starts[P] = N;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_graph_load_shard(const mars_graph_desc* desc, int32_t P, int32_t me,
+                                             int32_t device, mars_graph** out) {
+  if (!out) return fail(MARS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (!desc) return fail(MARS_EINVAL, "graph is NULL");
+  if (P < 1 || P > kMaxShards || me < 0 || me >= P)
+    return fail(MARS_EINVAL, "bad shard %d of %d (1 <= P <= %d)", me, P, kMaxShards);
+  if (desc->num_nodes < P) return fail(MARS_EINVAL, "fewer nodes than shards");
+  mars_graph* g = nullptr;
+  if (mars_status st = mars_graph_load(desc, 1, device, &g)) return st;
+  std::unique_ptr<mars_graph> guard(g);
+  const int32_t N = g->Nt;
+  // contiguous row blocks balanced by nnz (mars_shard_partition)
+  std::vector<int32_t> rp((size_t)N + 1);
+  CK(cudaMemcpy(rp.data(), g->rowptr, sizeof(int32_t) * (N + 1), cudaMemcpyDeviceToHost));
+  g->starts.assign(P + 1, 0);
+  if (mars_status st = mars_shard_partition(rp.data(), N, P, g->starts.data())) return st;
+  g->starts.resize(P);
+  const int32_t r0 = g->starts[me], r1 = me + 1 < P ? g->starts[me + 1] : N;
+  const int32_t n = r1 - r0;
+  g->sharded = true;
+  g->P = P;
+  g->me = me;
+  g->row_begin = r0;
+  g->row_end = r1;
+  g->local_nnz = (int64_t)rp[r1] - rp[r0];
+  {   // halo: distinct columns of the local rows owned by other shards
+    std::vector<int32_t> col((size_t)g->local_nnz);
+    CK(cudaMemcpy(col.data(), g->colind + rp[r0], sizeof(int32_t) * col.size(),
+                  cudaMemcpyDeviceToHost));
+    std::vector<uint8_t> seen((size_t)N, 0);
+    int64_t h = 0;
+    for (int32_t j : col)
+      if ((j < r0 || j >= r1) && !seen[j]) { seen[j] = 1; ++h; }
+    g->halo_rows = h;
+  }
+  // local view: rows [r0, r1) with local ids, global columns, the whole X
+  std::vector<int32_t> node_off = {0, n}, chunk_row, chunk_graph, graph_chunk = {0, 0};
+  for (int32_t r = 0; r < n; r += kChunkRows) {
+    chunk_row.push_back(r);
+    chunk_graph.push_back(0);
+  }
+  chunk_row.push_back(n);
+  graph_chunk[1] = (int32_t)chunk_graph.size();
+  const int nch = (int)chunk_graph.size();
+  cudaStream_t s = nullptr;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+  CK(palloc(&g->l_node_off, 2, s));
+  CK(palloc(&g->l_node_graph, (size_t)n, s));
+  CK(palloc(&g->l_chunk_row, (size_t)nch + 1, s));
+  CK(palloc(&g->l_chunk_graph, (size_t)nch, s));
+  CK(palloc(&g->l_graph_chunk, 2, s));
+  CK(cudaMemcpyAsync(g->l_node_off, node_off.data(), sizeof(int32_t) * 2, cudaMemcpyHostToDevice, s));
+  CK(cudaMemsetAsync(g->l_node_graph, 0, sizeof(int32_t) * n, s));
+  CK(cudaMemcpyAsync(g->l_chunk_row, chunk_row.data(), sizeof(int32_t) * (nch + 1), cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(g->l_chunk_graph, chunk_graph.data(), sizeof(int32_t) * nch, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(g->l_graph_chunk, graph_chunk.data(), sizeof(int32_t) * 2, cudaMemcpyHostToDevice, s));
+  CK(cudaStreamSynchronize(s));
+  g->dev_full = g->dev;
+  GraphDev& v = g->dev;
+  v.Nt = n;
+  v.nnz = g->local_nnz;
+  v.node_off = g->l_node_off;
+  v.node_graph = g->l_node_graph;
+  v.rowptr = g->rowptr + r0;             // global nnz offsets into the whole colind / vals
+  v.nchunks = nch;
+  v.chunk_row = g->l_chunk_row;
+  v.chunk_graph = g->l_chunk_graph;
+  v.graph_chunk = g->l_graph_chunk;
+  v.gsize = g->gsize;                    // N of the whole graph (readout mean, loss scale)
+  *out = guard.release();
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_graph_shard_info(const mars_graph* g, int32_t* P, int32_t* me,
+                                             int32_t* row_begin, int32_t* row_end,
+                                             int64_t* local_nnz, int64_t* halo_rows) {
+  if (mars_status st = check_graph(g)) return st;
+  if (P) *P = g->P;
+  if (me) *me = g->me;
+  if (row_begin) *row_begin = g->sharded ? g->row_begin : 0;
+  if (row_end) *row_end = g->sharded ? g->row_end : g->Nt;
+  if (local_nnz) *local_nnz = g->sharded ? g->local_nnz : g->nnz;
+  if (halo_rows) *halo_rows = g->sharded ? g->halo_rows : 0;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (mars_status st = check_graph(g)) return st;
+  if (!g->sharded) return fail(MARS_EINVAL, "graph was not loaded with mars_graph_load_shard");
+  if (m->sh.g) return fail(MARS_ESTATE, "model already attached to a shard");
+  if (m->comm) return fail(MARS_EINVAL, "a shard-attached model cannot also be data-parallel");
+  if (g->F != m->F || g->device != m->cfg.device) return fail(MARS_EINVAL, "F / device mismatch");
+  if (!(m->H == 128 || m->H == 256) || m->gemm_impl != MARS_GEMM_AUTO)
+    return fail(MARS_EINVAL, "row sharding needs hidden_dim in {128, 256} and the tcgen05 GEMMs");
+  CK(cudaSetDevice(m->cfg.device));
+  if (mars_status st = ensure_ws(m, g)) return st;
+  mars_dgi::Shard& sh = m->sh;
+  auto al = [&](void** p, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e == cudaSuccess) sh.owned.push_back(*p);
+    return e;
+  };
+  CK(al((void**)&sh.flags, sizeof(unsigned long long) * kMaxShards));
+  CK(al((void**)&sh.epoch, sizeof(unsigned long long)));
+  CK(al((void**)&sh.err, sizeof(int32_t)));
+  CK(al((void**)&sh.xbuf, sizeof(double) * 2 * (m->H + 1)));
+  CK(al(&sh.dY2, sizeof(float) * 2 * (size_t)g->dev.Nt * m->H));
+  CK(al((void**)&sh.gsum, sizeof(float) * (m->P + 1)));
+  // zeroed before any shard can connect (connecting is collective), so no
+  // early arrival signal is lost
+  CK(cudaMemset(sh.flags, 0, sizeof(unsigned long long) * kMaxShards));
+  CK(cudaMemset(sh.epoch, 0, sizeof(unsigned long long)));
+  CK(cudaMemset(sh.err, 0, sizeof(int32_t)));
+  CK(cudaMemset(sh.gsum, 0, sizeof(float) * (m->P + 1)));
+  CK(cudaDeviceSynchronize());
+  sh.g = g;
+  sh.guid = g->uid;
+  return MARS_OK;
+}
+
+extern "C" int64_t mars_shard_blob_bytes(void) { return (int64_t)sizeof(ShardBlob); }
+
+extern "C" mars_status mars_shard_export(const mars_dgi* m, void* blob) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!blob) return fail(MARS_EINVAL, "blob is NULL");
+  if (!m->sh.g) return fail(MARS_ESTATE, "mars_shard_attach first");
+  CK(cudaSetDevice(m->cfg.device));
+  ShardBlob b{};
+  b.magic = kShardBlobMagic;
+  b.P = m->sh.g->P;
+  b.me = m->sh.g->me;
+  b.device = m->cfg.device;
+  b.H = m->H;
+  b.graph_key = shard_key(m->sh.g);
+  for (int k = 0; k < kShardBufs; ++k) CK(cudaIpcGetMemHandle(&b.h[k], shard_buf(m, k)));
+  memcpy(blob, &b, sizeof b);
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_shard_connect(mars_dgi* m, const void* blobs) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!blobs) return fail(MARS_EINVAL, "blobs is NULL");
+  if (!m->sh.g) return fail(MARS_ESTATE, "mars_shard_attach first");
+  if (m->sh.connected) return fail(MARS_ESTATE, "already connected");
+  CK(cudaSetDevice(m->cfg.device));
+  const mars_graph* g = m->sh.g;
+  const ShardBlob* b = static_cast<const ShardBlob*>(blobs);
+  void* bufs[kMaxShards][kShardBufs] = {};
+  for (int q = 0; q < g->P; ++q) {
+    if (b[q].magic != kShardBlobMagic || b[q].P != g->P || b[q].me != q || b[q].H != m->H ||
+        b[q].graph_key != shard_key(g))
+      return fail(MARS_EINVAL, "shard blob %d does not match this graph / model", q);
+    for (int k = 0; k < kShardBufs; ++k) {
+      if (q == g->me) {
+        bufs[q][k] = shard_buf(m, k);
+        continue;
+      }
+      void* p = nullptr;
+      CK(cudaIpcOpenMemHandle(&p, b[q].h[k], cudaIpcMemLazyEnablePeerAccess));
+      m->sh.ipc.push_back(p);
+      bufs[q][k] = p;
+    }
+  }
+  shard_wire(m, bufs);
+  return shard_prepare(m);
+}
+
+extern "C" mars_status mars_shard_connect_local(mars_dgi* const* models, int32_t P) {
+  if (!models || P < 1 || P > kMaxShards) return fail(MARS_EINVAL, "bad model list");
+  void* bufs[kMaxShards][kShardBufs] = {};
+  for (int q = 0; q < P; ++q) {
+    mars_dgi* m = models[q];
+    if (mars_status st = check_dgi(m)) return st;
+    if (!m->sh.g) return fail(MARS_ESTATE, "model %d: mars_shard_attach first", q);
+    if (m->sh.connected) return fail(MARS_ESTATE, "model %d already connected", q);
+    if (m->sh.g->P != P || m->sh.g->me != q || m->H != models[0]->H ||
+        shard_key(m->sh.g) != shard_key(models[0]->sh.g))
+      return fail(MARS_EINVAL, "model %d is not shard %d of the same graph", q, q);
+    for (int k = 0; k < kShardBufs; ++k) bufs[q][k] = shard_buf(m, k);
+  }
+  for (int q = 0; q < P; ++q)          // peer access between distinct devices
+    for (int r = 0; r < P; ++r) {
+      const int dq = models[q]->cfg.device, dr = models[r]->cfg.device;
+      if (dq == dr) continue;
+      CK(cudaSetDevice(dq));
+      cudaError_t e = cudaDeviceEnablePeerAccess(dr, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+        return fail(MARS_ECUDA, "peer access %d -> %d: %s", dq, dr, cudaGetErrorString(e));
+      cudaGetLastError();
+    }
+  for (int q = 0; q < P; ++q) shard_wire(models[q], bufs);
+  for (int q = 0; q < P; ++q) {
+    CK(cudaSetDevice(models[q]->cfg.device));
+    if (mars_status st = shard_prepare(models[q])) return st;
+  }
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_read_step(mars_dgi* m, float* loss, float* grads) {
+  if (mars_status st = check_dgi(m)) return st;
+  CK(cudaSetDevice(m->cfg.device));
+  cudaStream_t s = m->stream;
+  float l = 0.f;
+  int32_t err = 0;
+  CK(cudaMemcpyAsync(&l, m->grads_final() + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+  if (grads)
+    CK(cudaMemcpyAsync(grads, m->grads_final(), sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
+  if (m->sh.err) CK(cudaMemcpyAsync(&err, m->sh.err, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (err) return fail(MARS_ECUDA, "shard barrier timed out (a peer shard did not step)");
+  if (loss) *loss = l;
   return MARS_OK;
 }
 

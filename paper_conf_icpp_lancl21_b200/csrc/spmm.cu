@@ -14,15 +14,27 @@
 //   fwd layer 1: T = X, neg rows gather X[pi[j]] (the corruption, fused)
 //   fwd layer l>1: act = PReLU_{a_{l-1}} applied on load (H_{l-1} never stored)
 //   bwd: epilogue dZ = dH ⊙ PReLU'(Z), dalpha partials Σ dH·min(Z,0) per block
+// Row-sharded graph (shard.cu): layers 2-3 and the backward
+// gather neighbour rows by GLOBAL column id from the owning shard's buffer
+// (PeerSrc: peer-mapped memory over NVLink, or CUDA IPC) -- the halo exchange
+// is fused into the aggregation; row i of the output is local.
 #include "common.cuh"
 #include "internal.cuh"
 #include "vec.cuh"
+
+#include <type_traits>
 
 namespace mars {
 namespace {
 
 constexpr int kSpmmThreads = 256;
-constexpr int kU = 4;           // neighbours whose gathers are in flight together
+#ifndef MARS_SPMM_MINB
+#define MARS_SPMM_MINB 0      // min resident blocks per SM for __launch_bounds__ (0: unset)
+#endif
+#ifndef MARS_SPMM_KU
+#define MARS_SPMM_KU 4
+#endif
+constexpr int kU = MARS_SPMM_KU;   // neighbours whose gathers are in flight together
 
 // C in {16, 32, 64, 128, 256} (mars.h restricts F and H to these widths).
 template <int C, typename T>
@@ -46,13 +58,131 @@ __device__ __forceinline__ void vprelu(float (&x)[V], float a) {
   for (int e = 0; e < V; ++e) x[e] = prelu(x[e], a);
 }
 
+// One row group (L lanes) per row, one block per RPB rows.  Measured and
+// rejected on the bench step: a persistent grid walking rows
+// i, i + NG, ... (+10-17 % fp32), and software pipelining across rows (the
+// next row's first (colind, val) chunk and the row after's rowptr in flight
+// during this row's gathers, +25-48 % fp32): ptxas keeps ~3 gathers per lane
+// in flight either way, so the saved index round trips are not the bound.
+
+// Sources of the gathered rows: pos row j, neg row (j, or perm[j] for layer 1).
+template <typename T, int C>
+struct StackedSrc {     // [pos; neg] stacked in one 2*Nt-row buffer
+  const T* base;
+  int32_t Nt;
+  __device__ __forceinline__ const T* pos(int32_t j) const { return base + (int64_t)j * C; }
+  __device__ __forceinline__ const T* neg(int32_t j, int32_t) const {
+    return base + ((int64_t)Nt + j) * C;
+  }
+};
+template <typename T, int C>
+struct PermSrc {        // layer 1: pos X[j], neg X[perm[j]]
+  const T* X;
+  __device__ __forceinline__ const T* pos(int32_t j) const { return X + (int64_t)j * C; }
+  __device__ __forceinline__ const T* neg(int32_t, int32_t jn) const { return X + (int64_t)jn * C; }
+};
+
+template <typename T, int C>
+struct PeerSrc {        // row-sharded graph: global row j lives on shard owner(j)
+  const PeerRows& pr;   // a __grid_constant__ kernel parameter (constant bank)
+  __device__ __forceinline__ int owner(int32_t j) const {
+    int p = 0;
+#pragma unroll
+    for (int q = 1; q < kMaxShards; ++q) p += j >= pr.start[q] ? 1 : 0;
+    return p;
+  }
+  __device__ __forceinline__ const T* pos(int32_t j) const {
+    const int p = owner(j);
+    return static_cast<const T*>(pr.base[p]) + (int64_t)(j - pr.start[p]) * C;
+  }
+  __device__ __forceinline__ const T* neg(int32_t j, int32_t) const {
+    const int p = owner(j);
+    const int32_t n = pr.start[p + 1] - pr.start[p];
+    return static_cast<const T*>(pr.base[p]) + ((int64_t)n + j - pr.start[p]) * C;
+  }
+};
+
+// Accumulates row (rb, re) of Â_n · act(T) for both branches: per chunk of L
+// neighbours each lane loads one (colind, val) pair (+ perm for layer 1),
+// broadcast by shuffles; full batches of kU neighbours issue all their
+// gathers before the FMAs, the remainder goes one neighbour at a time.
+template <class S, bool BOTH, bool ACT, bool PERM, typename T, class Src>
+__device__ __forceinline__ void row_gather(const Src& src, const int32_t* __restrict__ colind,
+                                           const float* __restrict__ vals,
+                                           const int32_t* __restrict__ perm, int32_t rb,
+                                           int32_t re, unsigned gmask, int sl, float a,
+                                           float (&accp)[S::NT][S::V],
+                                           float (&accn)[S::NT][S::V]) {
+  constexpr int V = S::V;
+  for (int32_t k0 = rb; k0 < re; k0 += S::L) {
+    const int32_t cnt = min(S::L, re - k0);
+    int32_t cj = 0, cjn = 0;
+    float cv = 0.f;
+    if (sl < cnt) {
+      cj = colind[k0 + sl];
+      cv = vals[k0 + sl];
+      if (PERM && BOTH) cjn = perm[cj];
+    }
+    int t = 0;
+    for (; t + kU <= cnt; t += kU) {
+      int32_t j[kU], jn[kU];
+      float w[kU];
+#pragma unroll
+      for (int u = 0; u < kU; ++u) {
+        j[u] = __shfl_sync(gmask, cj, t + u, S::L);
+        w[u] = __shfl_sync(gmask, cv, t + u, S::L);
+        jn[u] = (PERM && BOTH) ? __shfl_sync(gmask, cjn, t + u, S::L) : 0;
+      }
+      float xp[kU][S::NT][V], xn[kU][S::NT][V];
+#pragma unroll
+      for (int u = 0; u < kU; ++u)
+#pragma unroll
+        for (int q = 0; q < S::NT; ++q) {
+          const int c = (sl + q * S::L) * V;
+          Vec<T>::load(src.pos(j[u]) + c, xp[u][q]);
+          if (BOTH) Vec<T>::load(src.neg(j[u], jn[u]) + c, xn[u][q]);
+        }
+#pragma unroll
+      for (int u = 0; u < kU; ++u)
+#pragma unroll
+        for (int q = 0; q < S::NT; ++q) {
+          if (ACT) vprelu<V>(xp[u][q], a);
+          vfma<V>(accp[q], w[u], xp[u][q]);
+          if (BOTH) {
+            if (ACT) vprelu<V>(xn[u][q], a);
+            vfma<V>(accn[q], w[u], xn[u][q]);
+          }
+        }
+    }
+    for (; t < cnt; ++t) {
+      const int32_t j = __shfl_sync(gmask, cj, t, S::L);
+      const float w = __shfl_sync(gmask, cv, t, S::L);
+      const int32_t jn = (PERM && BOTH) ? __shfl_sync(gmask, cjn, t, S::L) : 0;
+#pragma unroll
+      for (int q = 0; q < S::NT; ++q) {
+        const int c = (sl + q * S::L) * V;
+        float x[V];
+        Vec<T>::load(src.pos(j) + c, x);
+        if (ACT) vprelu<V>(x, a);
+        vfma<V>(accp[q], w, x);
+        if (BOTH) {
+          Vec<T>::load(src.neg(j, jn) + c, x);
+          if (ACT) vprelu<V>(x, a);
+          vfma<V>(accn[q], w, x);
+        }
+      }
+    }
+  }
+}
+
 // MODE 0: layer 1 (neg rows gather X[perm[j]]), MODE 1: PReLU on load.
-template <int C, int MODE, bool BOTH, typename Tin, typename Tout>
-__global__ void __launch_bounds__(kSpmmThreads)
+// SH: row-sharded graph (layers 2-3): rows are gathered through PeerSrc.
+template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
+__global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
 k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const Tin* __restrict__ T,
            const int32_t* __restrict__ perm, const float* __restrict__ alpha, int act_layer,
-           int32_t Nt, Tout* __restrict__ Y) {
+           int32_t Nt, Tout* __restrict__ Y, const __grid_constant__ PeerRows pr) {
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
   const int lane = threadIdx.x & 31;
@@ -67,65 +197,15 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   for (int q = 0; q < S::NT; ++q)
 #pragma unroll
     for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
-  for (int32_t k0 = rb; k0 < re; k0 += S::L) {
-    const int32_t cnt = min(S::L, re - k0);
-    int32_t myj = 0, myjn = 0;
-    float myv = 0.f;
-    if (sl < cnt) {
-      myj = colind[k0 + sl];
-      myv = vals[k0 + sl];
-      if (BOTH) myjn = (MODE == 0) ? perm[myj] : Nt + myj;
-    }
-    int t = 0;
-    for (; t + kU <= cnt; t += kU) {
-      int32_t j[kU], jn[kU];
-      float w[kU];
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        j[u] = __shfl_sync(gmask, myj, t + u, S::L);
-        w[u] = __shfl_sync(gmask, myv, t + u, S::L);
-        jn[u] = BOTH ? __shfl_sync(gmask, myjn, t + u, S::L) : 0;
-      }
-      float xp[kU][S::NT][V], xn[kU][S::NT][V];
-#pragma unroll
-      for (int u = 0; u < kU; ++u)
-#pragma unroll
-        for (int q = 0; q < S::NT; ++q) {
-          const int c = (sl + q * S::L) * V;
-          Vec<Tin>::load(T + (int64_t)j[u] * C + c, xp[u][q]);
-          if (BOTH) Vec<Tin>::load(T + (int64_t)jn[u] * C + c, xn[u][q]);
-        }
-#pragma unroll
-      for (int u = 0; u < kU; ++u)
-#pragma unroll
-        for (int q = 0; q < S::NT; ++q) {
-          if (MODE == 1) vprelu<V>(xp[u][q], a);
-          vfma<V>(accp[q], w[u], xp[u][q]);
-          if (BOTH) {
-            if (MODE == 1) vprelu<V>(xn[u][q], a);
-            vfma<V>(accn[q], w[u], xn[u][q]);
-          }
-        }
-    }
-    for (; t < cnt; ++t) {
-      const int32_t j = __shfl_sync(gmask, myj, t, S::L);
-      const float w = __shfl_sync(gmask, myv, t, S::L);
-      const int32_t jn = BOTH ? __shfl_sync(gmask, myjn, t, S::L) : 0;
-#pragma unroll
-      for (int q = 0; q < S::NT; ++q) {
-        const int c = (sl + q * S::L) * V;
-        float x[V];
-        Vec<Tin>::load(T + (int64_t)j * C + c, x);
-        if (MODE == 1) vprelu<V>(x, a);
-        vfma<V>(accp[q], w, x);
-        if (BOTH) {
-          Vec<Tin>::load(T + (int64_t)jn * C + c, x);
-          if (MODE == 1) vprelu<V>(x, a);
-          vfma<V>(accn[q], w, x);
-        }
-      }
-    }
-  }
+  if (MODE == 0)
+    row_gather<S, BOTH, false, true, Tin>(PermSrc<Tin, C>{T}, colind, vals, perm, rb, re, gmask,
+                                          sl, a, accp, accn);
+  else if (SH)
+    row_gather<S, BOTH, true, false, Tin>(PeerSrc<Tin, C>{pr}, colind, vals, perm, rb, re, gmask,
+                                          sl, a, accp, accn);
+  else
+    row_gather<S, BOTH, true, false, Tin>(StackedSrc<Tin, C>{T, Nt}, colind, vals, perm, rb, re,
+                                          gmask, sl, a, accp, accn);
 #pragma unroll
   for (int q = 0; q < S::NT; ++q) {
     const int c = (sl + q * S::L) * V;
@@ -134,12 +214,12 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   }
 }
 
-template <int C, typename T>
-__global__ void __launch_bounds__(kSpmmThreads)
+template <int C, bool SH, typename T>
+__global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
 k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const T* __restrict__ dY, const T* __restrict__ Z,
            const float* __restrict__ alpha, int layer, int32_t Nt, T* __restrict__ dZ,
-           double* __restrict__ slots) {
+           double* __restrict__ slots, const __grid_constant__ PeerRows pr) {
   using S = SpmmShape<C, T>;
   constexpr int V = S::V;
   __shared__ double wpart[kSpmmThreads / 32];
@@ -156,54 +236,12 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
     for (int q = 0; q < S::NT; ++q)
 #pragma unroll
       for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
-    for (int32_t k0 = rb; k0 < re; k0 += S::L) {
-      const int32_t cnt = min(S::L, re - k0);
-      int32_t myj = 0;
-      float myv = 0.f;
-      if (sl < cnt) {
-        myj = colind[k0 + sl];
-        myv = vals[k0 + sl];
-      }
-      int t = 0;
-      for (; t + kU <= cnt; t += kU) {
-        int32_t j[kU];
-        float w[kU];
-#pragma unroll
-        for (int u = 0; u < kU; ++u) {
-          j[u] = __shfl_sync(gmask, myj, t + u, S::L);
-          w[u] = __shfl_sync(gmask, myv, t + u, S::L);
-        }
-        float xp[kU][S::NT][V], xn[kU][S::NT][V];
-#pragma unroll
-        for (int u = 0; u < kU; ++u)
-#pragma unroll
-          for (int q = 0; q < S::NT; ++q) {
-            const int c = (sl + q * S::L) * V;
-            Vec<T>::load(dY + (int64_t)j[u] * C + c, xp[u][q]);
-            Vec<T>::load(dY + ((int64_t)Nt + j[u]) * C + c, xn[u][q]);
-          }
-#pragma unroll
-        for (int u = 0; u < kU; ++u)
-#pragma unroll
-          for (int q = 0; q < S::NT; ++q) {
-            vfma<V>(accp[q], w[u], xp[u][q]);
-            vfma<V>(accn[q], w[u], xn[u][q]);
-          }
-      }
-      for (; t < cnt; ++t) {
-        const int32_t j = __shfl_sync(gmask, myj, t, S::L);
-        const float w = __shfl_sync(gmask, myv, t, S::L);
-#pragma unroll
-        for (int q = 0; q < S::NT; ++q) {
-          const int c = (sl + q * S::L) * V;
-          float x[V];
-          Vec<T>::load(dY + (int64_t)j * C + c, x);
-          vfma<V>(accp[q], w, x);
-          Vec<T>::load(dY + ((int64_t)Nt + j) * C + c, x);
-          vfma<V>(accn[q], w, x);
-        }
-      }
-    }
+    if (SH)
+      row_gather<S, true, false, false, T>(PeerSrc<T, C>{pr}, colind, vals, nullptr, rb, re,
+                                           gmask, sl, a, accp, accn);
+    else
+      row_gather<S, true, false, false, T>(StackedSrc<T, C>{dY, Nt}, colind, vals, nullptr, rb,
+                                           re, gmask, sl, a, accp, accn);
 #pragma unroll
     for (int q = 0; q < S::NT; ++q) {
       const int c = (sl + q * S::L) * V;
@@ -232,66 +270,81 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   }
 }
 
+template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
+cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
+                       int act_layer, Tout* Y, cudaStream_t s, const PeerRows& pr) {
+  using S = SpmmShape<C, Tin>;
+  k_spmm_fwd<C, MODE, BOTH, SH, Tin, Tout><<<cdiv(g.Nt, S::RPB), kSpmmThreads, 0, s>>>(
+      g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, pr);
+  return cudaGetLastError();
+}
+
 template <int C, typename Tin, typename Tout>
 cudaError_t fwd_c(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
-                  int act_layer, Tout* Y, int both, cudaStream_t s) {
-  using S = SpmmShape<C, Tin>;
-  const unsigned blocks = cdiv(g.Nt, S::RPB);
+                  int act_layer, Tout* Y, int both, cudaStream_t s, const PeerRows* peers) {
+  const PeerRows none{};
   if (act_layer < 0) {
-    if (both)
-      k_spmm_fwd<C, 0, true, Tin, Tout><<<blocks, kSpmmThreads, 0, s>>>(
-          g.rowptr, g.colind, g.vals, T, perm, alpha, 0, g.Nt, Y);
-    else
-      k_spmm_fwd<C, 0, false, Tin, Tout><<<blocks, kSpmmThreads, 0, s>>>(
-          g.rowptr, g.colind, g.vals, T, perm, alpha, 0, g.Nt, Y);
-  } else {
-    if (both)
-      k_spmm_fwd<C, 1, true, Tin, Tout><<<blocks, kSpmmThreads, 0, s>>>(
-          g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer, g.Nt, Y);
-    else
-      k_spmm_fwd<C, 1, false, Tin, Tout><<<blocks, kSpmmThreads, 0, s>>>(
-          g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer, g.Nt, Y);
+    if (peers) return cudaErrorInvalidValue;    // layer 1 reads the replicated X
+    return both ? fwd_launch<C, 0, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none)
+                : fwd_launch<C, 0, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none);
   }
-  return cudaGetLastError();
+  if constexpr ((C == 128 || C == 256) && std::is_same<Tin, Tout>::value) {
+    if (peers) {
+      if (!both) return cudaErrorInvalidValue;
+      return fwd_launch<C, 1, true, true, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, *peers);
+    }
+  }
+  if (peers) return cudaErrorInvalidValue;
+  return both ? fwd_launch<C, 1, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none)
+              : fwd_launch<C, 1, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none);
 }
 
 template <typename Tin, typename Tout>
 cudaError_t fwd_t(const GraphDev& g, int C, const void* T, const int32_t* perm, const float* alpha,
-                  int act_layer, void* Y, int both, cudaStream_t s) {
+                  int act_layer, void* Y, int both, cudaStream_t s, const PeerRows* pr) {
   const Tin* t = static_cast<const Tin*>(T);
   Tout* y = static_cast<Tout*>(Y);
   switch (C) {
-    case 16: return fwd_c<16, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s);
-    case 32: return fwd_c<32, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s);
-    case 64: return fwd_c<64, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s);
-    case 128: return fwd_c<128, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s);
-    case 256: return fwd_c<256, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s);
+    case 16: return fwd_c<16, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
+    case 32: return fwd_c<32, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
+    case 64: return fwd_c<64, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
+    case 128: return fwd_c<128, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
+    case 256: return fwd_c<256, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
     default: return cudaErrorInvalidValue;
   }
 }
 
 template <int C, typename T>
 cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha, int layer,
-                  T* dZ, double* slots, int* nslots, cudaStream_t s) {
+                  T* dZ, double* slots, int* nslots, cudaStream_t s, const PeerRows* peers) {
   using S = SpmmShape<C, T>;
   const unsigned blocks = cdiv(g.Nt, S::RPB);
-  k_spmm_bwd<C, T><<<blocks, kSpmmThreads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z, alpha,
-                                                   layer, g.Nt, dZ, slots);
   *nslots = (int)blocks;
+  if constexpr (C == 128 || C == 256) {
+    if (peers) {
+      k_spmm_bwd<C, true, T><<<blocks, kSpmmThreads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
+                                                             alpha, layer, g.Nt, dZ, slots, *peers);
+      return cudaGetLastError();
+    }
+  }
+  if (peers) return cudaErrorInvalidValue;
+  k_spmm_bwd<C, false, T><<<blocks, kSpmmThreads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z, alpha,
+                                                          layer, g.Nt, dZ, slots, PeerRows{});
   return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t bwd_t(const GraphDev& g, int C, const void* dY, const void* Z, const float* alpha,
-                  int layer, void* dZ, double* slots, int* nslots, cudaStream_t s) {
+                  int layer, void* dZ, double* slots, int* nslots, cudaStream_t s,
+                  const PeerRows* pr) {
   const T* d = static_cast<const T*>(dY);
   const T* z = static_cast<const T*>(Z);
   T* o = static_cast<T*>(dZ);
   switch (C) {
-    case 32: return bwd_c<32, T>(g, d, z, alpha, layer, o, slots, nslots, s);
-    case 64: return bwd_c<64, T>(g, d, z, alpha, layer, o, slots, nslots, s);
-    case 128: return bwd_c<128, T>(g, d, z, alpha, layer, o, slots, nslots, s);
-    case 256: return bwd_c<256, T>(g, d, z, alpha, layer, o, slots, nslots, s);
+    case 32: return bwd_c<32, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
+    case 64: return bwd_c<64, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
+    case 128: return bwd_c<128, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
+    case 256: return bwd_c<256, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -302,11 +355,15 @@ cudaError_t bwd_t(const GraphDev& g, int C, const void* dY, const void* Z, const
 // in_bf16 / out_bf16 select the storage type of T and Y.
 cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16,
                             const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
-                            int out_bf16, int both, cudaStream_t s, int* launches) {
+                            int out_bf16, int both, cudaStream_t s, int* launches,
+                            const PeerRows* peers) {
   count_launch(launches);
-  if (!in_bf16 && !out_bf16) return fwd_t<float, float>(g, C, T, perm, alpha_dev, act_layer, Y, both, s);
-  if (!in_bf16 && out_bf16) return fwd_t<float, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, both, s);
-  if (in_bf16 && out_bf16) return fwd_t<bf16, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, both, s);
+  if (!in_bf16 && !out_bf16)
+    return fwd_t<float, float>(g, C, T, perm, alpha_dev, act_layer, Y, both, s, peers);
+  if (!in_bf16 && out_bf16)
+    return fwd_t<float, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, both, s, peers);
+  if (in_bf16 && out_bf16)
+    return fwd_t<bf16, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, both, s, peers);
   return cudaErrorInvalidValue;
 }
 
@@ -315,10 +372,10 @@ int spmm_bwd_slots(const GraphDev& g) { return (int)cdiv(g.Nt, SpmmShape<256, fl
 
 cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16_,
                             const float* alpha_dev, int layer, void* dZ, double* slots,
-                            int* nslots, cudaStream_t s, int* launches) {
+                            int* nslots, cudaStream_t s, int* launches, const PeerRows* peers) {
   count_launch(launches);
-  if (bf16_) return bwd_t<bf16>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, s);
-  return bwd_t<float>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, s);
+  if (bf16_) return bwd_t<bf16>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, s, peers);
+  return bwd_t<float>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, s, peers);
 }
 
 }  // namespace mars

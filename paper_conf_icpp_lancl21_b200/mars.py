@@ -24,7 +24,7 @@ MARS_OK, MARS_EINVAL, MARS_ENOMEM, MARS_ECUDA, MARS_ENCCL, MARS_ENUMERIC, MARS_E
 MARS_FP32, MARS_BF16 = 0, 1
 _STATUS = {0: "OK", 1: "EINVAL", 2: "ENOMEM", 3: "ECUDA", 4: "ENCCL", 5: "ENUMERIC", 6: "ESTATE"}
 PHASES = ["perm", "spmm_fwd", "gemm_fwd", "head", "gemm_dw", "gemm_dy", "spmm_bwd", "allreduce",
-          "adam", "reduce"]
+          "adam", "reduce", "exchange"]
 
 
 class MarsError(RuntimeError):
@@ -90,6 +90,18 @@ SIGNATURES = {
                                        ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
                                        ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                        ctypes.c_int32, ctypes.c_void_p]),
+    "mars_dgi_read_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_graph_load_shard": (ctypes.c_int, [ctypes.POINTER(GraphDesc), ctypes.c_int32,
+                                             ctypes.c_int32, ctypes.c_int32,
+                                             ctypes.POINTER(ctypes.c_void_p)]),
+    "mars_graph_shard_info": (ctypes.c_int, [ctypes.c_void_p] + [ctypes.c_void_p] * 6),
+    "mars_shard_partition": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
+                                            ctypes.c_void_p]),
+    "mars_shard_attach": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_shard_blob_bytes": (ctypes.c_int64, []),
+    "mars_shard_export": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_shard_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_shard_connect_local": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int32]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -105,7 +117,10 @@ def lib():
             if not os.path.exists(LIB_PATH):
                 raise ImportError(f"{LIB_PATH} not built (run `make` or __graft_entry__.build())")
             L = ctypes.CDLL(LIB_PATH)
+            lenient = os.environ.get("MARS_BINDING_LENIENT") == "1"   # A/B of older builds
             for name, (res, args) in SIGNATURES.items():
+                if lenient and not hasattr(L, name):
+                    continue
                 fn = getattr(L, name)
                 fn.restype = res
                 fn.argtypes = args
@@ -191,6 +206,69 @@ def graph_load(graphs, device: int = 0) -> Graph:
     h = ctypes.c_void_p()
     _check(lib().mars_graph_load(descs, len(graphs), device, ctypes.byref(h)))
     return Graph(h, [int(g.num_nodes) for g in graphs], F)
+
+
+def _desc(g):
+    ip = np.ascontiguousarray(g.indptr, np.int64)
+    ix = np.ascontiguousarray(g.indices, np.int32)
+    X = np.ascontiguousarray(g.features, np.float32)
+    d = GraphDesc(int(g.num_nodes), ip.ctypes.data, ix.ctypes.data if ix.size else None,
+                  int(X.shape[1]), X.ctypes.data)
+    return d, (ip, ix, X)
+
+
+def graph_load_shard(graph, num_shards: int, shard: int, device: int = 0) -> Graph:
+    """mars_graph_load_shard: shard `shard` of `num_shards` row blocks of one op graph
+    (SURVEY §8(e)(ii)).  The Graph's sizes are the WHOLE graph's (the permutation
+    covers it); shard_info() gives the owned rows."""
+    d, keep = _desc(graph)
+    h = ctypes.c_void_p()
+    _check(lib().mars_graph_load_shard(ctypes.byref(d), int(num_shards), int(shard), device,
+                                       ctypes.byref(h)))
+    del keep
+    g = Graph(h, [int(graph.num_nodes)], d.feat_dim)
+    g.sharded = True
+    return g
+
+
+def shard_partition(rowptr, num_shards: int) -> np.ndarray:
+    """mars_shard_partition (host only): row starts [P+1] of the nnz-balanced split."""
+    rp = np.ascontiguousarray(rowptr, np.int32)
+    out = np.zeros(num_shards + 1, np.int32)
+    _check(lib().mars_shard_partition(_ptr(rp), rp.size - 1, int(num_shards), _ptr(out)))
+    return out
+
+
+def graph_shard_info(g: Graph):
+    P = ctypes.c_int32(); me = ctypes.c_int32(); r0 = ctypes.c_int32(); r1 = ctypes.c_int32()
+    z = ctypes.c_int64(); h = ctypes.c_int64()
+    _check(lib().mars_graph_shard_info(g.handle, ctypes.byref(P), ctypes.byref(me), ctypes.byref(r0),
+                                       ctypes.byref(r1), ctypes.byref(z), ctypes.byref(h)))
+    return dict(num_shards=P.value, shard=me.value, row_begin=r0.value, row_end=r1.value,
+                local_nnz=z.value, halo_rows=h.value)
+
+
+def shard_attach(m: "DGI", g: Graph):
+    _check(lib().mars_shard_attach(m.handle, g.handle))
+    m._shard_rows = graph_shard_info(g)["row_end"] - graph_shard_info(g)["row_begin"]
+
+
+def shard_export(m: "DGI") -> bytes:
+    buf = ctypes.create_string_buffer(int(lib().mars_shard_blob_bytes()))
+    _check(lib().mars_shard_export(m.handle, buf))
+    return buf.raw
+
+
+def shard_connect(m: "DGI", blobs):
+    """blobs: the P shards' export blobs in rank order (bytes each)."""
+    data = b"".join(blobs)
+    buf = ctypes.create_string_buffer(data, len(data))
+    _check(lib().mars_shard_connect(m.handle, buf))
+
+
+def shard_connect_local(models):
+    arr = (ctypes.c_void_p * len(models))(*[m.handle for m in models])
+    _check(lib().mars_shard_connect_local(arr, len(models)))
 
 
 def graph_export_csr(g: Graph, idx: int):
@@ -280,6 +358,14 @@ class DGI:
         self._last_nt = g.total_nodes
         return [(PHASES[int(i)], float(t)) for i, t in zip(ids[:n.value], ms[:n.value])]
 
+    def read_step(self, want_grads=True):
+        """mars_dgi_read_step: (loss, grads or None) of the most recent step."""
+        loss = ctypes.c_float()
+        grads = np.zeros(self.P, np.float32) if want_grads else None
+        _check(lib().mars_dgi_read_step(self.handle, ctypes.byref(loss),
+                                        None if grads is None else _ptr(grads)))
+        return loss.value, grads
+
     def last_launches(self) -> int:
         return int(lib().mars_dgi_last_launches(self.handle))
 
@@ -331,7 +417,7 @@ def dgi_step(m: DGI, g: Graph, step_index: int, pair_base: int = 0, global_batch
         res["perms"] = np.zeros(g.total_nodes, np.int32); out.perms = res["perms"].ctypes.data
     _check(lib().mars_dgi_step(m.handle, g.handle, step_index & (2 ** 64 - 1), int(pair_base), B,
                                ctypes.byref(out)))
-    m._last_nt = g.total_nodes
+    m._last_nt = getattr(m, "_shard_rows", None) if getattr(g, "sharded", False) else g.total_nodes
     if want_loss:
         res["loss"] = float(res["loss"][0])
     return res

@@ -14,6 +14,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def child(path):
     sys.path.insert(0, ROOT)
+    os.environ["MARS_BINDING_LENIENT"] = "1"
     import numpy as np
     import paper_conf_icpp_lancl21_b200.mars as M
     M.LIB_PATH = path
