@@ -35,6 +35,16 @@ sys.path.insert(0, ROOT)
 METRIC = "DGI contrastive steps/s on GNMT-shaped op graph; SpMM GB/s vs HBM peak"
 UNIT = "graph-steps/s"
 F, H = 64, 256
+# BASELINE.json configs as bench workloads: generator, default graphs per GPU, F, H.
+# "gnmt" is the metric's workload (the default line); the others are the
+# configs[] rows measured the same way.  "1m" is ONE graph of ~1.1M ops: one
+# GPU unsharded, or row-sharded over the ranks under torchrun.
+WORKLOADS = {
+    "gnmt": ("gnmt", 16, 64, 256, "GNMT-4 shaped training op graphs, T~U[20,50]"),
+    "inception": ("inception", 16, 64, 128, "Inception-V3 shaped training op graphs"),
+    "bert": ("bert", 8, 64, 256, "BERT-large shaped training op graphs"),
+    "1m": ("1m", 1, 64, 256, "1.1M-op GNMT stress graph (T=3000)"),
+}
 FFMA_TFLOPS_NOTE = "148 SM x 128 FP32 lanes x 2 flop x 1.965 GHz (B200_PROFILING.md counts)"
 
 
@@ -160,7 +170,10 @@ def run_reference(args):
         return 0
     import oracle
     from synth import graphs as SG
-    graphs = [SG.cached("gnmt", i) for i in range(args.graphs_per_gpu)]
+    gen = WORKLOADS[args.workload][0]
+    if args.workload == "1m":      # one GNMT graph stands in: a 1.1M-op fp64 step takes ~10 min
+        gen = "gnmt"
+    graphs = [SG.cached(gen, i) for i in range(args.graphs_per_gpu)]
     small = min(graphs, key=lambda g: g.num_nodes)
     tiny = SG.tiny(0)
     for w in range(args.warmup):                      # untimed (CPU has nothing to warm up)
@@ -175,14 +188,14 @@ def run_reference(args):
         p, m, v = oracle.adam(p, m, v, grads, k + 1)
     dt = time.perf_counter() - t0
     val = args.steps / dt
-    sample = (f"1 GNMT-shaped graph per step (the smallest of the workload's "
+    sample = (f"1 {gen}-shaped graph per step (the smallest of the workload's "
               f"{args.graphs_per_gpu}, N={small.num_nodes}), full DGI step + Adam in fp64")
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * dt / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
-            "config": {"workload": f"gnmt x{args.graphs_per_gpu} per GPU (sampled: 1 graph/step)",
-                       "F": F, "H": H},
+            "config": {"workload": f"{args.workload} x{args.graphs_per_gpu} per GPU "
+                                   f"(sampled: 1 graph/step)", "F": F, "H": H},
             "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
@@ -204,19 +217,38 @@ def run_mine(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     b = args.graphs_per_gpu
-    graphs = [SG.cached("gnmt", i) for i in dp.graph_indices(rank, world, b)]
-    uid = dp.broadcast_unique_id(mars.nccl_get_unique_id)
-    g = mars.graph_load(graphs, device=local)
+    gen, _, _, _, desc = WORKLOADS[args.workload]
+    sharded = args.workload == "1m" and world > 1
+    if args.workload == "1m":
+        graphs = [SG.make("1m", 0)]           # ~7 s to generate; one graph for the whole job
+    else:
+        graphs = [SG.cached(gen, i) for i in dp.graph_indices(rank, world, b)]
+    if sharded:
+        # rank r owns row block r of the one graph; the peers'
+        # activation buffers are opened over CUDA IPC (NVLink peer memory)
+        g = mars.graph_load_shard(graphs[0], world, rank, device=local)
+        m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local)
+        mars.shard_attach(m, g)
+        blobs = [None] * world
+        dist.all_gather_object(blobs, mars.shard_export(m))
+        mars.shard_connect(m, blobs)
+        shard_info = mars.graph_shard_info(g)
+        uid = None
+    else:
+        uid = dp.broadcast_unique_id(mars.nccl_get_unique_id)
+        g = mars.graph_load(graphs, device=local)
+        m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local, world_size=world,
+                            rank=rank, nccl_unique_id=uid)
+        shard_info = None
     info = g.info()
-    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local, world_size=world,
-                        rank=rank, nccl_unique_id=uid)
-    m.set_gemm_impl(args.gemm)
+    if not sharded:
+        m.set_gemm_impl(args.gemm)
     # a dedicated (non-legacy) stream: libmars launches and captures on it and
     # torch's CUDA events are recorded on it
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
     m.set_stream(stream.cuda_stream)
-    base, B = dp.pair_range(rank, world, b)
+    base, B = (0, 1) if sharded else dp.pair_range(rank, world, b)
     for w in range(args.warmup):
         m.step(g, w, base, B)
     torch.cuda.synchronize()
@@ -249,7 +281,8 @@ def run_mine(args):
         t = torch.tensor([ms], device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
-    value = world * b * args.steps / (ms / 1000.0)
+    # graph-steps per second of the whole job (the sharded 1m job is ONE graph)
+    value = (1 if sharded else world * b) * args.steps / (ms / 1000.0)
 
     # per-phase device time, CUDA events on the launching stream (same kernels, eager)
     nprof = max(1, min(args.steps, args.profile_steps))
@@ -262,6 +295,9 @@ def run_mine(args):
         prof_total += sum(t for _, t in ph)
     per_step = {k: sum(v) / nprof for k, v in acc.items()}
     N, Z = info["total_nodes"], info["nnz"]
+    if sharded:                       # per-rank accounting: the owned rows and their nnz
+        N = shard_info["row_end"] - shard_info["row_begin"]
+        Z = shard_info["local_nnz"]
     sp, gflops, gbytes = step_accounting(N, Z)
     pk = peaks()
     spmm_ms = per_step.get("spmm_fwd", 0) + per_step.get("spmm_bwd", 0)
@@ -313,7 +349,7 @@ def run_mine(args):
     # e2e through the public API: H2D of the step's graph batch from host memory,
     # CSR build, the step, D2H of the loss -- every step
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not sharded:
         # the step's inputs live in page-locked host memory (a data loader's
         # pinned batch); libmars copies them straight to the device
         class _Pinned:
@@ -351,7 +387,7 @@ def run_mine(args):
 
     # the bf16 path (MARS_BF16, 2e-2 parity bar) on the same workload, same timing
     b16 = None
-    if not args.no_bf16:
+    if not args.no_bf16 and not sharded:
         m16 = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local,
                               world_size=world, rank=rank, nccl_unique_id=uid,
                               precision=mars.MARS_BF16) if world == 1 else None
@@ -385,30 +421,43 @@ def run_mine(args):
             m16.free()
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and args.workload != "1m":
         import oracle
-        gr0 = graphs[0]
-        bo = oracle.Batch([gr0])
+        # a bounded sample of the workload: whole graphs of the step, one at a
+        # time, until ~10 s of single-thread CPU work (at most 4 graphs)
         p0 = oracle.xavier(args.seed, F, H).astype(np.float64)
         t0 = time.perf_counter()
-        loss, grads, _, _ = oracle.step_grads(bo, H, p0, bo.perms(args.seed, 0, 0))
-        oracle.adam(p0, np.zeros_like(p0), np.zeros_like(p0), grads, 1)
+        done = 0
+        for gr0 in graphs[:4]:
+            bo = oracle.Batch([gr0])
+            loss, grads, _, _ = oracle.step_grads(bo, H, p0, bo.perms(args.seed, 0, done))
+            oracle.adam(p0, np.zeros_like(p0), np.zeros_like(p0), grads, 1)
+            done += 1
+            if time.perf_counter() - t0 > 10.0:
+                break
         dt = time.perf_counter() - t0
-        cpu = {"value": 1.0 / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"1 of the {b} GNMT-shaped graphs of a step (graph 0, N={gr0.num_nodes}), "
+        cpu = {"value": done / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"{done} of the {b} {gen}-shaped graphs of a step (graphs 0..{done - 1}, "
+                         f"N={sum(x.num_nodes for x in graphs[:done])}), "
                          f"full fp64 DGI step + Adam, single thread, {dt:.1f} s"}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
-                "data": "synthetic",
-                "config": {"workload": f"gnmt x{b} per GPU (GNMT-4 shaped training op graphs, "
-                                       f"T~U[20,50])", "graphs_per_gpu": b, "F": F, "H": H,
+                "higher_is_better": True, "scaling": "strong" if sharded else "weak",
+                "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": (f"{args.workload}: one graph, row-sharded over {world} GPUs "
+                                        f"({desc})" if sharded else
+                                        f"{args.workload} x{b} per GPU ({desc})"),
+                           "graphs_per_gpu": b, "F": F, "H": H,
                            "nodes_per_gpu": N, "nnz_per_gpu": Z, "global_batch": B,
-                           "parallelism": f"dp{world}",
-                           "l2": "inputs larger than L2 (activations ~%.1f GB/step)"
-                                 % (2 * N * 4 * (F + 7 * H) / 1e9)},
+                           "parallelism": f"rowshard{world}" if sharded else f"dp{world}",
+                           "shard": shard_info,
+                           "l2": (("inputs larger than L2 (activations ~%.2f GB/step)"
+                                   if 2 * N * 4 * (F + 7 * H) > 126e6 else
+                                   "working set ~%.2f GB fits the 126 MB L2: a latency-bound "
+                                   "small-config number, no flush")
+                                  % (2 * N * 4 * (F + 7 * H) / 1e9))},
                 "roofline": roof, "rooflines": rooflines, "spmm": spmm_obj,
                 "phases_ms_per_step": per_step, "phase_share": shares,
                 "profiled_step_ms": prof_total / nprof,
@@ -428,7 +477,10 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="mine", choices=["mine", "reference"])
-    ap.add_argument("--graphs-per-gpu", type=int, default=16)
+    ap.add_argument("--workload", default="gnmt", choices=sorted(WORKLOADS),
+                    help="gnmt (the metric's workload, default), inception, bert, or 1m "
+                         "(one 1.1M-op graph; row-sharded under torchrun)")
+    ap.add_argument("--graphs-per-gpu", type=int, default=None)
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--gemm", default="auto", choices=["auto", "simt"],
                     help="dense-transform kernels: tcgen05 3xTF32 (auto) or FFMA (simt)")
@@ -440,6 +492,10 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    global F, H
+    _, bdef, F, H, _ = WORKLOADS[args.workload]
+    if args.graphs_per_gpu is None:
+        args.graphs_per_gpu = bdef
     if args.impl == "reference":
         return run_reference(args)
     return run_mine(args)

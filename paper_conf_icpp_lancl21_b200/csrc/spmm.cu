@@ -22,6 +22,7 @@
 #include "internal.cuh"
 #include "vec.cuh"
 
+#include <algorithm>
 #include <type_traits>
 
 namespace mars {
@@ -29,7 +30,7 @@ namespace {
 
 constexpr int kSpmmThreads = 256;
 #ifndef MARS_SPMM_MINB
-#define MARS_SPMM_MINB 0      // min resident blocks per SM for __launch_bounds__ (0: unset)
+#define MARS_SPMM_MINB 4      // resident 256-thread blocks per SM: caps registers at 64
 #endif
 #ifndef MARS_SPMM_KU
 #define MARS_SPMM_KU 4
@@ -58,12 +59,10 @@ __device__ __forceinline__ void vprelu(float (&x)[V], float a) {
   for (int e = 0; e < V; ++e) x[e] = prelu(x[e], a);
 }
 
-// One row group (L lanes) per row, one block per RPB rows.  Measured and
-// rejected on the bench step: a persistent grid walking rows
-// i, i + NG, ... (+10-17 % fp32), and software pipelining across rows (the
-// next row's first (colind, val) chunk and the row after's rowptr in flight
-// during this row's gathers, +25-48 % fp32): ptxas keeps ~3 gathers per lane
-// in flight either way, so the saved index round trips are not the bound.
+// Measured and rejected on the bench step: a persistent grid
+// interleaving rows i, i + NG, ... over all SMs (+10-17 % fp32), and software
+// pipelining across rows (next row's first (colind, val) chunk and the row
+// after's rowptr in flight during this row's gathers, +25-48 % fp32).
 
 // Sources of the gathered rows: pos row j, neg row (j, or perm[j] for layer 1).
 template <typename T, int C>
@@ -102,10 +101,58 @@ struct PeerSrc {        // row-sharded graph: global row j lives on shard owner(
   }
 };
 
+#ifndef MARS_SPMM_TAIL
+#define MARS_SPMM_TAIL 1
+#endif
+
+// One batch of K neighbours t .. t+K-1 of the current chunk: all 2K gathers
+// are issued before the FMAs.  Slots u >= nvalid re-gather neighbour t (a
+// valid row, usually an L1 hit) with weight 0, so the batch needs no branch
+// and its loads stay independent.  Adding 0·x leaves the ascending-order sum
+// unchanged.
+template <class S, int K, bool BOTH, bool ACT, bool PERM, typename T, class Src>
+__device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, int32_t cj,
+                                             float cv, int32_t cjn, unsigned gmask, int sl,
+                                             float a, float (&accp)[S::NT][S::V],
+                                             float (&accn)[S::NT][S::V]) {
+  constexpr int V = S::V;
+  int32_t j[K], jn[K];
+  float w[K];
+#pragma unroll
+  for (int u = 0; u < K; ++u) {
+    const int lane_u = u < nvalid ? t + u : t;
+    j[u] = __shfl_sync(gmask, cj, lane_u, S::L);
+    w[u] = __shfl_sync(gmask, cv, lane_u, S::L);
+    jn[u] = (PERM && BOTH) ? __shfl_sync(gmask, cjn, lane_u, S::L) : 0;
+    if (u >= nvalid) w[u] = 0.f;
+  }
+  float xp[K][S::NT][V], xn[K][S::NT][V];
+#pragma unroll
+  for (int u = 0; u < K; ++u)
+#pragma unroll
+    for (int q = 0; q < S::NT; ++q) {
+      const int c = (sl + q * S::L) * V;
+      Vec<T>::load(src.pos(j[u]) + c, xp[u][q]);
+      if (BOTH) Vec<T>::load(src.neg(j[u], jn[u]) + c, xn[u][q]);
+    }
+#pragma unroll
+  for (int u = 0; u < K; ++u)
+#pragma unroll
+    for (int q = 0; q < S::NT; ++q) {
+      if (ACT) vprelu<V>(xp[u][q], a);
+      vfma<V>(accp[q], w[u], xp[u][q]);
+      if (BOTH) {
+        if (ACT) vprelu<V>(xn[u][q], a);
+        vfma<V>(accn[q], w[u], xn[u][q]);
+      }
+    }
+}
+
 // Accumulates row (rb, re) of Â_n · act(T) for both branches: per chunk of L
 // neighbours each lane loads one (colind, val) pair (+ perm for layer 1),
-// broadcast by shuffles; full batches of kU neighbours issue all their
-// gathers before the FMAs, the remainder goes one neighbour at a time.
+// broadcast by shuffles, then batches of kU neighbours.  MARS_SPMM_TAIL
+// selects the last partial batch: 1 = one padded batch (default), 0 = one
+// neighbour at a time, 2 = a batch of 2 then 1.
 template <class S, bool BOTH, bool ACT, bool PERM, typename T, class Src>
 __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __restrict__ colind,
                                            const float* __restrict__ vals,
@@ -113,7 +160,6 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
                                            int32_t re, unsigned gmask, int sl, float a,
                                            float (&accp)[S::NT][S::V],
                                            float (&accn)[S::NT][S::V]) {
-  constexpr int V = S::V;
   for (int32_t k0 = rb; k0 < re; k0 += S::L) {
     const int32_t cnt = min(S::L, re - k0);
     int32_t cj = 0, cjn = 0;
@@ -123,74 +169,38 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
       cv = vals[k0 + sl];
       if (PERM && BOTH) cjn = perm[cj];
     }
+#if MARS_SPMM_TAIL == 1
+    for (int t = 0; t < cnt; t += kU)
+      gather_batch<S, kU, BOTH, ACT, PERM, T>(src, t, min(kU, cnt - t), cj, cv, cjn, gmask, sl,
+                                              a, accp, accn);
+#else
     int t = 0;
-    for (; t + kU <= cnt; t += kU) {
-      int32_t j[kU], jn[kU];
-      float w[kU];
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        j[u] = __shfl_sync(gmask, cj, t + u, S::L);
-        w[u] = __shfl_sync(gmask, cv, t + u, S::L);
-        jn[u] = (PERM && BOTH) ? __shfl_sync(gmask, cjn, t + u, S::L) : 0;
-      }
-      float xp[kU][S::NT][V], xn[kU][S::NT][V];
-#pragma unroll
-      for (int u = 0; u < kU; ++u)
-#pragma unroll
-        for (int q = 0; q < S::NT; ++q) {
-          const int c = (sl + q * S::L) * V;
-          Vec<T>::load(src.pos(j[u]) + c, xp[u][q]);
-          if (BOTH) Vec<T>::load(src.neg(j[u], jn[u]) + c, xn[u][q]);
-        }
-#pragma unroll
-      for (int u = 0; u < kU; ++u)
-#pragma unroll
-        for (int q = 0; q < S::NT; ++q) {
-          if (ACT) vprelu<V>(xp[u][q], a);
-          vfma<V>(accp[q], w[u], xp[u][q]);
-          if (BOTH) {
-            if (ACT) vprelu<V>(xn[u][q], a);
-            vfma<V>(accn[q], w[u], xn[u][q]);
-          }
-        }
+    for (; t + kU <= cnt; t += kU)
+      gather_batch<S, kU, BOTH, ACT, PERM, T>(src, t, kU, cj, cv, cjn, gmask, sl, a, accp, accn);
+#if MARS_SPMM_TAIL == 2
+    if (t + 2 <= cnt) {
+      gather_batch<S, 2, BOTH, ACT, PERM, T>(src, t, 2, cj, cv, cjn, gmask, sl, a, accp, accn);
+      t += 2;
     }
-    for (; t < cnt; ++t) {
-      const int32_t j = __shfl_sync(gmask, cj, t, S::L);
-      const float w = __shfl_sync(gmask, cv, t, S::L);
-      const int32_t jn = (PERM && BOTH) ? __shfl_sync(gmask, cjn, t, S::L) : 0;
-#pragma unroll
-      for (int q = 0; q < S::NT; ++q) {
-        const int c = (sl + q * S::L) * V;
-        float x[V];
-        Vec<T>::load(src.pos(j) + c, x);
-        if (ACT) vprelu<V>(x, a);
-        vfma<V>(accp[q], w, x);
-        if (BOTH) {
-          Vec<T>::load(src.neg(j, jn) + c, x);
-          if (ACT) vprelu<V>(x, a);
-          vfma<V>(accn[q], w, x);
-        }
-      }
-    }
+#endif
+    for (; t < cnt; ++t)
+      gather_batch<S, 1, BOTH, ACT, PERM, T>(src, t, 1, cj, cv, cjn, gmask, sl, a, accp, accn);
+#endif
   }
 }
 
+// Row bodies shared by the two kernel shapes below.
 // MODE 0: layer 1 (neg rows gather X[perm[j]]), MODE 1: PReLU on load.
 // SH: row-sharded graph (layers 2-3): rows are gathered through PeerSrc.
 template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
-__global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
-k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
-           const float* __restrict__ vals, const Tin* __restrict__ T,
-           const int32_t* __restrict__ perm, const float* __restrict__ alpha, int act_layer,
-           int32_t Nt, Tout* __restrict__ Y, const __grid_constant__ PeerRows pr) {
+__device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ rowptr,
+                                        const int32_t* __restrict__ colind,
+                                        const float* __restrict__ vals, const Tin* __restrict__ T,
+                                        const int32_t* __restrict__ perm, float a, int32_t Nt,
+                                        Tout* __restrict__ Y, const PeerRows& pr, unsigned gmask,
+                                        int sl) {
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
-  const int lane = threadIdx.x & 31;
-  const int sub = lane / S::L, sl = lane % S::L;
-  const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
-  const int32_t i = (int32_t)(((int64_t)blockIdx.x * kSpmmThreads + threadIdx.x) / 32) * S::RPW + sub;
-  if (i >= Nt) return;
-  const float a = (MODE == 1) ? alpha[act_layer] : 1.f;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
   float accp[S::NT][V], accn[S::NT][V];
 #pragma unroll
@@ -215,67 +225,147 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
 }
 
 template <int C, bool SH, typename T>
-__global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
+__device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ rowptr,
+                                        const int32_t* __restrict__ colind,
+                                        const float* __restrict__ vals, const T* __restrict__ dY,
+                                        const T* __restrict__ Z, float a, int32_t Nt,
+                                        T* __restrict__ dZ, const PeerRows& pr, unsigned gmask,
+                                        int sl, float& da) {
+  using S = SpmmShape<C, T>;
+  constexpr int V = S::V;
+  const int32_t rb = rowptr[i], re = rowptr[i + 1];
+  float accp[S::NT][V], accn[S::NT][V];
+#pragma unroll
+  for (int q = 0; q < S::NT; ++q)
+#pragma unroll
+    for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
+  if (SH)
+    row_gather<S, true, false, false, T>(PeerSrc<T, C>{pr}, colind, vals, nullptr, rb, re, gmask,
+                                         sl, a, accp, accn);
+  else
+    row_gather<S, true, false, false, T>(StackedSrc<T, C>{dY, Nt}, colind, vals, nullptr, rb, re,
+                                         gmask, sl, a, accp, accn);
+#pragma unroll
+  for (int q = 0; q < S::NT; ++q) {
+    const int c = (sl + q * S::L) * V;
+#pragma unroll
+    for (int br = 0; br < 2; ++br) {
+      const int64_t row = (int64_t)i + (br ? Nt : 0);
+      float z[V], o[V];
+      Vec<T>::load(Z + row * C + c, z);
+#pragma unroll
+      for (int e = 0; e < V; ++e) {
+        const float h = br ? accn[q][e] : accp[q][e];
+        o[e] = z[e] > 0.f ? h : a * h;
+        da += z[e] > 0.f ? 0.f : h * z[e];
+      }
+      StoreN<T, V>::store(dZ + row * C + c, o);
+    }
+  }
+}
+
+// Rows handled by block b: NW warps x RPW row groups.  BAND = false: one row
+// per group, blocks of consecutive rows (kSpmmThreads = 256).  BAND = true: a
+// persistent grid of one 1024-thread block per SM, block b sweeping the
+// contiguous band of rows [b·n, (b+1)·n) 32·RPW rows at a time, so the rows
+// its warps gather (op graphs are local: most neighbours lie within a few
+// dozen rows) were just read by the same SM and hit in its L1 instead of L2.
+template <int C, typename T, bool BAND>
+struct RowSched {
+  using S = SpmmShape<C, T>;
+  static constexpr int NW = BAND ? 32 : kSpmmThreads / 32;
+  static constexpr int RPB = S::RPW * NW;
+};
+
+#ifndef MARS_SPMM_BAND
+#define MARS_SPMM_BAND 0
+#endif
+constexpr int kBandThreads = 1024;
+
+template <int C, int MODE, bool BOTH, bool SH, bool BAND, typename Tin, typename Tout>
+__global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 : MARS_SPMM_MINB)
+k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
+           const float* __restrict__ vals, const Tin* __restrict__ T,
+           const int32_t* __restrict__ perm, const float* __restrict__ alpha, int act_layer,
+           int32_t Nt, Tout* __restrict__ Y, const __grid_constant__ PeerRows pr) {
+  using S = SpmmShape<C, Tin>;
+  using RS = RowSched<C, Tin, BAND>;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int sub = lane / S::L, sl = lane % S::L;
+  const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
+  const float a = (MODE == 1) ? alpha[act_layer] : 1.f;
+  if (!BAND) {
+    const int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub;
+    if (i < Nt) fwd_row<C, MODE, BOTH, SH>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+    return;
+  }
+  const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
+  const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
+  for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
+    fwd_row<C, MODE, BOTH, SH>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+}
+
+template <int C, bool SH, bool BAND, typename T>
+__global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 : MARS_SPMM_MINB)
 k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const T* __restrict__ dY, const T* __restrict__ Z,
            const float* __restrict__ alpha, int layer, int32_t Nt, T* __restrict__ dZ,
            double* __restrict__ slots, const __grid_constant__ PeerRows pr) {
   using S = SpmmShape<C, T>;
-  constexpr int V = S::V;
-  __shared__ double wpart[kSpmmThreads / 32];
-  const int lane = threadIdx.x & 31;
+  using RS = RowSched<C, T, BAND>;
+  __shared__ double wpart[RS::NW];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int sub = lane / S::L, sl = lane % S::L;
   const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
-  const int32_t i = (int32_t)(((int64_t)blockIdx.x * kSpmmThreads + threadIdx.x) / 32) * S::RPW + sub;
+  const float a = alpha[layer];
   float da = 0.f;
-  if (i < Nt) {
-    const float a = alpha[layer];
-    const int32_t rb = rowptr[i], re = rowptr[i + 1];
-    float accp[S::NT][V], accn[S::NT][V];
-#pragma unroll
-    for (int q = 0; q < S::NT; ++q)
-#pragma unroll
-      for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
-    if (SH)
-      row_gather<S, true, false, false, T>(PeerSrc<T, C>{pr}, colind, vals, nullptr, rb, re,
-                                           gmask, sl, a, accp, accn);
-    else
-      row_gather<S, true, false, false, T>(StackedSrc<T, C>{dY, Nt}, colind, vals, nullptr, rb,
-                                           re, gmask, sl, a, accp, accn);
-#pragma unroll
-    for (int q = 0; q < S::NT; ++q) {
-      const int c = (sl + q * S::L) * V;
-#pragma unroll
-      for (int br = 0; br < 2; ++br) {
-        const int64_t row = (int64_t)i + (br ? Nt : 0);
-        float z[V], o[V];
-        Vec<T>::load(Z + row * C + c, z);
-#pragma unroll
-        for (int e = 0; e < V; ++e) {
-          const float h = br ? accn[q][e] : accp[q][e];
-          o[e] = z[e] > 0.f ? h : a * h;
-          da += z[e] > 0.f ? 0.f : h * z[e];
-        }
-        StoreN<T, V>::store(dZ + row * C + c, o);
-      }
-    }
+  if (!BAND) {
+    const int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub;
+    if (i < Nt) bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, pr, gmask, sl, da);
+  } else {
+    const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
+    const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
+    for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
+      bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, pr, gmask, sl, da);
   }
   const double wd = warp_sum((double)da);
-  if (lane == 0) wpart[threadIdx.x >> 5] = wd;
+  if (lane == 0) wpart[w] = wd;
   __syncthreads();
   if (threadIdx.x == 0) {
     double t = 0.0;
-    for (int k = 0; k < kSpmmThreads / 32; ++k) t += wpart[k];
+    for (int k = 0; k < RS::NW; ++k) t += wpart[k];
     slots[blockIdx.x] = t;
   }
+}
+
+int spmm_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (!n) n = 148;
+  }
+  return n;
+}
+
+// Grid of a launch: banded (one block per SM, at most one per 32·RPW rows)
+// for the wide aggregations, blocks of consecutive rows otherwise (layer 1's
+// corrupted branch gathers X[pi[j]] at random, no band locality).
+template <int C, typename T, bool BAND>
+unsigned spmm_blocks(int32_t Nt) {
+  using RS = RowSched<C, T, BAND>;
+  if (!BAND) return cdiv(Nt, RS::RPB);
+  return (unsigned)std::max<int64_t>(1, std::min<int64_t>(spmm_sms(), cdiv(Nt, RS::RPB)));
 }
 
 template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
 cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
                        int act_layer, Tout* Y, cudaStream_t s, const PeerRows& pr) {
-  using S = SpmmShape<C, Tin>;
-  k_spmm_fwd<C, MODE, BOTH, SH, Tin, Tout><<<cdiv(g.Nt, S::RPB), kSpmmThreads, 0, s>>>(
-      g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, pr);
+  constexpr bool BAND = MARS_SPMM_BAND && MODE == 1;
+  k_spmm_fwd<C, MODE, BOTH, SH, BAND, Tin, Tout>
+      <<<spmm_blocks<C, Tin, BAND>(g.Nt), BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
+          g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, pr);
   return cudaGetLastError();
 }
 
@@ -317,19 +407,21 @@ cudaError_t fwd_t(const GraphDev& g, int C, const void* T, const int32_t* perm, 
 template <int C, typename T>
 cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha, int layer,
                   T* dZ, double* slots, int* nslots, cudaStream_t s, const PeerRows* peers) {
-  using S = SpmmShape<C, T>;
-  const unsigned blocks = cdiv(g.Nt, S::RPB);
+  constexpr bool BAND = MARS_SPMM_BAND;
+  const unsigned blocks = spmm_blocks<C, T, BAND>(g.Nt);
+  const unsigned threads = BAND ? kBandThreads : kSpmmThreads;
   *nslots = (int)blocks;
   if constexpr (C == 128 || C == 256) {
     if (peers) {
-      k_spmm_bwd<C, true, T><<<blocks, kSpmmThreads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
-                                                             alpha, layer, g.Nt, dZ, slots, *peers);
+      k_spmm_bwd<C, true, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
+                                                              alpha, layer, g.Nt, dZ, slots, *peers);
       return cudaGetLastError();
     }
   }
   if (peers) return cudaErrorInvalidValue;
-  k_spmm_bwd<C, false, T><<<blocks, kSpmmThreads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z, alpha,
-                                                          layer, g.Nt, dZ, slots, PeerRows{});
+  k_spmm_bwd<C, false, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
+                                                           alpha, layer, g.Nt, dZ, slots,
+                                                           PeerRows{});
   return cudaGetLastError();
 }
 
