@@ -183,7 +183,7 @@ __device__ __forceinline__ double softplus_d(double x) {
 // dl values are broadcast back.
 template <int NC, typename T>
 #ifndef MARS_SCORE_MINB
-#define MARS_SCORE_MINB 3
+#define MARS_SCORE_MINB 2
 #endif
 __global__ void __launch_bounds__(kWarps * 32, MARS_SCORE_MINB)
 k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
@@ -193,7 +193,10 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         double* __restrict__ dv_part, double* __restrict__ loss_part) {
   using RT = RowTile<NC, T>;
   constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER;
-  constexpr int NU = RT::RU >= 4 ? 2 : 1;          // nodes per iteration (2 NU rows)
+#ifndef MARS_SCORE_NU
+#define MARS_SCORE_NU 4     // 8 rows in flight per warp (A/B: profiles/r1s3_spmm_ab.md)
+#endif
+  constexpr int NU = RT::RU >= 4 ? MARS_SCORE_NU : 1;   // nodes per iteration (2 NU rows)
   __shared__ double sh_dv[kWarps][H];
   __shared__ double sh_loss[kWarps];
   const int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -407,6 +410,24 @@ __global__ void __launch_bounds__(1024) k_reduce_slots(const double* __restrict_
   if (threadIdx.x == 0) *out = (float)sh[0];
 }
 
+// Stage 1 of a long slot reduction: block b sums the contiguous range
+// [b·n/NB, (b+1)·n/NB) in a fixed order (per-thread strides, then a tree).
+constexpr int kRedParts = 128;
+__global__ void __launch_bounds__(256) k_reduce_part(const double* __restrict__ slots, int n,
+                                                     double* __restrict__ part) {
+  __shared__ double sh[256];
+  const int64_t b0 = (int64_t)n * blockIdx.x / kRedParts, b1 = (int64_t)n * (blockIdx.x + 1) / kRedParts;
+  double t = 0.0;
+  for (int64_t k = b0 + threadIdx.x; k < b1; k += 256) t += slots[k];
+  sh[threadIdx.x] = t;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (threadIdx.x < o) sh[threadIdx.x] += sh[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) part[blockIdx.x] = sh[0];
+}
+
 template <typename T>
 __global__ void k_prelu(const T* __restrict__ Z, const float* __restrict__ alpha, int layer,
                         float* __restrict__ out, int64_t n) {
@@ -478,7 +499,7 @@ cudaError_t head_t(const GraphDev& g, int H, const void* Z3, const float* M, con
 
 }  // namespace
 
-int head_slots(const GraphDev& g) { return 2 * g.nchunks + 1; }
+int head_slots(const GraphDev& g) { return 2 * g.nchunks + 1 + kRedParts; }   // + reduction scratch
 
 cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, const float* params_M,
                         const float* alpha_dev, const StepParams* sp, const HeadWork& w, void* dZ,
@@ -490,10 +511,15 @@ cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, con
   return head_t<float>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s, hs);
 }
 
-cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
+cudaError_t launch_reduce_slots(double* slots, int n, float* grad, cudaStream_t s,
                                 int* launches) {
-  count_launch(launches);
-  k_reduce_slots<<<1, 1024, 0, s>>>(slots, n, grad);
+  count_launch(launches, n > 8192 ? 2 : 1);
+  if (n > 8192) {   // long slot lists (one per SpMM warp-block): two stages, scratch after them
+    k_reduce_part<<<kRedParts, 256, 0, s>>>(slots, n, slots + n);
+    k_reduce_slots<<<1, 1024, 0, s>>>(slots + n, kRedParts, grad);
+  } else {
+    k_reduce_slots<<<1, 1024, 0, s>>>(slots, n, grad);
+  }
   return cudaGetLastError();
 }
 

@@ -217,7 +217,7 @@ cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16,
                         cudaStream_t s, int* launches, const HeadShard* hs = nullptr);
 int head_slots(const GraphDev& g);
 // grad[0] = Σ slots (fixed order, double)
-cudaError_t launch_reduce_slots(const double* slots, int n, float* grad, cudaStream_t s,
+cudaError_t launch_reduce_slots(double* slots, int n, float* grad, cudaStream_t s,
                                 int* launches);
 // H3 = PReLU(Z3) for the first `rows` rows (encode); Z fp32 or bf16, out fp32
 cudaError_t launch_prelu(const void* Z, int bf16, const float* alpha_dev, int layer, float* out,

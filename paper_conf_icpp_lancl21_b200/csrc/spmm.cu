@@ -28,9 +28,12 @@
 namespace mars {
 namespace {
 
-constexpr int kSpmmThreads = 256;
-#ifndef MARS_SPMM_MINB
-#define MARS_SPMM_MINB 4      // resident 256-thread blocks per SM: caps registers at 64
+#ifndef MARS_SPMM_THREADS
+#define MARS_SPMM_THREADS 32    // one warp per block: a slow (hub) row holds no other warps
+#endif
+constexpr int kSpmmThreads = MARS_SPMM_THREADS;
+#ifndef MARS_SPMM_MINB        // resident blocks per SM: caps registers at 64
+#define MARS_SPMM_MINB (1024 / MARS_SPMM_THREADS < 32 ? 1024 / MARS_SPMM_THREADS : 32)
 #endif
 #ifndef MARS_SPMM_KU
 #define MARS_SPMM_KU 4
@@ -110,7 +113,7 @@ struct PeerSrc {        // row-sharded graph: global row j lives on shard owner(
 // valid row, usually an L1 hit) with weight 0, so the batch needs no branch
 // and its loads stay independent.  Adding 0·x leaves the ascending-order sum
 // unchanged.
-template <class S, int K, bool BOTH, bool ACT, bool PERM, typename T, class Src>
+template <class S, int K, bool BOTH, int ACT, bool PERM, typename T, class Src>
 __device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, int32_t cj,
                                              float cv, int32_t cjn, unsigned gmask, int sl,
                                              float a, float (&accp)[S::NT][S::V],
@@ -125,6 +128,41 @@ __device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, 
     w[u] = __shfl_sync(gmask, cv, lane_u, S::L);
     jn[u] = (PERM && BOTH) ? __shfl_sync(gmask, cjn, lane_u, S::L) : 0;
     if (u >= nvalid) w[u] = 0.f;
+  }
+  if constexpr (ACT == 2) {
+    // PReLU on packed bf16 pairs before widening: max(x, bf16(a·x)), exact
+    // for 0 <= a <= 1 up to the bf16 rounding of a·x (the kernel selects
+    // this form at run time only for such a; bf16 path only)
+    typename Vec<T>::Raw rp[K][S::NT], rn[K][S::NT];
+#pragma unroll
+    for (int u = 0; u < K; ++u)
+#pragma unroll
+      for (int q = 0; q < S::NT; ++q) {
+        const int c = (sl + q * S::L) * V;
+        rp[u][q] = Vec<T>::ld(src.pos(j[u]) + c);
+        if (BOTH) rn[u][q] = Vec<T>::ld(src.neg(j[u], jn[u]) + c);
+      }
+    const __nv_bfloat162 a2 = __float2bfloat162_rn(a);
+    auto hp = [&](uint32_t& wv) {
+      __nv_bfloat162 x = *reinterpret_cast<__nv_bfloat162*>(&wv);
+      x = __hmax2(x, __hmul2(x, a2));
+      wv = *reinterpret_cast<uint32_t*>(&x);
+    };
+#pragma unroll
+    for (int u = 0; u < K; ++u)
+#pragma unroll
+      for (int q = 0; q < S::NT; ++q) {
+        float x[V];
+        hp(rp[u][q].x); hp(rp[u][q].y); hp(rp[u][q].z); hp(rp[u][q].w);
+        Vec<T>::cvt(rp[u][q], x);
+        vfma<V>(accp[q], w[u], x);
+        if (BOTH) {
+          hp(rn[u][q].x); hp(rn[u][q].y); hp(rn[u][q].z); hp(rn[u][q].w);
+          Vec<T>::cvt(rn[u][q], x);
+          vfma<V>(accn[q], w[u], x);
+        }
+      }
+    return;
   }
   float xp[K][S::NT][V], xn[K][S::NT][V];
 #pragma unroll
@@ -153,7 +191,7 @@ __device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, 
 // broadcast by shuffles, then batches of kU neighbours.  MARS_SPMM_TAIL
 // selects the last partial batch: 1 = one padded batch (default), 0 = one
 // neighbour at a time, 2 = a batch of 2 then 1.
-template <class S, bool BOTH, bool ACT, bool PERM, typename T, class Src>
+template <class S, bool BOTH, int ACT, bool PERM, typename T, class Src>
 __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __restrict__ colind,
                                            const float* __restrict__ vals,
                                            const int32_t* __restrict__ perm, int32_t rb,
@@ -192,7 +230,7 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
 // Row bodies shared by the two kernel shapes below.
 // MODE 0: layer 1 (neg rows gather X[perm[j]]), MODE 1: PReLU on load.
 // SH: row-sharded graph (layers 2-3): rows are gathered through PeerSrc.
-template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
+template <int C, int MODE, bool BOTH, bool SH, int ACT, typename Tin, typename Tout>
 __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ rowptr,
                                         const int32_t* __restrict__ colind,
                                         const float* __restrict__ vals, const Tin* __restrict__ T,
@@ -208,14 +246,14 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
 #pragma unroll
     for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
   if (MODE == 0)
-    row_gather<S, BOTH, false, true, Tin>(PermSrc<Tin, C>{T}, colind, vals, perm, rb, re, gmask,
-                                          sl, a, accp, accn);
+    row_gather<S, BOTH, 0, true, Tin>(PermSrc<Tin, C>{T}, colind, vals, perm, rb, re, gmask, sl,
+                                      a, accp, accn);
   else if (SH)
-    row_gather<S, BOTH, true, false, Tin>(PeerSrc<Tin, C>{pr}, colind, vals, perm, rb, re, gmask,
-                                          sl, a, accp, accn);
+    row_gather<S, BOTH, ACT, false, Tin>(PeerSrc<Tin, C>{pr}, colind, vals, perm, rb, re, gmask,
+                                         sl, a, accp, accn);
   else
-    row_gather<S, BOTH, true, false, Tin>(StackedSrc<Tin, C>{T, Nt}, colind, vals, perm, rb, re,
-                                          gmask, sl, a, accp, accn);
+    row_gather<S, BOTH, ACT, false, Tin>(StackedSrc<Tin, C>{T, Nt}, colind, vals, perm, rb, re,
+                                         gmask, sl, a, accp, accn);
 #pragma unroll
   for (int q = 0; q < S::NT; ++q) {
     const int c = (sl + q * S::L) * V;
@@ -296,13 +334,22 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   const float a = (MODE == 1) ? alpha[act_layer] : 1.f;
   if (!BAND) {
     const int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub;
-    if (i < Nt) fwd_row<C, MODE, BOTH, SH>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+    // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
+    if (i < Nt) {
+      if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
+        if (a >= 0.f && a <= 1.f) {
+          fwd_row<C, MODE, BOTH, SH, 2>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+          return;
+        }
+      }
+      fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+    }
     return;
   }
   const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
   const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
   for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-    fwd_row<C, MODE, BOTH, SH>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+    fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
 }
 
 template <int C, bool SH, bool BAND, typename T>
@@ -460,7 +507,8 @@ cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16
 }
 
 // fp32 rows per block is the smallest RPB (largest block count) of any config.
-int spmm_bwd_slots(const GraphDev& g) { return (int)cdiv(g.Nt, SpmmShape<256, float>::RPB) + 1; }
+// (+ 128 doubles of scratch for the two-stage reduction, head.cu)
+int spmm_bwd_slots(const GraphDev& g) { return (int)cdiv(g.Nt, SpmmShape<256, float>::RPB) + 1 + 128; }
 
 cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16_,
                             const float* alpha_dev, int layer, void* dZ, double* slots,
