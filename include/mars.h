@@ -127,10 +127,16 @@ MARS_API mars_status mars_nccl_get_unique_id(void* out128);
 /* Use `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream()) instead
  * of the library stream.  NULL restores the library stream. */
 MARS_API mars_status mars_dgi_set_stream(mars_dgi* m, void* cuda_stream);
-/* Dense-transform implementation (a6/a12).  MARS_GEMM_AUTO (default): tcgen05
- * tensor cores with 3xTF32 splitting (fp32-accurate) when H == 256 and
- * C_in in {64, 128, 256}, FFMA otherwise; MARS_GEMM_SIMT: always FFMA. */
-enum { MARS_GEMM_AUTO = 0, MARS_GEMM_SIMT = 1 };
+/* Dense-transform implementation (a6/a12) of the MARS_FP32 path.
+ * MARS_GEMM_AUTO (default), when H in {128, 256} and C_in in {64, 128, 256}:
+ *   tcgen05 tensor cores at fp32 accuracy -- the row GEMMs (Z = Y·W,
+ *   dY = dZ·Wᵀ) as 3xFP16 with exact power-of-two row / tensor scaling
+ *   (kind::f16, twice the tf32 rate), the weight gradient as 3xTF32;
+ *   FFMA otherwise.
+ * MARS_GEMM_SIMT: always FFMA.
+ * MARS_GEMM_3XTF32: every tensor-core GEMM as 3xTF32 (kind::tf32).
+ * (The MARS_BF16 path always uses its bf16 kernels.) */
+enum { MARS_GEMM_AUTO = 0, MARS_GEMM_SIMT = 1, MARS_GEMM_3XTF32 = 2 };
 MARS_API mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl);
 /* Enables (1) / disables (0) CUDA-Graph capture of the step (default 1). */
 MARS_API mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable);

@@ -32,6 +32,15 @@ __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 // PReLU (c6): slope 1 for z > 0, a otherwise.
 __device__ __forceinline__ float prelu(float z, float a) { return z > 0.f ? z : a * z; }
 
+// 3xFP16 operand scaling (gemm_tc3h.cu): 2^(14 - e), e = floor(log2 m), so
+// m·scale lies in [2^14, 2^15) (below fp16's 65504); 1 for m = 0 or non-finite.
+__device__ __forceinline__ float pow2_scale(float m) {
+  if (!(m > 0.f) || !(m < INFINITY)) return 1.f;
+  const int e = ilogbf(m);
+  const int sh = min(100, max(-100, 14 - e));
+  return ldexpf(1.f, sh);
+}
+
 // Launch counter bump used by every launcher (mars_dgi_last_launches).
 __host__ inline void count_launch(int* launches, int n = 1) {
   if (launches) *launches += n;

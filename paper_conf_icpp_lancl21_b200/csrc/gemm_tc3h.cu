@@ -1,0 +1,408 @@
+// a6 / a12, fp32 path: the row GEMMs of Eq. 1 -- Z_l = Y_l·W_l and
+// dY_l = dZ_l·W_lᵀ -- at fp32 accuracy on the kind::f16 tensor cores, which
+// run at twice the kind::tf32 rate (reading c18: fp32 reference precision).
+//
+// 3xFP16 with exact power-of-two scaling.  Every row r of A is scaled by
+// s_r = 2^(14 - e_r) (e_r = exponent of max_k |A[r][k]|) and the weights by
+// one per-tensor t = 2^(14 - e_W), so every scaled value lies below 2^15 (fp16
+// max 65504) and a value 2^-28 of its row maximum is still a normal fp16.
+// Then x = hi + lo with hi = fp16_rn(x), lo = fp16_rn(x - hi) (x - hi exact in
+// fp32), and D += A_hi·B_hi + A_hi·B_lo + A_lo·B_hi in fp32 TMEM, C = D / (s_r t)
+// (exact).  hi and lo carry 11 significant bits each, like tf32 hi/lo, so the
+// error budget of the 3xTF32 kernel holds: the dropped lo·lo
+// term and the rounding of lo are ~2^-22 relative to the row's scale.
+//
+// k_tc3h_rows: persistent over 128-row tiles.  Warp 0 TMA (fp32 A K-blocks of
+// 32 columns, 128-byte swizzle; pre-split fp16 B hi/lo, 64-byte swizzle),
+// warp 1 MMA issuer, warps 2-5 convert A in place (fp32 tile -> fp16 hi and lo
+// tiles in the UMMA 64-byte-swizzle K-major layout) and compute the next
+// tile's row maxima from global memory while doing so, warps 6-9 epilogue
+// (tcgen05.ld, per-row unscale, 128B-swizzled smem slabs, TMA store).
+#include <cuda_fp16.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+
+#include "common.cuh"
+#include "internal.cuh"
+#include "tc_ptx.cuh"
+
+namespace mars {
+namespace {
+
+using namespace tc;
+
+constexpr int kBM = 128;       // tile rows (UMMA M)
+constexpr int kBK = 32;        // K elements per stage: 128 B of fp32 staging, 64 B of fp16
+constexpr int kThreads = 320;  // 10 warps
+constexpr int kScaleSlots = 8; // per-tile row-scale slots in flight (converters run ahead)
+
+// Instruction descriptor, kind::f16 with fp16 A, B and fp32 D, K-major both.
+__host__ __device__ constexpr uint32_t idesc_f16(int M, int N) {
+  return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+template <int N>
+struct H3Cfg {
+#ifndef MARS_H3_STAGES256
+#define MARS_H3_STAGES256 4
+#endif
+  // N = 256: 4 stages of 48 KB fit with one epilogue slab per warp; else 5
+  static constexpr int kStages = N > 128 ? MARS_H3_STAGES256 : 5;
+  static constexpr int NSLAB = (N > 128 && kStages > 3) ? 1 : 2;
+  static constexpr int A_BYTES = kBM * kBK * 4;      // fp32 staging, later hi | lo (8 KB each)
+  static constexpr int B_BYTES = N * kBK * 2;        // fp16
+  static constexpr int STAGE = A_BYTES + 2 * B_BYTES;
+  static constexpr int SLAB = 32 * 32 * 4;
+  static constexpr int STAGING = 4 * NSLAB * SLAB;
+  static constexpr int SCALES = kScaleSlots * kBM * 4;       // 1 / s_r
+  static constexpr int SMEM = kStages * STAGE + STAGING + SCALES + 1024 + 256;
+  static constexpr uint32_t TMEM_COLS = (2 * N) <= 128 ? 128 : (2 * N) <= 256 ? 256 : 512;
+};
+
+__device__ __forceinline__ void conv_bar() {   // the 4 converter warps
+  asm volatile("bar.sync 1, 128;" ::: "memory");
+}
+
+__device__ __forceinline__ uint32_t pack_h2(float a, float b) {
+  __half2 h = __floats2half2_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+template <int N>
+__global__ void __launch_bounds__(kThreads, 1)
+k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBhi,
+            const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmC,
+            const float* __restrict__ rs, const float* __restrict__ inv_tb, int32_t M, int32_t K) {
+  using Cfg = H3Cfg<N>;
+  constexpr int S = Cfg::kStages;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint8_t* staging = smem + S * Cfg::STAGE;
+  float* rscale = reinterpret_cast<float*>(staging + Cfg::STAGING);     // [slots][128]: 1 / s_r
+  uint64_t* bars = reinterpret_cast<uint64_t*>(staging + Cfg::STAGING + Cfg::SCALES);
+  uint64_t* full = bars;                 // TMA landed              (1 + tx)
+  uint64_t* conv = bars + S;             // A converted             (4 warps)
+  uint64_t* empty = bars + 2 * S;        // MMA done with the stage (commit)
+  uint64_t* tfull = bars + 3 * S;        // accumulator ready       [2]
+  uint64_t* tempty = bars + 3 * S + 2;   // accumulator drained     [2] (4 warps)
+  uint64_t* sready = bars + 3 * S + 4;   // 1 / s_r of a tile published [slots] (4 converter warps)
+  uint64_t* sfree = sready + kScaleSlots;//   ... read by the epilogue     [slots] (4 epilogue warps)
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(sfree + kScaleSlots);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ntiles = (M + kBM - 1) / kBM;
+  const int nk = K / kBK;
+  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stB = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES + Cfg::B_BYTES; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 4);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 4);
+    }
+    for (int b = 0; b < kScaleSlots; ++b) {
+      mbar_init(&sready[b], 4);
+      mbar_init(&sfree[b], 4);
+    }
+    fence_mbar_init();
+    tma_prefetch(&tmA);
+    tma_prefetch(&tmBhi);
+    tma_prefetch(&tmBlo);
+    tma_prefetch(&tmC);
+  }
+  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer
+      int s = 0;
+      uint32_t ph = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x)
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&empty[s], ph ^ 1);
+          mbar_expect_tx(&full[s], Cfg::A_BYTES + 2 * Cfg::B_BYTES);
+          tma_load_2d(stA(s), &tmA, kb * kBK, t * kBM, &full[s]);
+          tma_load_2d(stB(s), &tmBhi, kb * kBK, 0, &full[s]);
+          tma_load_2d(stBlo(s), &tmBlo, kb * kBK, 0, &full[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {                                         // ---- MMA issuer
+      constexpr uint32_t idesc = idesc_f16(kBM, N);
+      int s = 0;
+      uint32_t ph = 0;
+      int acc = 0;
+      uint32_t aph = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        mbar_wait(&tempty[acc], aph ^ 1);
+        tc_fence_after();
+        const uint32_t d = tbase + acc * N;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&conv[s], ph);
+          tc_fence_after();
+          const uint32_t a = smem_u32(stA(s)), al = a + kBM * kBK * 2;
+          const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
+#pragma unroll
+          for (int k = 0; k < kBK / 16; ++k) {
+            // K-major, 64-byte swizzle: rows 64 B apart, 8-row groups 512 B (SBO)
+            const uint64_t ah = sdesc_sw64(a + 32 * k, 16, 512);
+            const uint64_t alo = sdesc_sw64(al + 32 * k, 16, 512);
+            const uint64_t bh = sdesc_sw64(b + 32 * k, 16, 512);
+            const uint64_t blo = sdesc_sw64(bl + 32 * k, 16, 512);
+            mma_f16(d, ah, bh, idesc, (kb | k) != 0);
+            mma_f16(d, ah, blo, idesc, 1);
+            mma_f16(d, alo, bh, idesc, 1);
+          }
+          mma_commit(&empty[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+        mma_commit(&tfull[acc]);
+        acc ^= 1;
+        if (acc == 0) aph ^= 1;
+      }
+    }
+  } else if (warp < 6) {                                     // ---- convert A (row ct per thread)
+    const int ct = threadIdx.x - 64;
+    int s = 0;
+    uint32_t ph = 0;
+    int it = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++it) {
+      const int slot = it % kScaleSlots;
+      const int64_t row = (int64_t)t * kBM + ct;
+      const float scale = row < M ? __ldg(rs + row) : 1.f;  // s_r (power of two) of row ct
+      if (it >= kScaleSlots) mbar_wait(&sfree[slot], ((it / kScaleSlots) - 1) & 1);
+      rscale[slot * kBM + ct] = 1.f / scale;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sready[slot]);
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&full[s], ph);
+        uint8_t* base = stA(s);
+        // read row ct of the fp32 staging tile (128-byte swizzle: chunk j of row r
+        // at r*128 + ((j ^ (r & 7)) << 4)) -> scaled hi / lo halves
+        uint4 hi[kBK / 8], lo[kBK / 8];
+#pragma unroll
+        for (int c = 0; c < kBK / 8; ++c) {
+          float x[8];
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int j = 2 * c + h;
+            const float4 v =
+                *reinterpret_cast<const float4*>(base + ct * 128 + ((j ^ (ct & 7)) << 4));
+            x[4 * h] = v.x * scale;
+            x[4 * h + 1] = v.y * scale;
+            x[4 * h + 2] = v.z * scale;
+            x[4 * h + 3] = v.w * scale;
+          }
+          float xh[8], xl[8];
+#pragma unroll
+          for (int e = 0; e < 8; ++e) {
+            xh[e] = __half2float(__float2half_rn(x[e]));
+            xl[e] = x[e] - xh[e];
+          }
+          hi[c] = make_uint4(pack_h2(xh[0], xh[1]), pack_h2(xh[2], xh[3]), pack_h2(xh[4], xh[5]),
+                             pack_h2(xh[6], xh[7]));
+          lo[c] = make_uint4(pack_h2(xl[0], xl[1]), pack_h2(xl[2], xl[3]), pack_h2(xl[4], xl[5]),
+                             pack_h2(xl[6], xl[7]));
+        }
+        conv_bar();                  // every converter has read its row before any write
+        // hi tile [0, 8 KB), lo tile [8 KB, 16 KB): 64-byte rows, 16-byte chunk c of
+        // row r at r*64 + ((c ^ ((r >> 1) & 3)) << 4)
+#pragma unroll
+        for (int c = 0; c < kBK / 8; ++c) {
+          const int off = ct * 64 + ((c ^ ((ct >> 1) & 3)) << 4);
+          *reinterpret_cast<uint4*>(base + off) = hi[c];
+          *reinterpret_cast<uint4*>(base + kBM * kBK * 2 + off) = lo[c];
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&conv[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp < 10) {                                    // ---- epilogue
+    const int q = warp & 3;
+    int acc = 0;
+    uint32_t aph = 0;
+    const float itb = *inv_tb;
+    uint8_t* slab0 = staging + q * Cfg::NSLAB * Cfg::SLAB;
+    int nslab = 0;
+    int it = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x, ++it) {
+      const int slot = it % kScaleSlots;
+      mbar_wait(&sready[slot], (it / kScaleSlots) & 1);
+      const float f = rscale[slot * kBM + q * 32 + lane] * itb;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sfree[slot]);
+      mbar_wait(&tfull[acc], aph);
+      tc_fence_after();
+#pragma unroll 1
+      for (int c0 = 0; c0 < N; c0 += 32, ++nslab) {
+        uint32_t r[32];
+        tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
+        uint8_t* slab = slab0 + (Cfg::NSLAB == 2 ? (nslab & 1) * Cfg::SLAB : 0);
+        if (lane == 0) {   // the store that last read this slab is done
+          if (Cfg::NSLAB == 2) bulk_wait_read<1>();
+          else bulk_wait_read<0>();
+        }
+        __syncwarp();
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          float4* dst = reinterpret_cast<float4*>(slab + lane * 128 + ((j ^ (lane & 7)) << 4));
+          *dst = make_float4(__uint_as_float(r[4 * j]) * f, __uint_as_float(r[4 * j + 1]) * f,
+                             __uint_as_float(r[4 * j + 2]) * f, __uint_as_float(r[4 * j + 3]) * f);
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_2d(&tmC, slab, c0, t * kBM + q * 32);
+          bulk_commit();
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);
+      acc ^= 1;
+      if (acc == 0) aph ^= 1;
+    }
+    if (lane == 0) bulk_wait<0>();
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tbase, Cfg::TMEM_COLS);
+  }
+}
+
+// ---------------------------------------------------------------- row scales
+// rs[r] = 2^(14 - e_r) of max_k |A[r][k]| (warp per row), for A not produced by
+// a kernel that writes its own row scales.
+__global__ void k_row_scale(const float* __restrict__ A, int64_t M, int K, float* __restrict__ rs) {
+  const int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (r >= M) return;
+  float m = 0.f;
+  for (int k = lane; k < K; k += 32) m = fmaxf(m, fabsf(A[r * K + k]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(kFull, m, o));
+  if (lane == 0) rs[r] = pow2_scale(m);
+}
+
+// ---------------------------------------------------------------- weights
+// max |W| -> 1 / t (one block; W has at most 256 x 256 entries)
+__global__ void __launch_bounds__(1024) k_wscale(const float* __restrict__ W, int n,
+                                                 float* __restrict__ wsc) {
+  __shared__ float sh[32];
+  float m = 0.f;
+  for (int e = threadIdx.x; e < n; e += 1024) m = fmaxf(m, fabsf(W[e]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(kFull, m, o));
+  if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    m = sh[threadIdx.x];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(kFull, m, o));
+    if (threadIdx.x == 0) {
+      const float t = pow2_scale(m);
+      wsc[0] = t;
+      wsc[1] = 1.f / t;
+    }
+  }
+}
+
+// Scaled fp16 hi / lo of Bt = Wᵀ [H × Cin] (forward) and B = W [Cin × H] (dY).
+__global__ void k_split_w3h(const float* __restrict__ W, int CIN, int H,
+                            const float* __restrict__ wsc, __half* __restrict__ Bt_hi,
+                            __half* __restrict__ Bt_lo, __half* __restrict__ B_hi,
+                            __half* __restrict__ B_lo) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;   // e = c * H + h
+  if (e >= (int64_t)CIN * H) return;
+  const int c = (int)(e / H), h = (int)(e % H);
+  const float x = W[e] * wsc[0];
+  const __half hi = __float2half_rn(x);
+  const __half lo = __float2half_rn(x - __half2float(hi));
+  B_hi[e] = hi;
+  B_lo[e] = lo;
+  Bt_hi[(int64_t)h * CIN + c] = hi;
+  Bt_lo[(int64_t)h * CIN + c] = lo;
+}
+
+template <int N>
+cudaError_t rows3h_n(const float* A, const float* rs, const __half* Bhi, const __half* Blo,
+                     const float* inv_tb, float* C, int64_t M, int K, cudaStream_t s) {
+  using Cfg = H3Cfg<N>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_tc3h_rows<N>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap ta, tbh, tbl, tc;
+  if (!tc_tmap(&ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, A, M, K, kBK, kBM,
+               CU_TENSOR_MAP_SWIZZLE_128B) ||
+      !tc_tmap(&tbh, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Bhi, N, K, kBK, N,
+               CU_TENSOR_MAP_SWIZZLE_64B) ||
+      !tc_tmap(&tbl, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Blo, N, K, kBK, N,
+               CU_TENSOR_MAP_SWIZZLE_64B) ||
+      !tc_tmap(&tc, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, C, M, N, 32, 32,
+               CU_TENSOR_MAP_SWIZZLE_128B))
+    return cudaErrorInvalidValue;
+  const int ntiles = (int)((M + kBM - 1) / kBM);
+  const int grid = std::min(ntiles, tc_num_sms());
+  k_tc3h_rows<N><<<grid, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, tc, rs, inv_tb, (int32_t)M, K);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+// wsc[2] = {t, 1/t}; Bt_* [H × CIN], B_* [CIN × H], fp16.
+cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void* Bt_hi,
+                               void* Bt_lo, void* B_hi, void* B_lo, cudaStream_t s,
+                               int* launches) {
+  count_launch(launches, 2);
+  k_wscale<<<1, 1024, 0, s>>>(W, CIN * H, wsc);
+  k_split_w3h<<<cdiv((int64_t)CIN * H, 256), 256, 0, s>>>(
+      W, CIN, H, wsc, static_cast<__half*>(Bt_hi), static_cast<__half*>(Bt_lo),
+      static_cast<__half*>(B_hi), static_cast<__half*>(B_lo));
+  return cudaGetLastError();
+}
+
+cudaError_t tc3h_row_scales(const float* A, int64_t M, int K, float* rs, cudaStream_t s,
+                            int* launches) {
+  count_launch(launches);
+  k_row_scale<<<cdiv(M * 32, 256), 256, 0, s>>>(A, M, K, rs);
+  return cudaGetLastError();
+}
+
+// C[M×N] = A[M×K] · Bᵀ, B = (B_hi + B_lo) / t [N×K] (fp16, scaled by t = 1 / inv_tb[0]),
+// rs[M] = the power-of-two row scales of A (2^(14 - e_r), see k_row_scale).
+cudaError_t tc3h_gemm_rows(const float* A, const float* rs, const void* B_hi, const void* B_lo,
+                           const float* inv_tb, float* C, int64_t M, int N, int K, cudaStream_t s,
+                           int* launches) {
+  count_launch(launches);
+  if (K % kBK || K > 256) return cudaErrorInvalidValue;
+  const __half* bh = static_cast<const __half*>(B_hi);
+  const __half* bl = static_cast<const __half*>(B_lo);
+  switch (N) {
+    case 64: return rows3h_n<64>(A, rs, bh, bl, inv_tb, C, M, K, s);
+    case 128: return rows3h_n<128>(A, rs, bh, bl, inv_tb, C, M, K, s);
+    case 256: return rows3h_n<256>(A, rs, bh, bl, inv_tb, C, M, K, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace mars

@@ -18,6 +18,8 @@
 #include "internal.cuh"
 #include "vec.cuh"
 
+#include <type_traits>
+
 namespace mars {
 namespace {
 
@@ -327,7 +329,7 @@ __global__ void __launch_bounds__(kWarps * 32, 3)
 k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
       const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
       const float* __restrict__ dl, const float* __restrict__ vf, const float* __restrict__ dmf,
-      int32_t Nt, T* __restrict__ dZ, double* __restrict__ slots) {
+      int32_t Nt, T* __restrict__ dZ, double* __restrict__ slots, float* __restrict__ rs) {
   using RT = RowTile<NC, T>;
   constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER, RU = RT::RU;
   __shared__ double wpart[kWarps];
@@ -362,7 +364,8 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
     }
     float daf = 0.f;
 #pragma unroll
-    for (int u = 0; u < RU; ++u)
+    for (int u = 0; u < RU; ++u) {
+      float mx = 0.f;
 #pragma unroll
       for (int q = 0; q < PER; ++q) {
         float o[V], z[V];
@@ -372,9 +375,16 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
           const float dh = fmaf(d[u], vg[q][e], mg[q][e]);
           o[e] = z[e] > 0.f ? dh : a * dh;
           daf += z[e] > 0.f ? 0.f : dh * z[e];
+          mx = fmaxf(mx, act ? fabsf(o[e]) : 0.f);
         }
         if (act && r + u < r1) StoreN<T, V>::store(dZ + (base + r + u) * H + (lane + q * LPR) * V, o);
       }
+      if (rs) {                     // row scale of the stored dZ3 row (3xFP16 dY GEMM)
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(kFull, mx, o));
+        if (lane == 0 && r + u < r1) rs[base + r + u] = pow2_scale(mx);
+      }
+    }
     da += (double)daf;
   }
   da = warp_sum(da);
@@ -477,7 +487,9 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
   k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.gsize, H, w.dm);
   k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
   k_dz3<NC, T><<<dim3(g.nchunks, 2), kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
-                                                          w.dl, w.v, w.dm, g.Nt, dZ, w.slots);
+                                                          w.dl, w.v, w.dm, g.Nt, dZ, w.slots,
+                                                          std::is_same<T, float>::value ? w.rs_dz3
+                                                                                        : nullptr);
   *nslots = 2 * g.nchunks;
   return cudaGetLastError();
 }

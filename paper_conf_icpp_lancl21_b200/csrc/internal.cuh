@@ -140,14 +140,16 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
 cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16,
                             const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
                             int out_bf16, int both, cudaStream_t s, int* launches,
-                            const PeerRows* peers = nullptr);
+                            const PeerRows* peers = nullptr, float* row_scale = nullptr);
+// row_scale (fp32 storage only, may be null): per stored row the power-of-two
+// scale 2^(14 - e) of its max |value| (operand scaling of gemm_tc3h.cu).
 // Backward aggregate dH = Â_n dY (Â_n symmetric) with the PReLU'(Z) epilogue:
 // dZ = dH ⊙ (Z > 0 ? 1 : a), dalpha partials Σ dH·min(Z,0) -> slots[gridDim].
 // dY, Z, dZ share one storage type (bf16 != 0: bf16).
 cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16,
                             const float* alpha_dev, int layer, void* dZ, double* slots,
                             int* nslots, cudaStream_t s, int* launches,
-                            const PeerRows* peers = nullptr);
+                            const PeerRows* peers = nullptr, float* row_scale = nullptr);
 int spmm_bwd_slots(const GraphDev& g);
 
 // ---------------------------------------------------------------- gemm_simt.cu
@@ -171,6 +173,15 @@ cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, f
 size_t tc_dw_partial_floats(int64_t R, int CIN);
 cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN, int H,
                        float* part, cudaStream_t s, int* launches);
+// gemm_tc3h.cu: 3xFP16 row GEMMs with power-of-two scaling (fp32 path)
+cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void* Bt_hi,
+                               void* Bt_lo, void* B_hi, void* B_lo, cudaStream_t s,
+                               int* launches);
+cudaError_t tc3h_gemm_rows(const float* A, const float* rs, const void* B_hi, const void* B_lo,
+                           const float* inv_tb, float* C, int64_t M, int N, int K, cudaStream_t s,
+                           int* launches);
+cudaError_t tc3h_row_scales(const float* A, int64_t M, int K, float* rs, cudaStream_t s,
+                            int* launches);
 bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,
              int64_t rows, int64_t cols, int box_cols, int box_rows, CUtensorMapSwizzle swz);
 int tc_num_sms();
@@ -200,6 +211,7 @@ struct HeadWork {
   float* dl;            // [2*Nt]
   double* loss_g;       // [G] per-graph loss (already / (2 N_g B))
   double* slots;        // [nslots] dalpha3 partials
+  float* rs_dz3;        // [2*Nt] power-of-two row scales of dZ3 (fp32 storage) or null
 };
 // Forward head + head backward: writes grads of M (dM) and the loss slot,
 // dZ3 into dZ, dalpha3 partials into w.slots.

@@ -226,6 +226,11 @@ struct Workspace {
   size_t tn_part_n = 0;
   // tcgen05 path: per-layer hi/lo weight splits (Wᵀ for the forward, W for dY)
   float *wt_hi[3] = {}, *wt_lo[3] = {}, *w_hi[3] = {}, *w_lo[3] = {};
+  // 3xFP16 row GEMMs: scaled fp16 hi/lo splits + {t, 1/t} per layer
+  void *h3_wt_hi[3] = {}, *h3_wt_lo[3] = {}, *h3_w_hi[3] = {}, *h3_w_lo[3] = {};
+  float* h3_wsc[3] = {};
+  float* h3_rsY[3] = {};              // [R] power-of-two row scales of Y_l (written by the SpMM)
+  float* h3_rsdZ = nullptr;           // [R] ... of dZ_l (written by the head / backward SpMM)
   float* dw_part = nullptr;
   // bf16 path: bf16 weight copies (Wᵀ for the forward, W for dY), dW partials.
   // (Activation buffers are sized for fp32 and hold bf16 in that mode.)
@@ -697,7 +702,8 @@ extern "C" mars_status mars_dgi_set_stream(mars_dgi* m, void* stream) {
 
 extern "C" mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl) {
   if (mars_status st = check_dgi(m)) return st;
-  if (impl != MARS_GEMM_AUTO && impl != MARS_GEMM_SIMT) return fail(MARS_EINVAL, "bad gemm impl");
+  if (impl != MARS_GEMM_AUTO && impl != MARS_GEMM_SIMT && impl != MARS_GEMM_3XTF32)
+    return fail(MARS_EINVAL, "bad gemm impl");
   if (impl != m->gemm_impl && m->exec) {
     cudaGraphExecDestroy(m->exec);
     m->exec = nullptr;
@@ -772,7 +778,14 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
     CK(al((void**)&w.wt_lo[l], sizeof(float) * n));
     CK(al((void**)&w.w_hi[l], sizeof(float) * n));
     CK(al((void**)&w.w_lo[l], sizeof(float) * n));
+    CK(al(&w.h3_wt_hi[l], 2 * n));
+    CK(al(&w.h3_wt_lo[l], 2 * n));
+    CK(al(&w.h3_w_hi[l], 2 * n));
+    CK(al(&w.h3_w_lo[l], 2 * n));
+    CK(al((void**)&w.h3_wsc[l], sizeof(float) * 2));
   }
+  for (int l = 0; l < 3; ++l) CK(al((void**)&w.h3_rsY[l], sizeof(float) * R));
+  CK(al((void**)&w.h3_rsdZ, sizeof(float) * R));
   CK(al((void**)&w.dw_part, sizeof(float) * std::max(tc_dw_partial_floats(R, F),
                                                       tc_dw_partial_floats(R, H))));
   if (m->cfg.precision == MARS_BF16) {
@@ -847,10 +860,14 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   MARK(MARS_PH_PERM);
   const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
+  const bool h3 = m->gemm_impl == MARS_GEMM_AUTO;       // 3xFP16 row GEMMs (fp32 path)
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
-    tc[l] = m->gemm_impl == 0 && tc_supported(Cin, H);
+    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
     if (b16) RET(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl));
+    else if (tc[l] && h3)
+      RET(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
+                             w.h3_w_hi[l], w.h3_w_lo[l], s, nl));
     else if (tc[l])
       RET(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, nl));
   }
@@ -864,9 +881,13 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
       MARK(MARS_PH_EXCHANGE);
     }
     RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.perm, alpha, l - 1, Ys[l], b16, 1, s, nl,
-                        shard && l > 0 ? &m->sh.z[l - 1] : nullptr));
+                        shard && l > 0 ? &m->sh.z[l - 1] : nullptr,
+                        tc[l] && h3 ? w.h3_rsY[l] : nullptr));
     MARK(MARS_PH_SPMM_FWD);
     if (b16) RET(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], R, H, Cin, s, nl));
+    else if (tc[l] && h3)
+      RET(tc3h_gemm_rows(Ys[l], w.h3_rsY[l], w.h3_wt_hi[l], w.h3_wt_lo[l], w.h3_wsc[l] + 1,
+                         w.Z[l], R, H, Cin, s, nl));
     else if (tc[l]) RET(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], R, H, Cin, s, nl));
     else RET(gemm_nn(Ys[l], W[l], w.Z[l], R, H, Cin, s, nl));
     MARK(MARS_PH_GEMM_FWD);
@@ -881,6 +902,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     hs.x_peers[0] = m->sh.x[0];
     hs.x_peers[1] = m->sh.x[1];
   }
+  w.hw.rs_dz3 = !b16 && tc[2] && h3 ? w.h3_rsdZ : nullptr;   // dZ3 row scales (3xFP16 dY GEMM)
   RET(launch_head(g, H, w.Z[2], b16, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl,
                   shard ? &hs : nullptr));
   RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
@@ -896,6 +918,9 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
       // sharded: the two backward aggregations use separate peer-visible dY buffers
       float* dYl = (shard && l == 1) ? static_cast<float*>(m->sh.dY2) : w.dY;
       if (b16) RET(tc16_gemm_rows(w.dZ, w.w16[l], dYl, R, Cin, H, s, nl));
+      else if (tc[l] && h3)
+        RET(tc3h_gemm_rows(w.dZ, w.h3_rsdZ, w.h3_w_hi[l], w.h3_w_lo[l], w.h3_wsc[l] + 1, dYl, R,
+                           Cin, H, s, nl));
       else if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], dYl, R, Cin, H, s, nl));
       else RET(gemm_nt(w.dZ, W[l], dYl, R, Cin, H, s, nl));
       MARK(MARS_PH_GEMM_DY);
@@ -904,7 +929,8 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
         MARK(MARS_PH_EXCHANGE);
       }
       RET(launch_spmm_bwd(g, Cin, dYl, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
-                          s, nl, shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr));
+                          s, nl, shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr,
+                          l == 2 && tc[1] && h3 ? w.h3_rsdZ : nullptr));
       MARK(MARS_PH_SPMM_BWD);
       RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
       MARK(MARS_PH_REDUCE);
@@ -1170,11 +1196,18 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     const void* T = l == 0 ? (const void*)gd.X : (const void*)w.Z[l - 1];
-    CK(launch_spmm_fwd(gd, Cin, T, b16 && l > 0, nullptr, alpha, l - 1, Ys[l], b16, 0, s, &nl));
+    const bool h3l = !b16 && m->gemm_impl == MARS_GEMM_AUTO && tc_supported(Cin, H);
+    CK(launch_spmm_fwd(gd, Cin, T, b16 && l > 0, nullptr, alpha, l - 1, Ys[l], b16, 0, s, &nl,
+                       nullptr, h3l ? w.h3_rsY[l] : nullptr));
     if (b16) {
       CK(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, &nl));
       CK(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
-    } else if (m->gemm_impl == 0 && tc_supported(Cin, H)) {
+    } else if (m->gemm_impl == MARS_GEMM_AUTO && tc_supported(Cin, H)) {
+      CK(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
+                            w.h3_w_hi[l], w.h3_w_lo[l], s, &nl));
+      CK(tc3h_gemm_rows(Ys[l], w.h3_rsY[l], w.h3_wt_hi[l], w.h3_wt_lo[l], w.h3_wsc[l] + 1, w.Z[l],
+                        gd.Nt, H, Cin, s, &nl));
+    } else if (m->gemm_impl == MARS_GEMM_3XTF32 && tc_supported(Cin, H)) {
       CK(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, &nl));
       CK(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
     } else {
@@ -1254,8 +1287,12 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
     return fail(MARS_ECUDA, "no CUDA device");
   }
   CK(cudaSetDevice(device));
-  const bool tcp = impl == MARS_GEMM_AUTO && (op == 0 ? tc_supported(K, N) || tc_supported(N, K)
+  const bool tcp = impl != MARS_GEMM_SIMT && (op == 0 ? tc_supported(K, N) || tc_supported(N, K)
                                                      : tc_supported(K, N));
+  const bool h3 = impl == MARS_GEMM_AUTO;
+  float *wsc = nullptr, *rs = nullptr;
+  CK(dalloc(&wsc, 2));
+  CK(dalloc(&rs, (size_t)M));
   size_t nA = (size_t)M * K, nB = op == 0 ? (size_t)N * K : (size_t)M * N;
   size_t nC = op == 0 ? (size_t)M * N : (size_t)K * N;
   float *dA, *dB, *dC, *bh, *bl, *bth, *btl, *part;
@@ -1276,6 +1313,12 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   auto run = [&]() -> cudaError_t {
     if (op == 0) {
+      if (tcp && h3) {   // B [N×K] = "W" with CIN = N, H = K: the dY orientation
+        cudaError_t e = tc3h_split_weights(dB, N, K, wsc, bth, btl, bh, bl, s, nullptr);
+        if (e != cudaSuccess) return e;
+        if ((e = tc3h_row_scales(dA, M, K, rs, s, nullptr)) != cudaSuccess) return e;
+        return tc3h_gemm_rows(dA, rs, bh, bl, wsc + 1, dC, M, N, K, s, nullptr);
+      }
       if (tcp) {
         cudaError_t e = tc_split_weights(dB, N, K, bth, btl, bh, bl, s, nullptr);
         if (e != cudaSuccess) return e;
@@ -1302,7 +1345,7 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   cudaEventDestroy(e1);
   cudaStreamDestroy(s);
   for (void* p : {(void*)dA, (void*)dB, (void*)dC, (void*)bh, (void*)bl, (void*)bth, (void*)btl,
-                  (void*)part, (void*)tpart})
+                  (void*)part, (void*)tpart, (void*)wsc, (void*)rs})
     cudaFree(p);
   return MARS_OK;
 }
@@ -1522,7 +1565,7 @@ extern "C" mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g) {
   if (m->sh.g) return fail(MARS_ESTATE, "model already attached to a shard");
   if (m->comm) return fail(MARS_EINVAL, "a shard-attached model cannot also be data-parallel");
   if (g->F != m->F || g->device != m->cfg.device) return fail(MARS_EINVAL, "F / device mismatch");
-  if (!(m->H == 128 || m->H == 256) || m->gemm_impl != MARS_GEMM_AUTO)
+  if (!(m->H == 128 || m->H == 256) || m->gemm_impl == MARS_GEMM_SIMT)
     return fail(MARS_EINVAL, "row sharding needs hidden_dim in {128, 256} and the tcgen05 GEMMs");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;

@@ -227,6 +227,21 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
   }
 }
 
+// Power-of-two row scale (gemm_tc3h.cu) of one stored row held by the L lanes
+// of a row group: max |x| over the group, lane 0 of the group writes it.
+template <class S, int NV>
+__device__ __forceinline__ void row_scale_out(const float (&x)[S::NT][NV], unsigned gmask, int sl,
+                                              float* __restrict__ dst) {
+  float m = 0.f;
+#pragma unroll
+  for (int q = 0; q < S::NT; ++q)
+#pragma unroll
+    for (int e = 0; e < NV; ++e) m = fmaxf(m, fabsf(x[q][e]));
+#pragma unroll
+  for (int o = S::L / 2; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gmask, m, o));
+  if (sl == 0) *dst = pow2_scale(m);
+}
+
 // Row bodies shared by the two kernel shapes below.
 // MODE 0: layer 1 (neg rows gather X[perm[j]]), MODE 1: PReLU on load.
 // SH: row-sharded graph (layers 2-3): rows are gathered through PeerSrc.
@@ -235,8 +250,8 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
                                         const int32_t* __restrict__ colind,
                                         const float* __restrict__ vals, const Tin* __restrict__ T,
                                         const int32_t* __restrict__ perm, float a, int32_t Nt,
-                                        Tout* __restrict__ Y, const PeerRows& pr, unsigned gmask,
-                                        int sl) {
+                                        Tout* __restrict__ Y, float* __restrict__ rs,
+                                        const PeerRows& pr, unsigned gmask, int sl) {
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
@@ -260,6 +275,10 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
     StoreN<Tout, V>::store(Y + (int64_t)i * C + c, accp[q]);
     if (BOTH) StoreN<Tout, V>::store(Y + ((int64_t)Nt + i) * C + c, accn[q]);
   }
+  if (rs) {                          // fp32 storage: row scales for the 3xFP16 GEMM
+    row_scale_out<S>(accp, gmask, sl, rs + i);
+    if (BOTH) row_scale_out<S>(accn, gmask, sl, rs + Nt + i);
+  }
 }
 
 template <int C, bool SH, typename T>
@@ -267,8 +286,8 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
                                         const int32_t* __restrict__ colind,
                                         const float* __restrict__ vals, const T* __restrict__ dY,
                                         const T* __restrict__ Z, float a, int32_t Nt,
-                                        T* __restrict__ dZ, const PeerRows& pr, unsigned gmask,
-                                        int sl, float& da) {
+                                        T* __restrict__ dZ, float* __restrict__ rs,
+                                        const PeerRows& pr, unsigned gmask, int sl, float& da) {
   using S = SpmmShape<C, T>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
@@ -283,22 +302,27 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
   else
     row_gather<S, true, false, false, T>(StackedSrc<T, C>{dY, Nt}, colind, vals, nullptr, rb, re,
                                          gmask, sl, a, accp, accn);
+  float o[2][S::NT][V];
 #pragma unroll
   for (int q = 0; q < S::NT; ++q) {
     const int c = (sl + q * S::L) * V;
 #pragma unroll
     for (int br = 0; br < 2; ++br) {
       const int64_t row = (int64_t)i + (br ? Nt : 0);
-      float z[V], o[V];
+      float z[V];
       Vec<T>::load(Z + row * C + c, z);
 #pragma unroll
       for (int e = 0; e < V; ++e) {
         const float h = br ? accn[q][e] : accp[q][e];
-        o[e] = z[e] > 0.f ? h : a * h;
+        o[br][q][e] = z[e] > 0.f ? h : a * h;
         da += z[e] > 0.f ? 0.f : h * z[e];
       }
-      StoreN<T, V>::store(dZ + row * C + c, o);
+      StoreN<T, V>::store(dZ + row * C + c, o[br][q]);
     }
+  }
+  if (rs) {
+    row_scale_out<S>(o[0], gmask, sl, rs + i);
+    row_scale_out<S>(o[1], gmask, sl, rs + Nt + i);
   }
 }
 
@@ -325,7 +349,8 @@ __global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 :
 k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const Tin* __restrict__ T,
            const int32_t* __restrict__ perm, const float* __restrict__ alpha, int act_layer,
-           int32_t Nt, Tout* __restrict__ Y, const __grid_constant__ PeerRows pr) {
+           int32_t Nt, Tout* __restrict__ Y, float* __restrict__ rs,
+           const __grid_constant__ PeerRows pr) {
   using S = SpmmShape<C, Tin>;
   using RS = RowSched<C, Tin, BAND>;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -338,18 +363,18 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
     if (i < Nt) {
       if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
         if (a >= 0.f && a <= 1.f) {
-          fwd_row<C, MODE, BOTH, SH, 2>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+          fwd_row<C, MODE, BOTH, SH, 2>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
           return;
         }
       }
-      fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+      fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
     }
     return;
   }
   const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
   const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
   for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-    fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, pr, gmask, sl);
+    fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
 }
 
 template <int C, bool SH, bool BAND, typename T>
@@ -357,7 +382,8 @@ __global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 :
 k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const T* __restrict__ dY, const T* __restrict__ Z,
            const float* __restrict__ alpha, int layer, int32_t Nt, T* __restrict__ dZ,
-           double* __restrict__ slots, const __grid_constant__ PeerRows pr) {
+           double* __restrict__ slots, float* __restrict__ rs,
+           const __grid_constant__ PeerRows pr) {
   using S = SpmmShape<C, T>;
   using RS = RowSched<C, T, BAND>;
   __shared__ double wpart[RS::NW];
@@ -368,12 +394,12 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   float da = 0.f;
   if (!BAND) {
     const int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub;
-    if (i < Nt) bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, pr, gmask, sl, da);
+    if (i < Nt) bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
   } else {
     const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
     const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
     for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-      bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, pr, gmask, sl, da);
+      bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
   }
   const double wd = warp_sum((double)da);
   if (lane == 0) wpart[w] = wd;
@@ -408,52 +434,54 @@ unsigned spmm_blocks(int32_t Nt) {
 
 template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
 cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
-                       int act_layer, Tout* Y, cudaStream_t s, const PeerRows& pr) {
+                       int act_layer, Tout* Y, float* rs, cudaStream_t s, const PeerRows& pr) {
   constexpr bool BAND = MARS_SPMM_BAND && MODE == 1;
   k_spmm_fwd<C, MODE, BOTH, SH, BAND, Tin, Tout>
       <<<spmm_blocks<C, Tin, BAND>(g.Nt), BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
-          g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, pr);
+          g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, rs, pr);
   return cudaGetLastError();
 }
 
 template <int C, typename Tin, typename Tout>
 cudaError_t fwd_c(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
-                  int act_layer, Tout* Y, int both, cudaStream_t s, const PeerRows* peers) {
+                  int act_layer, Tout* Y, float* rs, int both, cudaStream_t s,
+                  const PeerRows* peers) {
   const PeerRows none{};
   if (act_layer < 0) {
     if (peers) return cudaErrorInvalidValue;    // layer 1 reads the replicated X
-    return both ? fwd_launch<C, 0, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none)
-                : fwd_launch<C, 0, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none);
+    return both ? fwd_launch<C, 0, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, none)
+                : fwd_launch<C, 0, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, none);
   }
   if constexpr ((C == 128 || C == 256) && std::is_same<Tin, Tout>::value) {
     if (peers) {
       if (!both) return cudaErrorInvalidValue;
-      return fwd_launch<C, 1, true, true, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, *peers);
+      return fwd_launch<C, 1, true, true, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, *peers);
     }
   }
   if (peers) return cudaErrorInvalidValue;
-  return both ? fwd_launch<C, 1, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none)
-              : fwd_launch<C, 1, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, s, none);
+  return both ? fwd_launch<C, 1, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, none)
+              : fwd_launch<C, 1, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, none);
 }
 
 template <typename Tin, typename Tout>
 cudaError_t fwd_t(const GraphDev& g, int C, const void* T, const int32_t* perm, const float* alpha,
-                  int act_layer, void* Y, int both, cudaStream_t s, const PeerRows* pr) {
+                  int act_layer, void* Y, float* rs, int both, cudaStream_t s, const PeerRows* pr) {
   const Tin* t = static_cast<const Tin*>(T);
   Tout* y = static_cast<Tout*>(Y);
   switch (C) {
-    case 16: return fwd_c<16, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
-    case 32: return fwd_c<32, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
-    case 64: return fwd_c<64, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
-    case 128: return fwd_c<128, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
-    case 256: return fwd_c<256, Tin, Tout>(g, t, perm, alpha, act_layer, y, both, s, pr);
+    case 16: return fwd_c<16, Tin, Tout>(g, t, perm, alpha, act_layer, y, rs, both, s, pr);
+    case 32: return fwd_c<32, Tin, Tout>(g, t, perm, alpha, act_layer, y, rs, both, s, pr);
+    case 64: return fwd_c<64, Tin, Tout>(g, t, perm, alpha, act_layer, y, rs, both, s, pr);
+    case 128: return fwd_c<128, Tin, Tout>(g, t, perm, alpha, act_layer, y, rs, both, s, pr);
+    case 256: return fwd_c<256, Tin, Tout>(g, t, perm, alpha, act_layer, y, rs, both, s, pr);
     default: return cudaErrorInvalidValue;
   }
 }
 
 template <int C, typename T>
 cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha, int layer,
-                  T* dZ, double* slots, int* nslots, cudaStream_t s, const PeerRows* peers) {
+                  T* dZ, double* slots, int* nslots, float* rs, cudaStream_t s,
+                  const PeerRows* peers) {
   constexpr bool BAND = MARS_SPMM_BAND;
   const unsigned blocks = spmm_blocks<C, T, BAND>(g.Nt);
   const unsigned threads = BAND ? kBandThreads : kSpmmThreads;
@@ -461,29 +489,29 @@ cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha
   if constexpr (C == 128 || C == 256) {
     if (peers) {
       k_spmm_bwd<C, true, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
-                                                              alpha, layer, g.Nt, dZ, slots, *peers);
+                                                              alpha, layer, g.Nt, dZ, slots, rs, *peers);
       return cudaGetLastError();
     }
   }
   if (peers) return cudaErrorInvalidValue;
   k_spmm_bwd<C, false, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
-                                                           alpha, layer, g.Nt, dZ, slots,
+                                                           alpha, layer, g.Nt, dZ, slots, rs,
                                                            PeerRows{});
   return cudaGetLastError();
 }
 
 template <typename T>
 cudaError_t bwd_t(const GraphDev& g, int C, const void* dY, const void* Z, const float* alpha,
-                  int layer, void* dZ, double* slots, int* nslots, cudaStream_t s,
+                  int layer, void* dZ, double* slots, int* nslots, float* rs, cudaStream_t s,
                   const PeerRows* pr) {
   const T* d = static_cast<const T*>(dY);
   const T* z = static_cast<const T*>(Z);
   T* o = static_cast<T*>(dZ);
   switch (C) {
-    case 32: return bwd_c<32, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
-    case 64: return bwd_c<64, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
-    case 128: return bwd_c<128, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
-    case 256: return bwd_c<256, T>(g, d, z, alpha, layer, o, slots, nslots, s, pr);
+    case 32: return bwd_c<32, T>(g, d, z, alpha, layer, o, slots, nslots, rs, s, pr);
+    case 64: return bwd_c<64, T>(g, d, z, alpha, layer, o, slots, nslots, rs, s, pr);
+    case 128: return bwd_c<128, T>(g, d, z, alpha, layer, o, slots, nslots, rs, s, pr);
+    case 256: return bwd_c<256, T>(g, d, z, alpha, layer, o, slots, nslots, rs, s, pr);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -495,14 +523,14 @@ cudaError_t bwd_t(const GraphDev& g, int C, const void* dY, const void* Z, const
 cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16,
                             const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
                             int out_bf16, int both, cudaStream_t s, int* launches,
-                            const PeerRows* peers) {
+                            const PeerRows* peers, float* rs) {
   count_launch(launches);
   if (!in_bf16 && !out_bf16)
-    return fwd_t<float, float>(g, C, T, perm, alpha_dev, act_layer, Y, both, s, peers);
+    return fwd_t<float, float>(g, C, T, perm, alpha_dev, act_layer, Y, rs, both, s, peers);
   if (!in_bf16 && out_bf16)
-    return fwd_t<float, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, both, s, peers);
+    return fwd_t<float, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, nullptr, both, s, peers);
   if (in_bf16 && out_bf16)
-    return fwd_t<bf16, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, both, s, peers);
+    return fwd_t<bf16, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, nullptr, both, s, peers);
   return cudaErrorInvalidValue;
 }
 
@@ -512,10 +540,11 @@ int spmm_bwd_slots(const GraphDev& g) { return (int)cdiv(g.Nt, SpmmShape<256, fl
 
 cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16_,
                             const float* alpha_dev, int layer, void* dZ, double* slots,
-                            int* nslots, cudaStream_t s, int* launches, const PeerRows* peers) {
+                            int* nslots, cudaStream_t s, int* launches, const PeerRows* peers,
+                            float* rs) {
   count_launch(launches);
-  if (bf16_) return bwd_t<bf16>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, s, peers);
-  return bwd_t<float>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, s, peers);
+  if (bf16_) return bwd_t<bf16>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, nullptr, s, peers);
+  return bwd_t<float>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, rs, s, peers);
 }
 
 }  // namespace mars

@@ -341,8 +341,9 @@ class DGI:
         _check(lib().mars_dgi_set_stream(self.handle, stream_ptr))
 
     def set_gemm_impl(self, impl: str):
-        """'auto' (tcgen05 3xTF32 where supported) or 'simt' (FFMA everywhere)."""
-        _check(lib().mars_dgi_set_gemm_impl(self.handle, {"auto": 0, "simt": 1}[impl]))
+        """'auto' (tcgen05: 3xFP16 row GEMMs, 3xTF32 weight gradient, where
+        supported), 'simt' (FFMA everywhere) or '3xtf32' (every tcgen05 GEMM 3xTF32)."""
+        _check(lib().mars_dgi_set_gemm_impl(self.handle, GEMM_IMPLS[impl]))
 
     def set_graph_capture(self, enable: bool):
         _check(lib().mars_dgi_set_graph_capture(self.handle, 1 if enable else 0))
@@ -442,6 +443,9 @@ def dgi_export_activations(m: DGI, layer: int):
     return Y, Z
 
 
+GEMM_IMPLS = {"auto": 0, "simt": 1, "3xtf32": 2}   # MARS_GEMM_* (include/mars.h)
+
+
 def debug_gemm(op: str, A, B, impl: str = "auto", iters: int = 0, device: int = 0):
     """mars_debug_gemm: op 'rows' -> A[M×K]·Bᵀ (B [N×K]); op 'dw' -> Aᵀ·B (A [M×K],
     B [M×N]).  Returns (C, mean ms per launch)."""
@@ -455,7 +459,7 @@ def debug_gemm(op: str, A, B, impl: str = "auto", iters: int = 0, device: int = 
         N = B.shape[1]
         C = np.zeros((K, N), np.float32)
     ms = ctypes.c_float()
-    _check(lib().mars_debug_gemm(device, 0 if op == "rows" else 1, {"auto": 0, "simt": 1}[impl],
+    _check(lib().mars_debug_gemm(device, 0 if op == "rows" else 1, GEMM_IMPLS[impl],
                                  _ptr(A), _ptr(B), _ptr(C), M, N, K, iters, ctypes.byref(ms)))
     return C, ms.value
 

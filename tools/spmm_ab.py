@@ -24,6 +24,8 @@ def child(path):
     out = {}
     for prec in (M.MARS_FP32, M.MARS_BF16):
         m = M.dgi_create(in_dim=64, hidden_dim=256, seed=0, precision=prec)
+        if os.environ.get("MARS_AB_GEMM"):
+            m.set_gemm_impl(os.environ["MARS_AB_GEMM"])
         for k in range(3):
             m.step(g, k, 0)
         runs = [m.profile_step(g, 10 + k, 0) for k in range(7)]
@@ -53,4 +55,5 @@ if __name__ == "__main__":
             ph = d[prec]
             print(f"{os.path.basename(p):28s} {prec}  spmm_fwd {ph.get('spmm_fwd', 0):.4f}  "
                   f"spmm_bwd {ph.get('spmm_bwd', 0):.4f}  head {ph.get('head', 0):.4f}  "
-                  f"total {sum(ph.values()):.4f}", flush=True)
+                  f"gemm_fwd {ph.get('gemm_fwd', 0):.4f}  gemm_dy {ph.get('gemm_dy', 0):.4f}  "
+                  f"gemm_dw {ph.get('gemm_dw', 0):.4f}  total {sum(ph.values()):.4f}", flush=True)
