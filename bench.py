@@ -305,25 +305,48 @@ def run_mine(args):
     spmm_gbs = spmm_algo / (spmm_ms / 1e3) / 1e9 if spmm_ms else None
     shares = {k: v / sum(per_step.values()) for k, v in per_step.items()}
     step_total = sum(per_step.values())
-    gemm_ms = sum(per_step.get(k, 0) for k in ("gemm_fwd", "gemm_dw", "gemm_dy"))
+    rows_ms = per_step.get("gemm_fwd", 0) + per_step.get("gemm_dy", 0)
+    dw_ms = per_step.get("gemm_dw", 0)
     head_ms = per_step.get("head", 0)
-    fl = sum(gflops.values())
-    # 3xTF32: three tf32 MMAs per fp32 product, so the fp32-equivalent tensor
-    # peak is the tf32 peak / 3; tf32 = bf16 x (1.1 / 2.25) nominal ratio.
-    tf32_peak = pk["bf16_tflops"] * (1.1 / 2.25)
-    gemm_peak = tf32_peak / 3.0 if args.gemm == "auto" else pk["ffma_tflops"]
-    gemm_ach = fl / (gemm_ms / 1e3) / 1e12 if gemm_ms else None
+    auto = args.gemm == "auto"
+    # Row GEMMs (Z = Y·W, dY = dZ·Wᵀ): 3xFP16 on kind::f16 -- fp32-equivalent
+    # tensor peak bf16 / 3 = ~540 TF/s, ridge ~83 flop/B above their 64 flop/B
+    # (fp32 operands), so HBM bounds them: algorithmic bytes R·(K+N)·4 per GEMM.
+    rows_bytes = gbytes["gemm_fwd"] + gbytes["gemm_dy"]
+    rows_flops = gflops["gemm_fwd"] + gflops["gemm_dy"]
+    rows_gbs = rows_bytes / (rows_ms / 1e3) / 1e9 if rows_ms else None
+    # Weight gradient (dW = Yᵀ·dZ): 3xFP16 as well, same intensity (<= 64 flop/B
+    # against the ~83 flop/B ridge), so also HBM-bound: R·(Cin+H)·4 per GEMM.
+    dw_bytes = gbytes["gemm_dw"]
+    dw_gbs = dw_bytes / (dw_ms / 1e3) / 1e9 if dw_ms else None
+    dw_ach = gflops["gemm_dw"] / (dw_ms / 1e3) / 1e12 if dw_ms else None
     head_bytes = 16 * N * H                     # Z3 in, dZ3 out (stacked pos/neg)
     head_gbs = head_bytes / (head_ms / 1e3) / 1e9 if head_ms else None
+    if auto:
+        gemm_rows = {"kernel": "row GEMMs Z = Y·W, dY = dZ·Wᵀ (tcgen05 3xFP16, k_tc3h_rows)",
+                     "bound": "hbm", "achieved": rows_gbs, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                     "frac": rows_gbs / pk["hbm_gbs"] if rows_gbs else None, "traffic": None,
+                     "peak_source": pk["source"], "algorithmic_bytes_per_step": rows_bytes,
+                     "achieved_tflops_fp32_equiv": rows_flops / (rows_ms / 1e3) / 1e12 if rows_ms else None,
+                     "share_of_step": rows_ms / step_total}
+    else:
+        ach = rows_flops / (rows_ms / 1e3) / 1e12 if rows_ms else None
+        gemm_rows = {"kernel": "row GEMMs (FFMA)", "bound": "alu", "achieved": ach,
+                     "peak": pk["ffma_tflops"], "unit": "TFLOP/s",
+                     "frac": ach / pk["ffma_tflops"] if ach else None, "traffic": None,
+                     "peak_source": FFMA_TFLOPS_NOTE, "share_of_step": rows_ms / step_total}
     rooflines = {
-        "gemm": {"kernel": "dense transforms (Z = Y·W, dY = dZ·Wᵀ, dW = Yᵀ·dZ), "
-                           + ("tcgen05 3xTF32" if args.gemm == "auto" else "FFMA"),
-                 "bound": "tensor" if args.gemm == "auto" else "alu", "achieved": gemm_ach,
-                 "peak": gemm_peak, "unit": "TFLOP/s",
-                 "frac": gemm_ach / gemm_peak if gemm_ach else None, "traffic": None,
-                 "peak_source": ("measured bf16 x 1.1/2.25 (tf32) / 3 (3xTF32), fp32-equivalent"
-                                 if args.gemm == "auto" else FFMA_TFLOPS_NOTE),
-                 "algorithmic_flops_per_step": fl, "share_of_step": gemm_ms / step_total},
+        "gemm_rows": gemm_rows,
+        "gemm_dw": ({"kernel": "weight gradient dW = Yᵀ·dZ (tcgen05 3xFP16, k_tc3h_dw)",
+                     "bound": "hbm", "achieved": dw_gbs, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                     "frac": dw_gbs / pk["hbm_gbs"] if dw_gbs else None, "traffic": None,
+                     "peak_source": pk["source"], "algorithmic_bytes_per_step": dw_bytes,
+                     "achieved_tflops_fp32_equiv": dw_ach, "share_of_step": dw_ms / step_total}
+                    if auto else
+                    {"kernel": "weight gradient dW = Yᵀ·dZ (FFMA)", "bound": "alu",
+                     "achieved": dw_ach, "peak": pk["ffma_tflops"], "unit": "TFLOP/s",
+                     "frac": dw_ach / pk["ffma_tflops"] if dw_ach else None, "traffic": None,
+                     "peak_source": FFMA_TFLOPS_NOTE, "share_of_step": dw_ms / step_total}),
         "spmm": {"kernel": "spmm (fwd x3 + bwd x2)", "bound": "hbm", "achieved": spmm_gbs,
                  "peak": pk["hbm_gbs"], "unit": "GB/s",
                  "frac": spmm_gbs / pk["hbm_gbs"] if spmm_gbs else None, "traffic": None,
@@ -333,7 +356,8 @@ def run_mine(args):
                  "frac": head_gbs / pk["hbm_gbs"] if head_gbs else None, "traffic": None,
                  "peak_source": pk["source"], "share_of_step": head_ms / step_total},
     }
-    algo_bytes = {"gemm": sum(gbytes.values()), "spmm": spmm_algo, "head": head_bytes}
+    algo_bytes = {"gemm_rows": rows_bytes, "gemm_dw": gbytes["gemm_dw"], "spmm": spmm_algo,
+                  "head": head_bytes}
     for grp, r in rooflines.items():
         t = ncu_traffic("fp32", grp)
         if t is not None:
@@ -372,18 +396,28 @@ def run_mine(args):
         m2.step(gg, 0, base, B, want_loss=True)
         gg.free()
         torch.cuda.synchronize()
+        # Pipelined like a data loader: step k is enqueued (mars_dgi_step returns
+        # without waiting when no output is requested), then the NEXT batch's
+        # H2D copy + CSR build run on libmars's loader stream (copy engines and a
+        # few small kernels) while step k computes, then step k's loss is read
+        # back (D2H).  Every step's inputs are still copied inside the timed region.
         t0 = time.perf_counter()
+        gg = mars.graph_load(pinned, device=local)
         for k in range(ke):
-            gg = mars.graph_load(pinned, device=local)
-            m2.step(gg, 1 + k, base, B, want_loss=True)
+            m2.step(gg, 1 + k, base, B)
+            nxt = mars.graph_load(pinned, device=local) if k + 1 < ke else None
+            loss_k, _ = m2.read_step(want_grads=False)
             gg.free()
+            gg = nxt
         torch.cuda.synchronize()
         dt = time.perf_counter() - t0
         m2.free()
         e2e = {"value": b * ke / dt, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": 4, "steps": ke,
-               "note": "per step: mars_graph_load (H2D + CSR build) + mars_dgi_step + loss D2H, "
-                       "wall clock, rank-local (no allreduce)"}
+               "note": "per step: mars_graph_load (H2D from pinned host memory + CSR build on "
+                       "libmars's loader stream, overlapping the previous step's compute) + "
+                       "mars_dgi_step + loss D2H (mars_dgi_read_step); wall clock, rank-local "
+                       "(no allreduce)"}
 
     # the bf16 path (MARS_BF16, 2e-2 parity bar) on the same workload, same timing
     b16 = None
@@ -483,7 +517,7 @@ def main():
     ap.add_argument("--graphs-per-gpu", type=int, default=None)
     ap.add_argument("--seed", type=int, default=0)
     ap.add_argument("--gemm", default="auto", choices=["auto", "simt"],
-                    help="dense-transform kernels: tcgen05 3xTF32 (auto) or FFMA (simt)")
+                    help="dense-transform kernels: tcgen05 3xFP16 with power-of-two scaling (auto) or FFMA (simt)")
     ap.add_argument("--profile-steps", type=int, default=5)
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--no-e2e", action="store_true")

@@ -33,8 +33,11 @@ __device__ __forceinline__ int lane_id() { return threadIdx.x & 31; }
 __device__ __forceinline__ float prelu(float z, float a) { return z > 0.f ? z : a * z; }
 
 // 3xFP16 operand scaling (gemm_tc3h.cu): 2^(14 - e), e = floor(log2 m), so
-// m·scale lies in [2^14, 2^15) (below fp16's 65504); 1 for m = 0 or non-finite.
+// m·scale lies in [2^14, 2^15) (below fp16's 65504); 1 for non-finite m.
+// An all-zero row gets the largest scale 2^100 (its products stay 0, and a
+// min-reduction over row scales -- k_tc3h_dw -- is not pulled down by it).
 __device__ __forceinline__ float pow2_scale(float m) {
+  if (m == 0.f) return 0x1p100f;
   if (!(m > 0.f) || !(m < INFINITY)) return 1.f;
   const int e = ilogbf(m);
   const int sh = min(100, max(-100, 14 - e));

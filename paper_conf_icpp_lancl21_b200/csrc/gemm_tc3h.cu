@@ -69,6 +69,22 @@ __device__ __forceinline__ uint32_t pack_h2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
+// x = hi + lo for 8 scaled values: hi = fp16_rn(x) (packed in pairs), read
+// back as fp32 to form lo = x - hi exactly, lo rounded to fp16.
+__device__ __forceinline__ void split_h8(const float (&x)[8], uint4& hi, uint4& lo) {
+  uint32_t hw[4], lw[4];
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const __half2 h2 = __floats2half2_rn(x[2 * k], x[2 * k + 1]);
+    const float2 hf = __half22float2(h2);
+    const __half2 l2 = __floats2half2_rn(x[2 * k] - hf.x, x[2 * k + 1] - hf.y);
+    hw[k] = *reinterpret_cast<const uint32_t*>(&h2);
+    lw[k] = *reinterpret_cast<const uint32_t*>(&l2);
+  }
+  hi = make_uint4(hw[0], hw[1], hw[2], hw[3]);
+  lo = make_uint4(lw[0], lw[1], lw[2], lw[3]);
+}
+
 template <int N>
 __global__ void __launch_bounds__(kThreads, 1)
 k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBhi,
@@ -204,16 +220,7 @@ k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUt
             x[4 * h + 2] = v.z * scale;
             x[4 * h + 3] = v.w * scale;
           }
-          float xh[8], xl[8];
-#pragma unroll
-          for (int e = 0; e < 8; ++e) {
-            xh[e] = __half2float(__float2half_rn(x[e]));
-            xl[e] = x[e] - xh[e];
-          }
-          hi[c] = make_uint4(pack_h2(xh[0], xh[1]), pack_h2(xh[2], xh[3]), pack_h2(xh[4], xh[5]),
-                             pack_h2(xh[6], xh[7]));
-          lo[c] = make_uint4(pack_h2(xl[0], xl[1]), pack_h2(xl[2], xl[3]), pack_h2(xl[4], xl[5]),
-                             pack_h2(xl[6], xl[7]));
+          split_h8(x, hi[c], lo[c]);
         }
         conv_bar();                  // every converter has read its row before any write
         // hi tile [0, 8 KB), lo tile [8 KB, 16 KB): 64-byte rows, 16-byte chunk c of
@@ -367,6 +374,280 @@ cudaError_t rows3h_n(const float* A, const float* rs, const __half* Bhi, const _
   return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- k_tc3h_dw
+// dW partials per row chunk, 3xFP16: D[h][c] += Σ_r dZ[r][h]·Y[r][c] with both
+// operands MN-major (row-major activations, reduction over rows, no
+// transpose).  Scaling: one power of two per CTA and operand, the smallest row
+// scale of its chunk (min_r rs[r], rs written by the producing kernels), so
+// the chunk's largest |value| maps into [2^14, 2^15); the partial is unscaled
+// (exactly) before it is written.  TMA brings fp32 row tiles (boxes of 32
+// columns x 16 rows, 128-byte swizzle); converter warps 2..11 write scaled fp16
+// hi / lo tiles in the MN-major 128B-swizzle layout (64-column atoms, 8-row
+// groups); warps 4..11 also fold the 128-row TMEM work runs into an fp32
+// register master (as k_tc_dw2: bounded tensor-core accumulation runs).
+constexpr int kDwBK = 16;        // rows per stage = one K = 16 MMA step
+constexpr int kDwStages = 4;
+constexpr int kDwSub = 8;        // stages per TMEM work run (128 rows)
+
+template <int CINT, int HH>
+struct H3DwCfg {
+  static constexpr int NH = HH / 128;                 // 128-row halves of H (UMMA M)
+  static constexpr int BOX32 = 32 * kDwBK * 4;        // fp32 TMA box: 32 cols x 16 rows = 2 KB
+  static constexpr int ATOM = 64 * kDwBK * 2;         // fp16 MN atom column: 64 cols x 16 rows
+  static constexpr int A32 = (HH / 32) * BOX32;
+  static constexpr int B32 = (CINT / 32) * BOX32;
+  static constexpr int A16 = (HH / 64) * ATOM;
+  static constexpr int B16 = (CINT / 64) * ATOM;
+  static constexpr int STAGE = A32 + B32 + 2 * A16 + 2 * B16;
+  static constexpr int SMEM = kDwStages * STAGE + 1024 + 512;
+  static constexpr uint32_t TMEM_COLS = 2 * NH * CINT;
+  static constexpr int MCOLS = CINT / 2;              // columns per folding thread per half
+};
+
+__device__ __forceinline__ void dwconv_bar() {      // converter warps 2..11
+  asm volatile("bar.sync 2, 320;" ::: "memory");
+}
+
+template <int CINT, int HH>
+__global__ void __launch_bounds__(384, 1)
+k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
+          const float* __restrict__ rs_dz, const float* __restrict__ rs_y,
+          float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN) {
+  using Cfg = H3DwCfg<CINT, HH>;
+  constexpr int NH = Cfg::NH;
+  constexpr int S = kDwStages;
+  constexpr int MC = Cfg::MCOLS;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;
+  uint64_t* conv = bars + S;
+  uint64_t* empty = bars + 2 * S;
+  uint64_t* tfull = bars + 3 * S;        // [2]
+  uint64_t* tempty = bars + 3 * S + 2;   // [2]
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 4);
+  float* wmin = reinterpret_cast<float*>(bars + 3 * S + 6);   // [2][10] per-warp minima
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ntile = CIN / CINT;
+  const int chunk = blockIdx.x / ntile, c_off = (blockIdx.x % ntile) * CINT;
+  const int32_t r0 = chunk * rows_per_chunk;
+  const int32_t r1 = min(R, r0 + rows_per_chunk);
+  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
+  const int nsub = (nk + kDwSub - 1) / kDwSub;
+  auto stA32 = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stB32 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32; };
+  auto stA16 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32 + Cfg::B32; };  // hi, lo
+  auto stB16 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32 + Cfg::B32 + 2 * Cfg::A16; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 10);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 8);
+    }
+    fence_mbar_init();
+    tma_prefetch(&tmDZ);
+    tma_prefetch(&tmY);
+  }
+  if (warp == 1) tmem_alloc(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer
+      int s = 0;
+      uint32_t ph = 0;
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], Cfg::A32 + Cfg::B32);
+        const int32_t row = r0 + kb * kDwBK;
+#pragma unroll
+        for (int bx = 0; bx < HH / 32; ++bx)
+          tma_load_2d(stA32(s) + bx * Cfg::BOX32, &tmDZ, bx * 32, row, &full[s]);
+#pragma unroll
+        for (int bx = 0; bx < CINT / 32; ++bx)
+          tma_load_2d(stB32(s) + bx * Cfg::BOX32, &tmY, c_off + bx * 32, row, &full[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {                                         // ---- MMA issuer
+      constexpr uint32_t idesc = idesc_f16(kBM, CINT) | (1u << 15) | (1u << 16);   // MN-major
+      int s = 0;
+      uint32_t ph = 0;
+      for (int sub = 0; sub < nsub; ++sub) {
+        const int buf = sub & 1;
+        mbar_wait(&tempty[buf], ((sub >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t twork = tbase + buf * NH * CINT;
+        const int kb1 = min(nk, (sub + 1) * kDwSub);
+        for (int kb = sub * kDwSub; kb < kb1; ++kb) {
+          mbar_wait(&conv[s], ph);
+          tc_fence_after();
+          const uint32_t a = smem_u32(stA16(s)), al = a + Cfg::A16;
+          const uint32_t b = smem_u32(stB16(s)), bl = b + Cfg::B16;
+          // MN-major fp16, 128B swizzle: 8-row atoms (1 KB, SBO), 64-column
+          // blocks one atom column apart (LBO); one MMA (K = 16) spans two atoms
+          const uint64_t bh = sdesc_sw128(b, Cfg::ATOM, 1024);
+          const uint64_t blo = sdesc_sw128(bl, Cfg::ATOM, 1024);
+          const uint32_t first = kb == sub * kDwSub ? 0u : 1u;
+#pragma unroll
+          for (int h = 0; h < NH; ++h) {
+            const uint64_t ah = sdesc_sw128(a + h * 2 * Cfg::ATOM, Cfg::ATOM, 1024);
+            const uint64_t alo = sdesc_sw128(al + h * 2 * Cfg::ATOM, Cfg::ATOM, 1024);
+            const uint32_t d = twork + h * CINT;
+            mma_f16(d, ah, bh, idesc, first);
+            mma_f16(d, ah, blo, idesc, 1);
+            mma_f16(d, alo, bh, idesc, 1);
+          }
+          mma_commit(&empty[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+        mma_commit(&tfull[buf]);
+      }
+    }
+  } else {                         // ---- convert (warps 2..11); warps 4..11 also fold
+    const bool folder = warp >= 4;
+    const int ct = (warp - 2) * 32 + lane;
+    constexpr int NT = 10 * 32;
+    // chunk scales: min over the chunk's row scales of each operand
+    float mz = INFINITY, my = INFINITY;
+    for (int32_t r = r0 + ct; r < r1; r += NT) {
+      mz = fminf(mz, __ldg(rs_dz + r));
+      my = fminf(my, __ldg(rs_y + r));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      mz = fminf(mz, __shfl_xor_sync(kFull, mz, o));
+      my = fminf(my, __shfl_xor_sync(kFull, my, o));
+    }
+    if (lane == 0) {
+      wmin[warp - 2] = mz;
+      wmin[10 + warp - 2] = my;
+    }
+    dwconv_bar();
+    float sz = INFINITY, sy = INFINITY;
+#pragma unroll
+    for (int k = 0; k < 10; ++k) {
+      sz = fminf(sz, wmin[k]);
+      sy = fminf(sy, wmin[10 + k]);
+    }
+    if (!(sz < INFINITY)) sz = 1.f;          // empty chunk
+    if (!(sy < INFINITY)) sy = 1.f;
+
+    const int q = warp & 3, ch = (warp - 4) >> 2;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    float master[NH][MC];
+#pragma unroll
+    for (int h = 0; h < NH; ++h)
+#pragma unroll
+      for (int j = 0; j < MC; ++j) master[h][j] = 0.f;
+    int folded = 0;
+    auto fold = [&](int sub) {
+      const int buf = sub & 1;
+      mbar_wait(&tfull[buf], (sub >> 1) & 1);
+      tc_fence_after();
+      const uint32_t twork = tbase + buf * NH * CINT + ch * MC;
+#pragma unroll
+      for (int h = 0; h < NH; ++h)
+#pragma unroll
+        for (int c0 = 0; c0 < MC; c0 += 32) {
+          uint32_t w[32];
+          tmem_ld32(twork + lane_off + h * CINT + c0, w);
+          tmem_wait_ld();
+#pragma unroll
+          for (int j = 0; j < 32; ++j) master[h][c0 + j] += __uint_as_float(w[j]);
+        }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[buf]);
+    };
+    constexpr int NTA = kDwBK * HH / 8;                 // 8-column tasks of dZ per stage
+    constexpr int NTT = NTA + kDwBK * CINT / 8;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int kb = 0; kb < nk; ++kb) {
+      mbar_wait(&full[s], ph);
+      for (int i = ct; i < NTT; i += NT) {
+        const bool isA = i < NTA;
+        const int ii = isA ? i : i - NTA;
+        const int r = ii % kDwBK, c0 = (ii / kDwBK) * 8;
+        const uint8_t* src = (isA ? stA32(s) : stB32(s)) + (c0 / 32) * Cfg::BOX32 + r * 128;
+        const int w0 = (c0 % 32) / 4;
+        const float4 v0 = *reinterpret_cast<const float4*>(src + ((w0 ^ (r & 7)) << 4));
+        const float4 v1 = *reinterpret_cast<const float4*>(src + (((w0 + 1) ^ (r & 7)) << 4));
+        const float sc = isA ? sz : sy;
+        const float x[8] = {v0.x * sc, v0.y * sc, v0.z * sc, v0.w * sc,
+                            v1.x * sc, v1.y * sc, v1.z * sc, v1.w * sc};
+        uint4 hv, lv;
+        split_h8(x, hv, lv);
+        uint8_t* dst = (isA ? stA16(s) : stB16(s)) + (c0 / 64) * Cfg::ATOM + r * 128 +
+                       ((((c0 % 64) / 8) ^ (r & 7)) << 4);
+        *reinterpret_cast<uint4*>(dst) = hv;
+        *reinterpret_cast<uint4*>(dst + (isA ? Cfg::A16 : Cfg::B16)) = lv;
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&conv[s]);
+      if (++s == S) { s = 0; ph ^= 1; }
+      if (folder && (kb % kDwSub) == kDwSub / 2 && kb / kDwSub >= 1) fold(folded++);
+    }
+    if (folder) {
+      while (folded < nsub) fold(folded++);
+      const float inv = 1.f / (sz * sy);                   // exact (powers of two)
+      float* out = part + (int64_t)chunk * HH * CIN + c_off + ch * MC;
+#pragma unroll
+      for (int h = 0; h < NH; ++h) {
+        float4* dst = reinterpret_cast<float4*>(out + (int64_t)(h * 128 + q * 32 + lane) * CIN);
+#pragma unroll
+        for (int j = 0; j < MC / 4; ++j)
+          dst[j] = make_float4(master[h][4 * j] * inv, master[h][4 * j + 1] * inv,
+                               master[h][4 * j + 2] * inv, master[h][4 * j + 3] * inv);
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tbase, Cfg::TMEM_COLS);
+  }
+}
+
+__global__ void k_dw3h_reduce(const float* __restrict__ part, int nchunk, int CIN, int H,
+                              float* __restrict__ dW) {
+  dw_reduce_body(part, nchunk, CIN, H, dW);
+}
+
+template <int CINT, int HH>
+cudaError_t dw3h_c(const float* Y, const float* rs_y, const float* dZ, const float* rs_dz,
+                   float* part, int nchunk, int64_t R, int rows, int CIN, cudaStream_t s) {
+  using Cfg = H3DwCfg<CINT, HH>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_tc3h_dw<CINT, HH>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap tdz, ty;
+  if (!tc_tmap(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, HH, 32, kDwBK,
+               CU_TENSOR_MAP_SWIZZLE_128B) ||
+      !tc_tmap(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, CIN, 32, kDwBK,
+               CU_TENSOR_MAP_SWIZZLE_128B))
+    return cudaErrorInvalidValue;
+  k_tc3h_dw<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part,
+                                                                   (int32_t)R, rows, CIN);
+  return cudaGetLastError();
+}
+
 }  // namespace
 
 // wsc[2] = {t, 1/t}; Bt_* [H × CIN], B_* [CIN × H], fp16.
@@ -403,6 +684,31 @@ cudaError_t tc3h_gemm_rows(const float* A, const float* rs, const void* B_hi, co
     case 256: return rows3h_n<256>(A, rs, bh, bl, inv_tb, C, M, K, s);
     default: return cudaErrorInvalidValue;
   }
+}
+
+// dW [CIN × H] = Yᵀ dZ, Y [R × CIN], dZ [R × H] (H in {128, 256}), with the
+// power-of-two row scales rs_y / rs_dz of both operands (see k_tc3h_dw).
+cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, const float* rs_dz,
+                         float* dW, int64_t R, int CIN, int H, float* part, cudaStream_t s,
+                         int* launches) {
+  count_launch(launches, 2);
+  int nchunk = tc_dw_chunks(R, CIN);
+  int rows = (int)((R + nchunk - 1) / nchunk);
+  rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
+  nchunk = (int)((R + rows - 1) / rows);
+  cudaError_t e;
+  if (H != 128 && H != 256) return cudaErrorInvalidValue;
+  switch (CIN) {
+    case 64: e = H == 256 ? dw3h_c<64, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s)
+                          : dw3h_c<64, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s); break;
+    case 128:
+    case 256: e = H == 256 ? dw3h_c<128, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s)
+                           : dw3h_c<128, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s); break;
+    default: return cudaErrorInvalidValue;
+  }
+  if (e != cudaSuccess) return e;
+  k_dw3h_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
+  return cudaGetLastError();
 }
 
 }  // namespace mars

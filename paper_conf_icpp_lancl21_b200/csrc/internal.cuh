@@ -180,6 +180,10 @@ cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void*
 cudaError_t tc3h_gemm_rows(const float* A, const float* rs, const void* B_hi, const void* B_lo,
                            const float* inv_tb, float* C, int64_t M, int N, int K, cudaStream_t s,
                            int* launches);
+cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, const float* rs_dz,
+                         float* dW, int64_t R, int CIN, int H, float* part, cudaStream_t s,
+                         int* launches);
+int tc_dw_chunks(int64_t R, int CIN);
 cudaError_t tc3h_row_scales(const float* A, int64_t M, int K, float* rs, cudaStream_t s,
                             int* launches);
 bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,

@@ -911,6 +911,8 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   for (int l = 2; l >= 0; --l) {
     int Cin = l == 0 ? F : H;
     if (b16) RET(tc16_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, H, w.dw16_part, s, nl));
+    else if (tc[l] && h3)
+      RET(tc3h_gemm_dw(Ys[l], w.h3_rsY[l], w.dZ, w.h3_rsdZ, gW[l], R, Cin, H, w.dw_part, s, nl));
     else if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, H, w.dw_part, s, nl));
     else RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
     MARK(MARS_PH_GEMM_DW);
@@ -930,7 +932,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
       }
       RET(launch_spmm_bwd(g, Cin, dYl, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
                           s, nl, shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr,
-                          l == 2 && tc[1] && h3 ? w.h3_rsdZ : nullptr));
+                          tc[l - 1] && h3 ? w.h3_rsdZ : nullptr));
       MARK(MARS_PH_SPMM_BWD);
       RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
       MARK(MARS_PH_REDUCE);
@@ -1290,9 +1292,10 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   const bool tcp = impl != MARS_GEMM_SIMT && (op == 0 ? tc_supported(K, N) || tc_supported(N, K)
                                                      : tc_supported(K, N));
   const bool h3 = impl == MARS_GEMM_AUTO;
-  float *wsc = nullptr, *rs = nullptr;
+  float *wsc = nullptr, *rs = nullptr, *rs2 = nullptr;
   CK(dalloc(&wsc, 2));
   CK(dalloc(&rs, (size_t)M));
+  CK(dalloc(&rs2, (size_t)M));
   size_t nA = (size_t)M * K, nB = op == 0 ? (size_t)N * K : (size_t)M * N;
   size_t nC = op == 0 ? (size_t)M * N : (size_t)K * N;
   float *dA, *dB, *dC, *bh, *bl, *bth, *btl, *part;
@@ -1326,6 +1329,12 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
       }
       return gemm_nt(dA, dB, dC, M, N, K, s, nullptr);
     }
+    if (tcp && h3) {
+      cudaError_t e = tc3h_row_scales(dA, M, K, rs, s, nullptr);
+      if (e != cudaSuccess) return e;
+      if ((e = tc3h_row_scales(dB, M, N, rs2, s, nullptr)) != cudaSuccess) return e;
+      return tc3h_gemm_dw(dA, rs, dB, rs2, dC, M, K, N, part, s, nullptr);
+    }
     if (tcp) return tc_gemm_dw(dA, dB, dC, M, K, N, part, s, nullptr);
     return gemm_tn(dA, dB, dC, M, K, N, tpart, s, nullptr);
   };
@@ -1345,7 +1354,7 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   cudaEventDestroy(e1);
   cudaStreamDestroy(s);
   for (void* p : {(void*)dA, (void*)dB, (void*)dC, (void*)bh, (void*)bl, (void*)bth, (void*)btl,
-                  (void*)part, (void*)tpart, (void*)wsc, (void*)rs})
+                  (void*)part, (void*)tpart, (void*)wsc, (void*)rs, (void*)rs2})
     cudaFree(p);
   return MARS_OK;
 }
