@@ -573,6 +573,24 @@ bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void*
                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// Row-major [rows × cols] matrix viewed as 3-D {128-byte column block, rows,
+// column blocks}: one box {128 B, box_rows, nblk} lands as nblk consecutive
+// [box_rows × 128 B] blocks with the 128-byte swizzle -- e.g. the MN-major
+// 128B-swizzle atom columns of the UMMA layout -- in a single TMA request.
+bool tc_tmap_blocks(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,
+                    int64_t rows, int64_t cols, int box_rows, int nblk) {
+  if (!encode_fn()) return false;
+  const cuuint64_t bc = 128 / elem_bytes;            // columns per 128-byte block
+  cuuint64_t dims[3] = {bc, (cuuint64_t)rows, (cuuint64_t)(cols / bc)};
+  cuuint64_t strides[2] = {(cuuint64_t)cols * elem_bytes, 128};
+  cuuint32_t box[3] = {(cuuint32_t)bc, (cuuint32_t)box_rows, (cuuint32_t)nblk};
+  cuuint32_t es[3] = {1, 1, 1};
+  return g_encode(m, dt, 3, const_cast<void*>(base), dims, strides, box, es,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) ==
+         CUDA_SUCCESS;
+}
+
 int tc_num_sms() { return num_sms(); }
 
 bool tc_supported(int K_or_cin, int N_or_h) {

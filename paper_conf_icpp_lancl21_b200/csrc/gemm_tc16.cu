@@ -172,6 +172,9 @@ k_tc16_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUt
 }
 
 // ---------------------------------------------------------------- k_tc16_dw
+#ifndef MARS_DW16_3D
+#define MARS_DW16_3D 1   // one 3-D TMA box per operand and stage (vs one per 64-column atom)
+#endif
 constexpr int kDwBK = 16;        // rows per stage (one K = 16 MMA)
 constexpr int kDwStages = 8;
 constexpr int kSubKb = 8;        // stages per TMEM work run (128 rows)
@@ -242,12 +245,18 @@ k_tc16_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
         mbar_wait(&empty[s], ph ^ 1);
         mbar_expect_tx(&full[s], Cfg::A_BYTES + Cfg::B_BYTES);
         const int32_t row = r0 + kb * kDwBK;
+#if MARS_DW16_3D
+        // one 3-D box per operand: all 64-column atom columns of the stage
+        tma_load_3d(stA(s), &tmDZ, 0, row, 0, &full[s]);
+        tma_load_3d(stB(s), &tmY, 0, row, c_off / 64, &full[s]);
+#else
 #pragma unroll
         for (int bx = 0; bx < HH / 64; ++bx)
           tma_load_2d(stA(s) + bx * Cfg::BOX, &tmDZ, bx * 64, row, &full[s]);
 #pragma unroll
         for (int bx = 0; bx < CINT / 64; ++bx)
           tma_load_2d(stB(s) + bx * Cfg::BOX, &tmY, c_off + bx * 64, row, &full[s]);
+#endif
         if (++s == S) { s = 0; ph ^= 1; }
       }
     }
@@ -388,8 +397,14 @@ cudaError_t dw16_c(const void* Y, const void* dZ, float* part, int nchunk, int64
     attr = true;
   }
   CUtensorMap tdz, ty;
+#if MARS_DW16_3D
+  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, dZ, R, HH, kDwBK, HH / 64) ||
+      !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, Y, R, CIN, kDwBK, CINT / 64))
+    return cudaErrorInvalidValue;
+#else
   if (!tmap16(&tdz, dZ, R, HH, 64, kDwBK) || !tmap16(&ty, Y, R, CIN, 64, kDwBK))
     return cudaErrorInvalidValue;
+#endif
   k_tc16_dw<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, part, (int32_t)R, rows,
                                                                CIN);
   return cudaGetLastError();

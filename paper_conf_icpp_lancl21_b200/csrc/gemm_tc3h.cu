@@ -380,8 +380,9 @@ cudaError_t rows3h_n(const float* A, const float* rs, const __half* Bhi, const _
 // transpose).  Scaling: one power of two per CTA and operand, the smallest row
 // scale of its chunk (min_r rs[r], rs written by the producing kernels), so
 // the chunk's largest |value| maps into [2^14, 2^15); the partial is unscaled
-// (exactly) before it is written.  TMA brings fp32 row tiles (boxes of 32
-// columns x 16 rows, 128-byte swizzle); converter warps 2..11 write scaled fp16
+// (exactly) before it is written.  TMA brings fp32 row tiles (one 3-D box of
+// 16 rows x all 32-column 128B-swizzled blocks per operand and stage);
+// converter warps 2..11 write scaled fp16
 // hi / lo tiles in the MN-major 128B-swizzle layout (64-column atoms, 8-row
 // groups); warps 4..11 also fold the 128-row TMEM work runs into an fp32
 // register master (as k_tc_dw2: bounded tensor-core accumulation runs).
@@ -392,8 +393,8 @@ constexpr int kDwSub = 8;        // stages per TMEM work run (128 rows)
 template <int CINT, int HH>
 struct H3DwCfg {
   static constexpr int NH = HH / 128;                 // 128-row halves of H (UMMA M)
-  static constexpr int BOX32 = 32 * kDwBK * 4;        // fp32 TMA box: 32 cols x 16 rows = 2 KB
   static constexpr int ATOM = 64 * kDwBK * 2;         // fp16 MN atom column: 64 cols x 16 rows
+  static constexpr int BOX32 = 32 * kDwBK * 4;        // one 32-column fp32 block: 16 rows x 128 B
   static constexpr int A32 = (HH / 32) * BOX32;
   static constexpr int B32 = (CINT / 32) * BOX32;
   static constexpr int A16 = (HH / 64) * ATOM;
@@ -468,12 +469,10 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
         mbar_wait(&empty[s], ph ^ 1);
         mbar_expect_tx(&full[s], Cfg::A32 + Cfg::B32);
         const int32_t row = r0 + kb * kDwBK;
-#pragma unroll
-        for (int bx = 0; bx < HH / 32; ++bx)
-          tma_load_2d(stA32(s) + bx * Cfg::BOX32, &tmDZ, bx * 32, row, &full[s]);
-#pragma unroll
-        for (int bx = 0; bx < CINT / 32; ++bx)
-          tma_load_2d(stB32(s) + bx * Cfg::BOX32, &tmY, c_off + bx * 32, row, &full[s]);
+        // one 3-D box per operand: all 32-column (128-byte, swizzled) blocks of
+        // the stage in a single TMA request
+        tma_load_3d(stA32(s), &tmDZ, 0, row, 0, &full[s]);
+        tma_load_3d(stB32(s), &tmY, 0, row, c_off / 32, &full[s]);
         if (++s == S) { s = 0; ph ^= 1; }
       }
     }
@@ -638,10 +637,8 @@ cudaError_t dw3h_c(const float* Y, const float* rs_y, const float* dZ, const flo
     attr = true;
   }
   CUtensorMap tdz, ty;
-  if (!tc_tmap(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, HH, 32, kDwBK,
-               CU_TENSOR_MAP_SWIZZLE_128B) ||
-      !tc_tmap(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, CIN, 32, kDwBK,
-               CU_TENSOR_MAP_SWIZZLE_128B))
+  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, HH, kDwBK, HH / 32) ||
+      !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, CIN, kDwBK, CINT / 32))
     return cudaErrorInvalidValue;
   k_tc3h_dw<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part,
                                                                    (int32_t)R, rows, CIN);

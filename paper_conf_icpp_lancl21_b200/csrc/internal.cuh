@@ -189,6 +189,8 @@ cudaError_t tc3h_row_scales(const float* A, int64_t M, int K, float* rs, cudaStr
 bool tc_tmap(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,
              int64_t rows, int64_t cols, int box_cols, int box_rows, CUtensorMapSwizzle swz);
 int tc_num_sms();
+bool tc_tmap_blocks(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, const void* base,
+                    int64_t rows, int64_t cols, int box_rows, int nblk);
 
 // ---------------------------------------------------------------- gemm_tc16.cu
 // bf16 path (MARS_BF16): one kind::f16 MMA per k-step, bf16 operands, fp32

@@ -10,7 +10,7 @@ sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from ncu_table import rows  # noqa: E402
 
 GROUPS = {"gemm_rows": ("k_tc3h_rows", "k_tc_rows", "k_tc16_rows"),
-          "gemm_dw": ("k_tc_dw2", "k_tc16_dw"),
+          "gemm_dw": ("k_tc3h_dw", "k_tc_dw2", "k_tc16_dw"),
           "spmm": ("k_spmm_fwd", "k_spmm_bwd"),
           "head": ("k_colsum", "k_score", "k_dz3")}
 
