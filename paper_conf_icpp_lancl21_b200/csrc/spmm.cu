@@ -104,6 +104,9 @@ struct PeerSrc {        // row-sharded graph: global row j lives on shard owner(
   }
 };
 
+#ifndef MARS_SPMM_PERSIST
+#define MARS_SPMM_PERSIST 0   // > 0: resident grid of PERSIST waves of MINB blocks per SM
+#endif
 #ifndef MARS_SPMM_TAIL
 #define MARS_SPMM_TAIL 1
 #endif
@@ -358,13 +361,15 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
   const float a = (MODE == 1) ? alpha[act_layer] : 1.f;
   if (!BAND) {
-    const int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub;
-    // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
-    if (i < Nt) {
+    // MARS_SPMM_PERSIST: a resident grid walks rows i, i + gridDim·RPB, ...
+    // (no per-row block launches); otherwise one launch block per RPB rows
+    const int32_t step = MARS_SPMM_PERSIST ? (int32_t)gridDim.x * RS::RPB : Nt;
+    for (int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub; i < Nt; i += step) {
+      // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
       if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
         if (a >= 0.f && a <= 1.f) {
           fwd_row<C, MODE, BOTH, SH, 2>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
-          return;
+          continue;
         }
       }
       fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
@@ -393,8 +398,9 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   const float a = alpha[layer];
   float da = 0.f;
   if (!BAND) {
-    const int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub;
-    if (i < Nt) bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
+    const int32_t step = MARS_SPMM_PERSIST ? (int32_t)gridDim.x * RS::RPB : Nt;
+    for (int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub; i < Nt; i += step)
+      bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
   } else {
     const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
     const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
@@ -428,6 +434,10 @@ int spmm_sms() {
 template <int C, typename T, bool BAND>
 unsigned spmm_blocks(int32_t Nt) {
   using RS = RowSched<C, T, BAND>;
+  if (!BAND && MARS_SPMM_PERSIST)
+    return (unsigned)std::max<int64_t>(
+        1, std::min<int64_t>((int64_t)spmm_sms() * MARS_SPMM_MINB * MARS_SPMM_PERSIST,
+                             cdiv(Nt, RS::RPB)));
   if (!BAND) return cdiv(Nt, RS::RPB);
   return (unsigned)std::max<int64_t>(1, std::min<int64_t>(spmm_sms(), cdiv(Nt, RS::RPB)));
 }
