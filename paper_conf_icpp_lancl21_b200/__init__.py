@@ -5,6 +5,7 @@ package holds it and a thin ctypes binding (``mars.py``) with the ABI's names.
 It never imports ``oracle/`` and has no CPU fallback.
 """
 from .mars import (DGI, Graph, MarsError, MARS_BF16, MARS_FP32, PHASES, config_default,  # noqa: F401
+                   corruption_samples,
                    debug_gemm, dgi_create, dgi_export_activations, dgi_step, encode, free,
                    graph_export_csr, graph_load, graph_load_shard, graph_shard_info, lib,
                    nccl_get_unique_id, num_params, shard_attach, shard_connect,

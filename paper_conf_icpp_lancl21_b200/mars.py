@@ -188,6 +188,18 @@ class Graph:
             pass
 
 
+def corruption_samples(graphs, K: int):
+    """K corruption samples per graph (DESIGN.md reading
+    c20): each graph repeated K times consecutively, so with global_batch =
+    K·len(graphs) pair g·K + k draws its own permutation and the step's loss is
+    1/(2N)[Σ softplus(-l_i) + (1/K) Σ_k Σ_i softplus(l~_i^k)] per graph -- the
+    positive branch weighted once, each corruption sample 1/K (the positive
+    branch is recomputed per sample)."""
+    if K < 1:
+        raise ValueError("K >= 1")
+    return [g for g in graphs for _ in range(K)]
+
+
 def graph_load(graphs, device: int = 0) -> Graph:
     """mars_graph_load: graphs = iterable of objects with num_nodes, indptr (int64
     [N+1]), indices (int32), features (float32 [N, F])."""
