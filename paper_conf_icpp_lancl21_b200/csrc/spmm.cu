@@ -245,6 +245,41 @@ __device__ __forceinline__ void row_scale_out(const float (&x)[S::NT][NV], unsig
   if (sl == 0) *dst = pow2_scale(m);
 }
 
+#ifndef MARS_SPMM_PF
+#define MARS_SPMM_PF (3 << 20)   // L2-prefetch distance in bytes of one branch's rows (0: off)
+#endif
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+
+// Streams the inputs of row i + PF into L2 ahead of its block (PF = 3 MB of
+// one branch's rows: 3072 rows of 1 KB, 6144 of 512 B; measured, r1s3_spmm_ab.md): its
+// own source rows (pos + neg -- also the first-touch gathers of its
+// neighbours) now, and its colind / vals lines once its rowptr entry (loaded
+// now, used at the end of this row) has arrived.
+template <typename T, int C, bool NEG>
+__device__ __forceinline__ int32_t prefetch_rows_ahead(int32_t i, int32_t Nt,
+                                                       const int32_t* rowptr, const T* base,
+                                                       int sl) {
+  constexpr int PF = MARS_SPMM_PF / (C * (int)sizeof(T));
+  const int32_t ip = i + PF;
+  if (PF <= 0 || ip >= Nt) return -1;
+  constexpr int LINES = (C * (int)sizeof(T) + 127) / 128;    // 128-byte lines per branch row
+  if (sl < LINES) {
+    prefetch_l2(reinterpret_cast<const char*>(base + (int64_t)ip * C) + sl * 128);
+    if (NEG) prefetch_l2(reinterpret_cast<const char*>(base + ((int64_t)Nt + ip) * C) + sl * 128);
+  }
+  return __ldg(rowptr + ip);
+}
+__device__ __forceinline__ void prefetch_csr_ahead(int32_t rp, const int32_t* colind,
+                                                   const float* vals, int sl) {
+  if (MARS_SPMM_PF <= 0 || rp < 0) return;
+  if (sl == 0) {
+    prefetch_l2(colind + rp);
+    prefetch_l2(vals + rp);
+  }
+}
+
 // Row bodies shared by the two kernel shapes below.
 // MODE 0: layer 1 (neg rows gather X[perm[j]]), MODE 1: PReLU on load.
 // SH: row-sharded graph (layers 2-3): rows are gathered through PeerSrc.
@@ -258,6 +293,8 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
+  const int32_t rp_ahead =
+      SH ? -1 : prefetch_rows_ahead<Tin, C, MODE == 1 && BOTH>(i, Nt, rowptr, T, sl);
   float accp[S::NT][V], accn[S::NT][V];
 #pragma unroll
   for (int q = 0; q < S::NT; ++q)
@@ -278,6 +315,7 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
     StoreN<Tout, V>::store(Y + (int64_t)i * C + c, accp[q]);
     if (BOTH) StoreN<Tout, V>::store(Y + ((int64_t)Nt + i) * C + c, accn[q]);
   }
+  prefetch_csr_ahead(rp_ahead, colind, vals, sl);
   if (rs) {                          // fp32 storage: row scales for the 3xFP16 GEMM
     row_scale_out<S>(accp, gmask, sl, rs + i);
     if (BOTH) row_scale_out<S>(accn, gmask, sl, rs + Nt + i);
@@ -294,6 +332,11 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
   using S = SpmmShape<C, T>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
+  const int32_t rp_ahead = SH ? -1 : prefetch_rows_ahead<T, C, true>(i, Nt, rowptr, dY, sl);
+  if (MARS_SPMM_PF > 0 && sl < (C * (int)sizeof(T) + 127) / 128) {   // own Z rows (epilogue)
+    prefetch_l2(reinterpret_cast<const char*>(Z + (int64_t)i * C) + sl * 128);
+    prefetch_l2(reinterpret_cast<const char*>(Z + ((int64_t)Nt + i) * C) + sl * 128);
+  }
   float accp[S::NT][V], accn[S::NT][V];
 #pragma unroll
   for (int q = 0; q < S::NT; ++q)
@@ -323,6 +366,7 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
       StoreN<T, V>::store(dZ + row * C + c, o[br][q]);
     }
   }
+  prefetch_csr_ahead(rp_ahead, colind, vals, sl);
   if (rs) {
     row_scale_out<S>(o[0], gmask, sl, rs + i);
     row_scale_out<S>(o[1], gmask, sl, rs + Nt + i);
