@@ -63,8 +63,19 @@ __device__ __forceinline__ void dw_reduce_body(const float* __restrict__ part, i
   const int64_t n = (int64_t)H * CIN;
   const int64_t e = (int64_t)blockIdx.x * 32 + lane;     // e = h * CIN + c
   double t = 0.0;
-  if (e < n)
-    for (int k = j; k < nchunk; k += 8) t += (double)part[(int64_t)k * n + e];
+  if (e < n) {
+    // loads issued four at a time, summed in the fixed order k = j, j+8, ...
+    int k = j;
+    for (; k + 24 < nchunk; k += 32) {
+      const float a0 = part[(int64_t)k * n + e], a1 = part[(int64_t)(k + 8) * n + e];
+      const float a2 = part[(int64_t)(k + 16) * n + e], a3 = part[(int64_t)(k + 24) * n + e];
+      t += (double)a0;
+      t += (double)a1;
+      t += (double)a2;
+      t += (double)a3;
+    }
+    for (; k < nchunk; k += 8) t += (double)part[(int64_t)k * n + e];
+  }
   sh[j][lane] = t;
   __syncthreads();
   if (j == 0 && e < n) {
