@@ -131,7 +131,8 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
 
 // ---------------------------------------------------------------- spmm.cu
 // Forward aggregate of both branches: Y[i] = Σ_j a_ij act(T[j]), Y[Nt+i] = Σ_j a_ij
-// act(T[Nt+j]).  layer1: T = X (pos) and X[perm[j]] (neg), act = identity.
+// act(T[Nt+j]).  layer1: T = X (pos) and X[pi[j]] (neg), act = identity; `perm`
+// is then colperm[k] = pi[colind[k]] (launch_colperm), indexed like colind.
 // Otherwise act = PReLU(alpha[act_layer]).  neg_rows = 0 aggregates only the
 // positive branch (encode).
 // in_bf16 / out_bf16: storage type of T / Y (fp32 or bf16); fp32 accumulation.
@@ -151,6 +152,10 @@ cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void
                             int* nslots, cudaStream_t s, int* launches,
                             const PeerRows* peers = nullptr, float* row_scale = nullptr);
 int spmm_bwd_slots(const GraphDev& g);
+// Layer 1's corrupted-branch column ids: colperm[k] = pi[colind[k]] over the
+// view's entries (launch_spmm_fwd's `perm` argument for act_layer < 0).
+cudaError_t launch_colperm(const GraphDev& g, const int32_t* perm, int32_t* colperm,
+                           cudaStream_t s, int* launches);
 
 // ---------------------------------------------------------------- gemm_simt.cu
 // fp32 SIMT GEMMs (parity path).

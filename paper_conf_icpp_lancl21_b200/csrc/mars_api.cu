@@ -219,6 +219,7 @@ struct Workspace {
   float *Y1 = nullptr, *Z[3] = {nullptr, nullptr, nullptr}, *Y23[2] = {nullptr, nullptr};
   float *dZ = nullptr, *dY = nullptr;
   int32_t* perm = nullptr;
+  int32_t* colperm = nullptr;         // [nnz of the permuted view] pi[colind[k]] (layer 1)
   PermWork pw{};
   HeadWork hw{};
   double *slots[3] = {nullptr, nullptr, nullptr};
@@ -747,6 +748,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   CK(al((void**)&w.dZ, sizeof(float) * R * H));
   CK(al((void**)&w.dY, sizeof(float) * R * H));
   CK(al((void**)&w.perm, sizeof(int32_t) * Np));
+  CK(al((void**)&w.colperm, sizeof(int32_t) * (size_t)std::max<int64_t>(1, pv.nnz)));
   CK(al((void**)&w.pw.keys, sizeof(uint64_t) * Np));
   CK(al((void**)&w.pw.bucket, sizeof(int32_t) * Np));
   CK(al((void**)&w.pw.bcnt, sizeof(int32_t) * (nb + 1)));
@@ -857,6 +859,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM);
   // a row-sharded graph permutes the whole graph on every shard
   RET(launch_perm(gr->perm_view(), m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
+  RET(launch_colperm(g, w.perm, w.colperm, s, nl));
   MARK(MARS_PH_PERM);
   const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
@@ -880,7 +883,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
       RET(launch_shard_barrier(m->sh.sync, s, nl));   // peers' Z_{l-1} complete
       MARK(MARS_PH_EXCHANGE);
     }
-    RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.perm, alpha, l - 1, Ys[l], b16, 1, s, nl,
+    RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.colperm, alpha, l - 1, Ys[l], b16, 1, s, nl,
                         shard && l > 0 ? &m->sh.z[l - 1] : nullptr,
                         tc[l] && h3 ? w.h3_rsY[l] : nullptr));
     MARK(MARS_PH_SPMM_FWD);

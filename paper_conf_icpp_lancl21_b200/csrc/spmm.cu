@@ -208,7 +208,7 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
     if (sl < cnt) {
       cj = colind[k0 + sl];
       cv = vals[k0 + sl];
-      if (PERM && BOTH) cjn = perm[cj];
+      if (PERM && BOTH) cjn = perm[k0 + sl];   // colperm: pi[colind[k]], no dependent lookup
     }
 #if MARS_SPMM_TAIL == 1
     for (int t = 0; t < cnt; t += kU)
@@ -586,6 +586,25 @@ cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16
   if (in_bf16 && out_bf16)
     return fwd_t<bf16, bf16>(g, C, T, perm, alpha_dev, act_layer, Y, nullptr, both, s, peers);
   return cudaErrorInvalidValue;
+}
+
+// colperm[k] = pi[colind[k]] for the entries of the view's rows (layer 1's
+// corrupted gathers read it beside colind instead of a dependent pi lookup).
+__global__ void k_colperm(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
+                          const int32_t* __restrict__ perm, int64_t nnz,
+                          int32_t* __restrict__ colperm) {
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= nnz) return;
+  const int64_t k = rowptr[0] + t;
+  colperm[k] = perm[colind[k]];
+}
+
+cudaError_t launch_colperm(const GraphDev& g, const int32_t* perm, int32_t* colperm,
+                           cudaStream_t s, int* launches) {
+  count_launch(launches);
+  if (g.nnz > 0)
+    k_colperm<<<cdiv(g.nnz, 256), 256, 0, s>>>(g.rowptr, g.colind, perm, g.nnz, colperm);
+  return cudaGetLastError();
 }
 
 // fp32 rows per block is the smallest RPB (largest block count) of any config.
