@@ -141,11 +141,25 @@ __global__ void k_Mv(const float* __restrict__ M, const double* __restrict__ sd,
                      float* __restrict__ vf) {
   const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const double* s = sd + (int64_t)g * H;
+  // H <= 256: at most 8 columns per lane; every load of the 4 rows issued
+  // before the (fixed-order) sums
+  double sv[8];
+#pragma unroll
+  for (int q = 0; q < 8; ++q) sv[q] = lane + 32 * q < H ? s[lane + 32 * q] : 0.0;
+  float mv[4][8];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int r = blockIdx.y * 32 + w * 4 + i;
+#pragma unroll
+    for (int q = 0; q < 8; ++q)
+      mv[i][q] = lane + 32 * q < H ? M[(int64_t)r * H + lane + 32 * q] : 0.f;
+  }
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     const int r = blockIdx.y * 32 + w * 4 + i;
     double t = 0.0;
-    for (int c = lane; c < H; c += 32) t += (double)M[(int64_t)r * H + c] * s[c];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) t += (double)mv[i][q] * sv[q];
     t = warp_sum(t);
     if (lane == 0) vf[(int64_t)g * H + r] = (float)t;
   }
@@ -161,7 +175,19 @@ __global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dv
   const int c = blockIdx.y * 32 + lane;
   const double* dv = dvd + (int64_t)g * H;
   double acc = 0.0;
-  for (int r = w; r < H; r += kWarps) acc += (double)M[(int64_t)r * H + c] * dv[r];
+  // H <= 256: at most 32 rows per warp, loaded 8 at a time, summed in order
+  for (int r0 = w; r0 < H; r0 += 8 * kWarps) {
+    float mv[8];
+    double dd[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int r = r0 + q * kWarps;
+      mv[q] = r < H ? M[(int64_t)r * H + c] : 0.f;
+      dd[q] = r < H ? dv[r] : 0.0;
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) acc += (double)mv[q] * dd[q];
+  }
   sh[w][lane] = acc;
   __syncthreads();
   if (w == 0) {
@@ -309,7 +335,18 @@ __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ 
   if (e < (int64_t)H * H) {
     int r = (int)(e / H), c = (int)(e % H);
     double t = 0.0;
-    for (int g = 0; g < G; ++g) t += dvd[(int64_t)g * H + r] * sd[(int64_t)g * H + c];
+    int g = 0;
+    for (; g + 4 <= G; g += 4) {            // four graphs' loads in flight, summed in order
+      const double a0 = dvd[(int64_t)g * H + r], b0 = sd[(int64_t)g * H + c];
+      const double a1 = dvd[(int64_t)(g + 1) * H + r], b1 = sd[(int64_t)(g + 1) * H + c];
+      const double a2 = dvd[(int64_t)(g + 2) * H + r], b2 = sd[(int64_t)(g + 2) * H + c];
+      const double a3 = dvd[(int64_t)(g + 3) * H + r], b3 = sd[(int64_t)(g + 3) * H + c];
+      t += a0 * b0;
+      t += a1 * b1;
+      t += a2 * b2;
+      t += a3 * b3;
+    }
+    for (; g < G; ++g) t += dvd[(int64_t)g * H + r] * sd[(int64_t)g * H + c];
     gM[e] = (float)t;
   }
   if (e == 0) {
