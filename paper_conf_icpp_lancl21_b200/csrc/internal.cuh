@@ -39,6 +39,15 @@ struct GraphDev {
   const int32_t* chunk_graph;// [nchunks]
   const int32_t* graph_chunk;// [G+1] first chunk of each graph
   // permutation buckets
+  // long rows (degree > kLongRow, e.g. weight-read hubs): aggregated by one warp
+  // per segment of kLongSeg entries plus an in-order combine (spmm.cu); the
+  // main SpMM kernels skip them
+  int32_t nlong = 0;
+  int32_t nseg = 0;
+  const int32_t* long_rows = nullptr;  // [nlong] row ids (view-local)
+  const int32_t* long_seg = nullptr;   // [nlong + 1] first segment of each long row
+  const int32_t* seg_row = nullptr;    // [nseg] long-row index of each segment
+  float* long_part = nullptr;          // [nseg * 2 * 256] fp32 partial sums (scratch)
   int32_t nbuckets;
   const int32_t* bucket_off; // [G+1]
   const int32_t* bucket_log2;// [G]
@@ -130,6 +139,11 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
                         const PermWork& w, int32_t* perm_global, cudaStream_t s, int* launches);
 
 // ---------------------------------------------------------------- spmm.cu
+#ifndef MARS_LONG_ROW
+#define MARS_LONG_ROW 256
+#endif
+constexpr int kLongRow = MARS_LONG_ROW;   // rows with more entries are split into segments
+constexpr int kLongSeg = 128;   // entries per segment
 // Forward aggregate of both branches: Y[i] = Σ_j a_ij act(T[j]), Y[Nt+i] = Σ_j a_ij
 // act(T[Nt+j]).  layer1: T = X (pos) and X[pi[j]] (neg), act = identity; `perm`
 // is then colperm[k] = pi[colind[k]] (launch_colperm), indexed like colind.

@@ -202,7 +202,9 @@ struct mars_graph {
   GraphDev dev_full{};
   int32_t *l_node_off = nullptr, *l_node_graph = nullptr, *l_chunk_row = nullptr,
           *l_chunk_graph = nullptr, *l_graph_chunk = nullptr;
+  std::vector<void*> extra;         // long-row tables (cudaMalloc)
   ~mars_graph() {   // pool memory; mars_free synchronises the device first
+    for (void* p : extra) cudaFree(p);
     for (void* p : {(void*)node_off, (void*)node_graph, (void*)rowptr, (void*)colind, (void*)deg,
                     (void*)chunk_row, (void*)chunk_graph, (void*)graph_chunk, (void*)bucket_off,
                     (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X, (void*)gsize,
@@ -213,9 +215,50 @@ struct mars_graph {
   const GraphDev& perm_view() const { return sharded ? dev_full : dev; }
 };
 
+// Long rows of a view (degree > kLongRow, spmm.cu): host scan of its rowptr,
+// segment tables and the fp32 partial-sum scratch on the device.
+static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v) {
+  v.nlong = v.nseg = 0;
+  v.long_rows = v.long_seg = v.seg_row = nullptr;
+  v.long_part = nullptr;
+  if (v.Nt < 1) return cudaSuccess;
+  std::vector<int32_t> rp((size_t)v.Nt + 1);
+  cudaError_t e = cudaMemcpy(rp.data(), v.rowptr, sizeof(int32_t) * rp.size(), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return e;
+  std::vector<int32_t> rows, seg{0}, segrow;
+  for (int32_t i = 0; i < v.Nt; ++i) {
+    const int32_t d = rp[i + 1] - rp[i];
+    if (d <= kLongRow) continue;
+    const int32_t ns = (d + kLongSeg - 1) / kLongSeg;
+    for (int32_t k = 0; k < ns; ++k) segrow.push_back((int32_t)rows.size());
+    rows.push_back(i);
+    seg.push_back(seg.back() + ns);
+  }
+  if (rows.empty()) return cudaSuccess;
+  auto up = [&](const std::vector<int32_t>& h, const int32_t** d) -> cudaError_t {
+    void* p = nullptr;
+    cudaError_t e2 = cudaMalloc(&p, sizeof(int32_t) * h.size());
+    if (e2 != cudaSuccess) return e2;
+    gr->extra.push_back(p);
+    *d = static_cast<const int32_t*>(p);
+    return cudaMemcpy(p, h.data(), sizeof(int32_t) * h.size(), cudaMemcpyHostToDevice);
+  };
+  if ((e = up(rows, &v.long_rows)) || (e = up(seg, &v.long_seg)) || (e = up(segrow, &v.seg_row)))
+    return e;
+  void* part = nullptr;
+  if ((e = cudaMalloc(&part, sizeof(float) * (size_t)seg.back() * 2 * 256))) return e;
+  gr->extra.push_back(part);
+  v.long_part = static_cast<float*>(part);
+  v.nlong = (int32_t)rows.size();
+  v.nseg = seg.back();
+  return cudaSuccess;
+}
+
 struct Workspace {
   int32_t Nt = 0, G = 0, nchunks = 0, nbuckets = 0, F = 0, H = 0;
   int32_t Nperm = 0;      // rows of the permutation (the whole graph when row-sharded)
+  int64_t nnz_perm = 0;   // entries of the permuted view (colperm)
+  int32_t nlong = 0;      // long rows (dalpha slots of the backward aggregation)
   float *Y1 = nullptr, *Z[3] = {nullptr, nullptr, nullptr}, *Y23[2] = {nullptr, nullptr};
   float *dZ = nullptr, *dY = nullptr;
   int32_t* perm = nullptr;
@@ -561,6 +604,7 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   v.bucket_off = gr->bucket_off;
   v.bucket_log2 = gr->bucket_log2;
   v.gsize = gr->gsize;
+  CK(build_long_rows(gr, v));
   *out = guard.release();
   return MARS_OK;
 }
@@ -725,7 +769,8 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   Workspace& w = m->ws;
   const GraphDev& pv = g->perm_view();
   if (w.Nt >= g->dev.Nt && w.Nperm >= pv.Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks &&
-      w.nbuckets >= pv.nbuckets && w.F == m->F && w.H == m->H)
+      w.nbuckets >= pv.nbuckets && w.nnz_perm >= pv.nnz && w.nlong >= g->dev.nlong &&
+      w.F == m->F && w.H == m->H)
     return MARS_OK;
   if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
   if (m->exec) {
@@ -801,6 +846,8 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   }
   w.Nt = (int32_t)Nt;
   w.Nperm = (int32_t)Np;
+  w.nnz_perm = pv.nnz;
+  w.nlong = g->dev.nlong;
   w.G = G;
   w.nchunks = nch;
   w.nbuckets = nb;
@@ -1553,6 +1600,7 @@ extern "C" mars_status mars_graph_load_shard(const mars_graph_desc* desc, int32_
   v.chunk_graph = g->l_chunk_graph;
   v.graph_chunk = g->l_graph_chunk;
   v.gsize = g->gsize;                    // N of the whole graph (readout mean, loss scale)
+  CK(build_long_rows(g, v));             // of the local rows
   *out = guard.release();
   return MARS_OK;
 }

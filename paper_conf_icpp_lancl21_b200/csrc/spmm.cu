@@ -293,6 +293,7 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
+  if (re - rb > kLongRow) return;                     // long row: k_spmm_long_*
   const int32_t rp_ahead =
       SH ? -1 : prefetch_rows_ahead<Tin, C, MODE == 1 && BOTH>(i, Nt, rowptr, T, sl);
   float accp[S::NT][V], accn[S::NT][V];
@@ -332,6 +333,7 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
   using S = SpmmShape<C, T>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
+  if (re - rb > kLongRow) return;                     // long row: k_spmm_long_*
   const int32_t rp_ahead = SH ? -1 : prefetch_rows_ahead<T, C, true>(i, Nt, rowptr, dY, sl);
   if (MARS_SPMM_PF > 0 && sl < (C * (int)sizeof(T) + 127) / 128) {   // own Z rows (epilogue)
     prefetch_l2(reinterpret_cast<const char*>(Z + (int64_t)i * C) + sl * 128);
@@ -371,6 +373,194 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
     row_scale_out<S>(o[0], gmask, sl, rs + i);
     row_scale_out<S>(o[1], gmask, sl, rs + Nt + i);
   }
+}
+
+
+// ---------------------------------------------------------------- long rows
+// Rows with more than kLongRow entries (hubs: the weight reads of an unrolled
+// RNN, fan-out 2T; ~6000 in the 1.1M-op graph) would serialise hundreds of
+// gather round trips in one warp and become the kernel's tail.  The row kernels
+// skip them; here one warp per segment of kLongSeg entries aggregates into fp32
+// partials (same gathers, same activation), and one warp per long row sums its
+// segments in order -- deterministic -- and applies the row's epilogue.  The
+// sum order differs from a single ascending pass only by the segment
+// bracketing (fp32 accumulation either way).
+struct LongArgs {
+  const int32_t* long_rows;
+  const int32_t* long_seg;
+  const int32_t* seg_row;
+  float* part;
+};
+
+template <int C, int MODE, bool BOTH, bool SH, typename Tin>
+__global__ void __launch_bounds__(32)
+k_spmm_long_part(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
+                 const float* __restrict__ vals, const Tin* __restrict__ T,
+                 const int32_t* __restrict__ perm, const float* __restrict__ alpha,
+                 int act_layer, int32_t Nt, LongArgs la, const __grid_constant__ PeerRows pr) {
+  using S = SpmmShape<C, Tin>;
+  constexpr int V = S::V;
+  const int lane = threadIdx.x;
+  if (lane >= S::L) return;                          // one row group per warp
+  const int sl = lane;
+  const unsigned gmask = (S::L == 32) ? kFull : ((1u << S::L) - 1u);
+  const int seg = blockIdx.x;
+  const int lr = la.seg_row[seg];
+  const int32_t i = la.long_rows[lr];
+  const int32_t e0 = rowptr[i] + (seg - la.long_seg[lr]) * kLongSeg;
+  const int32_t e1 = min(rowptr[i + 1], e0 + kLongSeg);
+  const float a = MODE == 1 ? alpha[act_layer] : 1.f;   // bwd (MODE 2): no activation
+  float accp[S::NT][V], accn[S::NT][V];
+#pragma unroll
+  for (int q = 0; q < S::NT; ++q)
+#pragma unroll
+    for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
+  if (MODE == 0) {
+    row_gather<S, BOTH, 0, true, Tin>(PermSrc<Tin, C>{T}, colind, vals, perm, e0, e1, gmask, sl,
+                                      a, accp, accn);
+  } else if (MODE == 1) {
+    bool done = false;
+    if constexpr (std::is_same<Tin, bf16>::value) {
+      if (a >= 0.f && a <= 1.f) {
+        if (SH)
+          row_gather<S, BOTH, 2, false, Tin>(PeerSrc<Tin, C>{pr}, colind, vals, perm, e0, e1, gmask,
+                                             sl, a, accp, accn);
+        else
+          row_gather<S, BOTH, 2, false, Tin>(StackedSrc<Tin, C>{T, Nt}, colind, vals, perm, e0, e1,
+                                             gmask, sl, a, accp, accn);
+        done = true;
+      }
+    }
+    if (!done) {
+      if (SH)
+        row_gather<S, BOTH, 1, false, Tin>(PeerSrc<Tin, C>{pr}, colind, vals, perm, e0, e1, gmask,
+                                           sl, a, accp, accn);
+      else
+        row_gather<S, BOTH, 1, false, Tin>(StackedSrc<Tin, C>{T, Nt}, colind, vals, perm, e0, e1,
+                                           gmask, sl, a, accp, accn);
+    }
+  } else {
+    if (SH)
+      row_gather<S, true, 0, false, Tin>(PeerSrc<Tin, C>{pr}, colind, vals, nullptr, e0, e1, gmask,
+                                         sl, a, accp, accn);
+    else
+      row_gather<S, true, 0, false, Tin>(StackedSrc<Tin, C>{T, Nt}, colind, vals, nullptr, e0, e1,
+                                         gmask, sl, a, accp, accn);
+  }
+  float* out = la.part + (int64_t)seg * 2 * C;
+#pragma unroll
+  for (int q = 0; q < S::NT; ++q) {
+    const int c = (sl + q * S::L) * V;
+    StoreN<float, V>::store(out + c, accp[q]);
+    StoreN<float, V>::store(out + C + c, accn[q]);
+  }
+}
+
+// Combine: one warp per long row, segments summed in order.  FWD: store Y (+ the
+// row scales); else the backward epilogue (PReLU'(Z), dZ, dalpha partial into
+// slots[lr]).
+template <int C, bool FWD, bool BOTH, typename Tin, typename Tout>
+__global__ void __launch_bounds__(32)
+k_spmm_long_fin(const float* __restrict__ alpha, int layer, int32_t Nt, LongArgs la,
+                const Tin* __restrict__ Z, Tout* __restrict__ out, float* __restrict__ rs,
+                double* __restrict__ slots) {
+  using S = SpmmShape<C, Tout>;
+  constexpr int V = S::V;
+  const int lane = threadIdx.x;
+  const int lr = blockIdx.x;
+  if (lane >= S::L) return;                          // one row group per warp
+  const int sl = lane;
+  const unsigned gmask = (S::L == 32) ? kFull : ((1u << S::L) - 1u);
+  const int32_t i = la.long_rows[lr];
+  float acc[2][S::NT][V];
+#pragma unroll
+  for (int b = 0; b < 2; ++b)
+#pragma unroll
+    for (int q = 0; q < S::NT; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) acc[b][q][e] = 0.f;
+  for (int seg = la.long_seg[lr]; seg < la.long_seg[lr + 1]; ++seg) {
+    const float* p = la.part + (int64_t)seg * 2 * C;
+#pragma unroll
+    for (int b = 0; b < 2; ++b)
+#pragma unroll
+      for (int q = 0; q < S::NT; ++q) {
+        const float4* v4 = reinterpret_cast<const float4*>(p + b * C + (sl + q * S::L) * V);
+#pragma unroll
+        for (int e4 = 0; e4 < V / 4; ++e4) {
+          const float4 x = v4[e4];
+          acc[b][q][4 * e4] += x.x;
+          acc[b][q][4 * e4 + 1] += x.y;
+          acc[b][q][4 * e4 + 2] += x.z;
+          acc[b][q][4 * e4 + 3] += x.w;
+        }
+      }
+  }
+  if constexpr (FWD) {
+#pragma unroll
+    for (int q = 0; q < S::NT; ++q) {
+      const int c = (sl + q * S::L) * V;
+      StoreN<Tout, V>::store(out + (int64_t)i * C + c, acc[0][q]);
+      if (BOTH) StoreN<Tout, V>::store(out + ((int64_t)Nt + i) * C + c, acc[1][q]);
+    }
+    if (rs) {
+      row_scale_out<S>(acc[0], gmask, sl, rs + i);
+      if (BOTH) row_scale_out<S>(acc[1], gmask, sl, rs + Nt + i);
+    }
+  } else {
+  const float a = alpha[layer];
+  float da = 0.f;
+  float o[2][S::NT][V];
+#pragma unroll
+  for (int q = 0; q < S::NT; ++q) {
+    const int c = (sl + q * S::L) * V;
+#pragma unroll
+    for (int br = 0; br < 2; ++br) {
+      const int64_t row = (int64_t)i + (br ? Nt : 0);
+      float z[V];
+      Vec<Tin>::load(Z + row * C + c, z);
+#pragma unroll
+      for (int e = 0; e < V; ++e) {
+        const float h = acc[br][q][e];
+        o[br][q][e] = z[e] > 0.f ? h : a * h;
+        da += z[e] > 0.f ? 0.f : h * z[e];
+      }
+      StoreN<Tout, V>::store(out + row * C + c, o[br][q]);
+    }
+  }
+  if (rs) {
+    row_scale_out<S>(o[0], gmask, sl, rs + i);
+    row_scale_out<S>(o[1], gmask, sl, rs + Nt + i);
+  }
+  double dd = (double)da;
+#pragma unroll
+  for (int off = S::L / 2; off > 0; off >>= 1) dd += __shfl_xor_sync(gmask, dd, off);
+  if (sl == 0) slots[lr] = dd;
+  }
+}
+
+template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
+cudaError_t long_fwd(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
+                     int act_layer, Tout* Y, float* rs, cudaStream_t s, const PeerRows& pr) {
+  if (g.nlong == 0) return cudaSuccess;
+  const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
+  k_spmm_long_part<C, MODE, BOTH, SH, Tin><<<g.nseg, 32, 0, s>>>(
+      g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, la, pr);
+  k_spmm_long_fin<C, true, BOTH, Tin, Tout><<<g.nlong, 32, 0, s>>>(
+      alpha, 0, g.Nt, la, nullptr, Y, rs, nullptr);
+  return cudaGetLastError();
+}
+
+template <int C, bool SH, typename T>
+cudaError_t long_bwd(const GraphDev& g, const T* dY, const T* Z, const float* alpha, int layer,
+                     T* dZ, double* slots, float* rs, cudaStream_t s, const PeerRows& pr) {
+  if (g.nlong == 0) return cudaSuccess;
+  const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
+  k_spmm_long_part<C, 2, true, SH, T><<<g.nseg, 32, 0, s>>>(
+      g.rowptr, g.colind, g.vals, dY, nullptr, alpha, layer, g.Nt, la, pr);
+  k_spmm_long_fin<C, false, true, T, T><<<g.nlong, 32, 0, s>>>(alpha, layer, g.Nt, la, Z, dZ, rs,
+                                                                 slots);
+  return cudaGetLastError();
 }
 
 // Rows handled by block b: NW warps x RPW row groups.  BAND = false: one row
@@ -493,7 +683,8 @@ cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, con
   k_spmm_fwd<C, MODE, BOTH, SH, BAND, Tin, Tout>
       <<<spmm_blocks<C, Tin, BAND>(g.Nt), BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
           g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, rs, pr);
-  return cudaGetLastError();
+  if (cudaError_t e = cudaGetLastError()) return e;
+  return long_fwd<C, MODE, BOTH, SH, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, pr);
 }
 
 template <int C, typename Tin, typename Tout>
@@ -539,19 +730,21 @@ cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha
   constexpr bool BAND = MARS_SPMM_BAND;
   const unsigned blocks = spmm_blocks<C, T, BAND>(g.Nt);
   const unsigned threads = BAND ? kBandThreads : kSpmmThreads;
-  *nslots = (int)blocks;
+  *nslots = (int)blocks + g.nlong;                   // long rows' dalpha after the blocks'
   if constexpr (C == 128 || C == 256) {
     if (peers) {
       k_spmm_bwd<C, true, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
                                                               alpha, layer, g.Nt, dZ, slots, rs, *peers);
-      return cudaGetLastError();
+      if (cudaError_t e = cudaGetLastError()) return e;
+      return long_bwd<C, true, T>(g, dY, Z, alpha, layer, dZ, slots + blocks, rs, s, *peers);
     }
   }
   if (peers) return cudaErrorInvalidValue;
   k_spmm_bwd<C, false, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
                                                            alpha, layer, g.Nt, dZ, slots, rs,
                                                            PeerRows{});
-  return cudaGetLastError();
+  if (cudaError_t e = cudaGetLastError()) return e;
+  return long_bwd<C, false, T>(g, dY, Z, alpha, layer, dZ, slots + blocks, rs, s, PeerRows{});
 }
 
 template <typename T>
@@ -578,7 +771,7 @@ cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16
                             const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
                             int out_bf16, int both, cudaStream_t s, int* launches,
                             const PeerRows* peers, float* rs) {
-  count_launch(launches);
+  count_launch(launches, g.nlong ? 3 : 1);
   if (!in_bf16 && !out_bf16)
     return fwd_t<float, float>(g, C, T, perm, alpha_dev, act_layer, Y, rs, both, s, peers);
   if (!in_bf16 && out_bf16)
@@ -609,13 +802,15 @@ cudaError_t launch_colperm(const GraphDev& g, const int32_t* perm, int32_t* colp
 
 // fp32 rows per block is the smallest RPB (largest block count) of any config.
 // (+ 128 doubles of scratch for the two-stage reduction, head.cu)
-int spmm_bwd_slots(const GraphDev& g) { return (int)cdiv(g.Nt, SpmmShape<256, float>::RPB) + 1 + 128; }
+int spmm_bwd_slots(const GraphDev& g) {
+  return (int)cdiv(g.Nt, SpmmShape<256, float>::RPB) + 1 + g.nlong + 128;
+}
 
 cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void* Z, int bf16_,
                             const float* alpha_dev, int layer, void* dZ, double* slots,
                             int* nslots, cudaStream_t s, int* launches, const PeerRows* peers,
                             float* rs) {
-  count_launch(launches);
+  count_launch(launches, g.nlong ? 3 : 1);
   if (bf16_) return bwd_t<bf16>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, nullptr, s, peers);
   return bwd_t<float>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, rs, s, peers);
 }

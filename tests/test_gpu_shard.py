@@ -67,7 +67,18 @@ def test_shard_geometry():
 @pytest.mark.parametrize("name,P,H", [("inception", 2, 128), ("inception", 3, 128),
                                       ("gnmt", 4, 256)])
 def test_shard_step_matches_unsharded(name, P, H):
-    graph = SG.cached(name, 0)
+    _shard_case(SG.cached(name, 0), P, H)
+
+
+def test_shard_long_rows():
+    """A hub row of ~2600 entries (the long-row path of spmm.cu: segments
+    aggregated by several warps, combined in order) owned by one shard, its
+    halo gathered from the other shard."""
+    from tests.test_gpu_spmm_edge import star_graph
+    _shard_case(star_graph(), 2, 256)
+
+
+def _shard_case(graph, P, H):
     F, seed = 64, 5
     N = graph.num_nodes
     g1 = mars.graph_load([graph])

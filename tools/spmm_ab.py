@@ -19,11 +19,13 @@ def child(path):
     import paper_conf_icpp_lancl21_b200.mars as M
     M.LIB_PATH = path
     from synth import graphs as SG
-    gs = [SG.cached("gnmt", i) for i in range(16)]
+    wl = os.environ.get("MARS_AB_WORKLOAD", "gnmt")          # gnmt | inception | bert
+    gs = [SG.cached(wl, i) for i in range({"gnmt": 16, "inception": 16, "bert": 8}[wl])]
+    H = 128 if wl == "inception" else 256
     g = M.graph_load(gs)
     out = {}
     for prec in (M.MARS_FP32, M.MARS_BF16):
-        m = M.dgi_create(in_dim=64, hidden_dim=256, seed=0, precision=prec)
+        m = M.dgi_create(in_dim=64, hidden_dim=H, seed=0, precision=prec)
         if os.environ.get("MARS_AB_GEMM"):
             m.set_gemm_impl(os.environ["MARS_AB_GEMM"])
         for k in range(3):
