@@ -39,9 +39,10 @@ struct GraphDev {
   const int32_t* chunk_graph;// [nchunks]
   const int32_t* graph_chunk;// [G+1] first chunk of each graph
   // permutation buckets
-  // long rows (degree > kLongRow, e.g. weight-read hubs): aggregated by one warp
+  // long rows (degree > long_min, e.g. weight-read hubs): aggregated by one warp
   // per segment of kLongSeg entries plus an in-order combine (spmm.cu); the
   // main SpMM kernels skip them
+  int32_t long_min = 0x7fffffff;       // rows with more entries than this are long
   int32_t nlong = 0;
   int32_t nseg = 0;
   const int32_t* long_rows = nullptr;  // [nlong] row ids (view-local)
@@ -139,10 +140,12 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
                         const PermWork& w, int32_t* perm_global, cudaStream_t s, int* launches);
 
 // ---------------------------------------------------------------- spmm.cu
-#ifndef MARS_LONG_ROW
-#define MARS_LONG_ROW 256
-#endif
-constexpr int kLongRow = MARS_LONG_ROW;   // rows with more entries are split into segments
+// A row is long when its serial gather time would exceed about half the row
+// kernel's duration: degree > kLongFactor x rows per resident warp slot
+// (Nt / (SMs x 32)), clamped to [kLongMin, kLongMax] (graph load, mars_api.cu).
+constexpr int kLongFactor = 8;
+constexpr int kLongMin = 128;
+constexpr int kLongMax = 1024;
 constexpr int kLongSeg = 128;   // entries per segment
 // Forward aggregate of both branches: Y[i] = Σ_j a_ij act(T[j]), Y[Nt+i] = Σ_j a_ij
 // act(T[Nt+j]).  layer1: T = X (pos) and X[pi[j]] (neg), act = identity; `perm`

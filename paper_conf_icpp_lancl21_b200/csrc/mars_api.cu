@@ -215,20 +215,26 @@ struct mars_graph {
   const GraphDev& perm_view() const { return sharded ? dev_full : dev; }
 };
 
-// Long rows of a view (degree > kLongRow, spmm.cu): host scan of its rowptr,
+// Long rows of a view (degree > long_min, spmm.cu): host scan of its rowptr,
 // segment tables and the fp32 partial-sum scratch on the device.
 static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v) {
   v.nlong = v.nseg = 0;
+  v.long_min = 0x7fffffff;
   v.long_rows = v.long_seg = v.seg_row = nullptr;
   v.long_part = nullptr;
   if (v.Nt < 1) return cudaSuccess;
   std::vector<int32_t> rp((size_t)v.Nt + 1);
   cudaError_t e = cudaMemcpy(rp.data(), v.rowptr, sizeof(int32_t) * rp.size(), cudaMemcpyDeviceToHost);
   if (e != cudaSuccess) return e;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t per_slot = (int64_t)v.Nt / std::max(1, sms * 32);
+  v.long_min = (int32_t)std::min<int64_t>(kLongMax, std::max<int64_t>(kLongMin, kLongFactor * per_slot));
   std::vector<int32_t> rows, seg{0}, segrow;
   for (int32_t i = 0; i < v.Nt; ++i) {
     const int32_t d = rp[i + 1] - rp[i];
-    if (d <= kLongRow) continue;
+    if (d <= v.long_min) continue;
     const int32_t ns = (d + kLongSeg - 1) / kLongSeg;
     for (int32_t k = 0; k < ns; ++k) segrow.push_back((int32_t)rows.size());
     rows.push_back(i);

@@ -283,8 +283,9 @@ __device__ __forceinline__ void prefetch_csr_ahead(int32_t rp, const int32_t* co
 // Row bodies shared by the two kernel shapes below.
 // MODE 0: layer 1 (neg rows gather X[perm[j]]), MODE 1: PReLU on load.
 // SH: row-sharded graph (layers 2-3): rows are gathered through PeerSrc.
-template <int C, int MODE, bool BOTH, bool SH, int ACT, typename Tin, typename Tout>
-__device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ rowptr,
+template <int C, int MODE, bool BOTH, bool SH, int ACT, bool LONG, typename Tin, typename Tout>
+__device__ __forceinline__ void fwd_row(int32_t i, int32_t long_min,
+                                        const int32_t* __restrict__ rowptr,
                                         const int32_t* __restrict__ colind,
                                         const float* __restrict__ vals, const Tin* __restrict__ T,
                                         const int32_t* __restrict__ perm, float a, int32_t Nt,
@@ -293,7 +294,7 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
-  if (re - rb > kLongRow) return;                     // long row: k_spmm_long_*
+  if (LONG && re - rb > long_min) return;            // long row: segments + k_spmm_long_fin
   const int32_t rp_ahead =
       SH ? -1 : prefetch_rows_ahead<Tin, C, MODE == 1 && BOTH>(i, Nt, rowptr, T, sl);
   float accp[S::NT][V], accn[S::NT][V];
@@ -323,8 +324,9 @@ __device__ __forceinline__ void fwd_row(int32_t i, const int32_t* __restrict__ r
   }
 }
 
-template <int C, bool SH, typename T>
-__device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ rowptr,
+template <int C, bool SH, bool LONG, typename T>
+__device__ __forceinline__ void bwd_row(int32_t i, int32_t long_min,
+                                        const int32_t* __restrict__ rowptr,
                                         const int32_t* __restrict__ colind,
                                         const float* __restrict__ vals, const T* __restrict__ dY,
                                         const T* __restrict__ Z, float a, int32_t Nt,
@@ -333,7 +335,7 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
   using S = SpmmShape<C, T>;
   constexpr int V = S::V;
   const int32_t rb = rowptr[i], re = rowptr[i + 1];
-  if (re - rb > kLongRow) return;                     // long row: k_spmm_long_*
+  if (LONG && re - rb > long_min) return;            // long row: segments + k_spmm_long_fin
   const int32_t rp_ahead = SH ? -1 : prefetch_rows_ahead<T, C, true>(i, Nt, rowptr, dY, sl);
   if (MARS_SPMM_PF > 0 && sl < (C * (int)sizeof(T) + 127) / 128) {   // own Z rows (epilogue)
     prefetch_l2(reinterpret_cast<const char*>(Z + (int64_t)i * C) + sl * 128);
@@ -377,7 +379,7 @@ __device__ __forceinline__ void bwd_row(int32_t i, const int32_t* __restrict__ r
 
 
 // ---------------------------------------------------------------- long rows
-// Rows with more than kLongRow entries (hubs: the weight reads of an unrolled
+// Rows with more than long_min entries (hubs: the weight reads of an unrolled
 // RNN, fan-out 2T; ~6000 in the 1.1M-op graph) would serialise hundreds of
 // gather round trips in one warp and become the kernel's tail.  The row kernels
 // skip them; here one warp per segment of kLongSeg entries aggregates into fp32
@@ -392,24 +394,25 @@ struct LongArgs {
   float* part;
 };
 
+// Segment `seg` of a long row, run by the first warp-blocks of the row kernels'
+// grid (so the segments overlap the ordinary rows).
 template <int C, int MODE, bool BOTH, bool SH, typename Tin>
-__global__ void __launch_bounds__(32)
-k_spmm_long_part(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
-                 const float* __restrict__ vals, const Tin* __restrict__ T,
-                 const int32_t* __restrict__ perm, const float* __restrict__ alpha,
-                 int act_layer, int32_t Nt, LongArgs la, const __grid_constant__ PeerRows pr) {
+__device__ __forceinline__ void long_part_dev(int seg, const int32_t* __restrict__ rowptr,
+                                              const int32_t* __restrict__ colind,
+                                              const float* __restrict__ vals,
+                                              const Tin* __restrict__ T,
+                                              const int32_t* __restrict__ perm, float a,
+                                              int32_t Nt, const LongArgs& la, const PeerRows& pr) {
   using S = SpmmShape<C, Tin>;
   constexpr int V = S::V;
-  const int lane = threadIdx.x;
+  const int lane = threadIdx.x & 31;
   if (lane >= S::L) return;                          // one row group per warp
   const int sl = lane;
   const unsigned gmask = (S::L == 32) ? kFull : ((1u << S::L) - 1u);
-  const int seg = blockIdx.x;
   const int lr = la.seg_row[seg];
   const int32_t i = la.long_rows[lr];
   const int32_t e0 = rowptr[i] + (seg - la.long_seg[lr]) * kLongSeg;
   const int32_t e1 = min(rowptr[i + 1], e0 + kLongSeg);
-  const float a = MODE == 1 ? alpha[act_layer] : 1.f;   // bwd (MODE 2): no activation
   float accp[S::NT][V], accn[S::NT][V];
 #pragma unroll
   for (int q = 0; q < S::NT; ++q)
@@ -544,8 +547,6 @@ cudaError_t long_fwd(const GraphDev& g, const Tin* T, const int32_t* perm, const
                      int act_layer, Tout* Y, float* rs, cudaStream_t s, const PeerRows& pr) {
   if (g.nlong == 0) return cudaSuccess;
   const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
-  k_spmm_long_part<C, MODE, BOTH, SH, Tin><<<g.nseg, 32, 0, s>>>(
-      g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, la, pr);
   k_spmm_long_fin<C, true, BOTH, Tin, Tout><<<g.nlong, 32, 0, s>>>(
       alpha, 0, g.Nt, la, nullptr, Y, rs, nullptr);
   return cudaGetLastError();
@@ -556,8 +557,6 @@ cudaError_t long_bwd(const GraphDev& g, const T* dY, const T* Z, const float* al
                      T* dZ, double* slots, float* rs, cudaStream_t s, const PeerRows& pr) {
   if (g.nlong == 0) return cudaSuccess;
   const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
-  k_spmm_long_part<C, 2, true, SH, T><<<g.nseg, 32, 0, s>>>(
-      g.rowptr, g.colind, g.vals, dY, nullptr, alpha, layer, g.Nt, la, pr);
   k_spmm_long_fin<C, false, true, T, T><<<g.nlong, 32, 0, s>>>(alpha, layer, g.Nt, la, Z, dZ, rs,
                                                                  slots);
   return cudaGetLastError();
@@ -581,48 +580,57 @@ struct RowSched {
 #endif
 constexpr int kBandThreads = 1024;
 
-template <int C, int MODE, bool BOTH, bool SH, bool BAND, typename Tin, typename Tout>
+template <int C, int MODE, bool BOTH, bool SH, bool BAND, bool LONG, typename Tin, typename Tout>
 __global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 : MARS_SPMM_MINB)
 k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const Tin* __restrict__ T,
            const int32_t* __restrict__ perm, const float* __restrict__ alpha, int act_layer,
            int32_t Nt, Tout* __restrict__ Y, float* __restrict__ rs,
-           const __grid_constant__ PeerRows pr) {
+           const __grid_constant__ PeerRows pr, const __grid_constant__ LongArgs la, int32_t nseg,
+           int32_t long_min) {
   using S = SpmmShape<C, Tin>;
   using RS = RowSched<C, Tin, BAND>;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int sub = lane / S::L, sl = lane % S::L;
   const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
   const float a = (MODE == 1) ? alpha[act_layer] : 1.f;
+  if (LONG && (int32_t)blockIdx.x < nseg) {         // long-row segments first
+    long_part_dev<C, MODE, BOTH, SH, Tin>(blockIdx.x, rowptr, colind, vals, T, perm, a, Nt, la,
+                                          pr);
+    return;
+  }
+  const int32_t bid = LONG ? (int32_t)blockIdx.x - nseg : (int32_t)blockIdx.x;
+  const int32_t nblk = LONG ? (int32_t)gridDim.x - nseg : (int32_t)gridDim.x;
   if (!BAND) {
     // MARS_SPMM_PERSIST: a resident grid walks rows i, i + gridDim·RPB, ...
     // (no per-row block launches); otherwise one launch block per RPB rows
-    const int32_t step = MARS_SPMM_PERSIST ? (int32_t)gridDim.x * RS::RPB : Nt;
-    for (int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub; i < Nt; i += step) {
+    const int32_t step = MARS_SPMM_PERSIST ? nblk * RS::RPB : Nt;
+    for (int32_t i = bid * RS::RPB + w * S::RPW + sub; i < Nt; i += step) {
       // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
       if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
         if (a >= 0.f && a <= 1.f) {
-          fwd_row<C, MODE, BOTH, SH, 2>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
+          fwd_row<C, MODE, BOTH, SH, 2, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
           continue;
         }
       }
-      fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
+      fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
     }
     return;
   }
-  const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
-  const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
+  const int32_t n = (int32_t)((Nt + nblk - 1) / nblk);
+  const int32_t r0 = bid * n, r1 = min(Nt, r0 + n);
   for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-    fwd_row<C, MODE, BOTH, SH, 1>(i, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
+    fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
 }
 
-template <int C, bool SH, bool BAND, typename T>
+template <int C, bool SH, bool BAND, bool LONG, typename T>
 __global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 : MARS_SPMM_MINB)
 k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const T* __restrict__ dY, const T* __restrict__ Z,
            const float* __restrict__ alpha, int layer, int32_t Nt, T* __restrict__ dZ,
            double* __restrict__ slots, float* __restrict__ rs,
-           const __grid_constant__ PeerRows pr) {
+           const __grid_constant__ PeerRows pr, const __grid_constant__ LongArgs la, int32_t nseg,
+           int32_t long_min) {
   using S = SpmmShape<C, T>;
   using RS = RowSched<C, T, BAND>;
   __shared__ double wpart[RS::NW];
@@ -630,16 +638,23 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   const int sub = lane / S::L, sl = lane % S::L;
   const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
   const float a = alpha[layer];
+  if (LONG && (int32_t)blockIdx.x < nseg) {         // long-row segments first (no slot)
+    long_part_dev<C, 2, true, SH, T>(blockIdx.x, rowptr, colind, vals, dY, nullptr, 1.f, Nt, la,
+                                     pr);
+    return;
+  }
+  const int32_t bid = LONG ? (int32_t)blockIdx.x - nseg : (int32_t)blockIdx.x;
+  const int32_t nblk = LONG ? (int32_t)gridDim.x - nseg : (int32_t)gridDim.x;
   float da = 0.f;
   if (!BAND) {
-    const int32_t step = MARS_SPMM_PERSIST ? (int32_t)gridDim.x * RS::RPB : Nt;
-    for (int32_t i = (int32_t)blockIdx.x * RS::RPB + w * S::RPW + sub; i < Nt; i += step)
-      bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
+    const int32_t step = MARS_SPMM_PERSIST ? nblk * RS::RPB : Nt;
+    for (int32_t i = bid * RS::RPB + w * S::RPW + sub; i < Nt; i += step)
+      bwd_row<C, SH, LONG>(i, long_min, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
   } else {
-    const int32_t n = (int32_t)((Nt + gridDim.x - 1) / gridDim.x);
-    const int32_t r0 = (int32_t)blockIdx.x * n, r1 = min(Nt, r0 + n);
+    const int32_t n = (int32_t)((Nt + nblk - 1) / nblk);
+    const int32_t r0 = bid * n, r1 = min(Nt, r0 + n);
     for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-      bwd_row<C, SH>(i, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
+      bwd_row<C, SH, LONG>(i, long_min, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
   }
   const double wd = warp_sum((double)da);
   if (lane == 0) wpart[w] = wd;
@@ -647,7 +662,7 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
   if (threadIdx.x == 0) {
     double t = 0.0;
     for (int k = 0; k < RS::NW; ++k) t += wpart[k];
-    slots[blockIdx.x] = t;
+    slots[bid] = t;
   }
 }
 
@@ -680,9 +695,18 @@ template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
 cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
                        int act_layer, Tout* Y, float* rs, cudaStream_t s, const PeerRows& pr) {
   constexpr bool BAND = MARS_SPMM_BAND && MODE == 1;
-  k_spmm_fwd<C, MODE, BOTH, SH, BAND, Tin, Tout>
-      <<<spmm_blocks<C, Tin, BAND>(g.Nt), BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
-          g.rowptr, g.colind, g.vals, T, perm, alpha, act_layer < 0 ? 0 : act_layer, g.Nt, Y, rs, pr);
+  static_assert(BAND || kSpmmThreads == 32, "long-row segments run as one-warp blocks");
+  const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
+  const unsigned nb = spmm_blocks<C, Tin, BAND>(g.Nt);
+  const int al = act_layer < 0 ? 0 : act_layer;
+  if (g.nseg > 0)   // long rows: their segments run as the grid's first blocks
+    k_spmm_fwd<C, MODE, BOTH, SH, BAND, true, Tin, Tout>
+        <<<nb + g.nseg, BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
+            g.rowptr, g.colind, g.vals, T, perm, alpha, al, g.Nt, Y, rs, pr, la, g.nseg, g.long_min);
+  else
+    k_spmm_fwd<C, MODE, BOTH, SH, BAND, false, Tin, Tout>
+        <<<nb, BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
+            g.rowptr, g.colind, g.vals, T, perm, alpha, al, g.Nt, Y, rs, pr, la, 0, 0);
   if (cudaError_t e = cudaGetLastError()) return e;
   return long_fwd<C, MODE, BOTH, SH, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, pr);
 }
@@ -730,19 +754,29 @@ cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha
   constexpr bool BAND = MARS_SPMM_BAND;
   const unsigned blocks = spmm_blocks<C, T, BAND>(g.Nt);
   const unsigned threads = BAND ? kBandThreads : kSpmmThreads;
+  const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
   *nslots = (int)blocks + g.nlong;                   // long rows' dalpha after the blocks'
   if constexpr (C == 128 || C == 256) {
     if (peers) {
-      k_spmm_bwd<C, true, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
-                                                              alpha, layer, g.Nt, dZ, slots, rs, *peers);
+      if (g.nseg > 0)
+        k_spmm_bwd<C, true, BAND, true, T><<<blocks + g.nseg, threads, 0, s>>>(
+            g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, *peers, la,
+            g.nseg, g.long_min);
+      else
+        k_spmm_bwd<C, true, BAND, false, T><<<blocks, threads, 0, s>>>(
+            g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, *peers, la, 0, 0);
       if (cudaError_t e = cudaGetLastError()) return e;
       return long_bwd<C, true, T>(g, dY, Z, alpha, layer, dZ, slots + blocks, rs, s, *peers);
     }
   }
   if (peers) return cudaErrorInvalidValue;
-  k_spmm_bwd<C, false, BAND, T><<<blocks, threads, 0, s>>>(g.rowptr, g.colind, g.vals, dY, Z,
-                                                           alpha, layer, g.Nt, dZ, slots, rs,
-                                                           PeerRows{});
+  if (g.nseg > 0)
+    k_spmm_bwd<C, false, BAND, true, T><<<blocks + g.nseg, threads, 0, s>>>(
+        g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, PeerRows{}, la,
+        g.nseg, g.long_min);
+  else
+    k_spmm_bwd<C, false, BAND, false, T><<<blocks, threads, 0, s>>>(
+        g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, PeerRows{}, la, 0, 0);
   if (cudaError_t e = cudaGetLastError()) return e;
   return long_bwd<C, false, T>(g, dY, Z, alpha, layer, dZ, slots + blocks, rs, s, PeerRows{});
 }
@@ -771,7 +805,7 @@ cudaError_t launch_spmm_fwd(const GraphDev& g, int C, const void* T, int in_bf16
                             const int32_t* perm, const float* alpha_dev, int act_layer, void* Y,
                             int out_bf16, int both, cudaStream_t s, int* launches,
                             const PeerRows* peers, float* rs) {
-  count_launch(launches, g.nlong ? 3 : 1);
+  count_launch(launches, g.nlong ? 2 : 1);
   if (!in_bf16 && !out_bf16)
     return fwd_t<float, float>(g, C, T, perm, alpha_dev, act_layer, Y, rs, both, s, peers);
   if (!in_bf16 && out_bf16)
@@ -810,7 +844,7 @@ cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void
                             const float* alpha_dev, int layer, void* dZ, double* slots,
                             int* nslots, cudaStream_t s, int* launches, const PeerRows* peers,
                             float* rs) {
-  count_launch(launches, g.nlong ? 3 : 1);
+  count_launch(launches, g.nlong ? 2 : 1);
   if (bf16_) return bwd_t<bf16>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, nullptr, s, peers);
   return bwd_t<float>(g, C, dY, Z, alpha_dev, layer, dZ, slots, nslots, rs, s, peers);
 }
