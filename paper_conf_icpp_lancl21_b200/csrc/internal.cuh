@@ -171,6 +171,7 @@ cudaError_t launch_spmm_bwd(const GraphDev& g, int C, const void* dY, const void
 int spmm_bwd_slots(const GraphDev& g);
 // Layer 1's corrupted-branch column ids: colperm[k] = pi[colind[k]] over the
 // view's entries (launch_spmm_fwd's `perm` argument for act_layer < 0).
+cudaError_t launch_max_degree(const int32_t* rowptr, int32_t Nt, int32_t* out, cudaStream_t s);
 cudaError_t launch_colperm(const GraphDev& g, const int32_t* perm, int32_t* colperm,
                            cudaStream_t s, int* launches);
 

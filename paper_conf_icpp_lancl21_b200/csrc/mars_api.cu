@@ -204,7 +204,7 @@ struct mars_graph {
           *l_chunk_graph = nullptr, *l_graph_chunk = nullptr;
   std::vector<void*> extra;         // long-row tables (cudaMalloc)
   ~mars_graph() {   // pool memory; mars_free synchronises the device first
-    for (void* p : extra) cudaFree(p);
+    for (void* p : extra) cudaFreeAsync(p, nullptr);
     for (void* p : {(void*)node_off, (void*)node_graph, (void*)rowptr, (void*)colind, (void*)deg,
                     (void*)chunk_row, (void*)chunk_graph, (void*)graph_chunk, (void*)bucket_off,
                     (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X, (void*)gsize,
@@ -217,20 +217,38 @@ struct mars_graph {
 
 // Long rows of a view (degree > long_min, spmm.cu): host scan of its rowptr,
 // segment tables and the fp32 partial-sum scratch on the device.
-static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v) {
+// Everything on the loader's non-blocking stream `s` (no legacy-stream copies or
+// cudaMalloc, which would wait for a model's step running concurrently).
+static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s) {
   v.nlong = v.nseg = 0;
   v.long_min = 0x7fffffff;
   v.long_rows = v.long_seg = v.seg_row = nullptr;
   v.long_part = nullptr;
   if (v.Nt < 1) return cudaSuccess;
-  std::vector<int32_t> rp((size_t)v.Nt + 1);
-  cudaError_t e = cudaMemcpy(rp.data(), v.rowptr, sizeof(int32_t) * rp.size(), cudaMemcpyDeviceToHost);
-  if (e != cudaSuccess) return e;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t per_slot = (int64_t)v.Nt / std::max(1, sms * 32);
-  v.long_min = (int32_t)std::min<int64_t>(kLongMax, std::max<int64_t>(kLongMin, kLongFactor * per_slot));
+  const int32_t long_min =
+      (int32_t)std::min<int64_t>(kLongMax, std::max<int64_t>(kLongMin, kLongFactor * per_slot));
+  {   // most graphs have no long row: 4 bytes back instead of the whole rowptr
+    int32_t* dmax = nullptr;
+    int32_t hmax = 0;
+    cudaError_t e0 = cudaMallocAsync(&dmax, sizeof(int32_t), s);
+    if (e0 == cudaSuccess) e0 = launch_max_degree(v.rowptr, v.Nt, dmax, s);
+    if (e0 == cudaSuccess)
+      e0 = cudaMemcpyAsync(&hmax, dmax, sizeof(int32_t), cudaMemcpyDeviceToHost, s);
+    if (dmax) cudaFreeAsync(dmax, s);
+    if (e0 == cudaSuccess) e0 = cudaStreamSynchronize(s);
+    if (e0 != cudaSuccess) return e0;
+    if (hmax <= long_min) return cudaSuccess;
+  }
+  std::vector<int32_t> rp((size_t)v.Nt + 1);
+  cudaError_t e = cudaMemcpyAsync(rp.data(), v.rowptr, sizeof(int32_t) * rp.size(),
+                                  cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return e;
+  v.long_min = long_min;
   std::vector<int32_t> rows, seg{0}, segrow;
   for (int32_t i = 0; i < v.Nt; ++i) {
     const int32_t d = rp[i + 1] - rp[i];
@@ -243,21 +261,21 @@ static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v) {
   if (rows.empty()) return cudaSuccess;
   auto up = [&](const std::vector<int32_t>& h, const int32_t** d) -> cudaError_t {
     void* p = nullptr;
-    cudaError_t e2 = cudaMalloc(&p, sizeof(int32_t) * h.size());
+    cudaError_t e2 = cudaMallocAsync(&p, sizeof(int32_t) * h.size(), s);
     if (e2 != cudaSuccess) return e2;
     gr->extra.push_back(p);
     *d = static_cast<const int32_t*>(p);
-    return cudaMemcpy(p, h.data(), sizeof(int32_t) * h.size(), cudaMemcpyHostToDevice);
+    return cudaMemcpyAsync(p, h.data(), sizeof(int32_t) * h.size(), cudaMemcpyHostToDevice, s);
   };
   if ((e = up(rows, &v.long_rows)) || (e = up(seg, &v.long_seg)) || (e = up(segrow, &v.seg_row)))
     return e;
   void* part = nullptr;
-  if ((e = cudaMalloc(&part, sizeof(float) * (size_t)seg.back() * 2 * 256))) return e;
+  if ((e = cudaMallocAsync(&part, sizeof(float) * (size_t)seg.back() * 2 * 256, s))) return e;
   gr->extra.push_back(part);
   v.long_part = static_cast<float*>(part);
   v.nlong = (int32_t)rows.size();
   v.nseg = seg.back();
-  return cudaSuccess;
+  return cudaStreamSynchronize(s);   // the host vectors go out of scope
 }
 
 struct Workspace {
@@ -610,7 +628,7 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   v.bucket_off = gr->bucket_off;
   v.bucket_log2 = gr->bucket_log2;
   v.gsize = gr->gsize;
-  CK(build_long_rows(gr, v));
+  CK(build_long_rows(gr, v, s));
   *out = guard.release();
   return MARS_OK;
 }
@@ -1606,7 +1624,7 @@ extern "C" mars_status mars_graph_load_shard(const mars_graph_desc* desc, int32_
   v.chunk_graph = g->l_chunk_graph;
   v.graph_chunk = g->l_graph_chunk;
   v.gsize = g->gsize;                    // N of the whole graph (readout mean, loss scale)
-  CK(build_long_rows(g, v));             // of the local rows
+  CK(build_long_rows(g, v, s));          // of the local rows
   *out = guard.release();
   return MARS_OK;
 }

@@ -826,6 +826,23 @@ __global__ void k_colperm(const int32_t* __restrict__ rowptr, const int32_t* __r
   colperm[k] = perm[colind[k]];
 }
 
+// max over the view's rows of rowptr[i+1] - rowptr[i] (into *out, zeroed here).
+__global__ void k_max_degree(const int32_t* __restrict__ rowptr, int32_t Nt, int32_t* out) {
+  int32_t m = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < Nt;
+       i += (int64_t)gridDim.x * blockDim.x)
+    m = max(m, rowptr[i + 1] - rowptr[i]);
+  m = __reduce_max_sync(kFull, (unsigned)m);
+  if ((threadIdx.x & 31) == 0 && m > 0) atomicMax(out, m);
+}
+
+cudaError_t launch_max_degree(const int32_t* rowptr, int32_t Nt, int32_t* out, cudaStream_t s) {
+  cudaError_t e = cudaMemsetAsync(out, 0, sizeof(int32_t), s);
+  if (e != cudaSuccess) return e;
+  k_max_degree<<<std::min<unsigned>(cdiv(Nt, 256), 1184), 256, 0, s>>>(rowptr, Nt, out);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_colperm(const GraphDev& g, const int32_t* perm, int32_t* colperm,
                            cudaStream_t s, int* launches) {
   count_launch(launches);
