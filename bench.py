@@ -519,7 +519,7 @@ def main():
     ap.add_argument("--gemm", default="auto", choices=["auto", "simt"],
                     help="dense-transform kernels: tcgen05 3xFP16 with power-of-two scaling (auto) or FFMA (simt)")
     ap.add_argument("--profile-steps", type=int, default=5)
-    ap.add_argument("--e2e-steps", type=int, default=20)
+    ap.add_argument("--e2e-steps", type=int, default=40)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-bf16", action="store_true", help="skip the bf16-path measurement")
