@@ -9,7 +9,14 @@ graphs per GPU (one (graph, sample) pair each, weak scaling).  `value` counts
 per-graph DGI steps per second over the whole job (N x 16 x K / time).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
-  torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU, NCCL)
+  torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU)
+
+`--gpus N` without a torchrun environment re-launches itself under
+`python -m torch.distributed.run --nproc-per-node N` (fails loudly if fewer
+than N GPUs are visible).  Graphs are assigned to ranks by deterministic LPT
+on their size (dp.lpt_assign), each keeping its global pair index; the
+gradient exchange is libmars's peer-memory kernel (`--dp peer`, default) or
+an NCCL allreduce (`--dp nccl`).
 
 Device time: CUDA events on the stream the library launches on (torch's
 current stream, handed to libmars), barrier + synchronize on both sides, max
@@ -211,18 +218,25 @@ def run_mine(args):
     from synth import graphs as SG
 
     rank, world, local = dp.env()
+    if world > 1:                     # NCCL communicator lines (incl. nranks) in the log
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     if world != args.gpus:
-        args.gpus = world
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     b = args.graphs_per_gpu
     gen, _, _, _, desc = WORKLOADS[args.workload]
     sharded = args.workload == "1m" and world > 1
+    mine = None
     if args.workload == "1m":
         graphs = [SG.make("1m", 0)]           # ~7 s to generate; one graph for the whole job
     else:
-        graphs = [SG.cached(gen, i) for i in dp.graph_indices(rank, world, b)]
+        # LPT on graph size over the job's world*b graphs; graph i keeps pair index i
+        costs = [dp.graph_cost(SG.cached(gen, i)) for i in range(world * b)]
+        mine = dp.lpt_assign(costs, world, b)[rank]
+        graphs = [SG.cached(gen, i) for i in mine]
     if sharded:
         # rank r owns row block r of the one graph; the peers'
         # activation buffers are opened over CUDA IPC (NVLink peer memory)
@@ -235,10 +249,13 @@ def run_mine(args):
         shard_info = mars.graph_shard_info(g)
         uid = None
     else:
-        uid = dp.broadcast_unique_id(mars.nccl_get_unique_id)
+        uid = dp.broadcast_unique_id(mars.nccl_get_unique_id) if args.dp == "nccl" else None
         g = mars.graph_load(graphs, device=local)
+        g.set_pair_offsets(mine)
         m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local, world_size=world,
                             rank=rank, nccl_unique_id=uid)
+        if world > 1 and args.dp == "peer":
+            dp.connect_peers(m)
         shard_info = None
     info = g.info()
     if not sharded:
@@ -248,7 +265,7 @@ def run_mine(args):
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
     m.set_stream(stream.cuda_stream)
-    base, B = (0, 1) if sharded else dp.pair_range(rank, world, b)
+    base, B = (0, 1) if sharded else (0, world * b)
     for w in range(args.warmup):
         m.step(g, w, base, B)
     torch.cuda.synchronize()
@@ -386,6 +403,7 @@ def run_mine(args):
             pg.indices = torch.from_numpy(np.ascontiguousarray(gr.indices)).pin_memory().numpy()
             pg.features = torch.from_numpy(np.ascontiguousarray(gr.features)).pin_memory().numpy()
             pinned.append(pg)
+        offs = np.ascontiguousarray(mine, np.int64)
         h2d = sum(gr.indptr.nbytes + gr.indices.nbytes + gr.features.nbytes for gr in pinned)
         ke = max(1, min(args.steps, args.e2e_steps))
         m2 = mars.dgi_create(in_dim=F, hidden_dim=H, seed=args.seed, device=local,
@@ -393,6 +411,7 @@ def run_mine(args):
         m2.set_gemm_impl(args.gemm)
         m2.set_stream(stream.cuda_stream)
         gg = mars.graph_load(pinned, device=local)          # warm allocator pool
+        gg.set_pair_offsets(offs)
         m2.step(gg, 0, base, B, want_loss=True)
         gg.free()
         torch.cuda.synchronize()
@@ -403,9 +422,13 @@ def run_mine(args):
         # back (D2H).  Every step's inputs are still copied inside the timed region.
         t0 = time.perf_counter()
         gg = mars.graph_load(pinned, device=local)
+        gg.set_pair_offsets(offs)
         for k in range(ke):
             m2.step(gg, 1 + k, base, B)
-            nxt = mars.graph_load(pinned, device=local) if k + 1 < ke else None
+            nxt = None
+            if k + 1 < ke:
+                nxt = mars.graph_load(pinned, device=local)
+                nxt.set_pair_offsets(offs)
             loss_k, _ = m2.read_step(want_grads=False)
             gg.free()
             gg = nxt
@@ -486,6 +509,10 @@ def run_mine(args):
                            "graphs_per_gpu": b, "F": F, "H": H,
                            "nodes_per_gpu": N, "nnz_per_gpu": Z, "global_batch": B,
                            "parallelism": f"rowshard{world}" if sharded else f"dp{world}",
+                           "dp_exchange": None if sharded or world == 1 else
+                           ("libmars peer-memory kernel (rank-ordered fp64 sum over NVLink, "
+                            "2 device barriers)" if args.dp == "peer" else "NCCL allreduce"),
+                           "graph_assignment": None if sharded else "LPT on N+2E, global pair ids",
                            "shard": shard_info,
                            "l2": (("inputs larger than L2 (activations ~%.2f GB/step)"
                                    if 2 * N * 4 * (F + 7 * H) > 126e6 else
@@ -523,6 +550,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-bf16", action="store_true", help="skip the bf16-path measurement")
+    ap.add_argument("--dp", default="peer", choices=["peer", "nccl"],
+                    help="gradient exchange for N > 1: libmars peer-memory kernel or NCCL allreduce")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -530,9 +559,36 @@ def main():
     _, bdef, F, H, _ = WORKLOADS[args.workload]
     if args.graphs_per_gpu is None:
         args.graphs_per_gpu = bdef
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch(args)
     if args.impl == "reference":
         return run_reference(args)
     return run_mine(args)
+
+
+def relaunch(args):
+    """`--gpus N` outside torchrun: one rank per GPU under torch.distributed.run."""
+    import socket
+    try:
+        import torch
+        ngpu = torch.cuda.device_count()
+    except Exception:
+        ngpu = 0
+    if ngpu < args.gpus:
+        print(f"bench.py: --gpus {args.gpus} needs {args.gpus} visible GPUs, found {ngpu}",
+              file=sys.stderr, flush=True)
+        return 2
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")            # communicator lines (nranks) in the log
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr=127.0.0.1", f"--master-port={port}",
+           os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd, env=env)
 
 
 if __name__ == "__main__":

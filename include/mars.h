@@ -112,15 +112,20 @@ typedef struct {
   const float* init_params;   /* optional [P] host; NULL => Xavier-uniform(seed) */
   int32_t device;             /* CUDA device ordinal                           */
   int32_t world_size, rank;   /* data parallelism; 1, 0 for a single GPU       */
-  const void* nccl_unique_id; /* 128-byte ncclUniqueId; required when world_size > 1, optional with 1 (1-rank communicator) */
+  const void* nccl_unique_id; /* 128-byte ncclUniqueId: the gradient exchange is an NCCL
+                                 allreduce (optional with world_size 1: a 1-rank
+                                 communicator).  NULL with world_size > 1: peer-memory
+                                 exchange (mars_dp_export / mars_dp_connect below). */
 } mars_dgi_config;
 
 /* Fills cfg with the defaults above (F = 64, H = 256, L = 3, FP32, seed 0,
  * device 0, world 1). */
 MARS_API void mars_dgi_config_default(mars_dgi_config* cfg);
 /* Allocates params (init per c14 unless init_params), Adam state (m = v = 0,
- * t = 0) and a library stream on cfg->device; with world_size > 1 joins the
- * NCCL communicator (ncclCommInitRank; every rank must call collectively). */
+ * t = 0) and a library stream on cfg->device; with world_size > 1 and an
+ * nccl_unique_id joins the NCCL communicator (ncclCommInitRank; every rank
+ * must call collectively); with world_size > 1 and no id allocates the
+ * peer-visible buffers of the peer-memory exchange (connect before stepping). */
 MARS_API mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** out);
 /* Rank 0 only: writes a fresh 128-byte ncclUniqueId to out128. */
 MARS_API mars_status mars_nccl_get_unique_id(void* out128);
@@ -129,14 +134,12 @@ MARS_API mars_status mars_nccl_get_unique_id(void* out128);
 MARS_API mars_status mars_dgi_set_stream(mars_dgi* m, void* cuda_stream);
 /* Dense-transform implementation (a6/a12) of the MARS_FP32 path.
  * MARS_GEMM_AUTO (default), when H in {128, 256} and C_in in {64, 128, 256}:
- *   tcgen05 tensor cores at fp32 accuracy -- the row GEMMs (Z = Y·W,
- *   dY = dZ·Wᵀ) as 3xFP16 with exact power-of-two row / tensor scaling
- *   (kind::f16, twice the tf32 rate), the weight gradient as 3xTF32;
- *   FFMA otherwise.
- * MARS_GEMM_SIMT: always FFMA.
- * MARS_GEMM_3XTF32: every tensor-core GEMM as 3xTF32 (kind::tf32).
+ *   tcgen05 tensor cores at fp32 accuracy -- Z = Y·W, dY = dZ·Wᵀ and
+ *   dW = Yᵀ·dZ as 3xFP16 with exact power-of-two row / tensor scaling
+ *   (kind::f16); FFMA for the other widths (H in {32, 64}, C_in in {16, 32}).
+ * MARS_GEMM_SIMT: always FFMA (A/B comparisons).
  * (The MARS_BF16 path always uses its bf16 kernels.) */
-enum { MARS_GEMM_AUTO = 0, MARS_GEMM_SIMT = 1, MARS_GEMM_3XTF32 = 2 };
+enum { MARS_GEMM_AUTO = 0, MARS_GEMM_SIMT = 1 };
 MARS_API mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl);
 /* Enables (1) / disables (0) CUDA-Graph capture of the step (default 1). */
 MARS_API mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable);
@@ -183,6 +186,20 @@ MARS_API mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* embedd
  * `layer` in 1..3, stacked [pos; neg]: Y [2ΣN × C_in], Z [2ΣN × H] (host,
  * fp32; either may be NULL). */
 MARS_API mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t layer, float* Y, float* Z);
+/* Rows per branch (ΣN, or the shard's own rows) of the activations the last
+ * step saved -- the row count of the export hooks' [pos; neg] arrays is twice
+ * this; 0 after mars_encode (which overwrites them). */
+MARS_API mars_status mars_dgi_saved_rows(const mars_dgi* m, int64_t* rows_per_branch);
+/* Test hook (parity P3 at the bench size): with keep != 0 every later step also
+ * copies its backward intermediates -- dZ_l (l = 3, 2, 1) and dY_l = dZ_l W_lᵀ
+ * (l = 3, 2), which the step overwrites in place -- into separate device
+ * buffers (5 × 2ΣN × H elements, allocated on the next step).  A debugging aid:
+ * it adds 5 device-to-device copies per step.  keep = 0 releases them. */
+MARS_API mars_status mars_dgi_set_keep_backward(mars_dgi* m, int32_t keep);
+/* The last step's kept dZ_layer [2ΣN × H] and, for layer in {2, 3}, dY_layer
+ * [2ΣN × H] (host fp32; either may be NULL; dY must be NULL for layer 1).
+ * MARS_ESTATE unless keep_backward was on for that step. */
+MARS_API mars_status mars_dgi_export_backward(const mars_dgi* m, int32_t layer, float* dY, float* dZ);
 
 /* Checkpoint / resume: params, Adam m and v ([P] each) and step count t. */
 MARS_API mars_status mars_dgi_get_state(const mars_dgi* m, float* params, float* adam_m, float* adam_v,
@@ -224,6 +241,37 @@ MARS_API mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, uin
 MARS_API mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl, const float* A,
                                      const float* B, float* C, int64_t M, int32_t N, int32_t K,
                                      int32_t iters, float* ms);
+
+/* ------------------------------------------------------------------------ */
+/* Data parallelism over peer memory (a13): the R ranks of  */
+/* a job (one process per GPU, world_size R > 1, no nccl_unique_id) map each */
+/* other's gradient buffers (CUDA IPC; NVLink / NVSwitch between GPUs, or     */
+/* the same device).  After its backward every rank signals a device-side    */
+/* barrier, then sums the R partial gradient vectors (+ loss; each already   */
+/* scaled by 1/B_global) in rank order in fp64 -- identical on every rank, so */
+/* the replicated Adam keeps identical parameters -- and a second barrier     */
+/* releases the buffers for the next step.  One kernel reads the peers'      */
+/* partials directly: no staging copies, no host involvement, captured in    */
+/* the step's CUDA Graph.  A barrier wait longer than ~20 s sets an error     */
+/* flag (MARS_ECUDA from mars_dgi_read_step) instead of hanging.             */
+/* Protocol: mars_dgi_create (world_size R, rank r, same seed on every rank) */
+/* -> mars_dp_export (mars_dp_blob_bytes() bytes) -> all-gather the blobs in */
+/* rank order (e.g. torch.distributed) -> mars_dp_connect -> mars_dgi_step on */
+/* every rank with the same step index (steps wait on device for the peers). */
+/* ------------------------------------------------------------------------ */
+MARS_API int64_t mars_dp_blob_bytes(void);
+/* Writes this rank's CUDA IPC handles (gradients, barrier flags) into blob. */
+MARS_API mars_status mars_dp_export(const mars_dgi* m, void* blob);
+/* blobs: the R ranks' blobs concatenated in rank order.  EINVAL if they do
+ * not describe the same job (world size, ranks, parameter count). */
+MARS_API mars_status mars_dp_connect(mars_dgi* m, const void* blobs);
+
+/* Global pair indices of the graphs of a set (c15): graph i's corruption
+ * seed uses pair index global_pair_base + pair_offsets[i] (default i).  With
+ * a balanced (e.g. LPT) assignment of graphs to ranks, passing each graph's
+ * global index keeps every graph's corruption independent of the rank count.
+ * Host array [num_graphs], each >= 0.  Takes effect from the next step. */
+MARS_API mars_status mars_graph_set_pair_offsets(mars_graph* g, const int64_t* pair_offsets);
 
 /* Copies the most recent step's loss and global-mean gradient (the values
  * Adam consumed) to host memory (either may be NULL).  Synchronous.  For a

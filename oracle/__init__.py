@@ -76,6 +76,8 @@ def lib():
             L.oracle_spmm_rows.restype = None
             L.oracle_spmm_rows.argtypes = [ctypes.c_int32, i32p, i32p, ctypes.c_int32, f64p,
                                            ctypes.c_double, ctypes.c_int64, i64p, f64p]
+            L.oracle_prelu_backward.restype = ctypes.c_double
+            L.oracle_prelu_backward.argtypes = [ctypes.c_int64, f64p, f64p, ctypes.c_double, f64p]
             L.oracle_dense_anorm.restype = None
             L.oracle_dense_anorm.argtypes = [ctypes.c_int32, i32p, f64p]
             L.oracle_dense_step.restype = ctypes.c_double
@@ -232,6 +234,16 @@ def spmm_rows(batch: Batch, T, rows, alpha=None) -> np.ndarray:
     lib().oracle_spmm_rows(batch.Nt, batch.rowptr, batch.colind, T.shape[1], T,
                            float("nan") if alpha is None else float(alpha), rows.size, rows, out)
     return out
+
+
+def prelu_backward(dH, Z, alpha: float):
+    """Row a12's PReLU stage (c6): (dZ = dH ⊙ PReLU'(Z), Σ_{Z<=0} dH·Z)."""
+    dH = np.ascontiguousarray(dH, np.float64)
+    Z = np.ascontiguousarray(Z, np.float64)
+    assert dH.shape == Z.shape
+    dZ = np.zeros_like(dH)
+    da = lib().oracle_prelu_backward(dH.size, dH, Z, float(alpha), dZ)
+    return dZ, float(da)
 
 
 def encode(batch: Batch, H: int, params) -> np.ndarray:

@@ -36,11 +36,14 @@ __device__ __forceinline__ float prelu(float z, float a) { return z > 0.f ? z : 
 // m·scale lies in [2^14, 2^15) (below fp16's 65504); 1 for non-finite m.
 // An all-zero row gets the largest scale 2^100 (its products stay 0, and a
 // min-reduction over row scales -- k_tc3h_dw -- is not pulled down by it).
+// Large rows are never clamped (e <= 127 gives a normal 2^-113), so no finite
+// row can scale past fp16's range; tiny rows (e < -86) are clamped at 2^100
+// and keep their precision relative to 2^-86 (absolute, below ~2^-108).
 __device__ __forceinline__ float pow2_scale(float m) {
   if (m == 0.f) return 0x1p100f;
   if (!(m > 0.f) || !(m < INFINITY)) return 1.f;
   const int e = ilogbf(m);
-  const int sh = min(100, max(-100, 14 - e));
+  const int sh = min(100, 14 - e);
   return ldexpf(1.f, sh);
 }
 

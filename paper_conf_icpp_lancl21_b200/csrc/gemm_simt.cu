@@ -1,7 +1,9 @@
 // a6 / a12: the dense transforms of Eq. 1 (Z_l = Y_l · W_l) and their
 // backward (dY_l = dZ_l · W_lᵀ, dW_l = Y_lᵀ · dZ_l) in fp32 FFMA -- the fp32
-// reference-precision path (reading c18).  tf32 tensor cores cannot meet the
-// 1e-5 bar; the tcgen05 kernels (gemm_tc.cu) serve the bf16 path.
+// reference-precision path (reading c18) for the widths the tcgen05 kernels do
+// not cover (H in {32, 64}, C_in in {16, 32}: the tiny configuration) and for
+// MARS_GEMM_SIMT A/B runs; plain tf32 tensor cores could not meet the 1e-5
+// bar.
 //
 // gemm_nn / gemm_nt: 128-row CTA tiles, the whole W tile column block staged
 // through shared memory 16 K-rows at a time, 8×8 (or 8×4 / 4×4) register

@@ -8,9 +8,9 @@
 // max 65504) and a value 2^-28 of its row maximum is still a normal fp16.
 // Then x = hi + lo with hi = fp16_rn(x), lo = fp16_rn(x - hi) (x - hi exact in
 // fp32), and D += A_hi·B_hi + A_hi·B_lo + A_lo·B_hi in fp32 TMEM, C = D / (s_r t)
-// (exact).  hi and lo carry 11 significant bits each, like tf32 hi/lo, so the
-// error budget of the 3xTF32 kernel holds: the dropped lo·lo
-// term and the rounding of lo are ~2^-22 relative to the row's scale.
+// (exact).  hi and lo carry 11 significant bits each, so the dropped lo·lo
+// term and the rounding of lo are ~2^-22 relative to the row's scale
+// (the same budget as a 3xTF32 split, at twice its MMA rate).
 //
 // k_tc3h_rows: persistent over 128-row tiles.  Warp 0 TMA (fp32 A K-blocks of
 // 32 columns, 128-byte swizzle; pre-split fp16 B hi/lo, 64-byte swizzle),

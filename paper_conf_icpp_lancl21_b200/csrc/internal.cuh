@@ -16,9 +16,19 @@ struct StepParams {
   uint64_t step_index;
   int64_t pair_base;
   float inv_batch;      // 1 / global batch B
-  float adam_step_size; // lr / (1 - beta1^t)
-  float adam_bc2_sqrt;  // sqrt(1 - beta2^t)
   float pad;
+};
+
+// Adam's device-resident state (adam.cu): the step count and this step's bias
+// corrections, written by the guard kernel only when the loss and every
+// gradient are finite (otherwise skip = 1 and skipped counts the step).
+struct AdamDev {
+  int64_t t;            // completed updates (torch's state['step'])
+  int32_t skip;         // this step's update was skipped
+  int32_t skipped;      // total skipped updates
+  double clip_coef;     // min(1, clip / (||g|| + 1e-6))
+  float step_size;      // lr / (1 - beta1^t)
+  float bc2_sqrt;       // sqrt(1 - beta2^t)
 };
 
 // Device view of a loaded graph set (block-diagonal, global node ids).
@@ -53,6 +63,7 @@ struct GraphDev {
   const int32_t* bucket_off; // [G+1]
   const int32_t* bucket_log2;// [G]
   const int32_t* gsize;      // [G] node count N_g of each graph (all shards of a row-sharded graph)
+  const int64_t* pair_off;   // [G] pair index of graph g = pair_base + pair_off[g] (c15)
 };
 
 // ---------------------------------------------------------------- row sharding
@@ -87,9 +98,11 @@ cudaError_t launch_head_xsum(const PeerPtrs& x, int P, int H, int mode, const in
                              double* outd, float* outf, double* loss_g, cudaStream_t st,
                              int* launches);
 // out[k] = Σ_p g_p[k] (fp64, rank order) for k outside [keep_b, keep_e) and
-// k != n - 1; inside (dM, loss: already global on every shard) out[k] = g_me[k].
+// (unless sum_last) k != n - 1; the others (row-sharded graph: dM and the
+// loss, already global on every shard) out[k] = g_me[k].
 cudaError_t launch_grad_sum(const PeerPtrs& g, int P, int me, int64_t n, int64_t keep_b,
-                            int64_t keep_e, float* out, cudaStream_t st, int* launches);
+                            int64_t keep_e, int sum_last, float* out, cudaStream_t st,
+                            int* launches);
 
 // ---------------------------------------------------------------- builder.cu
 // Builds the CSR of Â for the packed set.  d_indptr: [Nt + G] int64 concatenated
@@ -185,17 +198,10 @@ size_t gemm_tn_partial_floats(int64_t R, int M, int N);
 cudaError_t gemm_tn(const float* A, const float* B, float* out, int64_t R, int M, int N,
                     double* partial, cudaStream_t s, int* launches);  // out[M×N] = Aᵀ B, A[R×M], B[R×N]
 
-// ---------------------------------------------------------------- gemm_tc.cu
-// 3xTF32 tcgen05 GEMMs (fp32-accurate).  Supported when H == 256 and
-// C_in in {64, 128, 256}.
+// ---------------------------------------------------------------- gemm_common.cu
+// tcgen05 GEMMs are specialised for H in {128, 256} and C_in in {64, 128, 256}.
 bool tc_supported(int cin, int h);
-cudaError_t tc_split_weights(const float* W, int CIN, int H, float* Bt_hi, float* Bt_lo,
-                             float* B_hi, float* B_lo, cudaStream_t s, int* launches);
-cudaError_t tc_gemm_rows(const float* A, const float* B_hi, const float* B_lo, float* C,
-                         int64_t M, int N, int K, cudaStream_t s, int* launches);
 size_t tc_dw_partial_floats(int64_t R, int CIN);
-cudaError_t tc_gemm_dw(const float* Y, const float* dZ, float* dW, int64_t R, int CIN, int H,
-                       float* part, cudaStream_t s, int* launches);
 // gemm_tc3h.cu: 3xFP16 row GEMMs with power-of-two scaling (fp32 path)
 cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void* Bt_hi,
                                void* Bt_lo, void* B_hi, void* B_lo, cudaStream_t s,
@@ -267,9 +273,10 @@ cudaError_t launch_prelu(const void* Z, int bf16, const float* alpha_dev, int la
 cudaError_t launch_upcast(const void* in, float* out, int64_t n, cudaStream_t s);
 
 // ---------------------------------------------------------------- adam.cu
+// grads: [P + 1], the loss at grads[P]; guard_part: adam_guard_doubles() doubles.
+int adam_guard_doubles();
 cudaError_t launch_adam(float* params, float* m, float* v, const float* grads, int64_t P,
-                        double beta1, double beta2, double eps, double clip_norm, double* norm_part,
-                        const StepParams* sp, cudaStream_t s, int* launches);
-cudaError_t launch_check_finite(const float* loss, int32_t* flag, cudaStream_t s, int* launches);
+                        double lr, double beta1, double beta2, double eps, double clip_norm,
+                        double* guard_part, AdamDev* st, cudaStream_t s, int* launches);
 
 }  // namespace mars

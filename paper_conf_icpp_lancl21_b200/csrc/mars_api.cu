@@ -191,6 +191,7 @@ struct mars_graph {
   int32_t *bucket_off = nullptr, *bucket_log2 = nullptr;
   float *vals = nullptr, *dinv = nullptr, *X = nullptr;
   int32_t* gsize = nullptr;
+  int64_t* pair_off = nullptr;      // [G] global pair index offsets (c15), default 0..G-1
   GraphDev dev{};
   // Row-sharded graph (mars_graph_load_shard): dev is the
   // view of this shard's rows [row_begin, row_end) (local row ids, global
@@ -202,21 +203,51 @@ struct mars_graph {
   GraphDev dev_full{};
   int32_t *l_node_off = nullptr, *l_node_graph = nullptr, *l_chunk_row = nullptr,
           *l_chunk_graph = nullptr, *l_graph_chunk = nullptr;
-  std::vector<void*> extra;         // long-row tables (cudaMalloc)
-  ~mars_graph() {   // pool memory; mars_free synchronises the device first
-    for (void* p : extra) cudaFreeAsync(p, nullptr);
+  std::vector<void*> extra;         // long-row tables (pool memory)
+  // Last use per stream: every step / encode that reads this graph records an
+  // event on its stream, so mars_free waits for exactly those uses (not for the
+  // whole device, which would serialise against other models' steps).
+  mutable std::mutex use_mu;
+  mutable std::vector<std::pair<cudaStream_t, cudaEvent_t>> uses;
+  void note_use(cudaStream_t s) const {
+    std::lock_guard<std::mutex> lk(use_mu);
+    for (auto& u : uses)
+      if (u.first == s) {
+        cudaEventRecord(u.second, s);
+        return;
+      }
+    cudaEvent_t e;
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
+      cudaGetLastError();
+      cudaStreamSynchronize(s);           // no event: wait for the stream instead
+      return;
+    }
+    cudaEventRecord(e, s);
+    uses.emplace_back(s, e);
+  }
+  ~mars_graph() {   // pool memory, freed on a private stream after the recorded uses
+    for (auto& u : uses) {
+      cudaEventSynchronize(u.second);
+      cudaEventDestroy(u.second);
+    }
+    cudaStream_t fs = nullptr;
+    if (cudaStreamCreateWithFlags(&fs, cudaStreamNonBlocking) != cudaSuccess) fs = nullptr;
+    for (void* p : extra) cudaFreeAsync(p, fs);
     for (void* p : {(void*)node_off, (void*)node_graph, (void*)rowptr, (void*)colind, (void*)deg,
                     (void*)chunk_row, (void*)chunk_graph, (void*)graph_chunk, (void*)bucket_off,
                     (void*)bucket_log2, (void*)vals, (void*)dinv, (void*)X, (void*)gsize,
-                    (void*)l_node_off, (void*)l_node_graph, (void*)l_chunk_row,
+                    (void*)pair_off, (void*)l_node_off, (void*)l_node_graph, (void*)l_chunk_row,
                     (void*)l_chunk_graph, (void*)l_graph_chunk})
-      if (p) cudaFreeAsync(p, nullptr);
+      if (p) cudaFreeAsync(p, fs);
+    if (fs) cudaStreamDestroy(fs);
   }
   const GraphDev& perm_view() const { return sharded ? dev_full : dev; }
 };
 
-// Long rows of a view (degree > long_min, spmm.cu): host scan of its rowptr,
-// segment tables and the fp32 partial-sum scratch on the device.
+// Long rows of a view (degree > long_min, spmm.cu): host scan of its rowptr and
+// the segment tables on the device (read-only; the fp32 partial-sum scratch
+// the segments write belongs to each model's Workspace, so models stepping the
+// same graph concurrently never share it).
 // Everything on the loader's non-blocking stream `s` (no legacy-stream copies or
 // cudaMalloc, which would wait for a model's step running concurrently).
 static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s) {
@@ -269,10 +300,6 @@ static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s) 
   };
   if ((e = up(rows, &v.long_rows)) || (e = up(seg, &v.long_seg)) || (e = up(segrow, &v.seg_row)))
     return e;
-  void* part = nullptr;
-  if ((e = cudaMallocAsync(&part, sizeof(float) * (size_t)seg.back() * 2 * 256, s))) return e;
-  gr->extra.push_back(part);
-  v.long_part = static_cast<float*>(part);
   v.nlong = (int32_t)rows.size();
   v.nseg = seg.back();
   return cudaStreamSynchronize(s);   // the host vectors go out of scope
@@ -283,6 +310,8 @@ struct Workspace {
   int32_t Nperm = 0;      // rows of the permutation (the whole graph when row-sharded)
   int64_t nnz_perm = 0;   // entries of the permuted view (colperm)
   int32_t nlong = 0;      // long rows (dalpha slots of the backward aggregation)
+  int32_t nseg = 0;       // long-row segments (long_part)
+  float* long_part = nullptr;   // [nseg * 2 * 256] fp32 segment partial sums (spmm.cu)
   float *Y1 = nullptr, *Z[3] = {nullptr, nullptr, nullptr}, *Y23[2] = {nullptr, nullptr};
   float *dZ = nullptr, *dY = nullptr;
   int32_t* perm = nullptr;
@@ -292,8 +321,6 @@ struct Workspace {
   double *slots[3] = {nullptr, nullptr, nullptr};
   double* tn_part = nullptr;
   size_t tn_part_n = 0;
-  // tcgen05 path: per-layer hi/lo weight splits (Wᵀ for the forward, W for dY)
-  float *wt_hi[3] = {}, *wt_lo[3] = {}, *w_hi[3] = {}, *w_lo[3] = {};
   // 3xFP16 row GEMMs: scaled fp16 hi/lo splits + {t, 1/t} per layer
   void *h3_wt_hi[3] = {}, *h3_wt_lo[3] = {}, *h3_w_hi[3] = {}, *h3_w_lo[3] = {};
   float* h3_wsc[3] = {};
@@ -317,11 +344,11 @@ struct mars_dgi {
   mars_dgi_config cfg{};
   int F = 0, H = 0;
   int64_t P = 0;
-  int64_t t = 0;
   cudaStream_t own_stream = nullptr, stream = nullptr;
   float *params = nullptr, *adam_m = nullptr, *adam_v = nullptr, *grads = nullptr;
-  double* norm_part = nullptr;
-  int32_t* finite_flag = nullptr;
+  double* guard_part = nullptr;      // [adam_guard_doubles()] finiteness / clip-norm partials
+  AdamDev* adam_st = nullptr;        // device-resident Adam step count + bias corrections
+  int32_t skipped_seen = 0;          // skipped updates already reported (MARS_ENUMERIC)
   StepParams* d_sp = nullptr;
   StepParams* h_sp = nullptr;       // pinned ring
   cudaEvent_t* sp_ev = nullptr;
@@ -329,13 +356,25 @@ struct mars_dgi {
   Workspace ws;
   const mars_graph* ws_graph = nullptr;
   bool capture = true;
-  int gemm_impl = 0;                // 0 auto (tcgen05 3xTF32 when supported), 1 SIMT FFMA
+  int gemm_impl = 0;                // 0 auto (tcgen05 3xFP16 when supported), 1 SIMT FFMA
   cudaGraphExec_t exec = nullptr;
   uint64_t exec_graph = 0;          // uid of the graph set the exec was captured for
   uint64_t prev_graph = 0;          // uid of the graph set of the previous step
   cudaStream_t exec_stream = nullptr;
   int64_t last_launches = 0, exec_launches = 0;
   int32_t last_Nt = 0;              // node count of the last step's graph set (export hook)
+  // keep_backward test hook: copies of dZ3, dZ2, dZ1 (kb_dZ[l]) and dY3, dY2
+  // (kb_dY[l - 1]) of the last step, 2 * kb_rows rows each
+  bool keep_bwd = false;
+  void *kb_dZ[3] = {}, *kb_dY[2] = {};
+  int64_t kb_rows = 0;              // rows per branch the buffers hold
+  int32_t kb_valid_Nt = 0;          // last_Nt of the step that filled them (0: none)
+  void kb_release() {
+    for (void*& p : kb_dZ) { if (p) cudaFree(p); p = nullptr; }
+    for (void*& p : kb_dY) { if (p) cudaFree(p); p = nullptr; }
+    kb_rows = 0;
+    kb_valid_Nt = 0;
+  }
   ncclComm_t comm = nullptr;
   // Row-sharded graph: the shard this model is attached to,
   // its peer-visible buffers, and the peers' buffers once connected.
@@ -355,14 +394,32 @@ struct mars_dgi {
     std::vector<void*> ipc;                // pointers opened with cudaIpcOpenMemHandle
     std::vector<void*> owned;
   } sh;
-  float* grads_final() const { return sh.connected ? sh.gsum : grads; }
+  // Data parallelism over peer memory (mars_dp_*): rank-ordered sum of the
+  // ranks' partial gradients (+ loss) between two device barriers.
+  struct Dp {
+    int32_t R = 1, me = 0;                 // world size, rank (R > 1: peer mode)
+    bool connected = false;
+    unsigned long long* flags = nullptr;   // [kMaxShards] arrival slots (peer-visible)
+    unsigned long long* epoch = nullptr;
+    int32_t* err = nullptr;
+    float* gsum = nullptr;                 // [P + 1] global gradient + loss
+    ShardSync sync{};
+    PeerPtrs grads{};
+    std::vector<void*> ipc, owned;
+  } dp;
+  float* grads_final() const {
+    return sh.connected ? sh.gsum : dp.connected ? dp.gsum : grads;
+  }
   ~mars_dgi() {
     if (exec) cudaGraphExecDestroy(exec);
+    kb_release();
     for (void* p : sh.ipc) cudaIpcCloseMemHandle(p);
     for (void* p : sh.owned) cudaFree(p);
+    for (void* p : dp.ipc) cudaIpcCloseMemHandle(p);
+    for (void* p : dp.owned) cudaFree(p);
     ws.release();
-    for (void* p : {(void*)params, (void*)adam_m, (void*)adam_v, (void*)grads, (void*)norm_part,
-                    (void*)finite_flag, (void*)d_sp})
+    for (void* p : {(void*)params, (void*)adam_m, (void*)adam_v, (void*)grads, (void*)guard_part,
+                    (void*)adam_st, (void*)d_sp})
       if (p) cudaFree(p);
     if (sp_ev) {
       for (int i = 0; i < sp_ring; ++i) cudaEventDestroy(sp_ev[i]);
@@ -503,6 +560,7 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   CK(palloc(&gr->bucket_off, (size_t)G + 1, s));
   CK(palloc(&gr->bucket_log2, (size_t)G, s));
   CK(palloc(&gr->gsize, (size_t)G, s));
+  CK(palloc(&gr->pair_off, (size_t)G, s));
 
   // Inputs in page-locked host memory are copied straight to the device;
   // otherwise they are packed into a pinned staging buffer first.
@@ -552,6 +610,9 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   std::vector<int32_t> gsize(G);
   for (int g = 0; g < G; ++g) gsize[g] = descs[g].num_nodes;
   CK(cudaMemcpyAsync(gr->gsize, gsize.data(), sizeof(int32_t) * G, cudaMemcpyHostToDevice, s));
+  std::vector<int64_t> poff(G);
+  for (int g = 0; g < G; ++g) poff[g] = g;
+  CK(cudaMemcpyAsync(gr->pair_off, poff.data(), sizeof(int64_t) * G, cudaMemcpyHostToDevice, s));
   k_node_graph<<<cdiv(Nt, 256), 256, 0, s>>>(gr->node_off, G, (int32_t)Nt, gr->node_graph);
   CK(cudaGetLastError());
 
@@ -628,6 +689,7 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   v.bucket_off = gr->bucket_off;
   v.bucket_log2 = gr->bucket_log2;
   v.gsize = gr->gsize;
+  v.pair_off = gr->pair_off;
   CK(build_long_rows(gr, v, s));
   *out = guard.release();
   return MARS_OK;
@@ -697,8 +759,8 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
     return fail(MARS_EINVAL, "MARS_BF16 needs hidden_dim in {128, 256} and in_dim in {64, 128, 256}");
   if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
     return fail(MARS_EINVAL, "bad world_size/rank");
-  if (cfg->world_size > 1 && !cfg->nccl_unique_id)
-    return fail(MARS_EINVAL, "world_size > 1 needs nccl_unique_id");
+  if (cfg->world_size > kMaxShards && !cfg->nccl_unique_id)
+    return fail(MARS_EINVAL, "peer-memory data parallelism supports world_size <= %d", kMaxShards);
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
     cudaGetLastError();
@@ -720,8 +782,8 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   CK(dalloc(&m->adam_m, m->P));
   CK(dalloc(&m->adam_v, m->P));
   CK(dalloc(&m->grads, m->P + 1));
-  CK(dalloc(&m->norm_part, 160));
-  CK(dalloc(&m->finite_flag, 1));
+  CK(dalloc(&m->guard_part, (size_t)adam_guard_doubles()));
+  CK(dalloc(&m->adam_st, 1));
   CK(dalloc(&m->d_sp, 1));
   CK(cudaMallocHost(&m->h_sp, sizeof(StepParams) * m->sp_ring));
   m->sp_ev = new cudaEvent_t[m->sp_ring];
@@ -733,6 +795,7 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   CK(cudaMemsetAsync(m->adam_m, 0, sizeof(float) * m->P, s));
   CK(cudaMemsetAsync(m->adam_v, 0, sizeof(float) * m->P, s));
   CK(cudaMemsetAsync(m->grads, 0, sizeof(float) * (m->P + 1), s));
+  CK(cudaMemsetAsync(m->adam_st, 0, sizeof(AdamDev), s));
   if (cfg->init_params) {
     CK(cudaMemcpyAsync(m->params, cfg->init_params, sizeof(float) * m->P, cudaMemcpyHostToDevice, s));
   } else {
@@ -748,9 +811,28 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
     CK(cudaGetLastError());
   }
   CK(cudaStreamSynchronize(s));
-  // world_size > 1 needs a communicator; with world_size == 1 an id may still
-  // be passed to run the (identity) allreduce path, which the tests use.
-  if (cfg->world_size > 1 || cfg->nccl_unique_id) {
+  if (cfg->world_size > 1 && !cfg->nccl_unique_id) {      // peer-memory exchange
+    mars_dgi::Dp& d = m->dp;
+    d.R = cfg->world_size;
+    d.me = cfg->rank;
+    auto al = [&](void** p, size_t bytes) -> cudaError_t {
+      cudaError_t e = cudaMalloc(p, bytes);
+      if (e == cudaSuccess) d.owned.push_back(*p);
+      return e;
+    };
+    CK(al((void**)&d.flags, sizeof(unsigned long long) * kMaxShards));
+    CK(al((void**)&d.epoch, sizeof(unsigned long long)));
+    CK(al((void**)&d.err, sizeof(int32_t)));
+    CK(al((void**)&d.gsum, sizeof(float) * (m->P + 1)));
+    CK(cudaMemset(d.flags, 0, sizeof(unsigned long long) * kMaxShards));
+    CK(cudaMemset(d.epoch, 0, sizeof(unsigned long long)));
+    CK(cudaMemset(d.err, 0, sizeof(int32_t)));
+    CK(cudaMemset(d.gsum, 0, sizeof(float) * (m->P + 1)));
+    CK(cudaDeviceSynchronize());
+  }
+  // an NCCL id makes the exchange an NCCL allreduce; with world_size == 1 an
+  // id may still be passed to run the (identity) allreduce path (tests).
+  if (cfg->nccl_unique_id) {
     if (!nccl_load()) return fail(MARS_ENCCL, "libnccl.so.2 not loadable");
     ncclUniqueId id;
     memcpy(&id, cfg->nccl_unique_id, sizeof id);
@@ -771,7 +853,7 @@ extern "C" mars_status mars_dgi_set_stream(mars_dgi* m, void* stream) {
 
 extern "C" mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl) {
   if (mars_status st = check_dgi(m)) return st;
-  if (impl != MARS_GEMM_AUTO && impl != MARS_GEMM_SIMT && impl != MARS_GEMM_3XTF32)
+  if (impl != MARS_GEMM_AUTO && impl != MARS_GEMM_SIMT)
     return fail(MARS_EINVAL, "bad gemm impl");
   if (impl != m->gemm_impl && m->exec) {
     cudaGraphExecDestroy(m->exec);
@@ -789,11 +871,29 @@ extern "C" mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable) {
 }
 
 // ---------------------------------------------------------------- workspaces
+static mars_status ensure_kb(mars_dgi* m, const mars_graph* g) {
+  if (!m->keep_bwd || m->kb_rows >= g->dev.Nt) return MARS_OK;
+  if (m->exec) {                 // a captured step without the copies
+    cudaGraphExecDestroy(m->exec);
+    m->exec = nullptr;
+    m->exec_graph = 0;
+  }
+  CK(cudaStreamSynchronize(m->stream));
+  m->kb_release();
+  const size_t bytes = sizeof(float) * 2 * (size_t)g->dev.Nt * m->H;
+  for (void*& p : m->kb_dZ) CK(cudaMalloc(&p, bytes));
+  for (void*& p : m->kb_dY) CK(cudaMalloc(&p, bytes));
+  m->kb_rows = g->dev.Nt;
+  return MARS_OK;
+}
+
 static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
+  if (mars_status st = ensure_kb(m, g)) return st;
   Workspace& w = m->ws;
   const GraphDev& pv = g->perm_view();
   if (w.Nt >= g->dev.Nt && w.Nperm >= pv.Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks &&
       w.nbuckets >= pv.nbuckets && w.nnz_perm >= pv.nnz && w.nlong >= g->dev.nlong &&
+      w.nseg >= g->dev.nseg &&
       w.F == m->F && w.H == m->H)
     return MARS_OK;
   if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
@@ -817,6 +917,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   CK(al((void**)&w.dZ, sizeof(float) * R * H));
   CK(al((void**)&w.dY, sizeof(float) * R * H));
   CK(al((void**)&w.perm, sizeof(int32_t) * Np));
+  CK(al((void**)&w.long_part, sizeof(float) * (size_t)g->dev.nseg * 2 * 256));
   CK(al((void**)&w.colperm, sizeof(int32_t) * (size_t)std::max<int64_t>(1, pv.nnz)));
   CK(al((void**)&w.pw.keys, sizeof(uint64_t) * Np));
   CK(al((void**)&w.pw.bucket, sizeof(int32_t) * Np));
@@ -845,10 +946,6 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   w.tn_part_n = tn;
   for (int l = 0; l < 3; ++l) {
     int64_t n = (int64_t)(l == 0 ? F : H) * H;
-    CK(al((void**)&w.wt_hi[l], sizeof(float) * n));
-    CK(al((void**)&w.wt_lo[l], sizeof(float) * n));
-    CK(al((void**)&w.w_hi[l], sizeof(float) * n));
-    CK(al((void**)&w.w_lo[l], sizeof(float) * n));
     CK(al(&w.h3_wt_hi[l], 2 * n));
     CK(al(&w.h3_wt_lo[l], 2 * n));
     CK(al(&w.h3_w_hi[l], 2 * n));
@@ -872,6 +969,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   w.Nperm = (int32_t)Np;
   w.nnz_perm = pv.nnz;
   w.nlong = g->dev.nlong;
+  w.nseg = g->dev.nseg;
   w.G = G;
   w.nchunks = nch;
   w.nbuckets = nb;
@@ -902,8 +1000,9 @@ struct Profiler {
 // Enqueues one full DGI step (a4-a14) on stream s.  Reads step scalars from m->d_sp.
 static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl,
                                 Profiler* prof = nullptr) {
-  const GraphDev& g = gr->dev;
   Workspace& w = m->ws;
+  GraphDev g = gr->dev;
+  g.long_part = w.long_part;
   const int F = m->F, H = m->H;
   const int64_t R = 2LL * g.Nt;
   float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
@@ -934,16 +1033,13 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   MARK(MARS_PH_PERM);
   const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
-  const bool h3 = m->gemm_impl == MARS_GEMM_AUTO;       // 3xFP16 row GEMMs (fp32 path)
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
     if (b16) RET(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl));
-    else if (tc[l] && h3)
+    else if (tc[l])
       RET(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
                              w.h3_w_hi[l], w.h3_w_lo[l], s, nl));
-    else if (tc[l])
-      RET(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, nl));
   }
   MARK(MARS_PH_GEMM_FWD);
   // a5-a7: forward, l = 1..3
@@ -956,13 +1052,12 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     }
     RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.colperm, alpha, l - 1, Ys[l], b16, 1, s, nl,
                         shard && l > 0 ? &m->sh.z[l - 1] : nullptr,
-                        tc[l] && h3 ? w.h3_rsY[l] : nullptr));
+                        tc[l] ? w.h3_rsY[l] : nullptr));
     MARK(MARS_PH_SPMM_FWD);
     if (b16) RET(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], R, H, Cin, s, nl));
-    else if (tc[l] && h3)
+    else if (tc[l])
       RET(tc3h_gemm_rows(Ys[l], w.h3_rsY[l], w.h3_wt_hi[l], w.h3_wt_lo[l], w.h3_wsc[l] + 1,
                          w.Z[l], R, H, Cin, s, nl));
-    else if (tc[l]) RET(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], R, H, Cin, s, nl));
     else RET(gemm_nn(Ys[l], W[l], w.Z[l], R, H, Cin, s, nl));
     MARK(MARS_PH_GEMM_FWD);
   }
@@ -976,29 +1071,32 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     hs.x_peers[0] = m->sh.x[0];
     hs.x_peers[1] = m->sh.x[1];
   }
-  w.hw.rs_dz3 = !b16 && tc[2] && h3 ? w.h3_rsdZ : nullptr;   // dZ3 row scales (3xFP16 dY GEMM)
+  w.hw.rs_dz3 = !b16 && tc[2] ? w.h3_rsdZ : nullptr;   // dZ3 row scales (3xFP16 dY GEMM)
   RET(launch_head(g, H, w.Z[2], b16, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl,
                   shard ? &hs : nullptr));
   RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
+  const size_t es = b16 ? 2 : 4;                         // storage bytes per element
+  const size_t kb_bytes = (size_t)R * H * es;
+  const bool kb = m->keep_bwd && m->kb_rows >= g.Nt;
+  if (kb) RET(cudaMemcpyAsync(m->kb_dZ[2], w.dZ, kb_bytes, cudaMemcpyDeviceToDevice, s));
   MARK(MARS_PH_HEAD);
   // a12: backward, l = 3..1
   for (int l = 2; l >= 0; --l) {
     int Cin = l == 0 ? F : H;
     if (b16) RET(tc16_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, H, w.dw16_part, s, nl));
-    else if (tc[l] && h3)
+    else if (tc[l])
       RET(tc3h_gemm_dw(Ys[l], w.h3_rsY[l], w.dZ, w.h3_rsdZ, gW[l], R, Cin, H, w.dw_part, s, nl));
-    else if (tc[l]) RET(tc_gemm_dw(Ys[l], w.dZ, gW[l], R, Cin, H, w.dw_part, s, nl));
     else RET(gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl));
     MARK(MARS_PH_GEMM_DW);
     if (l > 0) {
       // sharded: the two backward aggregations use separate peer-visible dY buffers
       float* dYl = (shard && l == 1) ? static_cast<float*>(m->sh.dY2) : w.dY;
       if (b16) RET(tc16_gemm_rows(w.dZ, w.w16[l], dYl, R, Cin, H, s, nl));
-      else if (tc[l] && h3)
+      else if (tc[l])
         RET(tc3h_gemm_rows(w.dZ, w.h3_rsdZ, w.h3_w_hi[l], w.h3_w_lo[l], w.h3_wsc[l] + 1, dYl, R,
                            Cin, H, s, nl));
-      else if (tc[l]) RET(tc_gemm_rows(w.dZ, w.w_hi[l], w.w_lo[l], dYl, R, Cin, H, s, nl));
       else RET(gemm_nt(w.dZ, W[l], dYl, R, Cin, H, s, nl));
+      if (kb) RET(cudaMemcpyAsync(m->kb_dY[l - 1], dYl, kb_bytes, cudaMemcpyDeviceToDevice, s));
       MARK(MARS_PH_GEMM_DY);
       if (shard) {
         RET(launch_shard_barrier(m->sh.sync, s, nl));  // peers' dY_l complete
@@ -1006,7 +1104,8 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
       }
       RET(launch_spmm_bwd(g, Cin, dYl, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
                           s, nl, shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr,
-                          tc[l - 1] && h3 ? w.h3_rsdZ : nullptr));
+                          tc[l - 1] ? w.h3_rsdZ : nullptr));
+      if (kb) RET(cudaMemcpyAsync(m->kb_dZ[l - 1], w.dZ, kb_bytes, cudaMemcpyDeviceToDevice, s));
       MARK(MARS_PH_SPMM_BWD);
       RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
       MARK(MARS_PH_REDUCE);
@@ -1019,18 +1118,28 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
     if (r != ncclSuccess) return cudaErrorUnknown;
     MARK(MARS_PH_ALLREDUCE);
   }
+  // a13 over peer memory: barrier (every rank's partials complete), rank-ordered
+  // fp64 sum of the partial gradients + loss, barrier (every rank has read
+  // them, so the next step may overwrite its own)
+  if (m->dp.connected) {
+    RET(launch_shard_barrier(m->dp.sync, s, nl));
+    RET(launch_grad_sum(m->dp.grads, m->dp.R, m->dp.me, m->P + 1, 0, 0, 1, m->dp.gsum, s, nl));
+    RET(launch_shard_barrier(m->dp.sync, s, nl));
+    MARK(MARS_PH_ALLREDUCE);
+  }
   // row-sharded: sum the shards' W / alpha partials in rank order (dM and the
   // loss are already global on every shard after the head exchange)
   if (shard) {
     RET(launch_shard_barrier(m->sh.sync, s, nl));
     const int64_t mb = (int64_t)F * H + 2LL * H * H;
     RET(launch_grad_sum(m->sh.grads, m->sh.sync.P, m->sh.sync.me, m->P + 1, mb, mb + (int64_t)H * H,
-                        m->sh.gsum, s, nl));
+                        0, m->sh.gsum, s, nl));
     MARK(MARS_PH_EXCHANGE);
   }
   // a14: Adam
-  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads_final(), m->P, m->cfg.beta1,
-                  m->cfg.beta2, m->cfg.eps, m->cfg.clip_norm, m->norm_part, m->d_sp, s, nl));
+  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads_final(), m->P, m->cfg.lr,
+                  m->cfg.beta1, m->cfg.beta2, m->cfg.eps, m->cfg.clip_norm, m->guard_part,
+                  m->adam_st, s, nl));
   MARK(MARS_PH_ADAM);
 #undef MARK
 #undef RET
@@ -1042,7 +1151,6 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
 static mars_status push_step_params(mars_dgi* m, uint64_t step_index, int64_t pair_base,
                                     int64_t global_batch) {
   cudaStream_t s = m->stream;
-  m->t += 1;
   int slot = m->sp_next;
   m->sp_next = (m->sp_next + 1) % m->sp_ring;
   CK(cudaEventSynchronize(m->sp_ev[slot]));
@@ -1050,13 +1158,18 @@ static mars_status push_step_params(mars_dgi* m, uint64_t step_index, int64_t pa
   sp.step_index = step_index;
   sp.pair_base = pair_base;
   sp.inv_batch = (float)(1.0 / (double)global_batch);
-  double bc1 = 1.0 - std::pow((double)m->cfg.beta1, (double)m->t);
-  double bc2 = 1.0 - std::pow((double)m->cfg.beta2, (double)m->t);
-  sp.adam_step_size = (float)((double)m->cfg.lr / bc1);
-  sp.adam_bc2_sqrt = (float)std::sqrt(bc2);
   CK(cudaMemcpyAsync(m->d_sp, &sp, sizeof sp, cudaMemcpyHostToDevice, s));
   CK(cudaEventRecord(m->sp_ev[slot], s));
   return MARS_OK;
+}
+
+// A guarded Adam update was skipped (non-finite loss or gradient, adam.cu)
+// since the last report: MARS_ENUMERIC once per skipped batch of steps.
+static mars_status check_skipped(mars_dgi* m, int32_t skipped) {
+  if (skipped <= m->skipped_seen) return MARS_OK;
+  const int32_t n = skipped - m->skipped_seen;
+  m->skipped_seen = skipped;
+  return fail(MARS_ENUMERIC, "non-finite loss or gradient: %d Adam update(s) skipped", n);
 }
 
 static mars_status check_step_args(mars_dgi* m, const mars_graph* g, int64_t global_batch) {
@@ -1065,6 +1178,8 @@ static mars_status check_step_args(mars_dgi* m, const mars_graph* g, int64_t glo
   if (g->F != m->F) return fail(MARS_EINVAL, "graph feat_dim %d != model in_dim %d", g->F, m->F);
   if (g->device != m->cfg.device) return fail(MARS_EINVAL, "graph and model on different devices");
   if (global_batch < g->G) return fail(MARS_EINVAL, "global_batch < graphs in this set");
+  if (m->dp.R > 1 && !m->dp.connected)
+    return fail(MARS_ESTATE, "peer-memory data parallelism: mars_dp_connect first");
   return MARS_OK;
 }
 
@@ -1084,6 +1199,7 @@ extern "C" mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, u
     cudaGetLastError();
     return fail(MARS_ECUDA, "profile step: %s", cudaGetErrorString(e));
   }
+  g->note_use(m->stream);
   CK(cudaStreamSynchronize(m->stream));
   int n = 0;
   for (size_t k = 1; k < prof.ev.size() && n < max_phases; ++k, ++n) {
@@ -1095,6 +1211,7 @@ extern "C" mars_status mars_dgi_profile_step(mars_dgi* m, const mars_graph* g, u
   *n_phases = n;
   m->last_launches = nl;
   m->last_Nt = g->dev.Nt;
+  m->kb_valid_Nt = m->keep_bwd ? g->dev.Nt : 0;
   return MARS_OK;
 }
 
@@ -1110,7 +1227,9 @@ extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t 
   cudaStream_t s = m->stream;
   if (out && (out->loss || out->grads || out->perms)) {
     float loss = 0.f;
+    int32_t skipped = 0;
     CK(cudaMemcpyAsync(&loss, m->grads_final() + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+    CK(cudaMemcpyAsync(&skipped, &m->adam_st->skipped, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
     if (out->grads)
       CK(cudaMemcpyAsync(out->grads, m->grads_final(), sizeof(float) * m->P,
                          cudaMemcpyDeviceToHost, s));
@@ -1122,6 +1241,7 @@ extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t 
         for (int32_t i = g->h_node_off[gi]; i < g->h_node_off[gi + 1]; ++i)
           out->perms[i] -= g->h_node_off[gi];
     if (out->loss) *out->loss = loss;
+    if (mars_status st = check_skipped(m, skipped)) return st;
     if (!std::isfinite(loss)) return fail(MARS_ENUMERIC, "non-finite loss");
   }
   return MARS_OK;
@@ -1190,11 +1310,13 @@ extern "C" mars_status mars_dgi_pretrain(mars_dgi* m, const mars_graph* g, uint6
   if (best_params) CK(cudaMemcpyAsync(best_params, best, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
   CK(cudaMemcpyAsync(&bl, d_bl, sizeof(float), cudaMemcpyDeviceToHost, s));
   CK(cudaMemcpyAsync(&bs, d_bs, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+  int32_t skipped = 0;
+  CK(cudaMemcpyAsync(&skipped, &m->adam_st->skipped, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   if (best_loss) *best_loss = bl;
   if (best_step) *best_step = bs;
   if (bs < 0) return fail(MARS_ENUMERIC, "no finite loss during pre-training");
-  return MARS_OK;
+  return check_skipped(m, skipped);
 }
 
 // Enqueues one step (graph replay or eager) after the step scalars.
@@ -1242,8 +1364,10 @@ static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_inde
                   cudaGetErrorString(e));
     }
   }
+  g->note_use(s);
   m->last_launches = nl;
   m->last_Nt = g->dev.Nt;
+  m->kb_valid_Nt = m->keep_bwd ? g->dev.Nt : 0;
   return MARS_OK;
 }
 
@@ -1260,8 +1384,9 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
   if (g->F != m->F) return fail(MARS_EINVAL, "feat_dim mismatch");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
-  const GraphDev& gd = g->dev;
   Workspace& w = m->ws;
+  GraphDev gd = g->dev;
+  gd.long_part = w.long_part;
   cudaStream_t s = m->stream;
   const int F = m->F, H = m->H;
   float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
@@ -1283,9 +1408,6 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
                             w.h3_w_hi[l], w.h3_w_lo[l], s, &nl));
       CK(tc3h_gemm_rows(Ys[l], w.h3_rsY[l], w.h3_wt_hi[l], w.h3_wt_lo[l], w.h3_wsc[l] + 1, w.Z[l],
                         gd.Nt, H, Cin, s, &nl));
-    } else if (m->gemm_impl == MARS_GEMM_3XTF32 && tc_supported(Cin, H)) {
-      CK(tc_split_weights(W[l], Cin, H, w.wt_hi[l], w.wt_lo[l], w.w_hi[l], w.w_lo[l], s, &nl));
-      CK(tc_gemm_rows(Ys[l], w.wt_hi[l], w.wt_lo[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
     } else {
       CK(gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
     }
@@ -1327,6 +1449,55 @@ extern "C" mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t la
   return MARS_OK;
 }
 
+extern "C" mars_status mars_dgi_saved_rows(const mars_dgi* m, int64_t* rows) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!rows) return fail(MARS_EINVAL, "rows is NULL");
+  *rows = m->last_Nt;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_set_keep_backward(mars_dgi* m, int32_t keep) {
+  if (mars_status st = check_dgi(m)) return st;
+  CK(cudaSetDevice(m->cfg.device));
+  if (m->exec) {                 // recapture with / without the copies
+    cudaGraphExecDestroy(m->exec);
+    m->exec = nullptr;
+    m->exec_graph = 0;
+  }
+  CK(cudaStreamSynchronize(m->stream));
+  m->keep_bwd = keep != 0;
+  if (!m->keep_bwd) m->kb_release();
+  m->kb_valid_Nt = 0;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_export_backward(const mars_dgi* m, int32_t layer, float* dY,
+                                                float* dZ) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (layer < 1 || layer > 3) return fail(MARS_EINVAL, "layer must be 1..3");
+  if (layer == 1 && dY) return fail(MARS_EINVAL, "there is no dY_1");
+  if (!m->kb_valid_Nt || m->kb_valid_Nt != m->last_Nt)
+    return fail(MARS_ESTATE, "the last step did not keep its backward intermediates");
+  CK(cudaSetDevice(m->cfg.device));
+  CK(cudaStreamSynchronize(m->stream));
+  const int64_t n = 2LL * m->kb_valid_Nt * m->H;
+  const void* srcs[2] = {layer >= 2 ? m->kb_dY[layer - 2] : nullptr, m->kb_dZ[layer - 1]};
+  float* dsts[2] = {dY, dZ};
+  for (int k = 0; k < 2; ++k) {
+    if (!dsts[k]) continue;
+    if (m->cfg.precision == MARS_BF16) {
+      float* tmp = nullptr;
+      CK(cudaMalloc(&tmp, sizeof(float) * n));
+      struct FT { float* p; ~FT() { cudaFree(p); } } ft{tmp};
+      CK(launch_upcast(srcs[k], tmp, n, nullptr));
+      CK(cudaMemcpy(dsts[k], tmp, sizeof(float) * n, cudaMemcpyDeviceToHost));
+    } else {
+      CK(cudaMemcpy(dsts[k], srcs[k], sizeof(float) * n, cudaMemcpyDeviceToHost));
+    }
+  }
+  return MARS_OK;
+}
+
 extern "C" mars_status mars_dgi_get_state(const mars_dgi* m, float* params, float* am, float* av,
                                           int64_t* t) {
   if (mars_status st = check_dgi(m)) return st;
@@ -1335,7 +1506,7 @@ extern "C" mars_status mars_dgi_get_state(const mars_dgi* m, float* params, floa
   if (params) CK(cudaMemcpy(params, m->params, sizeof(float) * m->P, cudaMemcpyDeviceToHost));
   if (am) CK(cudaMemcpy(am, m->adam_m, sizeof(float) * m->P, cudaMemcpyDeviceToHost));
   if (av) CK(cudaMemcpy(av, m->adam_v, sizeof(float) * m->P, cudaMemcpyDeviceToHost));
-  if (t) *t = m->t;
+  if (t) CK(cudaMemcpy(t, &m->adam_st->t, sizeof(int64_t), cudaMemcpyDeviceToHost));
   return MARS_OK;
 }
 
@@ -1348,7 +1519,7 @@ extern "C" mars_status mars_dgi_set_state(mars_dgi* m, const float* params, cons
   if (params) CK(cudaMemcpy(m->params, params, sizeof(float) * m->P, cudaMemcpyHostToDevice));
   if (am) CK(cudaMemcpy(m->adam_m, am, sizeof(float) * m->P, cudaMemcpyHostToDevice));
   if (av) CK(cudaMemcpy(m->adam_v, av, sizeof(float) * m->P, cudaMemcpyHostToDevice));
-  m->t = t;
+  CK(cudaMemcpy(&m->adam_st->t, &t, sizeof(int64_t), cudaMemcpyHostToDevice));
   return MARS_OK;
 }
 
@@ -1365,22 +1536,22 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   CK(cudaSetDevice(device));
   const bool tcp = impl != MARS_GEMM_SIMT && (op == 0 ? tc_supported(K, N) || tc_supported(N, K)
                                                      : tc_supported(K, N));
-  const bool h3 = impl == MARS_GEMM_AUTO;
   float *wsc = nullptr, *rs = nullptr, *rs2 = nullptr;
   CK(dalloc(&wsc, 2));
   CK(dalloc(&rs, (size_t)M));
   CK(dalloc(&rs2, (size_t)M));
   size_t nA = (size_t)M * K, nB = op == 0 ? (size_t)N * K : (size_t)M * N;
   size_t nC = op == 0 ? (size_t)M * N : (size_t)K * N;
-  float *dA, *dB, *dC, *bh, *bl, *bth, *btl, *part;
+  float *dA, *dB, *dC, *part;
+  void *bh, *bl, *bth, *btl;
   double* tpart;
   CK(dalloc(&dA, nA));
   CK(dalloc(&dB, nB));
   CK(dalloc(&dC, nC));
-  CK(dalloc(&bh, (size_t)N * K));
-  CK(dalloc(&bl, (size_t)N * K));
-  CK(dalloc(&bth, (size_t)N * K));
-  CK(dalloc(&btl, (size_t)N * K));
+  CK(dalloc((char**)&bh, (size_t)N * K * 2));
+  CK(dalloc((char**)&bl, (size_t)N * K * 2));
+  CK(dalloc((char**)&bth, (size_t)N * K * 2));
+  CK(dalloc((char**)&btl, (size_t)N * K * 2));
   size_t np = std::max(tc_dw_partial_floats(M, K), (size_t)1);
   CK(dalloc(&part, np));
   CK(dalloc(&tpart, gemm_tn_partial_floats(M, K, N)));
@@ -1390,26 +1561,20 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
   CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
   auto run = [&]() -> cudaError_t {
     if (op == 0) {
-      if (tcp && h3) {   // B [N×K] = "W" with CIN = N, H = K: the dY orientation
+      if (tcp) {   // B [N×K] = "W" with CIN = N, H = K: the dY orientation
         cudaError_t e = tc3h_split_weights(dB, N, K, wsc, bth, btl, bh, bl, s, nullptr);
         if (e != cudaSuccess) return e;
         if ((e = tc3h_row_scales(dA, M, K, rs, s, nullptr)) != cudaSuccess) return e;
         return tc3h_gemm_rows(dA, rs, bh, bl, wsc + 1, dC, M, N, K, s, nullptr);
       }
-      if (tcp) {
-        cudaError_t e = tc_split_weights(dB, N, K, bth, btl, bh, bl, s, nullptr);
-        if (e != cudaSuccess) return e;
-        return tc_gemm_rows(dA, bh, bl, dC, M, N, K, s, nullptr);
-      }
       return gemm_nt(dA, dB, dC, M, N, K, s, nullptr);
     }
-    if (tcp && h3) {
+    if (tcp) {
       cudaError_t e = tc3h_row_scales(dA, M, K, rs, s, nullptr);
       if (e != cudaSuccess) return e;
       if ((e = tc3h_row_scales(dB, M, N, rs2, s, nullptr)) != cudaSuccess) return e;
       return tc3h_gemm_dw(dA, rs, dB, rs2, dC, M, K, N, part, s, nullptr);
     }
-    if (tcp) return tc_gemm_dw(dA, dB, dC, M, K, N, part, s, nullptr);
     return gemm_tn(dA, dB, dC, M, K, N, tpart, s, nullptr);
   };
   cudaEvent_t e0, e1;
@@ -1755,20 +1920,106 @@ extern "C" mars_status mars_shard_connect_local(mars_dgi* const* models, int32_t
   return MARS_OK;
 }
 
+// ---------------------------------------------------------------- data parallel over peer memory
+namespace {
+constexpr uint64_t kDpBlobMagic = 0x4D41525344504231ULL;   // "MARSDPB1"
+struct DpBlob {
+  uint64_t magic;
+  int32_t R, me, device, pad;
+  int64_t P;
+  cudaIpcMemHandle_t grads, flags;
+};
+}  // namespace
+
+extern "C" int64_t mars_dp_blob_bytes(void) { return (int64_t)sizeof(DpBlob); }
+
+extern "C" mars_status mars_dp_export(const mars_dgi* m, void* blob) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!blob) return fail(MARS_EINVAL, "blob is NULL");
+  if (m->dp.R < 2) return fail(MARS_ESTATE, "model was not created for peer-memory data parallelism");
+  CK(cudaSetDevice(m->cfg.device));
+  DpBlob b{};
+  b.magic = kDpBlobMagic;
+  b.R = m->dp.R;
+  b.me = m->dp.me;
+  b.device = m->cfg.device;
+  b.P = m->P;
+  CK(cudaIpcGetMemHandle(&b.grads, m->grads));
+  CK(cudaIpcGetMemHandle(&b.flags, m->dp.flags));
+  memcpy(blob, &b, sizeof b);
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dp_connect(mars_dgi* m, const void* blobs) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!blobs) return fail(MARS_EINVAL, "blobs is NULL");
+  mars_dgi::Dp& d = m->dp;
+  if (d.R < 2) return fail(MARS_ESTATE, "model was not created for peer-memory data parallelism");
+  if (d.connected) return fail(MARS_ESTATE, "already connected");
+  CK(cudaSetDevice(m->cfg.device));
+  const DpBlob* b = static_cast<const DpBlob*>(blobs);
+  for (int q = 0; q < d.R; ++q)
+    if (b[q].magic != kDpBlobMagic || b[q].R != d.R || b[q].me != q || b[q].P != m->P)
+      return fail(MARS_EINVAL, "data-parallel blob %d does not match this job", q);
+  d.sync.P = d.R;
+  d.sync.me = d.me;
+  d.sync.epoch = d.epoch;
+  d.sync.err = d.err;
+  for (int q = 0; q < d.R; ++q) {
+    if (q == d.me) {
+      d.grads.p[q] = m->grads;
+      d.sync.flags[q] = d.flags;
+      continue;
+    }
+    void* pg = nullptr;
+    void* pf = nullptr;
+    CK(cudaIpcOpenMemHandle(&pg, b[q].grads, cudaIpcMemLazyEnablePeerAccess));
+    d.ipc.push_back(pg);
+    CK(cudaIpcOpenMemHandle(&pf, b[q].flags, cudaIpcMemLazyEnablePeerAccess));
+    d.ipc.push_back(pf);
+    d.grads.p[q] = pg;
+    d.sync.flags[q] = static_cast<unsigned long long*>(pf);
+  }
+  d.connected = true;
+  if (m->exec) {
+    cudaGraphExecDestroy(m->exec);
+    m->exec = nullptr;
+    m->exec_graph = 0;
+  }
+  // One process per rank: each barrier signals its peers before it waits, so a
+  // host thread blocked in a lazy module load (which waits for its own context
+  // to go idle) cannot deadlock the ranks.
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_graph_set_pair_offsets(mars_graph* g, const int64_t* off) {
+  if (mars_status st = check_graph(g)) return st;
+  if (!off) return fail(MARS_EINVAL, "pair_offsets is NULL");
+  for (int i = 0; i < g->G; ++i)
+    if (off[i] < 0) return fail(MARS_EINVAL, "negative pair offset");
+  CK(cudaSetDevice(g->device));
+  CK(cudaMemcpy(g->pair_off, off, sizeof(int64_t) * g->G, cudaMemcpyHostToDevice));
+  return MARS_OK;
+}
+
 extern "C" mars_status mars_dgi_read_step(mars_dgi* m, float* loss, float* grads) {
   if (mars_status st = check_dgi(m)) return st;
   CK(cudaSetDevice(m->cfg.device));
   cudaStream_t s = m->stream;
   float l = 0.f;
-  int32_t err = 0;
+  int32_t err = 0, skipped = 0;
   CK(cudaMemcpyAsync(&l, m->grads_final() + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&skipped, &m->adam_st->skipped, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   if (grads)
     CK(cudaMemcpyAsync(grads, m->grads_final(), sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
   if (m->sh.err) CK(cudaMemcpyAsync(&err, m->sh.err, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
+  int32_t derr = 0;
+  if (m->dp.err) CK(cudaMemcpyAsync(&derr, m->dp.err, sizeof(int32_t), cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
   if (err) return fail(MARS_ECUDA, "shard barrier timed out (a peer shard did not step)");
+  if (derr) return fail(MARS_ECUDA, "data-parallel barrier timed out (a peer rank did not step)");
   if (loss) *loss = l;
-  return MARS_OK;
+  return check_skipped(m, skipped);
 }
 
 extern "C" void mars_free(void* h) {
@@ -1777,7 +2028,6 @@ extern "C" void mars_free(void* h) {
   if (tag == kTagGraph) {
     auto* g = static_cast<mars_graph*>(h);
     cudaSetDevice(g->device);
-    cudaDeviceSynchronize();
     g->tag = kTagDead;
     delete g;
   } else if (tag == kTagDgi) {

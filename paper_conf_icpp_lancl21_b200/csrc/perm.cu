@@ -19,6 +19,7 @@ namespace {
 
 __global__ void k_perm_keys(const int32_t* __restrict__ node_graph,
                             const int32_t* __restrict__ node_off,
+                            const int64_t* __restrict__ pair_off,
                             const int32_t* __restrict__ bucket_off,
                             const int32_t* __restrict__ bucket_log2, int32_t Nt, uint64_t seed,
                             const StepParams* __restrict__ sp, uint64_t* __restrict__ keys,
@@ -26,7 +27,7 @@ __global__ void k_perm_keys(const int32_t* __restrict__ node_graph,
   int32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= Nt) return;
   int32_t g = node_graph[i];
-  uint64_t kg = sm64(sm64(sm64(seed) ^ sp->step_index) ^ (uint64_t)(sp->pair_base + g));
+  uint64_t kg = sm64(sm64(sm64(seed) ^ sp->step_index) ^ (uint64_t)(sp->pair_base + pair_off[g]));
   uint64_t key = sm64(kg ^ (uint64_t)(i - node_off[g]));
   int lb = bucket_log2[g];
   int32_t b = bucket_off[g] + (lb ? (int32_t)(key >> (64 - lb)) : 0);
@@ -67,7 +68,7 @@ cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp, 
   cudaError_t e;
   if ((e = cudaMemsetAsync(w.bcnt, 0, sizeof(int32_t) * (size_t)(g.nbuckets + 1), s))) return e;
   unsigned nb = cdiv(g.Nt, 256);
-  k_perm_keys<<<nb, 256, 0, s>>>(g.node_graph, g.node_off, g.bucket_off, g.bucket_log2, g.Nt,
+  k_perm_keys<<<nb, 256, 0, s>>>(g.node_graph, g.node_off, g.pair_off, g.bucket_off, g.bucket_log2, g.Nt,
                                  seed, sp, w.keys, w.bucket, w.bcnt);
   count_launch(launches);
   if ((e = scan_exclusive_i32(w.bcnt, w.bstart, g.nbuckets, w.scan_tmp, s, launches))) return e;

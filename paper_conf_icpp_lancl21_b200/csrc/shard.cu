@@ -16,8 +16,10 @@
 //     partials, gradient partials);
 //   - k_head_xsum: readout column sums (Eq. 4) and dv / loss (Eqs. 5-6) summed
 //     over shards in rank order (deterministic, identical on every shard);
-//   - k_grad_sum: the data-parallel-style gradient reduction over shards in
-//     rank order (fp64), so replicated Adam stays bit-identical across shards.
+//   - k_grad_sum: the gradient reduction over shards in rank order (fp64), so
+//     replicated Adam stays bit-identical across shards; the same kernel is
+//     the data-parallel gradient exchange over peer memory (a13, mars_dp_*),
+//     where every entry including the loss is a per-rank partial.
 #include "common.cuh"
 #include "internal.cuh"
 
@@ -83,10 +85,10 @@ __global__ void k_head_xsum(const __grid_constant__ PeerPtrs x, int P, int H, in
 }
 
 __global__ void k_grad_sum(const __grid_constant__ PeerPtrs g, int P, int me, int64_t n,
-                           int64_t keep_b, int64_t keep_e, float* __restrict__ out) {
+                           int64_t keep_b, int64_t keep_e, int sum_last, float* __restrict__ out) {
   const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (k >= n) return;
-  if ((k >= keep_b && k < keep_e) || k == n - 1) {
+  if ((k >= keep_b && k < keep_e) || (!sum_last && k == n - 1)) {
     out[k] = static_cast<const float*>(g.p[me])[k];
     return;
   }
@@ -112,9 +114,10 @@ cudaError_t launch_head_xsum(const PeerPtrs& x, int P, int H, int mode, const in
 }
 
 cudaError_t launch_grad_sum(const PeerPtrs& g, int P, int me, int64_t n, int64_t keep_b,
-                            int64_t keep_e, float* out, cudaStream_t st, int* launches) {
+                            int64_t keep_e, int sum_last, float* out, cudaStream_t st,
+                            int* launches) {
   count_launch(launches);
-  k_grad_sum<<<cdiv(n, 256), 256, 0, st>>>(g, P, me, n, keep_b, keep_e, out);
+  k_grad_sum<<<cdiv(n, 256), 256, 0, st>>>(g, P, me, n, keep_b, keep_e, sum_last, out);
   return cudaGetLastError();
 }
 

@@ -28,12 +28,9 @@
 namespace mars {
 namespace {
 
-#ifndef MARS_SPMM_THREADS
-#define MARS_SPMM_THREADS 32    // one warp per block: a slow (hub) row holds no other warps
-#endif
-constexpr int kSpmmThreads = MARS_SPMM_THREADS;
-#ifndef MARS_SPMM_MINB        // resident blocks per SM: caps registers at 64
-#define MARS_SPMM_MINB (1024 / MARS_SPMM_THREADS < 32 ? 1024 / MARS_SPMM_THREADS : 32)
+constexpr int kSpmmThreads = 32;   // one warp per block: a slow (hub) row holds no other warps
+#ifndef MARS_SPMM_MINB             // resident blocks per SM: caps registers at 64
+#define MARS_SPMM_MINB 32
 #endif
 #ifndef MARS_SPMM_KU
 #define MARS_SPMM_KU 4
@@ -103,13 +100,6 @@ struct PeerSrc {        // row-sharded graph: global row j lives on shard owner(
     return static_cast<const T*>(pr.base[p]) + ((int64_t)n + j - pr.start[p]) * C;
   }
 };
-
-#ifndef MARS_SPMM_PERSIST
-#define MARS_SPMM_PERSIST 0   // > 0: resident grid of PERSIST waves of MINB blocks per SM
-#endif
-#ifndef MARS_SPMM_TAIL
-#define MARS_SPMM_TAIL 1
-#endif
 
 // One batch of K neighbours t .. t+K-1 of the current chunk: all 2K gathers
 // are issued before the FMAs.  Slots u >= nvalid re-gather neighbour t (a
@@ -191,9 +181,9 @@ __device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, 
 
 // Accumulates row (rb, re) of Â_n · act(T) for both branches: per chunk of L
 // neighbours each lane loads one (colind, val) pair (+ perm for layer 1),
-// broadcast by shuffles, then batches of kU neighbours.  MARS_SPMM_TAIL
-// selects the last partial batch: 1 = one padded batch (default), 0 = one
-// neighbour at a time, 2 = a batch of 2 then 1.
+// broadcast by shuffles, then batches of kU neighbours; the last partial batch
+// is one padded batch (measured against a neighbour-at-a-time tail and
+// predicated tails).
 template <class S, bool BOTH, int ACT, bool PERM, typename T, class Src>
 __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __restrict__ colind,
                                            const float* __restrict__ vals,
@@ -210,23 +200,9 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
       cv = vals[k0 + sl];
       if (PERM && BOTH) cjn = perm[k0 + sl];   // colperm: pi[colind[k]], no dependent lookup
     }
-#if MARS_SPMM_TAIL == 1
     for (int t = 0; t < cnt; t += kU)
       gather_batch<S, kU, BOTH, ACT, PERM, T>(src, t, min(kU, cnt - t), cj, cv, cjn, gmask, sl,
                                               a, accp, accn);
-#else
-    int t = 0;
-    for (; t + kU <= cnt; t += kU)
-      gather_batch<S, kU, BOTH, ACT, PERM, T>(src, t, kU, cj, cv, cjn, gmask, sl, a, accp, accn);
-#if MARS_SPMM_TAIL == 2
-    if (t + 2 <= cnt) {
-      gather_batch<S, 2, BOTH, ACT, PERM, T>(src, t, 2, cj, cv, cjn, gmask, sl, a, accp, accn);
-      t += 2;
-    }
-#endif
-    for (; t < cnt; ++t)
-      gather_batch<S, 1, BOTH, ACT, PERM, T>(src, t, 1, cj, cv, cjn, gmask, sl, a, accp, accn);
-#endif
   }
 }
 
@@ -562,26 +538,13 @@ cudaError_t long_bwd(const GraphDev& g, const T* dY, const T* Z, const float* al
   return cudaGetLastError();
 }
 
-// Rows handled by block b: NW warps x RPW row groups.  BAND = false: one row
-// per group, blocks of consecutive rows (kSpmmThreads = 256).  BAND = true: a
-// persistent grid of one 1024-thread block per SM, block b sweeping the
-// contiguous band of rows [b·n, (b+1)·n) 32·RPW rows at a time, so the rows
-// its warps gather (op graphs are local: most neighbours lie within a few
-// dozen rows) were just read by the same SM and hit in its L1 instead of L2.
-template <int C, typename T, bool BAND>
-struct RowSched {
-  using S = SpmmShape<C, T>;
-  static constexpr int NW = BAND ? 32 : kSpmmThreads / 32;
-  static constexpr int RPB = S::RPW * NW;
-};
+// Rows handled by block b: one warp of RPW row groups (rows b·RPW ...).
+// Measured and rejected: multi-warp blocks, a persistent grid
+// walking rows i, i + NG, ..., and banded grids of one 1024-thread block per SM.
+static_assert(kSpmmThreads == 32, "long-row segments and the row map assume one-warp blocks");
 
-#ifndef MARS_SPMM_BAND
-#define MARS_SPMM_BAND 0
-#endif
-constexpr int kBandThreads = 1024;
-
-template <int C, int MODE, bool BOTH, bool SH, bool BAND, bool LONG, typename Tin, typename Tout>
-__global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 : MARS_SPMM_MINB)
+template <int C, int MODE, bool BOTH, bool SH, bool LONG, typename Tin, typename Tout>
+__global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
 k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const Tin* __restrict__ T,
            const int32_t* __restrict__ perm, const float* __restrict__ alpha, int act_layer,
@@ -589,7 +552,6 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
            const __grid_constant__ PeerRows pr, const __grid_constant__ LongArgs la, int32_t nseg,
            int32_t long_min) {
   using S = SpmmShape<C, Tin>;
-  using RS = RowSched<C, Tin, BAND>;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int sub = lane / S::L, sl = lane % S::L;
   const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
@@ -600,31 +562,22 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
     return;
   }
   const int32_t bid = LONG ? (int32_t)blockIdx.x - nseg : (int32_t)blockIdx.x;
-  const int32_t nblk = LONG ? (int32_t)gridDim.x - nseg : (int32_t)gridDim.x;
-  if (!BAND) {
-    // MARS_SPMM_PERSIST: a resident grid walks rows i, i + gridDim·RPB, ...
-    // (no per-row block launches); otherwise one launch block per RPB rows
-    const int32_t step = MARS_SPMM_PERSIST ? nblk * RS::RPB : Nt;
-    for (int32_t i = bid * RS::RPB + w * S::RPW + sub; i < Nt; i += step) {
-      // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
-      if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
-        if (a >= 0.f && a <= 1.f) {
-          fwd_row<C, MODE, BOTH, SH, 2, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
-          continue;
-        }
-      }
-      fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
+  const int32_t i = bid * S::RPB + w * S::RPW + sub;
+  if (i >= Nt) return;
+  // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
+  if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
+    if (a >= 0.f && a <= 1.f) {
+      fwd_row<C, MODE, BOTH, SH, 2, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs,
+                                          pr, gmask, sl);
+      return;
     }
-    return;
   }
-  const int32_t n = (int32_t)((Nt + nblk - 1) / nblk);
-  const int32_t r0 = bid * n, r1 = min(Nt, r0 + n);
-  for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-    fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr, gmask, sl);
+  fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr,
+                                      gmask, sl);
 }
 
-template <int C, bool SH, bool BAND, bool LONG, typename T>
-__global__ void __launch_bounds__(BAND ? kBandThreads : kSpmmThreads, BAND ? 1 : MARS_SPMM_MINB)
+template <int C, bool SH, bool LONG, typename T>
+__global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
 k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
            const float* __restrict__ vals, const T* __restrict__ dY, const T* __restrict__ Z,
            const float* __restrict__ alpha, int layer, int32_t Nt, T* __restrict__ dZ,
@@ -632,8 +585,6 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
            const __grid_constant__ PeerRows pr, const __grid_constant__ LongArgs la, int32_t nseg,
            int32_t long_min) {
   using S = SpmmShape<C, T>;
-  using RS = RowSched<C, T, BAND>;
-  __shared__ double wpart[RS::NW];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int sub = lane / S::L, sl = lane % S::L;
   const unsigned gmask = (S::L == 32) ? kFull : (((1u << S::L) - 1u) << (sub * S::L));
@@ -644,26 +595,12 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
     return;
   }
   const int32_t bid = LONG ? (int32_t)blockIdx.x - nseg : (int32_t)blockIdx.x;
-  const int32_t nblk = LONG ? (int32_t)gridDim.x - nseg : (int32_t)gridDim.x;
+  const int32_t i = bid * S::RPB + w * S::RPW + sub;
   float da = 0.f;
-  if (!BAND) {
-    const int32_t step = MARS_SPMM_PERSIST ? nblk * RS::RPB : Nt;
-    for (int32_t i = bid * RS::RPB + w * S::RPW + sub; i < Nt; i += step)
-      bwd_row<C, SH, LONG>(i, long_min, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
-  } else {
-    const int32_t n = (int32_t)((Nt + nblk - 1) / nblk);
-    const int32_t r0 = bid * n, r1 = min(Nt, r0 + n);
-    for (int32_t i = r0 + w * S::RPW + sub; i < r1; i += RS::RPB)
-      bwd_row<C, SH, LONG>(i, long_min, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
-  }
-  const double wd = warp_sum((double)da);
-  if (lane == 0) wpart[w] = wd;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double t = 0.0;
-    for (int k = 0; k < RS::NW; ++k) t += wpart[k];
-    slots[bid] = t;
-  }
+  if (i < Nt)
+    bwd_row<C, SH, LONG>(i, long_min, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
+  const double wd = warp_sum((double)da);   // the block is one warp
+  if (lane == 0) slots[bid] = wd;
 }
 
 int spmm_sms() {
@@ -677,35 +614,23 @@ int spmm_sms() {
   return n;
 }
 
-// Grid of a launch: banded (one block per SM, at most one per 32·RPW rows)
-// for the wide aggregations, blocks of consecutive rows otherwise (layer 1's
-// corrupted branch gathers X[pi[j]] at random, no band locality).
-template <int C, typename T, bool BAND>
+// One one-warp block per RPB rows.
+template <int C, typename T>
 unsigned spmm_blocks(int32_t Nt) {
-  using RS = RowSched<C, T, BAND>;
-  if (!BAND && MARS_SPMM_PERSIST)
-    return (unsigned)std::max<int64_t>(
-        1, std::min<int64_t>((int64_t)spmm_sms() * MARS_SPMM_MINB * MARS_SPMM_PERSIST,
-                             cdiv(Nt, RS::RPB)));
-  if (!BAND) return cdiv(Nt, RS::RPB);
-  return (unsigned)std::max<int64_t>(1, std::min<int64_t>(spmm_sms(), cdiv(Nt, RS::RPB)));
+  return cdiv(Nt, SpmmShape<C, T>::RPB);
 }
 
 template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
 cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
                        int act_layer, Tout* Y, float* rs, cudaStream_t s, const PeerRows& pr) {
-  constexpr bool BAND = MARS_SPMM_BAND && MODE == 1;
-  static_assert(BAND || kSpmmThreads == 32, "long-row segments run as one-warp blocks");
   const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
-  const unsigned nb = spmm_blocks<C, Tin, BAND>(g.Nt);
+  const unsigned nb = spmm_blocks<C, Tin>(g.Nt);
   const int al = act_layer < 0 ? 0 : act_layer;
   if (g.nseg > 0)   // long rows: their segments run as the grid's first blocks
-    k_spmm_fwd<C, MODE, BOTH, SH, BAND, true, Tin, Tout>
-        <<<nb + g.nseg, BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
-            g.rowptr, g.colind, g.vals, T, perm, alpha, al, g.Nt, Y, rs, pr, la, g.nseg, g.long_min);
+    k_spmm_fwd<C, MODE, BOTH, SH, true, Tin, Tout><<<nb + g.nseg, kSpmmThreads, 0, s>>>(
+        g.rowptr, g.colind, g.vals, T, perm, alpha, al, g.Nt, Y, rs, pr, la, g.nseg, g.long_min);
   else
-    k_spmm_fwd<C, MODE, BOTH, SH, BAND, false, Tin, Tout>
-        <<<nb, BAND ? kBandThreads : kSpmmThreads, 0, s>>>(
+    k_spmm_fwd<C, MODE, BOTH, SH, false, Tin, Tout><<<nb, kSpmmThreads, 0, s>>>(
             g.rowptr, g.colind, g.vals, T, perm, alpha, al, g.Nt, Y, rs, pr, la, 0, 0);
   if (cudaError_t e = cudaGetLastError()) return e;
   return long_fwd<C, MODE, BOTH, SH, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, pr);
@@ -751,19 +676,18 @@ template <int C, typename T>
 cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha, int layer,
                   T* dZ, double* slots, int* nslots, float* rs, cudaStream_t s,
                   const PeerRows* peers) {
-  constexpr bool BAND = MARS_SPMM_BAND;
-  const unsigned blocks = spmm_blocks<C, T, BAND>(g.Nt);
-  const unsigned threads = BAND ? kBandThreads : kSpmmThreads;
+  const unsigned blocks = spmm_blocks<C, T>(g.Nt);
+  const unsigned threads = kSpmmThreads;
   const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
   *nslots = (int)blocks + g.nlong;                   // long rows' dalpha after the blocks'
   if constexpr (C == 128 || C == 256) {
     if (peers) {
       if (g.nseg > 0)
-        k_spmm_bwd<C, true, BAND, true, T><<<blocks + g.nseg, threads, 0, s>>>(
+        k_spmm_bwd<C, true, true, T><<<blocks + g.nseg, threads, 0, s>>>(
             g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, *peers, la,
             g.nseg, g.long_min);
       else
-        k_spmm_bwd<C, true, BAND, false, T><<<blocks, threads, 0, s>>>(
+        k_spmm_bwd<C, true, false, T><<<blocks, threads, 0, s>>>(
             g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, *peers, la, 0, 0);
       if (cudaError_t e = cudaGetLastError()) return e;
       return long_bwd<C, true, T>(g, dY, Z, alpha, layer, dZ, slots + blocks, rs, s, *peers);
@@ -771,11 +695,11 @@ cudaError_t bwd_c(const GraphDev& g, const T* dY, const T* Z, const float* alpha
   }
   if (peers) return cudaErrorInvalidValue;
   if (g.nseg > 0)
-    k_spmm_bwd<C, false, BAND, true, T><<<blocks + g.nseg, threads, 0, s>>>(
+    k_spmm_bwd<C, false, true, T><<<blocks + g.nseg, threads, 0, s>>>(
         g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, PeerRows{}, la,
         g.nseg, g.long_min);
   else
-    k_spmm_bwd<C, false, BAND, false, T><<<blocks, threads, 0, s>>>(
+    k_spmm_bwd<C, false, false, T><<<blocks, threads, 0, s>>>(
         g.rowptr, g.colind, g.vals, dY, Z, alpha, layer, g.Nt, dZ, slots, rs, PeerRows{}, la, 0, 0);
   if (cudaError_t e = cudaGetLastError()) return e;
   return long_bwd<C, false, T>(g, dY, Z, alpha, layer, dZ, slots + blocks, rs, s, PeerRows{});

@@ -80,6 +80,10 @@ SIGNATURES = {
                                          ctypes.c_void_p]),
     "mars_dgi_export_activations": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32,
                                                    ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_saved_rows": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_set_keep_backward": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mars_dgi_export_backward": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32,
+                                                ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dgi_get_state": (ctypes.c_int, [ctypes.c_void_p] * 4 + [ctypes.c_void_p]),
     "mars_dgi_set_state": (ctypes.c_int, [ctypes.c_void_p] * 4 + [ctypes.c_int64]),
     "mars_dgi_profile_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
@@ -102,6 +106,10 @@ SIGNATURES = {
     "mars_shard_export": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_shard_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_shard_connect_local": (ctypes.c_int, [ctypes.POINTER(ctypes.c_void_p), ctypes.c_int32]),
+    "mars_dp_blob_bytes": (ctypes.c_int64, []),
+    "mars_dp_export": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dp_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_graph_set_pair_offsets": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -175,6 +183,13 @@ class Graph:
 
     def export_csr(self, idx):
         return graph_export_csr(self, idx)
+
+    def set_pair_offsets(self, offsets):
+        """mars_graph_set_pair_offsets: graph i uses pair index pair_base + offsets[i] (c15)."""
+        off = np.ascontiguousarray(offsets, np.int64)
+        if off.size != self.num_graphs:
+            raise ValueError("one offset per graph")
+        _check(lib().mars_graph_set_pair_offsets(self.handle, _ptr(off)))
 
     def free(self):
         if self.handle:
@@ -262,7 +277,6 @@ def graph_shard_info(g: Graph):
 
 def shard_attach(m: "DGI", g: Graph):
     _check(lib().mars_shard_attach(m.handle, g.handle))
-    m._shard_rows = graph_shard_info(g)["row_end"] - graph_shard_info(g)["row_begin"]
 
 
 def shard_export(m: "DGI") -> bytes:
@@ -281,6 +295,20 @@ def shard_connect(m: "DGI", blobs):
 def shard_connect_local(models):
     arr = (ctypes.c_void_p * len(models))(*[m.handle for m in models])
     _check(lib().mars_shard_connect_local(arr, len(models)))
+
+
+def dp_export(m: "DGI") -> bytes:
+    """mars_dp_export: this rank's blob for the peer-memory gradient exchange."""
+    buf = ctypes.create_string_buffer(int(lib().mars_dp_blob_bytes()))
+    _check(lib().mars_dp_export(m.handle, buf))
+    return buf.raw
+
+
+def dp_connect(m: "DGI", blobs):
+    """mars_dp_connect: blobs = every rank's dp_export() in rank order."""
+    data = b"".join(blobs)
+    buf = ctypes.create_string_buffer(data, len(data))
+    _check(lib().mars_dp_connect(m.handle, buf))
 
 
 def graph_export_csr(g: Graph, idx: int):
@@ -332,11 +360,30 @@ class DGI:
         _check(lib().mars_dgi_pretrain(self.handle, g.handle, step0 & (2 ** 64 - 1), int(n_steps),
                                        int(pair_base), B, _ptr(losses), _ptr(best),
                                        ctypes.byref(bl), ctypes.byref(bs)))
-        self._last_nt = g.total_nodes
         return dict(losses=losses, best_params=best, best_loss=bl.value, best_step=bs.value)
 
     def export_activations(self, layer: int):
         return dgi_export_activations(self, layer)
+
+    def saved_rows(self) -> int:
+        """Rows per branch of the last step's saved activations (0 after encode)."""
+        r = ctypes.c_int64()
+        _check(lib().mars_dgi_saved_rows(self.handle, ctypes.byref(r)))
+        return r.value
+
+    def set_keep_backward(self, keep: bool):
+        """Test hook: keep dZ_3..1 and dY_3, dY_2 of every later step."""
+        _check(lib().mars_dgi_set_keep_backward(self.handle, 1 if keep else 0))
+
+    def export_backward(self, layer: int):
+        """Test hook: (dY_layer or None for layer 1, dZ_layer) of the last step,
+        stacked [pos; neg], fp32."""
+        R = 2 * self.saved_rows()
+        dZ = np.zeros((R, self.H), np.float32)
+        dY = np.zeros((R, self.H), np.float32) if layer > 1 else None
+        _check(lib().mars_dgi_export_backward(self.handle, layer,
+                                              None if dY is None else _ptr(dY), _ptr(dZ)))
+        return dY, dZ
 
     def get_state(self):
         p = np.zeros(self.P, np.float32); m = np.zeros(self.P, np.float32)
@@ -353,8 +400,8 @@ class DGI:
         _check(lib().mars_dgi_set_stream(self.handle, stream_ptr))
 
     def set_gemm_impl(self, impl: str):
-        """'auto' (tcgen05: 3xFP16 row GEMMs, 3xTF32 weight gradient, where
-        supported), 'simt' (FFMA everywhere) or '3xtf32' (every tcgen05 GEMM 3xTF32)."""
+        """'auto' (tcgen05 3xFP16 GEMMs where the widths are supported) or
+        'simt' (FFMA everywhere)."""
         _check(lib().mars_dgi_set_gemm_impl(self.handle, GEMM_IMPLS[impl]))
 
     def set_graph_capture(self, enable: bool):
@@ -368,7 +415,6 @@ class DGI:
         _check(lib().mars_dgi_profile_step(self.handle, g.handle, step_index & (2 ** 64 - 1),
                                            int(pair_base), B, _ptr(ids), _ptr(ms), 256,
                                            ctypes.byref(n)))
-        self._last_nt = g.total_nodes
         return [(PHASES[int(i)], float(t)) for i, t in zip(ids[:n.value], ms[:n.value])]
 
     def read_step(self, want_grads=True):
@@ -430,7 +476,6 @@ def dgi_step(m: DGI, g: Graph, step_index: int, pair_base: int = 0, global_batch
         res["perms"] = np.zeros(g.total_nodes, np.int32); out.perms = res["perms"].ctypes.data
     _check(lib().mars_dgi_step(m.handle, g.handle, step_index & (2 ** 64 - 1), int(pair_base), B,
                                ctypes.byref(out)))
-    m._last_nt = getattr(m, "_shard_rows", None) if getattr(g, "sharded", False) else g.total_nodes
     if want_loss:
         res["loss"] = float(res["loss"][0])
     return res
@@ -439,15 +484,15 @@ def dgi_step(m: DGI, g: Graph, step_index: int, pair_base: int = 0, global_batch
 def encode(m: DGI, g: Graph) -> np.ndarray:
     out = np.zeros((g.total_nodes, m.H), np.float32)
     _check(lib().mars_encode(m.handle, g.handle, _ptr(out)))
-    m._last_nt = None          # encode overwrote the saved activations
     return out
 
 
 def dgi_export_activations(m: DGI, layer: int):
     """Test hook: the last step's (Y_l, Z_l), stacked [pos; neg], as fp32 arrays."""
-    if getattr(m, "_last_nt", None) is None:
-        raise MarsError(MARS_ESTATE, "no step has run")
-    R = 2 * m._last_nt
+    nt = m.saved_rows()
+    if nt == 0:
+        raise MarsError(MARS_ESTATE, "no step has run since the last encode")
+    R = 2 * nt
     cin = m.F if layer == 1 else m.H
     Y = np.zeros((R, cin), np.float32)
     Z = np.zeros((R, m.H), np.float32)
@@ -455,7 +500,7 @@ def dgi_export_activations(m: DGI, layer: int):
     return Y, Z
 
 
-GEMM_IMPLS = {"auto": 0, "simt": 1, "3xtf32": 2}   # MARS_GEMM_* (include/mars.h)
+GEMM_IMPLS = {"auto": 0, "simt": 1}   # MARS_GEMM_* (include/mars.h)
 
 
 def debug_gemm(op: str, A, B, impl: str = "auto", iters: int = 0, device: int = 0):

@@ -11,6 +11,7 @@ import pytest
 import oracle
 import paper_conf_icpp_lancl21_b200 as mars
 from synth import graphs as SG
+from tests import stagewise
 from tests.util import scaled_err, split_params
 
 pytestmark = pytest.mark.gpu
@@ -60,35 +61,17 @@ def test_bf16_step(name, H):
     print("bf16", name, res)
 
 
-def test_bf16_bench_config_sampled():
+def test_bf16_bench_config_stagewise():
+    """The bench workload on the bf16 path: every stage of the step (forward
+    rows, head, dZ / dY / dW / dalpha of all three layers) against the oracle
+    at the GPU's own bf16 stage inputs, 2e-2 (tests/stagewise.py)."""
     gs = [SG.cached("gnmt", i) for i in range(16)]
     F, H = 64, 256
-    g, m, b, p0, out = _run(gs, F, H, 0, B=16)
-    perms = b.perms(0, 0, 0)
-    assert np.array_equal(out["perms"], perms)
-    P = split_params(p0, F, H)
-    rng = np.random.default_rng(1)
-    rows = np.unique(np.concatenate([rng.integers(0, 2 * b.Nt, 300), [0, 2 * b.Nt - 1]]))
-    prev = oracle.layer1_input(b, perms)
-    for l in (1, 2, 3):
-        Y, Z = m.export_activations(l)
-        W = P[f"W{l}"].reshape(-1, H)
-        y = oracle.spmm_rows(b, prev, rows, None if l == 1 else P["alpha"][l - 2])
-        assert scaled_err(Y[rows], y) <= TOL
-        # the GEMM consumes bf16(W): compare against the bf16-rounded weights
-        Wb = W.astype(np.float32)
-        Wb = (Wb.view(np.uint32) + 0x7FFF + ((Wb.view(np.uint32) >> 16) & 1)) & 0xFFFF0000
-        Wb = Wb.astype(np.uint32).view(np.float32).astype(np.float64)
-        assert scaled_err(Z[rows], Y[rows].astype(np.float64) @ Wb) <= TOL
-        prev = Z
-    loss, s, dM, dZ3, da3 = oracle.head(b, H, p0, prev, B=16)
-    assert abs(out["loss"] - loss) / loss <= 1e-4
-    G = split_params(out["grads"], F, H)
-    assert scaled_err(G["M"].reshape(H, H), dM) <= TOL
-    Y3, _ = m.export_activations(3)
-    e = scaled_err(G["W3"].reshape(H, H), Y3.astype(np.float64).T @ dZ3)
-    print("bf16 bench-config dW3 stage-wise err", e)
-    assert e <= TOL
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=0, precision=mars.MARS_BF16)
+    stagewise.step_stagewise(m, g, gs, F, H, 0, step=0, base=0, B=16, bf16=True, tol=TOL,
+                             rng_seed=1)
+    m.free(); g.free()
 
 
 def test_bf16_training_decreases_loss():

@@ -1,6 +1,6 @@
 """Dense-transform kernels in isolation (mars_debug_gemm) vs fp64 numpy:
-tcgen05 3xFP16 ('auto' rows) and 3xTF32 ('3xtf32', and 'auto' dW) and FFMA
-paths, ragged row counts, both operand majors, wide dynamic ranges."""
+tcgen05 3xFP16 ('auto') and FFMA ('simt') paths, ragged row counts, both
+operand majors, wide dynamic ranges."""
 import numpy as np
 import pytest
 
@@ -10,7 +10,7 @@ from tests.util import scaled_err
 pytestmark = pytest.mark.gpu
 
 
-@pytest.mark.parametrize("impl", ["auto", "3xtf32", "simt"])
+@pytest.mark.parametrize("impl", ["auto", "simt"])
 @pytest.mark.parametrize("M,N,K", [(128, 256, 64), (1000, 256, 256), (4133, 256, 64),
                                    (777, 64, 256), (300, 128, 256)])
 def test_rows(impl, M, N, K):
@@ -45,35 +45,46 @@ def _row_err(C, ref):
     return float(np.max(num / den))
 
 
-@pytest.mark.parametrize("impl", ["auto", "3xtf32"])
 @pytest.mark.parametrize("N,K", [(256, 256), (64, 256), (256, 64)])
-def test_rows_dynamic_range(impl, N, K):
-    """Rows spanning 1e-30 .. 1e30 (far outside fp16's range; the 3xFP16 kernel
-    scales every row by a power of two), zero rows, and weights of magnitude
-    1e4 and 1e-6: every row accurate relative to its own scale."""
+def test_rows_dynamic_range(N, K):
+    """Rows spanning 1e-30 .. 1e30 and rows near the top of fp32's range
+    (max |x| up to 2^126: the 3xFP16 kernel scales every row by a power of two,
+    unclamped for large rows), zero rows, and weights of magnitude 1e4 and 1e-6:
+    every row accurate relative to its own scale."""
     rng = np.random.default_rng(N + K)
     M = 1031
     A = rng.standard_normal((M, K))
     A *= 10.0 ** rng.uniform(-30, 30, (M, 1))
     A[rng.integers(0, M, 7)] = 0.0
+    big = rng.integers(0, M, 9)
+    A[big] = rng.standard_normal((9, K)) * 2.0 ** rng.uniform(110, 122, (9, 1))
     A = A.astype(np.float32)
-    for wscale in (1e4, 1e-6):
+    for wscale in (1e-4, 1e-6):
         B = (rng.standard_normal((N, K)) * wscale).astype(np.float32)
-        C, _ = mars.debug_gemm("rows", A, B, impl)
+        C, _ = mars.debug_gemm("rows", A, B, "auto")
         ref = A.astype(np.float64) @ B.astype(np.float64).T
         e = _row_err(C, ref)
-        print(impl, N, K, wscale, e)
+        print(N, K, wscale, e)
         assert np.all(np.isfinite(C)) and e < 5e-6
 
 
-def test_timing_report():
-    rng = np.random.default_rng(0)
-    R = 419232
-    for K in (64, 256):
-        A = rng.standard_normal((R, K)).astype(np.float32)
-        W = rng.standard_normal((256, K)).astype(np.float32)
-        D = rng.standard_normal((R, 256)).astype(np.float32)
-        for impl in ("auto", "3xtf32", "simt"):
-            _, t1 = mars.debug_gemm("rows", A, W, impl, iters=5)
-            _, t2 = mars.debug_gemm("dw", A, D, impl, iters=5)
-            print(f"TIMING K={K} {impl}: rows {t1:.3f} ms  dw {t2:.3f} ms")
+@pytest.mark.parametrize("H,K", [(256, 64), (256, 256), (128, 128)])
+def test_dw_mixed_magnitude_columns(H, K):
+    """The weight gradient scales each operand by ONE power of two per row chunk
+    (the chunk's largest value), so its error bound is normwise
+    per chunk, not per element.  Columns whose magnitudes span 8 decades
+    (shape features normalised to ~1e-6 next to one-hot features) must still
+    meet the componentwise GEMM bound |err_ij| <= tol · Σ_r |A_ri| |B_rj|."""
+    rng = np.random.default_rng(H + K)
+    M = 20011
+    A = rng.standard_normal((M, K)) * 10.0 ** rng.uniform(-8, 0, (1, K))
+    B = rng.standard_normal((M, H)) * 10.0 ** rng.uniform(-4, 0, (1, H))
+    A = A.astype(np.float32)
+    B = B.astype(np.float32)
+    C, _ = mars.debug_gemm("dw", A, B, "auto")
+    A64, B64 = A.astype(np.float64), B.astype(np.float64)
+    ref = A64.T @ B64
+    bound = np.abs(A64).T @ np.abs(B64)
+    comp = float(np.max(np.abs(C - ref) / bound))
+    print("componentwise", H, K, comp, "normwise", scaled_err(C, ref))
+    assert comp < 2e-5

@@ -13,6 +13,7 @@ import pytest
 import oracle
 import paper_conf_icpp_lancl21_b200 as mars
 from synth import graphs as SG
+from tests import stagewise
 from tests.util import scaled_err, split_params
 
 pytestmark = pytest.mark.gpu
@@ -131,12 +132,14 @@ def _forward_backward_case(gs, F, H, seed, e2e_grads=True, step=0, base=0):
     flips = sum(int(np.sum((acts[k] > 0) != (ref[k] > 0))) for k in ("Z1", "Z2", "Z3"))
     res["sign_flips"] = flips
     if e2e_grads:
+        # the gate must be visible: on the well-conditioned sizes it is
+        # requested for, a sign disagreement fails the test outright
+        assert flips == 0, f"P4 gate: {flips} PReLU sign disagreements vs the fp64 forward"
         loss_e, grads_e, _ = oracle.backward(b, H, p0, ref)
         for name, blk in split_params(out["grads"], F, H).items():
             e = scaled_err(blk, split_params(grads_e, F, H)[name])
             res["P4_" + name] = e
-            if flips == 0:
-                assert e <= TOL, (name, e)
+            assert e <= TOL, (name, e)
     # Adam stage-wise: the oracle's Adam applied to the GPU's gradients
     p1, m1, v1, t1 = m.get_state()
     assert t1 == 1
@@ -169,40 +172,19 @@ def test_step_gnmt_stagewise():
     _forward_backward_case([SG.cached("gnmt", 0)], 64, 256, 2, e2e_grads=False)
 
 
-def test_bench_config_sampled():
-    """The bench workload (16 GNMT graphs, F=64, H=256) in the bench's launch
-    configuration: sampled rows of every layer stage-wise, the head (loss, dM,
-    dalpha3) from the GPU's Z3, permutations bit-exact."""
+def test_bench_config_stagewise():
+    """The bench workload (16 GNMT graphs, F=64, H=256, R = 419k stacked rows) in
+    the bench's launch configuration, every stage of the step against the oracle
+    at the GPU's own stage inputs (tests/stagewise.py): sampled Y_l / Z_l rows,
+    the head (loss, dM, dZ3, dalpha3), and all rows of dW3, dY3, dZ2, dalpha2,
+    dW2, dY2, dZ1, dalpha1, dW1 -- every backward kernel instantiation the
+    bench times (k_tc3h_dw<64,256> included)."""
     gs = [SG.cached("gnmt", i) for i in range(16)]
     F, H, seed = 64, 256, 0
-    g, m, b = _setup(gs, F, H, seed)
-    p0 = m.get_state()[0].astype(np.float64)
-    out = m.step(g, 1, 0, global_batch=16, want_loss=True, want_grads=True, want_perms=True)
-    perms = b.perms(seed, 1, 0)
-    assert np.array_equal(out["perms"], perms)
-    P = split_params(p0, F, H)
-    rng = np.random.default_rng(0)
-    rows = np.unique(np.concatenate([rng.integers(0, 2 * b.Nt, 300), [0, b.Nt - 1, b.Nt,
-                                                                      2 * b.Nt - 1]]))
-    prev = oracle.layer1_input(b, perms)
-    for l in (1, 2, 3):
-        Y, Z = m.export_activations(l)
-        W = P[f"W{l}"].reshape(-1, H)
-        y = oracle.spmm_rows(b, prev, rows, None if l == 1 else P["alpha"][l - 2])
-        assert scaled_err(Y[rows], y) <= TOL
-        assert scaled_err(Z[rows], Y[rows].astype(np.float64) @ W) <= TOL
-        prev = Z
-    loss, s, dM, dZ3, da3 = oracle.head(b, H, p0, prev, B=16)
-    assert abs(out["loss"] - loss) / loss <= TOL
-    G = split_params(out["grads"], F, H)
-    assert scaled_err(G["M"].reshape(H, H), dM) <= TOL
-    assert abs(G["alpha"][2] - da3) <= TOL * max(abs(da3), 1e-12) * 10
-    # dW3 = Y3ᵀ dZ3 over all 2ΣN = 419k rows (the longest reduction of the step),
-    # stage-wise from the GPU's Y3 and the oracle's dZ3
-    Y3, _ = m.export_activations(3)
-    e = scaled_err(G["W3"].reshape(H, H), Y3.astype(np.float64).T @ dZ3)
-    print("bench-config dW3 stage-wise err", e)
-    assert e <= TOL
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=seed)
+    stagewise.step_stagewise(m, g, gs, F, H, seed, step=1, base=0, B=16, bf16=False, tol=TOL)
+    m.free(); g.free()
 
 
 def test_capture_replay_matches_eager():
@@ -283,3 +265,50 @@ def test_nccl_allreduce_path_one_rank():
         lb = mb.step(g, t, 0, want_loss=True)["loss"]
         assert la == lb
     assert np.array_equal(ma.get_state()[0], mb.get_state()[0])
+
+
+def test_nonfinite_step_skips_adam():
+    """Guarded update (adam.cu): a step whose loss or gradient is non-finite
+    leaves params, Adam m / v and t untouched on the device, and the next read
+    reports MARS_ENUMERIC once; a later finite step updates normally."""
+    gs = [SG.tiny(0), SG.tiny(1)]
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=16, hidden_dim=32, seed=3)
+    m.step(g, 0, 0, want_loss=True)
+    p1, m1, v1, t1 = m.get_state()
+    assert t1 == 1
+    bad = p1.copy()
+    bad[5] = np.inf                                   # W1 entry -> non-finite forward
+    m.set_state(bad, m1, v1, t1)
+    for s in (1, 2):                                  # eager, then captured replay
+        with pytest.raises(mars.MarsError) as e:
+            m.step(g, s, 0, want_loss=True)
+        assert e.value.status == mars.mars.MARS_ENUMERIC
+        p2, m2, v2, t2 = m.get_state()
+        assert t2 == 1 and np.array_equal(m2, m1) and np.array_equal(v2, v1)
+        assert np.array_equal(p2[np.isfinite(bad)], bad[np.isfinite(bad)])
+    m.set_state(p1, m1, v1, t1)
+    m.step(g, 3, 0)                                   # no outputs requested: asynchronous
+    loss, _ = m.read_step(want_grads=False)           # reports the step, which was finite
+    assert np.isfinite(loss)
+    assert m.get_state()[3] == 2
+
+
+def test_two_models_share_a_graph_with_long_rows():
+    """Two models stepping the same graph set concurrently on their own streams
+    (the long-row segment scratch is per model): results equal the
+    same steps run one after the other."""
+    gs = [SG.cached("bert", 0)]
+    g = mars.graph_load(gs)
+    ref = []
+    for seed in (1, 2):
+        m = mars.dgi_create(in_dim=64, hidden_dim=256, seed=seed)
+        ref.append(m.step(g, 0, 0, want_loss=True, want_grads=True))
+        m.free()
+    ms = [mars.dgi_create(in_dim=64, hidden_dim=256, seed=seed) for seed in (1, 2)]
+    for m in ms:
+        m.set_graph_capture(False)
+        m.step(g, 0, 0)                               # both enqueued before either is read
+    for m, r in zip(ms, ref):
+        loss, grads = m.read_step()
+        assert loss == r["loss"] and np.array_equal(grads, r["grads"])

@@ -296,3 +296,88 @@ def test_xavier_bounds_and_alpha():
     assert np.all(np.abs(P["W1"]) <= b1) and np.all(np.abs(P["W2"]) <= b2)
     assert abs(P["W1"].mean()) < 0.01 and abs(P["M"].std() - b2 / math.sqrt(3)) < 0.005
     assert np.all(P["alpha"] == np.float32(0.25))
+
+
+def test_head_tail_finite_differences():
+    """oracle_head's tail (a11 + the PReLU stage of a12 at layer 3): dZ3 and
+    dalpha3 are the derivatives of its own loss w.r.t. Z3 and alpha3 --
+    pinned by central differences of that loss (entries with |Z3| > 1e-3, so no
+    step crosses the PReLU kink)."""
+    gl = [SG.tiny(0), SG.tiny(1)]
+    b = oracle.Batch(gl)
+    F, H = 16, 32
+    p = oracle.xavier(5, F, H).astype(np.float64)
+    p[-1] = 0.3
+    Z3 = oracle.forward(b, H, p, b.perms(5, 0, 0))["Z3"]
+    loss, s, dM, dZ3, da3 = oracle.head(b, H, p, Z3, B=2)
+    rng = np.random.default_rng(0)
+    h = 1e-6
+    cand = np.flatnonzero(np.abs(Z3.ravel()) > 1e-3)
+    for e in rng.choice(cand, 40, replace=False):
+        Zp = Z3.copy().ravel(); Zp[e] += h
+        Zm = Z3.copy().ravel(); Zm[e] -= h
+        fd = (oracle.head(b, H, p, Zp.reshape(Z3.shape), B=2)[0] -
+              oracle.head(b, H, p, Zm.reshape(Z3.shape), B=2)[0]) / (2 * h)
+        assert abs(fd - dZ3.ravel()[e]) <= 1e-7 * max(np.abs(dZ3).max(), 1e-30), e
+    q = p.copy(); q[-1] += h
+    lp = oracle.head(b, H, q, Z3, B=2)[0]
+    q[-1] -= 2 * h
+    lm = oracle.head(b, H, q, Z3, B=2)[0]
+    assert abs((lp - lm) / (2 * h) - da3) <= 1e-7 * max(abs(da3), 1e-12)
+
+
+def test_stagewise_backward_composes_to_oracle_backward():
+    """The stage functions the full-size GPU tests chain (oracle.head,
+    oracle.prelu_backward, oracle.spmm_rows with identity act, and the dense
+    products dW = Yᵀ dZ, dY = dZ Wᵀ of row a12) reproduce oracle_backward
+    (itself pinned by finite differences and torch autograd) on a batch."""
+    gl = [SG.tiny(i) for i in range(3)]
+    b = oracle.Batch(gl)
+    F, H = 16, 32
+    p = oracle.xavier(8, F, H).astype(np.float64)
+    p[-3:] = [0.2, 0.35, 0.1]
+    acts = oracle.forward(b, H, p, b.perms(8, 1, 4))
+    loss_ref, g_ref, _ = oracle.backward(b, H, p, acts, B=5)
+    P = split_params(p, F, H)
+    loss, s, dM, dZ, da3 = oracle.head(b, H, p, acts["Z3"], B=5)
+    g = {"M": dM.ravel(), "alpha": [0.0, 0.0, da3]}
+    rows = np.arange(2 * b.Nt)
+    for l in (3, 2, 1):
+        g[f"W{l}"] = (acts[f"Y{l}"].T @ dZ).ravel()
+        if l > 1:
+            dY = dZ @ P[f"W{l}"].reshape(-1, H).T
+            dH = oracle.spmm_rows(b, dY, rows)
+            dZ, g["alpha"][l - 2] = oracle.prelu_backward(dH, acts[f"Z{l - 1}"], P["alpha"][l - 2])
+    assert abs(loss - loss_ref) < 1e-14
+    for name, ref in split_params(g_ref, F, H).items():
+        assert scaled_err(np.asarray(g[name]), ref) < 1e-12, name
+
+
+def _sm64_py(z):
+    """splitmix64 mixer in Python integers -- a second implementation, checked
+    against the published reference vectors (tests/golden/splitmix64.json)."""
+    M = (1 << 64) - 1
+    z = (z + 0x9E3779B97F4A7C15) & M
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M
+    return z ^ (z >> 31)
+
+
+def test_xavier_against_independent_generator():
+    """Reading c14 computed a second way (Python integers + the stdlib's correctly
+    rounded float arithmetic, splitmix64 pinned by the reference vectors): every
+    entry of W1 and M at a few indices, both matrices' tags, bitwise."""
+    with open(os.path.join(GOLDEN, "splitmix64.json")) as f:
+        gold = json.load(f)
+    x = gold["seed"]
+    for want in gold["outputs"]:
+        assert _sm64_py(x) == want
+        x = (x + 0x9E3779B97F4A7C15) & ((1 << 64) - 1)
+    F, H, seed = 64, 256, 20211
+    p = split_params(oracle.xavier(seed, F, H), F, H)
+    for tag, name, fan_in in ((1, "W1", F), (2, "W2", H), (4, "M", H)):
+        b = float(np.float32(math.sqrt(6.0 / (fan_in + H))))
+        base = _sm64_py(seed ^ tag)
+        for idx in (0, 1, 255, 4097, fan_in * H - 1):
+            u = (_sm64_py(base ^ idx) >> 40) / 16777216.0
+            assert p[name][idx] == np.float32((2.0 * u - 1.0) * b), (name, idx)
