@@ -96,6 +96,18 @@ MARS_API mars_status mars_graph_size(const mars_graph* g, int32_t graph_idx, int
 MARS_API mars_status mars_graph_export_csr(const mars_graph* g, int32_t graph_idx, int32_t* rowptr,
                                   int32_t* colind, int32_t* deg, float* dinv, float* vals);
 
+/* NEXT-1 featuriser ("the operation type is encoded as a one-hot
+ * vector ... input and output shapes ... normalised"; reading c16): writes the
+ * feature matrix X [N x F] (host, row-major fp32) of one op graph from its op
+ * types [N] (>= 0; types >= F - 8 share the last type slot, "other") and shape
+ * dims [N x 8] (int64: the first input's 4 dims then the op's 4 output dims;
+ * <= 0 = absent / unknown).  Slots [0, F-8): one-hot type; [F-8, F): each dim
+ * divided by the largest dim of the graph (f32 of the double quotient), 0 for
+ * unknown dims.  Runs on `device`; synchronous; inputs borrowed.  EINVAL on
+ * N < 1, an unsupported F, or a negative type. */
+MARS_API mars_status mars_featurize(const int32_t* types, const int64_t* dims, int32_t num_nodes,
+                                    int32_t feat_dim, int32_t device, float* X);
+
 /* ------------------------------------------------------------------------ */
 /* The pre-training model: 3 GCN layers with PReLU (Eq. 1),     */
 /* sigmoid-mean readout (Eq. 4), bilinear discriminator (Eq. 5), BCE (Eq. 6), */

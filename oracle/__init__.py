@@ -78,6 +78,8 @@ def lib():
                                            ctypes.c_double, ctypes.c_int64, i64p, f64p]
             L.oracle_prelu_backward.restype = ctypes.c_double
             L.oracle_prelu_backward.argtypes = [ctypes.c_int64, f64p, f64p, ctypes.c_double, f64p]
+            L.oracle_featurize.restype = ctypes.c_int
+            L.oracle_featurize.argtypes = [ctypes.c_int32, ctypes.c_int32, i32p, i64p, f32p]
             L.oracle_dense_anorm.restype = None
             L.oracle_dense_anorm.argtypes = [ctypes.c_int32, i32p, f64p]
             L.oracle_dense_step.restype = ctypes.c_double
@@ -130,6 +132,17 @@ def perm(seed: int, step: int, pair: int, num_nodes: int) -> np.ndarray:
     lib().oracle_perm(ctypes.c_uint64(seed & (2**64 - 1)), ctypes.c_uint64(step & (2**64 - 1)),
                       ctypes.c_uint64(pair & (2**64 - 1)), int(num_nodes), out)
     return out[:num_nodes]
+
+
+def featurize(types, dims, F: int) -> np.ndarray:
+    """NEXT-1 featuriser (reading c16): X [N x F] from op types [N] and
+    shape dims [N x 8] (first input's 4, output's 4; <= 0 unknown)."""
+    types = np.ascontiguousarray(types, np.int32)
+    dims = np.ascontiguousarray(dims, np.int64).reshape(-1, 8)
+    X = np.zeros((types.size, F), np.float32)
+    if lib().oracle_featurize(types.size, F, types, dims, X) != 0:
+        raise ValueError("negative op type")
+    return X
 
 
 def xavier(seed: int, F: int, H: int) -> np.ndarray:

@@ -272,6 +272,12 @@ cudaError_t launch_prelu(const void* Z, int bf16, const float* alpha_dev, int la
 // fp32 copy of a bf16 array (export hooks)
 cudaError_t launch_upcast(const void* in, float* out, int64_t n, cudaStream_t s);
 
+// ---------------------------------------------------------------- featurize.cu
+// NEXT-1: X [N x F] from op types [N] and shape dims [N x 8] (device buffers);
+// dmax: one device u64 of scratch.
+cudaError_t launch_featurize(const int32_t* types, const int64_t* dims, int32_t N, int32_t F,
+                             unsigned long long* dmax, float* X, cudaStream_t s);
+
 // ---------------------------------------------------------------- adam.cu
 // grads: [P + 1], the loss at grads[P]; guard_part: adam_guard_doubles() doubles.
 int adam_guard_doubles();

@@ -735,6 +735,45 @@ extern "C" mars_status mars_graph_export_csr(const mars_graph* g, int32_t idx, i
   return MARS_OK;
 }
 
+// ---------------------------------------------------------------- featuriser (NEXT-1)
+extern "C" mars_status mars_featurize(const int32_t* types, const int64_t* dims, int32_t N,
+                                      int32_t F, int32_t device, float* X) {
+  if (!types || !dims || !X) return fail(MARS_EINVAL, "NULL argument");
+  if (N < 1) return fail(MARS_EINVAL, "N < 1");
+  if (!valid_F(F)) return fail(MARS_EINVAL, "feat_dim %d not in {16,32,64,128,256}", F);
+  for (int32_t i = 0; i < N; ++i)
+    if (types[i] < 0) return fail(MARS_EINVAL, "op %d: negative type", i);
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "no CUDA device (libmars has no CPU fallback)");
+  }
+  if (device < 0 || device >= ndev) return fail(MARS_EINVAL, "bad device %d", device);
+  CK(cudaSetDevice(device));
+  cudaStream_t s = nullptr;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+  int32_t* d_types = nullptr;
+  int64_t* d_dims = nullptr;
+  float* d_X = nullptr;
+  unsigned long long* d_max = nullptr;
+  struct F1 { void* p; cudaStream_t s; ~F1() { if (p) cudaFreeAsync(p, s); } };
+  CK(palloc(&d_types, (size_t)N, s));
+  F1 f1{d_types, s};
+  CK(palloc(&d_dims, 8 * (size_t)N, s));
+  F1 f2{d_dims, s};
+  CK(palloc(&d_X, (size_t)N * F, s));
+  F1 f3{d_X, s};
+  CK(palloc(&d_max, 1, s));
+  F1 f4{d_max, s};
+  CK(cudaMemcpyAsync(d_types, types, sizeof(int32_t) * N, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(d_dims, dims, sizeof(int64_t) * 8 * N, cudaMemcpyHostToDevice, s));
+  CK(launch_featurize(d_types, d_dims, N, F, d_max, d_X, s));
+  CK(cudaMemcpyAsync(X, d_X, sizeof(float) * (size_t)N * F, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  return MARS_OK;
+}
+
 // ---------------------------------------------------------------- model create
 extern "C" mars_status mars_nccl_get_unique_id(void* out128) {
   if (!out128) return fail(MARS_EINVAL, "out is NULL");

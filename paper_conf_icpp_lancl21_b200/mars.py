@@ -110,6 +110,8 @@ SIGNATURES = {
     "mars_dp_export": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dp_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_graph_set_pair_offsets": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_featurize": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
+                                      ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -213,6 +215,17 @@ def corruption_samples(graphs, K: int):
     if K < 1:
         raise ValueError("K >= 1")
     return [g for g in graphs for _ in range(K)]
+
+
+def featurize(types, dims, feat_dim: int, device: int = 0) -> np.ndarray:
+    """mars_featurize (NEXT-1): X [N x F] from op types [N] and shape dims [N x 8]."""
+    t = np.ascontiguousarray(types, np.int32)
+    d = np.ascontiguousarray(dims, np.int64).reshape(-1, 8)
+    if d.shape[0] != t.size:
+        raise ValueError("one dims row per op")
+    X = np.zeros((t.size, feat_dim), np.float32)
+    _check(lib().mars_featurize(_ptr(t), _ptr(d), t.size, int(feat_dim), device, _ptr(X)))
+    return X
 
 
 def graph_load(graphs, device: int = 0) -> Graph:

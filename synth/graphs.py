@@ -77,7 +77,9 @@ class OpGraph:
     indptr: np.ndarray          # int64 [N+1], directed data-flow CSR (u -> consumers)
     indices: np.ndarray         # int32 [E]
     features: np.ndarray        # float32 [N, F]
-    types: np.ndarray = field(default=None)   # int32 [N] op-type index (for inspection)
+    types: np.ndarray = field(default=None)   # int32 [N] op-type index
+    dims: np.ndarray = field(default=None)    # int64 [N, 8]: first input's 4 dims, own
+                                              # output's 4 dims, 0 = unknown / absent
 
     @property
     def num_edges(self) -> int:
@@ -183,7 +185,20 @@ class _Builder:
         in_shapes = [self.shape[self.inputs[i][0]] if self.inputs[i] else () for i in order]
         out_shapes = [self.shape[i] for i in order]
         X = featurize(types, in_shapes, out_shapes, F)
-        return OpGraph(name, N, indptr, dst.astype(np.int32), X, types)
+        return OpGraph(name, N, indptr, dst.astype(np.int32), X, types,
+                       shape_dims(in_shapes, out_shapes))
+
+
+def shape_dims(in_shapes, out_shapes):
+    """[N, 8] int64: the first input's and the output's first 4 dims (0 = absent)."""
+    N = len(in_shapes)
+    dims = np.zeros((N, 8), np.int64)
+    for i in range(N):
+        for j, d in enumerate(tuple(in_shapes[i])[:4]):
+            dims[i, j] = d
+        for j, d in enumerate(tuple(out_shapes[i])[:4]):
+            dims[i, 4 + j] = d
+    return dims
 
 
 def featurize(types, in_shapes, out_shapes, F):
@@ -231,7 +246,8 @@ def tiny(seed_index: int = 0, N: int = 64, F: int = 16) -> OpGraph:
     indptr = np.zeros(N + 1, np.int64)
     np.add.at(indptr, src[o] + 1, 1)
     X = featurize(types, in_shapes, out_shapes, F)
-    return OpGraph("tiny", N, np.cumsum(indptr), dst[o].astype(np.int32), X, types)
+    return OpGraph("tiny", N, np.cumsum(indptr), dst[o].astype(np.int32), X, types,
+                   shape_dims(in_shapes, out_shapes))
 
 
 # =========================================================================== GNMT
@@ -614,13 +630,15 @@ def cached(name: str, index: int = 0, cache_dir: str | None = None, **kw) -> OpG
     path = os.path.join(cache_dir, f"{name}_{index}{'_' + tag if tag else ''}.npz")
     if os.path.exists(path):
         z = np.load(path)
-        return OpGraph(name, int(z["N"]), z["indptr"], z["indices"], z["X"], z["types"])
+        if "dims" in z.files:
+            return OpGraph(name, int(z["N"]), z["indptr"], z["indices"], z["X"], z["types"],
+                           z["dims"])
     g = make(name, index, **kw)
     try:
         os.makedirs(cache_dir, exist_ok=True)
         tmp = path + f".tmp{os.getpid()}.npz"
         np.savez(tmp, N=g.num_nodes, indptr=g.indptr, indices=g.indices, X=g.features,
-                 types=g.types)
+                 types=g.types, dims=g.dims)
         os.replace(tmp, path)
     except OSError:
         pass

@@ -16,11 +16,11 @@ difference upstream cannot flip a PReLU branch downstream (reading c19):
            dZ_{l-1}      oracle.prelu_backward(oracle.spmm_rows(dY_l(GPU)), Z_{l-1}(GPU))
            dalpha_{l-1}  the same call's sum                       all rows
 
-Matrices use the scaled max-norm max|gpu - ref| / max|ref|.  The dalpha_l are
-sums over 2ΣN·H terms of both signs; they are compared relative to
-Σ|dH·min(Z,0)| (reading c21: the sum's own scale, the
-scalar analogue of the scaled max-norm), and their plain relative error is
-reported beside it.
+Matrices use the scaled max-norm max|gpu - ref| / max|ref|; the scalars
+(loss, dalpha_l) their relative error |gpu - ref| / |ref| (key "dalpha<l>").
+The dalpha_l are sums over 2ΣN·H terms of both signs, so their error is also
+reported against Σ|dH·min(Z,0)|, the sum's own scale ("dalpha<l>_cond",
+diagnostic only).
 """
 import numpy as np
 
@@ -99,8 +99,8 @@ def step_stagewise(m, g, gs, F, H, seed, step, base, B, bf16, tol, nrows=300, rn
     _, dZ = m.export_backward(3)
     res["dZ3"] = _scaled(dZ, dZ3_ref)
     terms = np.abs(np.minimum(Z3.astype(np.float64), 0.0) * (dZ3_ref / np.where(Z3 > 0, 1.0, alpha[2])))
-    res["dalpha3_rel"] = abs(G["alpha"][2] - da3) / max(abs(da3), 1e-30)
-    res["dalpha3"] = abs(G["alpha"][2] - da3) / max(float(terms.sum()), 1e-30)
+    res["dalpha3"] = abs(G["alpha"][2] - da3) / max(abs(da3), 1e-30)
+    res["dalpha3_cond"] = abs(G["alpha"][2] - da3) / max(float(terms.sum()), 1e-30)
     del dZ3_ref, terms, Z3
 
     # ---- layers 3, 2, 1: dW, dY, aggregation + PReLU' (all rows, chunked)
@@ -134,15 +134,15 @@ def step_stagewise(m, g, gs, F, H, seed, step, base, B, bf16, tol, nrows=300, rn
             da += part
             mag += float(np.sum(np.abs(dH * np.minimum(z, 0.0))))
         res[f"dZ{l - 1}"] = e.err
-        res[f"dalpha{l - 1}_rel"] = abs(G["alpha"][l - 2] - da) / max(abs(da), 1e-30)
-        res[f"dalpha{l - 1}"] = abs(G["alpha"][l - 2] - da) / max(mag, 1e-30)
+        res[f"dalpha{l - 1}"] = abs(G["alpha"][l - 2] - da) / max(abs(da), 1e-30)
+        res[f"dalpha{l - 1}_cond"] = abs(G["alpha"][l - 2] - da) / max(mag, 1e-30)
         del dY64, Zp
         dZ = dZn
     m.set_keep_backward(False)
     print({k: f"{v:.2e}" for k, v in res.items()})
     loss_tol = 1e-4 if bf16 else tol
     for k, v in res.items():
-        if k.endswith("_rel"):
+        if k.endswith("_cond"):
             continue
         assert v <= (loss_tol if k == "loss" else tol), (k, v, res)
     return res

@@ -312,3 +312,32 @@ def test_two_models_share_a_graph_with_long_rows():
     for m, r in zip(ms, ref):
         loss, grads = m.read_step()
         assert loss == r["loss"] and np.array_equal(grads, r["grads"])
+
+
+def test_pretrain_matches_oracle_loop():
+    """NEXT-1: mars_dgi_pretrain against the oracle's own pre-training
+    loop -- oracle.step_grads + oracle.adam per step from the same init,
+    tracking the lowest loss (earliest wins, c17) -- on tiny graphs, where the
+    end-to-end gradients are well-conditioned (P4): every loss, the arg-min
+    step and its parameter snapshot, and the final parameters at 1e-5."""
+    gs = [SG.tiny(0), SG.tiny(1)]
+    F, H, n, lr, seed = 16, 32, 12, 3e-3, 21
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=seed, lr=lr)
+    p = m.get_state()[0].astype(np.float64)
+    res = m.pretrain(g, n, step0=5)
+    b = oracle.Batch(gs)
+    mo, vo = np.zeros_like(p), np.zeros_like(p)
+    losses, snaps = [], []
+    for t in range(n):
+        snaps.append(p.copy())
+        loss, grads, _, _ = oracle.step_grads(b, H, p, b.perms(seed, 5 + t, 0))
+        losses.append(loss)
+        p, mo, vo = oracle.adam(p, mo, vo, grads, t + 1, lr=lr)
+    losses = np.array(losses)
+    assert np.max(np.abs(res["losses"] - losses) / losses) <= 1e-5
+    k = int(np.argmin(losses))
+    assert res["best_step"] == k
+    assert abs(res["best_loss"] - losses[k]) <= 1e-5 * losses[k]
+    assert scaled_err(res["best_params"], snaps[k]) <= 1e-5
+    assert scaled_err(m.get_state()[0], p) <= 1e-5
