@@ -22,6 +22,8 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "internal.cuh"
@@ -389,6 +391,10 @@ cudaError_t rows3h_n(const float* A, const float* rs, const __half* Bhi, const _
 constexpr int kDwBK = 16;        // rows per stage = one K = 16 MMA step
 constexpr int kDwStages = 4;
 constexpr int kDwSub = 8;        // stages per TMEM work run (128 rows)
+#ifndef MARS_DW_PAIR
+#define MARS_DW_PAIR 1
+#endif
+constexpr bool kDwPair = MARS_DW_PAIR != 0;   // C_in = H = 256 on a CTA pair (k_tc3h_dw_pair)
 
 template <int CINT, int HH>
 struct H3DwCfg {
@@ -620,6 +626,244 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
   }
 }
 
+// ---------------------------------------------------------------- k_tc3h_dw_pair
+// The C_in = H = 256 weight gradient on a CTA pair (cta_group::2), so that no
+// operand is converted twice.  With one CTA per 128-column tile of C_in (the
+// kernel above), both tiles of a row chunk convert the whole dZ tile: 1.5x the
+// conversion work the GEMM needs, and the fp32 -> fp16 hi / lo conversion is
+// what bounds this kernel.  Here the pair splits both operands instead: CTA r
+// converts dZ columns (h) [128r, 128r + 128) and Y columns (c) [128r, 128r +
+// 128) of every 16-row stage; the even CTA issues one M = 256 (h), N = 256 (c)
+// pair MMA per product that reads the A half and the B half of each CTA from
+// the same shared-memory offsets; CTA r's TMEM accumulates D[h][c] for its 128
+// h rows and all 256 c columns (256 fp32 columns, double-buffered).
+// Synchronisation: the MMA commits multicast to both CTAs' empty / tfull
+// barriers; the even CTA's converter (folder) warps arrive on its own conv
+// (tempty) barrier; the odd CTA's converters (folders) first meet at a named
+// barrier, then ONE thread arrives on the even CTA's barrier (remote arrive).
+// Scaling, folding and the partial layout are those of k_tc3h_dw.
+constexpr int kPairStages = 6;
+
+struct H3PairCfg {
+  static constexpr int ATOM = 64 * kDwBK * 2;          // fp16 MN atom column: 64 cols x 16 rows
+  static constexpr int BOX32 = 32 * kDwBK * 4;         // one 32-column fp32 block: 16 rows x 128 B
+  static constexpr int HALF = 128;                     // columns of each operand per CTA
+  static constexpr int A32 = (HALF / 32) * BOX32;      // 8 KB
+  static constexpr int B32 = (HALF / 32) * BOX32;
+  static constexpr int A16 = (HALF / 64) * ATOM;       // 4 KB (hi; lo follows)
+  static constexpr int B16 = (HALF / 64) * ATOM;
+  static constexpr int STAGE = A32 + B32 + 2 * A16 + 2 * B16;   // 32 KB
+  static constexpr int SMEM = kPairStages * STAGE + 1024 + 512;
+  static constexpr uint32_t TMEM_COLS = 512;           // 2 buffers x 256 fp32 columns
+  static constexpr int MC = 128;                       // columns per folding thread
+};
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1)
+k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
+               const float* __restrict__ rs_dz, const float* __restrict__ rs_y,
+               float* __restrict__ part, int32_t R, int32_t rows_per_chunk) {
+  using Cfg = H3PairCfg;
+  constexpr int S = kPairStages;
+  constexpr int MC = Cfg::MC;
+  constexpr int CIN = 256, HH = 256;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
+  uint64_t* full = bars;
+  uint64_t* conv = bars + S;             // even CTA: both CTAs' converters
+  uint64_t* empty = bars + 2 * S;
+  uint64_t* tfull = bars + 3 * S;        // [2]
+  uint64_t* tempty = bars + 3 * S + 2;   // [2] even CTA: both CTAs' folders
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 4);
+  float* wmin = reinterpret_cast<float*>(bars + 3 * S + 6);   // [2][10] per-warp minima
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const int chunk = blockIdx.x >> 1;
+  const int32_t r0 = chunk * rows_per_chunk;
+  const int32_t r1 = min(R, r0 + rows_per_chunk);
+  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
+  const int nsub = (nk + kDwSub - 1) / kDwSub;
+  auto stA32 = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stB32 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32; };
+  auto stA16 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32 + Cfg::B32; };  // hi, lo
+  auto stB16 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32 + Cfg::B32 + 2 * Cfg::A16; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 11);         // 10 local converter warps + 1 from the odd CTA
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 9);        // 8 local folder warps + 1 from the odd CTA
+    }
+    fence_mbar_init();
+    tma_prefetch(&tmDZ);
+    tma_prefetch(&tmY);
+  }
+  if (warp == 1) tmem_alloc_pair(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  cluster_sync();                        // peers' barriers initialised, TMEM allocated
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer (both CTAs)
+      int s = 0;
+      uint32_t ph = 0;
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&empty[s], ph ^ 1);
+        mbar_expect_tx(&full[s], Cfg::A32 + Cfg::B32);
+        const int32_t row = r0 + kb * kDwBK;
+        tma_load_3d(stA32(s), &tmDZ, 0, row, (int)rank * (Cfg::HALF / 32), &full[s]);
+        tma_load_3d(stB32(s), &tmY, 0, row, (int)rank * (Cfg::HALF / 32), &full[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {                            // ---- pair MMA issuer
+      constexpr uint32_t idesc = idesc_f16(2 * Cfg::HALF, CIN) | (1u << 15) | (1u << 16);
+      int s = 0;
+      uint32_t ph = 0;
+      for (int sub = 0; sub < nsub; ++sub) {
+        const int buf = sub & 1;
+        mbar_wait_cluster(&tempty[buf], ((sub >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t twork = tbase + buf * CIN;
+        const int kb1 = min(nk, (sub + 1) * kDwSub);
+        for (int kb = sub * kDwSub; kb < kb1; ++kb) {
+          mbar_wait_cluster(&conv[s], ph);
+          tc_fence_after();
+          const uint32_t a = smem_u32(stA16(s)), al = a + Cfg::A16;
+          const uint32_t b = smem_u32(stB16(s)), bl = b + Cfg::B16;
+          const uint64_t ah = sdesc_sw128(a, Cfg::ATOM, 1024);
+          const uint64_t alo = sdesc_sw128(al, Cfg::ATOM, 1024);
+          const uint64_t bh = sdesc_sw128(b, Cfg::ATOM, 1024);
+          const uint64_t blo = sdesc_sw128(bl, Cfg::ATOM, 1024);
+          const uint32_t first = kb == sub * kDwSub ? 0u : 1u;
+          mma_f16_pair(twork, ah, bh, idesc, first);
+          mma_f16_pair(twork, ah, blo, idesc, 1);
+          mma_f16_pair(twork, alo, bh, idesc, 1);
+          mma_commit_pair(&empty[s], 0x3);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+        mma_commit_pair(&tfull[buf], 0x3);
+      }
+    }
+  } else {                         // ---- convert (warps 2..11); warps 4..11 also fold
+    const bool folder = warp >= 4;
+    const int ct = (warp - 2) * 32 + lane;
+    constexpr int NT = 10 * 32;
+    float mz = INFINITY, my = INFINITY;
+    for (int32_t r = r0 + ct; r < r1; r += NT) {
+      mz = fminf(mz, __ldg(rs_dz + r));
+      my = fminf(my, __ldg(rs_y + r));
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      mz = fminf(mz, __shfl_xor_sync(kFull, mz, o));
+      my = fminf(my, __shfl_xor_sync(kFull, my, o));
+    }
+    if (lane == 0) {
+      wmin[warp - 2] = mz;
+      wmin[10 + warp - 2] = my;
+    }
+    dwconv_bar();
+    float sz = INFINITY, sy = INFINITY;
+#pragma unroll
+    for (int k = 0; k < 10; ++k) {
+      sz = fminf(sz, wmin[k]);
+      sy = fminf(sy, wmin[10 + k]);
+    }
+    if (!(sz < INFINITY)) sz = 1.f;          // empty chunk
+    if (!(sy < INFINITY)) sy = 1.f;
+    const uint32_t conv0 = mapa_u32(conv, 0), tempty0 = mapa_u32(tempty, 0);
+
+    const int q = warp & 3, ch = (warp - 4) >> 2;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    float master[MC];
+#pragma unroll
+    for (int j = 0; j < MC; ++j) master[j] = 0.f;
+    int folded = 0;
+    auto fold = [&](int sub) {
+      const int buf = sub & 1;
+      mbar_wait(&tfull[buf], (sub >> 1) & 1);
+      tc_fence_after();
+      const uint32_t twork = tbase + buf * CIN + ch * MC;
+#pragma unroll
+      for (int c0 = 0; c0 < MC; c0 += 32) {
+        uint32_t w[32];
+        tmem_ld32(twork + lane_off + c0, w);
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 32; ++j) master[c0 + j] += __uint_as_float(w[j]);
+      }
+      tc_fence_before();
+      if (rank == 0) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[buf]);
+      } else {
+        asm volatile("bar.sync 3, 256;" ::: "memory");      // the 8 folder warps
+        if (threadIdx.x == 4 * 32) mbar_arrive_cluster(tempty0 + buf * 8);
+      }
+    };
+    constexpr int NTA = kDwBK * Cfg::HALF / 8;          // 8-column tasks of dZ per stage
+    constexpr int NTT = 2 * NTA;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int kb = 0; kb < nk; ++kb) {
+      mbar_wait(&full[s], ph);
+      for (int i = ct; i < NTT; i += NT) {
+        const bool isA = i < NTA;
+        const int ii = isA ? i : i - NTA;
+        const int r = ii % kDwBK, c0 = (ii / kDwBK) * 8;
+        const uint8_t* src = (isA ? stA32(s) : stB32(s)) + (c0 / 32) * Cfg::BOX32 + r * 128;
+        const int w0 = (c0 % 32) / 4;
+        const float4 v0 = *reinterpret_cast<const float4*>(src + ((w0 ^ (r & 7)) << 4));
+        const float4 v1 = *reinterpret_cast<const float4*>(src + (((w0 + 1) ^ (r & 7)) << 4));
+        const float sc = isA ? sz : sy;
+        const float x[8] = {v0.x * sc, v0.y * sc, v0.z * sc, v0.w * sc,
+                            v1.x * sc, v1.y * sc, v1.z * sc, v1.w * sc};
+        uint4 hv, lv;
+        split_h8(x, hv, lv);
+        uint8_t* dst = (isA ? stA16(s) : stB16(s)) + (c0 / 64) * Cfg::ATOM + r * 128 +
+                       ((((c0 % 64) / 8) ^ (r & 7)) << 4);
+        *reinterpret_cast<uint4*>(dst) = hv;
+        *reinterpret_cast<uint4*>(dst + Cfg::A16) = lv;      // A16 == B16
+      }
+      fence_proxy_async_smem();
+      if (rank == 0) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&conv[s]);
+      } else {
+        dwconv_bar();                                        // the 10 converter warps
+        if (threadIdx.x == 2 * 32) mbar_arrive_cluster(conv0 + s * 8);
+      }
+      if (++s == S) { s = 0; ph ^= 1; }
+      if (folder && (kb % kDwSub) == kDwSub / 2 && kb / kDwSub >= 1) fold(folded++);
+    }
+    if (folder) {
+      while (folded < nsub) fold(folded++);
+      const float inv = 1.f / (sz * sy);                   // exact (powers of two)
+      float* out = part + (int64_t)chunk * HH * CIN +
+                   (int64_t)(rank * Cfg::HALF + q * 32 + lane) * CIN + ch * MC;
+      float4* dst = reinterpret_cast<float4*>(out);
+#pragma unroll
+      for (int j = 0; j < MC / 4; ++j)
+        dst[j] = make_float4(master[4 * j] * inv, master[4 * j + 1] * inv,
+                             master[4 * j + 2] * inv, master[4 * j + 3] * inv);
+    }
+  }
+  tc_fence_before();
+  cluster_sync();                        // both CTAs done with TMEM and the peer's barriers
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc_pair(tbase, Cfg::TMEM_COLS);
+  }
+}
+
 __global__ void k_dw3h_reduce(const float* __restrict__ part, int nchunk, int CIN, int H,
                               float* __restrict__ dW) {
   dw_reduce_body(part, nchunk, CIN, H, dW);
@@ -642,6 +886,52 @@ cudaError_t dw3h_c(const float* Y, const float* rs_y, const float* dZ, const flo
     return cudaErrorInvalidValue;
   k_tc3h_dw<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part,
                                                                    (int32_t)R, rows, CIN);
+  return cudaGetLastError();
+}
+
+// Co-resident CTA pairs of k_tc3h_dw_pair (cudaOccupancyMaxActiveClusters).
+int dw_pair_clusters() {
+  static int n = 0;
+  if (!n) {
+    cudaFuncSetAttribute(k_tc3h_dw_pair, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         H3PairCfg::SMEM);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * 74, 1, 1);
+    cfg.blockDim = dim3(384, 1, 1);
+    cfg.dynamicSmemBytes = H3PairCfg::SMEM;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int c = 0;
+    if (cudaOccupancyMaxActiveClusters(&c, k_tc3h_dw_pair, &cfg) != cudaSuccess || c < 1) {
+      cudaGetLastError();
+      c = tc_num_sms() / 2;
+    }
+    n = c;
+    if (getenv("MARS_DEBUG_DW")) fprintf(stderr, "k_tc3h_dw_pair: %d co-resident CTA pairs\n", n);
+  }
+  return n;
+}
+
+cudaError_t dw3h_pair(const float* Y, const float* rs_y, const float* dZ, const float* rs_dz,
+                      float* part, int nchunk, int64_t R, int rows, cudaStream_t s) {
+  using Cfg = H3PairCfg;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_tc3h_dw_pair, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap tdz, ty;
+  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, 256, kDwBK, Cfg::HALF / 32) ||
+      !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, 256, kDwBK, Cfg::HALF / 32))
+    return cudaErrorInvalidValue;
+  k_tc3h_dw_pair<<<2 * nchunk, 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part, (int32_t)R, rows);
   return cudaGetLastError();
 }
 
@@ -695,6 +985,18 @@ cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, con
   nchunk = (int)((R + rows - 1) / rows);
   cudaError_t e;
   if (H != 128 && H != 256) return cudaErrorInvalidValue;
+  if (CIN == 256 && H == 256 && kDwPair) {
+    // one wave: as many row chunks as CTA pairs can be co-resident (a pair
+    // needs both SMs of a TPC free; not every SM can be paired)
+    nchunk = std::min(tc_dw_chunks(R, CIN), dw_pair_clusters());
+    rows = (int)((R + nchunk - 1) / nchunk);
+    rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
+    nchunk = (int)((R + rows - 1) / rows);
+    e = dw3h_pair(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, s);
+    if (e != cudaSuccess) return e;
+    k_dw3h_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
+    return cudaGetLastError();
+  }
   switch (CIN) {
     case 64: e = H == 256 ? dw3h_c<64, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s)
                           : dw3h_c<64, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s); break;
