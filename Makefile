@@ -10,7 +10,7 @@ ARCH := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
            -Xptxas -warn-spills -I include -DMARS_BUILD
 
-all: $(LIB) oracle/liboracle.so
+all: $(LIB) oracle/liboracle.so oracle/liboracle_omp.so
 
 build/obj/%.o: $(SRC)/%.cu $(HDR)
 	@mkdir -p build/obj
@@ -22,7 +22,11 @@ $(LIB): $(OBJ)
 oracle/liboracle.so: oracle/mars_oracle.c
 	gcc -O2 -std=c11 -fPIC -shared -fno-fast-math -ffp-contract=off -o $@ $< -lm
 
+# the same source with -fopenmp: bench.py's multi-core cpu_baseline (bitwise = serial)
+oracle/liboracle_omp.so: oracle/mars_oracle.c
+	gcc -O2 -std=c11 -fPIC -shared -fno-fast-math -ffp-contract=off -fopenmp -o $@ $< -lm
+
 clean:
-	rm -rf build/obj $(LIB) oracle/liboracle.so
+	rm -rf build/obj $(LIB) oracle/liboracle.so oracle/liboracle_omp.so
 
 .PHONY: all clean

@@ -170,12 +170,37 @@ def dist_env():
     return rank, world, local
 
 
+def host_info():
+    """os.cpu_count() and the CPU model (lscpu), for the CPU-baseline lines."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.startswith("Model name:"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return {"cpu_count": os.cpu_count(), "model": model}
+
+
+def oracle_step_seconds(oracle, graphs, H, seed=0):
+    """Wall seconds of one full fp64 oracle DGI step + Adam on `graphs`."""
+    b = oracle.Batch(graphs)
+    p = oracle.xavier(seed, b.F, H).astype(np.float64)
+    t0 = time.perf_counter()
+    loss, grads, _, _ = oracle.step_grads(b, H, p, b.perms(seed, 0, 0))
+    oracle.adam(p, np.zeros_like(p), np.zeros_like(p), grads, 1)
+    return time.perf_counter() - t0
+
+
 def run_reference(args):
-    """The oracle (fp64, single thread) on the host cores, as it stands."""
+    """The oracle (fp64; its OpenMP build on every host core) as it stands."""
     rank, world, _ = dist_env()
     if rank != 0:
         return 0
     import oracle
+    oracle.set_variant("omp")
     from synth import graphs as SG
     gen = WORKLOADS[args.workload][0]
     if args.workload == "1m":      # one GNMT graph stands in: a 1.1M-op fp64 step takes ~10 min
@@ -196,15 +221,16 @@ def run_reference(args):
     dt = time.perf_counter() - t0
     val = args.steps / dt
     sample = (f"1 {gen}-shaped graph per step (the smallest of the workload's "
-              f"{args.graphs_per_gpu}, N={small.num_nodes}), full DGI step + Adam in fp64")
+              f"{args.graphs_per_gpu}, N={small.num_nodes}), full DGI step + Adam in fp64, "
+              f"OpenMP build on {os.cpu_count()} host threads")
     line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * dt / args.steps,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": f"{args.workload} x{args.graphs_per_gpu} per GPU "
                                    f"(sampled: 1 graph/step)", "F": F, "H": H},
-            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": sample},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": os.cpu_count(), "kind": "oracle",
+                             "sample": sample, "host": host_info()},
             "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -481,7 +507,8 @@ def run_mine(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline and args.workload != "1m":
         import oracle
         # a bounded sample of the workload: whole graphs of the step, one at a
-        # time, until ~10 s of single-thread CPU work (at most 4 graphs)
+        # time, with the oracle's OpenMP build on every host core, until ~10 s
+        old = oracle.set_variant("omp")
         p0 = oracle.xavier(args.seed, F, H).astype(np.float64)
         t0 = time.perf_counter()
         done = 0
@@ -493,10 +520,24 @@ def run_mine(args):
             if time.perf_counter() - t0 > 10.0:
                 break
         dt = time.perf_counter() - t0
-        cpu = {"value": done / dt, "unit": UNIT, "cores": 1, "kind": "oracle",
+        # SURVEY §8(d)'s oracle table: seconds per step of one graph of each
+        # config, OpenMP (all cores) and serial, beside the GPU's per-graph time
+        table = {}
+        for name, Fc, Hc in (("tiny", 16, 32), ("inception", 64, 128), ("gnmt", 64, 256)):
+            g1 = [SG.tiny(0)] if name == "tiny" else [SG.cached(name, 0)]
+            row = {"N": g1[0].num_nodes, "F": Fc, "H": Hc,
+                   "omp_s": oracle_step_seconds(oracle, g1, Hc)}
+            oracle.set_variant("serial")
+            row["serial_s"] = oracle_step_seconds(oracle, g1, Hc)
+            oracle.set_variant("omp")
+            table[name] = row
+        oracle.set_variant(old)
+        cpu = {"value": done / dt, "unit": UNIT, "cores": os.cpu_count(), "kind": "oracle",
                "sample": f"{done} of the {b} {gen}-shaped graphs of a step (graphs 0..{done - 1}, "
-                         f"N={sum(x.num_nodes for x in graphs[:done])}), "
-                         f"full fp64 DGI step + Adam, single thread, {dt:.1f} s"}
+                         f"N={sum(x.num_nodes for x in graphs[:done])}), full fp64 DGI step + Adam, "
+                         f"OpenMP build of the oracle on {os.cpu_count()} threads, {dt:.1f} s",
+               "host": host_info(), "oracle_s_per_step": table,
+               "gpu_s_per_graph_step": (ms / args.steps / 1000.0) / b}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,

@@ -23,8 +23,10 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "mars_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
 _lock = threading.Lock()
-_lib = None
+_libs = {}
+_variant = "serial"
 
 i32p = np.ctypeslib.ndpointer(dtype=np.int32, flags="C_CONTIGUOUS")
 i64p = np.ctypeslib.ndpointer(dtype=np.int64, flags="C_CONTIGUOUS")
@@ -32,21 +34,34 @@ f32p = np.ctypeslib.ndpointer(dtype=np.float32, flags="C_CONTIGUOUS")
 f64p = np.ctypeslib.ndpointer(dtype=np.float64, flags="C_CONTIGUOUS")
 
 
-def build(force: bool = False) -> str:
-    """Compile liboracle.so with gcc -O2 (no fast-math: IEEE double throughout)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        tmp = _LIB + f".tmp{os.getpid()}"
+def build(force: bool = False, variant: str = "serial") -> str:
+    """Compile liboracle.so with gcc -O2 (no fast-math: IEEE double throughout);
+    variant "omp": the same source with -fopenmp (liboracle_omp.so, for the
+    multi-core CPU baseline; bitwise identical results)."""
+    out = _LIB_OMP if variant == "omp" else _LIB
+    if force or not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(_SRC):
+        tmp = out + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-fno-fast-math",
-                               "-ffp-contract=off", "-o", tmp, _SRC, "-lm"])
-        os.replace(tmp, _LIB)
-    return _LIB
+                               "-ffp-contract=off"] + (["-fopenmp"] if variant == "omp" else []) +
+                              ["-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, out)
+    return out
+
+
+def set_variant(variant: str) -> str:
+    """Select the build every later call uses: "serial" (default) or "omp"
+    (OpenMP over the outer loops; OMP_NUM_THREADS threads).  Returns the old one."""
+    global _variant
+    if variant not in ("serial", "omp"):
+        raise ValueError(variant)
+    old, _variant = _variant, variant
+    return old
 
 
 def lib():
-    global _lib
     with _lock:
-        if _lib is None:
-            L = ctypes.CDLL(build())
+        if _variant not in _libs:
+            L = ctypes.CDLL(build(variant=_variant))
             L.oracle_sm64.restype = ctypes.c_uint64
             L.oracle_sm64.argtypes = [ctypes.c_uint64]
             L.oracle_csr.restype = ctypes.c_int64
@@ -85,8 +100,8 @@ def lib():
             L.oracle_dense_step.restype = ctypes.c_double
             L.oracle_dense_step.argtypes = [ctypes.c_int32, i32p, ctypes.c_int32, ctypes.c_int32,
                                             f64p, i32p, f64p, f64p, ctypes.c_void_p]
-            _lib = L
-    return _lib
+            _libs[_variant] = L
+    return _libs[_variant]
 
 
 def num_params(F: int, H: int) -> int:

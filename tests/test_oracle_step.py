@@ -381,3 +381,24 @@ def test_xavier_against_independent_generator():
         for idx in (0, 1, 255, 4097, fan_in * H - 1):
             u = (_sm64_py(base ^ idx) >> 40) / 16777216.0
             assert p[name][idx] == np.float32((2.0 * u - 1.0) * b), (name, idx)
+
+
+def test_openmp_build_is_bitwise_serial():
+    """The OpenMP build of the oracle (bench.py's multi-core CPU baseline) splits
+    only outer loops with disjoint outputs and keeps every summation order, so a
+    full step is bitwise the serial build's."""
+    for gl, F, H in (([SG.tiny(i) for i in range(3)], 16, 32),
+                     ([SG.cached("inception", 0)], 64, 32)):
+        b = oracle.Batch(gl)
+        p = oracle.xavier(4, F, H).astype(np.float64)
+        perms = b.perms(4, 2, 0)
+        ref = oracle.step_grads(b, H, p, perms)
+        old = oracle.set_variant("omp")
+        try:
+            got = oracle.step_grads(b, H, p, perms)
+        finally:
+            oracle.set_variant(old)
+        assert got[0] == ref[0]
+        assert got[1].tobytes() == ref[1].tobytes()
+        for k in ref[3]:
+            assert got[3][k].tobytes() == ref[3][k].tobytes(), k

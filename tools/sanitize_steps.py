@@ -1,0 +1,30 @@
+"""compute-sanitizer workload (tools/sanitize.sh): one eager step per case on
+small sets -- tiny (SIMT GEMMs), Inception x2 at H = 128 and one Inception
+graph at H = 256 (tcgen05 row / dW kernels, incl. the CTA-pair dW), both
+precisions, plus an encode and the featuriser.  Small so the instrumented run
+finishes in minutes."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import paper_conf_icpp_lancl21_b200 as mars  # noqa: E402
+from synth import graphs as SG  # noqa: E402
+
+cases = [([SG.tiny(0), SG.tiny(1)], 16, 32, mars.MARS_FP32),
+         ([SG.cached("inception", i) for i in range(2)], 64, 128, mars.MARS_FP32),
+         ([SG.cached("inception", 0)], 64, 256, mars.MARS_FP32),
+         ([SG.cached("inception", 0)], 64, 256, mars.MARS_BF16),
+         ([SG.cached("bert", 0)], 64, 256, mars.MARS_FP32)]          # long rows
+for gs, F, H, prec in cases:
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=1, precision=prec)
+    m.set_graph_capture(False)
+    out = m.step(g, 0, 0, want_loss=True)
+    emb = m.encode(g)
+    print(f"N={sum(x.num_nodes for x in gs)} F={F} H={H} prec={prec} loss={out['loss']:.6f} "
+          f"emb finite={bool(np.isfinite(emb).all())}", flush=True)
+    m.free(); g.free()
+g0 = SG.cached("tiny", 0)
+X = mars.featurize(g0.types, g0.dims, 16)
+print("featurize ok", X.shape, flush=True)
