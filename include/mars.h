@@ -278,12 +278,70 @@ MARS_API mars_status mars_dp_export(const mars_dgi* m, void* blob);
  * not describe the same job (world size, ranks, parameter count). */
 MARS_API mars_status mars_dp_connect(mars_dgi* m, const void* blobs);
 
+/* Reloads a graph set in place (a1-a3): graphs[i] must have the node count
+ * and feat_dim of the set's graph i (the edges may differ).  The new edges and
+ * features go into the existing device buffers -- no allocation unless more
+ * entries of Â are stored than before -- after every step already enqueued
+ * on the old contents (waited for on the device, not the host).  Models keep
+ * the CUDA Graphs they captured for this handle when the number of stored
+ * entries and the long-row structure are unchanged: a data loader that
+ * alternates two handles re-captures nothing.  Synchronous with respect to
+ * the host for the CSR build (it returns when the set is ready).  EINVAL on
+ * mismatched sizes or malformed input (the set's contents are then undefined
+ * until a successful reload). */
+MARS_API mars_status mars_graph_reload(mars_graph* g, const mars_graph_desc* graphs,
+                                       int32_t num_graphs);
+
 /* Global pair indices of the graphs of a set (c15): graph i's corruption
  * seed uses pair index global_pair_base + pair_offsets[i] (default i).  With
  * a balanced (e.g. LPT) assignment of graphs to ranks, passing each graph's
  * global index keeps every graph's corruption independent of the rank count.
  * Host array [num_graphs], each >= 0.  Takes effect from the next step. */
 MARS_API mars_status mars_graph_set_pair_offsets(mars_graph* g, const int64_t* pair_offsets);
+
+/* ------------------------------------------------------------------------ */
+/* NEXT-2: the segment-level sequence-to-sequence placer, forward (PAPER.md  */
+/* §3.3, Fig. 6; sizes P:L234; readings c22-c28 in DESIGN.md).  */
+/* The op embeddings (mars_encode's output, in op order) are split into      */
+/* segments of s ops; a bidirectional LSTM (enc_hidden per direction) encodes */
+/* a segment starting from the previous segment's final states; a            */
+/* unidirectional LSTM (2 x enc_hidden) with Bahdanau additive attention     */
+/* over the segment's encoder outputs decodes one device per op, feeding the */
+/* previous op's device embedding back (start token per segment); devices    */
+/* are drawn by Gumbel-max from softmax(W_o s_t + b_o) with counter-based    */
+/* splitmix64 noise, so a draw depends only on (sample_seed, sample, op).    */
+/* ------------------------------------------------------------------------ */
+typedef struct mars_placer mars_placer;
+typedef struct {
+  int32_t in_dim;             /* H: width of the op embeddings (multiple of 16)   */
+  int32_t enc_hidden;         /* encoder LSTM size per direction: 64, 128, 256 (c22: 256) */
+  int32_t attn_dim;           /* attention size, multiple of 128 (c27: 512)       */
+  int32_t dev_embed;          /* device-embedding size in [1, 256] (c25: 64)       */
+  int32_t num_devices;        /* D in [2, 64]                                     */
+  int32_t segment;            /* s in [1, 1024] (128)                     */
+  uint64_t seed;              /* init (c28)                                       */
+  const float* init_params;   /* optional [mars_placer_num_params] host           */
+  int32_t device;
+} mars_placer_config;
+/* Defaults: H 256, enc_hidden 256, attn 512, dev_embed 64, D 4, s 128, seed 0. */
+MARS_API void mars_placer_config_default(mars_placer_config* cfg);
+MARS_API int64_t mars_placer_num_params(const mars_placer_config* cfg);
+MARS_API mars_status mars_placer_create(const mars_placer_config* cfg, mars_placer** out);
+/* Flat fp32 parameters (layout: DESIGN.md §12): host buffers, synchronous. */
+MARS_API mars_status mars_placer_get_params(const mars_placer* p, float* params);
+MARS_API mars_status mars_placer_set_params(mars_placer* p, const float* params);
+/* The placer forward for num_samples (1..32) placements of one op graph:
+ * embeddings [N x in_dim] (host, op order).  forced [num_samples x N] (host,
+ * optional): teacher forcing -- the decoder consumes these devices and
+ * log pi / entropy are evaluated for them (PPO's re-evaluation of sampled
+ * placements).  Outputs (host, each optional) [num_samples x N]: placements
+ * (the drawn or forced device per op), logp = log pi(placement) per op,
+ * entropy of pi per op.  Synchronous.  EINVAL on bad sizes or a forced device
+ * outside [0, D). */
+MARS_API mars_status mars_placer_sample(mars_placer* p, const float* embeddings, int32_t num_ops,
+                                        int32_t num_samples, uint64_t sample_seed,
+                                        const int32_t* forced, int32_t* placements, float* logp,
+                                        float* entropy);
 
 /* Copies the most recent step's loss and global-mean gradient (the values
  * Adam consumed) to host memory (either may be NULL).  Synchronous.  For a
@@ -354,7 +412,7 @@ MARS_API mars_status mars_shard_connect_local(mars_dgi* const* models, int32_t n
 /* Kernel launches enqueued by the most recent mars_dgi_step (for reporting). */
 MARS_API int64_t mars_dgi_last_launches(const mars_dgi* m);
 
-/* Frees a mars_graph* or mars_dgi* (tag-checked; NULL is a no-op). */
+/* Frees a mars_graph*, mars_dgi* or mars_placer* (tag-checked; NULL is a no-op). */
 MARS_API void mars_free(void* handle);
 
 #ifdef __cplusplus

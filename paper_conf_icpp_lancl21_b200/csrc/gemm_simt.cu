@@ -32,7 +32,7 @@ k_gemm(const float* __restrict__ A, const float* __restrict__ B, float* __restri
   static_assert(TM % 4 == 0 && TN % 4 == 0, "float4 micro-tiles");
   __shared__ __align__(16) float As[kBK][BM];
   __shared__ __align__(16) float Bs[kBK][BN];
-  constexpr int TX = BN / TN, TY = BM / TM;
+  constexpr int TX = BN / TN;
   constexpr int GM = TM / 4, GN = TN / 4;          // float4 groups per thread
   const int tid = threadIdx.x;
   const int tx = tid % TX, ty = tid / TX;

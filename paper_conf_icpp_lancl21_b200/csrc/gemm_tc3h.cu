@@ -66,11 +66,6 @@ __device__ __forceinline__ void conv_bar() {   // the 4 converter warps
   asm volatile("bar.sync 1, 128;" ::: "memory");
 }
 
-__device__ __forceinline__ uint32_t pack_h2(float a, float b) {
-  __half2 h = __floats2half2_rn(a, b);
-  return *reinterpret_cast<uint32_t*>(&h);
-}
-
 // x = hi + lo for 8 scaled values: hi = fp16_rn(x) (packed in pairs), read
 // back as fp32 to form lo = x - hi exactly, lo rounded to fp16.
 __device__ __forceinline__ void split_h8(const float (&x)[8], uint4& hi, uint4& lo) {

@@ -278,6 +278,40 @@ cudaError_t launch_upcast(const void* in, float* out, int64_t n, cudaStream_t s)
 cudaError_t launch_featurize(const int32_t* types, const int64_t* dims, int32_t N, int32_t F,
                              unsigned long long* dmax, float* X, cudaStream_t s);
 
+// ---------------------------------------------------------------- placer.cu (NEXT-2)
+struct PlacerDims {
+  int32_t H;      // op-embedding width (the DGI encoder's H)
+  int32_t Hd;     // encoder LSTM size per direction (c22: 256; decoder = 2 Hd)
+  int32_t A;      // attention size (c27)
+  int32_t De;     // device-embedding size (c25)
+  int32_t D;      // devices
+};
+struct PlacerParams {   // views into the flat parameter vector (c28 layout)
+  float *enc_wih[2], *enc_whh[2], *enc_b[2];
+  float *wq, *wk, *v;
+  float *dec_wih, *dec_whh, *dec_b;
+  float *emb, *wo, *bo;
+};
+struct PlacerWork {     // device scratch sized for N ops and S samples
+  float* xp[2];         // [N x 4Hd]
+  float* enc;           // [N x 2Hd]
+  float* keys;          // [N x A]
+  float *seg_h, *seg_c; // [nseg x 2Hd]
+  float* hbuf;          // [2 x 2 x Hd]
+  float *sh, *sc;       // [2 x S x 2Hd], [S x 2Hd]
+  float *q, *ghh, *score, *ctx;   // [S x A], [S x 8Hd], [S x seg], [S x 2Hd]
+  unsigned int* bar;    // [2] grid-barrier counters
+};
+int64_t placer_num_params(const PlacerDims& d);
+PlacerParams placer_views(const PlacerDims& d, float* base);
+cudaError_t placer_init(const PlacerDims& d, float* params, uint64_t seed, cudaStream_t s);
+cudaError_t placer_prepare(const PlacerDims& d);
+// E [N x H] device; place / logp / ent [S x N] device; forced [S x N] device or null.
+cudaError_t placer_forward(const PlacerDims& d, const PlacerParams& w, const PlacerWork& ws,
+                           const float* E, int32_t N, int32_t seg, int32_t S, uint64_t sample_seed,
+                           const int32_t* forced, int32_t* place, float* logp, float* ent,
+                           cudaStream_t s, int* launches);
+
 // ---------------------------------------------------------------- adam.cu
 // grads: [P + 1], the loss at grads[P]; guard_part: adam_guard_doubles() doubles.
 int adam_guard_doubles();

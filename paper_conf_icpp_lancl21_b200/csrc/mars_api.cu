@@ -26,6 +26,7 @@ namespace {
 constexpr uint64_t kTagGraph = 0x4D41525347524150ULL;  // "MARSGRAP"
 constexpr uint64_t kTagDgi = 0x4D41525344474931ULL;    // "MARSDGI1"
 constexpr uint64_t kTagDead = 0xDEADDEADDEADDEADULL;
+constexpr uint64_t kTagPlacer = 0x4D415253504C4331ULL;  // "MARSPLC1"
 constexpr int kChunkRows = 256;   // deterministic reduction chunk (rows, within one graph)
 
 thread_local std::string g_err;
@@ -204,6 +205,9 @@ struct mars_graph {
   int32_t *l_node_off = nullptr, *l_node_graph = nullptr, *l_chunk_row = nullptr,
           *l_chunk_graph = nullptr, *l_graph_chunk = nullptr;
   std::vector<void*> extra;         // long-row tables (pool memory)
+  std::vector<int32_t> h_long[3];   // host copies: long rows, segment offsets, segment rows
+  int64_t nnz_cap = 0;              // entries colind / vals can hold (mars_graph_reload)
+  int64_t Et_load = 0;
   // Last use per stream: every step / encode that reads this graph records an
   // event on its stream, so mars_free waits for exactly those uses (not for the
   // whole device, which would serialise against other models' steps).
@@ -250,7 +254,10 @@ struct mars_graph {
 // same graph concurrently never share it).
 // Everything on the loader's non-blocking stream `s` (no legacy-stream copies or
 // cudaMalloc, which would wait for a model's step running concurrently).
-static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s) {
+static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s,
+                                   bool* changed = nullptr) {
+  const GraphDev old = v;
+  if (changed) *changed = true;
   v.nlong = v.nseg = 0;
   v.long_min = 0x7fffffff;
   v.long_rows = v.long_seg = v.seg_row = nullptr;
@@ -272,7 +279,11 @@ static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s) 
     if (dmax) cudaFreeAsync(dmax, s);
     if (e0 == cudaSuccess) e0 = cudaStreamSynchronize(s);
     if (e0 != cudaSuccess) return e0;
-    if (hmax <= long_min) return cudaSuccess;
+    if (hmax <= long_min) {
+      if (changed) *changed = old.nlong != 0;
+      for (auto& h : gr->h_long) h.clear();
+      return cudaSuccess;
+    }
   }
   std::vector<int32_t> rp((size_t)v.Nt + 1);
   cudaError_t e = cudaMemcpyAsync(rp.data(), v.rowptr, sizeof(int32_t) * rp.size(),
@@ -289,7 +300,20 @@ static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s) 
     rows.push_back(i);
     seg.push_back(seg.back() + ns);
   }
-  if (rows.empty()) return cudaSuccess;
+  if (rows.empty()) {
+    if (changed) *changed = old.nlong != 0;
+    for (auto& h : gr->h_long) h.clear();
+    return cudaSuccess;
+  }
+  if (old.nlong == (int32_t)rows.size() && old.long_min == long_min && gr->h_long[0] == rows &&
+      gr->h_long[1] == seg && gr->h_long[2] == segrow) {   // reload: tables unchanged
+    v = old;
+    if (changed) *changed = false;
+    return cudaSuccess;
+  }
+  gr->h_long[0] = rows;
+  gr->h_long[1] = seg;
+  gr->h_long[2] = segrow;
   auto up = [&](const std::vector<int32_t>& h, const int32_t** d) -> cudaError_t {
     void* p = nullptr;
     cudaError_t e2 = cudaMallocAsync(&p, sizeof(int32_t) * h.size(), s);
@@ -357,11 +381,51 @@ struct mars_dgi {
   const mars_graph* ws_graph = nullptr;
   bool capture = true;
   int gemm_impl = 0;                // 0 auto (tcgen05 3xFP16 when supported), 1 SIMT FFMA
-  cudaGraphExec_t exec = nullptr;
-  uint64_t exec_graph = 0;          // uid of the graph set the exec was captured for
-  uint64_t prev_graph = 0;          // uid of the graph set of the previous step
-  cudaStream_t exec_stream = nullptr;
-  int64_t last_launches = 0, exec_launches = 0;
+  // Captured steps, one per (graph set, stream), least recently used evicted:
+  // a loader that alternates a few graph handles (mars_graph_reload) replays
+  // each handle's graph instead of launching the step's kernels eagerly.
+  struct ExecEntry {
+    uint64_t uid;
+    cudaStream_t stream;
+    cudaGraphExec_t exec;
+    int64_t launches;
+    uint64_t last;
+  };
+  static constexpr int kExecCache = 4;
+  std::vector<ExecEntry> execs;
+  uint64_t exec_clock = 0;
+  uint64_t seen[kExecCache] = {};   // uids of recent steps (capture on a set's second step)
+  int seen_next = 0;
+  int64_t last_launches = 0;
+  void drop_execs() {
+    for (auto& e : execs) cudaGraphExecDestroy(e.exec);
+    execs.clear();
+  }
+  ExecEntry* find_exec(uint64_t uid, cudaStream_t s) {
+    for (auto& e : execs)
+      if (e.uid == uid && e.stream == s) return &e;
+    return nullptr;
+  }
+  bool seen_recently(uint64_t uid) const {
+    for (uint64_t u : seen)
+      if (u == uid) return true;
+    return false;
+  }
+  void note_seen(uint64_t uid) {
+    if (seen_recently(uid)) return;
+    seen[seen_next] = uid;
+    seen_next = (seen_next + 1) % kExecCache;
+  }
+  ExecEntry* add_exec(uint64_t uid, cudaStream_t s, cudaGraphExec_t ex, int64_t launches) {
+    if ((int)execs.size() >= kExecCache) {
+      auto lru = std::min_element(execs.begin(), execs.end(),
+                                  [](const ExecEntry& a, const ExecEntry& b) { return a.last < b.last; });
+      cudaGraphExecDestroy(lru->exec);
+      execs.erase(lru);
+    }
+    execs.push_back(ExecEntry{uid, s, ex, launches, ++exec_clock});
+    return &execs.back();
+  }
   int32_t last_Nt = 0;              // node count of the last step's graph set (export hook)
   // keep_backward test hook: copies of dZ3, dZ2, dZ1 (kb_dZ[l]) and dY3, dY2
   // (kb_dY[l - 1]) of the last step, 2 * kb_rows rows each
@@ -411,7 +475,7 @@ struct mars_dgi {
     return sh.connected ? sh.gsum : dp.connected ? dp.gsum : grads;
   }
   ~mars_dgi() {
-    if (exec) cudaGraphExecDestroy(exec);
+    drop_execs();
     kb_release();
     for (void* p : sh.ipc) cudaIpcCloseMemHandle(p);
     for (void* p : sh.owned) cudaFree(p);
@@ -667,6 +731,8 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   gr->nnz = gr->h_nnz_off[G];
   CK(palloc(&gr->colind, (size_t)gr->nnz, s));
   CK(palloc(&gr->vals, (size_t)gr->nnz, s));
+  gr->nnz_cap = gr->nnz;
+  gr->Et_load = Et;
   CK(build_csr_phase2(io, gr->colind, gr->vals, s));
   CK(cudaStreamSynchronize(s));
 
@@ -692,6 +758,132 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   v.pair_off = gr->pair_off;
   CK(build_long_rows(gr, v, s));
   *out = guard.release();
+  return MARS_OK;
+}
+
+// In-place reload (a1-a3 again) of a graph set with the same graphs' node
+// counts and feature width: new edges and features into the existing device
+// buffers, on a private stream that first waits (on the device) for every
+// recorded use of the old contents.  The handle keeps its identity -- and the
+// steps models captured for it stay valid -- unless the stored-entry count or
+// the long-row structure changed (then it gets a new identity).
+extern "C" mars_status mars_graph_reload(mars_graph* gr, const mars_graph_desc* descs, int32_t G) {
+  if (mars_status st = check_graph(gr)) return st;
+  if (gr->sharded) return fail(MARS_EINVAL, "a row-sharded graph cannot be reloaded");
+  if (!descs || G != gr->G) return fail(MARS_EINVAL, "reload needs the same number of graphs");
+  const int F = gr->F;
+  int64_t Et = 0;
+  for (int g = 0; g < G; ++g) {
+    const mars_graph_desc& d = descs[g];
+    if (d.num_nodes != gr->h_node_off[g + 1] - gr->h_node_off[g])
+      return fail(MARS_EINVAL, "graph %d: reload needs the same node count", g);
+    if (d.feat_dim != F) return fail(MARS_EINVAL, "graph %d: feat_dim mismatch", g);
+    if (!d.indptr || !d.features || (!d.indices && d.indptr[d.num_nodes] > 0))
+      return fail(MARS_EINVAL, "graph %d: NULL array", g);
+    if (d.indptr[0] != 0 || d.indptr[d.num_nodes] < 0)
+      return fail(MARS_EINVAL, "graph %d: malformed indptr", g);
+    Et += d.indptr[d.num_nodes];
+  }
+  const int64_t Nt = gr->Nt;
+  if (Nt + 2 * Et >= (int64_t)INT32_MAX - 1) return fail(MARS_EINVAL, "graph set too large");
+  CK(cudaSetDevice(gr->device));
+  cudaStream_t s = nullptr;
+  CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  struct SG { cudaStream_t s; ~SG() { cudaStreamDestroy(s); } } sg{s};
+  {   // the old contents stay until every recorded use of them has run
+    std::lock_guard<std::mutex> lk(gr->use_mu);
+    for (auto& u : gr->uses) CK(cudaStreamWaitEvent(s, u.second, 0));
+  }
+  std::vector<int64_t> edge_off(G + 1, 0);
+  for (int g = 0; g < G; ++g) edge_off[g + 1] = edge_off[g] + descs[g].indptr[descs[g].num_nodes];
+  std::vector<void*> scratch;
+  struct SF {
+    std::vector<void*>* v;
+    cudaStream_t s;
+    ~SF() { for (void* p : *v) cudaFreeAsync(p, s); }
+  } sf{&scratch, s};
+  auto salloc = [&](void** p, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMallocAsync(p, bytes ? bytes : 4, s);
+    if (e == cudaSuccess) scratch.push_back(*p);
+    return e;
+  };
+  int64_t* d_indptr = nullptr;
+  int32_t* d_idx = nullptr;
+  int64_t* d_edge_off = nullptr;
+  CK(salloc((void**)&d_indptr, sizeof(int64_t) * (size_t)(Nt + G)));
+  CK(salloc((void**)&d_idx, sizeof(int32_t) * (size_t)std::max<int64_t>(Et, 1)));
+  CK(salloc((void**)&d_edge_off, sizeof(int64_t) * (G + 1)));
+  for (int g = 0; g < G; ++g) {   // pinned inputs are copied directly, pageable ones staged by CUDA
+    const mars_graph_desc& d = descs[g];
+    const int32_t N = d.num_nodes;
+    CK(cudaMemcpyAsync(d_indptr + gr->h_node_off[g] + g, d.indptr, sizeof(int64_t) * (N + 1),
+                       cudaMemcpyHostToDevice, s));
+    if (d.indptr[N] > 0)
+      CK(cudaMemcpyAsync(d_idx + edge_off[g], d.indices, sizeof(int32_t) * d.indptr[N],
+                         cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(gr->X + (int64_t)gr->h_node_off[g] * F, d.features,
+                       sizeof(float) * (size_t)N * F, cudaMemcpyHostToDevice, s));
+  }
+  CK(cudaMemcpyAsync(d_edge_off, edge_off.data(), sizeof(int64_t) * (G + 1), cudaMemcpyHostToDevice, s));
+  BuilderIO io{};
+  io.G = G;
+  io.Nt = (int32_t)Nt;
+  io.Et = Et;
+  io.indptr = d_indptr;
+  io.indices = d_idx;
+  io.node_off = gr->node_off;
+  io.edge_off = d_edge_off;
+  io.node_graph = gr->node_graph;
+  const int64_t cap = Nt + 2 * Et;
+  CK(salloc((void**)&io.cnt, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.off_dup, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.cursor, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.buf, sizeof(int32_t) * cap));
+  CK(salloc((void**)&io.buf2, sizeof(int32_t) * cap));
+  CK(salloc((void**)&io.ucnt, sizeof(int32_t) * (Nt + 1)));
+  CK(salloc((void**)&io.err, sizeof(int32_t) * 2));
+  io.scan_tmp_bytes = scan_tmp_bytes(Nt + 1);
+  CK(salloc(&io.scan_tmp, io.scan_tmp_bytes));
+  io.rowptr = gr->rowptr;
+  io.deg = gr->deg;
+  io.dinv = gr->dinv;
+  CK(build_csr_phase1(io, s));
+  std::vector<int32_t> hbuf((size_t)G + 3);
+  int32_t* d_nnzoff = io.ucnt;
+  k_gather_rowptr<<<cdiv(G + 1, 256), 256, 0, s>>>(gr->rowptr, gr->node_off, G, d_nnzoff);
+  CK(cudaGetLastError());
+  CK(cudaMemcpyAsync(hbuf.data(), d_nnzoff, sizeof(int32_t) * (G + 1), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(hbuf.data() + G + 1, io.err, sizeof(int32_t) * 2, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (hbuf[G + 1]) {
+    gr->uid = g_graph_uid.fetch_add(1);   // contents undefined until a successful reload
+    return fail(MARS_EINVAL, "malformed graph input (code %d): %s", hbuf[G + 1],
+                (hbuf[G + 1] & 2) ? "edge index out of range" : "indptr inconsistent");
+  }
+  const int64_t nnz_old = gr->nnz;
+  for (int g = 0; g <= G; ++g) gr->h_nnz_off[g] = hbuf[g];
+  gr->nnz = gr->h_nnz_off[G];
+  bool same = gr->nnz == nnz_old;
+  if (gr->nnz > gr->nnz_cap) {          // more stored entries than the buffers hold
+    cudaFreeAsync(gr->colind, s);
+    cudaFreeAsync(gr->vals, s);
+    gr->colind = nullptr;
+    gr->vals = nullptr;
+    CK(palloc(&gr->colind, (size_t)gr->nnz, s));
+    CK(palloc(&gr->vals, (size_t)gr->nnz, s));
+    gr->nnz_cap = gr->nnz;
+    same = false;
+  }
+  CK(build_csr_phase2(io, gr->colind, gr->vals, s));
+  GraphDev& v = gr->dev;
+  v.nnz = gr->nnz;
+  v.colind = gr->colind;
+  v.vals = gr->vals;
+  bool lchanged = true;
+  CK(build_long_rows(gr, v, s, &lchanged));
+  CK(cudaStreamSynchronize(s));
+  gr->Et = Et;
+  if (!same || lchanged) gr->uid = g_graph_uid.fetch_add(1);   // captured steps are stale
   return MARS_OK;
 }
 
@@ -894,11 +1086,7 @@ extern "C" mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl) {
   if (mars_status st = check_dgi(m)) return st;
   if (impl != MARS_GEMM_AUTO && impl != MARS_GEMM_SIMT)
     return fail(MARS_EINVAL, "bad gemm impl");
-  if (impl != m->gemm_impl && m->exec) {
-    cudaGraphExecDestroy(m->exec);
-    m->exec = nullptr;
-    m->exec_graph = 0;
-  }
+  if (impl != m->gemm_impl) m->drop_execs();
   m->gemm_impl = impl;
   return MARS_OK;
 }
@@ -912,11 +1100,7 @@ extern "C" mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable) {
 // ---------------------------------------------------------------- workspaces
 static mars_status ensure_kb(mars_dgi* m, const mars_graph* g) {
   if (!m->keep_bwd || m->kb_rows >= g->dev.Nt) return MARS_OK;
-  if (m->exec) {                 // a captured step without the copies
-    cudaGraphExecDestroy(m->exec);
-    m->exec = nullptr;
-    m->exec_graph = 0;
-  }
+  m->drop_execs();                 // a captured step without the copies
   CK(cudaStreamSynchronize(m->stream));
   m->kb_release();
   const size_t bytes = sizeof(float) * 2 * (size_t)g->dev.Nt * m->H;
@@ -936,11 +1120,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
       w.F == m->F && w.H == m->H)
     return MARS_OK;
   if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
-  if (m->exec) {
-    cudaGraphExecDestroy(m->exec);
-    m->exec = nullptr;
-    m->exec_graph = 0;
-  }
+  m->drop_execs();
   CK(cudaStreamSynchronize(m->stream));
   w.release();
   int64_t Nt = g->dev.Nt, R = 2 * Nt, Np = pv.Nt;
@@ -1367,15 +1547,11 @@ static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_inde
   int nl = 0;
   // Capture once a graph set is stepped twice in a row (pre-training reuses one
   // set for many steps); a set seen once (streamed batches) runs eagerly.
-  bool replay = m->capture && ((m->exec && m->exec_graph == g->uid && m->exec_stream == s) ||
-                               m->prev_graph == g->uid);
-  m->prev_graph = g->uid;
+  mars_dgi::ExecEntry* ent = m->capture ? m->find_exec(g->uid, s) : nullptr;
+  const bool replay = m->capture && (ent || m->seen_recently(g->uid));
+  m->note_seen(g->uid);
   if (replay) {
-    if (!m->exec || m->exec_graph != g->uid || m->exec_stream != s) {
-      if (m->exec) {
-        cudaGraphExecDestroy(m->exec);
-        m->exec = nullptr;
-      }
+    if (!ent) {
       cudaGraph_t graph;
       CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
       cudaError_t e = enqueue_step(m, g, s, &nl);
@@ -1386,15 +1562,15 @@ static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_inde
         return fail(MARS_ECUDA, "step capture failed: %s",
                     cudaGetErrorString(e != cudaSuccess ? e : e2));
       }
-      cudaError_t e3 = cudaGraphInstantiate(&m->exec, graph, 0);
+      cudaGraphExec_t ex = nullptr;
+      cudaError_t e3 = cudaGraphInstantiate(&ex, graph, 0);
       cudaGraphDestroy(graph);
       CK(e3);
-      m->exec_graph = g->uid;
-      m->exec_stream = s;
-      m->exec_launches = nl;
+      ent = m->add_exec(g->uid, s, ex, nl);
     }
-    CK(cudaGraphLaunch(m->exec, s));
-    nl = (int)m->exec_launches;
+    ent->last = ++m->exec_clock;
+    CK(cudaGraphLaunch(ent->exec, s));
+    nl = (int)ent->launches;
   } else {
     cudaError_t e = enqueue_step(m, g, s, &nl);
     if (e != cudaSuccess) {
@@ -1498,11 +1674,7 @@ extern "C" mars_status mars_dgi_saved_rows(const mars_dgi* m, int64_t* rows) {
 extern "C" mars_status mars_dgi_set_keep_backward(mars_dgi* m, int32_t keep) {
   if (mars_status st = check_dgi(m)) return st;
   CK(cudaSetDevice(m->cfg.device));
-  if (m->exec) {                 // recapture with / without the copies
-    cudaGraphExecDestroy(m->exec);
-    m->exec = nullptr;
-    m->exec_graph = 0;
-  }
+  m->drop_execs();                 // recapture with / without the copies
   CK(cudaStreamSynchronize(m->stream));
   m->keep_bwd = keep != 0;
   if (!m->keep_bwd) m->kb_release();
@@ -1689,11 +1861,7 @@ void shard_wire(mars_dgi* m, void* const (*bufs)[kShardBufs]) {
     sh.grads.p[q] = bufs[q][6];
   }
   sh.connected = true;
-  if (m->exec) {          // a captured step of this graph predates the wiring
-    cudaGraphExecDestroy(m->exec);
-    m->exec = nullptr;
-    m->exec_graph = 0;
-  }
+  m->drop_execs();          // a captured step of this graph predates the wiring
 }
 
 // Captures the sharded step once at connect time and forces every kernel it
@@ -1730,12 +1898,10 @@ mars_status shard_prepare(mars_dgi* m) {
     cudaFuncAttributes fa;
     CK(cudaFuncGetAttributes(&fa, kp.func));
   }
-  if (m->exec) cudaGraphExecDestroy(m->exec);
-  m->exec = nullptr;
-  CK(cudaGraphInstantiate(&m->exec, graph, 0));
-  m->exec_graph = g->uid;
-  m->exec_stream = s;
-  m->exec_launches = nl;
+  m->drop_execs();
+  cudaGraphExec_t ex = nullptr;
+  CK(cudaGraphInstantiate(&ex, graph, 0));
+  m->add_exec(g->uid, s, ex, nl);
   return MARS_OK;
 }
 }  // namespace
@@ -2020,11 +2186,7 @@ extern "C" mars_status mars_dp_connect(mars_dgi* m, const void* blobs) {
     d.sync.flags[q] = static_cast<unsigned long long*>(pf);
   }
   d.connected = true;
-  if (m->exec) {
-    cudaGraphExecDestroy(m->exec);
-    m->exec = nullptr;
-    m->exec_graph = 0;
-  }
+  m->drop_execs();
   // One process per rank: each barrier signals its peers before it waits, so a
   // host thread blocked in a lazy module load (which waits for its own context
   // to go idle) cannot deadlock the ranks.
@@ -2061,6 +2223,187 @@ extern "C" mars_status mars_dgi_read_step(mars_dgi* m, float* loss, float* grads
   return check_skipped(m, skipped);
 }
 
+// ---------------------------------------------------------------- placer (NEXT-2)
+struct mars_placer {
+  uint64_t tag = kTagPlacer;
+  mars_placer_config cfg{};
+  PlacerDims d{};
+  int64_t P = 0;
+  float* params = nullptr;
+  PlacerParams w{};
+  PlacerWork ws{};
+  int64_t ws_N = 0, ws_S = 0, ws_seg = 0;
+  std::vector<void*> owned;
+  cudaStream_t stream = nullptr;
+  void release_ws() {
+    for (void* p : owned) cudaFree(p);
+    owned.clear();
+    ws = PlacerWork{};
+    ws_N = ws_S = ws_seg = 0;
+  }
+  ~mars_placer() {
+    if (stream) cudaStreamSynchronize(stream);
+    release_ws();
+    if (params) cudaFree(params);
+    if (stream) cudaStreamDestroy(stream);
+  }
+};
+
+static PlacerDims placer_dims(const mars_placer_config* c) {
+  return PlacerDims{c->in_dim, c->enc_hidden, c->attn_dim, c->dev_embed, c->num_devices};
+}
+
+extern "C" void mars_placer_config_default(mars_placer_config* c) {
+  if (!c) return;
+  memset(c, 0, sizeof *c);
+  c->in_dim = 256;
+  c->enc_hidden = 256;
+  c->attn_dim = 512;
+  c->dev_embed = 64;
+  c->num_devices = 4;
+  c->segment = 128;
+}
+
+extern "C" int64_t mars_placer_num_params(const mars_placer_config* c) {
+  return c ? placer_num_params(placer_dims(c)) : -1;
+}
+
+static mars_status check_placer_cfg(const mars_placer_config* c) {
+  if (!c) return fail(MARS_EINVAL, "NULL config");
+  if (c->in_dim < 16 || c->in_dim % 16) return fail(MARS_EINVAL, "in_dim must be a multiple of 16");
+  if (c->enc_hidden != 64 && c->enc_hidden != 128 && c->enc_hidden != 256)
+    return fail(MARS_EINVAL, "enc_hidden must be 64, 128 or 256");
+  if (c->attn_dim < 128 || c->attn_dim % 128) return fail(MARS_EINVAL, "attn_dim must be a multiple of 128");
+  if (c->dev_embed < 1 || c->dev_embed > 256) return fail(MARS_EINVAL, "dev_embed in [1, 256]");
+  if (c->num_devices < 2 || c->num_devices > 64) return fail(MARS_EINVAL, "num_devices in [2, 64]");
+  if (c->segment < 1 || c->segment > 1024) return fail(MARS_EINVAL, "segment in [1, 1024]");
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_placer_create(const mars_placer_config* cfg, mars_placer** out) {
+  if (!out) return fail(MARS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (mars_status st = check_placer_cfg(cfg)) return st;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(MARS_ECUDA, "no CUDA device (libmars has no CPU fallback)");
+  }
+  if (cfg->device < 0 || cfg->device >= ndev) return fail(MARS_EINVAL, "bad device");
+  CK(cudaSetDevice(cfg->device));
+  auto* p = new mars_placer();
+  std::unique_ptr<mars_placer> guard(p);
+  p->cfg = *cfg;
+  p->cfg.init_params = nullptr;
+  p->d = placer_dims(cfg);
+  p->P = placer_num_params(p->d);
+  CK(cudaStreamCreateWithFlags(&p->stream, cudaStreamNonBlocking));
+  CK(dalloc(&p->params, (size_t)p->P));
+  p->w = placer_views(p->d, p->params);
+  if (cfg->init_params)
+    CK(cudaMemcpyAsync(p->params, cfg->init_params, sizeof(float) * p->P, cudaMemcpyHostToDevice,
+                       p->stream));
+  else
+    CK(placer_init(p->d, p->params, cfg->seed, p->stream));
+  CK(placer_prepare(p->d));
+  CK(cudaStreamSynchronize(p->stream));
+  *out = guard.release();
+  return MARS_OK;
+}
+
+static mars_status check_placer(const mars_placer* p) {
+  if (!p || p->tag != kTagPlacer) return fail(MARS_ESTATE, "invalid or freed mars_placer handle");
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_placer_get_params(const mars_placer* p, float* params) {
+  if (mars_status st = check_placer(p)) return st;
+  if (!params) return fail(MARS_EINVAL, "params is NULL");
+  CK(cudaSetDevice(p->cfg.device));
+  CK(cudaStreamSynchronize(p->stream));
+  CK(cudaMemcpy(params, p->params, sizeof(float) * p->P, cudaMemcpyDeviceToHost));
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_placer_set_params(mars_placer* p, const float* params) {
+  if (mars_status st = check_placer(p)) return st;
+  if (!params) return fail(MARS_EINVAL, "params is NULL");
+  CK(cudaSetDevice(p->cfg.device));
+  CK(cudaStreamSynchronize(p->stream));
+  CK(cudaMemcpy(p->params, params, sizeof(float) * p->P, cudaMemcpyHostToDevice));
+  return MARS_OK;
+}
+
+static mars_status placer_ensure(mars_placer* p, int64_t N, int64_t S) {
+  const int64_t seg = p->cfg.segment;
+  if (p->ws_N >= N && p->ws_S >= S && p->ws_seg == seg) return MARS_OK;
+  CK(cudaStreamSynchronize(p->stream));
+  p->release_ws();
+  const PlacerDims& d = p->d;
+  const int64_t Hd = d.Hd, Hs = 2 * Hd, nseg = (N + seg - 1) / seg;
+  auto al = [&](float** q, size_t n) -> cudaError_t {
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(q), sizeof(float) * (n ? n : 1));
+    if (e == cudaSuccess) p->owned.push_back(*q);
+    return e;
+  };
+  PlacerWork& w = p->ws;
+  CK(al(&w.xp[0], N * 4 * Hd));
+  CK(al(&w.xp[1], N * 4 * Hd));
+  CK(al(&w.enc, N * Hs));
+  CK(al(&w.keys, N * d.A));
+  CK(al(&w.seg_h, nseg * Hs));
+  CK(al(&w.seg_c, nseg * Hs));
+  CK(al(&w.hbuf, 4 * Hd));
+  CK(al(&w.sh, 2 * S * Hs));
+  CK(al(&w.sc, S * Hs));
+  CK(al(&w.q, S * d.A));
+  CK(al(&w.ghh, S * 4 * Hs));
+  CK(al(&w.score, S * seg));
+  CK(al(&w.ctx, S * Hs));
+  CK(al(reinterpret_cast<float**>(&w.bar), 2));
+  p->ws_N = N;
+  p->ws_S = S;
+  p->ws_seg = seg;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_placer_sample(mars_placer* p, const float* emb, int32_t N,
+                                          int32_t num_samples, uint64_t sample_seed,
+                                          const int32_t* forced, int32_t* placements, float* logp,
+                                          float* entropy) {
+  if (mars_status st = check_placer(p)) return st;
+  if (!emb || N < 1) return fail(MARS_EINVAL, "need N >= 1 embeddings");
+  if (num_samples < 1 || num_samples > 32) return fail(MARS_EINVAL, "num_samples in [1, 32]");
+  if (forced)
+    for (int64_t e = 0; e < (int64_t)num_samples * N; ++e)
+      if (forced[e] < 0 || forced[e] >= p->d.D) return fail(MARS_EINVAL, "forced placement out of range");
+  CK(cudaSetDevice(p->cfg.device));
+  if (mars_status st = placer_ensure(p, N, num_samples)) return st;
+  cudaStream_t s = p->stream;
+  const int64_t SN = (int64_t)num_samples * N;
+  float* dE = nullptr;
+  int32_t *dF = nullptr, *dP = nullptr;
+  float *dL = nullptr, *dH = nullptr;
+  struct FreeAll { std::vector<void*> v; cudaStream_t s; ~FreeAll() { for (void* q : v) cudaFreeAsync(q, s); } } fa{{}, s};
+  CK(palloc(&dE, (size_t)N * p->d.H, s)); fa.v.push_back(dE);
+  CK(palloc(&dP, (size_t)SN, s)); fa.v.push_back(dP);
+  CK(palloc(&dL, (size_t)SN, s)); fa.v.push_back(dL);
+  CK(palloc(&dH, (size_t)SN, s)); fa.v.push_back(dH);
+  if (forced) {
+    CK(palloc(&dF, (size_t)SN, s)); fa.v.push_back(dF);
+    CK(cudaMemcpyAsync(dF, forced, sizeof(int32_t) * SN, cudaMemcpyHostToDevice, s));
+  }
+  CK(cudaMemcpyAsync(dE, emb, sizeof(float) * (size_t)N * p->d.H, cudaMemcpyHostToDevice, s));
+  int nl = 0;
+  CK(placer_forward(p->d, p->w, p->ws, dE, N, p->cfg.segment, num_samples, sample_seed, dF, dP, dL,
+                    dH, s, &nl));
+  if (placements) CK(cudaMemcpyAsync(placements, dP, sizeof(int32_t) * SN, cudaMemcpyDeviceToHost, s));
+  if (logp) CK(cudaMemcpyAsync(logp, dL, sizeof(float) * SN, cudaMemcpyDeviceToHost, s));
+  if (entropy) CK(cudaMemcpyAsync(entropy, dH, sizeof(float) * SN, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  return MARS_OK;
+}
+
 extern "C" void mars_free(void* h) {
   if (!h) return;
   uint64_t tag = *static_cast<uint64_t*>(h);
@@ -2075,5 +2418,10 @@ extern "C" void mars_free(void* h) {
     cudaStreamSynchronize(m->stream);
     m->tag = kTagDead;
     delete m;
+  } else if (tag == kTagPlacer) {
+    auto* p = static_cast<mars_placer*>(h);
+    cudaSetDevice(p->cfg.device);
+    p->tag = kTagDead;
+    delete p;
   }
 }

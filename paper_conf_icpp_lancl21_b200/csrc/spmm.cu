@@ -155,28 +155,28 @@ __device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, 
           vfma<V>(accn[q], w[u], x);
         }
       }
-    return;
-  }
-  float xp[K][S::NT][V], xn[K][S::NT][V];
+  } else {
+    float xp[K][S::NT][V], xn[K][S::NT][V];
 #pragma unroll
-  for (int u = 0; u < K; ++u)
+    for (int u = 0; u < K; ++u)
 #pragma unroll
-    for (int q = 0; q < S::NT; ++q) {
-      const int c = (sl + q * S::L) * V;
-      Vec<T>::load(src.pos(j[u]) + c, xp[u][q]);
-      if (BOTH) Vec<T>::load(src.neg(j[u], jn[u]) + c, xn[u][q]);
-    }
-#pragma unroll
-  for (int u = 0; u < K; ++u)
-#pragma unroll
-    for (int q = 0; q < S::NT; ++q) {
-      if (ACT) vprelu<V>(xp[u][q], a);
-      vfma<V>(accp[q], w[u], xp[u][q]);
-      if (BOTH) {
-        if (ACT) vprelu<V>(xn[u][q], a);
-        vfma<V>(accn[q], w[u], xn[u][q]);
+      for (int q = 0; q < S::NT; ++q) {
+        const int c = (sl + q * S::L) * V;
+        Vec<T>::load(src.pos(j[u]) + c, xp[u][q]);
+        if (BOTH) Vec<T>::load(src.neg(j[u], jn[u]) + c, xn[u][q]);
       }
-    }
+#pragma unroll
+    for (int u = 0; u < K; ++u)
+#pragma unroll
+      for (int q = 0; q < S::NT; ++q) {
+        if (ACT) vprelu<V>(xp[u][q], a);
+        vfma<V>(accp[q], w[u], xp[u][q]);
+        if (BOTH) {
+          if (ACT) vprelu<V>(xn[u][q], a);
+          vfma<V>(accn[q], w[u], xn[u][q]);
+        }
+      }
+  }
 }
 
 // Accumulates row (rb, re) of Â_n · act(T) for both branches: per chunk of L
@@ -601,17 +601,6 @@ k_spmm_bwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
     bwd_row<C, SH, LONG>(i, long_min, rowptr, colind, vals, dY, Z, a, Nt, dZ, rs, pr, gmask, sl, da);
   const double wd = warp_sum((double)da);   // the block is one warp
   if (lane == 0) slots[bid] = wd;
-}
-
-int spmm_sms() {
-  static int n = 0;
-  if (!n) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-    if (!n) n = 148;
-  }
-  return n;
 }
 
 // One one-warp block per RPB rows.

@@ -49,6 +49,14 @@ class DgiConfig(ctypes.Structure):
                 ("rank", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
 
 
+class PlacerConfig(ctypes.Structure):
+    _fields_ = [("in_dim", ctypes.c_int32), ("enc_hidden", ctypes.c_int32),
+                ("attn_dim", ctypes.c_int32), ("dev_embed", ctypes.c_int32),
+                ("num_devices", ctypes.c_int32), ("segment", ctypes.c_int32),
+                ("seed", ctypes.c_uint64), ("init_params", ctypes.c_void_p),
+                ("device", ctypes.c_int32)]
+
+
 class StepOut(ctypes.Structure):
     _fields_ = [("loss", ctypes.c_void_p), ("grads", ctypes.c_void_p), ("perms", ctypes.c_void_p)]
 
@@ -110,8 +118,18 @@ SIGNATURES = {
     "mars_dp_export": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dp_connect": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_graph_set_pair_offsets": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_graph_reload": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(GraphDesc), ctypes.c_int32]),
     "mars_featurize": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
                                       ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]),
+    "mars_placer_config_default": (None, [ctypes.POINTER(PlacerConfig)]),
+    "mars_placer_num_params": (ctypes.c_int64, [ctypes.POINTER(PlacerConfig)]),
+    "mars_placer_create": (ctypes.c_int, [ctypes.POINTER(PlacerConfig),
+                                          ctypes.POINTER(ctypes.c_void_p)]),
+    "mars_placer_get_params": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_placer_set_params": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_placer_sample": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
+                                          ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p,
+                                          ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -185,6 +203,17 @@ class Graph:
 
     def export_csr(self, idx):
         return graph_export_csr(self, idx)
+
+    def reload(self, graphs):
+        """mars_graph_reload: new contents (same node counts / F) in place."""
+        graphs = list(graphs)
+        descs = (GraphDesc * len(graphs))()
+        keep = []
+        for i, g in enumerate(graphs):
+            d, k = _desc(g)
+            descs[i] = d
+            keep.append(k)
+        _check(lib().mars_graph_reload(self.handle, descs, len(graphs)))
 
     def set_pair_offsets(self, offsets):
         """mars_graph_set_pair_offsets: graph i uses pair index pair_base + offsets[i] (c15)."""
@@ -514,6 +543,67 @@ def dgi_export_activations(m: DGI, layer: int):
 
 
 GEMM_IMPLS = {"auto": 0, "simt": 1}   # MARS_GEMM_* (include/mars.h)
+
+
+# ------------------------------------------------------------------ placer (NEXT-2)
+class Placer:
+    """The segment-level seq2seq placer (mars_placer*)."""
+
+    def __init__(self, handle, cfg: PlacerConfig):
+        self.handle = handle
+        self.cfg = cfg
+        self.P = int(lib().mars_placer_num_params(ctypes.byref(cfg)))
+
+    def get_params(self) -> np.ndarray:
+        p = np.zeros(self.P, np.float32)
+        _check(lib().mars_placer_get_params(self.handle, _ptr(p)))
+        return p
+
+    def set_params(self, params):
+        p = np.ascontiguousarray(params, np.float32)
+        _check(lib().mars_placer_set_params(self.handle, _ptr(p)))
+
+    def sample(self, embeddings, num_samples: int, sample_seed: int = 0, forced=None):
+        """mars_placer_sample: (placements [S x N] int32, logp [S x N], entropy [S x N])."""
+        E = np.ascontiguousarray(embeddings, np.float32)
+        N = E.shape[0]
+        S = int(num_samples)
+        f = None if forced is None else np.ascontiguousarray(forced, np.int32).reshape(S, N)
+        place = np.zeros((S, N), np.int32)
+        logp = np.zeros((S, N), np.float32)
+        ent = np.zeros((S, N), np.float32)
+        _check(lib().mars_placer_sample(self.handle, _ptr(E), N, S, sample_seed & (2 ** 64 - 1),
+                                        None if f is None else _ptr(f), _ptr(place), _ptr(logp),
+                                        _ptr(ent)))
+        return place, logp, ent
+
+    def free(self):
+        if self.handle:
+            lib().mars_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def placer_create(in_dim=256, enc_hidden=256, attn_dim=512, dev_embed=64, num_devices=4,
+                  segment=128, seed=0, init_params=None, device=0) -> Placer:
+    c = PlacerConfig()
+    lib().mars_placer_config_default(ctypes.byref(c))
+    c.in_dim, c.enc_hidden, c.attn_dim, c.dev_embed = in_dim, enc_hidden, attn_dim, dev_embed
+    c.num_devices, c.segment, c.seed, c.device = num_devices, segment, seed & (2 ** 64 - 1), device
+    keep = None
+    if init_params is not None:
+        keep = np.ascontiguousarray(init_params, np.float32)
+        c.init_params = keep.ctypes.data
+    h = ctypes.c_void_p()
+    _check(lib().mars_placer_create(ctypes.byref(c), ctypes.byref(h)))
+    c.init_params = None
+    del keep
+    return Placer(h, c)
 
 
 def debug_gemm(op: str, A, B, impl: str = "auto", iters: int = 0, device: int = 0):

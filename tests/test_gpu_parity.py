@@ -341,3 +341,36 @@ def test_pretrain_matches_oracle_loop():
     assert abs(res["best_loss"] - losses[k]) <= 1e-5 * losses[k]
     assert scaled_err(res["best_params"], snaps[k]) <= 1e-5
     assert scaled_err(m.get_state()[0], p) <= 1e-5
+
+
+def test_graph_reload_in_place():
+    """mars_graph_reload: new edges / features into the same handle (same node
+    counts) give exactly the results of a fresh load of them, also when the
+    captured step is replayed and when a step on the old contents is still in
+    flight (the reload waits for it on the device)."""
+    A = [SG.tiny(0), SG.tiny(1)]
+    Bs = [SG.tiny(2), SG.tiny(3)]                 # same N = 64 each, other edges / features
+    ref = {}
+    for name, gs in (("A", A), ("B", Bs)):
+        g = mars.graph_load(gs)
+        m = mars.dgi_create(in_dim=16, hidden_dim=32, seed=5)
+        ref[name] = [m.step(g, t, 0, want_loss=True, want_grads=True) for t in range(3)]
+    g = mars.graph_load(A)
+    m = mars.dgi_create(in_dim=16, hidden_dim=32, seed=5)
+    got = [m.step(g, 0, 0, want_loss=True, want_grads=True)]
+    g.reload(A)                                   # same contents: same identity, replay
+    got.append(m.step(g, 1, 0, want_loss=True, want_grads=True))
+    m.step(g, 2, 0)                               # in flight on the old contents ...
+    g.reload(Bs)                                  # ... while B is loaded in place
+    loss2, grads2 = m.read_step()
+    assert loss2 == ref["A"][2]["loss"] and np.array_equal(grads2, ref["A"][2]["grads"])
+    for t in range(2):
+        assert got[t]["loss"] == ref["A"][t]["loss"]
+        assert np.array_equal(got[t]["grads"], ref["A"][t]["grads"])
+    # a fresh model on the reloaded handle steps B exactly
+    m2 = mars.dgi_create(in_dim=16, hidden_dim=32, seed=5)
+    for t in range(3):
+        o = m2.step(g, t, 0, want_loss=True, want_grads=True)
+        assert o["loss"] == ref["B"][t]["loss"] and np.array_equal(o["grads"], ref["B"][t]["grads"])
+    with pytest.raises(mars.MarsError):
+        g.reload([SG.tiny(0)])                    # wrong graph count
