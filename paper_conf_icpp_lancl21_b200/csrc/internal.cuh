@@ -302,6 +302,49 @@ struct PlacerWork {     // device scratch sized for N ops and S samples
   float *q, *ghh, *score, *ctx;   // [S x A], [S x 8Hd], [S x seg], [S x 2Hd]
   unsigned int* bar;    // [2] grid-barrier counters
 };
+// Training forward: the decoder / encoder activations the backward needs and
+// the PPO output gradient (placer.cu, with placer_forward's `train`).
+struct PlacerTrain {
+  float *sv_hprev, *sv_cprev, *sv_gates, *sv_c, *sv_h, *sv_q, *sv_alpha, *sv_ctx;
+  int32_t* sv_prev;
+  float *esv_gates, *esv_c;            // encoder [2][N][4Hd], [2][N][Hd]
+  const float* logp_old;               // [S x N]
+  const float* adv;                    // [S]
+  float *dz, *lterm;                   // [S x N x D], [S x N]
+  float clip_eps, ent_coef;
+};
+// Backward pass state (placer_bwd.cu).
+struct PlacerBwd {
+  int32_t N, S, seg, Hd, Hs, Hin, A, D;
+  const float *wo, *v, *keys, *enc;    // weights / forward tensors
+  const float *wihT, *whhT, *wqT;      // decoder transposes [Hin x 4Hs], [Hs x 4Hs], [Hs x A]
+  const float* ewhhT[2];               // encoder W_hhᵀ [Hd x 4Hd]
+  const float *sv_gates, *sv_c, *sv_cprev, *sv_q, *sv_alpha;
+  const float* dz;
+  float *dg, *dx, *dq, *dvp;           // per (b, i): [SN x 4Hs], [SN x Hin], [SN x A], [SN x A]
+  float *dhr, *dcr, *dhr_part;         // [S x Hs]
+  float *dal, *de;                     // [S x seg]
+  float *dK, *denc;                    // [N x A], [N x Hs] (accumulated; zeroed first)
+  float *dinit_h, *dinit_c;            // [nseg x Hs]
+  const float *esv_gates, *esv_c;
+  float *edg;                          // [2][N][4Hd]
+  float *ehr, *ecr;                    // [2 x Hd]
+};
+cudaError_t placer_transpose(const float* in, int rows, int cols, float* out, cudaStream_t s);
+cudaError_t placer_bwd_decoder(const PlacerBwd& w, cudaStream_t s, int* launches);
+cudaError_t placer_bwd_encoder(const PlacerBwd& w, cudaStream_t s, int* launches);
+cudaError_t placer_colsum(const float* in, int64_t rows, int cols, float* out, cudaStream_t s);
+cudaError_t placer_emb_grad(const float* dx, const int32_t* prev, int64_t SN, int Hs, int Hin,
+                            int De, int D1, float* out, cudaStream_t s);
+cudaError_t placer_gather_rows(const float* in, const int32_t* order, int64_t rows, int cols,
+                               float* out, int scatter_add, cudaStream_t s);
+cudaError_t placer_add(float* a, const float* b, int64_t n, cudaStream_t s);
+cudaError_t placer_build_x(const float* ctx, const int32_t* prev, const float* emb, int64_t SN,
+                           int Hs, int De, float* X, cudaStream_t s);
+cudaError_t placer_gather_cols(const float* in, int64_t ld, int col0, const int32_t* order,
+                               int64_t rows, int cols, float* out, cudaStream_t s);
+cudaError_t placer_small_tn(const float* dz, const float* h, int64_t R, int D, int Hs, float* out,
+                            cudaStream_t s);
 int64_t placer_num_params(const PlacerDims& d);
 PlacerParams placer_views(const PlacerDims& d, float* base);
 cudaError_t placer_init(const PlacerDims& d, float* params, uint64_t seed, cudaStream_t s);
@@ -310,7 +353,7 @@ cudaError_t placer_prepare(const PlacerDims& d);
 cudaError_t placer_forward(const PlacerDims& d, const PlacerParams& w, const PlacerWork& ws,
                            const float* E, int32_t N, int32_t seg, int32_t S, uint64_t sample_seed,
                            const int32_t* forced, int32_t* place, float* logp, float* ent,
-                           cudaStream_t s, int* launches);
+                           cudaStream_t s, int* launches, const PlacerTrain* train = nullptr);
 
 // ---------------------------------------------------------------- adam.cu
 // grads: [P + 1], the loss at grads[P]; guard_part: adam_guard_doubles() doubles.

@@ -65,6 +65,8 @@ struct EncArgs {
   float* enc;                  // [N x 2Hd]
   float* seg_h;                // [nseg x 2Hd]
   float* seg_c;                // [nseg x 2Hd]
+  float* sv_gates;             // training: [2][N (step)][4Hd] post-activation i, f, g, o
+  float* sv_c;                 // training: [2][N (step)][Hd] cell state after the step
   unsigned int* bar;
   int32_t N, s, Hd;
 };
@@ -114,6 +116,14 @@ __global__ void __launch_bounds__(kThreads) k_enc(EncArgs a) {
       const float gg = tanhf(g[2 * kEncUnits + k]), og = sigm(g[3 * kEncUnits + k]);
       c_state = fg * c_state + ig * gg;
       const float hn = og * tanhf(c_state);
+      if (a.sv_gates) {
+        float* sg = a.sv_gates + ((int64_t)dir * a.N + t) * 4 * Hd;
+        sg[u0 + k] = ig;
+        sg[Hd + u0 + k] = fg;
+        sg[2 * Hd + u0 + k] = gg;
+        sg[3 * Hd + u0 + k] = og;
+        a.sv_c[((int64_t)dir * a.N + t) * Hd + u0 + k] = c_state;
+      }
       a.hbuf[(((t + 1) & 1) * 2 + dir) * Hd + u0 + k] = hn;
       a.enc[(int64_t)op * 2 * Hd + dir * Hd + u0 + k] = hn;
       if (t == j1 - 1) {                              // segment end: decoder init (c24)
@@ -150,6 +160,23 @@ struct DecArgs {
   int32_t* place;              // [S x N]
   float* logp;                 // [S x N]
   float* ent;                  // [S x N]
+  // training (NEXT-3): activations for the backward, per (sample b, op i)
+  float* sv_hprev;             // [S x N x Hs] decoder state entering op i
+  float* sv_cprev;             // [S x N x Hs]
+  float* sv_gates;             // [S x N x 4Hs] post-activation i, f, g, o
+  float* sv_c;                 // [S x N x Hs]
+  float* sv_h;                 // [S x N x Hs]
+  float* sv_q;                 // [S x N x A]
+  float* sv_alpha;             // [S x N x s]
+  float* sv_ctx;               // [S x N x Hs]
+  int32_t* sv_prev;            // [S x N] input device index of op i (D = start)
+  // PPO (c29): with logp_old / adv, dz [S x N x D] = dL/dlogits and the loss
+  // terms lterm [S x N] (-min(rho A, clip(rho) A) - c_ent H, before / (S N))
+  const float* logp_old;       // [S x N]
+  const float* adv;            // [S]
+  float* dz;
+  float* lterm;
+  float clip_eps, ent_coef;
   unsigned int* bar;
   uint64_t seed_key;           // sm64(sample_seed)
   int32_t N, s, S, Hs, A, De, D, nrows_a;   // nrows_a = A + 4 Hs
@@ -195,9 +222,27 @@ __device__ void finish_op(const DecArgs& a, const float* hs, int i, int32_t* pre
     }
     prev[b] = p;
     if (blockIdx.x == 0) {
-      a.place[(int64_t)b * a.N + i] = p;
-      a.logp[(int64_t)b * a.N + i] = (float)((double)z[p] - lse);
-      a.ent[(int64_t)b * a.N + i] = (float)en;
+      const int64_t bi = (int64_t)b * a.N + i;
+      a.place[bi] = p;
+      a.logp[bi] = (float)((double)z[p] - lse);
+      a.ent[bi] = (float)en;
+      if (a.dz) {
+        // L = -(1/n) sum min(rho A, clip(rho, 1-eps, 1+eps) A) - (c/n) sum H, n = S N;
+        // dL/dz_d = g (1[d = p] - pi_d) + (c/n) pi_d (log pi_d + H), g = dL/dlog pi(p)
+        const double n = (double)a.S * a.N;
+        const double A = a.adv[b];
+        const double lpn = (double)z[p] - lse;
+        const double rho = exp(lpn - (double)a.logp_old[bi]);
+        const double rc = fmin(fmax(rho, 1.0 - a.clip_eps), 1.0 + a.clip_eps);
+        const double un = rho * A, cl = rc * A;
+        const double g = un <= cl ? -rho * A / n : 0.0;   // the min picks the unclipped term
+        a.lterm[bi] = (float)(-fmin(un, cl) - (double)a.ent_coef * en);
+        for (int d = 0; d < a.D; ++d) {
+          const double lp = (double)z[d] - lse, pd = exp(lp);
+          a.dz[bi * a.D + d] = (float)(g * ((d == p ? 1.0 : 0.0) - pd) +
+                                       (double)a.ent_coef / n * pd * (lp + en));
+        }
+      }
     }
   }
   __syncthreads();
@@ -239,6 +284,11 @@ __global__ void __launch_bounds__(kThreads) k_dec(DecArgs a) {
         if (threadIdx.x < S) prev[threadIdx.x] = a.D;      // start token
         __syncthreads();
       }
+      if (a.sv_hprev && blockIdx.x == 0) {
+        for (int e = threadIdx.x; e < S * Hs; e += kThreads)
+          a.sv_hprev[((int64_t)(e / Hs) * a.N + i) * Hs + e % Hs] = hs[e];
+        if (threadIdx.x < S) a.sv_prev[(int64_t)threadIdx.x * a.N + i] = prev[threadIdx.x];
+      }
       // rows r in [0, A): q;  [A, A + 4Hs): W_hh s
       for (int r = blockIdx.x * (kThreads / 32) + warp; r < a.nrows_a; r += G * (kThreads / 32)) {
         const float* w = r < A ? a.wq + (int64_t)r * Hs : a.whh + (int64_t)(r - A) * Hs;
@@ -247,8 +297,12 @@ __global__ void __launch_bounds__(kThreads) k_dec(DecArgs a) {
           for (int c = lane; c < Hs; c += 32) acc = fmaf(w[c], hs[b * Hs + c], acc);
           acc = warp_sum(acc);
           if (lane == 0) {
-            if (r < A) a.q[b * A + r] = acc;
-            else a.ghh[(int64_t)b * 4 * Hs + (r - A)] = acc;
+            if (r < A) {
+              a.q[b * A + r] = acc;
+              if (a.sv_q) a.sv_q[((int64_t)b * a.N + i) * A + r] = acc;
+            } else {
+              a.ghh[(int64_t)b * 4 * Hs + (r - A)] = acc;
+            }
           }
         }
       }
@@ -282,6 +336,9 @@ __global__ void __launch_bounds__(kThreads) k_dec(DecArgs a) {
       for (int k = lane; k < len; k += 32) al[b * a.s + k] *= inv;
     }
     __syncthreads();
+    if (a.sv_alpha && blockIdx.x == 0)
+      for (int e = threadIdx.x; e < S * len; e += kThreads)
+        a.sv_alpha[((int64_t)(e / len) * a.N + i) * a.s + e % len] = al[(e / len) * a.s + e % len];
     {
       const int ncols = Hs / G > 0 ? Hs / G : 1;          // ctx columns of this CTA
       for (int e = threadIdx.x; e < S * ncols; e += kThreads) {
@@ -290,6 +347,7 @@ __global__ void __launch_bounds__(kThreads) k_dec(DecArgs a) {
         float acc = 0.f;
         for (int k = 0; k < len; ++k) acc = fmaf(al[b * a.s + k], a.enc[(int64_t)(j0 + k) * Hs + col], acc);
         a.ctx[b * Hs + col] = acc;
+        if (a.sv_ctx) a.sv_ctx[((int64_t)b * a.N + i) * Hs + col] = acc;
       }
     }
     grid_bar(a.bar, epoch);
@@ -321,8 +379,20 @@ __global__ void __launch_bounds__(kThreads) k_dec(DecArgs a) {
         const float g2 = tanhf(gg[2 * units + k]), og = sigm(gg[3 * units + k]);
         const float cp = first ? a.seg_c[(int64_t)j * Hs + u] : a.sc[b * Hs + u];
         const float cn = fg * cp + ig * g2;
+        const float hn = og * tanhf(cn);
         a.sc[b * Hs + u] = cn;
-        a.sh[(i & 1) * S * Hs + b * Hs + u] = og * tanhf(cn);
+        a.sh[(i & 1) * S * Hs + b * Hs + u] = hn;
+        if (a.sv_gates) {
+          const int64_t bi = (int64_t)b * a.N + i;
+          float* sg = a.sv_gates + bi * 4 * Hs;
+          sg[u] = ig;
+          sg[Hs + u] = fg;
+          sg[2 * Hs + u] = g2;
+          sg[3 * Hs + u] = og;
+          a.sv_cprev[bi * Hs + u] = cp;
+          a.sv_c[bi * Hs + u] = cn;
+          a.sv_h[bi * Hs + u] = hn;
+        }
       }
     }
     grid_bar(a.bar, epoch);
@@ -403,7 +473,7 @@ int placer_dec_grid(const PlacerDims& d) { return 2 * d.Hd / 4; }   // 4 decoder
 cudaError_t placer_forward(const PlacerDims& d, const PlacerParams& w, const PlacerWork& ws,
                            const float* E, int32_t N, int32_t seg, int32_t S, uint64_t sample_seed,
                            const int32_t* forced, int32_t* place, float* logp, float* ent,
-                           cudaStream_t s, int* launches) {
+                           cudaStream_t s, int* launches, const PlacerTrain* train) {
   const int Hs = 2 * d.Hd;
   cudaError_t e;
   // 1. encoder input projections (FFMA GEMMs)
@@ -426,6 +496,10 @@ cudaError_t placer_forward(const PlacerDims& d, const PlacerParams& w, const Pla
     a.N = N;
     a.s = seg;
     a.Hd = d.Hd;
+    if (train) {
+      a.sv_gates = train->esv_gates;
+      a.sv_c = train->esv_c;
+    }
     void* args[] = {&a};
     const int grid = 2 * d.Hd / kEncUnits;
     const size_t smem = placer_enc_smem(d);
@@ -461,6 +535,23 @@ cudaError_t placer_forward(const PlacerDims& d, const PlacerParams& w, const Pla
     a.ent = ent;
     a.bar = ws.bar + 1;
     a.seed_key = sm64(sample_seed);
+    if (train) {
+      a.sv_hprev = train->sv_hprev;
+      a.sv_cprev = train->sv_cprev;
+      a.sv_gates = train->sv_gates;
+      a.sv_c = train->sv_c;
+      a.sv_h = train->sv_h;
+      a.sv_q = train->sv_q;
+      a.sv_alpha = train->sv_alpha;
+      a.sv_ctx = train->sv_ctx;
+      a.sv_prev = train->sv_prev;
+      a.logp_old = train->logp_old;
+      a.adv = train->adv;
+      a.dz = train->dz;
+      a.lterm = train->lterm;
+      a.clip_eps = train->clip_eps;
+      a.ent_coef = train->ent_coef;
+    }
     a.N = N;
     a.s = seg;
     a.S = S;
