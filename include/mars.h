@@ -343,6 +343,21 @@ MARS_API mars_status mars_placer_sample(mars_placer* p, const float* embeddings,
                                         const int32_t* forced, int32_t* placements, float* logp,
                                         float* entropy);
 
+/* NEXT-3 (§3.4; readings c29-c31): the PPO loss
+ * of S placements re-evaluated under the current policy (teacher forcing) --
+ *   L = -(1/(S N)) sum_{b,i} min(rho A_b, clip(rho, 1 - eps, 1 + eps) A_b)
+ *       - ent_coef (1/(S N)) sum_{b,i} H_bi,   rho = exp(log pi(p_bi) - logp_old_bi)
+ * -- and its gradient by backpropagation through time: grads [P] (the flat
+ * parameter layout, host, optional) and dL/d embeddings [N x in_dim] (host,
+ * optional; continues into the GCN encoder for the joint update).
+ * placements / logp_old [S x N], adv [S]: host.  in_dim must be 32, 64 or a
+ * multiple of 128.  Synchronous. */
+MARS_API mars_status mars_placer_ppo_grad(mars_placer* p, const float* embeddings, int32_t num_ops,
+                                          int32_t num_samples, const int32_t* placements,
+                                          const float* logp_old, const float* adv,
+                                          float clip_eps, float ent_coef, float* loss,
+                                          float* grads, float* d_embeddings);
+
 /* Copies the most recent step's loss and global-mean gradient (the values
  * Adam consumed) to host memory (either may be NULL).  Synchronous.  For a
  * row-sharded model, ECUDA if a cross-shard barrier timed out. */

@@ -2234,6 +2234,21 @@ struct mars_placer {
   PlacerWork ws{};
   int64_t ws_N = 0, ws_S = 0, ws_seg = 0;
   std::vector<void*> owned;
+  // training (NEXT-3): saved activations, backward state, gradient vector
+  PlacerTrain tr{};
+  PlacerBwd bw{};
+  float *grads = nullptr, *wT = nullptr, *X = nullptr, *tmpNH = nullptr, *ebuf = nullptr;
+  double* part = nullptr;
+  int32_t* order_b = nullptr;
+  int64_t tr_N = 0, tr_S = 0;
+  std::vector<void*> tr_owned;
+  void release_tr() {
+    for (void* q : tr_owned) cudaFree(q);
+    tr_owned.clear();
+    tr = PlacerTrain{};
+    bw = PlacerBwd{};
+    tr_N = tr_S = 0;
+  }
   cudaStream_t stream = nullptr;
   void release_ws() {
     for (void* p : owned) cudaFree(p);
@@ -2244,6 +2259,7 @@ struct mars_placer {
   ~mars_placer() {
     if (stream) cudaStreamSynchronize(stream);
     release_ws();
+    release_tr();
     if (params) cudaFree(params);
     if (stream) cudaStreamDestroy(stream);
   }
@@ -2364,6 +2380,214 @@ static mars_status placer_ensure(mars_placer* p, int64_t N, int64_t S) {
   p->ws_N = N;
   p->ws_S = S;
   p->ws_seg = seg;
+  return MARS_OK;
+}
+
+// Training workspace for N ops and S samples (saved activations, backward).
+static mars_status placer_ensure_train(mars_placer* p, int64_t N, int64_t S) {
+  if (p->tr_N >= N && p->tr_S >= S && p->tr_N == N && p->tr_S == S) return MARS_OK;
+  CK(cudaStreamSynchronize(p->stream));
+  p->release_tr();
+  const PlacerDims& d = p->d;
+  const int64_t Hd = d.Hd, Hs = 2 * Hd, Hin = Hs + d.De, A = d.A, seg = p->cfg.segment;
+  const int64_t SN = S * N, nseg = (N + seg - 1) / seg;
+  auto al = [&](void** q, size_t bytes) -> cudaError_t {
+    cudaError_t e = cudaMalloc(q, bytes ? bytes : 8);
+    if (e == cudaSuccess) p->tr_owned.push_back(*q);
+    return e;
+  };
+  auto alf = [&](float** q, int64_t n) { return al(reinterpret_cast<void**>(q), sizeof(float) * n); };
+  PlacerTrain& t = p->tr;
+  CK(alf(&t.sv_hprev, SN * Hs));
+  CK(alf(&t.sv_cprev, SN * Hs));
+  CK(alf(&t.sv_gates, SN * 4 * Hs));
+  CK(alf(&t.sv_c, SN * Hs));
+  CK(alf(&t.sv_h, SN * Hs));
+  CK(alf(&t.sv_q, SN * A));
+  CK(alf(&t.sv_alpha, SN * seg));
+  CK(alf(&t.sv_ctx, SN * Hs));
+  CK(al(reinterpret_cast<void**>(&t.sv_prev), sizeof(int32_t) * SN));
+  CK(alf(&t.esv_gates, 2 * N * 4 * Hd));
+  CK(alf(&t.esv_c, 2 * N * Hd));
+  CK(alf(&t.dz, SN * d.D));
+  CK(alf(&t.lterm, SN));
+  CK(alf(const_cast<float**>(&t.logp_old), SN));
+  CK(alf(const_cast<float**>(&t.adv), S));
+  PlacerBwd& b = p->bw;
+  CK(alf(&b.dg, SN * 4 * Hs));
+  CK(alf(&b.dx, SN * Hin));
+  CK(alf(&b.dq, SN * A));
+  CK(alf(&b.dvp, SN * A));
+  CK(alf(&b.dhr, S * Hs));
+  CK(alf(&b.dcr, S * Hs));
+  CK(alf(&b.dhr_part, S * Hs));
+  CK(alf(&b.dal, S * seg));
+  CK(alf(&b.de, S * seg));
+  CK(alf(&b.dK, N * A));
+  CK(alf(&b.denc, N * Hs));
+  CK(alf(&b.dinit_h, nseg * Hs));
+  CK(alf(&b.dinit_c, nseg * Hs));
+  CK(alf(&b.edg, 2 * N * 4 * Hd));
+  CK(alf(&b.ehr, 2 * Hd));
+  CK(alf(&b.ecr, 2 * Hd));
+  CK(alf(&p->grads, p->P + 1));
+  // transposes: W_ihᵀ [Hin x 4Hs], W_hhᵀ [Hs x 4Hs], W_qᵀ [Hs x A], enc W_hhᵀ x2 [Hd x 4Hd]
+  CK(alf(&p->wT, Hin * 4 * Hs + Hs * 4 * Hs + Hs * A + 2 * Hd * 4 * Hd));
+  CK(alf(&p->X, SN * std::max<int64_t>(Hin, Hs)));
+  CK(alf(&p->tmpNH, N * std::max<int64_t>(Hs, d.H)));
+  CK(alf(&p->ebuf, 2 * N * std::max<int64_t>(Hd, d.H)));
+  size_t pt = 0;
+  const int64_t shapes[][3] = {{SN, 4 * Hs, Hin}, {SN, 4 * Hs, Hs}, {SN, A, Hs}, {N, A, Hs},
+                               {N, 4 * Hd, d.H}, {N, 4 * Hd, Hd}};
+  for (auto& sh : shapes) pt = std::max(pt, gemm_tn_partial_floats(sh[0], (int)sh[1], (int)sh[2]));
+  CK(al(reinterpret_cast<void**>(&p->part), sizeof(double) * pt));
+  CK(al(reinterpret_cast<void**>(&p->order_b), sizeof(int32_t) * N));
+  {   // backward-direction op order of the encoder steps (c23)
+    std::vector<int32_t> ord((size_t)N);
+    for (int64_t t2 = 0; t2 < N; ++t2) {
+      const int64_t j0 = (t2 / seg) * seg, j1 = std::min(N, j0 + seg);
+      ord[t2] = (int32_t)(j1 - 1 - (t2 - j0));
+    }
+    CK(cudaMemcpy(p->order_b, ord.data(), sizeof(int32_t) * N, cudaMemcpyHostToDevice));
+  }
+  b.N = (int32_t)N;
+  b.S = (int32_t)S;
+  b.seg = (int32_t)seg;
+  b.Hd = (int32_t)Hd;
+  b.Hs = (int32_t)Hs;
+  b.Hin = (int32_t)Hin;
+  b.A = (int32_t)A;
+  b.D = d.D;
+  b.wo = p->w.wo;
+  b.v = p->w.v;
+  b.keys = p->ws.keys;
+  b.enc = p->ws.enc;
+  b.wihT = p->wT;
+  b.whhT = p->wT + Hin * 4 * Hs;
+  b.wqT = b.whhT + Hs * 4 * Hs;
+  b.ewhhT[0] = b.wqT + Hs * A;
+  b.ewhhT[1] = b.ewhhT[0] + Hd * 4 * Hd;
+  b.sv_gates = t.sv_gates;
+  b.sv_c = t.sv_c;
+  b.sv_cprev = t.sv_cprev;
+  b.sv_q = t.sv_q;
+  b.sv_alpha = t.sv_alpha;
+  b.dz = t.dz;
+  b.esv_gates = t.esv_gates;
+  b.esv_c = t.esv_c;
+  p->tr_N = N;
+  p->tr_S = S;
+  return MARS_OK;
+}
+
+// The PPO loss (c29) of S teacher-forced placements and its gradient: placer
+// forward with activations saved, dL/dlogits, BPTT through the decoder and the
+// encoder, weight gradients by GEMMs / fixed-order sums.  Leaves the gradient
+// [P] and the loss (at [P]) in p->grads and dL/dE [N x H] in p->tmpNH.
+static mars_status placer_loss_grad(mars_placer* p, const float* dE_in, int32_t N, int32_t S,
+                                    const int32_t* dplace, float clip_eps, float ent_coef, int* nl) {
+  cudaStream_t s = p->stream;
+  const PlacerDims& d = p->d;
+  const int64_t Hd = d.Hd, Hs = 2 * Hd, Hin = Hs + d.De, A = d.A, SN = (int64_t)S * N;
+  PlacerTrain& t = p->tr;
+  PlacerBwd& b = p->bw;
+  b.keys = p->ws.keys;                    // the forward workspace may have been regrown
+  b.enc = p->ws.enc;
+  b.wo = p->w.wo;
+  b.v = p->w.v;
+  t.clip_eps = clip_eps;
+  t.ent_coef = ent_coef;
+  // forward with teacher forcing; place / logp / ent outputs into scratch rows of X
+  int32_t* dP = reinterpret_cast<int32_t*>(p->X);
+  float* dL = p->X + SN;
+  float* dH = p->X + 2 * SN;
+  CK(placer_forward(d, p->w, p->ws, dE_in, N, p->cfg.segment, S, 0, dplace, dP, dL, dH, s, nl, &t));
+  // transposed weights
+  CK(placer_transpose(p->w.dec_wih, (int)(4 * Hs), (int)Hin, const_cast<float*>(b.wihT), s));
+  CK(placer_transpose(p->w.dec_whh, (int)(4 * Hs), (int)Hs, const_cast<float*>(b.whhT), s));
+  CK(placer_transpose(p->w.wq, (int)A, (int)Hs, const_cast<float*>(b.wqT), s));
+  for (int dir = 0; dir < 2; ++dir)
+    CK(placer_transpose(p->w.enc_whh[dir], (int)(4 * Hd), (int)Hd, const_cast<float*>(b.ewhhT[dir]), s));
+  CK(cudaMemsetAsync(b.dK, 0, sizeof(float) * N * A, s));
+  CK(cudaMemsetAsync(b.denc, 0, sizeof(float) * N * Hs, s));
+  CK(placer_bwd_decoder(b, s, nl));
+  // decoder weight gradients
+  PlacerParams G = placer_views(d, p->grads);
+  CK(placer_build_x(t.sv_ctx, t.sv_prev, p->w.emb, SN, (int)Hs, d.De, p->X, s));
+  CK(gemm_tn(b.dg, p->X, G.dec_wih, SN, (int)(4 * Hs), (int)Hin, p->part, s, nl));
+  CK(gemm_tn(b.dg, t.sv_hprev, G.dec_whh, SN, (int)(4 * Hs), (int)Hs, p->part, s, nl));
+  CK(placer_colsum(b.dg, SN, (int)(4 * Hs), G.dec_b, s));
+  CK(gemm_tn(b.dq, t.sv_hprev, G.wq, SN, (int)A, (int)Hs, p->part, s, nl));
+  CK(placer_colsum(b.dvp, SN, (int)A, G.v, s));
+  CK(placer_small_tn(t.dz, t.sv_h, SN, d.D, (int)Hs, G.wo, s));
+  CK(placer_colsum(t.dz, SN, d.D, G.bo, s));
+  CK(placer_emb_grad(b.dx, t.sv_prev, SN, (int)Hs, (int)Hin, d.De, d.D + 1, G.emb, s));
+  CK(gemm_tn(b.dK, p->ws.enc, G.wk, N, (int)A, (int)Hs, p->part, s, nl));
+  CK(gemm_nn(b.dK, p->w.wk, p->tmpNH, N, (int)Hs, (int)A, s, nl));     // d(K)/d(enc)
+  CK(placer_add(b.denc, p->tmpNH, N * Hs, s));
+  // encoder BPTT and its gradients
+  CK(placer_bwd_encoder(b, s, nl));
+  float* Eb = p->ebuf;                      // E in the backward direction's step order
+  CK(placer_gather_rows(dE_in, p->order_b, N, d.H, Eb, 0, s));
+  CK(gemm_tn(b.edg, dE_in, G.enc_wih[0], N, (int)(4 * Hd), d.H, p->part, s, nl));
+  CK(gemm_tn(b.edg + N * 4 * Hd, Eb, G.enc_wih[1], N, (int)(4 * Hd), d.H, p->part, s, nl));
+  for (int dir = 0; dir < 2; ++dir) {
+    float* hs = p->ebuf;                    // h of each step of this direction, step order
+    CK(placer_gather_cols(p->ws.enc, Hs, dir * (int)Hd, dir ? p->order_b : nullptr, N, (int)Hd, hs, s));
+    const float* edg = b.edg + (int64_t)dir * N * 4 * Hd;
+    if (N > 1)
+      CK(gemm_tn(edg + 4 * Hd, hs, G.enc_whh[dir], N - 1, (int)(4 * Hd), (int)Hd, p->part, s, nl));
+    else
+      CK(cudaMemsetAsync(G.enc_whh[dir], 0, sizeof(float) * 4 * Hd * Hd, s));
+    CK(placer_colsum(edg, N, (int)(4 * Hd), G.enc_b[dir], s));
+  }
+  // dL/dE: forward direction in op order, backward direction scattered by its order
+  CK(gemm_nn(b.edg, p->w.enc_wih[0], p->tmpNH, N, d.H, (int)(4 * Hd), s, nl));
+  CK(gemm_nn(b.edg + N * 4 * Hd, p->w.enc_wih[1], p->ebuf, N, d.H, (int)(4 * Hd), s, nl));
+  CK(placer_gather_rows(p->ebuf, p->order_b, N, d.H, p->tmpNH, 1, s));
+  // the loss: sum of the per-op terms / (S N), fixed order
+  CK(placer_colsum(t.lterm, SN, 1, p->grads + p->P, s));
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_placer_ppo_grad(mars_placer* p, const float* emb, int32_t N,
+                                            int32_t num_samples, const int32_t* placements,
+                                            const float* logp_old, const float* adv,
+                                            float clip_eps, float ent_coef, float* loss,
+                                            float* grads, float* demb) {
+  if (mars_status st = check_placer(p)) return st;
+  if (!emb || !placements || !logp_old || !adv || N < 1)
+    return fail(MARS_EINVAL, "NULL input or N < 1");
+  if (num_samples < 1 || num_samples > 32) return fail(MARS_EINVAL, "num_samples in [1, 32]");
+  const int64_t SN = (int64_t)num_samples * N;
+  for (int64_t e = 0; e < SN; ++e)
+    if (placements[e] < 0 || placements[e] >= p->d.D) return fail(MARS_EINVAL, "placement out of range");
+  const int H = p->d.H;
+  if (!(H == 32 || H == 64 || H % 128 == 0))
+    return fail(MARS_EINVAL, "training needs in_dim in {32, 64} or a multiple of 128");
+  CK(cudaSetDevice(p->cfg.device));
+  if (mars_status st = placer_ensure(p, N, num_samples)) return st;
+  if (mars_status st = placer_ensure_train(p, N, num_samples)) return st;
+  cudaStream_t s = p->stream;
+  float* dE = nullptr;
+  int32_t* dPl = nullptr;
+  struct FreeAll { std::vector<void*> v; cudaStream_t s; ~FreeAll() { for (void* q : v) cudaFreeAsync(q, s); } } fa{{}, s};
+  CK(palloc(&dE, (size_t)N * H, s)); fa.v.push_back(dE);
+  CK(palloc(&dPl, (size_t)SN, s)); fa.v.push_back(dPl);
+  CK(cudaMemcpyAsync(dE, emb, sizeof(float) * (size_t)N * H, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(dPl, placements, sizeof(int32_t) * SN, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(const_cast<float*>(p->tr.logp_old), logp_old, sizeof(float) * SN,
+                     cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(const_cast<float*>(p->tr.adv), adv, sizeof(float) * num_samples,
+                     cudaMemcpyHostToDevice, s));
+  int nl = 0;
+  if (mars_status st = placer_loss_grad(p, dE, N, num_samples, dPl, clip_eps, ent_coef, &nl)) return st;
+  float lsum = 0.f;
+  CK(cudaMemcpyAsync(&lsum, p->grads + p->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+  if (grads) CK(cudaMemcpyAsync(grads, p->grads, sizeof(float) * p->P, cudaMemcpyDeviceToHost, s));
+  if (demb) CK(cudaMemcpyAsync(demb, p->tmpNH, sizeof(float) * (size_t)N * H, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (loss) *loss = (float)((double)lsum / (double)SN);
   return MARS_OK;
 }
 

@@ -67,12 +67,12 @@ __global__ void kb_xt(PlacerBwd w, int i) {
   const int b = warp / (Hin + Hs), o = warp % (Hin + Hs);
   const float* dg = w.dg + ((int64_t)b * w.N + i) * R;
   const float* wt = o < Hin ? w.wihT + (int64_t)o * R : w.whhT + (int64_t)(o - Hin) * R;
-  float acc = 0.f;
-  for (int r = lane; r < R; r += 32) acc = fmaf(wt[r], dg[r], acc);
+  double acc = 0.0;                 // dctx feeds the attention backward's cancellation
+  for (int r = lane; r < R; r += 32) acc += (double)wt[r] * (double)dg[r];
   acc = warp_sum(acc);
   if (lane == 0) {
-    if (o < Hin) w.dx[((int64_t)b * w.N + i) * Hin + o] = acc;
-    else w.dhr_part[(int64_t)b * Hs + (o - Hin)] = acc;
+    if (o < Hin) w.dx[((int64_t)b * w.N + i) * Hin + o] = (float)acc;
+    else w.dhr_part[(int64_t)b * Hs + (o - Hin)] = (float)acc;
   }
 }
 
@@ -83,46 +83,47 @@ __global__ void kb_dalpha(PlacerBwd w, int i, int j0, int len) {
   const int b = warp / len, k = warp % len;
   const float* dctx = w.dx + ((int64_t)b * w.N + i) * w.Hin;
   const float* en = w.enc + (int64_t)(j0 + k) * w.Hs;
-  float acc = 0.f;
-  for (int c = lane; c < w.Hs; c += 32) acc = fmaf(dctx[c], en[c], acc);
+  double acc = 0.0;
+  for (int c = lane; c < w.Hs; c += 32) acc += (double)dctx[c] * (double)en[c];
   acc = warp_sum(acc);
-  if (lane == 0) w.dal[(int64_t)b * w.seg + k] = acc;
+  if (lane == 0) w.dal[(int64_t)b * w.seg + k] = (float)acc;
 }
 
 // grid (S, cdiv(A, kT)): de_k (every block, redundant), then per a:
 // dq[b][a] = sum_k de_k v_a (1 - u_ka²), dvp[b][i][a] = sum_k de_k u_ka,
 // u_ka = tanh(q_a + K_{j0+k, a}); block (b, 0) also stores de.
 __global__ void kb_datt(PlacerBwd w, int i, int j0, int len) {
-  __shared__ float de[1024];
-  __shared__ float red[kT / 32];
+  // the softmax backward cancels (dalpha_k - sum alpha dalpha): double for the
+  // sums and de, so the query gradient keeps fp32-level relative accuracy
+  __shared__ double de[1024];
+  __shared__ double red[kT / 32];
   const int b = blockIdx.x;
   const int64_t bi = (int64_t)b * w.N + i;
   const float* al = w.sv_alpha + bi * w.seg;
-  float part = 0.f;
-  for (int k = threadIdx.x; k < len; k += kT) part = fmaf(al[k], w.dal[(int64_t)b * w.seg + k], part);
-  // fixed-order block reduction
-  part = warp_sum(part);
+  double part = 0.0;
+  for (int k = threadIdx.x; k < len; k += kT) part += (double)al[k] * (double)w.dal[(int64_t)b * w.seg + k];
+  part = warp_sum(part);                        // fixed-order block reduction
   if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = part;
   __syncthreads();
-  float sum = 0.f;
+  double sum = 0.0;
   for (int q = 0; q < kT / 32; ++q) sum += red[q];
   for (int k = threadIdx.x; k < len; k += kT) {
-    const float d = al[k] * (w.dal[(int64_t)b * w.seg + k] - sum);
+    const double d = (double)al[k] * ((double)w.dal[(int64_t)b * w.seg + k] - sum);
     de[k] = d;
-    if (blockIdx.y == 0) w.de[(int64_t)b * w.seg + k] = d;
+    if (blockIdx.y == 0) w.de[(int64_t)b * w.seg + k] = (float)d;
   }
   __syncthreads();
   const int a = blockIdx.y * kT + threadIdx.x;
   if (a >= w.A) return;
   const float qa = w.sv_q[bi * w.A + a], va = w.v[a];
-  float dq = 0.f, dv = 0.f;
+  double dq = 0.0, dv = 0.0;
   for (int k = 0; k < len; ++k) {
     const float u = tanhf(qa + w.keys[(int64_t)(j0 + k) * w.A + a]);
-    dq = fmaf(de[k] * va, 1.f - u * u, dq);
-    dv = fmaf(de[k], u, dv);
+    dq += de[k] * (double)(va * (1.f - u * u));
+    dv += de[k] * (double)u;
   }
-  w.dq[bi * w.A + a] = dq;
-  w.dvp[bi * w.A + a] = dv;
+  w.dq[bi * w.A + a] = (float)dq;
+  w.dvp[bi * w.A + a] = (float)dv;
 }
 
 // grid (cdiv(len * (A + Hs), kT)): e < len * A: dK[j0 + k][a] += sum_b de_bk v_a (1 - u²);

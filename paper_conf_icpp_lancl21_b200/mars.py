@@ -130,6 +130,10 @@ SIGNATURES = {
     "mars_placer_sample": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
                                           ctypes.c_int32, ctypes.c_uint64, ctypes.c_void_p,
                                           ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_placer_ppo_grad": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
+                                            ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
+                                            ctypes.c_void_p, ctypes.c_float, ctypes.c_float,
+                                            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -576,6 +580,22 @@ class Placer:
                                         None if f is None else _ptr(f), _ptr(place), _ptr(logp),
                                         _ptr(ent)))
         return place, logp, ent
+
+    def ppo_grad(self, embeddings, placements, logp_old, adv, clip_eps=0.2, ent_coef=0.001):
+        """mars_placer_ppo_grad: (loss, grads [P], dL/dE [N x H])."""
+        E = np.ascontiguousarray(embeddings, np.float32)
+        N = E.shape[0]
+        pl = np.ascontiguousarray(placements, np.int32)
+        S = pl.shape[0]
+        lo = np.ascontiguousarray(logp_old, np.float32).reshape(S, N)
+        ad = np.ascontiguousarray(adv, np.float32).reshape(S)
+        loss = np.zeros(1, np.float32)
+        g = np.zeros(self.P, np.float32)
+        dE = np.zeros_like(E)
+        _check(lib().mars_placer_ppo_grad(self.handle, _ptr(E), N, S, _ptr(pl), _ptr(lo), _ptr(ad),
+                                          float(clip_eps), float(ent_coef), _ptr(loss), _ptr(g),
+                                          _ptr(dE)))
+        return float(loss[0]), g, dE
 
     def free(self):
         if self.handle:
