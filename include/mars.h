@@ -343,6 +343,14 @@ MARS_API mars_status mars_placer_sample(mars_placer* p, const float* embeddings,
                                         const int32_t* forced, int32_t* placements, float* logp,
                                         float* entropy);
 
+/* The encoder's vector-Jacobian product (NEXT-3's joint update): the gradient
+ * [P] (flat layout, host; dM = 0) of sum(dE ⊙ H3) with H3 = mars_encode(m, g)
+ * at the current parameters, for an external loss's dL/dH3 = dE [ΣN x H] (host).
+ * fp32 models; unsharded graphs; synchronous.  Overwrites the step's saved
+ * activations. */
+MARS_API mars_status mars_dgi_encoder_vjp(mars_dgi* m, const mars_graph* g, const float* dE,
+                                          float* grads);
+
 /* NEXT-3 (§3.4; readings c29-c31): the PPO loss
  * of S placements re-evaluated under the current policy (teacher forcing) --
  *   L = -(1/(S N)) sum_{b,i} min(rho A_b, clip(rho, 1 - eps, 1 + eps) A_b)
@@ -357,6 +365,44 @@ MARS_API mars_status mars_placer_ppo_grad(mars_placer* p, const float* embedding
                                           const float* logp_old, const float* adv,
                                           float clip_eps, float ent_coef, float* loss,
                                           float* grads, float* d_embeddings);
+
+/* NEXT-3: PPO training of the placer (c29-c32).  One
+ * iteration: sample policies x samples_per_policy placements from the current
+ * policy, measure each with the synthetic per-step-time model (c30: per-device
+ * compute + received bytes, out of memory -> 100 s), Eq. 7 advantages over the
+ * placements in sampling order with the baseline carried across iterations,
+ * then `epochs` passes over a seeded shuffle in `minibatches` minibatches: the
+ * PPO loss gradient (mars_placer_ppo_grad) clipped to clip_norm and an Adam
+ * step (lr 3e-4).  Defaults are the paper's. */
+typedef struct mars_ppo mars_ppo;
+typedef struct {
+  float clip_eps, ent_coef, lr, beta1, beta2, adam_eps, clip_norm, mu;
+  int32_t samples_per_policy, policies, minibatches, epochs;
+  uint64_t seed;
+  float capacity_bytes;       /* device memory of the step-time model (c30)      */
+} mars_ppo_config;
+MARS_API void mars_ppo_config_default(mars_ppo_config* cfg);
+/* encoder: the DGI-pre-trained GCN to train jointly (NULL: placer only). */
+MARS_API mars_status mars_ppo_create(mars_placer* placer, mars_dgi* encoder,
+                                     const mars_ppo_config* cfg, mars_ppo** out);
+/* One iteration on one op graph: embeddings [N x in_dim] (host), shape dims
+ * [N x 8] and the directed data-flow CSR (indptr [N+1], indices) for the
+ * step-time model.  Optional host outputs: placements [S x N], step_times [S],
+ * advantages [S] (S = policies x samples_per_policy), mean minibatch loss. */
+MARS_API mars_status mars_ppo_iteration(mars_ppo* o, const float* embeddings, int32_t num_ops,
+                                        const int64_t* dims, const int64_t* indptr,
+                                        const int32_t* indices, int32_t* placements,
+                                        float* step_times, float* advantages, float* mean_loss);
+/* The joint update of Mars ("jointly train the two components ... end
+ * to end"): the embeddings are the encoder's (mars_encode on the device, one
+ * op graph in g) and every minibatch also back-propagates dL/dE through the
+ * three GCN layers (the stacked backward of the DGI step with a zero
+ * corrupted half) into an Adam step of the encoder (its own Adam state,
+ * the PPO lr / clip).  fp32, single-GPU encoders. */
+MARS_API mars_status mars_ppo_iteration_joint(mars_ppo* o, const mars_graph* g, const int64_t* dims,
+                                              const int64_t* indptr, const int32_t* indices,
+                                              int32_t* placements, float* step_times,
+                                              float* advantages, float* mean_loss);
 
 /* Copies the most recent step's loss and global-mean gradient (the values
  * Adam consumed) to host memory (either may be NULL).  Synchronous.  For a
@@ -427,7 +473,7 @@ MARS_API mars_status mars_shard_connect_local(mars_dgi* const* models, int32_t n
 /* Kernel launches enqueued by the most recent mars_dgi_step (for reporting). */
 MARS_API int64_t mars_dgi_last_launches(const mars_dgi* m);
 
-/* Frees a mars_graph*, mars_dgi* or mars_placer* (tag-checked; NULL is a no-op). */
+/* Frees a mars_graph*, mars_dgi*, mars_placer* or mars_ppo* (tag-checked; NULL is a no-op). */
 MARS_API void mars_free(void* handle);
 
 #ifdef __cplusplus

@@ -339,6 +339,10 @@ cudaError_t placer_emb_grad(const float* dx, const int32_t* prev, int64_t SN, in
 cudaError_t placer_gather_rows(const float* in, const int32_t* order, int64_t rows, int cols,
                                float* out, int scatter_add, cudaStream_t s);
 cudaError_t placer_add(float* a, const float* b, int64_t n, cudaStream_t s);
+// NEXT-3 environment (c30): out[b] = per-step seconds of placement b (place [S x N]).
+cudaError_t launch_step_time(const int32_t* place, int32_t S, int32_t N, const int64_t* dims,
+                             const int64_t* indptr, const int32_t* indices, int D,
+                             double capacity, double* out, cudaStream_t s);
 cudaError_t placer_build_x(const float* ctx, const int32_t* prev, const float* emb, int64_t SN,
                            int Hs, int De, float* X, cudaStream_t s);
 cudaError_t placer_gather_cols(const float* in, int64_t ld, int col0, const int32_t* order,

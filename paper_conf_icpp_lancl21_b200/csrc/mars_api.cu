@@ -27,6 +27,7 @@ constexpr uint64_t kTagGraph = 0x4D41525347524150ULL;  // "MARSGRAP"
 constexpr uint64_t kTagDgi = 0x4D41525344474931ULL;    // "MARSDGI1"
 constexpr uint64_t kTagDead = 0xDEADDEADDEADDEADULL;
 constexpr uint64_t kTagPlacer = 0x4D415253504C4331ULL;  // "MARSPLC1"
+constexpr uint64_t kTagPpo = 0x4D41525350504F31ULL;     // "MARSPPO1"
 constexpr int kChunkRows = 256;   // deterministic reduction chunk (rows, within one graph)
 
 thread_local std::string g_err;
@@ -1591,6 +1592,42 @@ extern "C" int64_t mars_dgi_last_launches(const mars_dgi* m) {
 }
 
 // ---------------------------------------------------------------- encode (a15)
+// Forward of the positive branch only (a15): Y_l, Z_l of rows [0, ΣN) and
+// H3 = PReLU(Z3) into w.dY (the embeddings, device).
+static cudaError_t enqueue_encode(mars_dgi* m, const mars_graph* g, cudaStream_t s, int* nl) {
+  Workspace& w = m->ws;
+  GraphDev gd = g->dev;
+  gd.long_part = w.long_part;
+  const int F = m->F, H = m->H;
+  float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
+  float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
+  float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
+  const bool b16 = m->cfg.precision == MARS_BF16;
+  cudaError_t e;
+  for (int l = 0; l < 3; ++l) {
+    int Cin = l == 0 ? F : H;
+    const void* T = l == 0 ? (const void*)gd.X : (const void*)w.Z[l - 1];
+    const bool h3l = !b16 && m->gemm_impl == MARS_GEMM_AUTO && tc_supported(Cin, H);
+    if ((e = launch_spmm_fwd(gd, Cin, T, b16 && l > 0, nullptr, alpha, l - 1, Ys[l], b16, 0, s, nl,
+                             nullptr, h3l ? w.h3_rsY[l] : nullptr)))
+      return e;
+    if (b16) {
+      if ((e = tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl))) return e;
+      if ((e = tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], gd.Nt, H, Cin, s, nl))) return e;
+    } else if (h3l) {
+      if ((e = tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
+                                  w.h3_w_hi[l], w.h3_w_lo[l], s, nl)))
+        return e;
+      if ((e = tc3h_gemm_rows(Ys[l], w.h3_rsY[l], w.h3_wt_hi[l], w.h3_wt_lo[l], w.h3_wsc[l] + 1,
+                              w.Z[l], gd.Nt, H, Cin, s, nl)))
+        return e;
+    } else if ((e = gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, nl))) {
+      return e;
+    }
+  }
+  return launch_prelu(w.Z[2], b16, alpha, 2, w.dY, (int64_t)gd.Nt * H, s, nl);
+}
+
 extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb) {
   if (mars_status st = check_dgi(m)) return st;
   if (mars_status st = check_graph(g)) return st;
@@ -1599,39 +1636,104 @@ extern "C" mars_status mars_encode(mars_dgi* m, const mars_graph* g, float* emb)
   if (g->F != m->F) return fail(MARS_EINVAL, "feat_dim mismatch");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
-  Workspace& w = m->ws;
-  GraphDev gd = g->dev;
-  gd.long_part = w.long_part;
   cudaStream_t s = m->stream;
-  const int F = m->F, H = m->H;
-  float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
-  float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
-  float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
   int nl = 0;
-  const bool b16 = m->cfg.precision == MARS_BF16;
-  for (int l = 0; l < 3; ++l) {
-    int Cin = l == 0 ? F : H;
-    const void* T = l == 0 ? (const void*)gd.X : (const void*)w.Z[l - 1];
-    const bool h3l = !b16 && m->gemm_impl == MARS_GEMM_AUTO && tc_supported(Cin, H);
-    CK(launch_spmm_fwd(gd, Cin, T, b16 && l > 0, nullptr, alpha, l - 1, Ys[l], b16, 0, s, &nl,
-                       nullptr, h3l ? w.h3_rsY[l] : nullptr));
-    if (b16) {
-      CK(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, &nl));
-      CK(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
-    } else if (m->gemm_impl == MARS_GEMM_AUTO && tc_supported(Cin, H)) {
-      CK(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
-                            w.h3_w_hi[l], w.h3_w_lo[l], s, &nl));
-      CK(tc3h_gemm_rows(Ys[l], w.h3_rsY[l], w.h3_wt_hi[l], w.h3_wt_lo[l], w.h3_wsc[l] + 1, w.Z[l],
-                        gd.Nt, H, Cin, s, &nl));
-    } else {
-      CK(gemm_nn(Ys[l], W[l], w.Z[l], gd.Nt, H, Cin, s, &nl));
-    }
-  }
-  CK(launch_prelu(w.Z[2], b16, alpha, 2, w.dY, (int64_t)gd.Nt * H, s, &nl));
-  CK(cudaMemcpyAsync(emb, w.dY, sizeof(float) * (size_t)gd.Nt * H, cudaMemcpyDeviceToHost, s));
+  CK(enqueue_encode(m, g, s, &nl));
+  CK(cudaMemcpyAsync(emb, m->ws.dY, sizeof(float) * (size_t)g->dev.Nt * m->H,
+                     cudaMemcpyDeviceToHost, s));
   CK(cudaStreamSynchronize(s));
+  g->note_use(s);
   m->last_Nt = 0;
   return MARS_OK;
+}
+
+namespace {
+// Joint training (NEXT-3): dZ3 of the stacked layout from dL/dH3 of the
+// positive rows: rows r < Nt: dE ⊙ PReLU'(Z3), rows >= Nt: 0; the 3xFP16 row
+// scales; per-row dalpha3 terms sum_c dE min(Z3, 0) into slots[r] (fixed order).
+__global__ void k_dz3_from_dE(const float* __restrict__ dE, const float* __restrict__ Z3,
+                              const float* __restrict__ alpha, int32_t Nt, int H,
+                              float* __restrict__ dZ, float* __restrict__ rs,
+                              double* __restrict__ slots) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (warp >= 2 * Nt) return;
+  const int64_t r = warp;
+  const float a = alpha[2];
+  float mx = 0.f;
+  double da = 0.0;
+  for (int c = lane; c < H; c += 32) {
+    float d = 0.f;
+    if (r < Nt) {
+      const float z = Z3[r * H + c], g = dE[r * H + c];
+      d = z > 0.f ? g : a * g;
+      if (!(z > 0.f)) da += (double)g * (double)z;
+    }
+    dZ[r * H + c] = d;
+    mx = fmaxf(mx, fabsf(d));
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(kFull, mx, o));
+  da = warp_sum(da);
+  if (lane == 0) {
+    if (rs) rs[r] = pow2_scale(mx);
+    if (r < Nt) slots[r] = da;
+  }
+}
+__global__ void k_fill_f(float* __restrict__ p, int64_t n, float v) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = v;
+}
+}  // namespace
+
+// Backward of the encoder from dL/dH3 of the positive rows (the placer's dE):
+// gradients of W1..3 and alpha into m->grads (dM = 0, loss slot 0), by the
+// stacked backward chain of the step with a zero corrupted half.  fp32 models.
+static cudaError_t enqueue_encoder_backward(mars_dgi* m, const mars_graph* gr, const float* dE,
+                                            cudaStream_t s, int* nl) {
+  Workspace& w = m->ws;
+  GraphDev g = gr->dev;
+  g.long_part = w.long_part;
+  const int F = m->F, H = m->H;
+  const int64_t Nt = g.Nt, R = 2 * Nt;
+  float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
+  float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
+  float* gW[3] = {m->grads, m->grads + (int64_t)F * H, m->grads + (int64_t)F * H + (int64_t)H * H};
+  float* galpha = m->grads + (int64_t)F * H + 3LL * H * H;
+  float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
+  cudaError_t e;
+  // the corrupted half of the saved activations is zero (and its row scales neutral)
+  if ((e = cudaMemsetAsync(w.Y1 + Nt * F, 0, sizeof(float) * Nt * F, s))) return e;
+  for (int l = 0; l < 2; ++l)
+    if ((e = cudaMemsetAsync(w.Y23[l] + Nt * H, 0, sizeof(float) * Nt * H, s))) return e;
+  for (int l = 0; l < 3; ++l) {
+    if ((e = cudaMemsetAsync(w.Z[l] + Nt * H, 0, sizeof(float) * Nt * H, s))) return e;
+    k_fill_f<<<cdiv(Nt, 256), 256, 0, s>>>(w.h3_rsY[l] + Nt, Nt, 0x1p100f);
+  }
+  if ((e = cudaMemsetAsync(m->grads, 0, sizeof(float) * (m->P + 1), s))) return e;
+  bool tc[3];
+  for (int l = 0; l < 3; ++l) tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(l == 0 ? F : H, H);
+  k_dz3_from_dE<<<cdiv(R * 32, 256), 256, 0, s>>>(dE, w.Z[2], alpha, (int32_t)Nt, H, w.dZ,
+                                                   tc[2] ? w.h3_rsdZ : nullptr, w.slots[2]);
+  count_launch(nl, 2 + 3);
+  if ((e = launch_reduce_slots(w.slots[2], (int)Nt, galpha + 2, s, nl))) return e;
+  int ns = 0;
+  for (int l = 2; l >= 0; --l) {
+    const int Cin = l == 0 ? F : H;
+    if (tc[l]) e = tc3h_gemm_dw(Ys[l], w.h3_rsY[l], w.dZ, w.h3_rsdZ, gW[l], R, Cin, H, w.dw_part, s, nl);
+    else e = gemm_tn(Ys[l], w.dZ, gW[l], R, Cin, H, w.tn_part, s, nl);
+    if (e) return e;
+    if (l > 0) {
+      if (tc[l]) e = tc3h_gemm_rows(w.dZ, w.h3_rsdZ, w.h3_w_hi[l], w.h3_w_lo[l], w.h3_wsc[l] + 1,
+                                    w.dY, R, Cin, H, s, nl);
+      else e = gemm_nt(w.dZ, W[l], w.dY, R, Cin, H, s, nl);
+      if (e) return e;
+      if ((e = launch_spmm_bwd(g, Cin, w.dY, w.Z[l - 1], 0, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
+                               s, nl, nullptr, tc[l - 1] ? w.h3_rsdZ : nullptr)))
+        return e;
+      if ((e = launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl))) return e;
+    }
+  }
+  return cudaSuccess;
 }
 
 // ---------------------------------------------------------------- hooks / state
@@ -2628,6 +2730,278 @@ extern "C" mars_status mars_placer_sample(mars_placer* p, const float* emb, int3
   return MARS_OK;
 }
 
+extern "C" mars_status mars_dgi_encoder_vjp(mars_dgi* m, const mars_graph* g, const float* dE,
+                                            float* grads) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (mars_status st = check_graph(g)) return st;
+  if (!dE || !grads) return fail(MARS_EINVAL, "NULL argument");
+  if (g->sharded || g->F != m->F) return fail(MARS_EINVAL, "unsharded graph of the model's F");
+  if (m->cfg.precision != MARS_FP32) return fail(MARS_EINVAL, "fp32 models only");
+  CK(cudaSetDevice(m->cfg.device));
+  if (mars_status st = ensure_ws(m, g)) return st;
+  cudaStream_t s = m->stream;
+  float* d = nullptr;
+  const size_t n = (size_t)g->dev.Nt * m->H;
+  CK(palloc(&d, n, s));
+  struct F1 { float* p; cudaStream_t s; ~F1() { cudaFreeAsync(p, s); } } f1{d, s};
+  CK(cudaMemcpyAsync(d, dE, sizeof(float) * n, cudaMemcpyHostToDevice, s));
+  int nl = 0;
+  CK(enqueue_encode(m, g, s, &nl));
+  CK(enqueue_encoder_backward(m, g, d, s, &nl));
+  CK(cudaMemcpyAsync(grads, m->grads, sizeof(float) * m->P, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  g->note_use(s);
+  m->last_Nt = 0;
+  return MARS_OK;
+}
+
+// ---------------------------------------------------------------- PPO (NEXT-3)
+struct mars_ppo {
+  uint64_t tag = kTagPpo;
+  mars_ppo_config cfg{};
+  mars_placer* p = nullptr;
+  mars_dgi* enc = nullptr;           // joint update of the GCN encoder (NULL: placer only)
+  float *m = nullptr, *v = nullptr;  // Adam state of the placer
+  double* guard = nullptr;
+  AdamDev* st = nullptr;
+  float *em = nullptr, *ev = nullptr;    // Adam state of the encoder (joint training)
+  double* eguard = nullptr;
+  AdamDev* est = nullptr;
+  double baseline = 0.0;             // Eq. 7's B_{t-1}
+  bool has_baseline = false;
+  int64_t iteration = 0;
+  ~mars_ppo() {
+    for (void* q : {(void*)m, (void*)v, (void*)guard, (void*)st, (void*)em, (void*)ev,
+                    (void*)eguard, (void*)est})
+      if (q) cudaFree(q);
+  }
+};
+
+extern "C" void mars_ppo_config_default(mars_ppo_config* c) {
+  if (!c) return;
+  memset(c, 0, sizeof *c);
+  c->clip_eps = 0.2f;
+  c->ent_coef = 0.001f;
+  c->lr = 3e-4f;
+  c->beta1 = 0.9f;
+  c->beta2 = 0.999f;
+  c->adam_eps = 1e-8f;
+  c->clip_norm = 1.0f;
+  c->mu = 0.99f;
+  c->samples_per_policy = 10;
+  c->policies = 2;
+  c->minibatches = 4;
+  c->epochs = 3;
+  c->capacity_bytes = 12e9f;
+}
+
+extern "C" mars_status mars_ppo_create(mars_placer* p, mars_dgi* enc, const mars_ppo_config* cfg,
+                                       mars_ppo** out) {
+  if (!out) return fail(MARS_EINVAL, "out is NULL");
+  *out = nullptr;
+  if (mars_status st = check_placer(p)) return st;
+  if (enc) {
+    if (mars_status st = check_dgi(enc)) return st;
+    if (enc->H != p->d.H) return fail(MARS_EINVAL, "encoder hidden_dim != placer in_dim");
+    if (enc->cfg.device != p->cfg.device) return fail(MARS_EINVAL, "encoder and placer on different devices");
+  }
+  if (!cfg) return fail(MARS_EINVAL, "NULL config");
+  const int S = cfg->samples_per_policy * cfg->policies;
+  if (cfg->samples_per_policy < 1 || cfg->policies < 1 || cfg->minibatches < 1 ||
+      cfg->epochs < 1 || S % cfg->minibatches || S / cfg->minibatches > 32 ||
+      cfg->samples_per_policy > 32)
+    return fail(MARS_EINVAL, "bad PPO schedule (samples / minibatches)");
+  if (p->d.D > 16) return fail(MARS_EINVAL, "the step-time model supports <= 16 devices");
+  CK(cudaSetDevice(p->cfg.device));
+  auto* o = new mars_ppo();
+  std::unique_ptr<mars_ppo> guard(o);
+  o->cfg = *cfg;
+  o->p = p;
+  o->enc = enc;
+  CK(dalloc(&o->m, (size_t)p->P));
+  CK(dalloc(&o->v, (size_t)p->P));
+  CK(dalloc(&o->guard, (size_t)adam_guard_doubles()));
+  CK(dalloc(&o->st, 1));
+  CK(cudaMemset(o->m, 0, sizeof(float) * p->P));
+  CK(cudaMemset(o->v, 0, sizeof(float) * p->P));
+  CK(cudaMemset(o->st, 0, sizeof(AdamDev)));
+  if (enc) {
+    if (enc->cfg.precision != MARS_FP32) return fail(MARS_EINVAL, "joint training needs an fp32 encoder");
+    if (enc->sh.g || enc->dp.R > 1 || enc->comm)
+      return fail(MARS_EINVAL, "joint training needs a single-GPU, unsharded encoder");
+    CK(dalloc(&o->em, (size_t)enc->P));
+    CK(dalloc(&o->ev, (size_t)enc->P));
+    CK(dalloc(&o->eguard, (size_t)adam_guard_doubles()));
+    CK(dalloc(&o->est, 1));
+    CK(cudaMemset(o->em, 0, sizeof(float) * enc->P));
+    CK(cudaMemset(o->ev, 0, sizeof(float) * enc->P));
+    CK(cudaMemset(o->est, 0, sizeof(AdamDev)));
+  }
+  *out = guard.release();
+  return MARS_OK;
+}
+
+static mars_status check_ppo(const mars_ppo* o) {
+  if (!o || o->tag != kTagPpo) return fail(MARS_ESTATE, "invalid or freed mars_ppo handle");
+  return check_placer(o->p);
+}
+
+// One PPO iteration (readings c29-c32): sample policies x samples
+// placements from the current policy, measure them (c30), Eq. 7 advantages in
+// sampling order (c31), then `epochs` passes over a seeded shuffle of the
+// placements in `minibatches` equal minibatches: per minibatch the PPO loss
+// gradient (mars_placer_ppo_grad's path), clipped to clip_norm, and an Adam step.
+static mars_status ppo_iteration(mars_ppo* o, const float* emb, const mars_graph* g, int32_t N,
+                                 const int64_t* dims, const int64_t* indptr,
+                                 const int32_t* indices, int32_t* placements_out,
+                                 float* step_times_out, float* adv_out, float* mean_loss) {
+  mars_placer* p = o->p;
+  mars_dgi* enc = o->enc;
+  const mars_ppo_config& c = o->cfg;
+  if ((!emb && !g) || !dims || !indptr || N < 1) return fail(MARS_EINVAL, "NULL input or N < 1");
+  const int H = p->d.H;
+  if (!(H == 32 || H == 64 || H % 128 == 0))
+    return fail(MARS_EINVAL, "training needs in_dim in {32, 64} or a multiple of 128");
+  const int S = c.samples_per_policy * c.policies, mb = S / c.minibatches;
+  const int64_t E = indptr[N];
+  CK(cudaSetDevice(p->cfg.device));
+  cudaStream_t s = p->stream;
+  if (mars_status st = placer_ensure(p, N, std::max(S, c.samples_per_policy))) return st;
+  if (mars_status st = placer_ensure_train(p, N, mb)) return st;
+  float* dE = nullptr;
+  int32_t *dPl = nullptr, *dMb = nullptr, *dIdx = nullptr;
+  float *dLp = nullptr, *dEnt = nullptr;
+  int64_t *dDims = nullptr, *dIp = nullptr;
+  double* dT = nullptr;
+  struct FreeAll { std::vector<void*> v; cudaStream_t s; ~FreeAll() { for (void* q : v) cudaFreeAsync(q, s); } } fa{{}, s};
+  CK(palloc(&dE, (size_t)N * H, s)); fa.v.push_back(dE);
+  CK(palloc(&dPl, (size_t)S * N, s)); fa.v.push_back(dPl);
+  CK(palloc(&dMb, (size_t)mb * N, s)); fa.v.push_back(dMb);
+  CK(palloc(&dLp, (size_t)S * N, s)); fa.v.push_back(dLp);
+  CK(palloc(&dEnt, (size_t)S * N, s)); fa.v.push_back(dEnt);
+  CK(palloc(&dDims, (size_t)N * 8, s)); fa.v.push_back(dDims);
+  CK(palloc(&dIp, (size_t)N + 1, s)); fa.v.push_back(dIp);
+  CK(palloc(&dIdx, (size_t)std::max<int64_t>(E, 1), s)); fa.v.push_back(dIdx);
+  CK(palloc(&dT, (size_t)S, s)); fa.v.push_back(dT);
+  if (enc) {                        // joint: the embeddings are the GCN encoder's, on the device
+    CK(cudaStreamSynchronize(enc->stream));
+    if (mars_status st = ensure_ws(enc, g)) return st;
+    CK(enqueue_encode(enc, g, s, nullptr));
+    CK(cudaMemcpyAsync(dE, enc->ws.dY, sizeof(float) * (size_t)N * H, cudaMemcpyDeviceToDevice, s));
+  } else {
+    CK(cudaMemcpyAsync(dE, emb, sizeof(float) * (size_t)N * H, cudaMemcpyHostToDevice, s));
+  }
+  CK(cudaMemcpyAsync(dDims, dims, sizeof(int64_t) * N * 8, cudaMemcpyHostToDevice, s));
+  CK(cudaMemcpyAsync(dIp, indptr, sizeof(int64_t) * (N + 1), cudaMemcpyHostToDevice, s));
+  if (E > 0) CK(cudaMemcpyAsync(dIdx, indices, sizeof(int32_t) * E, cudaMemcpyHostToDevice, s));
+  int nl = 0;
+  // 1. sample: `policies` draws of samples_per_policy placements, each its own seed
+  for (int q = 0; q < c.policies; ++q) {
+    const uint64_t seed = sm64(sm64(c.seed ^ 0x50504F53ULL) ^ (uint64_t)(o->iteration * c.policies + q));
+    const int64_t off = (int64_t)q * c.samples_per_policy * N;
+    CK(placer_forward(p->d, p->w, p->ws, dE, N, p->cfg.segment, c.samples_per_policy, seed,
+                      nullptr, dPl + off, dLp + off, dEnt + off, s, &nl));
+  }
+  // 2. the environment (c30) and Eq. 7 (c31) in sampling order
+  CK(launch_step_time(dPl, S, N, dDims, dIp, dIdx, p->d.D, (double)c.capacity_bytes, dT, s));
+  std::vector<double> times(S);
+  std::vector<float> lp_old((size_t)S * N);
+  CK(cudaMemcpyAsync(times.data(), dT, sizeof(double) * S, cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(lp_old.data(), dLp, sizeof(float) * S * N, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  std::vector<float> adv(S);
+  for (int b = 0; b < S; ++b) {
+    const double R = -std::sqrt(times[b]);
+    o->baseline = o->has_baseline ? (1.0 - c.mu) * R + c.mu * o->baseline : R;
+    o->has_baseline = true;
+    adv[b] = (float)(R - o->baseline);
+  }
+  // 3. epochs x minibatches over a seeded shuffle (c32: Fisher-Yates on splitmix64)
+  double loss_sum = 0.0;
+  int nsteps = 0;
+  std::vector<int32_t> order(S);
+  std::vector<float> adv_mb(mb), lp_mb((size_t)mb * N);
+  for (int ep = 0; ep < c.epochs; ++ep) {
+    for (int b = 0; b < S; ++b) order[b] = b;
+    const uint64_t key = sm64(sm64(c.seed ^ 0x53485546ULL) ^ (uint64_t)(o->iteration * c.epochs + ep));
+    for (int b = S - 1; b > 0; --b) {
+      const int r = (int)(sm64(key ^ (uint64_t)b) % (uint64_t)(b + 1));
+      std::swap(order[b], order[r]);
+    }
+    for (int k = 0; k < c.minibatches; ++k) {
+      for (int q = 0; q < mb; ++q) {
+        const int b = order[k * mb + q];
+        CK(cudaMemcpyAsync(dMb + (int64_t)q * N, dPl + (int64_t)b * N, sizeof(int32_t) * N,
+                           cudaMemcpyDeviceToDevice, s));
+        adv_mb[q] = adv[b];
+        memcpy(lp_mb.data() + (size_t)q * N, lp_old.data() + (size_t)b * N, sizeof(float) * N);
+      }
+      CK(cudaMemcpyAsync(const_cast<float*>(p->tr.logp_old), lp_mb.data(), sizeof(float) * mb * N,
+                         cudaMemcpyHostToDevice, s));
+      CK(cudaMemcpyAsync(const_cast<float*>(p->tr.adv), adv_mb.data(), sizeof(float) * mb,
+                         cudaMemcpyHostToDevice, s));
+      const float* Ecur = dE;
+      if (enc) {                     // the encoder's current embeddings
+        CK(enqueue_encode(enc, g, s, &nl));
+        Ecur = enc->ws.dY;
+      }
+      if (mars_status st = placer_loss_grad(p, Ecur, N, mb, dMb, c.clip_eps, c.ent_coef, &nl)) return st;
+      if (enc) {                     // dL/dE (p->tmpNH) on through the GCN, then its Adam step
+        CK(enqueue_encoder_backward(enc, g, p->tmpNH, s, &nl));
+        CK(launch_adam(enc->params, o->em, o->ev, enc->grads, enc->P, c.lr, c.beta1, c.beta2,
+                       c.adam_eps, c.clip_norm, o->eguard, o->est, s, &nl));
+      }
+      CK(launch_adam(p->params, o->m, o->v, p->grads, p->P, c.lr, c.beta1, c.beta2, c.adam_eps,
+                     c.clip_norm, o->guard, o->st, s, &nl));
+      float lsum = 0.f;
+      CK(cudaMemcpyAsync(&lsum, p->grads + p->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+      CK(cudaStreamSynchronize(s));       // the host-side staging buffers are reused
+      loss_sum += (double)lsum / ((double)mb * N);
+      ++nsteps;
+    }
+  }
+  if (placements_out)
+    CK(cudaMemcpyAsync(placements_out, dPl, sizeof(int32_t) * S * N, cudaMemcpyDeviceToHost, s));
+  CK(cudaStreamSynchronize(s));
+  if (step_times_out)
+    for (int b = 0; b < S; ++b) step_times_out[b] = (float)times[b];
+  if (adv_out) memcpy(adv_out, adv.data(), sizeof(float) * S);
+  if (mean_loss) *mean_loss = (float)(loss_sum / nsteps);
+  o->iteration += 1;
+  int32_t skipped = 0, eskipped = 0;
+  CK(cudaMemcpy(&skipped, &o->st->skipped, sizeof(int32_t), cudaMemcpyDeviceToHost));
+  if (enc) CK(cudaMemcpy(&eskipped, &o->est->skipped, sizeof(int32_t), cudaMemcpyDeviceToHost));
+  if (skipped || eskipped)
+    return fail(MARS_ENUMERIC, "non-finite PPO gradient: %d update(s) skipped", skipped + eskipped);
+  if (enc) g->note_use(s);
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_ppo_iteration(mars_ppo* o, const float* emb, int32_t N,
+                                          const int64_t* dims, const int64_t* indptr,
+                                          const int32_t* indices, int32_t* placements_out,
+                                          float* step_times_out, float* adv_out, float* mean_loss) {
+  if (mars_status st = check_ppo(o)) return st;
+  if (o->enc) return fail(MARS_ESTATE, "a joint PPO handle takes mars_ppo_iteration_joint");
+  return ppo_iteration(o, emb, nullptr, N, dims, indptr, indices, placements_out, step_times_out,
+                       adv_out, mean_loss);
+}
+
+extern "C" mars_status mars_ppo_iteration_joint(mars_ppo* o, const mars_graph* g,
+                                                const int64_t* dims, const int64_t* indptr,
+                                                const int32_t* indices, int32_t* placements_out,
+                                                float* step_times_out, float* adv_out,
+                                                float* mean_loss) {
+  if (mars_status st = check_ppo(o)) return st;
+  if (!o->enc) return fail(MARS_ESTATE, "mars_ppo_create was given no encoder");
+  if (mars_status st = check_graph(g)) return st;
+  if (mars_status st = check_dgi(o->enc)) return st;
+  if (g->G != 1 || g->sharded || g->F != o->enc->F)
+    return fail(MARS_EINVAL, "joint training takes one unsharded op graph of the encoder's F");
+  return ppo_iteration(o, nullptr, g, g->Nt, dims, indptr, indices, placements_out,
+                       step_times_out, adv_out, mean_loss);
+}
+
 extern "C" void mars_free(void* h) {
   if (!h) return;
   uint64_t tag = *static_cast<uint64_t*>(h);
@@ -2642,6 +3016,10 @@ extern "C" void mars_free(void* h) {
     cudaStreamSynchronize(m->stream);
     m->tag = kTagDead;
     delete m;
+  } else if (tag == kTagPpo) {
+    auto* o = static_cast<mars_ppo*>(h);
+    o->tag = kTagDead;
+    delete o;
   } else if (tag == kTagPlacer) {
     auto* p = static_cast<mars_placer*>(h);
     cudaSetDevice(p->cfg.device);

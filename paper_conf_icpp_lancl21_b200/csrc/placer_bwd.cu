@@ -376,3 +376,70 @@ cudaError_t placer_add(float* a, const float* b, int64_t n, cudaStream_t s) {
 }
 
 }  // namespace mars
+
+namespace mars {
+namespace {
+
+// NEXT-3's environment (reading c30): per-step seconds of each placement under a
+// synthetic cost model.  One block per placement; thread t sums a fixed
+// contiguous range of ops into per-device compute / resident bytes / received
+// bytes, then the block combines the threads in order (deterministic, double).
+__global__ void __launch_bounds__(256)
+k_step_time(const int32_t* __restrict__ place, int32_t N, const int64_t* __restrict__ dims,
+            const int64_t* __restrict__ indptr, const int32_t* __restrict__ indices, int D,
+            double capacity, double* __restrict__ out) {
+  extern __shared__ double sh[];                 // [256][3 D]
+  const int b = blockIdx.x, t = threadIdx.x;
+  const int32_t* p = place + (int64_t)b * N;
+  double* mine = sh + (int64_t)t * 3 * D;
+  for (int k = 0; k < 3 * D; ++k) mine[k] = 0.0;
+  const int64_t per = (N + 255) / 256;
+  const int64_t u0 = t * per, u1 = min((int64_t)N, u0 + per);
+  for (int64_t u = u0; u < u1; ++u) {
+    double sz = 1.0;
+    for (int j = 4; j < 8; ++j) {
+      const int64_t dd = dims[u * 8 + j];
+      if (dd > 0) sz *= (double)dd;
+    }
+    const int du = p[u];
+    mine[du] += sz * 1e-12;                      // compute
+    mine[D + du] += sz * 4.0;                    // resident bytes
+    for (int64_t e = indptr[u]; e < indptr[u + 1]; ++e) {
+      const int dv = p[indices[e]];
+      if (dv != du) mine[2 * D + dv] += sz * 4.0 / 12e9;   // received by the consumer's device
+    }
+  }
+  __syncthreads();
+  if (t == 0) {
+    double worst = 0.0;
+    bool oom = false;
+    for (int dv = 0; dv < D; ++dv) {
+      double c = 0.0, m = 0.0, r = 0.0;
+      for (int q = 0; q < 256; ++q) {
+        c += sh[(int64_t)q * 3 * D + dv];
+        m += sh[(int64_t)q * 3 * D + D + dv];
+        r += sh[(int64_t)q * 3 * D + 2 * D + dv];
+      }
+      if (m > capacity) oom = true;
+      worst = fmax(worst, c + r);
+    }
+    out[b] = oom ? 100.0 : worst;
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_step_time(const int32_t* place, int32_t S, int32_t N, const int64_t* dims,
+                             const int64_t* indptr, const int32_t* indices, int D,
+                             double capacity, double* out, cudaStream_t s) {
+  const size_t smem = sizeof(double) * 256 * 3 * D;
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(k_step_time, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+  k_step_time<<<S, 256, smem, s>>>(place, N, dims, indptr, indices, D, capacity, out);
+  return cudaGetLastError();
+}
+
+}  // namespace mars

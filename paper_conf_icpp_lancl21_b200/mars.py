@@ -57,6 +57,15 @@ class PlacerConfig(ctypes.Structure):
                 ("device", ctypes.c_int32)]
 
 
+class PpoConfig(ctypes.Structure):
+    _fields_ = [("clip_eps", ctypes.c_float), ("ent_coef", ctypes.c_float), ("lr", ctypes.c_float),
+                ("beta1", ctypes.c_float), ("beta2", ctypes.c_float), ("adam_eps", ctypes.c_float),
+                ("clip_norm", ctypes.c_float), ("mu", ctypes.c_float),
+                ("samples_per_policy", ctypes.c_int32), ("policies", ctypes.c_int32),
+                ("minibatches", ctypes.c_int32), ("epochs", ctypes.c_int32),
+                ("seed", ctypes.c_uint64), ("capacity_bytes", ctypes.c_float)]
+
+
 class StepOut(ctypes.Structure):
     _fields_ = [("loss", ctypes.c_void_p), ("grads", ctypes.c_void_p), ("perms", ctypes.c_void_p)]
 
@@ -134,6 +143,18 @@ SIGNATURES = {
                                             ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
                                             ctypes.c_void_p, ctypes.c_float, ctypes.c_float,
                                             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_ppo_config_default": (None, [ctypes.POINTER(PpoConfig)]),
+    "mars_ppo_create": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.POINTER(PpoConfig),
+                                       ctypes.POINTER(ctypes.c_void_p)]),
+    "mars_ppo_iteration": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,
+                                          ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                          ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                          ctypes.c_void_p]),
+    "mars_dgi_encoder_vjp": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                            ctypes.c_void_p]),
+    "mars_ppo_iteration_joint": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                                ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p,
+                                                ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
     "mars_free": (None, [ctypes.c_void_p]),
 }
 
@@ -411,6 +432,13 @@ class DGI:
     def export_activations(self, layer: int):
         return dgi_export_activations(self, layer)
 
+    def encoder_vjp(self, g: Graph, dE):
+        """mars_dgi_encoder_vjp: gradient [P] of sum(dE * encode(g))."""
+        d = np.ascontiguousarray(dE, np.float32)
+        out = np.zeros(self.P, np.float32)
+        _check(lib().mars_dgi_encoder_vjp(self.handle, g.handle, _ptr(d), _ptr(out)))
+        return out
+
     def saved_rows(self) -> int:
         """Rows per branch of the last step's saved activations (0 after encode)."""
         r = ctypes.c_int64()
@@ -646,3 +674,74 @@ def debug_gemm(op: str, A, B, impl: str = "auto", iters: int = 0, device: int = 
 
 def free(handle_obj):
     handle_obj.free()
+
+
+# ------------------------------------------------------------------ PPO (NEXT-3)
+class Ppo:
+    """PPO training of a placer (mars_ppo*)."""
+
+    def __init__(self, handle, cfg: PpoConfig, placer: "Placer"):
+        self.handle, self.cfg, self.placer = handle, cfg, placer
+
+    @property
+    def num_samples(self):
+        return self.cfg.samples_per_policy * self.cfg.policies
+
+    def iteration(self, embeddings, graph):
+        """mars_ppo_iteration on one op graph (an object with num_nodes, indptr,
+        indices and dims [N x 8]).  Returns dict(placements, step_times,
+        advantages, loss)."""
+        E = np.ascontiguousarray(embeddings, np.float32)
+        N = E.shape[0]
+        dims = np.ascontiguousarray(graph.dims, np.int64).reshape(N, 8)
+        ip = np.ascontiguousarray(graph.indptr, np.int64)
+        ix = np.ascontiguousarray(graph.indices, np.int32)
+        S = self.num_samples
+        pl = np.zeros((S, N), np.int32)
+        t = np.zeros(S, np.float32)
+        a = np.zeros(S, np.float32)
+        loss = np.zeros(1, np.float32)
+        _check(lib().mars_ppo_iteration(self.handle, _ptr(E), N, _ptr(dims), _ptr(ip),
+                                        _ptr(ix) if ix.size else None, _ptr(pl), _ptr(t), _ptr(a),
+                                        _ptr(loss)))
+        return dict(placements=pl, step_times=t, advantages=a, loss=float(loss[0]))
+
+    def iteration_joint(self, g: Graph, graph):
+        """mars_ppo_iteration_joint: the encoder's embeddings of the loaded op graph
+        g (one graph), the step-time model from `graph` (dims, indptr, indices)."""
+        N = g.total_nodes
+        dims = np.ascontiguousarray(graph.dims, np.int64).reshape(N, 8)
+        ip = np.ascontiguousarray(graph.indptr, np.int64)
+        ix = np.ascontiguousarray(graph.indices, np.int32)
+        S = self.num_samples
+        pl = np.zeros((S, N), np.int32)
+        t = np.zeros(S, np.float32)
+        a = np.zeros(S, np.float32)
+        loss = np.zeros(1, np.float32)
+        _check(lib().mars_ppo_iteration_joint(self.handle, g.handle, _ptr(dims), _ptr(ip),
+                                              _ptr(ix) if ix.size else None, _ptr(pl), _ptr(t),
+                                              _ptr(a), _ptr(loss)))
+        return dict(placements=pl, step_times=t, advantages=a, loss=float(loss[0]))
+
+    def free(self):
+        if self.handle:
+            lib().mars_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def ppo_create(placer: Placer, encoder: "DGI | None" = None, **kw) -> Ppo:
+    c = PpoConfig()
+    lib().mars_ppo_config_default(ctypes.byref(c))
+    for k, v in kw.items():
+        setattr(c, k, v)
+    h = ctypes.c_void_p()
+    _check(lib().mars_ppo_create(placer.handle, None if encoder is None else encoder.handle,
+                                 ctypes.byref(c), ctypes.byref(h)))
+    return Ppo(h, c, placer)
+
