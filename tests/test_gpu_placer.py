@@ -97,3 +97,9 @@ def test_placer_paper_sizes_on_encoder_output():
     D = 4 devices, S = 4 samples, on an Inception-V3 op graph's embeddings."""
     E = _embeddings()
     _check(E, 4, 7, 99)
+
+
+def test_placer_gnmt_graph():
+    """A GNMT-4 op graph (~12k ops, 93 segments) at paper sizes, S = 2."""
+    E = _embeddings("gnmt")
+    _check(E, 2, 8, 41)

@@ -196,3 +196,28 @@ def test_joint_ppo_iteration_runs_and_moves_both():
     times = [ppo.step_time(out["placements"][b], g0.dims, g0.indptr, g0.indices, 4, 3e8)
              for b in range(8)]
     assert np.allclose(out["step_times"], times, rtol=1e-6)
+
+
+def test_ppo_grad_paper_sizes():
+    """P:L234 sizes (bi-LSTM 2 x 256, decoder 512, attention 512, device
+    embedding 64, s = 128, D = 4) on 300 ops (a ragged last segment), H = 256:
+    the PPO gradient of every block and dL/dE at 1e-5 of torch fp64 autograd."""
+    N, seg, S, H = 300, 128, 2, 256
+    dims = dict(H=H, Hd=256, A=512, De=64, D=4)
+    p = mars.placer_create(seed=6, in_dim=H)
+    rng = np.random.default_rng(11)
+    E = (0.3 * rng.standard_normal((N, H))).astype(np.float32)
+    place, logp, _ = p.sample(E, S, 5)
+    params1 = (p.get_params() + 0.01 * rng.standard_normal(p.P)).astype(np.float32)
+    p.set_params(params1)
+    adv = np.array([1.2, -0.7], np.float32)
+    loss, g, dE = p.ppo_grad(E, place, logp, adv)
+    L, gp, gE = ppo.ppo_grads(E.astype(np.float64), params1.astype(np.float64), dims, seg, place,
+                              logp.astype(np.float64), adv.astype(np.float64))
+    res = {"loss": abs(loss - L) / abs(L), "dE": scaled_err(dE, gE)}
+    for name, blk in _blocks(g, dims).items():
+        res[name] = scaled_err(blk, _blocks(gp, dims)[name])
+    print("paper sizes", {k: f"{v:.2e}" for k, v in res.items()})
+    bad = {k: v for k, v in res.items() if v > 1e-5}
+    assert not bad, bad
+    p.free()

@@ -11,7 +11,7 @@ timeout 300 python bench.py --impl reference --steps 2 --warmup 3 > $out/referen
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $out/launches.csv \
   python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --profile-steps 1 > /dev/null 2>&1; echo "launches rc $?"
 LIB=paper_conf_icpp_lancl21_b200/libmars.so
-K='regex:k_tc3h_rows|k_tc3h_dw|k_tc_rows|k_tc_dw2|k_tc16_rows|k_tc16_dw|k_spmm_fwd|k_spmm_bwd|k_dz3|k_score|k_colsum'
+K='regex:k_tc3h_rows|k_tc3h_dw|k_tc16_rows|k_tc16_dw|k_spmm_fwd|k_spmm_bwd|k_dz3|k_score|k_colsum'
 rep=${NCU_REP_DIR:-/tmp}    # large .ncu-rep files stay on the box; summaries come back
 timeout 900 ncu --set full --clock-control none --import-source on -f -k "$K" -c 17 -o $rep/full_fp32 \
   python tools/step_once.py $LIB fp32 1 > /dev/null 2>&1; echo "full fp32 rc $?"
@@ -19,5 +19,5 @@ timeout 900 ncu --set full --clock-control none --import-source on -f -k "$K" -c
   python tools/step_once.py $LIB bf16 1 > /dev/null 2>&1; echo "full bf16 rc $?"
 python tools/ncu_table.py $rep/full_fp32.ncu-rep > $out/ncu_full_fp32.txt 2>&1
 python tools/ncu_table.py $rep/full_bf16.ncu-rep > $out/ncu_full_bf16.txt 2>&1
-python tools/traffic_from_ncu.py r1 $rep/full_fp32.ncu-rep $rep/full_bf16.ncu-rep && cp profiles/r1_traffic.json $out/
+python tools/traffic_from_ncu.py $tag $rep/full_fp32.ncu-rep $rep/full_bf16.ncu-rep && cp profiles/${tag}_traffic.json $out/
 ls -la $out
