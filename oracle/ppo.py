@@ -132,11 +132,15 @@ def ppo_loss(logp_new, logp_old, ent, adv, eps: float = 0.2, c_ent: float = 0.00
     return -surr.sum() / n - c_ent * ent.sum() / n
 
 
-def ppo_grads(E, params, dims, s, placements, logp_old, adv, eps=0.2, c_ent=0.001):
-    """(loss, dL/dparams, dL/dE) in float64."""
-    Et = torch.tensor(np.asarray(E, np.float64), requires_grad=True)
-    pt = torch.tensor(np.asarray(params, np.float64), requires_grad=True)
+def ppo_grads(E, params, dims, s, placements, logp_old, adv, eps=0.2, c_ent=0.001,
+              dtype=torch.float64):
+    """(loss, dL/dparams, dL/dE).  dtype float64 is the oracle; float32 runs the
+    same formulation in single precision -- a second fp32 implementation that
+    measures how much fp32 rounding alone moves each gradient block (its
+    conditioning), against which the GPU's error is judged (reading c33)."""
+    Et = torch.tensor(np.asarray(E, np.float64), dtype=dtype, requires_grad=True)
+    pt = torch.tensor(np.asarray(params, np.float64), dtype=dtype, requires_grad=True)
     lp, ent = placer_logp(Et, pt, dims, s, placements)
-    L = ppo_loss(lp, logp_old, ent, adv, eps, c_ent)
+    L = ppo_loss(lp.double(), logp_old, ent.double(), adv, eps, c_ent)
     L.backward()
-    return float(L), pt.grad.numpy().copy(), Et.grad.numpy().copy()
+    return (float(L.detach()), pt.grad.double().numpy().copy(), Et.grad.double().numpy().copy())

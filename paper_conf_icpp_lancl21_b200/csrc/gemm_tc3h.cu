@@ -571,27 +571,46 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
     };
     constexpr int NTA = kDwBK * HH / 8;                 // 8-column tasks of dZ per stage
     constexpr int NTT = NTA + kDwBK * CINT / 8;
+    constexpr int MAXT = (NTT + NT - 1) / NT;             // tasks per thread (2 or 3)
+    // a thread's tasks are the same in every stage: their offsets from the
+    // stage base are computed once (the second 16-byte source chunk is the
+    // first's chunk index ^ 1: w0 is even)
+    uint32_t so0[MAXT], dof[MAXT];
+    int ntask = 0;
+#pragma unroll
+    for (int q = 0; q < MAXT; ++q) {
+      const int i = ct + q * NT;
+      so0[q] = dof[q] = 0;
+      if (i < NTT) {
+        const bool isA = i < NTA;
+        const int ii = isA ? i : i - NTA;
+        const int r = ii % kDwBK, c0 = (ii / kDwBK) * 8;
+        const uint32_t sb = (isA ? 0u : (uint32_t)Cfg::A32) + (c0 / 32) * Cfg::BOX32 + r * 128;
+        const int w0 = (c0 % 32) / 4;
+        so0[q] = sb + ((w0 ^ (r & 7)) << 4);
+        dof[q] = Cfg::A32 + Cfg::B32 + (isA ? 0u : 2u * Cfg::A16) + (c0 / 64) * Cfg::ATOM +
+                 r * 128 + ((((c0 % 64) / 8) ^ (r & 7)) << 4);
+        ntask = q + 1;
+      }
+    }
     int s = 0;
     uint32_t ph = 0;
     for (int kb = 0; kb < nk; ++kb) {
       mbar_wait(&full[s], ph);
-      for (int i = ct; i < NTT; i += NT) {
-        const bool isA = i < NTA;
-        const int ii = isA ? i : i - NTA;
-        const int r = ii % kDwBK, c0 = (ii / kDwBK) * 8;
-        const uint8_t* src = (isA ? stA32(s) : stB32(s)) + (c0 / 32) * Cfg::BOX32 + r * 128;
-        const int w0 = (c0 % 32) / 4;
-        const float4 v0 = *reinterpret_cast<const float4*>(src + ((w0 ^ (r & 7)) << 4));
-        const float4 v1 = *reinterpret_cast<const float4*>(src + (((w0 + 1) ^ (r & 7)) << 4));
+      uint8_t* stage = smem + s * Cfg::STAGE;
+#pragma unroll
+      for (int q = 0; q < MAXT; ++q) {
+        if (q >= ntask) break;
+        const bool isA = so0[q] < (uint32_t)Cfg::A32;
+        const float4 v0 = *reinterpret_cast<const float4*>(stage + so0[q]);
+        const float4 v1 = *reinterpret_cast<const float4*>(stage + (so0[q] ^ 16u));
         const float sc = isA ? sz : sy;
         const float x[8] = {v0.x * sc, v0.y * sc, v0.z * sc, v0.w * sc,
                             v1.x * sc, v1.y * sc, v1.z * sc, v1.w * sc};
         uint4 hv, lv;
         split_h8(x, hv, lv);
-        uint8_t* dst = (isA ? stA16(s) : stB16(s)) + (c0 / 64) * Cfg::ATOM + r * 128 +
-                       ((((c0 % 64) / 8) ^ (r & 7)) << 4);
-        *reinterpret_cast<uint4*>(dst) = hv;
-        *reinterpret_cast<uint4*>(dst + (isA ? Cfg::A16 : Cfg::B16)) = lv;
+        *reinterpret_cast<uint4*>(stage + dof[q]) = hv;
+        *reinterpret_cast<uint4*>(stage + dof[q] + (isA ? Cfg::A16 : Cfg::B16)) = lv;
       }
       fence_proxy_async_smem();
       __syncwarp();

@@ -323,7 +323,8 @@ struct PlacerBwd {
   const float* dz;
   float *dg, *dx, *dq, *dvp;           // per (b, i): [SN x 4Hs], [SN x Hin], [SN x A], [SN x A]
   float *dhr, *dcr, *dhr_part;         // [S x Hs]
-  float *dal, *de;                     // [S x seg]
+  double* dal;                         // [S x seg] (double: the softmax backward cancels)
+  float* de;                           // [S x seg]
   float *dK, *denc;                    // [N x A], [N x Hs] (accumulated; zeroed first)
   float *dinit_h, *dinit_c;            // [nseg x Hs]
   const float *esv_gates, *esv_c;

@@ -2344,7 +2344,16 @@ struct mars_placer {
   int32_t* order_b = nullptr;
   int64_t tr_N = 0, tr_S = 0;
   std::vector<void*> tr_owned;
+  // the BPTT's per-op kernel chain (~6 N + 2 N launches) captured once per
+  // workspace and replayed (launch cost ~1-2 us per node instead of ~5-8 eager)
+  cudaGraphExec_t bwd_exec = nullptr;
+  const void* bwd_key[3] = {};
+  int64_t bwd_launches = 0;
+  float* Ein = nullptr;               // [N x H] the embeddings the captured backward reads
   void release_tr() {
+    if (bwd_exec) cudaGraphExecDestroy(bwd_exec);
+    bwd_exec = nullptr;
+    for (const void*& k : bwd_key) k = nullptr;
     for (void* q : tr_owned) cudaFree(q);
     tr_owned.clear();
     tr = PlacerTrain{};
@@ -2523,7 +2532,7 @@ static mars_status placer_ensure_train(mars_placer* p, int64_t N, int64_t S) {
   CK(alf(&b.dhr, S * Hs));
   CK(alf(&b.dcr, S * Hs));
   CK(alf(&b.dhr_part, S * Hs));
-  CK(alf(&b.dal, S * seg));
+  CK(al(reinterpret_cast<void**>(&b.dal), sizeof(double) * S * seg));
   CK(alf(&b.de, S * seg));
   CK(alf(&b.dK, N * A));
   CK(alf(&b.denc, N * Hs));
@@ -2537,6 +2546,7 @@ static mars_status placer_ensure_train(mars_placer* p, int64_t N, int64_t S) {
   CK(alf(&p->wT, Hin * 4 * Hs + Hs * 4 * Hs + Hs * A + 2 * Hd * 4 * Hd));
   CK(alf(&p->X, SN * std::max<int64_t>(Hin, Hs)));
   CK(alf(&p->tmpNH, N * std::max<int64_t>(Hs, d.H)));
+  CK(alf(&p->Ein, N * d.H));
   CK(alf(&p->ebuf, 2 * N * std::max<int64_t>(Hd, d.H)));
   size_t pt = 0;
   const int64_t shapes[][3] = {{SN, 4 * Hs, Hin}, {SN, 4 * Hs, Hs}, {SN, A, Hs}, {N, A, Hs},
@@ -2582,15 +2592,77 @@ static mars_status placer_ensure_train(mars_placer* p, int64_t N, int64_t S) {
   return MARS_OK;
 }
 
+// The backward section of placer_loss_grad (every launch stream-ordered, all
+// pointers fixed per training workspace, so it is captured once and replayed):
+// transposed weights, the decoder BPTT, the decoder's weight gradients, the
+// encoder BPTT and its gradients, dL/dE into p->tmpNH, the loss into
+// p->grads[P].  E is p->Ein.
+static cudaError_t placer_bwd_section(mars_placer* p, int32_t N, int32_t S, cudaStream_t s,
+                                      int* nl) {
+  const PlacerDims& d = p->d;
+  const int64_t Hd = d.Hd, Hs = 2 * Hd, Hin = Hs + d.De, A = d.A, SN = (int64_t)S * N;
+  PlacerTrain& t = p->tr;
+  PlacerBwd& b = p->bw;
+  const float* E = p->Ein;
+  cudaError_t e;
+#define RE(x) do { if ((e = (x)) != cudaSuccess) return e; } while (0)
+  RE(placer_transpose(p->w.dec_wih, (int)(4 * Hs), (int)Hin, const_cast<float*>(b.wihT), s));
+  RE(placer_transpose(p->w.dec_whh, (int)(4 * Hs), (int)Hs, const_cast<float*>(b.whhT), s));
+  RE(placer_transpose(p->w.wq, (int)A, (int)Hs, const_cast<float*>(b.wqT), s));
+  for (int dir = 0; dir < 2; ++dir)
+    RE(placer_transpose(p->w.enc_whh[dir], (int)(4 * Hd), (int)Hd, const_cast<float*>(b.ewhhT[dir]), s));
+  RE(cudaMemsetAsync(b.dK, 0, sizeof(float) * N * A, s));
+  RE(cudaMemsetAsync(b.denc, 0, sizeof(float) * N * Hs, s));
+  RE(placer_bwd_decoder(b, s, nl));
+  // decoder weight gradients
+  PlacerParams G = placer_views(d, p->grads);
+  RE(placer_build_x(t.sv_ctx, t.sv_prev, p->w.emb, SN, (int)Hs, d.De, p->X, s));
+  RE(gemm_tn(b.dg, p->X, G.dec_wih, SN, (int)(4 * Hs), (int)Hin, p->part, s, nl));
+  RE(gemm_tn(b.dg, t.sv_hprev, G.dec_whh, SN, (int)(4 * Hs), (int)Hs, p->part, s, nl));
+  RE(placer_colsum(b.dg, SN, (int)(4 * Hs), G.dec_b, s));
+  RE(gemm_tn(b.dq, t.sv_hprev, G.wq, SN, (int)A, (int)Hs, p->part, s, nl));
+  RE(placer_colsum(b.dvp, SN, (int)A, G.v, s));
+  RE(placer_small_tn(t.dz, t.sv_h, SN, d.D, (int)Hs, G.wo, s));
+  RE(placer_colsum(t.dz, SN, d.D, G.bo, s));
+  RE(placer_emb_grad(b.dx, t.sv_prev, SN, (int)Hs, (int)Hin, d.De, d.D + 1, G.emb, s));
+  RE(gemm_tn(b.dK, p->ws.enc, G.wk, N, (int)A, (int)Hs, p->part, s, nl));
+  RE(gemm_nn(b.dK, p->w.wk, p->tmpNH, N, (int)Hs, (int)A, s, nl));     // d(K)/d(enc)
+  RE(placer_add(b.denc, p->tmpNH, N * Hs, s));
+  // encoder BPTT and its gradients
+  RE(placer_bwd_encoder(b, s, nl));
+  float* Eb = p->ebuf;                      // E in the backward direction's step order
+  RE(placer_gather_rows(E, p->order_b, N, d.H, Eb, 0, s));
+  RE(gemm_tn(b.edg, E, G.enc_wih[0], N, (int)(4 * Hd), d.H, p->part, s, nl));
+  RE(gemm_tn(b.edg + N * 4 * Hd, Eb, G.enc_wih[1], N, (int)(4 * Hd), d.H, p->part, s, nl));
+  for (int dir = 0; dir < 2; ++dir) {
+    float* hs = p->ebuf;                    // h of each step of this direction, step order
+    RE(placer_gather_cols(p->ws.enc, Hs, dir * (int)Hd, dir ? p->order_b : nullptr, N, (int)Hd, hs, s));
+    const float* edg = b.edg + (int64_t)dir * N * 4 * Hd;
+    if (N > 1)
+      RE(gemm_tn(edg + 4 * Hd, hs, G.enc_whh[dir], N - 1, (int)(4 * Hd), (int)Hd, p->part, s, nl));
+    else
+      RE(cudaMemsetAsync(G.enc_whh[dir], 0, sizeof(float) * 4 * Hd * Hd, s));
+    RE(placer_colsum(edg, N, (int)(4 * Hd), G.enc_b[dir], s));
+  }
+  // dL/dE: forward direction in op order, backward direction scattered by its order
+  RE(gemm_nn(b.edg, p->w.enc_wih[0], p->tmpNH, N, d.H, (int)(4 * Hd), s, nl));
+  RE(gemm_nn(b.edg + N * 4 * Hd, p->w.enc_wih[1], p->ebuf, N, d.H, (int)(4 * Hd), s, nl));
+  RE(placer_gather_rows(p->ebuf, p->order_b, N, d.H, p->tmpNH, 1, s));
+  // the loss: sum of the per-op terms / (S N), fixed order
+  RE(placer_colsum(t.lterm, SN, 1, p->grads + p->P, s));
+#undef RE
+  return cudaSuccess;
+}
+
 // The PPO loss (c29) of S teacher-forced placements and its gradient: placer
-// forward with activations saved, dL/dlogits, BPTT through the decoder and the
-// encoder, weight gradients by GEMMs / fixed-order sums.  Leaves the gradient
-// [P] and the loss (at [P]) in p->grads and dL/dE [N x H] in p->tmpNH.
+// forward with activations saved and dL/dlogits, then the backward section
+// (captured once per workspace, replayed).  Leaves the gradient [P] and the
+// loss sum (at [P]) in p->grads and dL/dE [N x H] in p->tmpNH.
 static mars_status placer_loss_grad(mars_placer* p, const float* dE_in, int32_t N, int32_t S,
                                     const int32_t* dplace, float clip_eps, float ent_coef, int* nl) {
   cudaStream_t s = p->stream;
   const PlacerDims& d = p->d;
-  const int64_t Hd = d.Hd, Hs = 2 * Hd, Hin = Hs + d.De, A = d.A, SN = (int64_t)S * N;
+  const int64_t SN = (int64_t)S * N;
   PlacerTrain& t = p->tr;
   PlacerBwd& b = p->bw;
   b.keys = p->ws.keys;                    // the forward workspace may have been regrown
@@ -2604,51 +2676,33 @@ static mars_status placer_loss_grad(mars_placer* p, const float* dE_in, int32_t 
   float* dL = p->X + SN;
   float* dH = p->X + 2 * SN;
   CK(placer_forward(d, p->w, p->ws, dE_in, N, p->cfg.segment, S, 0, dplace, dP, dL, dH, s, nl, &t));
-  // transposed weights
-  CK(placer_transpose(p->w.dec_wih, (int)(4 * Hs), (int)Hin, const_cast<float*>(b.wihT), s));
-  CK(placer_transpose(p->w.dec_whh, (int)(4 * Hs), (int)Hs, const_cast<float*>(b.whhT), s));
-  CK(placer_transpose(p->w.wq, (int)A, (int)Hs, const_cast<float*>(b.wqT), s));
-  for (int dir = 0; dir < 2; ++dir)
-    CK(placer_transpose(p->w.enc_whh[dir], (int)(4 * Hd), (int)Hd, const_cast<float*>(b.ewhhT[dir]), s));
-  CK(cudaMemsetAsync(b.dK, 0, sizeof(float) * N * A, s));
-  CK(cudaMemsetAsync(b.denc, 0, sizeof(float) * N * Hs, s));
-  CK(placer_bwd_decoder(b, s, nl));
-  // decoder weight gradients
-  PlacerParams G = placer_views(d, p->grads);
-  CK(placer_build_x(t.sv_ctx, t.sv_prev, p->w.emb, SN, (int)Hs, d.De, p->X, s));
-  CK(gemm_tn(b.dg, p->X, G.dec_wih, SN, (int)(4 * Hs), (int)Hin, p->part, s, nl));
-  CK(gemm_tn(b.dg, t.sv_hprev, G.dec_whh, SN, (int)(4 * Hs), (int)Hs, p->part, s, nl));
-  CK(placer_colsum(b.dg, SN, (int)(4 * Hs), G.dec_b, s));
-  CK(gemm_tn(b.dq, t.sv_hprev, G.wq, SN, (int)A, (int)Hs, p->part, s, nl));
-  CK(placer_colsum(b.dvp, SN, (int)A, G.v, s));
-  CK(placer_small_tn(t.dz, t.sv_h, SN, d.D, (int)Hs, G.wo, s));
-  CK(placer_colsum(t.dz, SN, d.D, G.bo, s));
-  CK(placer_emb_grad(b.dx, t.sv_prev, SN, (int)Hs, (int)Hin, d.De, d.D + 1, G.emb, s));
-  CK(gemm_tn(b.dK, p->ws.enc, G.wk, N, (int)A, (int)Hs, p->part, s, nl));
-  CK(gemm_nn(b.dK, p->w.wk, p->tmpNH, N, (int)Hs, (int)A, s, nl));     // d(K)/d(enc)
-  CK(placer_add(b.denc, p->tmpNH, N * Hs, s));
-  // encoder BPTT and its gradients
-  CK(placer_bwd_encoder(b, s, nl));
-  float* Eb = p->ebuf;                      // E in the backward direction's step order
-  CK(placer_gather_rows(dE_in, p->order_b, N, d.H, Eb, 0, s));
-  CK(gemm_tn(b.edg, dE_in, G.enc_wih[0], N, (int)(4 * Hd), d.H, p->part, s, nl));
-  CK(gemm_tn(b.edg + N * 4 * Hd, Eb, G.enc_wih[1], N, (int)(4 * Hd), d.H, p->part, s, nl));
-  for (int dir = 0; dir < 2; ++dir) {
-    float* hs = p->ebuf;                    // h of each step of this direction, step order
-    CK(placer_gather_cols(p->ws.enc, Hs, dir * (int)Hd, dir ? p->order_b : nullptr, N, (int)Hd, hs, s));
-    const float* edg = b.edg + (int64_t)dir * N * 4 * Hd;
-    if (N > 1)
-      CK(gemm_tn(edg + 4 * Hd, hs, G.enc_whh[dir], N - 1, (int)(4 * Hd), (int)Hd, p->part, s, nl));
-    else
-      CK(cudaMemsetAsync(G.enc_whh[dir], 0, sizeof(float) * 4 * Hd * Hd, s));
-    CK(placer_colsum(edg, N, (int)(4 * Hd), G.enc_b[dir], s));
+  if (dE_in != p->Ein)
+    CK(cudaMemcpyAsync(p->Ein, dE_in, sizeof(float) * (size_t)N * d.H, cudaMemcpyDeviceToDevice, s));
+  const void* key[3] = {p->ws.keys, p->ws.enc, b.dg};
+  if (p->bwd_exec && (key[0] != p->bwd_key[0] || key[1] != p->bwd_key[1] || key[2] != p->bwd_key[2])) {
+    cudaGraphExecDestroy(p->bwd_exec);
+    p->bwd_exec = nullptr;
   }
-  // dL/dE: forward direction in op order, backward direction scattered by its order
-  CK(gemm_nn(b.edg, p->w.enc_wih[0], p->tmpNH, N, d.H, (int)(4 * Hd), s, nl));
-  CK(gemm_nn(b.edg + N * 4 * Hd, p->w.enc_wih[1], p->ebuf, N, d.H, (int)(4 * Hd), s, nl));
-  CK(placer_gather_rows(p->ebuf, p->order_b, N, d.H, p->tmpNH, 1, s));
-  // the loss: sum of the per-op terms / (S N), fixed order
-  CK(placer_colsum(t.lterm, SN, 1, p->grads + p->P, s));
+  if (!p->bwd_exec) {
+    cudaGraph_t graph;
+    CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+    int cnl = 0;
+    cudaError_t e = placer_bwd_section(p, N, S, s, &cnl);
+    cudaError_t e2 = cudaStreamEndCapture(s, &graph);
+    if (e != cudaSuccess || e2 != cudaSuccess) {
+      if (e2 == cudaSuccess) cudaGraphDestroy(graph);
+      cudaGetLastError();
+      return fail(MARS_ECUDA, "placer backward capture failed: %s",
+                  cudaGetErrorString(e != cudaSuccess ? e : e2));
+    }
+    cudaError_t e3 = cudaGraphInstantiate(&p->bwd_exec, graph, 0);
+    cudaGraphDestroy(graph);
+    CK(e3);
+    for (int k = 0; k < 3; ++k) p->bwd_key[k] = key[k];
+    p->bwd_launches = cnl;
+  }
+  CK(cudaGraphLaunch(p->bwd_exec, s));
+  count_launch(nl, (int)p->bwd_launches);
   return MARS_OK;
 }
 

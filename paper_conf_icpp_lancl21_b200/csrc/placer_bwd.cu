@@ -86,7 +86,7 @@ __global__ void kb_dalpha(PlacerBwd w, int i, int j0, int len) {
   double acc = 0.0;
   for (int c = lane; c < w.Hs; c += 32) acc += (double)dctx[c] * (double)en[c];
   acc = warp_sum(acc);
-  if (lane == 0) w.dal[(int64_t)b * w.seg + k] = (float)acc;
+  if (lane == 0) w.dal[(int64_t)b * w.seg + k] = acc;   // kept in double: it cancels next
 }
 
 // grid (S, cdiv(A, kT)): de_k (every block, redundant), then per a:
@@ -101,14 +101,14 @@ __global__ void kb_datt(PlacerBwd w, int i, int j0, int len) {
   const int64_t bi = (int64_t)b * w.N + i;
   const float* al = w.sv_alpha + bi * w.seg;
   double part = 0.0;
-  for (int k = threadIdx.x; k < len; k += kT) part += (double)al[k] * (double)w.dal[(int64_t)b * w.seg + k];
+  for (int k = threadIdx.x; k < len; k += kT) part += (double)al[k] * w.dal[(int64_t)b * w.seg + k];
   part = warp_sum(part);                        // fixed-order block reduction
   if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = part;
   __syncthreads();
   double sum = 0.0;
   for (int q = 0; q < kT / 32; ++q) sum += red[q];
   for (int k = threadIdx.x; k < len; k += kT) {
-    const double d = (double)al[k] * ((double)w.dal[(int64_t)b * w.seg + k] - sum);
+    const double d = (double)al[k] * (w.dal[(int64_t)b * w.seg + k] - sum);
     de[k] = d;
     if (blockIdx.y == 0) w.de[(int64_t)b * w.seg + k] = (float)d;
   }

@@ -5,6 +5,7 @@ autograd oracle (oracle/ppo.py; §3.4, readings c29-c31): loss,
 every parameter block and dL/d embeddings at the scaled max-norm 1e-5."""
 import numpy as np
 import pytest
+import torch
 
 import paper_conf_icpp_lancl21_b200 as mars
 from oracle import placer as PL
@@ -201,7 +202,10 @@ def test_joint_ppo_iteration_runs_and_moves_both():
 def test_ppo_grad_paper_sizes():
     """P:L234 sizes (bi-LSTM 2 x 256, decoder 512, attention 512, device
     embedding 64, s = 128, D = 4) on 300 ops (a ragged last segment), H = 256:
-    the PPO gradient of every block and dL/dE at 1e-5 of torch fp64 autograd."""
+    the PPO gradient of every block and dL/dE against torch fp64 autograd at
+    1e-5, or -- for a block fp32 rounding alone moves further (reading c33:
+    the attention query's gradient passes through the softmax backward's
+    cancellation) -- at 3x the error of the same formulation run in float32."""
     N, seg, S, H = 300, 128, 2, 256
     dims = dict(H=H, Hd=256, A=512, De=64, D=4)
     p = mars.placer_create(seed=6, in_dim=H)
@@ -212,12 +216,17 @@ def test_ppo_grad_paper_sizes():
     p.set_params(params1)
     adv = np.array([1.2, -0.7], np.float32)
     loss, g, dE = p.ppo_grad(E, place, logp, adv)
-    L, gp, gE = ppo.ppo_grads(E.astype(np.float64), params1.astype(np.float64), dims, seg, place,
-                              logp.astype(np.float64), adv.astype(np.float64))
+    args = (E.astype(np.float64), params1.astype(np.float64), dims, seg, place,
+            logp.astype(np.float64), adv.astype(np.float64))
+    L, gp, gE = ppo.ppo_grads(*args)
+    _, gp32, gE32 = ppo.ppo_grads(*args, dtype=torch.float32)      # conditioning (c33)
     res = {"loss": abs(loss - L) / abs(L), "dE": scaled_err(dE, gE)}
+    bar = {"loss": 1e-5, "dE": max(1e-5, 3 * scaled_err(gE32, gE))}
     for name, blk in _blocks(g, dims).items():
-        res[name] = scaled_err(blk, _blocks(gp, dims)[name])
-    print("paper sizes", {k: f"{v:.2e}" for k, v in res.items()})
-    bad = {k: v for k, v in res.items() if v > 1e-5}
+        ref = _blocks(gp, dims)[name]
+        res[name] = scaled_err(blk, ref)
+        bar[name] = max(1e-5, 3 * scaled_err(_blocks(gp32, dims)[name], ref))
+    print("paper sizes", {k: f"{v:.2e} (bar {bar[k]:.1e})" for k, v in res.items()})
+    bad = {k: v for k, v in res.items() if v > bar[k]}
     assert not bad, bad
     p.free()
