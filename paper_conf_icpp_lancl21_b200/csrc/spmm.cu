@@ -38,10 +38,14 @@ constexpr int kSpmmThreads = 32;   // one warp per block: a slow (hub) row holds
 constexpr int kU = MARS_SPMM_KU;   // neighbours whose gathers are in flight together
 
 // C in {16, 32, 64, 128, 256} (mars.h restricts F and H to these widths).
+#ifndef MARS_SPMM_LMAX_BF16
+#define MARS_SPMM_LMAX_BF16 32     // lanes per bf16 row at most (A/B: 16 = two rows per warp)
+#endif
 template <int C, typename T>
 struct SpmmShape {
   static constexpr int V = Vec<T>::N;                     // elements per 16-byte load
-  static constexpr int L = (C / V) < 32 ? (C / V) : 32;   // lanes per row
+  static constexpr int LMAX = std::is_same<T, float>::value ? 32 : MARS_SPMM_LMAX_BF16;
+  static constexpr int L = (C / V) < LMAX ? (C / V) : LMAX;   // lanes per row
   static constexpr int RPW = 32 / L;                      // rows per warp
   static constexpr int NT = C / (V * L);                  // vectors per lane per branch
   static constexpr int RPB = RPW * (kSpmmThreads / 32);   // rows per block

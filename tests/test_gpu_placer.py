@@ -103,3 +103,29 @@ def test_placer_gnmt_graph():
     """A GNMT-4 op graph (~12k ops, 93 segments) at paper sizes, S = 2."""
     E = _embeddings("gnmt")
     _check(E, 2, 8, 41)
+
+
+def test_placer_and_ppo_argument_validation():
+    with pytest.raises(mars.MarsError):
+        mars.placer_create(enc_hidden=48)                 # 64, 128 or 256 only
+    with pytest.raises(mars.MarsError):
+        mars.placer_create(num_devices=1)
+    p = mars.placer_create(in_dim=32, enc_hidden=64, attn_dim=128, dev_embed=8, num_devices=3,
+                           segment=8)
+    E = np.zeros((10, 32), np.float32)
+    with pytest.raises(mars.MarsError):
+        p.sample(E, 33, 0)                                # 1..32 samples
+    with pytest.raises(mars.MarsError):
+        p.sample(E, 2, 0, forced=np.full((2, 10), 3))     # device outside [0, D)
+    with pytest.raises(mars.MarsError):
+        mars.ppo_create(p, samples_per_policy=3, policies=1, minibatches=2)   # 3 % 2 != 0
+    enc = mars.dgi_create(in_dim=16, hidden_dim=64, seed=1)
+    with pytest.raises(mars.MarsError):
+        mars.ppo_create(p, enc)                           # encoder H != placer in_dim
+    o = mars.ppo_create(p, samples_per_policy=2, policies=1, minibatches=1, epochs=1)
+    g = mars.graph_load([SG.tiny(0)])
+    with pytest.raises(mars.MarsError):
+        o.iteration_joint(g, SG.tiny(0))                  # created without an encoder
+    h = p.handle
+    p.free()
+    assert mars.mars.lib().mars_placer_get_params(h, None) == mars.mars.MARS_ESTATE  # tag poisoned
