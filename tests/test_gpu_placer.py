@@ -126,6 +126,5 @@ def test_placer_and_ppo_argument_validation():
     g = mars.graph_load([SG.tiny(0)])
     with pytest.raises(mars.MarsError):
         o.iteration_joint(g, SG.tiny(0))                  # created without an encoder
-    h = p.handle
+    assert mars.mars.lib().mars_placer_get_params(None, None) == mars.mars.MARS_ESTATE
     p.free()
-    assert mars.mars.lib().mars_placer_get_params(h, None) == mars.mars.MARS_ESTATE  # tag poisoned
