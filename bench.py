@@ -255,7 +255,7 @@ def run_mine(args):
     b = args.graphs_per_gpu
     gen, _, _, _, desc = WORKLOADS[args.workload]
     sharded = args.workload == "1m" and world > 1
-    mine = None
+    mine = [0]
     if args.workload == "1m":
         graphs = [SG.make("1m", 0)]           # ~7 s to generate; one graph for the whole job
     else:

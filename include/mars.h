@@ -156,11 +156,49 @@ MARS_API mars_status mars_dgi_set_gemm_impl(mars_dgi* m, int32_t impl);
 /* Enables (1) / disables (0) CUDA-Graph capture of the step (default 1). */
 MARS_API mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable);
 
+/* NEXT-4 contrastive variants ("there are many choices of the
+ * corruption function, readout function and loss function in contrastive
+ * learning ... other contrastive learning methods should also work"; the
+ * GraphSAGE encoder of [33]).  Readings c34-c37:
+ *   num_neg     K >= 1 corruption samples per graph, all scored against ONE
+ *               positive branch (c34): L_g = 1/(2N)[Σ softplus(-l_i) + (1/K)
+ *               Σ_k Σ softplus(l~_i^k)]; sample k of graph g draws pair index
+ *               pair_base + pair_off(g) K + k (k = 0..K-1), so K samples of a
+ *               graph reproduce mars_step on K consecutive copies of it (c20)
+ *               while computing the positive branch once.  Activations hold
+ *               K + 1 blocks of ΣN rows (rounded up to an even count).
+ *   corruption  MARS_CORRUPT_PERMUTE: X~ = X[pi] (DGI, Eq. 2, default);
+ *               MARS_CORRUPT_MASK: X~ = X ⊙ Bernoulli keep mask, each feature
+ *               zeroed with probability mask_rate (counter-based, c35).
+ *   readout     MARS_READOUT_SIGMOID_MEAN: s = sig(mean H3) (Eq. 4, default);
+ *               MARS_READOUT_MEAN: s = mean H3 (c36).
+ *   aggregator  MARS_AGG_GCN: Â = D^-1/2 (A v Aᵀ + I) D^-1/2 (Eq. 1, default);
+ *               MARS_AGG_SAGE_GCN: Â = D^-1 (A v Aᵀ + I), the GraphSAGE mean
+ *               aggregator over the node and its neighbours (c37); the
+ *               backward uses Âᵀ.  mars_encode / mars_dgi_encoder_vjp follow it.
+ * The default {1, PERMUTE, 0, SIGMOID_MEAN, GCN} is the paper's DGI step. */
+enum { MARS_CORRUPT_PERMUTE = 0, MARS_CORRUPT_MASK = 1 };
+enum { MARS_READOUT_SIGMOID_MEAN = 0, MARS_READOUT_MEAN = 1 };
+enum { MARS_AGG_GCN = 0, MARS_AGG_SAGE_GCN = 1 };
+typedef struct {
+  int32_t num_neg;            /* K in [1, 64]                                      */
+  int32_t corruption;         /* MARS_CORRUPT_*                                    */
+  float mask_rate;            /* MARS_CORRUPT_MASK: in [0, 1]                      */
+  int32_t readout;            /* MARS_READOUT_*                                    */
+  int32_t aggregator;         /* MARS_AGG_*                                        */
+} mars_contrastive;
+/* Sets the variant for later steps / encodes (the workspace and captured steps
+ * are rebuilt on the next call).  EINVAL on an out-of-range field; ESTATE on a
+ * row-shard-attached model (the sharded step runs the default only). */
+MARS_API mars_status mars_dgi_set_contrastive(mars_dgi* m, const mars_contrastive* c);
+MARS_API mars_status mars_dgi_get_contrastive(const mars_dgi* m, mars_contrastive* c);
+
 /* Optional outputs of a step (host pointers; NULL = not requested). */
 typedef struct {
   float* loss;                /* [1]  L averaged over the GLOBAL batch (c15)    */
   float* grads;               /* [P]  global-batch mean gradient BEFORE Adam    */
-  int32_t* perms;             /* [ΣN] corruption permutations, LOCAL indices    */
+  int32_t* perms;             /* [K x ΣN] corruption permutations (sample-major),
+                                 LOCAL indices; EINVAL with MARS_CORRUPT_MASK  */
 } mars_step_out;
 
 /* One DGI step over every graph of `g` (each graph = one (graph, sample) pair,

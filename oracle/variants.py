@@ -1,0 +1,159 @@
+"""CPU oracle of the NEXT-4 contrastive variants ("there
+are many choices of the corruption function, readout function and loss
+function ... other contrastive learning methods should also work"; GraphSAGE
+in [33]) -- TEST INFRASTRUCTURE ONLY, like the rest of oracle/: only
+tests/ may import it.
+
+Plain PyTorch CPU ops in float64 with autograd (the chain rule as a library
+primitive, as in oracle/ppo.py), one graph at a time, step by step in the
+paper's order -- Eq. 1 encoder, Eq. 2 corruption, Eq. 4 readout, Eq. 5
+discriminator, Eq. 6 loss -- with the variant's choices.  Readings
+(DESIGN.md §3):
+
+  c34  K corruption samples share one positive branch: L_g = 1/(2N)[Σ_i
+       softplus(-l_i) + (1/K) Σ_k Σ_i softplus(l~_i^k)], L = (1/B) Σ_g L_g;
+       sample k of graph g uses pair index pair_base + pair_off[g] K + k.
+  c35  feature masking: X~ = X ⊙ keep, keep[i][f] iff u >= rate with u =
+       (sm64(sm64(key ^ 0x6D61736B) ^ (i F + f)) >> 40) 2^-24 and key =
+       sm64(sm64(sm64(seed) ^ step) ^ pair) (the c12 sample key).
+  c36  mean readout: s = (1/N) Σ_i h_i (no sigmoid).
+  c37  SAGE-GCN aggregation: Â = D^-1 (A v Aᵀ + I), D the row sums (the
+       GraphSAGE mean aggregator over the node and its neighbours).
+
+The corruption permutations are oracle.perm's (the C oracle, c12).  Parity
+pins: tests/test_oracle_variants.py (the default variant against the C
+oracle's step; K samples against the C oracle on K copies; masking rates 0 and
+1 in closed form; the readouts and aggregators against the C oracle's encoder
+plus a hand-written numpy head, brute-force loops, and finite differences).
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import perm as _perm
+
+M64 = (1 << 64) - 1
+
+
+def _sm64(z: int) -> int:
+    z = (z + 0x9E3779B97F4A7C15) & M64
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M64
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M64
+    return z ^ (z >> 31)
+
+
+def _sm64_np(z):
+    z = (z + np.uint64(0x9E3779B97F4A7C15)).astype(np.uint64)
+    z = ((z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)).astype(np.uint64)
+    z = ((z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)).astype(np.uint64)
+    return z ^ (z >> np.uint64(31))
+
+
+def mask_keep(seed: int, step: int, pair: int, N: int, F: int, rate: float) -> np.ndarray:
+    """c35: the [N x F] keep mask of one (graph, sample) pair.  rate is taken as
+    the float32 the ABI stores, compared in double."""
+    key = _sm64(_sm64(_sm64(seed & M64) ^ (step & M64)) ^ (pair & M64))
+    km = np.uint64(_sm64(key ^ 0x6D61736B))
+    e = np.arange(N * F, dtype=np.uint64)
+    u = (_sm64_np(km ^ e) >> np.uint64(40)).astype(np.float64) * (1.0 / 16777216.0)
+    return (u >= float(np.float32(rate))).reshape(N, F)
+
+
+def adjacency(g) -> np.ndarray:
+    """Â = A v Aᵀ + I, binary (Eq. 1; readings c1-c3)."""
+    N = g.num_nodes
+    A = np.zeros((N, N))
+    for u in range(N):
+        for e in range(int(g.indptr[u]), int(g.indptr[u + 1])):
+            v = int(g.indices[e])
+            A[u, v] = A[v, u] = 1.0
+    np.fill_diagonal(A, 1.0)
+    return A
+
+
+def normalise(A: np.ndarray, aggregator: str) -> np.ndarray:
+    d = A.sum(1)
+    if aggregator == "gcn":          # D^-1/2 Â D^-1/2 (Eq. 1)
+        r = 1.0 / np.sqrt(d)
+        return r[:, None] * A * r[None, :]
+    if aggregator == "sage_gcn":     # D^-1 Â (c37)
+        return A / d[:, None]
+    raise ValueError(aggregator)
+
+
+def unpack(p, F: int, H: int):
+    o = 0
+    out = []
+    for n, shp in ((F * H, (F, H)), (H * H, (H, H)), (H * H, (H, H)), (H * H, (H, H))):
+        out.append(p[o:o + n].view(*shp))
+        o += n
+    out.append(p[o:o + 3])
+    return out          # W1, W2, W3, M, alpha
+
+
+def encoder(An, X, W, alpha):
+    """Eq. 1 x 3 with PReLU (c10)."""
+    h = X
+    for l in range(3):
+        h = torch.nn.functional.prelu(An @ (h @ W[l]), alpha[l:l + 1])
+    return h
+
+
+def corrupted(g, X, seed, step, pair, corruption, mask_rate):
+    N, F = X.shape
+    if corruption == "permute":      # Eq. 2, c12
+        pi = _perm(seed, step, pair, N).astype(np.int64)
+        return X[torch.from_numpy(pi)]
+    if corruption == "mask":         # c35
+        return X * torch.from_numpy(mask_keep(seed, step, pair, N, F, mask_rate).astype(np.float64))
+    raise ValueError(corruption)
+
+
+def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: int = 0,
+               B: float | None = None, num_neg: int = 1, corruption: str = "permute",
+               mask_rate: float = 0.0, readout: str = "sigmoid_mean", aggregator: str = "gcn",
+               pair_off=None, sparse: bool = False):
+    """(loss, dL/dparams) of one step over a graph set (c34-c37).  B = number of
+    graphs the loss is averaged over (default: len(graphs)); pair_off[g]
+    defaults to g.  sparse: Â as a torch sparse matrix (larger graphs)."""
+    p = torch.tensor(np.asarray(params, np.float64), requires_grad=True)
+    W1, W2, W3, M, al = unpack(p, F, H)
+    W = (W1, W2, W3)
+    B = float(len(graphs) if B is None else B)
+    K = int(num_neg)
+    sp = torch.nn.functional.softplus
+    loss = torch.zeros((), dtype=torch.float64)
+    for gi, g in enumerate(graphs):
+        An_np = normalise(adjacency(g), aggregator)
+        An = torch.from_numpy(An_np)
+        if sparse:
+            An = An.to_sparse()
+        X = torch.tensor(np.asarray(g.features, np.float64))
+        N = g.num_nodes
+        Hp = encoder(An, X, W, al)
+        m = Hp.mean(0)                                   # Eq. 4
+        s = torch.sigmoid(m) if readout == "sigmoid_mean" else m
+        if readout not in ("sigmoid_mean", "mean"):
+            raise ValueError(readout)
+        v = M @ s                                        # Eq. 5: l_i = h_iᵀ M s
+        pos = sp(-(Hp @ v)).sum()
+        neg = torch.zeros((), dtype=torch.float64)
+        po = gi if pair_off is None else int(pair_off[gi])
+        for k in range(K):
+            Xt = corrupted(g, X, seed, step, pair_base + po * K + k, corruption, mask_rate)
+            neg = neg + sp(encoder(An, Xt, W, al) @ v).sum()
+        loss = loss + (pos + neg / K) / (2.0 * N) / B    # Eq. 6 with c34
+    loss.backward()
+    return float(loss.detach()), p.grad.numpy().copy()
+
+
+def encode(graphs, params, F: int, H: int, aggregator: str = "gcn"):
+    """a15 under the variant's aggregator: H3 of every node, stacked."""
+    p = torch.tensor(np.asarray(params, np.float64))
+    W1, W2, W3, _, al = unpack(p, F, H)
+    out = []
+    for g in graphs:
+        An = torch.from_numpy(normalise(adjacency(g), aggregator))
+        out.append(encoder(An, torch.tensor(np.asarray(g.features, np.float64)), (W1, W2, W3), al))
+    return torch.cat(out).numpy()

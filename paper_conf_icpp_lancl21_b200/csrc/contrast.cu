@@ -1,0 +1,118 @@
+// NEXT-4 contrastive variants ("there are many choices of the corruption
+// function, readout function and loss function ... other contrastive learning
+// methods should also work"; GraphSAGE in [33]).  Readings
+// c34-c37 in DESIGN.md §3:
+//   c34  K corruption samples per graph share ONE positive branch: the stacked
+//        activations hold [pos; neg_1; ...; neg_K (; zero pad to an even block
+//        count)], sample k of graph g draws pair index pair_base + pair_off[g] K
+//        + (k - 1) -- the same permutations as K consecutive copies of the graph
+//        in the batch API (c20), so both formulations give the same loss.
+//   c35  feature-masking corruption: X~[i][f] = X[i][f] keep(i, f), keep iff
+//        u >= rate, u = (sm64(sm64(k ^ 0x6D61736B) ^ (i F + f)) >> 40) 2^-24,
+//        k the sample's key sm64(sm64(sm64(seed) ^ step) ^ pair) (c12).
+//   c37  SAGE-GCN aggregation: Â = D^-1 (A v Aᵀ + I) (row mean over the
+//        neighbourhood with the node itself); the backward uses Âᵀ, the same
+//        pattern with 1/deg of the column.
+// The corrupted inputs are materialised (one pass over X per block) and layer
+// 1 aggregates the stacked blocks like layers 2-3 (PReLU slope 1 = identity).
+#include "common.cuh"
+#include "internal.cuh"
+
+namespace mars {
+namespace {
+
+__global__ void k_pair_off_k(const int64_t* __restrict__ pair_off, int32_t G, int32_t K,
+                             int64_t* __restrict__ out) {
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= (int64_t)G * K) return;
+  const int32_t k = (int32_t)(t / G), g = (int32_t)(t % G);
+  out[t] = pair_off[g] * K + k;
+}
+
+// one thread per 4 consecutive features of one row of Xs
+__global__ void k_corrupt(const float* __restrict__ X, const int32_t* __restrict__ node_graph,
+                          const int32_t* __restrict__ node_off, int32_t Nt, int32_t G, int32_t F,
+                          int32_t K, int32_t nb, int32_t corruption, double rate, uint64_t seed,
+                          const StepParams* __restrict__ sp, const int64_t* __restrict__ pair_off_k,
+                          const int32_t* __restrict__ perms, float* __restrict__ Xs) {
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int32_t Fq = F / 4;
+  if (t >= (int64_t)nb * Nt * Fq) return;
+  const int64_t r = t / Fq;
+  const int32_t f0 = (int32_t)(t % Fq) * 4;
+  const int32_t b = (int32_t)(r / Nt), i = (int32_t)(r % Nt);
+  float4 o = make_float4(0.f, 0.f, 0.f, 0.f);
+  if (b == 0) {
+    o = *reinterpret_cast<const float4*>(X + (int64_t)i * F + f0);
+  } else if (b <= K) {
+    if (corruption == 0) {
+      const int32_t src = perms[(int64_t)(b - 1) * Nt + i];
+      o = *reinterpret_cast<const float4*>(X + (int64_t)src * F + f0);
+    } else {
+      const int32_t g = node_graph[i];
+      const uint64_t pair = (uint64_t)(sp->pair_base + pair_off_k[(int64_t)(b - 1) * G + g]);
+      const uint64_t kg = sm64(sm64(sm64(seed) ^ sp->step_index) ^ pair);
+      const uint64_t km = sm64(kg ^ 0x6D61736BULL);
+      const uint64_t e0 = (uint64_t)(i - node_off[g]) * (uint64_t)F + (uint64_t)f0;
+      const float4 x = *reinterpret_cast<const float4*>(X + (int64_t)i * F + f0);
+      const float xv[4] = {x.x, x.y, x.z, x.w};
+      float ov[4];
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        const double u = (double)(sm64(km ^ (e0 + c)) >> 40) * (1.0 / 16777216.0);
+        ov[c] = u >= rate ? xv[c] : 0.f;
+      }
+      o = make_float4(ov[0], ov[1], ov[2], ov[3]);
+    }
+  }
+  *reinterpret_cast<float4*>(Xs + r * F + f0) = o;
+}
+
+__global__ void k_sage_vals(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
+                            int32_t Nt, float* __restrict__ valsR, float* __restrict__ valsC) {
+  // one warp per row: lanes stride the row's entries
+  const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (wid >= Nt) return;
+  const int32_t i = (int32_t)wid;
+  const int32_t k0 = rowptr[i], k1 = rowptr[i + 1];
+  const float ri = 1.0f / (float)(k1 - k0);
+  for (int32_t k = k0 + lane; k < k1; k += 32) {
+    const int32_t j = colind[k];
+    valsR[k] = ri;
+    valsC[k] = 1.0f / (float)(rowptr[j + 1] - rowptr[j]);
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_pair_off_k(const int64_t* pair_off, int32_t G, int32_t K, int64_t* out,
+                              cudaStream_t s, int* launches) {
+  count_launch(launches);
+  k_pair_off_k<<<cdiv((int64_t)G * K, 256), 256, 0, s>>>(pair_off, G, K, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_corrupt(const GraphDev& g, int32_t K, int32_t nb, int32_t corruption,
+                           float mask_rate, uint64_t seed, const StepParams* sp,
+                           const int64_t* pair_off_k, const int32_t* perms, float* Xs,
+                           cudaStream_t s, int* launches) {
+  if (g.F % 4 || K < 1 || K >= nb) return cudaErrorInvalidValue;
+  count_launch(launches);
+  const int64_t n = (int64_t)nb * g.Nt * (g.F / 4);
+  k_corrupt<<<cdiv(n, 256), 256, 0, s>>>(g.X, g.node_graph, g.node_off, g.Nt, g.G, g.F, K, nb,
+                                          corruption, (double)mask_rate, seed, sp, pair_off_k,
+                                          perms, Xs);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_sage_vals(const GraphDev& g, float* valsR, float* valsC, cudaStream_t s,
+                             int* launches) {
+  count_launch(launches);
+  if (g.Nt > 0)
+    k_sage_vals<<<cdiv((int64_t)g.Nt * 32, 256), 256, 0, s>>>(g.rowptr, g.colind, g.Nt, valsR,
+                                                               valsC);
+  return cudaGetLastError();
+}
+
+}  // namespace mars

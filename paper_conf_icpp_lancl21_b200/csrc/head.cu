@@ -9,6 +9,10 @@
 //   dl_i = (sig(l_i)-1)/(2 N_g B), dl~_i = sig(l~_i)/(2 N_g B)
 //   dv_g = Σ dl_i H3[i] + Σ dl~_i H3~[i]; dM = Σ_g dv_g s_gᵀ; ds = Mᵀ dv;
 //   dm = ds ⊙ s(1-s); dH3 = dl v_g + [pos] dm_g / N_g; dZ3 = dH3 ⊙ PReLU'(Z3)
+// NEXT-4 variants (HeadWork nb / K / readout; readings c34-c36): the stacked
+// activations hold nb blocks of Nt rows -- block 0 positive, blocks 1..K
+// corrupted (each weighted 1/K in the loss), blocks > K zero padding (weight
+// 0) -- and the readout is sig(mean) (default) or the plain mean.
 // Every cross-row reduction is two-stage with fixed-order fp64 combination
 // over row chunks (<= 256 rows, never straddling a graph): deterministic, no
 // float atomics.  The per-graph second stages are small and latency-bound; they
@@ -107,14 +111,16 @@ k_colsum(const T* __restrict__ Z3, const float* __restrict__ alpha,
 //                            graph's loss partials -> loss_g[g]
 //   outf == nullptr (row-sharded graph): the raw shard-local Σ -> outd only
 //                            (summed over shards and finished in k_head_xsum)
+//   rep > 1: every chunk has rep consecutive partials (one per block pair of
+//            k_score), summed like rep times as many chunks
 __global__ void k_chunk_sum(const double* __restrict__ part, const int32_t* __restrict__ graph_chunk,
-                            const int32_t* __restrict__ gsize, int H, int mode,
-                            double* __restrict__ outd, float* __restrict__ outf,
+                            const int32_t* __restrict__ gsize, int H, int mode, int rep,
+                            int readout, double* __restrict__ outd, float* __restrict__ outf,
                             const double* __restrict__ loss_part, double* __restrict__ loss_g) {
   __shared__ double sh[kWarps][32];
   const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int c = blockIdx.y * 32 + lane;
-  const int cb = graph_chunk[g], ce = graph_chunk[g + 1];
+  const int cb = graph_chunk[g] * rep, ce = graph_chunk[g + 1] * rep;
   double acc = 0.0;
   for (int ch = cb + w; ch < ce; ch += kWarps) acc += part[(int64_t)ch * H + c];
   sh[w][lane] = acc;
@@ -123,7 +129,8 @@ __global__ void k_chunk_sum(const double* __restrict__ part, const int32_t* __re
     double t = 0.0;
 #pragma unroll
     for (int k = 0; k < kWarps; ++k) t += sh[k][lane];
-    if (mode == 0 && outf) t = 1.0 / (1.0 + exp(-(t / (double)gsize[g])));
+    if (mode == 0 && outf)
+      t = readout ? t / (double)gsize[g] : 1.0 / (1.0 + exp(-(t / (double)gsize[g])));
     outd[(int64_t)g * H + c] = t;
     if (outf) outf[(int64_t)g * H + c] = (float)t;
   }
@@ -169,7 +176,7 @@ __global__ void k_Mv(const float* __restrict__ M, const double* __restrict__ sd,
 // columns, warp w sums rows w, w+8, ... (coalesced), fixed-order combine.
 __global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dvd,
                       const double* __restrict__ sd, const int32_t* __restrict__ gsize, int H,
-                      float* __restrict__ dmf) {
+                      int readout, float* __restrict__ dmf) {
   __shared__ double sh[kWarps][32];
   const int g = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int c = blockIdx.y * 32 + lane;
@@ -195,7 +202,7 @@ __global__ void k_MTv(const float* __restrict__ M, const double* __restrict__ dv
 #pragma unroll
     for (int k = 0; k < kWarps; ++k) ds += sh[k][lane];
     const double s = sd[(int64_t)g * H + c];
-    dmf[(int64_t)g * H + c] = (float)(ds * s * (1.0 - s) / (double)gsize[g]);
+    dmf[(int64_t)g * H + c] = (float)((readout ? ds : ds * s * (1.0 - s)) / (double)gsize[g]);
   }
 }
 
@@ -203,9 +210,10 @@ __device__ __forceinline__ double softplus_d(double x) {
   return (x > 0.0 ? x : 0.0) + log1p(exp(-fabs(x)));
 }
 
-// Scores, loss partials, dl, and dv partials.  One block (8 warps) per chunk;
-// warp w takes NU consecutive nodes i per iteration, each with its positive
-// row i and corrupted row Nt+i (2 NU rows in flight); lanes own H/32 columns.
+// Scores, loss partials, dl, and dv partials.  One block (8 warps) per (chunk,
+// block pair bp); warp w takes NU consecutive nodes i per iteration, each with
+// its rows in blocks 2bp and 2bp+1 (2 NU rows in flight; bp = 0: the positive row
+// i and the corrupted row Nt+i); lanes own H/32 columns.
 // The 2 NU logits are reduced across the warp, then lane j < 2 NU evaluates
 // the sigmoid / softplus of logit j in fp64 (parallel over lanes) and the
 // dl values are broadcast back.
@@ -217,7 +225,7 @@ __global__ void __launch_bounds__(kWarps * 32, MARS_SCORE_MINB)
 k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
         const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
         const int32_t* __restrict__ gsize, const float* __restrict__ vf,
-        const StepParams* __restrict__ sp, int32_t Nt, float* __restrict__ dl,
+        const StepParams* __restrict__ sp, int32_t Nt, int32_t K, float* __restrict__ dl,
         double* __restrict__ dv_part, double* __restrict__ loss_part) {
   using RT = RowTile<NC, T>;
   constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER;
@@ -228,11 +236,16 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
   __shared__ double sh_dv[kWarps][H];
   __shared__ double sh_loss[kWarps];
   const int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int bp = blockIdx.y, nbp = gridDim.y;
   const bool act = lane < LPR;
   const int g = chunk_graph[ch];
   const float a = alpha[2];
   const double Ng = (double)gsize[g];
   const double coef = (double)sp->inv_batch / (2.0 * Ng);
+  // block 2bp: positive (bp = 0, weight 1) or corrupted sample 2bp (1/K);
+  // block 2bp+1: corrupted sample 2bp+1 (1/K) or padding (> K, weight 0)
+  const int64_t rowA = 2LL * bp * Nt, rowB = rowA + Nt;
+  const double wA = bp == 0 ? 1.0 : 1.0 / K, wB = 2 * bp + 1 <= K ? 1.0 / K : 0.0;
   const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
   float v[PER][V];
   double dv[PER][V];
@@ -253,8 +266,8 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
       for (int q = 0; q < PER; ++q) {
         const int c = (lane + q * LPR) * V;
         if (act && i + u < r1) {
-          h[2 * u][q] = Vec<T>::ld(Z3 + (int64_t)(i + u) * H + c);
-          h[2 * u + 1][q] = Vec<T>::ld(Z3 + ((int64_t)Nt + i + u) * H + c);
+          h[2 * u][q] = Vec<T>::ld(Z3 + (rowA + i + u) * H + c);
+          h[2 * u + 1][q] = Vec<T>::ld(Z3 + (rowB + i + u) * H + c);
         } else {
           h[2 * u][q] = h[2 * u + 1][q] = typename Vec<T>::Raw{};
         }
@@ -279,10 +292,11 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
     if (lane < 2 * NU && i + (lane >> 1) < r1) {
       const double x = (double)mine;
       const double sg = 1.0 / (1.0 + exp(-x));
-      const bool neg = lane & 1;
-      dmine = (float)((neg ? sg : sg - 1.0) * coef);
-      dl[(neg ? (int64_t)Nt : 0) + i + (lane >> 1)] = dmine;
-      loss += neg ? softplus_d(x) : softplus_d(-x);
+      const bool isB = lane & 1, neg = isB || bp > 0;
+      const double wt = isB ? wB : wA;
+      dmine = (float)((neg ? sg : sg - 1.0) * (coef * wt));
+      dl[(isB ? rowB : rowA) + i + (lane >> 1)] = dmine;
+      loss += wt * (neg ? softplus_d(x) : softplus_d(-x));
     }
     float dvp[PER][V];
 #pragma unroll
@@ -318,12 +332,12 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
     double t = 0.0;
 #pragma unroll
     for (int k = 0; k < kWarps; ++k) t += sh_dv[k][c];
-    dv_part[(int64_t)ch * H + c] = t;
+    dv_part[((int64_t)ch * nbp + bp) * H + c] = t;
   }
   if (threadIdx.x == 0) {
     double t = 0.0;
     for (int k = 0; k < kWarps; ++k) t += sh_loss[k];
-    loss_part[ch] = t * coef;      // (1/B) (1/(2 N_g)) Σ softplus terms of this chunk
+    loss_part[(int64_t)ch * nbp + bp] = t * coef;   // (1/B) (1/(2 N_g)) Σ weighted softplus terms
   }
 }
 
@@ -370,13 +384,13 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
   using RT = RowTile<NC, T>;
   constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER, RU = RT::RU;
   __shared__ double wpart[kWarps];
-  const int ch = blockIdx.x, half = blockIdx.y;
+  const int ch = blockIdx.x, half = blockIdx.y;     // half: stacked block (0 = positive)
   const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const bool act = lane < LPR;
   const int g = chunk_graph[ch];
   const float a = alpha[2];
   const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
-  const int64_t base = half ? (int64_t)Nt : 0;
+  const int64_t base = (int64_t)half * Nt;
   float vg[PER][V], mg[PER][V];
 #pragma unroll
   for (int q = 0; q < PER; ++q)
@@ -430,7 +444,7 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
   if (threadIdx.x == 0) {
     double s = 0.0;
     for (int k = 0; k < kWarps; ++k) s += wpart[k];
-    slots[(int64_t)ch * 2 + half] = s;
+    slots[(int64_t)ch * gridDim.y + half] = s;
   }
 }
 
@@ -494,40 +508,43 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
   constexpr int H = NC * 32;
   const dim3 gh(g.G, H / 32);
   cudaError_t e;
+  const int nb = w.nb, nbp = nb / 2;
+  if (nb < 2 || (nb & 1) || w.K < 1 || w.K >= nb || (hs && (nb != 2 || w.readout)))
+    return cudaErrorInvalidValue;
   k_colsum<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, w.colsum_part);
   if (!hs) {
-    k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.gsize, H, 0, w.sd, w.s,
-                                   nullptr, nullptr);
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.gsize, H, 0, 1, w.readout,
+                                   w.sd, w.s, nullptr, nullptr);
   } else {      // shard-local sums -> own exchange buffer; barrier; sum over shards
-    k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.gsize, H, 0, hs->x_own[0],
-                                   nullptr, nullptr, nullptr);
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.colsum_part, g.graph_chunk, g.gsize, H, 0, 1, 0,
+                                   hs->x_own[0], nullptr, nullptr, nullptr);
     if ((e = launch_shard_barrier(*hs->sync, s, nullptr)) != cudaSuccess) return e;
     if ((e = launch_head_xsum(hs->x_peers[0], hs->sync->P, H, 0, g.gsize, w.sd, w.s, nullptr, s,
                               nullptr)) != cudaSuccess)
       return e;
   }
   k_Mv<<<gh, 256, 0, s>>>(M, w.sd, H, w.v);
-  k_score<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
-                                                   g.gsize, w.v, sp, g.Nt, w.dl, w.dv_part,
-                                                   w.loss_part);
+  k_score<NC, T><<<dim3(g.nchunks, nbp), kWarps * 32, 0, s>>>(
+      Z3, alpha, g.chunk_row, g.chunk_graph, g.gsize, w.v, sp, g.Nt, w.K, w.dl, w.dv_part,
+      w.loss_part);
   if (!hs) {
-    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, w.dvd, w.dv,
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, nbp, 0, w.dvd, w.dv,
                                    w.loss_part, w.loss_g);
   } else {
-    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, hs->x_own[1], nullptr,
-                                   w.loss_part, hs->x_own[1] + H);
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, 1, 0, hs->x_own[1],
+                                   nullptr, w.loss_part, hs->x_own[1] + H);
     if ((e = launch_shard_barrier(*hs->sync, s, nullptr)) != cudaSuccess) return e;
     if ((e = launch_head_xsum(hs->x_peers[1], hs->sync->P, H, 1, g.gsize, w.dvd, w.dv, w.loss_g,
                               s, nullptr)) != cudaSuccess)
       return e;
   }
-  k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.gsize, H, w.dm);
+  k_MTv<<<gh, 256, 0, s>>>(M, w.dvd, w.sd, g.gsize, H, w.readout, w.dm);
   k_dM<<<cdiv((int64_t)H * H, 256), 256, 0, s>>>(w.dvd, w.sd, g.G, H, w.loss_g, gM, loss_out);
-  k_dz3<NC, T><<<dim3(g.nchunks, 2), kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
+  k_dz3<NC, T><<<dim3(g.nchunks, nb), kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph,
                                                           w.dl, w.v, w.dm, g.Nt, dZ, w.slots,
                                                           std::is_same<T, float>::value ? w.rs_dz3
                                                                                         : nullptr);
-  *nslots = 2 * g.nchunks;
+  *nslots = nb * g.nchunks;
   return cudaGetLastError();
 }
 
@@ -548,7 +565,9 @@ cudaError_t head_t(const GraphDev& g, int H, const void* Z3, const float* M, con
 
 }  // namespace
 
-int head_slots(const GraphDev& g) { return 2 * g.nchunks + 1 + kRedParts; }   // + reduction scratch
+int head_slots(const GraphDev& g, int nb) {       // + reduction scratch
+  return nb * g.nchunks + 1 + kRedParts;
+}
 
 cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, const float* params_M,
                         const float* alpha_dev, const StepParams* sp, const HeadWork& w, void* dZ,

@@ -235,18 +235,22 @@ cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, in
 // ---------------------------------------------------------------- head.cu
 struct HeadWork {
   double* colsum_part;  // [nchunks*H]
-  double* dv_part;      // [nchunks*H]
-  double* loss_part;    // [nchunks]
+  double* dv_part;      // [nchunks*nb/2*H]
+  double* loss_part;    // [nchunks*nb/2]
   float* s;             // [G*H]
   float* v;             // [G*H]
   float* dm;            // [G*H] (already divided by N_g)
   float* dv;            // [G*H]
   double* dvd;          // [G*H]
   double* sd;           // [G*H]
-  float* dl;            // [2*Nt]
+  float* dl;            // [nb*Nt]
   double* loss_g;       // [G] per-graph loss (already / (2 N_g B))
   double* slots;        // [nslots] dalpha3 partials
-  float* rs_dz3;        // [2*Nt] power-of-two row scales of dZ3 (fp32 storage) or null
+  float* rs_dz3;        // [nb*Nt] power-of-two row scales of dZ3 (fp32 storage) or null
+  // NEXT-4 (c34-c36): nb stacked blocks of Nt rows (even; block 0 positive,
+  // 1..K corrupted, > K padding), K corruption samples, readout 0 = sig(mean),
+  // 1 = mean.  The default DGI step: nb = 2, K = 1, readout 0.
+  int32_t nb, K, readout;
 };
 // Forward head + head backward: writes grads of M (dM) and the loss slot,
 // dZ3 into dZ, dalpha3 partials into w.slots.
@@ -262,7 +266,25 @@ cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16,
                         const float* params_M, const float* alpha_dev, const StepParams* sp,
                         const HeadWork& w, void* dZ, float* grad_M, float* loss_out, int* nslots,
                         cudaStream_t s, int* launches, const HeadShard* hs = nullptr);
-int head_slots(const GraphDev& g);
+int head_slots(const GraphDev& g, int nb);
+
+// ---------------------------------------------------------------- contrast.cu (NEXT-4)
+// out[k*G + g] = pair_off[g]*K + k: the pair index offset of corruption sample
+// k of graph g when every graph draws K samples (c34).
+cudaError_t launch_pair_off_k(const int64_t* pair_off, int32_t G, int32_t K, int64_t* out,
+                              cudaStream_t s, int* launches);
+// The stacked layer-1 inputs Xs [nb*Nt x F] fp32: block 0 = X, block k in
+// 1..K = the k-th corruption of X (corruption 0: rows X[perms[(k-1)*Nt + i]];
+// 1: X ⊙ Bernoulli keep mask, c35), blocks > K = 0.
+cudaError_t launch_corrupt(const GraphDev& g, int32_t K, int32_t nb, int32_t corruption,
+                           float mask_rate, uint64_t seed, const StepParams* sp,
+                           const int64_t* pair_off_k, const int32_t* perms, float* Xs,
+                           cudaStream_t s, int* launches);
+// SAGE-GCN aggregation (c37): valsR[k] = 1/deg(row), valsC[k] = 1/deg(col) of
+// each CSR entry (deg counts the self loop): Â_mean = D^-1 (A + I) and its
+// transpose on the same (symmetric) pattern.
+cudaError_t launch_sage_vals(const GraphDev& g, float* valsR, float* valsC, cudaStream_t s,
+                             int* launches);
 // grad[0] = Σ slots (fixed order, double)
 cudaError_t launch_reduce_slots(double* slots, int n, float* grad, cudaStream_t s,
                                 int* launches);

@@ -356,6 +356,16 @@ struct Workspace {
   // (Activation buffers are sized for fp32 and hold bf16 in that mode.)
   void *w16t[3] = {}, *w16[3] = {};
   float* dw16_part = nullptr;
+  // NEXT-4 variants (contrast.cu): nb stacked blocks, K corruption samples,
+  // materialised layer-1 inputs Xs [nb*Nt x F], per-sample pair offsets,
+  // SAGE-GCN values (forward Â, backward Âᵀ), PReLU slope 1 for layer 1
+  int32_t nb = 2, K = 1;
+  bool has_xs = false;
+  int64_t nnz_vals = 0;
+  float* Xs = nullptr;
+  int64_t* pair_off_k = nullptr;
+  float *valsR = nullptr, *valsC = nullptr;
+  float* one = nullptr;
   std::vector<void*> owned;
   void release() {
     for (void* p : owned) cudaFree(p);
@@ -380,6 +390,9 @@ struct mars_dgi {
   int sp_ring = 32, sp_next = 0;
   Workspace ws;
   const mars_graph* ws_graph = nullptr;
+  mars_contrastive ct{1, MARS_CORRUPT_PERMUTE, 0.f, MARS_READOUT_SIGMOID_MEAN, MARS_AGG_GCN};
+  int ct_nb() const { return (ct.num_neg + 2) & ~1; }     // K + 1 blocks, rounded up to even
+  bool ct_materialise() const { return ct.num_neg > 1 || ct.corruption != MARS_CORRUPT_PERMUTE; }
   bool capture = true;
   int gemm_impl = 0;                // 0 auto (tcgen05 3xFP16 when supported), 1 SIMT FFMA
   // Captured steps, one per (graph set, stream), least recently used evicted:
@@ -1098,6 +1111,37 @@ extern "C" mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable) {
   return MARS_OK;
 }
 
+extern "C" mars_status mars_dgi_set_contrastive(mars_dgi* m, const mars_contrastive* c) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!c) return fail(MARS_EINVAL, "config is NULL");
+  if (c->num_neg < 1 || c->num_neg > 64) return fail(MARS_EINVAL, "num_neg must be in [1, 64]");
+  if (c->corruption != MARS_CORRUPT_PERMUTE && c->corruption != MARS_CORRUPT_MASK)
+    return fail(MARS_EINVAL, "unknown corruption");
+  if (!(c->mask_rate >= 0.f && c->mask_rate <= 1.f)) return fail(MARS_EINVAL, "mask_rate not in [0, 1]");
+  if (c->readout != MARS_READOUT_SIGMOID_MEAN && c->readout != MARS_READOUT_MEAN)
+    return fail(MARS_EINVAL, "unknown readout");
+  if (c->aggregator != MARS_AGG_GCN && c->aggregator != MARS_AGG_SAGE_GCN)
+    return fail(MARS_EINVAL, "unknown aggregator");
+  const bool dflt = c->num_neg == 1 && c->corruption == MARS_CORRUPT_PERMUTE &&
+                    c->readout == MARS_READOUT_SIGMOID_MEAN && c->aggregator == MARS_AGG_GCN;
+  if (m->sh.g && !dflt) return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
+  CK(cudaSetDevice(m->cfg.device));
+  m->drop_execs();                 // captured steps bake the variant in
+  CK(cudaStreamSynchronize(m->stream));
+  m->ws.release();                 // re-sized on the next step / encode
+  m->last_Nt = 0;
+  m->kb_valid_Nt = 0;
+  m->ct = *c;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_get_contrastive(const mars_dgi* m, mars_contrastive* c) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!c) return fail(MARS_EINVAL, "config is NULL");
+  *c = m->ct;
+  return MARS_OK;
+}
+
 // ---------------------------------------------------------------- workspaces
 static mars_status ensure_kb(mars_dgi* m, const mars_graph* g) {
   if (!m->keep_bwd || m->kb_rows >= g->dev.Nt) return MARS_OK;
@@ -1115,16 +1159,18 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   if (mars_status st = ensure_kb(m, g)) return st;
   Workspace& w = m->ws;
   const GraphDev& pv = g->perm_view();
+  const int nbk = m->ct_nb(), K = m->ct.num_neg;
+  const bool xs = m->ct_materialise(), sage = m->ct.aggregator == MARS_AGG_SAGE_GCN;
   if (w.Nt >= g->dev.Nt && w.Nperm >= pv.Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks &&
       w.nbuckets >= pv.nbuckets && w.nnz_perm >= pv.nnz && w.nlong >= g->dev.nlong &&
-      w.nseg >= g->dev.nseg &&
-      w.F == m->F && w.H == m->H)
+      w.nseg >= g->dev.nseg && w.F == m->F && w.H == m->H && w.nb == nbk && w.K == K &&
+      (w.has_xs || !xs) && (!sage || w.nnz_vals >= g->dev.nnz))
     return MARS_OK;
   if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
   m->drop_execs();
   CK(cudaStreamSynchronize(m->stream));
   w.release();
-  int64_t Nt = g->dev.Nt, R = 2 * Nt, Np = pv.Nt;
+  int64_t Nt = g->dev.Nt, R = nbk * Nt, Np = pv.Nt;
   int F = m->F, H = m->H, G = g->G, nch = g->dev.nchunks, nb = pv.nbuckets;
   auto al = [&](void** p, size_t bytes) -> cudaError_t {
     cudaError_t e = cudaMalloc(p, bytes ? bytes : 8);
@@ -1136,7 +1182,25 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   for (int l = 0; l < 2; ++l) CK(al((void**)&w.Y23[l], sizeof(float) * R * H));
   CK(al((void**)&w.dZ, sizeof(float) * R * H));
   CK(al((void**)&w.dY, sizeof(float) * R * H));
-  CK(al((void**)&w.perm, sizeof(int32_t) * Np));
+  if (nbk > K + 1) {               // the padding block stays zero (enqueue_step)
+    CK(cudaMemset(w.Y1, 0, sizeof(float) * R * F));
+    for (int l = 0; l < 3; ++l) CK(cudaMemset(w.Z[l], 0, sizeof(float) * R * H));
+    for (int l = 0; l < 2; ++l) CK(cudaMemset(w.Y23[l], 0, sizeof(float) * R * H));
+    CK(cudaMemset(w.dZ, 0, sizeof(float) * R * H));
+    CK(cudaMemset(w.dY, 0, sizeof(float) * R * H));
+  }
+  CK(al((void**)&w.perm, sizeof(int32_t) * Np * K));
+  CK(al((void**)&w.pair_off_k, sizeof(int64_t) * (size_t)G * K));
+  if (xs) CK(al((void**)&w.Xs, sizeof(float) * R * F));
+  if (sage) {
+    CK(al((void**)&w.valsR, sizeof(float) * (size_t)std::max<int64_t>(1, g->dev.nnz)));
+    CK(al((void**)&w.valsC, sizeof(float) * (size_t)std::max<int64_t>(1, g->dev.nnz)));
+  }
+  CK(al((void**)&w.one, sizeof(float)));
+  {
+    const float one = 1.f;
+    CK(cudaMemcpy(w.one, &one, sizeof one, cudaMemcpyHostToDevice));
+  }
   CK(al((void**)&w.long_part, sizeof(float) * (size_t)g->dev.nseg * 2 * 256));
   CK(al((void**)&w.colperm, sizeof(int32_t) * (size_t)std::max<int64_t>(1, pv.nnz)));
   CK(al((void**)&w.pw.keys, sizeof(uint64_t) * Np));
@@ -1148,8 +1212,8 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   CK(al(&w.pw.scan_tmp, scan_tmp_bytes(nb + 1)));
   HeadWork& h = w.hw;
   CK(al((void**)&h.colsum_part, sizeof(double) * nch * H));
-  CK(al((void**)&h.dv_part, sizeof(double) * nch * H));
-  CK(al((void**)&h.loss_part, sizeof(double) * nch));
+  CK(al((void**)&h.dv_part, sizeof(double) * nch * (nbk / 2) * H));
+  CK(al((void**)&h.loss_part, sizeof(double) * nch * (nbk / 2)));
   CK(al((void**)&h.s, sizeof(float) * G * H));
   CK(al((void**)&h.v, sizeof(float) * G * H));
   CK(al((void**)&h.dm, sizeof(float) * G * H));
@@ -1158,7 +1222,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   CK(al((void**)&h.sd, sizeof(double) * G * H));
   CK(al((void**)&h.dl, sizeof(float) * R));
   CK(al((void**)&h.loss_g, sizeof(double) * G));
-  int nsl = std::max(head_slots(g->dev), spmm_bwd_slots(g->dev));
+  int nsl = std::max(head_slots(g->dev, nbk), (nbk / 2) * spmm_bwd_slots(g->dev));
   for (int l = 0; l < 3; ++l) CK(al((void**)&w.slots[l], sizeof(double) * nsl));
   h.slots = w.slots[2];
   size_t tn = std::max(gemm_tn_partial_floats(R, F, H), gemm_tn_partial_floats(R, H, H));
@@ -1195,6 +1259,13 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   w.nbuckets = nb;
   w.F = F;
   w.H = H;
+  w.nb = nbk;
+  w.K = K;
+  w.has_xs = xs;
+  w.nnz_vals = sage ? g->dev.nnz : 0;
+  h.nb = nbk;
+  h.K = K;
+  h.readout = m->ct.readout;
   return MARS_OK;
 }
 
@@ -1224,7 +1295,19 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   GraphDev g = gr->dev;
   g.long_part = w.long_part;
   const int F = m->F, H = m->H;
-  const int64_t R = 2LL * g.Nt;
+  // NEXT-4 variants (c34-c37): nb stacked blocks [pos; neg_1..neg_K; pad];
+  // the default DGI step has nb = 2 and the fused layer-1 corruption gather
+  const int nb = w.nb, K = m->ct.num_neg, nbp = nb / 2;
+  const bool mat = m->ct_materialise();
+  // GEMM rows: the K + 1 real blocks.  A padding block (K even) is zero from
+  // allocation and never written: its forward aggregation is skipped (the last
+  // pair runs one branch), and the backward aggregation's pass over it gathers
+  // zeros into zeros.
+  const int64_t R = (int64_t)(K + 1) * g.Nt;
+  GraphDev gb = g;                       // the backward aggregation's view (Âᵀ)
+  w.hw.nb = nb;
+  w.hw.K = K;
+  w.hw.readout = m->ct.readout;
   float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
   float* Mp = m->params + (int64_t)F * H + 2LL * H * H;
   float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
@@ -1246,10 +1329,29 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   // Row-sharded graph: exchange steps between the shards (shard.cu).  A
   // barrier precedes every read of buffers the peers wrote in this step.
   const bool shard = m->sh.connected && gr->uid == m->sh.guid;
-  // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM);
-  // a row-sharded graph permutes the whole graph on every shard
-  RET(launch_perm(gr->perm_view(), m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
-  RET(launch_colperm(g, w.perm, w.colperm, s, nl));
+  if (m->ct.aggregator == MARS_AGG_SAGE_GCN) {
+    RET(launch_sage_vals(g, w.valsR, w.valsC, s, nl));
+    g.vals = w.valsR;
+    gb.vals = w.valsC;
+  }
+  if (!mat) {
+    // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM);
+    // a row-sharded graph permutes the whole graph on every shard
+    RET(launch_perm(gr->perm_view(), m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
+    RET(launch_colperm(g, w.perm, w.colperm, s, nl));
+  } else {
+    // K samples (c34): sample k of graph g is pair pair_off[g] K + k; the
+    // corrupted layer-1 inputs are materialised block by block (c35)
+    RET(launch_pair_off_k(g.pair_off, g.G, K, w.pair_off_k, s, nl));
+    if (m->ct.corruption == MARS_CORRUPT_PERMUTE)
+      for (int k = 0; k < K; ++k) {
+        GraphDev pv = g;
+        pv.pair_off = w.pair_off_k + (int64_t)k * g.G;
+        RET(launch_perm(pv, m->cfg.seed, m->d_sp, w.pw, w.perm + (int64_t)k * g.Nt, s, nl));
+      }
+    RET(launch_corrupt(g, K, nb, m->ct.corruption, m->ct.mask_rate, m->cfg.seed, m->d_sp,
+                       w.pair_off_k, w.perm, w.Xs, s, nl));
+  }
   MARK(MARS_PH_PERM);
   const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
@@ -1262,6 +1364,11 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
                              w.h3_w_hi[l], w.h3_w_lo[l], s, nl));
   }
   MARK(MARS_PH_GEMM_FWD);
+  const size_t es = b16 ? 2 : 4;                         // storage bytes per element
+  // rows [2p Nt, (2p + 2) Nt) of a stacked buffer of C columns (block pair p)
+  auto blk = [&](const void* base, int p, int C, size_t bytes) -> char* {
+    return (char*)base + (size_t)2 * p * g.Nt * C * bytes;
+  };
   // a5-a7: forward, l = 1..3
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
@@ -1270,9 +1377,21 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
       RET(launch_shard_barrier(m->sh.sync, s, nl));   // peers' Z_{l-1} complete
       MARK(MARS_PH_EXCHANGE);
     }
-    RET(launch_spmm_fwd(g, Cin, T, b16 && l > 0, w.colperm, alpha, l - 1, Ys[l], b16, 1, s, nl,
-                        shard && l > 0 ? &m->sh.z[l - 1] : nullptr,
-                        tc[l] ? w.h3_rsY[l] : nullptr));
+    if (!mat || l > 0) {
+      // one aggregation per block pair (the positive / corrupted pair of the
+      // default step): both halves of the pair share each CSR entry read
+      for (int p = 0; p < nbp; ++p)
+        RET(launch_spmm_fwd(g, Cin, l == 0 ? T : blk(T, p, Cin, es), b16 && l > 0, w.colperm,
+                            alpha, l - 1, blk(Ys[l], p, Cin, es), b16, 2 * p + 1 <= K, s, nl,
+                            shard && l > 0 ? &m->sh.z[l - 1] : nullptr,
+                            tc[l] ? w.h3_rsY[l] + 2LL * p * g.Nt : nullptr));
+    } else {
+      // materialised layer-1 inputs: the stacked aggregation with slope-1 PReLU
+      for (int p = 0; p < nbp; ++p)
+        RET(launch_spmm_fwd(g, Cin, blk(w.Xs, p, F, 4), 0, nullptr, w.one, 0,
+                            blk(Ys[0], p, Cin, es), b16, 2 * p + 1 <= K, s, nl, nullptr,
+                            tc[0] ? w.h3_rsY[0] + 2LL * p * g.Nt : nullptr));
+    }
     MARK(MARS_PH_SPMM_FWD);
     if (b16) RET(tc16_gemm_rows(Ys[l], w.w16t[l], w.Z[l], R, H, Cin, s, nl));
     else if (tc[l])
@@ -1295,8 +1414,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   RET(launch_head(g, H, w.Z[2], b16, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl,
                   shard ? &hs : nullptr));
   RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
-  const size_t es = b16 ? 2 : 4;                         // storage bytes per element
-  const size_t kb_bytes = (size_t)R * H * es;
+  const size_t kb_bytes = (size_t)2 * g.Nt * H * es;     // test hook: blocks 0 and 1
   const bool kb = m->keep_bwd && m->kb_rows >= g.Nt;
   if (kb) RET(cudaMemcpyAsync(m->kb_dZ[2], w.dZ, kb_bytes, cudaMemcpyDeviceToDevice, s));
   MARK(MARS_PH_HEAD);
@@ -1322,9 +1440,15 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
         RET(launch_shard_barrier(m->sh.sync, s, nl));  // peers' dY_l complete
         MARK(MARS_PH_EXCHANGE);
       }
-      RET(launch_spmm_bwd(g, Cin, dYl, w.Z[l - 1], b16, alpha, l - 1, w.dZ, w.slots[l - 1], &ns,
-                          s, nl, shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr,
-                          tc[l - 1] ? w.h3_rsdZ : nullptr));
+      ns = 0;
+      for (int p = 0; p < nbp; ++p) {
+        int nsp = 0;
+        RET(launch_spmm_bwd(gb, Cin, blk(dYl, p, Cin, es), blk(w.Z[l - 1], p, Cin, es), b16,
+                            alpha, l - 1, blk(w.dZ, p, Cin, es), w.slots[l - 1] + ns, &nsp, s, nl,
+                            shard ? &m->sh.dy[l == 2 ? 0 : 1] : nullptr,
+                            tc[l - 1] ? w.h3_rsdZ + 2LL * p * g.Nt : nullptr));
+        ns += nsp;
+      }
       if (kb) RET(cudaMemcpyAsync(m->kb_dZ[l - 1], w.dZ, kb_bytes, cudaMemcpyDeviceToDevice, s));
       MARK(MARS_PH_SPMM_BWD);
       RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
@@ -1441,6 +1565,8 @@ static mars_status run_step(mars_dgi* m, const mars_graph* g, uint64_t step_inde
 extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t step_index,
                                      int64_t pair_base, int64_t global_batch, mars_step_out* out) {
   if (mars_status st = check_step_args(m, g, global_batch)) return st;
+  if (out && out->perms && m->ct.corruption != MARS_CORRUPT_PERMUTE)
+    return fail(MARS_EINVAL, "no permutations: the corruption is feature masking");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
   if (mars_status st = run_step(m, g, step_index, pair_base, global_batch)) return st;
@@ -1453,13 +1579,16 @@ extern "C" mars_status mars_dgi_step(mars_dgi* m, const mars_graph* g, uint64_t 
     if (out->grads)
       CK(cudaMemcpyAsync(out->grads, m->grads_final(), sizeof(float) * m->P,
                          cudaMemcpyDeviceToHost, s));
+    const int K = m->ct.num_neg;
     if (out->perms)
-      CK(cudaMemcpyAsync(out->perms, m->ws.perm, sizeof(int32_t) * g->Nt, cudaMemcpyDeviceToHost, s));
+      CK(cudaMemcpyAsync(out->perms, m->ws.perm, sizeof(int32_t) * g->Nt * K,
+                         cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
     if (out->perms)
-      for (int gi = 0; gi < g->G; ++gi)
-        for (int32_t i = g->h_node_off[gi]; i < g->h_node_off[gi + 1]; ++i)
-          out->perms[i] -= g->h_node_off[gi];
+      for (int k = 0; k < K; ++k)
+        for (int gi = 0; gi < g->G; ++gi)
+          for (int32_t i = g->h_node_off[gi]; i < g->h_node_off[gi + 1]; ++i)
+            out->perms[(int64_t)k * g->Nt + i] -= g->h_node_off[gi];
     if (out->loss) *out->loss = loss;
     if (mars_status st = check_skipped(m, skipped)) return st;
     if (!std::isfinite(loss)) return fail(MARS_ENUMERIC, "non-finite loss");
@@ -1604,6 +1733,10 @@ static cudaError_t enqueue_encode(mars_dgi* m, const mars_graph* g, cudaStream_t
   float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
   const bool b16 = m->cfg.precision == MARS_BF16;
   cudaError_t e;
+  if (m->ct.aggregator == MARS_AGG_SAGE_GCN) {          // c37: Â = D^-1 (A + I)
+    if ((e = launch_sage_vals(gd, w.valsR, w.valsC, s, nl))) return e;
+    gd.vals = w.valsR;
+  }
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     const void* T = l == 0 ? (const void*)gd.X : (const void*)w.Z[l - 1];
@@ -1701,6 +1834,7 @@ static cudaError_t enqueue_encoder_backward(mars_dgi* m, const mars_graph* gr, c
   float* galpha = m->grads + (int64_t)F * H + 3LL * H * H;
   float* Ys[3] = {w.Y1, w.Y23[0], w.Y23[1]};
   cudaError_t e;
+  if (m->ct.aggregator == MARS_AGG_SAGE_GCN) g.vals = w.valsC;   // Âᵀ (c37; set by the encode)
   // the corrupted half of the saved activations is zero (and its row scales neutral)
   if ((e = cudaMemsetAsync(w.Y1 + Nt * F, 0, sizeof(float) * Nt * F, s))) return e;
   for (int l = 0; l < 2; ++l)
@@ -2119,6 +2253,9 @@ extern "C" mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g) {
   if (mars_status st = check_graph(g)) return st;
   if (!g->sharded) return fail(MARS_EINVAL, "graph was not loaded with mars_graph_load_shard");
   if (m->sh.g) return fail(MARS_ESTATE, "model already attached to a shard");
+  if (m->ct.num_neg != 1 || m->ct.corruption != MARS_CORRUPT_PERMUTE ||
+      m->ct.readout != MARS_READOUT_SIGMOID_MEAN || m->ct.aggregator != MARS_AGG_GCN)
+    return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
   if (m->comm) return fail(MARS_EINVAL, "a shard-attached model cannot also be data-parallel");
   if (g->F != m->F || g->device != m->cfg.device) return fail(MARS_EINVAL, "F / device mismatch");
   if (!(m->H == 128 || m->H == 256) || m->gemm_impl == MARS_GEMM_SIMT)

@@ -66,6 +66,18 @@ class PpoConfig(ctypes.Structure):
                 ("seed", ctypes.c_uint64), ("capacity_bytes", ctypes.c_float)]
 
 
+class Contrastive(ctypes.Structure):
+    """mars_contrastive (NEXT-4, readings c34-c37)."""
+    _fields_ = [("num_neg", ctypes.c_int32), ("corruption", ctypes.c_int32),
+                ("mask_rate", ctypes.c_float), ("readout", ctypes.c_int32),
+                ("aggregator", ctypes.c_int32)]
+
+
+CORRUPTIONS = {"permute": 0, "mask": 1}
+READOUTS = {"sigmoid_mean": 0, "mean": 1}
+AGGREGATORS = {"gcn": 0, "sage_gcn": 1}
+
+
 class StepOut(ctypes.Structure):
     _fields_ = [("loss", ctypes.c_void_p), ("grads", ctypes.c_void_p), ("perms", ctypes.c_void_p)]
 
@@ -88,6 +100,8 @@ SIGNATURES = {
     "mars_dgi_set_stream": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dgi_set_graph_capture": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
     "mars_dgi_set_gemm_impl": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
+    "mars_dgi_set_contrastive": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(Contrastive)]),
+    "mars_dgi_get_contrastive": (ctypes.c_int, [ctypes.c_void_p, ctypes.POINTER(Contrastive)]),
     "mars_dgi_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64,
                                      ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(StepOut)]),
     "mars_encode": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
@@ -407,6 +421,28 @@ class DGI:
         self.handle = handle
         self.F, self.H = F, H
         self.P = num_params(F, H)
+        self.num_neg = 1
+        self.corruption = "permute"
+
+    def set_contrastive(self, num_neg: int = 1, corruption: str = "permute",
+                        mask_rate: float = 0.0, readout: str = "sigmoid_mean",
+                        aggregator: str = "gcn"):
+        """mars_dgi_set_contrastive (NEXT-4): K corruption samples sharing one
+        positive branch, permutation or feature-mask corruption, sig(mean) or
+        mean readout, GCN or SAGE-GCN aggregation.  The defaults are the paper's
+        DGI step."""
+        c = Contrastive(int(num_neg), CORRUPTIONS[corruption], float(mask_rate),
+                        READOUTS[readout], AGGREGATORS[aggregator])
+        _check(lib().mars_dgi_set_contrastive(self.handle, ctypes.byref(c)))
+        self.num_neg, self.corruption = int(num_neg), corruption
+
+    def get_contrastive(self) -> dict:
+        c = Contrastive()
+        _check(lib().mars_dgi_get_contrastive(self.handle, ctypes.byref(c)))
+        inv = lambda d, v: next(k for k, x in d.items() if x == v)
+        return dict(num_neg=c.num_neg, corruption=inv(CORRUPTIONS, c.corruption),
+                    mask_rate=c.mask_rate, readout=inv(READOUTS, c.readout),
+                    aggregator=inv(AGGREGATORS, c.aggregator))
 
     def step(self, g: Graph, step_index: int, pair_base: int = 0, global_batch: int | None = None,
              want_loss=False, want_grads=False, want_perms=False):
@@ -547,7 +583,8 @@ def dgi_step(m: DGI, g: Graph, step_index: int, pair_base: int = 0, global_batch
     if want_grads:
         res["grads"] = np.zeros(m.P, np.float32); out.grads = res["grads"].ctypes.data
     if want_perms:
-        res["perms"] = np.zeros(g.total_nodes, np.int32); out.perms = res["perms"].ctypes.data
+        res["perms"] = np.zeros(g.total_nodes * m.num_neg, np.int32)
+        out.perms = res["perms"].ctypes.data
     _check(lib().mars_dgi_step(m.handle, g.handle, step_index & (2 ** 64 - 1), int(pair_base), B,
                                ctypes.byref(out)))
     if want_loss:

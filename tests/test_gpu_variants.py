@@ -1,0 +1,203 @@
+"""GPU parity of the NEXT-4 contrastive variants (mars_dgi_set_contrastive;
+readings c34-c37) against the variant oracle (oracle/variants.py, float64
+autograd), through the C ABI: K corruption samples sharing one positive
+branch, feature-masking corruption, the mean readout and the SAGE-GCN
+aggregator, alone and combined, fp32 (<= 1e-5 scaled) and bf16
+(2e-2).  At the GNMT bench size, where the fp64 oracle is too slow end to end,
+the shared-positive step is checked against the same K samples run as K
+copies of the graph (c20) -- a property that holds at any size."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from oracle import variants as V
+import paper_conf_icpp_lancl21_b200 as mars
+from synth import graphs as SG
+from tests.util import scaled_err
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+
+
+def _graphs(F):
+    # several chunks (<= 256 rows) per graph and a ragged tail
+    return [SG.tiny(0, N=300, F=F), SG.tiny(1, N=77, F=F), SG.tiny(2, N=517, F=F)]
+
+
+def _run(gs, F, H, variant, seed=5, step=3, pair_base=0, precision=mars.MARS_FP32):
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=seed, precision=precision)
+    m.set_contrastive(**variant)
+    p0 = m.get_state()[0].astype(np.float64)
+    out = m.step(g, step, pair_base, want_loss=True, want_grads=True,
+                 want_perms=variant.get("corruption", "permute") == "permute")
+    m.free(); g.free()
+    return p0, out
+
+
+VARIANTS = [
+    dict(num_neg=2),
+    dict(num_neg=3),
+    dict(num_neg=4),
+    dict(corruption="mask", mask_rate=0.25),
+    dict(num_neg=3, corruption="mask", mask_rate=0.5),
+    dict(readout="mean"),
+    dict(aggregator="sage_gcn"),
+    dict(num_neg=2, readout="mean", aggregator="sage_gcn"),
+]
+
+
+@pytest.mark.parametrize("F,H", [(16, 32), (64, 128)])
+@pytest.mark.parametrize("variant", VARIANTS, ids=lambda v: "-".join(f"{k}={x}" for k, x in v.items()))
+def test_variant_step_vs_oracle(variant, F, H):
+    gs = _graphs(F)
+    seed, step, pb = 5, 3, 11
+    p0, out = _run(gs, F, H, variant, seed, step, pb)
+    loss, grads = V.step_grads(gs, p0, F, H, seed, step, pair_base=pb, sparse=True, **variant)
+    assert abs(out["loss"] - loss) / abs(loss) <= TOL
+    assert scaled_err(out["grads"], grads) <= TOL, scaled_err(out["grads"], grads)
+    if "perms" in out:
+        K = variant.get("num_neg", 1)
+        Nt = sum(g.num_nodes for g in gs)
+        perms = out["perms"].reshape(K, Nt)
+        off = 0
+        for gi, g in enumerate(gs):
+            for k in range(K):
+                ref = oracle.perm(seed, step, pb + gi * K + k, g.num_nodes)
+                assert np.array_equal(perms[k, off:off + g.num_nodes], ref)
+            off += g.num_nodes
+
+
+def _cancellation(gs, p, F, H, seed, step, num_neg=1, corruption="permute", mask_rate=0.0,
+                  readout="sigmoid_mean", aggregator="gcn"):
+    """max over graphs of (|Σ_pos dl h| + (1/K) Σ_k |Σ dl~ h~|) / |dv| (max-norms):
+    how much dv = Σ dl h -- the sum every gradient flows through -- cancels."""
+    pt = torch.tensor(p)
+    W1, W2, W3, M, al = V.unpack(pt, F, H)
+    worst = 0.0
+    for gi, g in enumerate(gs):
+        An = torch.from_numpy(V.normalise(V.adjacency(g), aggregator))
+        X = torch.tensor(np.asarray(g.features, np.float64))
+        Hp = V.encoder(An, X, (W1, W2, W3), al)
+        s = torch.sigmoid(Hp.mean(0)) if readout == "sigmoid_mean" else Hp.mean(0)
+        v = M @ s
+        a = ((torch.sigmoid(Hp @ v) - 1)[:, None] * Hp).sum(0)
+        parts, tot = [a.abs().max()], a.clone()
+        for k in range(num_neg):
+            Hn = V.encoder(An, V.corrupted(g, X, seed, step, gi * num_neg + k, corruption,
+                                           mask_rate), (W1, W2, W3), al)
+            b = (torch.sigmoid(Hn @ v)[:, None] * Hn).sum(0) / num_neg
+            parts.append(b.abs().max())
+            tot = tot + b
+        worst = max(worst, float(sum(parts) / tot.abs().max()))
+    return worst
+
+
+@pytest.mark.parametrize("variant", [dict(num_neg=3), dict(num_neg=3, readout="mean"),
+                                     dict(corruption="mask", mask_rate=0.25, aggregator="sage_gcn")],
+                         ids=lambda v: "-".join(f"{k}={x}" for k, x in v.items()))
+def test_variant_bf16(variant):
+    """bf16 storage + bf16 MMAs end to end against fp64.  The 2e-2 bar of
+    DESIGN.md §6 is a stage-wise bar; end to end, bf16 rounding of H3 enters
+    every gradient through dv = Σ dl_i h_i, a difference of positive and
+    corrupted sums that cancels more or less depending on the variant (the
+    plain-mean readout gives scores near 0, dl near -1/2 and +1/2, and several
+    times the cancellation of sig(mean)).  So the variant is held to 2e-2 or to
+    1.5 x the default step's own end-to-end bf16 error scaled by the ratio of
+    the two cancellation factors, whichever is larger (the c33 rule: the bar
+    follows the conditioning)."""
+    gs = _graphs(64)
+    errs, canc = {}, {}
+    for name, v in (("default", {}), ("variant", variant)):
+        p0, out = _run(gs, 64, 128, v, precision=mars.MARS_BF16)
+        loss, grads = V.step_grads(gs, p0, 64, 128, 5, 3, sparse=True, **v)
+        errs[name] = (abs(out["loss"] - loss) / abs(loss), scaled_err(out["grads"], grads))
+        canc[name] = _cancellation(gs, p0, 64, 128, 5, 3, **v)
+    bar = max(2e-2, 1.5 * errs["default"][1] * max(1.0, canc["variant"] / canc["default"]))
+    print("bf16 end to end (loss, grads):", errs, "cancellation:", canc, "bar:", bar)
+    assert errs["variant"][0] <= 2e-2
+    assert errs["variant"][1] <= bar
+
+
+def test_default_variant_is_the_dgi_step():
+    """set_contrastive() with the defaults gives the same step, bit for bit."""
+    gs = _graphs(64)
+    _, a = _run(gs, 64, 256, {})
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=64, hidden_dim=256, seed=5)
+    b = m.step(g, 3, 0, want_loss=True, want_grads=True)
+    assert a["loss"] == b["loss"] and np.array_equal(a["grads"], b["grads"])
+    m.free(); g.free()
+
+
+@pytest.mark.parametrize("K", [2, 4])
+def test_shared_positive_equals_k_copies_at_gnmt_size(K):
+    """c34 = c20 at the bench's graph size (H = 256, tcgen05 GEMMs): one
+    positive branch + K samples vs the K-copies batch, same permutations."""
+    gs = [SG.cached("gnmt", 0)]
+    F, H, seed, step = 64, 256, 7, 2
+    _, a = _run(gs, F, H, dict(num_neg=K), seed, step)
+    gc = mars.graph_load(mars.corruption_samples(gs, K))
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=seed)
+    b = m.step(gc, step, 0, global_batch=K, want_loss=True, want_grads=True, want_perms=True)
+    m.free(); gc.free()
+    N = gs[0].num_nodes
+    assert np.array_equal(a["perms"], b["perms"])          # sample k = copy k, pair k
+    assert abs(a["loss"] - b["loss"]) / abs(b["loss"]) <= 1e-6
+    err = scaled_err(a["grads"], b["grads"])
+    print(f"K={K} N={N}: shared vs copies grads scaled err {err:.2e}")
+    assert err <= 1e-5
+
+
+def test_captured_replay_matches_eager():
+    """The captured step (second step on a set) replays the variant schedule."""
+    gs = _graphs(64)
+    variant = dict(num_neg=3, corruption="mask", mask_rate=0.3, aggregator="sage_gcn")
+    res = []
+    for cap in (True, False):
+        g = mars.graph_load(gs)
+        m = mars.dgi_create(in_dim=64, hidden_dim=128, seed=2)
+        m.set_graph_capture(cap)
+        m.set_contrastive(**variant)
+        losses = [m.step(g, s, 0, want_loss=True)["loss"] for s in range(4)]
+        res.append((losses, m.get_state()[0]))
+        m.free(); g.free()
+    assert res[0][0] == res[1][0]
+    assert np.array_equal(res[0][1], res[1][1])
+
+
+def test_sage_encode_and_vjp():
+    gs = _graphs(64)
+    F, H = 64, 128
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=4)
+    m.set_contrastive(aggregator="sage_gcn")
+    p0 = m.get_state()[0].astype(np.float64)
+    emb = m.encode(g)
+    ref = V.encode(gs, p0, F, H, aggregator="sage_gcn")
+    assert scaled_err(emb, ref) <= TOL
+    dE = np.random.default_rng(0).standard_normal(emb.shape).astype(np.float32)
+    got = m.encoder_vjp(g, dE)
+    p = torch.tensor(p0, requires_grad=True)
+    W1, W2, W3, _, al = V.unpack(p, F, H)
+    out, o = [], 0
+    for gr in gs:
+        An = torch.from_numpy(V.normalise(V.adjacency(gr), "sage_gcn"))
+        out.append(V.encoder(An, torch.tensor(np.asarray(gr.features, np.float64)), (W1, W2, W3), al))
+    (torch.cat(out) * torch.tensor(dE, dtype=torch.float64)).sum().backward()
+    assert scaled_err(got, p.grad.numpy()) <= TOL
+    m.free(); g.free()
+
+
+def test_variant_errors():
+    m = mars.dgi_create(in_dim=16, hidden_dim=32)
+    for bad in (dict(num_neg=0), dict(num_neg=65), dict(mask_rate=1.5, corruption="mask")):
+        with pytest.raises(mars.MarsError):
+            m.set_contrastive(**bad)
+    m.set_contrastive(corruption="mask", mask_rate=0.1)
+    g = mars.graph_load([SG.tiny(0)])
+    with pytest.raises(mars.MarsError):
+        m.step(g, 0, 0, want_perms=True)       # masking has no permutations
+    assert m.get_contrastive()["corruption"] == "mask"
+    m.free(); g.free()
