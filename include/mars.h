@@ -128,7 +128,22 @@ typedef struct {
                                  allreduce (optional with world_size 1: a 1-rank
                                  communicator).  NULL with world_size > 1: peer-memory
                                  exchange (mars_dp_export / mars_dp_connect below). */
+  int32_t encoder;            /* MARS_ENCODER_GCN (Eq. 1, default) or MARS_ENCODER_SAGE */
 } mars_dgi_config;
+
+/* The graph encoder (NEXT-4: "[33] uses GraphSAGE as the graph encoder",
+ * P:L222; reading c38).  MARS_ENCODER_SAGE: GraphSAGE with the mean
+ * aggregator and a root weight, per layer Z = H W_s + (Â_N H) W_n, Â_N =
+ * D_N^-1 (A v Aᵀ) over the neighbours without the node itself (an isolated
+ * node aggregates 0), PReLU as in Eq. 1, no bias.  Parameters [W1s F×H |
+ * W1n F×H | W2s | W2n | W3s | W3n (H×H each) | M H×H | α1 α2 α3]; default init
+ * U(-b, b), b = sqrt(6 / (2 C_in + H)) for both halves of a layer (Xavier on
+ * the concatenated [2 C_in × H] map), b = sqrt(6 / 2H) for M, tags 1..7 in
+ * layout order (c14's generator), α = 0.25.  MARS_FP32 only; not row-sharded;
+ * the contrastive variants apply except the SAGE-GCN aggregator; no
+ * mars_dgi_encoder_vjp (so no joint PPO update).  The hooks export, per layer,
+ * the GEMM input H_{l-1} (X~ stacked for layer 1) as "Y". */
+enum { MARS_ENCODER_GCN = 0, MARS_ENCODER_SAGE = 1 };
 
 /* Fills cfg with the defaults above (F = 64, H = 256, L = 3, FP32, seed 0,
  * device 0, world 1). */
@@ -139,6 +154,8 @@ MARS_API void mars_dgi_config_default(mars_dgi_config* cfg);
  * must call collectively); with world_size > 1 and no id allocates the
  * peer-visible buffers of the peer-memory exchange (connect before stepping). */
 MARS_API mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** out);
+/* Parameter count P of the model (mars_num_params for MARS_ENCODER_GCN). */
+MARS_API int64_t mars_dgi_num_params(const mars_dgi* m);
 /* Rank 0 only: writes a fresh 128-byte ncclUniqueId to out128. */
 MARS_API mars_status mars_nccl_get_unique_id(void* out128);
 /* Use `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream()) instead

@@ -19,6 +19,12 @@ discriminator, Eq. 6 loss -- with the variant's choices.  Readings
   c36  mean readout: s = (1/N) Σ_i h_i (no sigmoid).
   c37  SAGE-GCN aggregation: Â = D^-1 (A v Aᵀ + I), D the row sums (the
        GraphSAGE mean aggregator over the node and its neighbours).
+  c38  SAGE-mean encoder (GraphSAGE, mean aggregator with a root weight, no
+       bias): h' = PReLU(h W_s + (Â_N h) W_n), Â_N = D_N^-1 (A v Aᵀ) without
+       self loops (an isolated node aggregates 0); parameters [W1s | W1n | W2s |
+       W2n | W3s | W3n | M | α], init U(-b, b) with b = f32(sqrt(6 / (2 C_in +
+       H))) per layer (sqrt(6 / 2H) for M), tags 1..7 in layout order (c14's
+       generator), α = 0.25.
 
 The corruption permutations are oracle.perm's (the C oracle, c12).  Parity
 pins: tests/test_oracle_variants.py (the default variant against the C
@@ -82,6 +88,51 @@ def normalise(A: np.ndarray, aggregator: str) -> np.ndarray:
     raise ValueError(aggregator)
 
 
+def num_params(F: int, H: int, encoder: str = "gcn") -> int:
+    return F * H + 3 * H * H + 3 + (F * H + 2 * H * H if encoder == "sage" else 0)
+
+
+def sage_init(seed: int, F: int, H: int) -> np.ndarray:
+    """c38: W1s W1n W2s W2n W3s W3n M with c14's generator, tags 1..7."""
+    out = []
+    for t in range(1, 8):
+        fin = F if t <= 2 else H
+        fan = 2 * H if t == 7 else 2 * fin + H
+        b = float(np.float32(np.sqrt(6.0 / fan)))
+        base = np.uint64(_sm64((seed ^ t) & M64))
+        z = _sm64_np(base ^ np.arange(fin * H, dtype=np.uint64))
+        u = (z >> np.uint64(40)).astype(np.float64) * (1.0 / 16777216.0)
+        out.append(((2.0 * u - 1.0) * b).astype(np.float32))
+    out.append(np.full(3, 0.25, np.float32))
+    return np.concatenate(out)
+
+
+def unpack_sage(p, F: int, H: int):
+    """((W1s, W1n), (W2s, W2n), (W3s, W3n)), M, alpha (c38 layout)."""
+    o, mats = 0, []
+    for fin in (F, F, H, H, H, H, H):
+        mats.append(p[o:o + fin * H].view(fin, H))
+        o += fin * H
+    return ((mats[0], mats[1]), (mats[2], mats[3]), (mats[4], mats[5])), mats[6], p[o:o + 3]
+
+
+def neighbour_mean(g) -> np.ndarray:
+    """Â_N = D_N^-1 (A v Aᵀ), no self loops; rows of isolated nodes are 0 (c38)."""
+    A = adjacency(g)
+    np.fill_diagonal(A, 0.0)
+    d = A.sum(1)
+    return A / np.where(d > 0, d, 1.0)[:, None]
+
+
+def encoder_sage(AN, X, Wp, alpha):
+    """c38 x 3: h' = PReLU(h W_s + (Â_N h) W_n)."""
+    h = X
+    for l in range(3):
+        Ws, Wn = Wp[l]
+        h = torch.nn.functional.prelu(h @ Ws + AN @ (h @ Wn), alpha[l:l + 1])
+    return h
+
+
 def unpack(p, F: int, H: int):
     o = 0
     out = []
@@ -100,6 +151,9 @@ def encoder(An, X, W, alpha):
     return h
 
 
+_encoder_gcn = encoder        # (step_grads' `encoder` argument shadows the name)
+
+
 def corrupted(g, X, seed, step, pair, corruption, mask_rate):
     N, F = X.shape
     if corruption == "permute":      # Eq. 2, c12
@@ -113,25 +167,30 @@ def corrupted(g, X, seed, step, pair, corruption, mask_rate):
 def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: int = 0,
                B: float | None = None, num_neg: int = 1, corruption: str = "permute",
                mask_rate: float = 0.0, readout: str = "sigmoid_mean", aggregator: str = "gcn",
-               pair_off=None, sparse: bool = False):
-    """(loss, dL/dparams) of one step over a graph set (c34-c37).  B = number of
+               pair_off=None, sparse: bool = False, encoder: str = "gcn"):
+    """(loss, dL/dparams) of one step over a graph set (c34-c38).  B = number of
     graphs the loss is averaged over (default: len(graphs)); pair_off[g]
-    defaults to g.  sparse: Â as a torch sparse matrix (larger graphs)."""
+    defaults to g.  sparse: Â as a torch sparse matrix (larger graphs).
+    encoder "sage": the c38 encoder (aggregator unused)."""
     p = torch.tensor(np.asarray(params, np.float64), requires_grad=True)
-    W1, W2, W3, M, al = unpack(p, F, H)
-    W = (W1, W2, W3)
+    if encoder == "sage":
+        Wp, M, al = unpack_sage(p, F, H)
+        enc = lambda A_, X_: encoder_sage(A_, X_, Wp, al)   # noqa: E731
+    else:
+        W1, W2, W3, M, al = unpack(p, F, H)
+        enc = lambda A_, X_: _encoder_gcn(A_, X_, (W1, W2, W3), al)   # noqa: E731
     B = float(len(graphs) if B is None else B)
     K = int(num_neg)
     sp = torch.nn.functional.softplus
     loss = torch.zeros((), dtype=torch.float64)
     for gi, g in enumerate(graphs):
-        An_np = normalise(adjacency(g), aggregator)
+        An_np = neighbour_mean(g) if encoder == "sage" else normalise(adjacency(g), aggregator)
         An = torch.from_numpy(An_np)
         if sparse:
             An = An.to_sparse()
         X = torch.tensor(np.asarray(g.features, np.float64))
         N = g.num_nodes
-        Hp = encoder(An, X, W, al)
+        Hp = enc(An, X)
         m = Hp.mean(0)                                   # Eq. 4
         s = torch.sigmoid(m) if readout == "sigmoid_mean" else m
         if readout not in ("sigmoid_mean", "mean"):
@@ -142,18 +201,23 @@ def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: 
         po = gi if pair_off is None else int(pair_off[gi])
         for k in range(K):
             Xt = corrupted(g, X, seed, step, pair_base + po * K + k, corruption, mask_rate)
-            neg = neg + sp(encoder(An, Xt, W, al) @ v).sum()
+            neg = neg + sp(enc(An, Xt) @ v).sum()
         loss = loss + (pos + neg / K) / (2.0 * N) / B    # Eq. 6 with c34
     loss.backward()
     return float(loss.detach()), p.grad.numpy().copy()
 
 
-def encode(graphs, params, F: int, H: int, aggregator: str = "gcn"):
-    """a15 under the variant's aggregator: H3 of every node, stacked."""
+def encode(graphs, params, F: int, H: int, aggregator: str = "gcn", encoder_: str = "gcn"):
+    """a15 under the variant's aggregator / encoder: H3 of every node, stacked."""
     p = torch.tensor(np.asarray(params, np.float64))
-    W1, W2, W3, _, al = unpack(p, F, H)
     out = []
     for g in graphs:
-        An = torch.from_numpy(normalise(adjacency(g), aggregator))
-        out.append(encoder(An, torch.tensor(np.asarray(g.features, np.float64)), (W1, W2, W3), al))
+        X = torch.tensor(np.asarray(g.features, np.float64))
+        if encoder_ == "sage":
+            Wp, _, al = unpack_sage(p, F, H)
+            out.append(encoder_sage(torch.from_numpy(neighbour_mean(g)), X, Wp, al))
+        else:
+            W1, W2, W3, _, al = unpack(p, F, H)
+            An = torch.from_numpy(normalise(adjacency(g), aggregator))
+            out.append(encoder(An, X, (W1, W2, W3), al))
     return torch.cat(out).numpy()

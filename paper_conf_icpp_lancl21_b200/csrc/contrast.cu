@@ -13,6 +13,10 @@
 //   c37  SAGE-GCN aggregation: Â = D^-1 (A v Aᵀ + I) (row mean over the
 //        neighbourhood with the node itself); the backward uses Âᵀ, the same
 //        pattern with 1/deg of the column.
+//   c38  SAGE-mean encoder (GraphSAGE with a root weight): Z = H W_s +
+//        (Â_N H) W_n, Â_N = D_N^-1 (A v Aᵀ) without self loops; computed
+//        GEMM-first as Z_i = U_s[i] + Σ_j Â_N[i][j] U_n[j] (U = H [W_s | W_n])
+//        by ONE aggregation whose self entry is redirected to the U_s rows.
 // The corrupted inputs are materialised (one pass over X per block) and layer
 // 1 aggregates the stacked blocks like layers 2-3 (PReLU slope 1 = identity).
 #include "common.cuh"
@@ -84,7 +88,79 @@ __global__ void k_sage_vals(const int32_t* __restrict__ rowptr, const int32_t* _
   }
 }
 
+// SAGE-mean encoder (c38): per CSR entry k of row i with column j,
+//   colS[k] = j == i ? self_off + i : j         (self entry -> the root rows)
+//   vf[k]   = j == i ? 1 : 1/(deg_i - 1)        Z_i = U_s[i] + mean_j U_n[j]
+//   vb[k]   = j == i ? 1 : 1/(deg_j - 1)        its transpose (backward)
+//   vn[k]   = j == i ? 0 : 1/(deg_j - 1)        Â_Nᵀ alone (dW_n)
+// deg counts the self loop, so deg - 1 is the neighbour count (>= 1 for every
+// neighbour entry).
+__global__ void k_sage_csr(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
+                           int32_t Nt, int64_t self_off, int32_t* __restrict__ colS,
+                           float* __restrict__ vf, float* __restrict__ vb, float* __restrict__ vn) {
+  const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (wid >= Nt) return;
+  const int32_t i = (int32_t)wid;
+  const int32_t k0 = rowptr[i], k1 = rowptr[i + 1];
+  const float ri = k1 - k0 > 1 ? 1.0f / (float)(k1 - k0 - 1) : 0.f;
+  for (int32_t k = k0 + lane; k < k1; k += 32) {
+    const int32_t j = colind[k];
+    if (j == i) {
+      colS[k] = (int32_t)(self_off + i);
+      vf[k] = 1.f;
+      if (vb) vb[k] = 1.f;
+      if (vn) vn[k] = 0.f;
+    } else {
+      const float rj = 1.0f / (float)(rowptr[j + 1] - rowptr[j] - 1);
+      colS[k] = j;
+      vf[k] = ri;
+      if (vb) vb[k] = rj;
+      if (vn) vn[k] = rj;
+    }
+  }
+}
+
+// One warp per row of C columns: out = PReLU_a(in) (a = *slope; out may be
+// null) and the row's power-of-two scale (rs may be null) for the 3xFP16 GEMMs.
+__global__ void k_rowprep(const float* __restrict__ in, int64_t rows, int C,
+                          const float* __restrict__ slope, float* __restrict__ out,
+                          float* __restrict__ rs) {
+  const int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (r >= rows) return;
+  const float a = *slope;
+  float m = 0.f;
+  for (int c = lane * 4; c < C; c += 128) {
+    const float4 x = *reinterpret_cast<const float4*>(in + r * C + c);
+    const float4 y = make_float4(x.x > 0.f ? x.x : a * x.x, x.y > 0.f ? x.y : a * x.y,
+                                 x.z > 0.f ? x.z : a * x.z, x.w > 0.f ? x.w : a * x.w);
+    if (out) *reinterpret_cast<float4*>(out + r * C + c) = y;
+    m = fmaxf(m, fmaxf(fmaxf(fabsf(y.x), fabsf(y.y)), fmaxf(fabsf(y.z), fabsf(y.w))));
+  }
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if (rs && lane == 0) rs[r] = pow2_scale(m);
+}
+
 }  // namespace
+
+cudaError_t launch_sage_csr(const GraphDev& g, int64_t self_off, int32_t* colS, float* vf,
+                            float* vb, float* vn, cudaStream_t s, int* launches) {
+  count_launch(launches);
+  if (g.Nt > 0)
+    k_sage_csr<<<cdiv((int64_t)g.Nt * 32, 256), 256, 0, s>>>(g.rowptr, g.colind, g.Nt, self_off,
+                                                              colS, vf, vb, vn);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_rowprep(const float* in, int64_t rows, int C, const float* slope, float* out,
+                           float* rs, cudaStream_t s, int* launches) {
+  if (C % 4) return cudaErrorInvalidValue;
+  count_launch(launches);
+  if (rows > 0)
+    k_rowprep<<<cdiv(rows * 32, 256), 256, 0, s>>>(in, rows, C, slope, out, rs);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_pair_off_k(const int64_t* pair_off, int32_t G, int32_t K, int64_t* out,
                               cudaStream_t s, int* launches) {

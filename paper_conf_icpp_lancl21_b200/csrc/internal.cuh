@@ -285,6 +285,15 @@ cudaError_t launch_corrupt(const GraphDev& g, int32_t K, int32_t nb, int32_t cor
 // transpose on the same (symmetric) pattern.
 cudaError_t launch_sage_vals(const GraphDev& g, float* valsR, float* valsC, cudaStream_t s,
                              int* launches);
+// SAGE-mean encoder (c38): the redirected CSR (self entry -> row self_off + i
+// of the stacked [U_n; U_s] operand) with forward values (1 self, 1/deg_N(i)
+// neighbours), backward values (1, 1/deg_N(j)) and neighbour-only transpose
+// values (0, 1/deg_N(j)); vb / vn may be null.
+cudaError_t launch_sage_csr(const GraphDev& g, int64_t self_off, int32_t* colS, float* vf,
+                            float* vb, float* vn, cudaStream_t s, int* launches);
+// out = PReLU_{*slope}(in) row by row (out may be null) + power-of-two row scales (rs may be null).
+cudaError_t launch_rowprep(const float* in, int64_t rows, int C, const float* slope, float* out,
+                           float* rs, cudaStream_t s, int* launches);
 // grad[0] = Σ slots (fixed order, double)
 cudaError_t launch_reduce_slots(double* slots, int n, float* grad, cudaStream_t s,
                                 int* launches);

@@ -366,6 +366,15 @@ struct Workspace {
   int64_t* pair_off_k = nullptr;
   float *valsR = nullptr, *valsC = nullptr;
   float* one = nullptr;
+  // SAGE-mean encoder (c38): U = [U_n; U_s] and V = [V_n; V_s] ([2 nb Nt x H]),
+  // the redirected CSR (colS) and its three value arrays, G's row scales,
+  // the six weight matrices' 3xFP16 splits
+  float *sU = nullptr, *sV = nullptr;
+  int32_t* sColS = nullptr;
+  float *sVf = nullptr, *sVb = nullptr, *sVn = nullptr;
+  float* rsG = nullptr;
+  void *s3_wt_hi[6] = {}, *s3_wt_lo[6] = {}, *s3_w_hi[6] = {}, *s3_w_lo[6] = {};
+  float* s3_wsc[6] = {};
   std::vector<void*> owned;
   void release() {
     for (void* p : owned) cudaFree(p);
@@ -391,8 +400,11 @@ struct mars_dgi {
   Workspace ws;
   const mars_graph* ws_graph = nullptr;
   mars_contrastive ct{1, MARS_CORRUPT_PERMUTE, 0.f, MARS_READOUT_SIGMOID_MEAN, MARS_AGG_GCN};
+  bool sage = false;                // MARS_ENCODER_SAGE (c38)
   int ct_nb() const { return (ct.num_neg + 2) & ~1; }     // K + 1 blocks, rounded up to even
-  bool ct_materialise() const { return ct.num_neg > 1 || ct.corruption != MARS_CORRUPT_PERMUTE; }
+  bool ct_materialise() const {
+    return sage || ct.num_neg > 1 || ct.corruption != MARS_CORRUPT_PERMUTE;
+  }
   bool capture = true;
   int gemm_impl = 0;                // 0 auto (tcgen05 3xFP16 when supported), 1 SIMT FFMA
   // Captured steps, one per (graph set, stream), least recently used evicted:
@@ -981,6 +993,10 @@ extern "C" mars_status mars_featurize(const int32_t* types, const int64_t* dims,
 }
 
 // ---------------------------------------------------------------- model create
+extern "C" int64_t mars_dgi_num_params(const mars_dgi* m) {
+  return (m && m->tag == kTagDgi) ? m->P : -1;
+}
+
 extern "C" mars_status mars_nccl_get_unique_id(void* out128) {
   if (!out128) return fail(MARS_EINVAL, "out is NULL");
   if (!nccl_load()) return fail(MARS_ENCCL, "libnccl.so.2 not loadable");
@@ -1004,6 +1020,10 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
     return fail(MARS_EINVAL, "MARS_BF16 needs hidden_dim in {128, 256} and in_dim in {64, 128, 256}");
   if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
     return fail(MARS_EINVAL, "bad world_size/rank");
+  if (cfg->encoder != MARS_ENCODER_GCN && cfg->encoder != MARS_ENCODER_SAGE)
+    return fail(MARS_EINVAL, "unknown encoder %d", cfg->encoder);
+  if (cfg->encoder == MARS_ENCODER_SAGE && cfg->precision != MARS_FP32)
+    return fail(MARS_EINVAL, "the SAGE encoder runs MARS_FP32 only");
   if (cfg->world_size > kMaxShards && !cfg->nccl_unique_id)
     return fail(MARS_EINVAL, "peer-memory data parallelism supports world_size <= %d", kMaxShards);
   int ndev = 0;
@@ -1020,7 +1040,8 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   m->cfg.nccl_unique_id = nullptr;
   m->F = cfg->in_dim;
   m->H = cfg->hidden_dim;
-  m->P = mars_num_params(m->F, m->H);
+  m->sage = cfg->encoder == MARS_ENCODER_SAGE;
+  m->P = mars_num_params(m->F, m->H) + (m->sage ? (int64_t)m->F * m->H + 2LL * m->H * m->H : 0);
   CK(cudaStreamCreateWithFlags(&m->own_stream, cudaStreamNonBlocking));
   m->stream = m->own_stream;
   CK(dalloc(&m->params, m->P));
@@ -1043,12 +1064,24 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   CK(cudaMemsetAsync(m->adam_st, 0, sizeof(AdamDev), s));
   if (cfg->init_params) {
     CK(cudaMemcpyAsync(m->params, cfg->init_params, sizeof(float) * m->P, cudaMemcpyHostToDevice, s));
-  } else {
+  } else if (!m->sage) {
     int64_t off = 0;
     for (int t = 1; t <= 4; ++t) {
       int fin = t == 1 ? m->F : m->H;
       int64_t n = (int64_t)fin * m->H;
       float b = (float)std::sqrt(6.0 / (double)(fin + m->H));
+      k_xavier<<<cdiv(n, 256), 256, 0, s>>>(m->params + off, n, cfg->seed, (uint64_t)t, b);
+      off += n;
+    }
+    k_fill<<<1, 32, 0, s>>>(m->params + off, 3, 0.25f);
+    CK(cudaGetLastError());
+  } else {                         // c38: W1s W1n W2s W2n W3s W3n M, tags 1..7
+    int64_t off = 0;
+    for (int t = 1; t <= 7; ++t) {
+      const int fin = t <= 2 ? m->F : m->H;
+      const int64_t n = (int64_t)fin * m->H;
+      const double fan = t == 7 ? 2.0 * m->H : 2.0 * fin + m->H;
+      const float b = (float)std::sqrt(6.0 / fan);
       k_xavier<<<cdiv(n, 256), 256, 0, s>>>(m->params + off, n, cfg->seed, (uint64_t)t, b);
       off += n;
     }
@@ -1125,6 +1158,8 @@ extern "C" mars_status mars_dgi_set_contrastive(mars_dgi* m, const mars_contrast
   const bool dflt = c->num_neg == 1 && c->corruption == MARS_CORRUPT_PERMUTE &&
                     c->readout == MARS_READOUT_SIGMOID_MEAN && c->aggregator == MARS_AGG_GCN;
   if (m->sh.g && !dflt) return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
+  if (m->sage && c->aggregator != MARS_AGG_GCN)
+    return fail(MARS_EINVAL, "the SAGE encoder has its own aggregation (aggregator must be GCN)");
   CK(cudaSetDevice(m->cfg.device));
   m->drop_execs();                 // captured steps bake the variant in
   CK(cudaStreamSynchronize(m->stream));
@@ -1161,10 +1196,12 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   const GraphDev& pv = g->perm_view();
   const int nbk = m->ct_nb(), K = m->ct.num_neg;
   const bool xs = m->ct_materialise(), sage = m->ct.aggregator == MARS_AGG_SAGE_GCN;
+  const bool smean = m->sage;
   if (w.Nt >= g->dev.Nt && w.Nperm >= pv.Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks &&
       w.nbuckets >= pv.nbuckets && w.nnz_perm >= pv.nnz && w.nlong >= g->dev.nlong &&
       w.nseg >= g->dev.nseg && w.F == m->F && w.H == m->H && w.nb == nbk && w.K == K &&
-      (w.has_xs || !xs) && (!sage || w.nnz_vals >= g->dev.nnz))
+      (w.has_xs || !xs) && (!sage || w.nnz_vals >= g->dev.nnz) &&
+      (!smean || (w.sU && w.nnz_vals >= g->dev.nnz)))
     return MARS_OK;
   if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
   m->drop_execs();
@@ -1195,6 +1232,26 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   if (sage) {
     CK(al((void**)&w.valsR, sizeof(float) * (size_t)std::max<int64_t>(1, g->dev.nnz)));
     CK(al((void**)&w.valsC, sizeof(float) * (size_t)std::max<int64_t>(1, g->dev.nnz)));
+  }
+  if (smean) {
+    const size_t z = (size_t)std::max<int64_t>(1, g->dev.nnz);
+    CK(al((void**)&w.sU, sizeof(float) * 2 * R * H));
+    CK(al((void**)&w.sV, sizeof(float) * 2 * R * H));
+    CK(cudaMemset(w.sU, 0, sizeof(float) * 2 * R * H));    // padding rows stay zero
+    CK(cudaMemset(w.sV, 0, sizeof(float) * 2 * R * H));
+    CK(al((void**)&w.sColS, sizeof(int32_t) * z));
+    CK(al((void**)&w.sVf, sizeof(float) * z));
+    CK(al((void**)&w.sVb, sizeof(float) * z));
+    CK(al((void**)&w.sVn, sizeof(float) * z));
+    CK(al((void**)&w.rsG, sizeof(float) * R));
+    for (int t = 0; t < 6; ++t) {
+      const int64_t n = (int64_t)(t < 2 ? F : H) * H;
+      CK(al(&w.s3_wt_hi[t], 2 * n));
+      CK(al(&w.s3_wt_lo[t], 2 * n));
+      CK(al(&w.s3_w_hi[t], 2 * n));
+      CK(al(&w.s3_w_lo[t], 2 * n));
+      CK(al((void**)&w.s3_wsc[t], sizeof(float) * 2));
+    }
   }
   CK(al((void**)&w.one, sizeof(float)));
   {
@@ -1262,7 +1319,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   w.nb = nbk;
   w.K = K;
   w.has_xs = xs;
-  w.nnz_vals = sage ? g->dev.nnz : 0;
+  w.nnz_vals = (sage || smean) ? g->dev.nnz : 0;
   h.nb = nbk;
   h.K = K;
   h.readout = m->ct.readout;
@@ -1288,9 +1345,172 @@ struct Profiler {
   }
 };
 
+// The SAGE-mean encoder's step (c38, MARS_ENCODER_SAGE), GEMM-first per layer:
+//   A_0 = X~ stacked (materialised, c34/c35), A_l = PReLU(Z_l) (+ row scales)
+//   U_n = A W_n, U_s = A W_s                    (rows [0, R) / [nb Nt, nb Nt + R) of U)
+//   Z   = one aggregation over the redirected CSR: Z_i = U_s[i] + Σ_j U_n[j] / deg_N(i)
+// head as in the GCN step; backward per layer, from dZ:
+//   G   = Â_Nᵀ dZ (neighbour-only transpose; its row scales for the GEMM)
+//   dW_s = Aᵀ dZ, dW_n = Aᵀ G
+//   V_n = dZ W_nᵀ, V_s = dZ W_sᵀ; dZ_{l-1} = (V_s[i] + Σ_j V_n[j] / deg_N(j)) ⊙ PReLU'(Z_{l-1})
+//   (the same redirected CSR with the transpose's values, PReLU' and dα fused).
+static cudaError_t enqueue_step_sage(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl,
+                                     Profiler* prof) {
+  Workspace& w = m->ws;
+  GraphDev g = gr->dev;
+  g.long_part = w.long_part;
+  const int F = m->F, H = m->H;
+  const int nb = w.nb, K = m->ct.num_neg, nbp = nb / 2;
+  const int64_t Nt = g.Nt, Rb = (int64_t)nb * Nt, R = (int64_t)(K + 1) * Nt;
+  float* P = m->params;
+  float* Gd = m->grads;
+  const int64_t o1 = (int64_t)F * H, o2 = (int64_t)H * H;
+  // W[l][0] = W_ls, W[l][1] = W_ln (layout c38)
+  float* W[3][2] = {{P, P + o1}, {P + 2 * o1, P + 2 * o1 + o2}, {P + 2 * o1 + 2 * o2, P + 2 * o1 + 3 * o2}};
+  float* gW[3][2] = {{Gd, Gd + o1}, {Gd + 2 * o1, Gd + 2 * o1 + o2},
+                     {Gd + 2 * o1 + 2 * o2, Gd + 2 * o1 + 3 * o2}};
+  float* Mp = P + 2 * o1 + 4 * o2;
+  float* alpha = Mp + o2;
+  float* gM = Gd + 2 * o1 + 4 * o2;
+  float* galpha = gM + o2;
+  float* gloss = Gd + m->P;
+  float* A[3] = {w.Xs, w.Y23[0], w.Y23[1]};       // GEMM inputs of the three layers
+  cudaError_t e;
+#define RET(x)                                  \
+  do {                                          \
+    if ((e = (x)) != cudaSuccess) return e;     \
+  } while (0)
+#define MARK(ph)                                \
+  do {                                          \
+    if (prof) RET(prof->mark(ph, s));           \
+  } while (0)
+  MARK(-1);
+  w.hw.nb = nb;
+  w.hw.K = K;
+  w.hw.readout = m->ct.readout;
+  // corrupted inputs + the redirected CSR (self entry -> row Rb + i)
+  RET(launch_pair_off_k(g.pair_off, g.G, K, w.pair_off_k, s, nl));
+  if (m->ct.corruption == MARS_CORRUPT_PERMUTE)
+    for (int k = 0; k < K; ++k) {
+      GraphDev pv = g;
+      pv.pair_off = w.pair_off_k + (int64_t)k * g.G;
+      RET(launch_perm(pv, m->cfg.seed, m->d_sp, w.pw, w.perm + (int64_t)k * Nt, s, nl));
+    }
+  RET(launch_corrupt(g, K, nb, m->ct.corruption, m->ct.mask_rate, m->cfg.seed, m->d_sp,
+                     w.pair_off_k, w.perm, w.Xs, s, nl));
+  RET(launch_sage_csr(g, Rb, w.sColS, w.sVf, w.sVb, w.sVn, s, nl));
+  MARK(MARS_PH_PERM);
+  GraphDev gf = g, gbk = g, gn = g;
+  gf.colind = w.sColS;
+  gf.vals = w.sVf;
+  gbk.colind = w.sColS;
+  gbk.vals = w.sVb;
+  gn.vals = w.sVn;
+  bool tc[3];
+  for (int l = 0; l < 3; ++l) {
+    const int Cin = l == 0 ? F : H;
+    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
+    if (tc[l])
+      for (int h = 0; h < 2; ++h) {
+        const int t = 2 * l + h;
+        RET(tc3h_split_weights(W[l][h], Cin, H, w.s3_wsc[t], w.s3_wt_hi[t], w.s3_wt_lo[t],
+                               w.s3_w_hi[t], w.s3_w_lo[t], s, nl));
+      }
+  }
+  MARK(MARS_PH_GEMM_FWD);
+  float* U[2] = {w.sU + Rb * H, w.sU};           // [0]: U_s, [1]: U_n
+  float* Vv[2] = {w.sV + Rb * H, w.sV};          // [0]: V_s, [1]: V_n
+  auto blk = [&](float* base, int p, int C) { return base + (int64_t)2 * p * Nt * C; };
+  // forward
+  for (int l = 0; l < 3; ++l) {
+    const int Cin = l == 0 ? F : H;
+    if (l == 0) {
+      if (tc[0]) RET(launch_rowprep(w.Xs, R, F, w.one, nullptr, w.h3_rsY[0], s, nl));
+    } else {
+      RET(launch_rowprep(w.Z[l - 1], R, H, alpha + (l - 1), A[l], tc[l] ? w.h3_rsY[l] : nullptr,
+                         s, nl));
+    }
+    for (int h = 0; h < 2; ++h) {
+      const int t = 2 * l + h;
+      if (tc[l])
+        RET(tc3h_gemm_rows(A[l], w.h3_rsY[l], w.s3_wt_hi[t], w.s3_wt_lo[t], w.s3_wsc[t] + 1, U[h],
+                           R, H, Cin, s, nl));
+      else RET(gemm_nn(A[l], W[l][h], U[h], R, H, Cin, s, nl));
+    }
+    MARK(MARS_PH_GEMM_FWD);
+    for (int p = 0; p < nbp; ++p)
+      RET(launch_spmm_fwd(gf, H, blk(w.sU, p, H), 0, nullptr, w.one, 0, blk(w.Z[l], p, H), 0,
+                          2 * p + 1 <= K, s, nl, nullptr, nullptr));
+    MARK(MARS_PH_SPMM_FWD);
+  }
+  // head (a8-a11) -> dZ3
+  int ns = 0;
+  w.hw.rs_dz3 = tc[2] ? w.h3_rsdZ : nullptr;
+  RET(launch_head(g, H, w.Z[2], 0, Mp, alpha, m->d_sp, w.hw, w.dZ, gM, gloss, &ns, s, nl, nullptr));
+  RET(launch_reduce_slots(w.slots[2], ns, galpha + 2, s, nl));
+  MARK(MARS_PH_HEAD);
+  // backward
+  for (int l = 2; l >= 0; --l) {
+    const int Cin = l == 0 ? F : H;
+    for (int p = 0; p < nbp; ++p)        // G = Â_Nᵀ dZ
+      RET(launch_spmm_fwd(gn, H, blk(w.dZ, p, H), 0, nullptr, w.one, 0, blk(w.dY, p, H), 0,
+                          2 * p + 1 <= K, s, nl, nullptr, tc[l] ? w.rsG + 2LL * p * Nt : nullptr));
+    MARK(MARS_PH_SPMM_BWD);
+    if (tc[l]) {
+      RET(tc3h_gemm_dw(A[l], w.h3_rsY[l], w.dZ, w.h3_rsdZ, gW[l][0], R, Cin, H, w.dw_part, s, nl));
+      RET(tc3h_gemm_dw(A[l], w.h3_rsY[l], w.dY, w.rsG, gW[l][1], R, Cin, H, w.dw_part, s, nl));
+    } else {
+      RET(gemm_tn(A[l], w.dZ, gW[l][0], R, Cin, H, w.tn_part, s, nl));
+      RET(gemm_tn(A[l], w.dY, gW[l][1], R, Cin, H, w.tn_part, s, nl));
+    }
+    MARK(MARS_PH_GEMM_DW);
+    if (l > 0) {
+      for (int h = 0; h < 2; ++h) {
+        const int t = 2 * l + h;
+        if (tc[l])
+          RET(tc3h_gemm_rows(w.dZ, w.h3_rsdZ, w.s3_w_hi[t], w.s3_w_lo[t], w.s3_wsc[t] + 1, Vv[h], R,
+                             Cin, H, s, nl));
+        else RET(gemm_nt(w.dZ, W[l][h], Vv[h], R, Cin, H, s, nl));
+      }
+      MARK(MARS_PH_GEMM_DY);
+      ns = 0;
+      for (int p = 0; p < nbp; ++p) {
+        int nsp = 0;
+        RET(launch_spmm_bwd(gbk, Cin, blk(w.sV, p, Cin), blk(w.Z[l - 1], p, Cin), 0, alpha, l - 1,
+                            blk(w.dZ, p, Cin), w.slots[l - 1] + ns, &nsp, s, nl, nullptr,
+                            tc[l - 1] ? w.h3_rsdZ + 2LL * p * Nt : nullptr));
+        ns += nsp;
+      }
+      MARK(MARS_PH_SPMM_BWD);
+      RET(launch_reduce_slots(w.slots[l - 1], ns, galpha + (l - 1), s, nl));
+      MARK(MARS_PH_REDUCE);
+    }
+  }
+  if (m->comm) {
+    ncclResult_t r = g_nccl.AllReduce(m->grads, m->grads, (size_t)(m->P + 1), ncclFloat32, ncclSum,
+                                      m->comm, s);
+    if (r != ncclSuccess) return cudaErrorUnknown;
+    MARK(MARS_PH_ALLREDUCE);
+  }
+  if (m->dp.connected) {
+    RET(launch_shard_barrier(m->dp.sync, s, nl));
+    RET(launch_grad_sum(m->dp.grads, m->dp.R, m->dp.me, m->P + 1, 0, 0, 1, m->dp.gsum, s, nl));
+    RET(launch_shard_barrier(m->dp.sync, s, nl));
+    MARK(MARS_PH_ALLREDUCE);
+  }
+  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads_final(), m->P, m->cfg.lr,
+                  m->cfg.beta1, m->cfg.beta2, m->cfg.eps, m->cfg.clip_norm, m->guard_part,
+                  m->adam_st, s, nl));
+  MARK(MARS_PH_ADAM);
+#undef MARK
+#undef RET
+  return cudaSuccess;
+}
+
 // Enqueues one full DGI step (a4-a14) on stream s.  Reads step scalars from m->d_sp.
 static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl,
                                 Profiler* prof = nullptr) {
+  if (m->sage) return enqueue_step_sage(m, gr, s, nl, prof);
   Workspace& w = m->ws;
   GraphDev g = gr->dev;
   g.long_part = w.long_part;
@@ -1723,7 +1943,55 @@ extern "C" int64_t mars_dgi_last_launches(const mars_dgi* m) {
 // ---------------------------------------------------------------- encode (a15)
 // Forward of the positive branch only (a15): Y_l, Z_l of rows [0, ΣN) and
 // H3 = PReLU(Z3) into w.dY (the embeddings, device).
+// a15 under the SAGE-mean encoder (c38): the positive branch only, the
+// redirected CSR's self entries pointing at row Nt + i of [U_n; U_s].
+static cudaError_t enqueue_encode_sage(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl) {
+  Workspace& w = m->ws;
+  GraphDev g = gr->dev;
+  g.long_part = w.long_part;
+  const int F = m->F, H = m->H;
+  const int64_t Nt = g.Nt, o1 = (int64_t)F * H, o2 = (int64_t)H * H;
+  float* P = m->params;
+  float* W[3][2] = {{P, P + o1}, {P + 2 * o1, P + 2 * o1 + o2}, {P + 2 * o1 + 2 * o2, P + 2 * o1 + 3 * o2}};
+  float* alpha = P + 2 * o1 + 5 * o2;
+  const float* A[3] = {g.X, w.Y23[0], w.Y23[1]};
+  float* U[2] = {w.sU + Nt * H, w.sU};
+  cudaError_t e;
+  if ((e = launch_sage_csr(g, Nt, w.sColS, w.sVf, nullptr, nullptr, s, nl))) return e;
+  GraphDev gf = g;
+  gf.colind = w.sColS;
+  gf.vals = w.sVf;
+  for (int l = 0; l < 3; ++l) {
+    const int Cin = l == 0 ? F : H;
+    const bool tc = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
+    if (l == 0) {
+      if (tc && (e = launch_rowprep(g.X, Nt, F, w.one, nullptr, w.h3_rsY[0], s, nl))) return e;
+    } else if ((e = launch_rowprep(w.Z[l - 1], Nt, H, alpha + (l - 1), w.Y23[l - 1],
+                                   tc ? w.h3_rsY[l] : nullptr, s, nl))) {
+      return e;
+    }
+    for (int h = 0; h < 2; ++h) {
+      const int t = 2 * l + h;
+      if (tc) {
+        if ((e = tc3h_split_weights(W[l][h], Cin, H, w.s3_wsc[t], w.s3_wt_hi[t], w.s3_wt_lo[t],
+                                    w.s3_w_hi[t], w.s3_w_lo[t], s, nl)))
+          return e;
+        if ((e = tc3h_gemm_rows(A[l], w.h3_rsY[l], w.s3_wt_hi[t], w.s3_wt_lo[t], w.s3_wsc[t] + 1,
+                                U[h], Nt, H, Cin, s, nl)))
+          return e;
+      } else if ((e = gemm_nn(A[l], W[l][h], U[h], Nt, H, Cin, s, nl))) {
+        return e;
+      }
+    }
+    if ((e = launch_spmm_fwd(gf, H, w.sU, 0, nullptr, w.one, 0, w.Z[l], 0, 0, s, nl, nullptr,
+                             nullptr)))
+      return e;
+  }
+  return launch_prelu(w.Z[2], 0, alpha, 2, w.dY, Nt * H, s, nl);
+}
+
 static cudaError_t enqueue_encode(mars_dgi* m, const mars_graph* g, cudaStream_t s, int* nl) {
+  if (m->sage) return enqueue_encode_sage(m, g, s, nl);
   Workspace& w = m->ws;
   GraphDev gd = g->dev;
   gd.long_part = w.long_part;
@@ -1879,7 +2147,7 @@ extern "C" mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t la
   CK(cudaSetDevice(m->cfg.device));
   CK(cudaStreamSynchronize(m->stream));
   int64_t R = 2LL * m->last_Nt;
-  const float* Ys[3] = {m->ws.Y1, m->ws.Y23[0], m->ws.Y23[1]};
+  const float* Ys[3] = {m->sage ? m->ws.Xs : m->ws.Y1, m->ws.Y23[0], m->ws.Y23[1]};
   int Cin = layer == 1 ? m->F : m->H;
   if (m->cfg.precision == MARS_BF16) {     // upcast bf16 storage through a scratch buffer
     float* tmp = nullptr;
@@ -1909,6 +2177,7 @@ extern "C" mars_status mars_dgi_saved_rows(const mars_dgi* m, int64_t* rows) {
 
 extern "C" mars_status mars_dgi_set_keep_backward(mars_dgi* m, int32_t keep) {
   if (mars_status st = check_dgi(m)) return st;
+  if (m->sage && keep) return fail(MARS_EINVAL, "no backward hook for the SAGE encoder");
   CK(cudaSetDevice(m->cfg.device));
   m->drop_execs();                 // recapture with / without the copies
   CK(cudaStreamSynchronize(m->stream));
@@ -2253,6 +2522,7 @@ extern "C" mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g) {
   if (mars_status st = check_graph(g)) return st;
   if (!g->sharded) return fail(MARS_EINVAL, "graph was not loaded with mars_graph_load_shard");
   if (m->sh.g) return fail(MARS_ESTATE, "model already attached to a shard");
+  if (m->sage) return fail(MARS_EINVAL, "row sharding runs the GCN encoder only");
   if (m->ct.num_neg != 1 || m->ct.corruption != MARS_CORRUPT_PERMUTE ||
       m->ct.readout != MARS_READOUT_SIGMOID_MEAN || m->ct.aggregator != MARS_AGG_GCN)
     return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
@@ -2928,6 +3198,7 @@ extern "C" mars_status mars_dgi_encoder_vjp(mars_dgi* m, const mars_graph* g, co
   if (!dE || !grads) return fail(MARS_EINVAL, "NULL argument");
   if (g->sharded || g->F != m->F) return fail(MARS_EINVAL, "unsharded graph of the model's F");
   if (m->cfg.precision != MARS_FP32) return fail(MARS_EINVAL, "fp32 models only");
+  if (m->sage) return fail(MARS_EINVAL, "no encoder VJP for the SAGE encoder");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
   cudaStream_t s = m->stream;
@@ -2994,6 +3265,7 @@ extern "C" mars_status mars_ppo_create(mars_placer* p, mars_dgi* enc, const mars
   if (enc) {
     if (mars_status st = check_dgi(enc)) return st;
     if (enc->H != p->d.H) return fail(MARS_EINVAL, "encoder hidden_dim != placer in_dim");
+    if (enc->sage) return fail(MARS_EINVAL, "the joint update needs the GCN encoder (no SAGE VJP)");
     if (enc->cfg.device != p->cfg.device) return fail(MARS_EINVAL, "encoder and placer on different devices");
   }
   if (!cfg) return fail(MARS_EINVAL, "NULL config");

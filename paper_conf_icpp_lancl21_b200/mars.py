@@ -46,7 +46,8 @@ class DgiConfig(ctypes.Structure):
                 ("eps", ctypes.c_double), ("clip_norm", ctypes.c_double),
                 ("seed", ctypes.c_uint64), ("init_params", ctypes.c_void_p),
                 ("device", ctypes.c_int32), ("world_size", ctypes.c_int32),
-                ("rank", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p)]
+                ("rank", ctypes.c_int32), ("nccl_unique_id", ctypes.c_void_p),
+                ("encoder", ctypes.c_int32)]
 
 
 class PlacerConfig(ctypes.Structure):
@@ -76,6 +77,7 @@ class Contrastive(ctypes.Structure):
 CORRUPTIONS = {"permute": 0, "mask": 1}
 READOUTS = {"sigmoid_mean": 0, "mean": 1}
 AGGREGATORS = {"gcn": 0, "sage_gcn": 1}
+ENCODERS = {"gcn": 0, "sage": 1}
 
 
 class StepOut(ctypes.Structure):
@@ -96,6 +98,7 @@ SIGNATURES = {
     "mars_graph_export_csr": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32] + [ctypes.c_void_p] * 5),
     "mars_dgi_config_default": (None, [ctypes.POINTER(DgiConfig)]),
     "mars_dgi_create": (ctypes.c_int, [ctypes.POINTER(DgiConfig), ctypes.POINTER(ctypes.c_void_p)]),
+    "mars_dgi_num_params": (ctypes.c_int64, [ctypes.c_void_p]),
     "mars_nccl_get_unique_id": (ctypes.c_int, [ctypes.c_void_p]),
     "mars_dgi_set_stream": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
     "mars_dgi_set_graph_capture": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int32]),
@@ -420,7 +423,7 @@ class DGI:
     def __init__(self, handle, F, H):
         self.handle = handle
         self.F, self.H = F, H
-        self.P = num_params(F, H)
+        self.P = int(lib().mars_dgi_num_params(handle))
         self.num_neg = 1
         self.corruption = "permute"
 
@@ -552,8 +555,9 @@ class DGI:
 
 def dgi_create(in_dim=64, hidden_dim=256, precision=MARS_FP32, lr=1e-3, beta1=0.9, beta2=0.999,
                eps=1e-8, clip_norm=0.0, seed=0, init_params=None, device=0, world_size=1, rank=0,
-               nccl_unique_id: bytes | None = None) -> DGI:
+               nccl_unique_id: bytes | None = None, encoder: str = "gcn") -> DGI:
     c = config_default()
+    c.encoder = ENCODERS[encoder]
     c.in_dim, c.hidden_dim, c.num_layers, c.precision = in_dim, hidden_dim, 3, precision
     c.lr, c.beta1, c.beta2, c.eps, c.clip_norm = lr, beta1, beta2, eps, clip_norm
     c.seed = seed & (2 ** 64 - 1)

@@ -1,10 +1,12 @@
-"""Pins for the NEXT-4 variant oracle (oracle/variants.py; readings c34-c37):
+"""Pins for the NEXT-4 variant oracle (oracle/variants.py; readings c34-c38):
 the default variant against the C oracle's step, K shared-positive samples
 against the C oracle on K copies of each graph (c20), feature masking at rates
 0 and 1 in closed form, the readouts against the C oracle's encoder plus a
 hand-written numpy head, the SAGE-GCN encoder against brute-force loops and
-its constant-feature special case, and every variant's gradient against
-central finite differences."""
+its constant-feature special case, the SAGE-mean encoder (c38) against
+brute-force loops, its W_n = 0 and constant-feature special cases and its
+init layout, and every variant's gradient against central finite
+differences."""
 import math
 from types import SimpleNamespace
 
@@ -184,4 +186,118 @@ def test_variant_gradients_finite_differences(kw):
         pm[i] -= h
         fd = (V.step_grads(gs, pp, F, H, SEED, STEP, **kw)[0]
               - V.step_grads(gs, pm, F, H, SEED, STEP, **kw)[0]) / (2 * h)
+        assert abs(fd - grads[i]) <= 1e-7 + 1e-5 * abs(grads[i]), (i, fd, grads[i])
+
+
+# ----------------------------------------------------------------- SAGE-mean (c38)
+def _sage_params(seed=21):
+    return V.sage_init(seed, F, H).astype(np.float64)
+
+
+def _sage_blocks(p):
+    o, mats = 0, []
+    for fin in (F, F, H, H, H, H):
+        mats.append(p[o:o + fin * H].reshape(fin, H))
+        o += fin * H
+    return [(mats[0], mats[1]), (mats[2], mats[3]), (mats[4], mats[5])], p[-3:]
+
+
+def test_sage_init_layout_and_bounds():
+    p = V.sage_init(3, F, H)
+    assert p.size == V.num_params(F, H, "sage") == F * H + 3 * H * H + 3 + F * H + 2 * H * H
+    o = 0
+    for t, fin in enumerate((F, F, H, H, H, H, H), start=1):
+        blk = p[o:o + fin * H]
+        b = np.float32(np.sqrt(6.0 / (2 * H if t == 7 else 2 * fin + H)))
+        assert np.all(np.abs(blk) <= b) and np.std(blk) > 0.5 * b / np.sqrt(3)
+        o += fin * H
+    assert np.array_equal(p[-3:], np.full(3, 0.25, np.float32))
+    # W_s and W_n of a layer are different draws
+    assert not np.array_equal(p[:F * H], p[F * H:2 * F * H])
+
+
+def test_sage_mean_encoder_brute_force_loops():
+    """c38 as per-node loops: h_i' = PReLU(h_i W_s + mean_{j in N(i)} h_j W_n),
+    N(i) the neighbours without i; a node without neighbours aggregates 0."""
+    g = SG.tiny(5, N=26)
+    p = _sage_params()
+    Wp, al = _sage_blocks(p)
+    nb = [set() for _ in range(g.num_nodes)]
+    for u in range(g.num_nodes):
+        for e in range(int(g.indptr[u]), int(g.indptr[u + 1])):
+            v = int(g.indices[e])
+            if v != u:
+                nb[u].add(v)
+                nb[v].add(u)
+    h = np.asarray(g.features, np.float64)
+    for l in range(3):
+        out = np.zeros((g.num_nodes, H))
+        for i in range(g.num_nodes):
+            agg = sum(h[j] for j in sorted(nb[i])) / len(nb[i]) if nb[i] else np.zeros(h.shape[1])
+            out[i] = _prelu(h[i] @ Wp[l][0] + agg @ Wp[l][1], al[l])
+        h = out
+    got = V.encode([g], p, F, H, encoder_="sage")
+    assert np.max(np.abs(got - h)) < 1e-12 * max(1.0, np.max(np.abs(h)))
+
+
+def test_sage_special_cases():
+    """W_n = 0: the graph drops out (a per-node 3-layer PReLU MLP with W_s).
+    Constant feature rows: the neighbour mean is the row itself, so a node with
+    neighbours is the MLP with W_s + W_n and an isolated node the MLP with W_s."""
+    g = SG.tiny(6, N=30)
+    p = _sage_params(4)
+    Wp, al = _sage_blocks(p)
+
+    def mlp(x, mats):
+        h = x
+        for l, Wl in enumerate(mats):
+            h = _prelu(h @ Wl, al[l])
+        return h
+    X = np.asarray(g.features, np.float64)
+    q = p.copy()                             # zero the W_n blocks
+    offs, o = [], 0
+    for fin in (F, F, H, H, H, H):
+        offs.append((o, fin))
+        o += fin * H
+    for k in (1, 3, 5):
+        q[offs[k][0]:offs[k][0] + offs[k][1] * H] = 0.0
+    got = V.encode([g], q, F, H, encoder_="sage")
+    want = mlp(X.astype(np.float32).astype(np.float64), [w[0] for w in Wp])
+    assert np.max(np.abs(got - want)) < 1e-12 * max(1.0, np.max(np.abs(want)))
+    # constant rows; node 0 made isolated by removing its edges
+    x = np.random.default_rng(2).standard_normal(F).astype(np.float32)
+    N = g.num_nodes
+    keep = [(u, int(g.indices[e])) for u in range(N)
+            for e in range(int(g.indptr[u]), int(g.indptr[u + 1]))
+            if u != 0 and int(g.indices[e]) != 0]
+    indptr = np.zeros(N + 1, np.int64)
+    for u, _ in keep:
+        indptr[u + 1] += 1
+    gi = SimpleNamespace(num_nodes=N, indptr=np.cumsum(indptr),
+                         indices=np.array([v for _, v in keep], np.int32),
+                         features=np.tile(x, (N, 1)))
+    got = V.encode([gi], p, F, H, encoder_="sage")
+    both = mlp(x.astype(np.float64), [w[0] + w[1] for w in Wp])
+    root = mlp(x.astype(np.float64), [w[0] for w in Wp])
+    deg = V.neighbour_mean(gi).sum(1)
+    for i in range(N):
+        want = both if deg[i] > 0 else root
+        assert np.max(np.abs(got[i] - want)) < 1e-12 * max(1.0, np.max(np.abs(want)))
+    assert deg[0] == 0
+
+
+@pytest.mark.parametrize("kw", [dict(), dict(num_neg=2, corruption="mask", mask_rate=0.3),
+                                dict(readout="mean", num_neg=3)])
+def test_sage_gradients_finite_differences(kw):
+    gs, p = [SG.tiny(7, N=17)], _sage_params(8)
+    _, grads = V.step_grads(gs, p, F, H, SEED, STEP, encoder="sage", **kw)
+    rng = np.random.default_rng(3)
+    idx = list(rng.choice(p.size - 3, 6, replace=False)) + [F * H + 5, p.size - 2]
+    for i in idx:
+        h = 1e-5
+        pp, pm = p.copy(), p.copy()
+        pp[i] += h
+        pm[i] -= h
+        fd = (V.step_grads(gs, pp, F, H, SEED, STEP, encoder="sage", **kw)[0]
+              - V.step_grads(gs, pm, F, H, SEED, STEP, encoder="sage", **kw)[0]) / (2 * h)
         assert abs(fd - grads[i]) <= 1e-7 + 1e-5 * abs(grads[i]), (i, fd, grads[i])

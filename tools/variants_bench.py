@@ -2,7 +2,8 @@
 (GNMT x16 per GPU, F = 64, H = 256, fp32): the default DGI step, K = 4
 corruption samples with ONE positive branch (c34) against the same K samples
 run as K copies of every graph (c20, the positive branch recomputed K times),
-feature masking, the mean readout and SAGE-GCN aggregation.  CUDA events on the
+feature masking, the mean readout, SAGE-GCN aggregation and the SAGE-mean
+encoder (c38).  CUDA events on the
 library's stream around `steps` captured steps after a warm-up; inputs larger
 than L2.  Prints one JSON line per case."""
 import json
@@ -20,9 +21,9 @@ stream = torch.cuda.Stream()
 torch.cuda.set_stream(stream)
 
 
-def run(name, graphs, variant, batch):
+def run(name, graphs, variant, batch, encoder="gcn"):
     g = mars.graph_load(graphs)
-    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=1)
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=1, encoder=encoder)
     m.set_stream(stream.cuda_stream)
     m.set_contrastive(**variant)
     for s in range(warm):
@@ -51,3 +52,5 @@ run("K=2 shared positive", base, dict(num_neg=2), B)
 run("mask 0.2", base, dict(corruption="mask", mask_rate=0.2), B)
 run("readout mean", base, dict(readout="mean"), B)
 run("SAGE-GCN", base, dict(aggregator="sage_gcn"), B)
+run("SAGE-mean encoder", base, {}, B, encoder="sage")
+run("SAGE-mean encoder, K=3", base, dict(num_neg=3), B, encoder="sage")
