@@ -656,7 +656,10 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 // (tempty) barrier; the odd CTA's converters (folders) first meet at a named
 // barrier, then ONE thread arrives on the even CTA's barrier (remote arrive).
 // Scaling, folding and the partial layout are those of k_tc3h_dw.
-constexpr int kPairStages = 6;
+#ifndef MARS_PAIR_STAGES
+#define MARS_PAIR_STAGES 6
+#endif
+constexpr int kPairStages = MARS_PAIR_STAGES;
 
 struct H3PairCfg {
   static constexpr int ATOM = 64 * kDwBK * 2;          // fp16 MN atom column: 64 cols x 16 rows
