@@ -307,14 +307,16 @@ def run_mine(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
-    ev0.record(stream)
+    # one event between consecutive steps: the whole region for the value, the
+    # per-step spread for the p10 / p50 / p90 report
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    evs[0].record(stream)
     for k in range(args.steps):
         m.step(g, args.warmup + k, base, B)
-    ev1.record(stream)
-    ev1.synchronize()
-    ms = ev0.elapsed_time(ev1)
+        evs[k + 1].record(stream)
+    evs[-1].synchronize()
+    ms = evs[0].elapsed_time(evs[-1])
+    step_ms = np.array([evs[k].elapsed_time(evs[k + 1]) for k in range(args.steps)])
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -487,6 +489,7 @@ def run_mine(args):
             for w in range(args.warmup):
                 m16.step(g, w, base, B)
             torch.cuda.synchronize()
+            ev0, ev1 = evs[0], evs[-1]
             ev0.record(stream)
             for k in range(args.steps):
                 m16.step(g, args.warmup + k, base, B)
@@ -571,6 +574,10 @@ def run_mine(args):
                 "roofline": roof, "rooflines": rooflines, "spmm": spmm_obj,
                 "phases_ms_per_step": per_step, "phase_share": shares,
                 "profiled_step_ms": prof_total / nprof,
+                "step_ms_percentiles": {"p10": float(np.percentile(step_ms, 10)),
+                                        "p50": float(np.percentile(step_ms, 50)),
+                                        "p90": float(np.percentile(step_ms, 90)),
+                                        "of": "rank 0's timed steps (events between steps)"},
                 "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "gpu_launches": launches,
                 "bf16": b16}
         print(json.dumps(line), flush=True)

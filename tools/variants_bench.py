@@ -51,6 +51,8 @@ print(json.dumps({"shared_over_copies_speedup": copies / shared}), flush=True)
 run("K=2 shared positive", base, dict(num_neg=2), B)
 run("mask 0.2", base, dict(corruption="mask", mask_rate=0.2), B)
 run("readout mean", base, dict(readout="mean"), B)
+run("InfoNCE", base, dict(loss="infonce"), B)
+run("InfoNCE, K=4", base, dict(num_neg=4, loss="infonce"), B)
 run("SAGE-GCN", base, dict(aggregator="sage_gcn"), B)
 run("SAGE-mean encoder", base, {}, B, encoder="sage")
 run("SAGE-mean encoder, K=3", base, dict(num_neg=3), B, encoder="sage")
