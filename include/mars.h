@@ -193,16 +193,22 @@ MARS_API mars_status mars_dgi_set_graph_capture(mars_dgi* m, int32_t enable);
  *               MARS_AGG_SAGE_GCN: Â = D^-1 (A v Aᵀ + I), the GraphSAGE mean
  *               aggregator over the node and its neighbours (c37); the
  *               backward uses Âᵀ.  mars_encode / mars_dgi_encoder_vjp follow it.
- * The default {1, PERMUTE, 0, SIGMOID_MEAN, GCN} is the paper's DGI step. */
+ *   loss        MARS_LOSS_BCE: Eq. 6 (default); MARS_LOSS_INFONCE: per node, its
+ *               positive score against its K corrupted counterparts, L = (1/B)
+ *               Σ_g (1/N) Σ_i [log Σ_{k=0..K} e^{l_ik} - l_i0] (k = 0 the
+ *               positive, c39).
+ * The default {1, PERMUTE, 0, SIGMOID_MEAN, GCN, BCE} is the paper's DGI step. */
 enum { MARS_CORRUPT_PERMUTE = 0, MARS_CORRUPT_MASK = 1 };
 enum { MARS_READOUT_SIGMOID_MEAN = 0, MARS_READOUT_MEAN = 1 };
 enum { MARS_AGG_GCN = 0, MARS_AGG_SAGE_GCN = 1 };
+enum { MARS_LOSS_BCE = 0, MARS_LOSS_INFONCE = 1 };
 typedef struct {
   int32_t num_neg;            /* K in [1, 64]                                      */
   int32_t corruption;         /* MARS_CORRUPT_*                                    */
   float mask_rate;            /* MARS_CORRUPT_MASK: in [0, 1]                      */
   int32_t readout;            /* MARS_READOUT_*                                    */
   int32_t aggregator;         /* MARS_AGG_*                                        */
+  int32_t loss;               /* MARS_LOSS_*                                       */
 } mars_contrastive;
 /* Sets the variant for later steps / encodes (the workspace and captured steps
  * are rebuilt on the next call).  EINVAL on an out-of-range field; ESTATE on a

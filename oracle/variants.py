@@ -25,6 +25,9 @@ discriminator, Eq. 6 loss -- with the variant's choices.  Readings
        W2n | W3s | W3n | M | α], init U(-b, b) with b = f32(sqrt(6 / (2 C_in +
        H))) per layer (sqrt(6 / 2H) for M), tags 1..7 in layout order (c14's
        generator), α = 0.25.
+  c39  InfoNCE loss: per node i, softmax over its K + 1 logits (k = 0 the
+       positive, k = 1..K its corrupted counterparts, same node index);
+       L = (1/B) Σ_g (1/N_g) Σ_i [log Σ_k e^{l_ik} - l_i0].
 
 The corruption permutations are oracle.perm's (the C oracle, c12).  Parity
 pins: tests/test_oracle_variants.py (the default variant against the C
@@ -167,7 +170,7 @@ def corrupted(g, X, seed, step, pair, corruption, mask_rate):
 def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: int = 0,
                B: float | None = None, num_neg: int = 1, corruption: str = "permute",
                mask_rate: float = 0.0, readout: str = "sigmoid_mean", aggregator: str = "gcn",
-               pair_off=None, sparse: bool = False, encoder: str = "gcn"):
+               pair_off=None, sparse: bool = False, encoder: str = "gcn", loss: str = "bce"):
     """(loss, dL/dparams) of one step over a graph set (c34-c38).  B = number of
     graphs the loss is averaged over (default: len(graphs)); pair_off[g]
     defaults to g.  sparse: Â as a torch sparse matrix (larger graphs).
@@ -182,7 +185,7 @@ def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: 
     B = float(len(graphs) if B is None else B)
     K = int(num_neg)
     sp = torch.nn.functional.softplus
-    loss = torch.zeros((), dtype=torch.float64)
+    total = torch.zeros((), dtype=torch.float64)
     for gi, g in enumerate(graphs):
         An_np = neighbour_mean(g) if encoder == "sage" else normalise(adjacency(g), aggregator)
         An = torch.from_numpy(An_np)
@@ -196,15 +199,25 @@ def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: 
         if readout not in ("sigmoid_mean", "mean"):
             raise ValueError(readout)
         v = M @ s                                        # Eq. 5: l_i = h_iᵀ M s
+        po = gi if pair_off is None else int(pair_off[gi])
+        if loss == "infonce":                            # c39
+            logits = [Hp @ v]
+            for k in range(K):
+                Xt = corrupted(g, X, seed, step, pair_base + po * K + k, corruption, mask_rate)
+                logits.append(enc(An, Xt) @ v)
+            Lg = torch.stack(logits)                     # [K + 1, N]
+            total = total + (torch.logsumexp(Lg, 0) - Lg[0]).sum() / N / B
+            continue
+        if loss != "bce":
+            raise ValueError(loss)
         pos = sp(-(Hp @ v)).sum()
         neg = torch.zeros((), dtype=torch.float64)
-        po = gi if pair_off is None else int(pair_off[gi])
         for k in range(K):
             Xt = corrupted(g, X, seed, step, pair_base + po * K + k, corruption, mask_rate)
             neg = neg + sp(enc(An, Xt) @ v).sum()
-        loss = loss + (pos + neg / K) / (2.0 * N) / B    # Eq. 6 with c34
-    loss.backward()
-    return float(loss.detach()), p.grad.numpy().copy()
+        total = total + (pos + neg / K) / (2.0 * N) / B  # Eq. 6 with c34
+    total.backward()
+    return float(total.detach()), p.grad.numpy().copy()
 
 
 def encode(graphs, params, F: int, H: int, aggregator: str = "gcn", encoder_: str = "gcn"):

@@ -341,6 +341,153 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
   }
 }
 
+// ---- InfoNCE (c39): per node i, one positive logit l_i0 (block 0) against
+// its K corrupted counterparts l_ik (blocks 1..K, same node index):
+//   L = (1/B) Σ_g (1/N_g) Σ_i [log Σ_k e^{l_ik} - l_i0]
+//   dl_i0 = (p_i0 - 1)/(N_g B), dl_ik = p_ik/(N_g B), p = softmax over k.
+// Three passes replace k_score: logits of every real row, the per-node
+// softmax (dl, loss partials), and the dv partials Σ dl h.
+template <int NC, typename T>
+__global__ void __launch_bounds__(kWarps * 32, 3)
+k_logits(const T* __restrict__ Z3, const float* __restrict__ alpha,
+         const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
+         const float* __restrict__ vf, int32_t Nt, float* __restrict__ lg) {
+  using RT = RowTile<NC, T>;
+  constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER, RU = RT::RU;
+  const int ch = blockIdx.x, w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool act = lane < LPR;
+  const int g = chunk_graph[ch];
+  const float a = alpha[2];
+  const int64_t base = (int64_t)blockIdx.y * Nt;
+  const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
+  float v[PER][V];
+#pragma unroll
+  for (int q = 0; q < PER; ++q)
+#pragma unroll
+    for (int e = 0; e < V; ++e) v[q][e] = act ? vf[(int64_t)g * H + (lane + q * LPR) * V + e] : 0.f;
+  for (int32_t r = r0 + w * RU; r < r1; r += kWarps * RU) {
+    typename Vec<T>::Raw zr[RU][PER];
+#pragma unroll
+    for (int u = 0; u < RU; ++u)
+#pragma unroll
+      for (int q = 0; q < PER; ++q)
+        zr[u][q] = (act && r + u < r1) ? Vec<T>::ld(Z3 + (base + r + u) * H + (lane + q * LPR) * V)
+                                       : typename Vec<T>::Raw{};
+#pragma unroll
+    for (int u = 0; u < RU; ++u) {
+      float t = 0.f;
+#pragma unroll
+      for (int q = 0; q < PER; ++q) {
+        float x[V];
+        Vec<T>::cvt(zr[u][q], x);
+#pragma unroll
+        for (int e = 0; e < V; ++e) t = fmaf(prelu(x[e], a), v[q][e], t);
+      }
+      t = warp_sum(t);
+      if (lane == 0 && r + u < r1) lg[base + r + u] = t;
+    }
+  }
+}
+
+// One block per chunk, one thread per node: softmax over the node's K + 1
+// logits (fp64), dl in place of the logits (0 on padding blocks), and the
+// chunk's loss partial at loss_part[ch * (K + 1)] (the other K slots 0, so the
+// dv reduction's rep = K + 1 sums it once).
+__global__ void __launch_bounds__(256)
+k_nce(const int32_t* __restrict__ chunk_row, const int32_t* __restrict__ chunk_graph,
+      const int32_t* __restrict__ gsize, const StepParams* __restrict__ sp, int32_t Nt, int32_t K,
+      int32_t nb, float* __restrict__ dl, double* __restrict__ loss_part) {
+  __shared__ double sh[256];
+  const int ch = blockIdx.x;
+  const int32_t r = chunk_row[ch] + threadIdx.x, r1 = chunk_row[ch + 1];
+  const double coef = (double)sp->inv_batch / (double)gsize[chunk_graph[ch]];
+  double loss = 0.0;
+  if (r < r1) {
+    double m = -INFINITY;
+    for (int k = 0; k <= K; ++k) m = fmax(m, (double)dl[(int64_t)k * Nt + r]);
+    double se = 0.0;
+    for (int k = 0; k <= K; ++k) se += exp((double)dl[(int64_t)k * Nt + r] - m);
+    const double lse = m + log(se);
+    const double l0 = (double)dl[r];
+    loss = lse - l0;
+    for (int k = 0; k <= K; ++k) {
+      const int64_t o = (int64_t)k * Nt + r;
+      const double p = exp((double)dl[o] - lse);
+      dl[o] = (float)(coef * (k == 0 ? p - 1.0 : p));
+    }
+    for (int k = K + 1; k < nb; ++k) dl[(int64_t)k * Nt + r] = 0.f;
+  }
+  sh[threadIdx.x] = loss;
+  __syncthreads();
+  for (int o = 128; o > 0; o >>= 1) {
+    if (threadIdx.x < o) sh[threadIdx.x] += sh[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x <= K) loss_part[(int64_t)ch * (K + 1) + threadIdx.x] = threadIdx.x ? 0.0 : sh[0] * coef;
+}
+
+// dv partials Σ_rows dl_i H3_i per (chunk, block b in 0..K) -> part[(ch (K+1) + b) H]
+template <int NC, typename T>
+__global__ void __launch_bounds__(kWarps * 32, 3)
+k_dvp(const T* __restrict__ Z3, const float* __restrict__ alpha,
+      const int32_t* __restrict__ chunk_row, const float* __restrict__ dl, int32_t Nt,
+      double* __restrict__ part) {
+  using RT = RowTile<NC, T>;
+  constexpr int H = RT::H, V = RT::V, LPR = RT::LPR, PER = RT::PER, RU = RT::RU;
+  __shared__ double sh[kWarps][H];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int ch = blockIdx.x;
+  const float a = alpha[2];
+  const int64_t base = (int64_t)blockIdx.y * Nt;
+  const int32_t r0 = chunk_row[ch], r1 = chunk_row[ch + 1];
+  const bool act = lane < LPR;
+  double d[PER][V];
+#pragma unroll
+  for (int q = 0; q < PER; ++q)
+#pragma unroll
+    for (int e = 0; e < V; ++e) d[q][e] = 0.0;
+  for (int32_t r = r0 + w * RU; r < r1; r += kWarps * RU) {
+    typename Vec<T>::Raw xr[RU][PER];
+    float c[RU];
+#pragma unroll
+    for (int u = 0; u < RU; ++u) {
+      c[u] = r + u < r1 ? dl[base + r + u] : 0.f;
+#pragma unroll
+      for (int q = 0; q < PER; ++q)
+        xr[u][q] = (act && r + u < r1) ? Vec<T>::ld(Z3 + (base + r + u) * H + (lane + q * LPR) * V)
+                                       : typename Vec<T>::Raw{};
+    }
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      float f[V];
+#pragma unroll
+      for (int e = 0; e < V; ++e) f[e] = 0.f;
+#pragma unroll
+      for (int u = 0; u < RU; ++u) {
+        float x[V];
+        Vec<T>::cvt(xr[u][q], x);
+#pragma unroll
+        for (int e = 0; e < V; ++e) f[e] = fmaf(c[u], prelu(x[e], a), f[e]);
+      }
+#pragma unroll
+      for (int e = 0; e < V; ++e) d[q][e] += (double)f[e];
+    }
+  }
+  if (act) {
+#pragma unroll
+    for (int q = 0; q < PER; ++q)
+#pragma unroll
+      for (int e = 0; e < V; ++e) sh[w][(lane + q * LPR) * V + e] = d[q][e];
+  }
+  __syncthreads();
+  for (int cc = threadIdx.x; cc < H; cc += kWarps * 32) {
+    double t = 0.0;
+#pragma unroll
+    for (int k = 0; k < kWarps; ++k) t += sh[k][cc];
+    part[((int64_t)ch * gridDim.y + blockIdx.y) * H + cc] = t;
+  }
+}
+
 // dM[r][c] = Σ_g dv_g[r] s_g[c] (fixed order); block 0 also writes the loss.
 __global__ void k_dM(const double* __restrict__ dvd, const double* __restrict__ sd, int G, int H,
                      const double* __restrict__ loss_g, float* __restrict__ gM,
@@ -509,7 +656,7 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
   const dim3 gh(g.G, H / 32);
   cudaError_t e;
   const int nb = w.nb, nbp = nb / 2;
-  if (nb < 2 || (nb & 1) || w.K < 1 || w.K >= nb || (hs && (nb != 2 || w.readout)))
+  if (nb < 2 || (nb & 1) || w.K < 1 || w.K >= nb || (hs && (nb != 2 || w.readout || w.loss)))
     return cudaErrorInvalidValue;
   k_colsum<NC, T><<<g.nchunks, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, w.colsum_part);
   if (!hs) {
@@ -524,13 +671,25 @@ cudaError_t head_nc(const GraphDev& g, const T* Z3, const float* M, const float*
       return e;
   }
   k_Mv<<<gh, 256, 0, s>>>(M, w.sd, H, w.v);
-  k_score<NC, T><<<dim3(g.nchunks, nbp), kWarps * 32, 0, s>>>(
-      Z3, alpha, g.chunk_row, g.chunk_graph, g.gsize, w.v, sp, g.Nt, w.K, w.dl, w.dv_part,
-      w.loss_part);
-  if (!hs) {
+  if (w.loss) {                   // InfoNCE (c39)
+    const dim3 gk(g.nchunks, w.K + 1);
+    k_logits<NC, T><<<gk, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, g.chunk_graph, w.v, g.Nt,
+                                                w.dl);
+    k_nce<<<g.nchunks, 256, 0, s>>>(g.chunk_row, g.chunk_graph, g.gsize, sp, g.Nt, w.K, nb, w.dl,
+                                    w.loss_part);
+    k_dvp<NC, T><<<gk, kWarps * 32, 0, s>>>(Z3, alpha, g.chunk_row, w.dl, g.Nt, w.dv_part);
+    k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, w.K + 1, 0, w.dvd,
+                                   w.dv, w.loss_part, w.loss_g);
+  } else if (!hs) {
+    k_score<NC, T><<<dim3(g.nchunks, nbp), kWarps * 32, 0, s>>>(
+        Z3, alpha, g.chunk_row, g.chunk_graph, g.gsize, w.v, sp, g.Nt, w.K, w.dl, w.dv_part,
+        w.loss_part);
     k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, nbp, 0, w.dvd, w.dv,
                                    w.loss_part, w.loss_g);
   } else {
+    k_score<NC, T><<<dim3(g.nchunks, nbp), kWarps * 32, 0, s>>>(
+        Z3, alpha, g.chunk_row, g.chunk_graph, g.gsize, w.v, sp, g.Nt, w.K, w.dl, w.dv_part,
+        w.loss_part);
     k_chunk_sum<<<gh, 256, 0, s>>>(w.dv_part, g.graph_chunk, g.gsize, H, 1, 1, 0, hs->x_own[1],
                                    nullptr, w.loss_part, hs->x_own[1] + H);
     if ((e = launch_shard_barrier(*hs->sync, s, nullptr)) != cudaSuccess) return e;
@@ -573,7 +732,7 @@ cudaError_t launch_head(const GraphDev& g, int H, const void* Z3, int bf16_, con
                         const float* alpha_dev, const StepParams* sp, const HeadWork& w, void* dZ,
                         float* grad_M, float* loss_out, int* nslots, cudaStream_t s,
                         int* launches, const HeadShard* hs) {
-  count_launch(launches, hs ? 12 : 8);
+  count_launch(launches, hs ? 12 : w.loss ? 10 : 8);
   if (bf16_)
     return head_t<bf16>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s, hs);
   return head_t<float>(g, H, Z3, params_M, alpha_dev, sp, w, dZ, grad_M, loss_out, nslots, s, hs);

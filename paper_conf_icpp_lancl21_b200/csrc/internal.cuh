@@ -235,8 +235,8 @@ cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, in
 // ---------------------------------------------------------------- head.cu
 struct HeadWork {
   double* colsum_part;  // [nchunks*H]
-  double* dv_part;      // [nchunks*nb/2*H]
-  double* loss_part;    // [nchunks*nb/2]
+  double* dv_part;      // [nchunks*nb*H]
+  double* loss_part;    // [nchunks*nb]
   float* s;             // [G*H]
   float* v;             // [G*H]
   float* dm;            // [G*H] (already divided by N_g)
@@ -247,10 +247,11 @@ struct HeadWork {
   double* loss_g;       // [G] per-graph loss (already / (2 N_g B))
   double* slots;        // [nslots] dalpha3 partials
   float* rs_dz3;        // [nb*Nt] power-of-two row scales of dZ3 (fp32 storage) or null
-  // NEXT-4 (c34-c36): nb stacked blocks of Nt rows (even; block 0 positive,
-  // 1..K corrupted, > K padding), K corruption samples, readout 0 = sig(mean),
-  // 1 = mean.  The default DGI step: nb = 2, K = 1, readout 0.
-  int32_t nb, K, readout;
+  // NEXT-4 (c34-c36, c39): nb stacked blocks of Nt rows (even; block 0
+  // positive, 1..K corrupted, > K padding), K corruption samples, readout
+  // 0 = sig(mean), 1 = mean; loss 0 = BCE (Eq. 6), 1 = InfoNCE.  The default
+  // DGI step: nb = 2, K = 1, readout 0, loss 0.
+  int32_t nb, K, readout, loss;
 };
 // Forward head + head backward: writes grads of M (dM) and the loss slot,
 // dZ3 into dZ, dalpha3 partials into w.slots.

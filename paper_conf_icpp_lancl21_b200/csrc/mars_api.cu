@@ -399,7 +399,8 @@ struct mars_dgi {
   int sp_ring = 32, sp_next = 0;
   Workspace ws;
   const mars_graph* ws_graph = nullptr;
-  mars_contrastive ct{1, MARS_CORRUPT_PERMUTE, 0.f, MARS_READOUT_SIGMOID_MEAN, MARS_AGG_GCN};
+  mars_contrastive ct{1, MARS_CORRUPT_PERMUTE, 0.f, MARS_READOUT_SIGMOID_MEAN, MARS_AGG_GCN,
+                      MARS_LOSS_BCE};
   bool sage = false;                // MARS_ENCODER_SAGE (c38)
   int ct_nb() const { return (ct.num_neg + 2) & ~1; }     // K + 1 blocks, rounded up to even
   bool ct_materialise() const {
@@ -1155,8 +1156,10 @@ extern "C" mars_status mars_dgi_set_contrastive(mars_dgi* m, const mars_contrast
     return fail(MARS_EINVAL, "unknown readout");
   if (c->aggregator != MARS_AGG_GCN && c->aggregator != MARS_AGG_SAGE_GCN)
     return fail(MARS_EINVAL, "unknown aggregator");
+  if (c->loss != MARS_LOSS_BCE && c->loss != MARS_LOSS_INFONCE) return fail(MARS_EINVAL, "unknown loss");
   const bool dflt = c->num_neg == 1 && c->corruption == MARS_CORRUPT_PERMUTE &&
-                    c->readout == MARS_READOUT_SIGMOID_MEAN && c->aggregator == MARS_AGG_GCN;
+                    c->readout == MARS_READOUT_SIGMOID_MEAN && c->aggregator == MARS_AGG_GCN &&
+                    c->loss == MARS_LOSS_BCE;
   if (m->sh.g && !dflt) return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
   if (m->sage && c->aggregator != MARS_AGG_GCN)
     return fail(MARS_EINVAL, "the SAGE encoder has its own aggregation (aggregator must be GCN)");
@@ -1269,8 +1272,8 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   CK(al(&w.pw.scan_tmp, scan_tmp_bytes(nb + 1)));
   HeadWork& h = w.hw;
   CK(al((void**)&h.colsum_part, sizeof(double) * nch * H));
-  CK(al((void**)&h.dv_part, sizeof(double) * nch * (nbk / 2) * H));
-  CK(al((void**)&h.loss_part, sizeof(double) * nch * (nbk / 2)));
+  CK(al((void**)&h.dv_part, sizeof(double) * nch * nbk * H));
+  CK(al((void**)&h.loss_part, sizeof(double) * nch * nbk));
   CK(al((void**)&h.s, sizeof(float) * G * H));
   CK(al((void**)&h.v, sizeof(float) * G * H));
   CK(al((void**)&h.dm, sizeof(float) * G * H));
@@ -1323,6 +1326,7 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   h.nb = nbk;
   h.K = K;
   h.readout = m->ct.readout;
+  h.loss = m->ct.loss;
   return MARS_OK;
 }
 
@@ -1388,6 +1392,7 @@ static cudaError_t enqueue_step_sage(mars_dgi* m, const mars_graph* gr, cudaStre
   w.hw.nb = nb;
   w.hw.K = K;
   w.hw.readout = m->ct.readout;
+  w.hw.loss = m->ct.loss;
   // corrupted inputs + the redirected CSR (self entry -> row Rb + i)
   RET(launch_pair_off_k(g.pair_off, g.G, K, w.pair_off_k, s, nl));
   if (m->ct.corruption == MARS_CORRUPT_PERMUTE)
@@ -1528,6 +1533,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   w.hw.nb = nb;
   w.hw.K = K;
   w.hw.readout = m->ct.readout;
+  w.hw.loss = m->ct.loss;
   float* W[3] = {m->params, m->params + (int64_t)F * H, m->params + (int64_t)F * H + (int64_t)H * H};
   float* Mp = m->params + (int64_t)F * H + 2LL * H * H;
   float* alpha = m->params + (int64_t)F * H + 3LL * H * H;
@@ -2524,7 +2530,8 @@ extern "C" mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g) {
   if (m->sh.g) return fail(MARS_ESTATE, "model already attached to a shard");
   if (m->sage) return fail(MARS_EINVAL, "row sharding runs the GCN encoder only");
   if (m->ct.num_neg != 1 || m->ct.corruption != MARS_CORRUPT_PERMUTE ||
-      m->ct.readout != MARS_READOUT_SIGMOID_MEAN || m->ct.aggregator != MARS_AGG_GCN)
+      m->ct.readout != MARS_READOUT_SIGMOID_MEAN || m->ct.aggregator != MARS_AGG_GCN ||
+      m->ct.loss != MARS_LOSS_BCE)
     return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
   if (m->comm) return fail(MARS_EINVAL, "a shard-attached model cannot also be data-parallel");
   if (g->F != m->F || g->device != m->cfg.device) return fail(MARS_EINVAL, "F / device mismatch");

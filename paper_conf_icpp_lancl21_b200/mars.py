@@ -71,12 +71,13 @@ class Contrastive(ctypes.Structure):
     """mars_contrastive (NEXT-4, readings c34-c37)."""
     _fields_ = [("num_neg", ctypes.c_int32), ("corruption", ctypes.c_int32),
                 ("mask_rate", ctypes.c_float), ("readout", ctypes.c_int32),
-                ("aggregator", ctypes.c_int32)]
+                ("aggregator", ctypes.c_int32), ("loss", ctypes.c_int32)]
 
 
 CORRUPTIONS = {"permute": 0, "mask": 1}
 READOUTS = {"sigmoid_mean": 0, "mean": 1}
 AGGREGATORS = {"gcn": 0, "sage_gcn": 1}
+LOSSES = {"bce": 0, "infonce": 1}
 ENCODERS = {"gcn": 0, "sage": 1}
 
 
@@ -429,13 +430,13 @@ class DGI:
 
     def set_contrastive(self, num_neg: int = 1, corruption: str = "permute",
                         mask_rate: float = 0.0, readout: str = "sigmoid_mean",
-                        aggregator: str = "gcn"):
+                        aggregator: str = "gcn", loss: str = "bce"):
         """mars_dgi_set_contrastive (NEXT-4): K corruption samples sharing one
         positive branch, permutation or feature-mask corruption, sig(mean) or
         mean readout, GCN or SAGE-GCN aggregation.  The defaults are the paper's
         DGI step."""
         c = Contrastive(int(num_neg), CORRUPTIONS[corruption], float(mask_rate),
-                        READOUTS[readout], AGGREGATORS[aggregator])
+                        READOUTS[readout], AGGREGATORS[aggregator], LOSSES[loss])
         _check(lib().mars_dgi_set_contrastive(self.handle, ctypes.byref(c)))
         self.num_neg, self.corruption = int(num_neg), corruption
 
@@ -445,7 +446,7 @@ class DGI:
         inv = lambda d, v: next(k for k, x in d.items() if x == v)
         return dict(num_neg=c.num_neg, corruption=inv(CORRUPTIONS, c.corruption),
                     mask_rate=c.mask_rate, readout=inv(READOUTS, c.readout),
-                    aggregator=inv(AGGREGATORS, c.aggregator))
+                    aggregator=inv(AGGREGATORS, c.aggregator), loss=inv(LOSSES, c.loss))
 
     def step(self, g: Graph, step_index: int, pair_base: int = 0, global_batch: int | None = None,
              want_loss=False, want_grads=False, want_perms=False):

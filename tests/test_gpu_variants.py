@@ -1,8 +1,8 @@
 """GPU parity of the NEXT-4 contrastive variants (mars_dgi_set_contrastive;
-readings c34-c37) against the variant oracle (oracle/variants.py, float64
+readings c34-c39) against the variant oracle (oracle/variants.py, float64
 autograd), through the C ABI: K corruption samples sharing one positive
-branch, feature-masking corruption, the mean readout and the SAGE-GCN
-aggregator, alone and combined, fp32 (<= 1e-5 scaled) and bf16
+branch, feature-masking corruption, the mean readout, the SAGE-GCN
+aggregator and the InfoNCE loss, alone and combined, and the SAGE-mean encoder, fp32 (<= 1e-5 scaled) and bf16
 (2e-2).  At the GNMT bench size, where the fp64 oracle is too slow end to end,
 the shared-positive step is checked against the same K samples run as K
 copies of the graph (c20) -- a property that holds at any size."""
@@ -46,6 +46,9 @@ VARIANTS = [
     dict(readout="mean"),
     dict(aggregator="sage_gcn"),
     dict(num_neg=2, readout="mean", aggregator="sage_gcn"),
+    dict(loss="infonce"),
+    dict(num_neg=3, loss="infonce"),
+    dict(num_neg=2, corruption="mask", mask_rate=0.2, readout="mean", loss="infonce"),
 ]
 
 
@@ -237,7 +240,7 @@ def test_sage_init_bit_exact():
 @pytest.mark.parametrize("F,H,impl", SIZES)
 @pytest.mark.parametrize("variant", [dict(), dict(num_neg=3), dict(num_neg=2, corruption="mask",
                                                                    mask_rate=0.3),
-                                     dict(readout="mean")],
+                                     dict(readout="mean"), dict(num_neg=2, loss="infonce")],
                          ids=lambda v: "-".join(f"{k}={x}" for k, x in v.items()) or "default")
 def test_sage_step_vs_oracle(variant, F, H, impl):
     gs = _graphs(F)

@@ -1,4 +1,4 @@
-"""Pins for the NEXT-4 variant oracle (oracle/variants.py; readings c34-c38):
+"""Pins for the NEXT-4 variant oracle (oracle/variants.py; readings c34-c39):
 the default variant against the C oracle's step, K shared-positive samples
 against the C oracle on K copies of each graph (c20), feature masking at rates
 0 and 1 in closed form, the readouts against the C oracle's encoder plus a
@@ -300,4 +300,47 @@ def test_sage_gradients_finite_differences(kw):
         pm[i] -= h
         fd = (V.step_grads(gs, pp, F, H, SEED, STEP, encoder="sage", **kw)[0]
               - V.step_grads(gs, pm, F, H, SEED, STEP, encoder="sage", **kw)[0]) / (2 * h)
+        assert abs(fd - grads[i]) <= 1e-7 + 1e-5 * abs(grads[i]), (i, fd, grads[i])
+
+
+# ----------------------------------------------------------------- InfoNCE (c39)
+@pytest.mark.parametrize("K", [1, 3])
+def test_infonce_against_c_encoder_and_numpy(K):
+    """Forward loss from the C oracle's embeddings with the softmax written out
+    in numpy; K = 1 is also checked against its closed form softplus(l~ - l)."""
+    gs, p = _graphs(), _params()
+    M = p[F * H + 2 * H * H:F * H + 3 * H * H].reshape(H, H)
+    want = 0.0
+    for gi, g in enumerate(gs):
+        Hp = _c_encode(g, p)
+        v = M @ (1 / (1 + np.exp(-Hp.mean(0))))
+        L = [Hp @ v]
+        for k in range(K):
+            pi = oracle.perm(SEED, STEP, gi * K + k, g.num_nodes)
+            L.append(_c_encode(_with_features(g, np.asarray(g.features)[pi]), p) @ v)
+        L = np.array(L)
+        m = L.max(0)
+        lse = m + np.log(np.exp(L - m).sum(0))
+        per = lse - L[0]
+        if K == 1:
+            assert np.max(np.abs(per - _softplus(L[1] - L[0]))) < 1e-13
+        want += per.mean() / len(gs)
+    vl, _ = V.step_grads(gs, p, F, H, SEED, STEP, num_neg=K, loss="infonce")
+    assert abs(vl - want) < 1e-12
+
+
+@pytest.mark.parametrize("kw", [dict(num_neg=1), dict(num_neg=3, readout="mean"),
+                                dict(num_neg=2, encoder="sage")])
+def test_infonce_gradients_finite_differences(kw):
+    gs = [SG.tiny(8, N=19)]
+    p = _sage_params(5) if kw.get("encoder") == "sage" else _params(6)
+    _, grads = V.step_grads(gs, p, F, H, SEED, STEP, loss="infonce", **kw)
+    rng = np.random.default_rng(4)
+    for i in list(rng.choice(p.size - 3, 6, replace=False)) + [p.size - 1]:
+        h = 1e-5
+        pp, pm = p.copy(), p.copy()
+        pp[i] += h
+        pm[i] -= h
+        fd = (V.step_grads(gs, pp, F, H, SEED, STEP, loss="infonce", **kw)[0]
+              - V.step_grads(gs, pm, F, H, SEED, STEP, loss="infonce", **kw)[0]) / (2 * h)
         assert abs(fd - grads[i]) <= 1e-7 + 1e-5 * abs(grads[i]), (i, fd, grads[i])
