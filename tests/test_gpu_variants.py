@@ -290,3 +290,48 @@ def test_sage_captured_replay_matches_eager():
 def test_sage_config_errors():
     with pytest.raises(mars.MarsError):
         mars.dgi_create(in_dim=64, hidden_dim=128, encoder="sage", precision=mars.MARS_BF16)
+
+
+def _edge_graphs(F):
+    """A one-node graph, a graph with isolated nodes (no edges at all for some
+    ops) and a small DAG -- degenerate neighbourhoods for every aggregator."""
+    rng = np.random.default_rng(7)
+
+    class G:
+        pass
+    one = G()
+    one.num_nodes, one.indptr, one.indices = 1, np.zeros(2, np.int64), np.zeros(0, np.int32)
+    one.features = rng.random((1, F), dtype=np.float32)
+    iso = G()
+    N = 40
+    src = np.array([3, 3, 7, 10, 10, 11, 20], np.int64)
+    dst = np.array([4, 5, 8, 11, 12, 12, 21], np.int32)
+    indptr = np.zeros(N + 1, np.int64)
+    np.add.at(indptr, src + 1, 1)
+    iso.num_nodes, iso.indptr, iso.indices = N, np.cumsum(indptr), dst
+    iso.features = rng.random((N, F), dtype=np.float32)
+    return [one, iso, SG.tiny(3, N=61, F=F)]
+
+
+@pytest.mark.parametrize("encoder,variant", [("gcn", dict(num_neg=2, loss="infonce")),
+                                             ("gcn", dict(num_neg=3, aggregator="sage_gcn",
+                                                          readout="mean")),
+                                             ("sage", dict(num_neg=2, corruption="mask",
+                                                           mask_rate=0.4)),
+                                             ("sage", dict(loss="infonce"))])
+def test_variants_degenerate_graphs(encoder, variant):
+    gs = _edge_graphs(16)
+    g = mars.graph_load(gs)
+    m = mars.dgi_create(in_dim=16, hidden_dim=32, seed=9, encoder=encoder)
+    m.set_contrastive(**variant)
+    p0 = m.get_state()[0].astype(np.float64)
+    out = m.step(g, 1, 2, want_loss=True, want_grads=True)
+    emb = m.encode(g)
+    p1 = m.get_state()[0].astype(np.float64)          # after the step's Adam update
+    m.free(); g.free()
+    loss, grads = V.step_grads(gs, p0, 16, 32, 9, 1, pair_base=2, encoder=encoder, **variant)
+    assert np.isfinite(out["loss"]) and np.all(np.isfinite(out["grads"]))
+    assert abs(out["loss"] - loss) / abs(loss) <= TOL
+    assert scaled_err(out["grads"], grads) <= TOL
+    assert scaled_err(emb, V.encode(gs, p1, 16, 32, aggregator=variant.get("aggregator", "gcn"),
+                                    encoder_=encoder)) <= TOL
