@@ -28,9 +28,6 @@
 namespace mars {
 namespace {
 
-#ifndef MARS_SPMM_G4
-#define MARS_SPMM_G4 0             // A/B: TMA gather4-staged forward (C = 256, fp32)
-#endif
 constexpr int kSpmmThreads = 32;   // one warp per block: a slow (hub) row holds no other warps
 #ifndef MARS_SPMM_MINB             // resident blocks per SM: caps registers at 64
 #define MARS_SPMM_MINB 32
@@ -648,194 +645,6 @@ cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, con
   return long_fwd<C, MODE, BOTH, SH, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, pr);
 }
 
-#if MARS_SPMM_G4
-// ---------------------------------------------------------------- TMA gather4 staging (A/B)
-// Experimental forward aggregation for C = 256 fp32, layers 2-3: every warp
-// stages its own neighbour rows with `cp.async.bulk.tensor.2d ... tile::gather4`
-// (4 rows of the positive and 4 of the corrupted branch per group) into a
-// private shared-memory ring and FMAs from shared memory.  Rows are strided
-// over the grid's warps; a row's entries form ceil(deg / 4) groups (the last
-// padded with weight-0 repeats of its first neighbour).  The issue cursor runs
-// up to the ring size ahead of the consume cursor.
-}  // namespace
-}  // namespace mars
-#include "tc_ptx.cuh"
-namespace mars {
-namespace {
-namespace g4 {
-constexpr int kWarps = 8;
-constexpr int C = 256;
-constexpr int ROWB = C * 4;
-constexpr int SLOT = 8 * ROWB;                                    // 8 KB
-constexpr int SPW = (225 * 1024) / (kWarps * (SLOT + 32));        // slots per warp
-constexpr int SMEM = kWarps * SPW * (SLOT + 32) + 1024;
-struct Meta {
-  float w[4];
-  int32_t row;     // output row, or -1 if not the row's last group
-  int32_t pad[3];
-};
-}  // namespace g4
-
-__device__ __forceinline__ void g4_load(uint32_t dst, const CUtensorMap* tm, int32_t r0, int32_t r1,
-                                        int32_t r2, int32_t r3, uint32_t bar) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(dst),
-      "l"(reinterpret_cast<uint64_t>(tm)), "r"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3), "r"(bar)
-      : "memory");
-}
-
-__global__ void __launch_bounds__(32 * g4::kWarps, 1)
-k_spmm_fwd_g4(const __grid_constant__ CUtensorMap tm, const int32_t* __restrict__ rowptr,
-              const int32_t* __restrict__ colind, const float* __restrict__ vals,
-              const float* __restrict__ alpha, int act_layer, int32_t Nt, float* __restrict__ Y,
-              float* __restrict__ rs) {
-  using namespace tc;
-  constexpr int S = g4::SPW;
-  extern __shared__ uint8_t smem_raw[];
-  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint8_t* ring = smem + warp * S * g4::SLOT;
-  g4::Meta* meta = reinterpret_cast<g4::Meta*>(smem + g4::kWarps * S * g4::SLOT) + warp * S;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + g4::kWarps * S * (g4::SLOT + 32)) + warp * S;
-  if (lane == 0) {
-    for (int k = 0; k < S; ++k) mbar_init(&full[k], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncwarp();
-  const float a = alpha[act_layer];
-  const int32_t NW = gridDim.x * g4::kWarps;
-  // issue cursor: row ri, entry k (absolute), row end re; CSR chunk in lanes
-  int32_t ri = blockIdx.x * g4::kWarps + warp, k = 0, re = 0, cb = 0;
-  int32_t mycol = 0;
-  float myval = 0.f;
-  bool idone = ri >= Nt;
-  if (!idone) {
-    k = rowptr[ri];
-    re = rowptr[ri + 1];
-    cb = k;
-    mycol = k + lane < re ? colind[k + lane] : 0;
-    myval = k + lane < re ? vals[k + lane] : 0.f;
-  }
-  int64_t gi = 0, gc = 0;           // groups issued / consumed
-  float accp[8], accn[8];
-#pragma unroll
-  for (int e = 0; e < 8; ++e) accp[e] = accn[e] = 0.f;
-  for (;;) {
-    // issue while the ring has room
-    while (!idone && gi < gc + S) {
-      const int slot = (int)(gi % S);
-      const int off = k - cb;                        // chunk-relative first entry (< 32)
-      const int n = min(4, re - k);
-      int32_t j[4];
-      float w[4];
-#pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int src = off + (u < n ? u : 0);
-        j[u] = __shfl_sync(kFull, mycol, src);
-        w[u] = __shfl_sync(kFull, myval, src);
-        if (u >= n) w[u] = 0.f;
-      }
-      const bool last = k + n >= re;
-      if (lane == 0) {
-        g4::Meta& m = meta[slot];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) m.w[u] = w[u];
-        m.row = last ? ri : -1;
-        const uint32_t bar = smem_u32(&full[slot]);
-        const uint32_t dst = smem_u32(ring + slot * g4::SLOT);
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        mbar_expect_tx(&full[slot], g4::SLOT);
-        g4_load(dst, &tm, j[0], j[1], j[2], j[3], bar);
-        g4_load(dst + 4 * g4::ROWB, &tm, Nt + j[0], Nt + j[1], Nt + j[2], Nt + j[3], bar);
-      }
-      ++gi;
-      k += n;
-      if (k >= re) {                                 // next row of this warp
-        ri += NW;
-        if (ri >= Nt) {
-          idone = true;
-        } else {
-          k = rowptr[ri];
-          re = rowptr[ri + 1];
-          cb = k;
-          mycol = k + lane < re ? colind[k + lane] : 0;
-          myval = k + lane < re ? vals[k + lane] : 0.f;
-        }
-      } else if (k - cb + 4 > 32) {                  // refill the chunk window
-        cb = k;
-        mycol = k + lane < re ? colind[k + lane] : 0;
-        myval = k + lane < re ? vals[k + lane] : 0.f;
-      }
-    }
-    if (gc == gi) break;                             // everything consumed
-    // consume group gc
-    const int slot = (int)(gc % S);
-    mbar_wait(&full[slot], (uint32_t)((gc / S) & 1));
-    const g4::Meta m = meta[slot];
-    const uint8_t* base = ring + slot * g4::SLOT;
-#pragma unroll
-    for (int u = 0; u < 4; ++u) {
-      const float4* pp = reinterpret_cast<const float4*>(base + u * g4::ROWB);
-      const float4* pn = reinterpret_cast<const float4*>(base + (4 + u) * g4::ROWB);
-      const float4 p0 = pp[lane], p1 = pp[32 + lane], n0 = pn[lane], n1 = pn[32 + lane];
-      const float xp[8] = {p0.x, p0.y, p0.z, p0.w, p1.x, p1.y, p1.z, p1.w};
-      const float xn[8] = {n0.x, n0.y, n0.z, n0.w, n1.x, n1.y, n1.z, n1.w};
-#pragma unroll
-      for (int e = 0; e < 8; ++e) {
-        accp[e] = fmaf(m.w[u], prelu(xp[e], a), accp[e]);
-        accn[e] = fmaf(m.w[u], prelu(xn[e], a), accn[e]);
-      }
-    }
-    __syncwarp();
-    ++gc;
-    if (m.row >= 0) {                                // the row's last group: store
-      const int64_t rp = m.row, rn = (int64_t)Nt + m.row;
-      reinterpret_cast<float4*>(Y + rp * g4::C)[lane] = make_float4(accp[0], accp[1], accp[2], accp[3]);
-      reinterpret_cast<float4*>(Y + rp * g4::C)[32 + lane] = make_float4(accp[4], accp[5], accp[6], accp[7]);
-      reinterpret_cast<float4*>(Y + rn * g4::C)[lane] = make_float4(accn[0], accn[1], accn[2], accn[3]);
-      reinterpret_cast<float4*>(Y + rn * g4::C)[32 + lane] = make_float4(accn[4], accn[5], accn[6], accn[7]);
-      if (rs) {
-        float mp = 0.f, mn = 0.f;
-#pragma unroll
-        for (int e = 0; e < 8; ++e) {
-          mp = fmaxf(mp, fabsf(accp[e]));
-          mn = fmaxf(mn, fabsf(accn[e]));
-        }
-        for (int o = 16; o > 0; o >>= 1) {
-          mp = fmaxf(mp, __shfl_xor_sync(kFull, mp, o));
-          mn = fmaxf(mn, __shfl_xor_sync(kFull, mn, o));
-        }
-        if (lane == 0) {
-          rs[rp] = pow2_scale(mp);
-          rs[rn] = pow2_scale(mn);
-        }
-      }
-#pragma unroll
-      for (int e = 0; e < 8; ++e) accp[e] = accn[e] = 0.f;
-    }
-  }
-}
-
-cudaError_t fwd_g4(const GraphDev& g, const float* T, const float* alpha, int act_layer, float* Y,
-                   float* rs, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_spmm_fwd_g4, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         g4::SMEM);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
-  CUtensorMap tm;
-  if (!tc_tmap(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, T, 2LL * g.Nt, g4::C, g4::C, 1,
-               CU_TENSOR_MAP_SWIZZLE_NONE))
-    return cudaErrorInvalidValue;
-  k_spmm_fwd_g4<<<tc_num_sms(), 32 * g4::kWarps, g4::SMEM, s>>>(tm, g.rowptr, g.colind, g.vals,
-                                                                 alpha, act_layer, g.Nt, Y, rs);
-  return cudaGetLastError();
-}
-#endif
-
 template <int C, typename Tin, typename Tout>
 cudaError_t fwd_c(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
                   int act_layer, Tout* Y, float* rs, int both, cudaStream_t s,
@@ -853,10 +662,6 @@ cudaError_t fwd_c(const GraphDev& g, const Tin* T, const int32_t* perm, const fl
     }
   }
   if (peers) return cudaErrorInvalidValue;
-#if MARS_SPMM_G4
-  if constexpr (C == 256 && std::is_same<Tin, float>::value && std::is_same<Tout, float>::value)
-    if (both && g.nseg == 0) return fwd_g4(g, T, alpha, act_layer, Y, rs, s);
-#endif
   return both ? fwd_launch<C, 1, true, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, none)
               : fwd_launch<C, 1, false, false, Tin, Tout>(g, T, perm, alpha, act_layer, Y, rs, s, none);
 }
