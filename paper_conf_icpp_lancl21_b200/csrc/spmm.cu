@@ -547,17 +547,6 @@ cudaError_t long_bwd(const GraphDev& g, const T* dY, const T* Z, const float* al
 // walking rows i, i + NG, ..., and banded grids of one 1024-thread block per SM.
 static_assert(kSpmmThreads == 32, "long-row segments and the row map assume one-warp blocks");
 
-// Row groups per forward block for narrow rows (A/B knob; 1 = one group).
-#ifndef MARS_SPMM_ITERS
-#define MARS_SPMM_ITERS 1
-#endif
-#ifndef MARS_SPMM_ITER_CMAX
-#define MARS_SPMM_ITER_CMAX 64
-#endif
-template <int C>
-struct FwdIters {
-  static constexpr int N = C <= MARS_SPMM_ITER_CMAX ? MARS_SPMM_ITERS : 1;
-};
 
 template <int C, int MODE, bool BOTH, bool SH, bool LONG, typename Tin, typename Tout>
 __global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
@@ -578,22 +567,18 @@ k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colin
     return;
   }
   const int32_t bid = LONG ? (int32_t)blockIdx.x - nseg : (int32_t)blockIdx.x;
-  constexpr int IT = FwdIters<C>::N;
-#pragma unroll 1
-  for (int it = 0; it < IT; ++it) {
-    const int32_t i = (bid * IT + it) * S::RPB + w * S::RPW + sub;
-    if (i >= Nt) return;
-    // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
-    if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
-      if (a >= 0.f && a <= 1.f) {
-        fwd_row<C, MODE, BOTH, SH, 2, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y,
-                                            rs, pr, gmask, sl);
-        continue;
-      }
+  const int32_t i = bid * S::RPB + w * S::RPW + sub;
+  if (i >= Nt) return;
+  // bf16 storage: PReLU on packed pairs when 0 <= a <= 1 (uniform branch)
+  if constexpr (MODE == 1 && std::is_same<Tin, bf16>::value) {
+    if (a >= 0.f && a <= 1.f) {
+      fwd_row<C, MODE, BOTH, SH, 2, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs,
+                                          pr, gmask, sl);
+      return;
     }
-    fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs,
-                                        pr, gmask, sl);
   }
+  fwd_row<C, MODE, BOTH, SH, 1, LONG>(i, long_min, rowptr, colind, vals, T, perm, a, Nt, Y, rs, pr,
+                                      gmask, sl);
 }
 
 template <int C, bool SH, bool LONG, typename T>
@@ -633,7 +618,7 @@ template <int C, int MODE, bool BOTH, bool SH, typename Tin, typename Tout>
 cudaError_t fwd_launch(const GraphDev& g, const Tin* T, const int32_t* perm, const float* alpha,
                        int act_layer, Tout* Y, float* rs, cudaStream_t s, const PeerRows& pr) {
   const LongArgs la{g.long_rows, g.long_seg, g.seg_row, g.long_part};
-  const unsigned nb = cdiv(g.Nt, (int64_t)SpmmShape<C, Tin>::RPB * FwdIters<C>::N);
+  const unsigned nb = spmm_blocks<C, Tin>(g.Nt);
   const int al = act_layer < 0 ? 0 : act_layer;
   if (g.nseg > 0)   // long rows: their segments run as the grid's first blocks
     k_spmm_fwd<C, MODE, BOTH, SH, true, Tin, Tout><<<nb + g.nseg, kSpmmThreads, 0, s>>>(
