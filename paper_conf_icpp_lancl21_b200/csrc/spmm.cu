@@ -547,7 +547,6 @@ cudaError_t long_bwd(const GraphDev& g, const T* dY, const T* Z, const float* al
 // walking rows i, i + NG, ..., and banded grids of one 1024-thread block per SM.
 static_assert(kSpmmThreads == 32, "long-row segments and the row map assume one-warp blocks");
 
-
 template <int C, int MODE, bool BOTH, bool SH, bool LONG, typename Tin, typename Tout>
 __global__ void __launch_bounds__(kSpmmThreads, MARS_SPMM_MINB)
 k_spmm_fwd(const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
