@@ -534,7 +534,8 @@ def run_mine(args):
         # SURVEY §8(d)'s oracle table: seconds per step of one graph of each
         # config, OpenMP (all cores) and serial, beside the GPU's per-graph time
         table = {}
-        for name, Fc, Hc in (("tiny", 16, 32), ("inception", 64, 128), ("gnmt", 64, 256)):
+        for name, Fc, Hc in (("tiny", 16, 32), ("inception", 64, 128), ("gnmt", 64, 256),
+                             ("bert", 64, 256)):
             g1 = [SG.tiny(0)] if name == "tiny" else [SG.cached(name, 0)]
             row = {"N": g1[0].num_nodes, "F": Fc, "H": Hc,
                    "omp_s": oracle_step_seconds(oracle, g1, Hc)}
