@@ -1161,6 +1161,7 @@ extern "C" mars_status mars_dgi_set_contrastive(mars_dgi* m, const mars_contrast
                     c->readout == MARS_READOUT_SIGMOID_MEAN && c->aggregator == MARS_AGG_GCN &&
                     c->loss == MARS_LOSS_BCE;
   if (m->sh.g && !dflt) return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
+  if (memcmp(c, &m->ct, sizeof *c) == 0) return MARS_OK;     // unchanged: keep workspace and graphs
   if (m->sage && c->aggregator != MARS_AGG_GCN)
     return fail(MARS_EINVAL, "the SAGE encoder has its own aggregation (aggregator must be GCN)");
   CK(cudaSetDevice(m->cfg.device));

@@ -168,3 +168,25 @@ def test_shard_misuse_rejected():
     m2 = mars.dgi_create(in_dim=64, hidden_dim=128, seed=0)
     with pytest.raises(mars.MarsError):
         mars.shard_attach(m2, plain)                        # not a shard graph
+
+
+def test_shard_contrastive_variants_rejected():
+    """A row-sharded model runs the default DGI step only: re-setting the
+    default is a no-op (the attached workspace is kept and the step still
+    runs), any NEXT-4 variant or the SAGE encoder is refused."""
+    graph = SG.cached("inception", 0)
+    gs, ms = _sharded(graph, 2, 64, 128, 3)
+    ms[0].set_contrastive()
+    for bad in (dict(num_neg=2), dict(readout="mean"), dict(loss="infonce"),
+                dict(aggregator="sage_gcn")):
+        with pytest.raises(mars.MarsError):
+            ms[0].set_contrastive(**bad)
+    out = _step_all(gs, ms, 0)
+    assert all(np.isfinite(o[0]) for o in out)
+    ms_sage = mars.dgi_create(in_dim=64, hidden_dim=128, seed=3, encoder="sage")
+    with pytest.raises(mars.MarsError):
+        mars.shard_attach(ms_sage, mars.graph_load_shard(graph, 2, 0))
+    for m in ms + [ms_sage]:
+        m.free()
+    for g in gs:
+        g.free()
