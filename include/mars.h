@@ -128,7 +128,7 @@ typedef struct {
                                  allreduce (optional with world_size 1: a 1-rank
                                  communicator).  NULL with world_size > 1: peer-memory
                                  exchange (mars_dp_export / mars_dp_connect below). */
-  int32_t encoder;            /* MARS_ENCODER_GCN (Eq. 1, default) or MARS_ENCODER_SAGE */
+  int32_t encoder;            /* MARS_ENCODER_GCN (Eq. 1, default), _SAGE or _SAGE_POOL */
 } mars_dgi_config;
 
 /* The graph encoder (NEXT-4: "[33] uses GraphSAGE as the graph encoder",
@@ -143,7 +143,15 @@ typedef struct {
  * the contrastive variants apply except the SAGE-GCN aggregator; no
  * mars_dgi_encoder_vjp (so no joint PPO update).  The hooks export, per layer,
  * the GEMM input H_{l-1} (X~ stacked for layer 1) as "Y". */
-enum { MARS_ENCODER_GCN = 0, MARS_ENCODER_SAGE = 1 };
+/* MARS_ENCODER_SAGE_POOL: GraphSAGE with the pooling aggregator (the encoder
+ * of [33]; reading c40): per layer P = ReLU(h W_p + b_p), agg_i = element-wise
+ * max of P over the neighbours of i without i (0 for an isolated node),
+ * h' = PReLU(h W_s + agg W_n).  Parameters per layer [W_s C_in×H | W_n H×H |
+ * W_p C_in×H | b_p H], then [M H×H | α1 α2 α3]; default init U(-b, b) with
+ * b = sqrt(6 / (C_in + 2H)) for W_s and W_n, sqrt(6 / (C_in + H)) for W_p,
+ * b_p = 0, sqrt(6 / 2H) for M, tags 1..10 over the matrices in layout order,
+ * α = 0.25.  Same restrictions as MARS_ENCODER_SAGE. */
+enum { MARS_ENCODER_GCN = 0, MARS_ENCODER_SAGE = 1, MARS_ENCODER_SAGE_POOL = 2 };
 
 /* Fills cfg with the defaults above (F = 64, H = 256, L = 3, FP32, seed 0,
  * device 0, world 1). */

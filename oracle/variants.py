@@ -25,6 +25,14 @@ discriminator, Eq. 6 loss -- with the variant's choices.  Readings
        W2n | W3s | W3n | M | α], init U(-b, b) with b = f32(sqrt(6 / (2 C_in +
        H))) per layer (sqrt(6 / 2H) for M), tags 1..7 in layout order (c14's
        generator), α = 0.25.
+  c40  SAGE-pool encoder (GraphSAGE's pooling aggregator, the encoder of
+       [33]): P = ReLU(h W_p + b_p); agg_i = max_{j in N(i)} P_j element-wise
+       over the neighbours without the node (0 for an isolated node);
+       h' = PReLU(h W_s + agg W_n).  Parameters per layer [W_s C x H | W_n H x H
+       | W_p C x H | b_p H], then M and α; init U(-b, b) with b =
+       f32(sqrt(6 / (C + 2H))) for W_s and W_n, f32(sqrt(6 / (C + H))) for W_p,
+       b_p = 0, f32(sqrt(6 / 2H)) for M, tags 1..10 over the matrices in layout
+       order (c14's generator), α = 0.25.
   c39  InfoNCE loss: per node i, softmax over its K + 1 logits (k = 0 the
        positive, k = 1..K its corrupted counterparts, same node index);
        L = (1/B) Σ_g (1/N_g) Σ_i [log Σ_k e^{l_ik} - l_i0].
@@ -92,7 +100,65 @@ def normalise(A: np.ndarray, aggregator: str) -> np.ndarray:
 
 
 def num_params(F: int, H: int, encoder: str = "gcn") -> int:
+    if encoder == "sage_pool":
+        return 2 * F * H + 8 * H * H + 3 * H + 3
     return F * H + 3 * H * H + 3 + (F * H + 2 * H * H if encoder == "sage" else 0)
+
+
+def _xavier_block(seed: int, tag: int, n: int, fan: float):
+    b = float(np.float32(np.sqrt(6.0 / fan)))
+    base = np.uint64(_sm64((seed ^ tag) & M64))
+    z = _sm64_np(base ^ np.arange(n, dtype=np.uint64))
+    u = (z >> np.uint64(40)).astype(np.float64) * (1.0 / 16777216.0)
+    return ((2.0 * u - 1.0) * b).astype(np.float32)
+
+
+def sage_pool_init(seed: int, F: int, H: int) -> np.ndarray:
+    """c40: per layer W_s, W_n, W_p (tags 3l+1..3l+3), b_p = 0; M tag 10; α."""
+    out = []
+    for l in range(3):
+        C = F if l == 0 else H
+        out.append(_xavier_block(seed, 3 * l + 1, C * H, C + 2 * H))
+        out.append(_xavier_block(seed, 3 * l + 2, H * H, C + 2 * H))
+        out.append(_xavier_block(seed, 3 * l + 3, C * H, C + H))
+        out.append(np.zeros(H, np.float32))
+    out.append(_xavier_block(seed, 10, H * H, 2 * H))
+    out.append(np.full(3, 0.25, np.float32))
+    return np.concatenate(out)
+
+
+def unpack_sage_pool(p, F: int, H: int):
+    """[(W_s, W_n, W_p, b_p) per layer], M, alpha (c40 layout)."""
+    o, layers = 0, []
+    for l in range(3):
+        C = F if l == 0 else H
+        Ws = p[o:o + C * H].view(C, H); o += C * H
+        Wn = p[o:o + H * H].view(H, H); o += H * H
+        Wp = p[o:o + C * H].view(C, H); o += C * H
+        bp = p[o:o + H]; o += H
+        layers.append((Ws, Wn, Wp, bp))
+    M = p[o:o + H * H].view(H, H); o += H * H
+    return layers, M, p[o:o + 3]
+
+
+def neighbour_lists(g):
+    """N(i) of A v Aᵀ without self loops, ascending."""
+    A = adjacency(g)
+    np.fill_diagonal(A, 0.0)
+    return [np.nonzero(A[i])[0] for i in range(g.num_nodes)]
+
+
+def encoder_sage_pool(nbrs, X, layers, alpha):
+    """c40 x 3 (torch, autograd through the element-wise max)."""
+    h = X
+    for l in range(3):
+        Ws, Wn, Wp, bp = layers[l]
+        P = torch.relu(h @ Wp + bp)
+        zero = torch.zeros(P.shape[1], dtype=P.dtype)
+        agg = torch.stack([P[torch.from_numpy(nb)].max(0).values if len(nb) else zero
+                           for nb in nbrs])
+        h = torch.nn.functional.prelu(h @ Ws + agg @ Wn, alpha[l:l + 1])
+    return h
 
 
 def sage_init(seed: int, F: int, H: int) -> np.ndarray:
@@ -163,35 +229,45 @@ def corrupted(g, X, seed, step, pair, corruption, mask_rate):
         pi = _perm(seed, step, pair, N).astype(np.int64)
         return X[torch.from_numpy(pi)]
     if corruption == "mask":         # c35
-        return X * torch.from_numpy(mask_keep(seed, step, pair, N, F, mask_rate).astype(np.float64))
+        return X * torch.from_numpy(mask_keep(seed, step, pair, N, F, mask_rate)).to(X.dtype)
     raise ValueError(corruption)
 
 
 def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: int = 0,
                B: float | None = None, num_neg: int = 1, corruption: str = "permute",
                mask_rate: float = 0.0, readout: str = "sigmoid_mean", aggregator: str = "gcn",
-               pair_off=None, sparse: bool = False, encoder: str = "gcn", loss: str = "bce"):
+               pair_off=None, sparse: bool = False, encoder: str = "gcn", loss: str = "bce",
+               dtype=torch.float64):
     """(loss, dL/dparams) of one step over a graph set (c34-c38).  B = number of
     graphs the loss is averaged over (default: len(graphs)); pair_off[g]
     defaults to g.  sparse: Â as a torch sparse matrix (larger graphs).
-    encoder "sage": the c38 encoder (aggregator unused)."""
-    p = torch.tensor(np.asarray(params, np.float64), requires_grad=True)
+    encoder "sage": the c38 encoder (aggregator unused).  dtype float64 is the
+    oracle; float32 runs the same formulation in single precision -- a second
+    fp32 implementation that measures how much fp32 rounding alone moves the
+    result (the conditioning), as oracle/ppo.py does (reading c33)."""
+    p = torch.tensor(np.asarray(params, np.float64), dtype=dtype, requires_grad=True)
     if encoder == "sage":
         Wp, M, al = unpack_sage(p, F, H)
         enc = lambda A_, X_: encoder_sage(A_, X_, Wp, al)   # noqa: E731
+    elif encoder == "sage_pool":
+        layers, M, al = unpack_sage_pool(p, F, H)
+        enc = lambda A_, X_: encoder_sage_pool(A_, X_, layers, al)   # noqa: E731
     else:
         W1, W2, W3, M, al = unpack(p, F, H)
         enc = lambda A_, X_: _encoder_gcn(A_, X_, (W1, W2, W3), al)   # noqa: E731
     B = float(len(graphs) if B is None else B)
     K = int(num_neg)
     sp = torch.nn.functional.softplus
-    total = torch.zeros((), dtype=torch.float64)
+    total = torch.zeros((), dtype=dtype)
     for gi, g in enumerate(graphs):
-        An_np = neighbour_mean(g) if encoder == "sage" else normalise(adjacency(g), aggregator)
-        An = torch.from_numpy(An_np)
-        if sparse:
+        if encoder == "sage_pool":
+            An = neighbour_lists(g)                      # the encoder takes neighbour lists
+        else:
+            An_np = neighbour_mean(g) if encoder == "sage" else normalise(adjacency(g), aggregator)
+            An = torch.from_numpy(An_np).to(dtype)
+        if sparse and encoder != "sage_pool":
             An = An.to_sparse()
-        X = torch.tensor(np.asarray(g.features, np.float64))
+        X = torch.tensor(np.asarray(g.features, np.float64), dtype=dtype)
         N = g.num_nodes
         Hp = enc(An, X)
         m = Hp.mean(0)                                   # Eq. 4
@@ -217,7 +293,7 @@ def step_grads(graphs, params, F: int, H: int, seed: int, step: int, pair_base: 
             neg = neg + sp(enc(An, Xt) @ v).sum()
         total = total + (pos + neg / K) / (2.0 * N) / B  # Eq. 6 with c34
     total.backward()
-    return float(total.detach()), p.grad.numpy().copy()
+    return float(total.detach()), p.grad.double().numpy().copy()
 
 
 def encode(graphs, params, F: int, H: int, aggregator: str = "gcn", encoder_: str = "gcn"):
@@ -229,6 +305,9 @@ def encode(graphs, params, F: int, H: int, aggregator: str = "gcn", encoder_: st
         if encoder_ == "sage":
             Wp, _, al = unpack_sage(p, F, H)
             out.append(encoder_sage(torch.from_numpy(neighbour_mean(g)), X, Wp, al))
+        elif encoder_ == "sage_pool":
+            layers, _, al = unpack_sage_pool(p, F, H)
+            out.append(encoder_sage_pool(neighbour_lists(g), X, layers, al))
         else:
             W1, W2, W3, _, al = unpack(p, F, H)
             An = torch.from_numpy(normalise(adjacency(g), aggregator))

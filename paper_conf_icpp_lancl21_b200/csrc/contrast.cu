@@ -17,6 +17,9 @@
 //        (Â_N H) W_n, Â_N = D_N^-1 (A v Aᵀ) without self loops; computed
 //        GEMM-first as Z_i = U_s[i] + Σ_j Â_N[i][j] U_n[j] (U = H [W_s | W_n])
 //        by ONE aggregation whose self entry is redirected to the U_s rows.
+//   c40  SAGE-pool encoder: P = ReLU(h W_p + b_p), agg = element-wise max of
+//        P over the neighbours (argmax kept for the backward), h' = PReLU(h W_s
+//        + agg W_n).
 // The corrupted inputs are materialised (one pass over X per block) and layer
 // 1 aggregates the stacked blocks like layers 2-3 (PReLU slope 1 = identity).
 #include "common.cuh"
@@ -142,7 +145,161 @@ __global__ void k_rowprep(const float* __restrict__ in, int64_t rows, int C,
   if (rs && lane == 0) rs[r] = pow2_scale(m);
 }
 
+// ---- SAGE-pool encoder (c40).  One warp per row of the stacked activations
+// (row r = block b, node i = r - b Nt; neighbours in the same block); lanes
+// stride the H columns.
+// agg[r][c] = max_{j in N(i), j != i} ReLU(U[b Nt + j][c] + bp[c]) (0 without
+// neighbours), idx[r][c] = the first j (ascending) attaining it (-1 without).
+__global__ void k_maxagg(const float* __restrict__ U, const float* __restrict__ bp,
+                         const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
+                         int32_t Nt, int64_t R, int H, float* __restrict__ agg,
+                         int32_t* __restrict__ idx, float* __restrict__ rs) {
+  const int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (r >= R) return;
+  const int64_t base = r / Nt * Nt;
+  const int32_t i = (int32_t)(r - base);
+  const int32_t k0 = rowptr[i], k1 = rowptr[i + 1];
+  float amax = 0.f;
+  for (int c = lane; c < H; c += 32) {
+    const float b = bp[c];
+    float m = -1.f;
+    int32_t a = -1;
+    for (int32_t k = k0; k < k1; ++k) {
+      const int32_t j = colind[k];
+      if (j == i) continue;
+      const float v = fmaxf(U[(base + j) * H + c] + b, 0.f);
+      if (v > m) {
+        m = v;
+        a = j;
+      }
+    }
+    const float o = a < 0 ? 0.f : m;
+    agg[r * H + c] = o;
+    idx[r * H + c] = a;
+    amax = fmaxf(amax, o);
+  }
+  for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
+  if (rs && lane == 0) rs[r] = pow2_scale(amax);
+}
+
+// dU[r][c] = [U[r][c] + bp[c] > 0] Σ_{i in N(j), i != j, idx[b Nt + i][c] == j}
+// dagg[b Nt + i][c] (row r = b Nt + j; the pattern is symmetric, so the rows
+// whose max j won are among j's own neighbours; ascending i: deterministic).
+__global__ void k_maxagg_bwd(const float* __restrict__ dagg, const int32_t* __restrict__ idx,
+                             const float* __restrict__ U, const float* __restrict__ bp,
+                             const int32_t* __restrict__ rowptr,
+                             const int32_t* __restrict__ colind, int32_t Nt, int64_t R, int H,
+                             float* __restrict__ dU, float* __restrict__ rs) {
+  const int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (r >= R) return;
+  const int64_t base = r / Nt * Nt;
+  const int32_t j = (int32_t)(r - base);
+  const int32_t k0 = rowptr[j], k1 = rowptr[j + 1];
+  float amax = 0.f;
+  for (int c = lane; c < H; c += 32) {
+    float acc = 0.f;
+    for (int32_t k = k0; k < k1; ++k) {
+      const int32_t i = colind[k];
+      if (i == j) continue;
+      const int64_t e = (base + i) * H + c;
+      if (idx[e] == j) acc += dagg[e];
+    }
+    const float o = U[r * H + c] + bp[c] > 0.f ? acc : 0.f;
+    dU[r * H + c] = o;
+    amax = fmaxf(amax, fabsf(o));
+  }
+  for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
+  if (rs && lane == 0) rs[r] = pow2_scale(amax);
+}
+
+__global__ void k_add4(const float4* __restrict__ a, const float4* __restrict__ b,
+                       float4* __restrict__ out, int64_t n4) {
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= n4) return;
+  const float4 x = a[t], y = b[t];
+  out[t] = make_float4(x.x + y.x, x.y + y.y, x.z + y.z, x.w + y.w);
+}
+
+// dZ = (d1 + d2) ⊙ PReLU'_a(Z) row by row (8 rows per 256-thread block) with
+// the row's power-of-two scale and the block's dα partial Σ_{Z<=0} (d1+d2) Z.
+__global__ void __launch_bounds__(256) k_add_prelu_bwd(const float* __restrict__ d1,
+                                                       const float* __restrict__ d2,
+                                                       const float* __restrict__ Z,
+                                                       const float* __restrict__ alpha, int layer,
+                                                       int64_t R, int H, float* __restrict__ dZ,
+                                                       float* __restrict__ rs,
+                                                       double* __restrict__ slots) {
+  __shared__ double sh[8];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t r = (int64_t)blockIdx.x * 8 + w;
+  const float a = alpha[layer];
+  double da = 0.0;
+  float amax = 0.f;
+  if (r < R) {
+    for (int c = lane; c < H; c += 32) {
+      const int64_t e = r * H + c;
+      const float h = d1[e] + d2[e], z = Z[e];
+      const float o = z > 0.f ? h : a * h;
+      dZ[e] = o;
+      da += z > 0.f ? 0.0 : (double)(h * z);
+      amax = fmaxf(amax, fabsf(o));
+    }
+    for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
+    if (rs && lane == 0) rs[r] = pow2_scale(amax);
+  }
+  da = warp_sum(da);
+  if (lane == 0) sh[w] = da;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int k = 0; k < 8; ++k) t += sh[k];
+    slots[blockIdx.x] = t;
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_maxagg(const GraphDev& g, const float* U, const float* bp, int64_t R, int H,
+                          float* agg, int32_t* idx, float* rs, cudaStream_t s, int* launches) {
+  count_launch(launches);
+  if (R > 0)
+    k_maxagg<<<cdiv(R * 32, 256), 256, 0, s>>>(U, bp, g.rowptr, g.colind, g.Nt, R, H, agg, idx, rs);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_maxagg_bwd(const GraphDev& g, const float* dagg, const int32_t* idx,
+                              const float* U, const float* bp, int64_t R, int H, float* dU,
+                              float* rs, cudaStream_t s, int* launches) {
+  count_launch(launches);
+  if (R > 0)
+    k_maxagg_bwd<<<cdiv(R * 32, 256), 256, 0, s>>>(dagg, idx, U, bp, g.rowptr, g.colind, g.Nt, R,
+                                                   H, dU, rs);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_add(const float* a, const float* b, float* out, int64_t n, cudaStream_t s,
+                       int* launches) {
+  if (n % 4) return cudaErrorInvalidValue;
+  count_launch(launches);
+  if (n > 0)
+    k_add4<<<cdiv(n / 4, 256), 256, 0, s>>>(reinterpret_cast<const float4*>(a),
+                                            reinterpret_cast<const float4*>(b),
+                                            reinterpret_cast<float4*>(out), n / 4);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_add_prelu_bwd(const float* d1, const float* d2, const float* Z,
+                                 const float* alpha, int layer, int64_t R, int H, float* dZ,
+                                 float* rs, double* slots, int* nslots, cudaStream_t s,
+                                 int* launches) {
+  count_launch(launches);
+  *nslots = (int)cdiv(R, 8);
+  if (R > 0)
+    k_add_prelu_bwd<<<cdiv(R, 8), 256, 0, s>>>(d1, d2, Z, alpha, layer, R, H, dZ, rs, slots);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_sage_csr(const GraphDev& g, int64_t self_off, int32_t* colS, float* vf,
                             float* vb, float* vn, cudaStream_t s, int* launches) {

@@ -292,6 +292,22 @@ cudaError_t launch_sage_vals(const GraphDev& g, float* valsR, float* valsC, cuda
 // values (0, 1/deg_N(j)); vb / vn may be null.
 cudaError_t launch_sage_csr(const GraphDev& g, int64_t self_off, int32_t* colS, float* vf,
                             float* vb, float* vn, cudaStream_t s, int* launches);
+// SAGE-pool encoder (c40), over the R stacked rows (blocks of Nt rows, each
+// aggregating within its block): the element-wise max aggregation of
+// ReLU(U + bp) with its argmax, its backward (gradient routed to the argmax,
+// masked by ReLU'), z = a + b, and dZ = (d1 + d2) ⊙ PReLU' with dα block
+// partials (cdiv(R, 8) slots).  rs (row scales) may be null.
+cudaError_t launch_maxagg(const GraphDev& g, const float* U, const float* bp, int64_t R, int H,
+                          float* agg, int32_t* idx, float* rs, cudaStream_t s, int* launches);
+cudaError_t launch_maxagg_bwd(const GraphDev& g, const float* dagg, const int32_t* idx,
+                              const float* U, const float* bp, int64_t R, int H, float* dU,
+                              float* rs, cudaStream_t s, int* launches);
+cudaError_t launch_add(const float* a, const float* b, float* out, int64_t n, cudaStream_t s,
+                       int* launches);
+cudaError_t launch_add_prelu_bwd(const float* d1, const float* d2, const float* Z,
+                                 const float* alpha, int layer, int64_t R, int H, float* dZ,
+                                 float* rs, double* slots, int* nslots, cudaStream_t s,
+                                 int* launches);
 // out = PReLU_{*slope}(in) row by row (out may be null) + power-of-two row scales (rs may be null).
 cudaError_t launch_rowprep(const float* in, int64_t rows, int C, const float* slope, float* out,
                            float* rs, cudaStream_t s, int* launches);

@@ -375,6 +375,15 @@ struct Workspace {
   float* rsG = nullptr;
   void *s3_wt_hi[6] = {}, *s3_wt_lo[6] = {}, *s3_w_hi[6] = {}, *s3_w_lo[6] = {};
   float* s3_wsc[6] = {};
+  // SAGE-pool encoder (c40): per layer U_p = A W_p, the max aggregation, its
+  // argmax and row scales; scratch U_s / V (forward) = dA_s / dA_p (backward),
+  // dU_p and its row scales, a ones column (the pool-bias gradient), the nine
+  // weight matrices' 3xFP16 splits
+  float *pUP[3] = {}, *pAGG[3] = {}, *pRsAGG[3] = {};
+  int32_t* pIDX[3] = {};
+  float *pUS = nullptr, *pVV = nullptr, *pDUP = nullptr, *pRsDUP = nullptr, *pOnes = nullptr;
+  void *p3_wt_hi[9] = {}, *p3_wt_lo[9] = {}, *p3_w_hi[9] = {}, *p3_w_lo[9] = {};
+  float* p3_wsc[9] = {};
   std::vector<void*> owned;
   void release() {
     for (void* p : owned) cudaFree(p);
@@ -402,9 +411,10 @@ struct mars_dgi {
   mars_contrastive ct{1, MARS_CORRUPT_PERMUTE, 0.f, MARS_READOUT_SIGMOID_MEAN, MARS_AGG_GCN,
                       MARS_LOSS_BCE};
   bool sage = false;                // MARS_ENCODER_SAGE (c38)
+  bool pool = false;                // MARS_ENCODER_SAGE_POOL (c40)
   int ct_nb() const { return (ct.num_neg + 2) & ~1; }     // K + 1 blocks, rounded up to even
   bool ct_materialise() const {
-    return sage || ct.num_neg > 1 || ct.corruption != MARS_CORRUPT_PERMUTE;
+    return sage || pool || ct.num_neg > 1 || ct.corruption != MARS_CORRUPT_PERMUTE;
   }
   bool capture = true;
   int gemm_impl = 0;                // 0 auto (tcgen05 3xFP16 when supported), 1 SIMT FFMA
@@ -1021,10 +1031,11 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
     return fail(MARS_EINVAL, "MARS_BF16 needs hidden_dim in {128, 256} and in_dim in {64, 128, 256}");
   if (cfg->world_size < 1 || cfg->rank < 0 || cfg->rank >= cfg->world_size)
     return fail(MARS_EINVAL, "bad world_size/rank");
-  if (cfg->encoder != MARS_ENCODER_GCN && cfg->encoder != MARS_ENCODER_SAGE)
+  if (cfg->encoder != MARS_ENCODER_GCN && cfg->encoder != MARS_ENCODER_SAGE &&
+      cfg->encoder != MARS_ENCODER_SAGE_POOL)
     return fail(MARS_EINVAL, "unknown encoder %d", cfg->encoder);
-  if (cfg->encoder == MARS_ENCODER_SAGE && cfg->precision != MARS_FP32)
-    return fail(MARS_EINVAL, "the SAGE encoder runs MARS_FP32 only");
+  if (cfg->encoder != MARS_ENCODER_GCN && cfg->precision != MARS_FP32)
+    return fail(MARS_EINVAL, "the SAGE encoders run MARS_FP32 only");
   if (cfg->world_size > kMaxShards && !cfg->nccl_unique_id)
     return fail(MARS_EINVAL, "peer-memory data parallelism supports world_size <= %d", kMaxShards);
   int ndev = 0;
@@ -1042,7 +1053,10 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   m->F = cfg->in_dim;
   m->H = cfg->hidden_dim;
   m->sage = cfg->encoder == MARS_ENCODER_SAGE;
-  m->P = mars_num_params(m->F, m->H) + (m->sage ? (int64_t)m->F * m->H + 2LL * m->H * m->H : 0);
+  m->pool = cfg->encoder == MARS_ENCODER_SAGE_POOL;
+  m->P = m->pool ? 2LL * m->F * m->H + 8LL * m->H * m->H + 3LL * m->H + 3
+                 : mars_num_params(m->F, m->H) +
+                       (m->sage ? (int64_t)m->F * m->H + 2LL * m->H * m->H : 0);
   CK(cudaStreamCreateWithFlags(&m->own_stream, cudaStreamNonBlocking));
   m->stream = m->own_stream;
   CK(dalloc(&m->params, m->P));
@@ -1065,6 +1079,25 @@ extern "C" mars_status mars_dgi_create(const mars_dgi_config* cfg, mars_dgi** ou
   CK(cudaMemsetAsync(m->adam_st, 0, sizeof(AdamDev), s));
   if (cfg->init_params) {
     CK(cudaMemcpyAsync(m->params, cfg->init_params, sizeof(float) * m->P, cudaMemcpyHostToDevice, s));
+  } else if (m->pool) {            // c40: per layer W_s, W_n, W_p (tags 3l+1..3l+3), b_p = 0; M
+    const int F = m->F, H = m->H;
+    int64_t off = 0;
+    auto xav = [&](int tag, int64_t n, double fan) {
+      const float b = (float)std::sqrt(6.0 / fan);
+      k_xavier<<<cdiv(n, 256), 256, 0, s>>>(m->params + off, n, cfg->seed, (uint64_t)tag, b);
+      off += n;
+    };
+    for (int l = 0; l < 3; ++l) {
+      const int C = l == 0 ? F : H;
+      xav(3 * l + 1, (int64_t)C * H, (double)C + 2.0 * H);
+      xav(3 * l + 2, (int64_t)H * H, (double)C + 2.0 * H);
+      xav(3 * l + 3, (int64_t)C * H, (double)C + H);
+      CK(cudaMemsetAsync(m->params + off, 0, sizeof(float) * H, s));
+      off += H;
+    }
+    xav(10, (int64_t)H * H, 2.0 * H);
+    k_fill<<<1, 32, 0, s>>>(m->params + off, 3, 0.25f);
+    CK(cudaGetLastError());
   } else if (!m->sage) {
     int64_t off = 0;
     for (int t = 1; t <= 4; ++t) {
@@ -1162,8 +1195,8 @@ extern "C" mars_status mars_dgi_set_contrastive(mars_dgi* m, const mars_contrast
                     c->loss == MARS_LOSS_BCE;
   if (m->sh.g && !dflt) return fail(MARS_ESTATE, "a row-sharded model runs the default step only");
   if (memcmp(c, &m->ct, sizeof *c) == 0) return MARS_OK;     // unchanged: keep workspace and graphs
-  if (m->sage && c->aggregator != MARS_AGG_GCN)
-    return fail(MARS_EINVAL, "the SAGE encoder has its own aggregation (aggregator must be GCN)");
+  if ((m->sage || m->pool) && c->aggregator != MARS_AGG_GCN)
+    return fail(MARS_EINVAL, "the SAGE encoders have their own aggregation (aggregator must be GCN)");
   CK(cudaSetDevice(m->cfg.device));
   m->drop_execs();                 // captured steps bake the variant in
   CK(cudaStreamSynchronize(m->stream));
@@ -1200,12 +1233,12 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
   const GraphDev& pv = g->perm_view();
   const int nbk = m->ct_nb(), K = m->ct.num_neg;
   const bool xs = m->ct_materialise(), sage = m->ct.aggregator == MARS_AGG_SAGE_GCN;
-  const bool smean = m->sage;
+  const bool smean = m->sage, spool = m->pool;
   if (w.Nt >= g->dev.Nt && w.Nperm >= pv.Nt && w.G >= g->G && w.nchunks >= g->dev.nchunks &&
       w.nbuckets >= pv.nbuckets && w.nnz_perm >= pv.nnz && w.nlong >= g->dev.nlong &&
       w.nseg >= g->dev.nseg && w.F == m->F && w.H == m->H && w.nb == nbk && w.K == K &&
       (w.has_xs || !xs) && (!sage || w.nnz_vals >= g->dev.nnz) &&
-      (!smean || (w.sU && w.nnz_vals >= g->dev.nnz)))
+      (!smean || (w.sU && w.nnz_vals >= g->dev.nnz)) && (!spool || w.pUS))
     return MARS_OK;
   if (m->sh.g) return fail(MARS_ESTATE, "workspace of a shard-attached model cannot grow");
   m->drop_execs();
@@ -1256,6 +1289,30 @@ static mars_status ensure_ws(mars_dgi* m, const mars_graph* g) {
       CK(al(&w.s3_w_lo[t], 2 * n));
       CK(al((void**)&w.s3_wsc[t], sizeof(float) * 2));
     }
+  }
+  if (spool) {
+    for (int l = 0; l < 3; ++l) {
+      CK(al((void**)&w.pUP[l], sizeof(float) * R * H));
+      CK(al((void**)&w.pAGG[l], sizeof(float) * R * H));
+      CK(al((void**)&w.pIDX[l], sizeof(int32_t) * R * H));
+      CK(al((void**)&w.pRsAGG[l], sizeof(float) * R));
+    }
+    CK(al((void**)&w.pUS, sizeof(float) * R * H));
+    CK(al((void**)&w.pVV, sizeof(float) * R * H));
+    CK(al((void**)&w.pDUP, sizeof(float) * R * H));
+    CK(al((void**)&w.pRsDUP, sizeof(float) * R));
+    CK(al((void**)&w.pOnes, sizeof(float) * R));
+    k_fill<<<cdiv(R, 256), 256>>>(w.pOnes, R, 1.f);
+    CK(cudaGetLastError());
+    for (int t = 0; t < 9; ++t) {
+      const int64_t n = (int64_t)(t < 3 && t != 1 ? F : H) * H;    // layer 1: W_s, W_p are F x H
+      CK(al(&w.p3_wt_hi[t], 2 * n));
+      CK(al(&w.p3_wt_lo[t], 2 * n));
+      CK(al(&w.p3_w_hi[t], 2 * n));
+      CK(al(&w.p3_w_lo[t], 2 * n));
+      CK(al((void**)&w.p3_wsc[t], sizeof(float) * 2));
+    }
+    CK(cudaDeviceSynchronize());
   }
   CK(al((void**)&w.one, sizeof(float)));
   {
@@ -1349,6 +1406,198 @@ struct Profiler {
     for (cudaEvent_t e : ev) cudaEventDestroy(e);
   }
 };
+
+// Parameter blocks of the SAGE-pool encoder (c40): W_s, W_n, W_p, b_p of
+// layer l, then M and α.
+struct PoolParams {
+  float *Ws[3], *Wn[3], *Wp[3], *bp[3], *M, *alpha;
+};
+static PoolParams pool_params(float* P, int F, int H) {
+  PoolParams q{};
+  int64_t o = 0;
+  for (int l = 0; l < 3; ++l) {
+    const int64_t C = l == 0 ? F : H;
+    q.Ws[l] = P + o; o += C * H;
+    q.Wn[l] = P + o; o += (int64_t)H * H;
+    q.Wp[l] = P + o; o += C * H;
+    q.bp[l] = P + o; o += H;
+  }
+  q.M = P + o;
+  q.alpha = P + o + (int64_t)H * H;
+  return q;
+}
+
+// Row GEMM out[R x N] = A[R x K] W (W [K x N]) on the 3xFP16 tensor cores when
+// the widths allow (split t of the workspace), else FFMA.
+static cudaError_t pool_gemm(Workspace& w, bool tc, int t, const float* A, const float* rsA,
+                             const float* W, float* out, int64_t R, int N, int K, cudaStream_t s,
+                             int* nl) {
+  if (tc) return tc3h_gemm_rows(A, rsA, w.p3_wt_hi[t], w.p3_wt_lo[t], w.p3_wsc[t] + 1, out, R, N, K, s, nl);
+  return gemm_nn(A, W, out, R, N, K, s, nl);
+}
+// out[R x K] = D[R x N] Wᵀ (W [K x N]).
+static cudaError_t pool_gemm_t(Workspace& w, bool tc, int t, const float* D, const float* rsD,
+                               const float* W, float* out, int64_t R, int K, int N, cudaStream_t s,
+                               int* nl) {
+  if (tc) return tc3h_gemm_rows(D, rsD, w.p3_w_hi[t], w.p3_w_lo[t], w.p3_wsc[t] + 1, out, R, K, N, s, nl);
+  return gemm_nt(D, W, out, R, K, N, s, nl);
+}
+// dW [K x N] = Aᵀ D.
+static cudaError_t pool_dw(Workspace& w, bool tc, const float* A, const float* rsA, const float* D,
+                           const float* rsD, float* dW, int64_t R, int K, int N, cudaStream_t s,
+                           int* nl) {
+  if (tc) return tc3h_gemm_dw(A, rsA, D, rsD, dW, R, K, N, w.dw_part, s, nl);
+  return gemm_tn(A, D, dW, R, K, N, w.tn_part, s, nl);
+}
+
+// One SAGE-pool layer forward over R rows of A (C columns): Z = A W_s +
+// maxagg(ReLU(A W_p + b_p)) W_n.
+static cudaError_t pool_layer_fwd(mars_dgi* m, const GraphDev& g, const PoolParams& q, int l,
+                                  const float* A, const float* rsA, float* Z, int64_t R,
+                                  cudaStream_t s, int* nl) {
+  Workspace& w = m->ws;
+  const int H = m->H, C = l == 0 ? m->F : H;
+  const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+  const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(H, H);
+  cudaError_t e;
+  if ((e = pool_gemm(w, tcC, 3 * l + 2, A, rsA, q.Wp[l], w.pUP[l], R, H, C, s, nl))) return e;
+  if ((e = launch_maxagg(g, w.pUP[l], q.bp[l], R, H, w.pAGG[l], w.pIDX[l],
+                         tcH ? w.pRsAGG[l] : nullptr, s, nl)))
+    return e;
+  if ((e = pool_gemm(w, tcC, 3 * l, A, rsA, q.Ws[l], w.pUS, R, H, C, s, nl))) return e;
+  if ((e = pool_gemm(w, tcH, 3 * l + 1, w.pAGG[l], w.pRsAGG[l], q.Wn[l], w.pVV, R, H, H, s, nl)))
+    return e;
+  return launch_add(w.pUS, w.pVV, Z, R * H, s, nl);
+}
+
+static cudaError_t pool_splits(mars_dgi* m, const PoolParams& q, cudaStream_t s, int* nl) {
+  Workspace& w = m->ws;
+  const int F = m->F, H = m->H;
+  cudaError_t e;
+  for (int l = 0; l < 3; ++l) {
+    const int C = l == 0 ? F : H;
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(H, H);
+    const float* Wm[3] = {q.Ws[l], q.Wn[l], q.Wp[l]};
+    for (int h = 0; h < 3; ++h) {
+      const int K = h == 1 ? H : C;
+      if (!(h == 1 ? tcH : tcC)) continue;
+      const int t = 3 * l + h;
+      if ((e = tc3h_split_weights(Wm[h], K, H, w.p3_wsc[t], w.p3_wt_hi[t], w.p3_wt_lo[t],
+                                  w.p3_w_hi[t], w.p3_w_lo[t], s, nl)))
+        return e;
+    }
+  }
+  return cudaSuccess;
+}
+
+// The SAGE-pool encoder's step (c40).  Forward per layer as pool_layer_fwd;
+// the head as in the GCN step; backward per layer, from dZ:
+//   dW_s = Aᵀ dZ, dW_n = aggᵀ dZ, dagg = dZ W_nᵀ, dU_p = maxagg_bwd(dagg),
+//   dW_p = Aᵀ dU_p, db_p = 1ᵀ dU_p, and for l > 1
+//   dZ_{l-1} = (dZ W_sᵀ + dU_p W_pᵀ) ⊙ PReLU'(Z_{l-1}) with dα fused.
+static cudaError_t enqueue_step_pool(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl,
+                                     Profiler* prof) {
+  Workspace& w = m->ws;
+  GraphDev g = gr->dev;
+  g.long_part = w.long_part;
+  const int F = m->F, H = m->H;
+  const int nb = w.nb, K = m->ct.num_neg;
+  const int64_t Nt = g.Nt, R = (int64_t)(K + 1) * Nt;
+  const PoolParams q = pool_params(m->params, F, H), gq = pool_params(m->grads, F, H);
+  float* gloss = m->grads + m->P;
+  float* A[3] = {w.Xs, w.Y23[0], w.Y23[1]};
+  cudaError_t e;
+#define RET(x)                                  \
+  do {                                          \
+    if ((e = (x)) != cudaSuccess) return e;     \
+  } while (0)
+#define MARK(ph)                                \
+  do {                                          \
+    if (prof) RET(prof->mark(ph, s));           \
+  } while (0)
+  MARK(-1);
+  w.hw.nb = nb;
+  w.hw.K = K;
+  w.hw.readout = m->ct.readout;
+  w.hw.loss = m->ct.loss;
+  RET(launch_pair_off_k(g.pair_off, g.G, K, w.pair_off_k, s, nl));
+  if (m->ct.corruption == MARS_CORRUPT_PERMUTE)
+    for (int k = 0; k < K; ++k) {
+      GraphDev pv = g;
+      pv.pair_off = w.pair_off_k + (int64_t)k * g.G;
+      RET(launch_perm(pv, m->cfg.seed, m->d_sp, w.pw, w.perm + (int64_t)k * Nt, s, nl));
+    }
+  RET(launch_corrupt(g, K, nb, m->ct.corruption, m->ct.mask_rate, m->cfg.seed, m->d_sp,
+                     w.pair_off_k, w.perm, w.Xs, s, nl));
+  MARK(MARS_PH_PERM);
+  RET(pool_splits(m, q, s, nl));
+  MARK(MARS_PH_GEMM_FWD);
+  for (int l = 0; l < 3; ++l) {
+    const int C = l == 0 ? F : H;
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    if (l == 0) {
+      if (tcC) RET(launch_rowprep(w.Xs, R, F, w.one, nullptr, w.h3_rsY[0], s, nl));
+    } else {
+      RET(launch_rowprep(w.Z[l - 1], R, H, q.alpha + (l - 1), A[l], tcC ? w.h3_rsY[l] : nullptr,
+                         s, nl));
+    }
+    RET(pool_layer_fwd(m, g, q, l, A[l], w.h3_rsY[l], w.Z[l], R, s, nl));
+    MARK(MARS_PH_GEMM_FWD);
+  }
+  const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(H, H);
+  int ns = 0;
+  w.hw.rs_dz3 = tcH ? w.h3_rsdZ : nullptr;
+  RET(launch_head(g, H, w.Z[2], 0, q.M, q.alpha, m->d_sp, w.hw, w.dZ, gq.M, gloss, &ns, s, nl,
+                  nullptr));
+  RET(launch_reduce_slots(w.slots[2], ns, gq.alpha + 2, s, nl));
+  MARK(MARS_PH_HEAD);
+  for (int l = 2; l >= 0; --l) {
+    const int C = l == 0 ? F : H;
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    RET(pool_dw(w, tcC, A[l], w.h3_rsY[l], w.dZ, w.h3_rsdZ, gq.Ws[l], R, C, H, s, nl));
+    RET(pool_dw(w, tcH, w.pAGG[l], w.pRsAGG[l], w.dZ, w.h3_rsdZ, gq.Wn[l], R, H, H, s, nl));
+    MARK(MARS_PH_GEMM_DW);
+    RET(pool_gemm_t(w, tcH, 3 * l + 1, w.dZ, w.h3_rsdZ, q.Wn[l], w.dY, R, H, H, s, nl));   // dagg
+    MARK(MARS_PH_GEMM_DY);
+    RET(launch_maxagg_bwd(g, w.dY, w.pIDX[l], w.pUP[l], q.bp[l], R, H, w.pDUP,
+                          tcC ? w.pRsDUP : nullptr, s, nl));
+    MARK(MARS_PH_SPMM_BWD);
+    RET(pool_dw(w, tcC, A[l], w.h3_rsY[l], w.pDUP, w.pRsDUP, gq.Wp[l], R, C, H, s, nl));
+    RET(gemm_tn(w.pOnes, w.pDUP, gq.bp[l], R, 1, H, w.tn_part, s, nl));               // db_p
+    MARK(MARS_PH_GEMM_DW);
+    if (l > 0) {
+      RET(pool_gemm_t(w, tcC, 3 * l, w.dZ, w.h3_rsdZ, q.Ws[l], w.pUS, R, C, H, s, nl));     // dA_s
+      RET(pool_gemm_t(w, tcC, 3 * l + 2, w.pDUP, w.pRsDUP, q.Wp[l], w.pVV, R, C, H, s, nl));  // dA_p
+      MARK(MARS_PH_GEMM_DY);
+      const bool tcP = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(l - 1 == 0 ? F : H, H);
+      RET(launch_add_prelu_bwd(w.pUS, w.pVV, w.Z[l - 1], q.alpha, l - 1, R, H, w.dZ,
+                               tcP || tcH ? w.h3_rsdZ : nullptr, w.slots[l - 1], &ns, s, nl));
+      MARK(MARS_PH_SPMM_BWD);
+      RET(launch_reduce_slots(w.slots[l - 1], ns, gq.alpha + (l - 1), s, nl));
+      MARK(MARS_PH_REDUCE);
+    }
+  }
+  if (m->comm) {
+    ncclResult_t r = g_nccl.AllReduce(m->grads, m->grads, (size_t)(m->P + 1), ncclFloat32, ncclSum,
+                                      m->comm, s);
+    if (r != ncclSuccess) return cudaErrorUnknown;
+    MARK(MARS_PH_ALLREDUCE);
+  }
+  if (m->dp.connected) {
+    RET(launch_shard_barrier(m->dp.sync, s, nl));
+    RET(launch_grad_sum(m->dp.grads, m->dp.R, m->dp.me, m->P + 1, 0, 0, 1, m->dp.gsum, s, nl));
+    RET(launch_shard_barrier(m->dp.sync, s, nl));
+    MARK(MARS_PH_ALLREDUCE);
+  }
+  RET(launch_adam(m->params, m->adam_m, m->adam_v, m->grads_final(), m->P, m->cfg.lr,
+                  m->cfg.beta1, m->cfg.beta2, m->cfg.eps, m->cfg.clip_norm, m->guard_part,
+                  m->adam_st, s, nl));
+  MARK(MARS_PH_ADAM);
+#undef MARK
+#undef RET
+  return cudaSuccess;
+}
 
 // The SAGE-mean encoder's step (c38, MARS_ENCODER_SAGE), GEMM-first per layer:
 //   A_0 = X~ stacked (materialised, c34/c35), A_l = PReLU(Z_l) (+ row scales)
@@ -1517,6 +1766,7 @@ static cudaError_t enqueue_step_sage(mars_dgi* m, const mars_graph* gr, cudaStre
 static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl,
                                 Profiler* prof = nullptr) {
   if (m->sage) return enqueue_step_sage(m, gr, s, nl, prof);
+  if (m->pool) return enqueue_step_pool(m, gr, s, nl, prof);
   Workspace& w = m->ws;
   GraphDev g = gr->dev;
   g.long_part = w.long_part;
@@ -1997,8 +2247,34 @@ static cudaError_t enqueue_encode_sage(mars_dgi* m, const mars_graph* gr, cudaSt
   return launch_prelu(w.Z[2], 0, alpha, 2, w.dY, Nt * H, s, nl);
 }
 
+// a15 under the SAGE-pool encoder (c40): the positive rows only.
+static cudaError_t enqueue_encode_pool(mars_dgi* m, const mars_graph* gr, cudaStream_t s, int* nl) {
+  Workspace& w = m->ws;
+  GraphDev g = gr->dev;
+  g.long_part = w.long_part;
+  const int F = m->F, H = m->H;
+  const int64_t Nt = g.Nt;
+  const PoolParams q = pool_params(m->params, F, H);
+  const float* A[3] = {g.X, w.Y23[0], w.Y23[1]};
+  cudaError_t e;
+  if ((e = pool_splits(m, q, s, nl))) return e;
+  for (int l = 0; l < 3; ++l) {
+    const int C = l == 0 ? F : H;
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    if (l == 0) {
+      if (tcC && (e = launch_rowprep(g.X, Nt, F, w.one, nullptr, w.h3_rsY[0], s, nl))) return e;
+    } else if ((e = launch_rowprep(w.Z[l - 1], Nt, H, q.alpha + (l - 1), w.Y23[l - 1],
+                                   tcC ? w.h3_rsY[l] : nullptr, s, nl))) {
+      return e;
+    }
+    if ((e = pool_layer_fwd(m, g, q, l, A[l], w.h3_rsY[l], w.Z[l], Nt, s, nl))) return e;
+  }
+  return launch_prelu(w.Z[2], 0, q.alpha, 2, w.dY, Nt * H, s, nl);
+}
+
 static cudaError_t enqueue_encode(mars_dgi* m, const mars_graph* g, cudaStream_t s, int* nl) {
   if (m->sage) return enqueue_encode_sage(m, g, s, nl);
+  if (m->pool) return enqueue_encode_pool(m, g, s, nl);
   Workspace& w = m->ws;
   GraphDev gd = g->dev;
   gd.long_part = w.long_part;
@@ -2154,7 +2430,7 @@ extern "C" mars_status mars_dgi_export_activations(const mars_dgi* m, int32_t la
   CK(cudaSetDevice(m->cfg.device));
   CK(cudaStreamSynchronize(m->stream));
   int64_t R = 2LL * m->last_Nt;
-  const float* Ys[3] = {m->sage ? m->ws.Xs : m->ws.Y1, m->ws.Y23[0], m->ws.Y23[1]};
+  const float* Ys[3] = {(m->sage || m->pool) ? m->ws.Xs : m->ws.Y1, m->ws.Y23[0], m->ws.Y23[1]};
   int Cin = layer == 1 ? m->F : m->H;
   if (m->cfg.precision == MARS_BF16) {     // upcast bf16 storage through a scratch buffer
     float* tmp = nullptr;
@@ -2184,7 +2460,7 @@ extern "C" mars_status mars_dgi_saved_rows(const mars_dgi* m, int64_t* rows) {
 
 extern "C" mars_status mars_dgi_set_keep_backward(mars_dgi* m, int32_t keep) {
   if (mars_status st = check_dgi(m)) return st;
-  if (m->sage && keep) return fail(MARS_EINVAL, "no backward hook for the SAGE encoder");
+  if ((m->sage || m->pool) && keep) return fail(MARS_EINVAL, "no backward hook for the SAGE encoders");
   CK(cudaSetDevice(m->cfg.device));
   m->drop_execs();                 // recapture with / without the copies
   CK(cudaStreamSynchronize(m->stream));
@@ -2529,7 +2805,7 @@ extern "C" mars_status mars_shard_attach(mars_dgi* m, const mars_graph* g) {
   if (mars_status st = check_graph(g)) return st;
   if (!g->sharded) return fail(MARS_EINVAL, "graph was not loaded with mars_graph_load_shard");
   if (m->sh.g) return fail(MARS_ESTATE, "model already attached to a shard");
-  if (m->sage) return fail(MARS_EINVAL, "row sharding runs the GCN encoder only");
+  if (m->sage || m->pool) return fail(MARS_EINVAL, "row sharding runs the GCN encoder only");
   if (m->ct.num_neg != 1 || m->ct.corruption != MARS_CORRUPT_PERMUTE ||
       m->ct.readout != MARS_READOUT_SIGMOID_MEAN || m->ct.aggregator != MARS_AGG_GCN ||
       m->ct.loss != MARS_LOSS_BCE)
@@ -3206,7 +3482,7 @@ extern "C" mars_status mars_dgi_encoder_vjp(mars_dgi* m, const mars_graph* g, co
   if (!dE || !grads) return fail(MARS_EINVAL, "NULL argument");
   if (g->sharded || g->F != m->F) return fail(MARS_EINVAL, "unsharded graph of the model's F");
   if (m->cfg.precision != MARS_FP32) return fail(MARS_EINVAL, "fp32 models only");
-  if (m->sage) return fail(MARS_EINVAL, "no encoder VJP for the SAGE encoder");
+  if (m->sage || m->pool) return fail(MARS_EINVAL, "no encoder VJP for the SAGE encoders");
   CK(cudaSetDevice(m->cfg.device));
   if (mars_status st = ensure_ws(m, g)) return st;
   cudaStream_t s = m->stream;
@@ -3273,7 +3549,8 @@ extern "C" mars_status mars_ppo_create(mars_placer* p, mars_dgi* enc, const mars
   if (enc) {
     if (mars_status st = check_dgi(enc)) return st;
     if (enc->H != p->d.H) return fail(MARS_EINVAL, "encoder hidden_dim != placer in_dim");
-    if (enc->sage) return fail(MARS_EINVAL, "the joint update needs the GCN encoder (no SAGE VJP)");
+    if (enc->sage || enc->pool)
+      return fail(MARS_EINVAL, "the joint update needs the GCN encoder (no SAGE VJP)");
     if (enc->cfg.device != p->cfg.device) return fail(MARS_EINVAL, "encoder and placer on different devices");
   }
   if (!cfg) return fail(MARS_EINVAL, "NULL config");

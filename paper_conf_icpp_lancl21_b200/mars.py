@@ -78,7 +78,7 @@ CORRUPTIONS = {"permute": 0, "mask": 1}
 READOUTS = {"sigmoid_mean": 0, "mean": 1}
 AGGREGATORS = {"gcn": 0, "sage_gcn": 1}
 LOSSES = {"bce": 0, "infonce": 1}
-ENCODERS = {"gcn": 0, "sage": 1}
+ENCODERS = {"gcn": 0, "sage": 1, "sage_pool": 2}
 
 
 class StepOut(ctypes.Structure):

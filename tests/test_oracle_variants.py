@@ -344,3 +344,98 @@ def test_infonce_gradients_finite_differences(kw):
         fd = (V.step_grads(gs, pp, F, H, SEED, STEP, loss="infonce", **kw)[0]
               - V.step_grads(gs, pm, F, H, SEED, STEP, loss="infonce", **kw)[0]) / (2 * h)
         assert abs(fd - grads[i]) <= 1e-7 + 1e-5 * abs(grads[i]), (i, fd, grads[i])
+
+
+# ----------------------------------------------------------------- SAGE-pool (c40)
+def _pool_blocks(p):
+    o, layers = 0, []
+    for l in range(3):
+        C = F if l == 0 else H
+        Ws = p[o:o + C * H].reshape(C, H); o += C * H
+        Wn = p[o:o + H * H].reshape(H, H); o += H * H
+        Wp = p[o:o + C * H].reshape(C, H); o += C * H
+        bp = p[o:o + H]; o += H
+        layers.append((Ws, Wn, Wp, bp))
+    return layers, p[-3:]
+
+
+def test_sage_pool_init_layout():
+    p = V.sage_pool_init(3, F, H)
+    assert p.size == V.num_params(F, H, "sage_pool")
+    layers, al = _pool_blocks(p.astype(np.float64))
+    for l, (Ws, Wn, Wp, bp) in enumerate(layers):
+        C = F if l == 0 else H
+        assert np.all(np.abs(Ws) <= np.float32(np.sqrt(6.0 / (C + 2 * H))))
+        assert np.all(np.abs(Wp) <= np.float32(np.sqrt(6.0 / (C + H))))
+        assert np.all(bp == 0)
+    assert np.array_equal(al, np.full(3, 0.25))
+
+
+def test_sage_pool_encoder_brute_force_loops():
+    """c40 as per-node loops: P = ReLU(h W_p + b); agg_i = element-wise max over
+    the neighbours (0 when there are none); h' = PReLU(h W_s + agg W_n)."""
+    g = SG.tiny(5, N=26)
+    p = V.sage_pool_init(21, F, H).astype(np.float64)
+    rng = np.random.default_rng(0)
+    layers, al = _pool_blocks(p)
+    layers = [(Ws, Wn, Wp, rng.standard_normal(H) * 0.1) for Ws, Wn, Wp, _ in layers]
+    q = p.copy()                                     # non-zero biases
+    o = 0
+    for l in range(3):
+        C = F if l == 0 else H
+        o += 2 * C * H + H * H
+        q[o:o + H] = layers[l][3]
+        o += H
+    nb = [set() for _ in range(g.num_nodes)]
+    for u in range(g.num_nodes):
+        for e in range(int(g.indptr[u]), int(g.indptr[u + 1])):
+            v = int(g.indices[e])
+            if v != u:
+                nb[u].add(v); nb[v].add(u)
+    h = np.asarray(g.features, np.float64)
+    for l in range(3):
+        Ws, Wn, Wp, bp = layers[l]
+        P = np.maximum(h @ Wp + bp, 0.0)
+        out = np.zeros((g.num_nodes, H))
+        for i in range(g.num_nodes):
+            agg = np.max(P[sorted(nb[i])], axis=0) if nb[i] else np.zeros(H)
+            out[i] = _prelu(h[i] @ Ws + agg @ Wn, al[l])
+        h = out
+    got = V.encode([g], q, F, H, encoder_="sage_pool")
+    assert np.max(np.abs(got - h)) < 1e-12 * max(1.0, np.max(np.abs(h)))
+
+
+def test_sage_pool_wn_zero_is_an_mlp():
+    g = SG.tiny(6, N=30)
+    p = V.sage_pool_init(4, F, H).astype(np.float64)
+    layers, al = _pool_blocks(p)
+    q = p.copy()
+    o = 0
+    for l in range(3):
+        C = F if l == 0 else H
+        q[o + C * H:o + C * H + H * H] = 0.0         # W_n = 0
+        o += 2 * C * H + H * H + H
+    h = np.asarray(g.features, np.float64)
+    for l in range(3):
+        h = _prelu(h @ layers[l][0], al[l])
+    got = V.encode([g], q, F, H, encoder_="sage_pool")
+    assert np.max(np.abs(got - h)) < 1e-12 * max(1.0, np.max(np.abs(h)))
+
+
+@pytest.mark.parametrize("kw", [dict(), dict(num_neg=2, corruption="mask", mask_rate=0.3),
+                                dict(num_neg=2, loss="infonce")])
+def test_sage_pool_gradients_finite_differences(kw):
+    gs = [SG.tiny(7, N=17)]
+    p = V.sage_pool_init(8, F, H).astype(np.float64)
+    _, grads = V.step_grads(gs, p, F, H, SEED, STEP, encoder="sage_pool", **kw)
+    rng = np.random.default_rng(5)
+    # weights of every block incl. W_p and the pool bias b_p of layer 1
+    idx = list(rng.choice(p.size - 3, 6, replace=False)) + [2 * F * H + H * H + 3, p.size - 1]
+    for i in idx:
+        h = 1e-6
+        pp, pm = p.copy(), p.copy()
+        pp[i] += h
+        pm[i] -= h
+        fd = (V.step_grads(gs, pp, F, H, SEED, STEP, encoder="sage_pool", **kw)[0]
+              - V.step_grads(gs, pm, F, H, SEED, STEP, encoder="sage_pool", **kw)[0]) / (2 * h)
+        assert abs(fd - grads[i]) <= 1e-7 + 1e-5 * abs(grads[i]), (i, fd, grads[i])

@@ -56,3 +56,4 @@ run("InfoNCE, K=4", base, dict(num_neg=4, loss="infonce"), B)
 run("SAGE-GCN", base, dict(aggregator="sage_gcn"), B)
 run("SAGE-mean encoder", base, {}, B, encoder="sage")
 run("SAGE-mean encoder, K=3", base, dict(num_neg=3), B, encoder="sage")
+run("SAGE-pool encoder", base, {}, B, encoder="sage_pool")
