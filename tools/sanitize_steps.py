@@ -26,7 +26,10 @@ variants = [([SG.tiny(0), SG.tiny(1)], 16, 32, mars.MARS_FP32, "gcn",
             ([SG.cached("inception", 0)], 64, 256, mars.MARS_BF16, "gcn", dict(num_neg=2)),
             ([SG.tiny(0), SG.tiny(1)], 16, 32, mars.MARS_FP32, "sage", dict(num_neg=2)),
             ([SG.cached("inception", 0)], 64, 256, mars.MARS_FP32, "sage",
-             dict(num_neg=4, corruption="mask", mask_rate=0.2))]
+             dict(num_neg=4, corruption="mask", mask_rate=0.2)),
+            ([SG.tiny(0), SG.tiny(1)], 16, 32, mars.MARS_FP32, "sage_pool", dict(num_neg=2)),
+            ([SG.cached("inception", 0)], 64, 128, mars.MARS_FP32, "sage_pool",
+             dict(num_neg=3, loss="infonce"))]
 only = os.environ.get("MARS_SAN_ONLY", "")
 runs = ([] if only == "variants" else [(gs, F, H, p, "gcn", {}) for gs, F, H, p in cases]) + \
     ([] if only == "default" else variants)
