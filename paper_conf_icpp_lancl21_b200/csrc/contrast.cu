@@ -150,34 +150,54 @@ __global__ void k_rowprep(const float* __restrict__ in, int64_t rows, int C,
 // stride the H columns.
 // agg[r][c] = max_{j in N(i), j != i} ReLU(U[b Nt + j][c] + bp[c]) (0 without
 // neighbours), idx[r][c] = the first j (ascending) attaining it (-1 without).
+// Lanes own 4-column slices (16-byte loads), neighbours in the outer loop.
+template <int H>
 __global__ void k_maxagg(const float* __restrict__ U, const float* __restrict__ bp,
                          const int32_t* __restrict__ rowptr, const int32_t* __restrict__ colind,
-                         int32_t Nt, int64_t R, int H, float* __restrict__ agg,
+                         int32_t Nt, int64_t R, float* __restrict__ agg,
                          int32_t* __restrict__ idx, float* __restrict__ rs) {
+  constexpr int LPR = H / 4 < 32 ? H / 4 : 32, PER = H / (4 * LPR);
   const int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (r >= R) return;
+  const bool act = lane < LPR;
   const int64_t base = r / Nt * Nt;
   const int32_t i = (int32_t)(r - base);
   const int32_t k0 = rowptr[i], k1 = rowptr[i + 1];
-  float amax = 0.f;
-  for (int c = lane; c < H; c += 32) {
-    const float b = bp[c];
-    float m = -1.f;
-    int32_t a = -1;
-    for (int32_t k = k0; k < k1; ++k) {
-      const int32_t j = colind[k];
-      if (j == i) continue;
-      const float v = fmaxf(U[(base + j) * H + c] + b, 0.f);
-      if (v > m) {
-        m = v;
-        a = j;
+  float b[PER][4], m[PER][4];
+  int32_t a[PER][4];
+#pragma unroll
+  for (int q = 0; q < PER; ++q) {
+    const float4 bv = act ? reinterpret_cast<const float4*>(bp)[lane + q * LPR] : float4{};
+    b[q][0] = bv.x; b[q][1] = bv.y; b[q][2] = bv.z; b[q][3] = bv.w;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) { m[q][e] = -1.f; a[q][e] = -1; }
+  }
+  for (int32_t k = k0; k < k1; ++k) {
+    const int32_t j = colind[k];
+    if (j == i || !act) continue;
+    const float4* row = reinterpret_cast<const float4*>(U + (base + j) * H);
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const float4 u = row[lane + q * LPR];
+      const float x[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float v = fmaxf(x[e] + b[q][e], 0.f);
+        if (v > m[q][e]) { m[q][e] = v; a[q][e] = j; }
       }
     }
-    const float o = a < 0 ? 0.f : m;
-    agg[r * H + c] = o;
-    idx[r * H + c] = a;
-    amax = fmaxf(amax, o);
+  }
+  float amax = 0.f;
+  if (act) {
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      float o[4];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) { o[e] = a[q][e] < 0 ? 0.f : m[q][e]; amax = fmaxf(amax, o[e]); }
+      reinterpret_cast<float4*>(agg + r * H)[lane + q * LPR] = make_float4(o[0], o[1], o[2], o[3]);
+      reinterpret_cast<int4*>(idx + r * H)[lane + q * LPR] = make_int4(a[q][0], a[q][1], a[q][2], a[q][3]);
+    }
   }
   for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
   if (rs && lane == 0) rs[r] = pow2_scale(amax);
@@ -186,29 +206,53 @@ __global__ void k_maxagg(const float* __restrict__ U, const float* __restrict__ 
 // dU[r][c] = [U[r][c] + bp[c] > 0] Σ_{i in N(j), i != j, idx[b Nt + i][c] == j}
 // dagg[b Nt + i][c] (row r = b Nt + j; the pattern is symmetric, so the rows
 // whose max j won are among j's own neighbours; ascending i: deterministic).
+template <int H>
 __global__ void k_maxagg_bwd(const float* __restrict__ dagg, const int32_t* __restrict__ idx,
                              const float* __restrict__ U, const float* __restrict__ bp,
                              const int32_t* __restrict__ rowptr,
-                             const int32_t* __restrict__ colind, int32_t Nt, int64_t R, int H,
+                             const int32_t* __restrict__ colind, int32_t Nt, int64_t R,
                              float* __restrict__ dU, float* __restrict__ rs) {
+  constexpr int LPR = H / 4 < 32 ? H / 4 : 32, PER = H / (4 * LPR);
   const int64_t r = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int lane = threadIdx.x & 31;
   if (r >= R) return;
+  const bool act = lane < LPR;
   const int64_t base = r / Nt * Nt;
   const int32_t j = (int32_t)(r - base);
   const int32_t k0 = rowptr[j], k1 = rowptr[j + 1];
-  float amax = 0.f;
-  for (int c = lane; c < H; c += 32) {
-    float acc = 0.f;
-    for (int32_t k = k0; k < k1; ++k) {
-      const int32_t i = colind[k];
-      if (i == j) continue;
-      const int64_t e = (base + i) * H + c;
-      if (idx[e] == j) acc += dagg[e];
+  float acc[PER][4];
+#pragma unroll
+  for (int q = 0; q < PER; ++q)
+#pragma unroll
+    for (int e = 0; e < 4; ++e) acc[q][e] = 0.f;
+  for (int32_t k = k0; k < k1; ++k) {
+    const int32_t i = colind[k];
+    if (i == j || !act) continue;
+    const int4* ix = reinterpret_cast<const int4*>(idx + (base + i) * H);
+    const float4* dg = reinterpret_cast<const float4*>(dagg + (base + i) * H);
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const int4 w = ix[lane + q * LPR];
+      if (w.x != j && w.y != j && w.z != j && w.w != j) continue;
+      const float4 d = dg[lane + q * LPR];
+      if (w.x == j) acc[q][0] += d.x;
+      if (w.y == j) acc[q][1] += d.y;
+      if (w.z == j) acc[q][2] += d.z;
+      if (w.w == j) acc[q][3] += d.w;
     }
-    const float o = U[r * H + c] + bp[c] > 0.f ? acc : 0.f;
-    dU[r * H + c] = o;
-    amax = fmaxf(amax, fabsf(o));
+  }
+  float amax = 0.f;
+  if (act) {
+#pragma unroll
+    for (int q = 0; q < PER; ++q) {
+      const float4 u = reinterpret_cast<const float4*>(U + r * H)[lane + q * LPR];
+      const float4 bv = reinterpret_cast<const float4*>(bp)[lane + q * LPR];
+      const float o[4] = {u.x + bv.x > 0.f ? acc[q][0] : 0.f, u.y + bv.y > 0.f ? acc[q][1] : 0.f,
+                          u.z + bv.z > 0.f ? acc[q][2] : 0.f, u.w + bv.w > 0.f ? acc[q][3] : 0.f};
+#pragma unroll
+      for (int e = 0; e < 4; ++e) amax = fmaxf(amax, fabsf(o[e]));
+      reinterpret_cast<float4*>(dU + r * H)[lane + q * LPR] = make_float4(o[0], o[1], o[2], o[3]);
+    }
   }
   for (int o = 16; o > 0; o >>= 1) amax = fmaxf(amax, __shfl_xor_sync(0xffffffffu, amax, o));
   if (rs && lane == 0) rs[r] = pow2_scale(amax);
@@ -264,8 +308,15 @@ __global__ void __launch_bounds__(256) k_add_prelu_bwd(const float* __restrict__
 cudaError_t launch_maxagg(const GraphDev& g, const float* U, const float* bp, int64_t R, int H,
                           float* agg, int32_t* idx, float* rs, cudaStream_t s, int* launches) {
   count_launch(launches);
-  if (R > 0)
-    k_maxagg<<<cdiv(R * 32, 256), 256, 0, s>>>(U, bp, g.rowptr, g.colind, g.Nt, R, H, agg, idx, rs);
+  if (R <= 0) return cudaSuccess;
+  const unsigned nb = cdiv(R * 32, 256);
+  switch (H) {
+#define MAXAGG(HH) \
+  case HH: k_maxagg<HH><<<nb, 256, 0, s>>>(U, bp, g.rowptr, g.colind, g.Nt, R, agg, idx, rs); break;
+    MAXAGG(32) MAXAGG(64) MAXAGG(128) MAXAGG(256)
+#undef MAXAGG
+    default: return cudaErrorInvalidValue;
+  }
   return cudaGetLastError();
 }
 
@@ -273,9 +324,17 @@ cudaError_t launch_maxagg_bwd(const GraphDev& g, const float* dagg, const int32_
                               const float* U, const float* bp, int64_t R, int H, float* dU,
                               float* rs, cudaStream_t s, int* launches) {
   count_launch(launches);
-  if (R > 0)
-    k_maxagg_bwd<<<cdiv(R * 32, 256), 256, 0, s>>>(dagg, idx, U, bp, g.rowptr, g.colind, g.Nt, R,
-                                                   H, dU, rs);
+  if (R <= 0) return cudaSuccess;
+  const unsigned nb = cdiv(R * 32, 256);
+  switch (H) {
+#define MAXBWD(HH)                                                                             \
+  case HH:                                                                                     \
+    k_maxagg_bwd<HH><<<nb, 256, 0, s>>>(dagg, idx, U, bp, g.rowptr, g.colind, g.Nt, R, dU, rs); \
+    break;
+    MAXBWD(32) MAXBWD(64) MAXBWD(128) MAXBWD(256)
+#undef MAXBWD
+    default: return cudaErrorInvalidValue;
+  }
   return cudaGetLastError();
 }
 
