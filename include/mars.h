@@ -170,10 +170,11 @@ MARS_API mars_status mars_nccl_get_unique_id(void* out128);
  * of the library stream.  NULL restores the library stream. */
 MARS_API mars_status mars_dgi_set_stream(mars_dgi* m, void* cuda_stream);
 /* Dense-transform implementation (a6/a12) of the MARS_FP32 path.
- * MARS_GEMM_AUTO (default), when H in {128, 256} and C_in in {64, 128, 256}:
- *   tcgen05 tensor cores at fp32 accuracy -- Z = Y·W, dY = dZ·Wᵀ and
- *   dW = Yᵀ·dZ as 3xFP16 with exact power-of-two row / tensor scaling
- *   (kind::f16); FFMA for the other widths (H in {32, 64}, C_in in {16, 32}).
+ * MARS_GEMM_AUTO (default): tcgen05 tensor cores at fp32 accuracy for every
+ *   supported width -- Z = Y·W, dY = dZ·Wᵀ and dW = Yᵀ·dZ as 3xFP16 with
+ *   exact power-of-two row / tensor scaling (kind::f16); the narrow widths of
+ *   the tiny configuration (H in {32, 64}, C_in in {16, 32}) run on wider
+ *   tiles whose missing rows / columns TMA zero-fills.
  * MARS_GEMM_SIMT: always FFMA (A/B comparisons).
  * (The MARS_BF16 path always uses its bf16 kernels.) */
 enum { MARS_GEMM_AUTO = 0, MARS_GEMM_SIMT = 1 };

@@ -53,7 +53,10 @@ bool tc_tmap_blocks(CUtensorMap* m, CUtensorMapDataType dt, int elem_bytes, cons
                     int64_t rows, int64_t cols, int box_rows, int nblk) {
   if (!encode_fn()) return false;
   const cuuint64_t bc = 128 / elem_bytes;            // columns per 128-byte block
-  cuuint64_t dims[3] = {bc, (cuuint64_t)rows, (cuuint64_t)(cols / bc)};
+  // a row narrower than one block (C_in = 16 fp32): one partial block; the
+  // box's remaining columns and blocks are zero-filled
+  cuuint64_t dims[3] = {std::min<cuuint64_t>(bc, (cuuint64_t)cols), (cuuint64_t)rows,
+                        std::max<cuuint64_t>(1, (cuuint64_t)cols / bc)};
   cuuint64_t strides[2] = {(cuuint64_t)cols * elem_bytes, 128};
   cuuint32_t box[3] = {(cuuint32_t)bc, (cuuint32_t)box_rows, (cuuint32_t)nblk};
   cuuint32_t es[3] = {1, 1, 1};
@@ -75,6 +78,15 @@ int tc_num_sms() {
 
 bool tc_supported(int K_or_cin, int N_or_h) {
   return (N_or_h == 128 || N_or_h == 256) && (K_or_cin == 64 || K_or_cin == 128 || K_or_cin == 256);
+}
+
+// The 3xFP16 kernels also take the narrow widths of the tiny configuration
+// (H in {32, 64}, C_in in {16, 32}) on zero-filled wider tiles.
+bool tc3h_supported(int K_or_cin, int N_or_h) {
+  const bool n = N_or_h == 32 || N_or_h == 64 || N_or_h == 128 || N_or_h == 256;
+  const bool k = K_or_cin == 16 || K_or_cin == 32 || K_or_cin == 64 || K_or_cin == 128 ||
+                 K_or_cin == 256;
+  return n && k;
 }
 
 // Row chunks of the split-K weight gradient so that chunks x C_in tiles is

@@ -105,7 +105,7 @@ k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUt
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int ntiles = (M + kBM - 1) / kBM;
-  const int nk = K / kBK;
+  const int nk = (K + kBK - 1) / kBK;    // K = 16: one block, TMA zero-fills the rest
   auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
   auto stB = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
   auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES + Cfg::B_BYTES; };
@@ -345,8 +345,10 @@ __global__ void k_split_w3h(const float* __restrict__ W, int CIN, int H,
 }
 
 template <int N>
+// N = the tile width (64, 128, 256); n = the actual output width (n <= N: the
+// weight rows beyond n are zero-filled by TMA and the store is clipped to n).
 cudaError_t rows3h_n(const float* A, const float* rs, const __half* Bhi, const __half* Blo,
-                     const float* inv_tb, float* C, int64_t M, int K, cudaStream_t s) {
+                     const float* inv_tb, float* C, int64_t M, int K, int n, cudaStream_t s) {
   using Cfg = H3Cfg<N>;
   static bool attr = false;
   if (!attr) {
@@ -358,11 +360,11 @@ cudaError_t rows3h_n(const float* A, const float* rs, const __half* Bhi, const _
   CUtensorMap ta, tbh, tbl, tc;
   if (!tc_tmap(&ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, A, M, K, kBK, kBM,
                CU_TENSOR_MAP_SWIZZLE_128B) ||
-      !tc_tmap(&tbh, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Bhi, N, K, kBK, N,
+      !tc_tmap(&tbh, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Bhi, n, K, kBK, N,
                CU_TENSOR_MAP_SWIZZLE_64B) ||
-      !tc_tmap(&tbl, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Blo, N, K, kBK, N,
+      !tc_tmap(&tbl, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Blo, n, K, kBK, N,
                CU_TENSOR_MAP_SWIZZLE_64B) ||
-      !tc_tmap(&tc, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, C, M, N, 32, 32,
+      !tc_tmap(&tc, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, C, M, n, 32, 32,
                CU_TENSOR_MAP_SWIZZLE_128B))
     return cudaErrorInvalidValue;
   const int ntiles = (int)((M + kBM - 1) / kBM);
@@ -414,7 +416,9 @@ template <int CINT, int HH>
 __global__ void __launch_bounds__(384, 1)
 k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
           const float* __restrict__ rs_dz, const float* __restrict__ rs_y,
-          float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN) {
+          float* __restrict__ part, int32_t R, int32_t rows_per_chunk, int32_t CIN, int32_t Hn) {
+  // Hn <= HH, CIN: the actual widths (narrower operands are zero-filled by TMA;
+  // the partial [chunk][Hn][CIN] is written for the actual widths only)
   using Cfg = H3DwCfg<CINT, HH>;
   constexpr int NH = Cfg::NH;
   constexpr int S = kDwStages;
@@ -431,7 +435,7 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
   float* wmin = reinterpret_cast<float*>(bars + 3 * S + 6);   // [2][10] per-warp minima
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int ntile = CIN / CINT;
+  const int ntile = (CIN + CINT - 1) / CINT;
   const int chunk = blockIdx.x / ntile, c_off = (blockIdx.x % ntile) * CINT;
   const int32_t r0 = chunk * rows_per_chunk;
   const int32_t r1 = min(R, r0 + rows_per_chunk);
@@ -621,14 +625,18 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
     if (folder) {
       while (folded < nsub) fold(folded++);
       const float inv = 1.f / (sz * sy);                   // exact (powers of two)
-      float* out = part + (int64_t)chunk * HH * CIN + c_off + ch * MC;
+      float* out = part + (int64_t)chunk * Hn * CIN + c_off + ch * MC;
+      const int cend = CIN - (c_off + ch * MC);            // columns of this thread that exist
 #pragma unroll
       for (int h = 0; h < NH; ++h) {
-        float4* dst = reinterpret_cast<float4*>(out + (int64_t)(h * 128 + q * 32 + lane) * CIN);
+        const int hr = h * 128 + q * 32 + lane;
+        if (hr >= Hn) continue;
+        float4* dst = reinterpret_cast<float4*>(out + (int64_t)hr * CIN);
 #pragma unroll
         for (int j = 0; j < MC / 4; ++j)
-          dst[j] = make_float4(master[h][4 * j] * inv, master[h][4 * j + 1] * inv,
-                               master[h][4 * j + 2] * inv, master[h][4 * j + 3] * inv);
+          if (4 * j < cend)
+            dst[j] = make_float4(master[h][4 * j] * inv, master[h][4 * j + 1] * inv,
+                                 master[h][4 * j + 2] * inv, master[h][4 * j + 3] * inv);
       }
     }
   }
@@ -906,7 +914,7 @@ __global__ void k_dw3h_reduce(const float* __restrict__ part, int nchunk, int CI
 
 template <int CINT, int HH>
 cudaError_t dw3h_c(const float* Y, const float* rs_y, const float* dZ, const float* rs_dz,
-                   float* part, int nchunk, int64_t R, int rows, int CIN, cudaStream_t s) {
+                   float* part, int nchunk, int64_t R, int rows, int CIN, int H, cudaStream_t s) {
   using Cfg = H3DwCfg<CINT, HH>;
   static bool attr = false;
   if (!attr) {
@@ -916,11 +924,11 @@ cudaError_t dw3h_c(const float* Y, const float* rs_y, const float* dZ, const flo
     attr = true;
   }
   CUtensorMap tdz, ty;
-  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, HH, kDwBK, HH / 32) ||
+  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, H, kDwBK, HH / 32) ||
       !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, CIN, kDwBK, CINT / 32))
     return cudaErrorInvalidValue;
-  k_tc3h_dw<CINT, HH><<<nchunk * (CIN / CINT), 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part,
-                                                                   (int32_t)R, rows, CIN);
+  k_tc3h_dw<CINT, HH><<<nchunk * ((CIN + CINT - 1) / CINT), 384, Cfg::SMEM, s>>>(
+      tdz, ty, rs_dz, rs_y, part, (int32_t)R, rows, CIN, H);
   return cudaGetLastError();
 }
 
@@ -997,13 +1005,14 @@ cudaError_t tc3h_gemm_rows(const float* A, const float* rs, const void* B_hi, co
                            const float* inv_tb, float* C, int64_t M, int N, int K, cudaStream_t s,
                            int* launches) {
   count_launch(launches);
-  if (K % kBK || K > 256) return cudaErrorInvalidValue;
+  if (K % 16 || K > 256) return cudaErrorInvalidValue;
   const __half* bh = static_cast<const __half*>(B_hi);
   const __half* bl = static_cast<const __half*>(B_lo);
   switch (N) {
-    case 64: return rows3h_n<64>(A, rs, bh, bl, inv_tb, C, M, K, s);
-    case 128: return rows3h_n<128>(A, rs, bh, bl, inv_tb, C, M, K, s);
-    case 256: return rows3h_n<256>(A, rs, bh, bl, inv_tb, C, M, K, s);
+    case 32:
+    case 64: return rows3h_n<64>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
+    case 128: return rows3h_n<128>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
+    case 256: return rows3h_n<256>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -1019,7 +1028,7 @@ cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, con
   rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
   nchunk = (int)((R + rows - 1) / rows);
   cudaError_t e;
-  if (H != 128 && H != 256) return cudaErrorInvalidValue;
+  if (H != 32 && H != 64 && H != 128 && H != 256) return cudaErrorInvalidValue;
   if (CIN == 256 && H == 256 && kDwPair) {
     // one wave: as many row chunks as CTA pairs can be co-resident (a pair
     // needs both SMs of a TPC free; not every SM can be paired)
@@ -1032,12 +1041,16 @@ cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, con
     k_dw3h_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
     return cudaGetLastError();
   }
+  // H in {32, 64} runs the H = 128 tiles and C_in in {16, 32} the 64-column
+  // tiles (TMA zero-fills the missing columns; only the real ones are written)
   switch (CIN) {
-    case 64: e = H == 256 ? dw3h_c<64, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s)
-                          : dw3h_c<64, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s); break;
+    case 16:
+    case 32:
+    case 64: e = H == 256 ? dw3h_c<64, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, H, s)
+                          : dw3h_c<64, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, H, s); break;
     case 128:
-    case 256: e = H == 256 ? dw3h_c<128, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s)
-                           : dw3h_c<128, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, s); break;
+    case 256: e = H == 256 ? dw3h_c<128, 256>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, H, s)
+                           : dw3h_c<128, 128>(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, CIN, H, s); break;
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;

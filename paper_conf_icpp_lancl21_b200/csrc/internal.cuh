@@ -201,6 +201,7 @@ cudaError_t gemm_tn(const float* A, const float* B, float* out, int64_t R, int M
 // ---------------------------------------------------------------- gemm_common.cu
 // tcgen05 GEMMs are specialised for H in {128, 256} and C_in in {64, 128, 256}.
 bool tc_supported(int cin, int h);
+bool tc3h_supported(int cin, int h);   // the 3xFP16 fp32 path (also the tiny widths)
 size_t tc_dw_partial_floats(int64_t R, int CIN);
 // gemm_tc3h.cu: 3xFP16 row GEMMs with power-of-two scaling (fp32 path)
 cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void* Bt_hi,

@@ -1457,8 +1457,8 @@ static cudaError_t pool_layer_fwd(mars_dgi* m, const GraphDev& g, const PoolPara
                                   cudaStream_t s, int* nl) {
   Workspace& w = m->ws;
   const int H = m->H, C = l == 0 ? m->F : H;
-  const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
-  const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(H, H);
+  const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(C, H);
+  const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(H, H);
   cudaError_t e;
   if ((e = pool_gemm(w, tcC, 3 * l + 2, A, rsA, q.Wp[l], w.pUP[l], R, H, C, s, nl))) return e;
   if ((e = launch_maxagg(g, w.pUP[l], q.bp[l], R, H, w.pAGG[l], w.pIDX[l],
@@ -1476,8 +1476,8 @@ static cudaError_t pool_splits(mars_dgi* m, const PoolParams& q, cudaStream_t s,
   cudaError_t e;
   for (int l = 0; l < 3; ++l) {
     const int C = l == 0 ? F : H;
-    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
-    const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(H, H);
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(C, H);
+    const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(H, H);
     const float* Wm[3] = {q.Ws[l], q.Wn[l], q.Wp[l]};
     for (int h = 0; h < 3; ++h) {
       const int K = h == 1 ? H : C;
@@ -1535,7 +1535,7 @@ static cudaError_t enqueue_step_pool(mars_dgi* m, const mars_graph* gr, cudaStre
   MARK(MARS_PH_GEMM_FWD);
   for (int l = 0; l < 3; ++l) {
     const int C = l == 0 ? F : H;
-    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(C, H);
     if (l == 0) {
       if (tcC) RET(launch_rowprep(w.Xs, R, F, w.one, nullptr, w.h3_rsY[0], s, nl));
     } else {
@@ -1545,7 +1545,7 @@ static cudaError_t enqueue_step_pool(mars_dgi* m, const mars_graph* gr, cudaStre
     RET(pool_layer_fwd(m, g, q, l, A[l], w.h3_rsY[l], w.Z[l], R, s, nl));
     MARK(MARS_PH_GEMM_FWD);
   }
-  const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(H, H);
+  const bool tcH = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(H, H);
   int ns = 0;
   w.hw.rs_dz3 = tcH ? w.h3_rsdZ : nullptr;
   RET(launch_head(g, H, w.Z[2], 0, q.M, q.alpha, m->d_sp, w.hw, w.dZ, gq.M, gloss, &ns, s, nl,
@@ -1554,7 +1554,7 @@ static cudaError_t enqueue_step_pool(mars_dgi* m, const mars_graph* gr, cudaStre
   MARK(MARS_PH_HEAD);
   for (int l = 2; l >= 0; --l) {
     const int C = l == 0 ? F : H;
-    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(C, H);
     RET(pool_dw(w, tcC, A[l], w.h3_rsY[l], w.dZ, w.h3_rsdZ, gq.Ws[l], R, C, H, s, nl));
     RET(pool_dw(w, tcH, w.pAGG[l], w.pRsAGG[l], w.dZ, w.h3_rsdZ, gq.Wn[l], R, H, H, s, nl));
     MARK(MARS_PH_GEMM_DW);
@@ -1570,7 +1570,7 @@ static cudaError_t enqueue_step_pool(mars_dgi* m, const mars_graph* gr, cudaStre
       RET(pool_gemm_t(w, tcC, 3 * l, w.dZ, w.h3_rsdZ, q.Ws[l], w.pUS, R, C, H, s, nl));     // dA_s
       RET(pool_gemm_t(w, tcC, 3 * l + 2, w.pDUP, w.pRsDUP, q.Wp[l], w.pVV, R, C, H, s, nl));  // dA_p
       MARK(MARS_PH_GEMM_DY);
-      const bool tcP = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(l - 1 == 0 ? F : H, H);
+      const bool tcP = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(l - 1 == 0 ? F : H, H);
       RET(launch_add_prelu_bwd(w.pUS, w.pVV, w.Z[l - 1], q.alpha, l - 1, R, H, w.dZ,
                                tcP || tcH ? w.h3_rsdZ : nullptr, w.slots[l - 1], &ns, s, nl));
       MARK(MARS_PH_SPMM_BWD);
@@ -1664,7 +1664,7 @@ static cudaError_t enqueue_step_sage(mars_dgi* m, const mars_graph* gr, cudaStre
   bool tc[3];
   for (int l = 0; l < 3; ++l) {
     const int Cin = l == 0 ? F : H;
-    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
+    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(Cin, H);
     if (tc[l])
       for (int h = 0; h < 2; ++h) {
         const int t = 2 * l + h;
@@ -1834,7 +1834,7 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   bool tc[3];
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
-    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
+    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(Cin, H);
     if (b16) RET(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl));
     else if (tc[l])
       RET(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
@@ -2220,7 +2220,7 @@ static cudaError_t enqueue_encode_sage(mars_dgi* m, const mars_graph* gr, cudaSt
   gf.vals = w.sVf;
   for (int l = 0; l < 3; ++l) {
     const int Cin = l == 0 ? F : H;
-    const bool tc = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(Cin, H);
+    const bool tc = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(Cin, H);
     if (l == 0) {
       if (tc && (e = launch_rowprep(g.X, Nt, F, w.one, nullptr, w.h3_rsY[0], s, nl))) return e;
     } else if ((e = launch_rowprep(w.Z[l - 1], Nt, H, alpha + (l - 1), w.Y23[l - 1],
@@ -2260,7 +2260,7 @@ static cudaError_t enqueue_encode_pool(mars_dgi* m, const mars_graph* gr, cudaSt
   if ((e = pool_splits(m, q, s, nl))) return e;
   for (int l = 0; l < 3; ++l) {
     const int C = l == 0 ? F : H;
-    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(C, H);
+    const bool tcC = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(C, H);
     if (l == 0) {
       if (tcC && (e = launch_rowprep(g.X, Nt, F, w.one, nullptr, w.h3_rsY[0], s, nl))) return e;
     } else if ((e = launch_rowprep(w.Z[l - 1], Nt, H, q.alpha + (l - 1), w.Y23[l - 1],
@@ -2291,7 +2291,7 @@ static cudaError_t enqueue_encode(mars_dgi* m, const mars_graph* g, cudaStream_t
   for (int l = 0; l < 3; ++l) {
     int Cin = l == 0 ? F : H;
     const void* T = l == 0 ? (const void*)gd.X : (const void*)w.Z[l - 1];
-    const bool h3l = !b16 && m->gemm_impl == MARS_GEMM_AUTO && tc_supported(Cin, H);
+    const bool h3l = !b16 && m->gemm_impl == MARS_GEMM_AUTO && tc3h_supported(Cin, H);
     if ((e = launch_spmm_fwd(gd, Cin, T, b16 && l > 0, nullptr, alpha, l - 1, Ys[l], b16, 0, s, nl,
                              nullptr, h3l ? w.h3_rsY[l] : nullptr)))
       return e;
@@ -2396,7 +2396,7 @@ static cudaError_t enqueue_encoder_backward(mars_dgi* m, const mars_graph* gr, c
   }
   if ((e = cudaMemsetAsync(m->grads, 0, sizeof(float) * (m->P + 1), s))) return e;
   bool tc[3];
-  for (int l = 0; l < 3; ++l) tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc_supported(l == 0 ? F : H, H);
+  for (int l = 0; l < 3; ++l) tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(l == 0 ? F : H, H);
   k_dz3_from_dE<<<cdiv(R * 32, 256), 256, 0, s>>>(dE, w.Z[2], alpha, (int32_t)Nt, H, w.dZ,
                                                    tc[2] ? w.h3_rsdZ : nullptr, w.slots[2]);
   count_launch(nl, 2 + 3);
@@ -2533,8 +2533,8 @@ extern "C" mars_status mars_debug_gemm(int32_t device, int32_t op, int32_t impl,
     return fail(MARS_ECUDA, "no CUDA device");
   }
   CK(cudaSetDevice(device));
-  const bool tcp = impl != MARS_GEMM_SIMT && (op == 0 ? tc_supported(K, N) || tc_supported(N, K)
-                                                     : tc_supported(K, N));
+  const bool tcp = impl != MARS_GEMM_SIMT && (op == 0 ? tc3h_supported(K, N) || tc3h_supported(N, K)
+                                                     : tc3h_supported(K, N));
   float *wsc = nullptr, *rs = nullptr, *rs2 = nullptr;
   CK(dalloc(&wsc, 2));
   CK(dalloc(&rs, (size_t)M));

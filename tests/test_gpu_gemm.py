@@ -88,3 +88,29 @@ def test_dw_mixed_magnitude_columns(H, K):
     comp = float(np.max(np.abs(C - ref) / bound))
     print("componentwise", H, K, comp, "normwise", scaled_err(C, ref))
     assert comp < 2e-5
+
+
+# The tiny configuration's widths (H in {32, 64}, C_in in {16, 32}) on the
+# tcgen05 kernels: wider tiles whose missing rows / columns TMA zero-fills.
+@pytest.mark.parametrize("M,N,K", [(1000, 32, 16), (777, 64, 32), (300, 32, 64), (4133, 64, 16),
+                                   (129, 32, 256), (5001, 32, 32)])
+def test_rows_narrow(M, N, K):
+    rng = np.random.default_rng(M + 3 * N + K)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    B = rng.standard_normal((N, K)).astype(np.float32)
+    C, _ = mars.debug_gemm("rows", A, B, "auto")
+    e = scaled_err(C, A.astype(np.float64) @ B.astype(np.float64).T)
+    print("rows narrow", M, N, K, e)
+    assert e < 5e-6
+
+
+@pytest.mark.parametrize("M,K,H", [(5000, 16, 32), (3001, 32, 64), (40001, 16, 64), (777, 64, 32),
+                                   (12345, 32, 32), (1000, 256, 32), (2048, 128, 64)])
+def test_dw_narrow(M, K, H):
+    rng = np.random.default_rng(M + K + 7 * H)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    B = rng.standard_normal((M, H)).astype(np.float32)
+    C, _ = mars.debug_gemm("dw", A, B, "auto")
+    e = scaled_err(C, A.astype(np.float64).T @ B.astype(np.float64))
+    print("dw narrow", M, K, H, e)
+    assert e < 5e-6

@@ -58,7 +58,50 @@ VARIANTS = [
 # dW1 / dW2 by ~1e-4 -- the default step behaves the same (its H = 256 gate is
 # stage-wise, tests/stagewise.py: every stage <= 1.4e-6 on these graphs) -- so
 # the H = 256 variant logic is checked end to end on the FFMA GEMMs.
-SIZES = [(16, 32, "auto"), (64, 128, "auto"), (64, 256, "simt")]
+SIZES = [(16, 32, "auto"), (16, 32, "simt"), (64, 128, "auto"), (64, 256, "simt")]
+
+
+def _noise_spread(gs, p0, F, H, seed, step, pb, variant, encoder="gcn", eps=1e-6, seeds=3):
+    """Conditioning probe for the tcgen05 (3xFP16) path: the largest change of
+    the fp64 oracle's gradient when every pre-activation Z of the encoder is
+    perturbed by relative noise eps (the 3xFP16 rounding scale), over a few
+    draws.  A PReLU kink within that noise of zero flips the branch."""
+    kw = dict(pair_base=pb, encoder=encoder, sparse=encoder != "sage_pool", **variant)
+    _, g0 = V.step_grads(gs, p0, F, H, seed, step, **kw)
+    worst = 0.0
+    for sd in range(seeds):
+        gen = torch.Generator().manual_seed(sd)
+        noise = lambda z: z * (1 + eps * torch.randn(z.shape, generator=gen, dtype=z.dtype))  # noqa
+
+        def gcn(An, X, W, alpha):
+            h = X
+            for l in range(3):
+                h = torch.nn.functional.prelu(noise(An @ (h @ W[l])), alpha[l:l + 1])
+            return h
+
+        def sage(AN, X, Wp, alpha):
+            h = X
+            for l in range(3):
+                Ws, Wn = Wp[l]
+                h = torch.nn.functional.prelu(noise(h @ Ws + AN @ (h @ Wn)), alpha[l:l + 1])
+            return h
+        saved = (V._encoder_gcn, V.encoder_sage)
+        V._encoder_gcn, V.encoder_sage = gcn, sage
+        try:
+            _, g1 = V.step_grads(gs, p0, F, H, seed, step, **kw)
+        finally:
+            V._encoder_gcn, V.encoder_sage = saved
+        worst = max(worst, scaled_err(g1, g0))
+    return worst
+
+
+def _grad_bar(impl, gs, p0, F, H, seed, step, pb, variant, encoder="gcn"):
+    """1e-5, or on the tcgen05 path 3 x the conditioning probe if larger (the
+    c33 rule): the FFMA GEMMs' ~1e-7 rounding flips no kink on
+    these graphs, 3xFP16's ~1e-6 can."""
+    if impl != "auto":
+        return TOL
+    return max(TOL, 3 * _noise_spread(gs, p0, F, H, seed, step, pb, variant, encoder))
 
 
 @pytest.mark.parametrize("F,H,impl", SIZES)
@@ -69,7 +112,11 @@ def test_variant_step_vs_oracle(variant, F, H, impl):
     p0, out = _run(gs, F, H, variant, seed, step, pb, impl=impl)
     loss, grads = V.step_grads(gs, p0, F, H, seed, step, pair_base=pb, sparse=True, **variant)
     assert abs(out["loss"] - loss) / abs(loss) <= TOL
-    assert scaled_err(out["grads"], grads) <= TOL, scaled_err(out["grads"], grads)
+    err = scaled_err(out["grads"], grads)
+    if err > TOL:                       # only then is the (slower) conditioning probe needed
+        bar = _grad_bar(impl, gs, p0, F, H, seed, step, pb, variant)
+        print(f"{variant} F={F} H={H} {impl}: grads err {err:.2e}, conditioning bar {bar:.2e}")
+        assert err <= bar, (err, bar)
     if "perms" in out:
         K = variant.get("num_neg", 1)
         Nt = sum(g.num_nodes for g in gs)
@@ -249,7 +296,10 @@ def test_sage_step_vs_oracle(variant, F, H, impl):
                                **variant)
     assert abs(out["loss"] - loss) / abs(loss) <= TOL
     err = scaled_err(out["grads"], grads)
-    assert err <= TOL, err
+    if err > TOL:
+        bar = _grad_bar(impl, gs, p0, F, H, 6, 2, 4, variant, encoder="sage")
+        print(f"sage {variant} F={F} H={H} {impl}: grads err {err:.2e}, conditioning bar {bar:.2e}")
+        assert err <= bar, (err, bar)
 
 
 def test_sage_encode_vs_oracle_and_hooks():
@@ -332,7 +382,11 @@ def test_variants_degenerate_graphs(encoder, variant):
     loss, grads = V.step_grads(gs, p0, 16, 32, 9, 1, pair_base=2, encoder=encoder, **variant)
     assert np.isfinite(out["loss"]) and np.all(np.isfinite(out["grads"]))
     assert abs(out["loss"] - loss) / abs(loss) <= TOL
-    assert scaled_err(out["grads"], grads) <= TOL
+    err = scaled_err(out["grads"], grads)
+    if err > TOL:
+        bar = _grad_bar("auto", gs, p0, 16, 32, 9, 1, 2, variant, encoder)
+        print(f"degenerate {encoder} {variant}: grads err {err:.2e}, conditioning bar {bar:.2e}")
+        assert err <= bar, (err, bar)
     assert scaled_err(emb, V.encode(gs, p1, 16, 32, aggregator=variant.get("aggregator", "gcn"),
                                     encoder_=encoder)) <= TOL
 
@@ -425,7 +479,7 @@ def test_sage_pool_step_vs_oracle(variant, F, H, impl):
     loss, grads = V.step_grads(gs, p0, F, H, 6, 2, **kw)
     _, g32 = V.step_grads(gs, p0, F, H, 6, 2, dtype=torch.float32, **kw)
     cond = scaled_err(g32, grads)
-    if impl == "auto" and H > 32:                       # tcgen05 3xFP16 GEMMs
+    if impl == "auto":                                  # tcgen05 3xFP16 GEMMs
         cond = max(cond, _pool_noise_spread(gs, p0, F, H, variant))
     err = scaled_err(out["grads"], grads)
     print(f"sage_pool {variant} F={F} H={H} {impl}: grads err {err:.2e}, conditioning {cond:.2e}")
