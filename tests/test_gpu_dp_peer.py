@@ -39,7 +39,7 @@ def _graphs():
     return [SG.cached("inception", i) for i in range(WORLD * PER)]
 
 
-def _worker(rank, port, q):
+def _worker(rank, port, q, variant=None):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank),
                       WORLD_SIZE=str(WORLD), LOCAL_RANK="0")
     import torch.distributed as dist
@@ -53,6 +53,8 @@ def _worker(rank, port, q):
         g.set_pair_offsets(mine)                   # global pair index = global graph index
         m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=SEED, device=0, world_size=WORLD,
                             rank=rank)
+        if variant:
+            m.set_contrastive(**variant)
         dp.connect_peers(m)
         dist.barrier()
         out = []
@@ -112,3 +114,41 @@ def test_two_process_peer_dp_matches_single_process():
             assert abs(loss_dp - loss_o) <= 1e-5 * abs(loss_o)
             assert scaled_err(grads_dp, grads_o) <= 1e-5
     assert scaled_err(res[0][2], m.get_state()[0]) <= 1e-5
+
+
+@pytest.mark.timeout(600)
+def test_two_process_peer_dp_contrastive_variant():
+    """NEXT-4 under the peer exchange: K = 3 corruption samples per graph
+    sharing the positive branch (sample k of graph g = pair g K + k with the
+    global g) and the InfoNCE loss; both ranks bitwise identical and equal to
+    the single-process step on all four graphs."""
+    variant = dict(num_neg=3, loss="infonce", corruption="mask", mask_rate=0.2)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, port, q, variant)) for r in range(WORLD)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(WORLD):
+        r, mine, out, params, err = q.get(timeout=500)
+        res[r] = (mine, out, params, err)
+    for p in procs:
+        p.join(timeout=60)
+    for r in range(WORLD):
+        assert res[r][3] is None, res[r][3]
+    for t in range(STEPS):
+        assert res[0][1][t][0] == res[1][1][t][0]
+        assert np.array_equal(res[0][1][t][1], res[1][1][t][1])
+    import paper_conf_icpp_lancl21_b200 as mars
+    g = mars.graph_load(_graphs())
+    m = mars.dgi_create(in_dim=F, hidden_dim=H, seed=SEED)
+    m.set_contrastive(**variant)
+    for t in range(STEPS):
+        o = m.step(g, t, 0, want_loss=True, want_grads=True)
+        loss_dp, grads_dp = res[0][1][t]
+        assert abs(loss_dp - o["loss"]) <= 1e-5 * abs(o["loss"]), t
+        e = scaled_err(grads_dp, o["grads"])
+        print("variant step", t, "dp vs single-process grads", e)
+        assert e <= 1e-5, t
+    m.free(); g.free()
