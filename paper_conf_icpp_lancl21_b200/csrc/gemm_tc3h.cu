@@ -290,6 +290,307 @@ k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUt
   }
 }
 
+// ---------------------------------------------------------------- k_tc3h_rows_pair
+// Z = A·Bᵀ for N = 256 on CTA pairs (cta_group::2): each CTA of a pair owns
+// one 128-row tile of A and HALF of the weight operand (N rows 128r ..
+// 128r + 127), so per K-block a CTA loads 16 KB of A and 16 KB of B hi / lo
+// instead of 16 + 32 KB, and every pair MMA (M = 256: both CTAs' A tiles;
+// N = 256: both CTAs' B halves) reads each B half from the CTA that holds it
+// -- a third less shared-memory traffic per row tile than k_tc3h_rows.
+// Roles as in k_tc3h_rows (warp 0 TMA, warp 1 MMA -- the even CTA issues --
+// warps 2-5 convert their own A rows in place, warps 6-9 drain their own
+// TMEM rows); the odd CTA's converters and epilogue warps meet at a named
+// barrier and one thread arrives on the even CTA's conv / tempty barrier.
+#ifndef MARS_ROWS_PAIR
+#define MARS_ROWS_PAIR 1
+#endif
+constexpr int kRpStages = 6;
+struct H3RowsPairCfg {
+  static constexpr int N = 256, NHALF = 128;
+  static constexpr int A_BYTES = kBM * kBK * 4;       // fp32 staging, later hi | lo (8 KB each)
+  static constexpr int B_BYTES = NHALF * kBK * 2;     // one fp16 half tile (8 KB)
+  static constexpr int STAGE = A_BYTES + 2 * B_BYTES; // 32 KB
+  static constexpr int SLAB = 32 * 32 * 4;
+  static constexpr int STAGING = 4 * SLAB;            // one slab per epilogue warp
+  static constexpr int SCALES = kScaleSlots * kBM * 4;
+  static constexpr int SMEM = kRpStages * STAGE + STAGING + SCALES + 1024 + 512;
+  static constexpr uint32_t TMEM_COLS = 512;
+};
+
+__device__ __forceinline__ void rp_epi_bar() {     // the 4 epilogue warps
+  asm volatile("bar.sync 2, 128;" ::: "memory");
+}
+
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+k_tc3h_rows_pair(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBhi,
+                 const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmC,
+                 const float* __restrict__ rs, const float* __restrict__ inv_tb, int32_t M,
+                 int32_t K) {
+  using Cfg = H3RowsPairCfg;
+  constexpr int S = kRpStages, N = Cfg::N;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
+  uint8_t* staging = smem + S * Cfg::STAGE;
+  float* rscale = reinterpret_cast<float*>(staging + Cfg::STAGING);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(staging + Cfg::STAGING + Cfg::SCALES);
+  uint64_t* full = bars;                 // TMA landed (this CTA)
+  uint64_t* conv = bars + S;             // even CTA: both CTAs' converters (4 + 1)
+  uint64_t* empty = bars + 2 * S;        // pair MMAs done with the stage (multicast commit)
+  uint64_t* tfull = bars + 3 * S;        // [2] accumulator ready (multicast commit)
+  uint64_t* tempty = bars + 3 * S + 2;   // [2] even CTA: both CTAs' epilogues (4 + 1)
+  uint64_t* sready = bars + 3 * S + 4;   // [slots] local
+  uint64_t* sfree = sready + kScaleSlots;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(sfree + kScaleSlots);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_rank();
+  const int ntiles = (M + kBM - 1) / kBM;
+  const int npair = (ntiles + 1) / 2;
+  const int nclu = gridDim.x / 2, clu = blockIdx.x / 2;
+  const int nk = (K + kBK - 1) / kBK;
+  auto stA = [&](int s) { return smem + s * Cfg::STAGE; };
+  auto stB = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES; };
+  auto stBlo = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A_BYTES + Cfg::B_BYTES; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 5);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 5);
+    }
+    for (int b = 0; b < kScaleSlots; ++b) {
+      mbar_init(&sready[b], 4);
+      mbar_init(&sfree[b], 4);
+    }
+    fence_mbar_init();
+    tma_prefetch(&tmA);
+    tma_prefetch(&tmBhi);
+    tma_prefetch(&tmBlo);
+    tma_prefetch(&tmC);
+  }
+  if (warp == 1) tmem_alloc_pair(tslot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tbase = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {                                         // ---- TMA producer (both CTAs)
+      int s = 0;
+      uint32_t ph = 0;
+      for (int pt = clu; pt < npair; pt += nclu) {
+        const int t = 2 * pt + (int)rank;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&empty[s], ph ^ 1);
+          mbar_expect_tx(&full[s], Cfg::A_BYTES + 2 * Cfg::B_BYTES);
+          tma_load_2d(stA(s), &tmA, kb * kBK, t * kBM, &full[s]);
+          tma_load_2d(stB(s), &tmBhi, kb * kBK, (int)rank * Cfg::NHALF, &full[s]);
+          tma_load_2d(stBlo(s), &tmBlo, kb * kBK, (int)rank * Cfg::NHALF, &full[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {                            // ---- pair MMA issuer
+      constexpr uint32_t idesc = idesc_f16(2 * kBM, N);
+      int s = 0;
+      uint32_t ph = 0;
+      int acc = 0;
+      uint32_t aph = 0;
+      for (int pt = clu; pt < npair; pt += nclu) {
+        mbar_wait_cluster(&tempty[acc], aph ^ 1);
+        tc_fence_after();
+        const uint32_t d = tbase + acc * N;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait_cluster(&conv[s], ph);
+          tc_fence_after();
+          const uint32_t a = smem_u32(stA(s)), al = a + kBM * kBK * 2;
+          const uint32_t b = smem_u32(stB(s)), bl = smem_u32(stBlo(s));
+#pragma unroll
+          for (int k = 0; k < kBK / 16; ++k) {
+            const uint64_t ah = sdesc_sw64(a + 32 * k, 16, 512);
+            const uint64_t alo = sdesc_sw64(al + 32 * k, 16, 512);
+            const uint64_t bh = sdesc_sw64(b + 32 * k, 16, 512);
+            const uint64_t blo = sdesc_sw64(bl + 32 * k, 16, 512);
+            mma_f16_pair(d, ah, bh, idesc, (kb | k) != 0);
+            mma_f16_pair(d, ah, blo, idesc, 1);
+            mma_f16_pair(d, alo, bh, idesc, 1);
+          }
+          mma_commit_pair(&empty[s], 0x3);
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+        mma_commit_pair(&tfull[acc], 0x3);
+        acc ^= 1;
+        if (acc == 0) aph ^= 1;
+      }
+    }
+  } else if (warp < 6) {                                     // ---- convert own A rows
+    const int ct = threadIdx.x - 64;
+    const uint32_t conv0 = mapa_u32(conv, 0);
+    int s = 0;
+    uint32_t ph = 0;
+    int it = 0;
+    for (int pt = clu; pt < npair; pt += nclu, ++it) {
+      const int t = 2 * pt + (int)rank;
+      const int slot = it % kScaleSlots;
+      const int64_t row = (int64_t)t * kBM + ct;
+      const float scale = row < M ? __ldg(rs + row) : 1.f;
+      if (it >= kScaleSlots) mbar_wait(&sfree[slot], ((it / kScaleSlots) - 1) & 1);
+      rscale[slot * kBM + ct] = 1.f / scale;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sready[slot]);
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&full[s], ph);
+        uint8_t* base = stA(s);
+        uint4 hi[kBK / 8], lo[kBK / 8];
+#pragma unroll
+        for (int c = 0; c < kBK / 8; ++c) {
+          float x[8];
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int j = 2 * c + h;
+            const float4 v =
+                *reinterpret_cast<const float4*>(base + ct * 128 + ((j ^ (ct & 7)) << 4));
+            x[4 * h] = v.x * scale;
+            x[4 * h + 1] = v.y * scale;
+            x[4 * h + 2] = v.z * scale;
+            x[4 * h + 3] = v.w * scale;
+          }
+          split_h8(x, hi[c], lo[c]);
+        }
+        conv_bar();                  // every converter has read its row before any write
+#pragma unroll
+        for (int c = 0; c < kBK / 8; ++c) {
+          const int off = ct * 64 + ((c ^ ((ct >> 1) & 3)) << 4);
+          *reinterpret_cast<uint4*>(base + off) = hi[c];
+          *reinterpret_cast<uint4*>(base + kBM * kBK * 2 + off) = lo[c];
+        }
+        fence_proxy_async_smem();
+        if (rank == 0) {
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&conv[s]);
+        } else {
+          conv_bar();                                        // the 4 converter warps
+          if (threadIdx.x == 64) mbar_arrive_cluster(conv0 + s * 8);
+        }
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp < 10) {                                    // ---- epilogue (own rows)
+    const int q = warp & 3;
+    const uint32_t tempty0 = mapa_u32(tempty, 0);
+    int acc = 0;
+    uint32_t aph = 0;
+    const float itb = *inv_tb;
+    uint8_t* slab = staging + q * Cfg::SLAB;
+    int it = 0;
+    for (int pt = clu; pt < npair; pt += nclu, ++it) {
+      const int t = 2 * pt + (int)rank;
+      const int slot = it % kScaleSlots;
+      mbar_wait(&sready[slot], (it / kScaleSlots) & 1);
+      const float f = rscale[slot * kBM + q * 32 + lane] * itb;
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&sfree[slot]);
+      mbar_wait(&tfull[acc], aph);
+      tc_fence_after();
+#pragma unroll 1
+      for (int c0 = 0; c0 < N; c0 += 32) {
+        uint32_t r[32];
+        tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
+        if (lane == 0) bulk_wait_read<0>();   // the store that last read this slab is done
+        __syncwarp();
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          float4* dst = reinterpret_cast<float4*>(slab + lane * 128 + ((j ^ (lane & 7)) << 4));
+          *dst = make_float4(__uint_as_float(r[4 * j]) * f, __uint_as_float(r[4 * j + 1]) * f,
+                             __uint_as_float(r[4 * j + 2]) * f, __uint_as_float(r[4 * j + 3]) * f);
+        }
+        fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_2d(&tmC, slab, c0, t * kBM + q * 32);
+          bulk_commit();
+        }
+      }
+      tc_fence_before();
+      if (rank == 0) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&tempty[acc]);
+      } else {
+        rp_epi_bar();
+        if (threadIdx.x == 6 * 32) mbar_arrive_cluster(tempty0 + acc * 8);
+      }
+      acc ^= 1;
+      if (acc == 0) aph ^= 1;
+    }
+    if (lane == 0) bulk_wait<0>();
+  }
+  tc_fence_before();
+  cluster_sync();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc_pair(tbase, Cfg::TMEM_COLS);
+  }
+}
+
+int rows_pair_clusters() {
+  static int n = 0;
+  if (!n) {
+    cudaFuncSetAttribute(k_tc3h_rows_pair, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         H3RowsPairCfg::SMEM);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * 74, 1, 1);
+    cfg.blockDim = dim3(kThreads, 1, 1);
+    cfg.dynamicSmemBytes = H3RowsPairCfg::SMEM;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    int c = 0;
+    if (cudaOccupancyMaxActiveClusters(&c, k_tc3h_rows_pair, &cfg) != cudaSuccess || c < 1) {
+      cudaGetLastError();
+      c = tc_num_sms() / 2;
+    }
+    n = c;
+  }
+  return n;
+}
+
+cudaError_t rows3h_pair(const float* A, const float* rs, const __half* Bhi, const __half* Blo,
+                        const float* inv_tb, float* C, int64_t M, int K, cudaStream_t s) {
+  using Cfg = H3RowsPairCfg;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k_tc3h_rows_pair,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap ta, tbh, tbl, tc;
+  if (!tc_tmap(&ta, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, A, M, K, kBK, kBM,
+               CU_TENSOR_MAP_SWIZZLE_128B) ||
+      !tc_tmap(&tbh, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Bhi, Cfg::N, K, kBK, Cfg::NHALF,
+               CU_TENSOR_MAP_SWIZZLE_64B) ||
+      !tc_tmap(&tbl, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, Blo, Cfg::N, K, kBK, Cfg::NHALF,
+               CU_TENSOR_MAP_SWIZZLE_64B) ||
+      !tc_tmap(&tc, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, C, M, Cfg::N, 32, 32,
+               CU_TENSOR_MAP_SWIZZLE_128B))
+    return cudaErrorInvalidValue;
+  const int ntiles = (int)((M + kBM - 1) / kBM);
+  const int npair = (ntiles + 1) / 2;
+  const int nclu = std::min(npair, rows_pair_clusters());
+  k_tc3h_rows_pair<<<2 * nclu, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, tc, rs, inv_tb, (int32_t)M, K);
+  return cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- row scales
 // rs[r] = 2^(14 - e_r) of max_k |A[r][k]| (warp per row), for A not produced by
 // a kernel that writes its own row scales.
@@ -1012,7 +1313,10 @@ cudaError_t tc3h_gemm_rows(const float* A, const float* rs, const void* B_hi, co
     case 32:
     case 64: return rows3h_n<64>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
     case 128: return rows3h_n<128>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
-    case 256: return rows3h_n<256>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
+    case 256:
+      if (MARS_ROWS_PAIR && M >= 2 * kBM * tc_num_sms())   // CTA pairs for the large launches
+        return rows3h_pair(A, rs, bh, bl, inv_tb, C, M, K, s);
+      return rows3h_n<256>(A, rs, bh, bl, inv_tb, C, M, K, N, s);
     default: return cudaErrorInvalidValue;
   }
 }

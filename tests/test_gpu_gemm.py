@@ -114,3 +114,19 @@ def test_dw_narrow(M, K, H):
     e = scaled_err(C, A.astype(np.float64).T @ B.astype(np.float64))
     print("dw narrow", M, K, H, e)
     assert e < 5e-6
+
+
+# Large launches (M >= 2 x 128 x SMs) run the CTA-pair row kernel
+# (k_tc3h_rows_pair: half the weight operand per CTA, cta_group::2 MMAs),
+# including an odd tile count (the odd CTA's last tile is empty).
+@pytest.mark.parametrize("M,K", [(100003, 256), (419232, 256), (77777, 64), (38144, 128)])
+def test_rows_pair(M, K):
+    rng = np.random.default_rng(M + K)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    A[::7] *= 1e-20                                  # rows of very different magnitude
+    B = rng.standard_normal((256, K)).astype(np.float32)
+    C, _ = mars.debug_gemm("rows", A, B, "auto")
+    ref = A.astype(np.float64) @ B.astype(np.float64).T
+    e = _row_err(C, ref)
+    print("rows pair", M, K, e)
+    assert e < 5e-6
