@@ -304,14 +304,21 @@ k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUt
 #ifndef MARS_ROWS_PAIR
 #define MARS_ROWS_PAIR 1
 #endif
-constexpr int kRpStages = 6;
+#ifndef MARS_RP_STAGES
+#define MARS_RP_STAGES 6
+#endif
+#ifndef MARS_RP_SLABS
+#define MARS_RP_SLABS 1
+#endif
+constexpr int kRpStages = MARS_RP_STAGES;
 struct H3RowsPairCfg {
   static constexpr int N = 256, NHALF = 128;
   static constexpr int A_BYTES = kBM * kBK * 4;       // fp32 staging, later hi | lo (8 KB each)
   static constexpr int B_BYTES = NHALF * kBK * 2;     // one fp16 half tile (8 KB)
   static constexpr int STAGE = A_BYTES + 2 * B_BYTES; // 32 KB
   static constexpr int SLAB = 32 * 32 * 4;
-  static constexpr int STAGING = 4 * SLAB;            // one slab per epilogue warp
+  static constexpr int NSLAB = MARS_RP_SLABS;
+  static constexpr int STAGING = 4 * NSLAB * SLAB;    // slabs per epilogue warp
   static constexpr int SCALES = kScaleSlots * kBM * 4;
   static constexpr int SMEM = kRpStages * STAGE + STAGING + SCALES + 1024 + 512;
   static constexpr uint32_t TMEM_COLS = 512;
@@ -486,7 +493,8 @@ k_tc3h_rows_pair(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
     int acc = 0;
     uint32_t aph = 0;
     const float itb = *inv_tb;
-    uint8_t* slab = staging + q * Cfg::SLAB;
+    uint8_t* slab0 = staging + q * Cfg::NSLAB * Cfg::SLAB;
+    int nslab = 0;
     int it = 0;
     for (int pt = clu; pt < npair; pt += nclu, ++it) {
       const int t = 2 * pt + (int)rank;
@@ -498,10 +506,14 @@ k_tc3h_rows_pair(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       mbar_wait(&tfull[acc], aph);
       tc_fence_after();
 #pragma unroll 1
-      for (int c0 = 0; c0 < N; c0 += 32) {
+      for (int c0 = 0; c0 < N; c0 += 32, ++nslab) {
         uint32_t r[32];
         tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
-        if (lane == 0) bulk_wait_read<0>();   // the store that last read this slab is done
+        uint8_t* slab = slab0 + (Cfg::NSLAB == 2 ? (nslab & 1) * Cfg::SLAB : 0);
+        if (lane == 0) {                      // the store that last read this slab is done
+          if (Cfg::NSLAB == 2) bulk_wait_read<1>();
+          else bulk_wait_read<0>();
+        }
         __syncwarp();
         tmem_wait_ld();
 #pragma unroll
