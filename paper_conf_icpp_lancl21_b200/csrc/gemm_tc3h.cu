@@ -704,7 +704,10 @@ constexpr int kDwSub = 8;        // stages per TMEM work run (128 rows)
 #ifndef MARS_DW_PAIR
 #define MARS_DW_PAIR 1
 #endif
-constexpr bool kDwPair = MARS_DW_PAIR != 0;   // C_in = H = 256 on a CTA pair (k_tc3h_dw_pair)
+constexpr bool kDwPair = MARS_DW_PAIR != 0;
+#ifndef MARS_DW_NG
+#define MARS_DW_NG 1          // converter groups of k_tc3h_dw working on alternate stages
+#endif   // C_in = H = 256 on a CTA pair (k_tc3h_dw_pair)
 
 template <int CINT, int HH>
 struct H3DwCfg {
@@ -762,7 +765,7 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&conv[s], 10);
+      mbar_init(&conv[s], 10 / MARS_DW_NG);   // the converter warps of the stage's group
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -886,54 +889,61 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[buf]);
     };
+    // converter group: warps 2 + GW g .. 2 + GW g + GW - 1 convert stages kb = g (mod NG)
+    constexpr int NG = MARS_DW_NG, GW = 10 / NG, GT = GW * 32;
+    static_assert(10 % NG == 0 && NG <= kDwStages && NG <= kDwSub, "converter groups");
+    const int grp = (warp - 2) / GW;
+    const int gt = ct - grp * GT;                        // thread index within the group
     constexpr int NTA = kDwBK * HH / 8;                 // 8-column tasks of dZ per stage
     constexpr int NTT = NTA + kDwBK * CINT / 8;
-    constexpr int MAXT = (NTT + NT - 1) / NT;             // tasks per thread (2 or 3)
+    constexpr int MAXT = (NTT + GT - 1) / GT;             // tasks per thread
     // a thread's tasks are the same in every stage: their offsets from the
     // stage base are computed once (the second 16-byte source chunk is the
     // first's chunk index ^ 1: w0 is even)
     uint32_t so0[MAXT], dof[MAXT];
     int ntask = 0;
 #pragma unroll
-    for (int q = 0; q < MAXT; ++q) {
-      const int i = ct + q * NT;
-      so0[q] = dof[q] = 0;
+    for (int t = 0; t < MAXT; ++t) {
+      const int i = gt + t * GT;
+      so0[t] = dof[t] = 0;
       if (i < NTT) {
         const bool isA = i < NTA;
         const int ii = isA ? i : i - NTA;
         const int r = ii % kDwBK, c0 = (ii / kDwBK) * 8;
         const uint32_t sb = (isA ? 0u : (uint32_t)Cfg::A32) + (c0 / 32) * Cfg::BOX32 + r * 128;
         const int w0 = (c0 % 32) / 4;
-        so0[q] = sb + ((w0 ^ (r & 7)) << 4);
-        dof[q] = Cfg::A32 + Cfg::B32 + (isA ? 0u : 2u * Cfg::A16) + (c0 / 64) * Cfg::ATOM +
+        so0[t] = sb + ((w0 ^ (r & 7)) << 4);
+        dof[t] = Cfg::A32 + Cfg::B32 + (isA ? 0u : 2u * Cfg::A16) + (c0 / 64) * Cfg::ATOM +
                  r * 128 + ((((c0 % 64) / 8) ^ (r & 7)) << 4);
-        ntask = q + 1;
+        ntask = t + 1;
       }
     }
-    int s = 0;
+    int s = grp;
     uint32_t ph = 0;
-    for (int kb = 0; kb < nk; ++kb) {
+    for (int kb = grp; kb < nk; kb += NG) {
       mbar_wait(&full[s], ph);
       uint8_t* stage = smem + s * Cfg::STAGE;
 #pragma unroll
-      for (int q = 0; q < MAXT; ++q) {
-        if (q >= ntask) break;
-        const bool isA = so0[q] < (uint32_t)Cfg::A32;
-        const float4 v0 = *reinterpret_cast<const float4*>(stage + so0[q]);
-        const float4 v1 = *reinterpret_cast<const float4*>(stage + (so0[q] ^ 16u));
+      for (int t = 0; t < MAXT; ++t) {
+        if (t >= ntask) break;
+        const bool isA = so0[t] < (uint32_t)Cfg::A32;
+        const float4 v0 = *reinterpret_cast<const float4*>(stage + so0[t]);
+        const float4 v1 = *reinterpret_cast<const float4*>(stage + (so0[t] ^ 16u));
         const float sc = isA ? sz : sy;
         const float x[8] = {v0.x * sc, v0.y * sc, v0.z * sc, v0.w * sc,
                             v1.x * sc, v1.y * sc, v1.z * sc, v1.w * sc};
         uint4 hv, lv;
         split_h8(x, hv, lv);
-        *reinterpret_cast<uint4*>(stage + dof[q]) = hv;
-        *reinterpret_cast<uint4*>(stage + dof[q] + (isA ? Cfg::A16 : Cfg::B16)) = lv;
+        *reinterpret_cast<uint4*>(stage + dof[t]) = hv;
+        *reinterpret_cast<uint4*>(stage + dof[t] + (isA ? Cfg::A16 : Cfg::B16)) = lv;
       }
       fence_proxy_async_smem();
       __syncwarp();
       if (lane == 0) mbar_arrive(&conv[s]);
-      if (++s == S) { s = 0; ph ^= 1; }
-      if (folder && (kb % kDwSub) == kDwSub / 2 && kb / kDwSub >= 1) fold(folded++);
+      s += NG;
+      if (s >= S) { s -= S; ph ^= 1; }
+      // fold run j once the conversion has passed the middle of run j + 1
+      while (folder && folded < nsub && kb >= (folded + 1) * kDwSub + kDwSub / 2) fold(folded++);
     }
     if (folder) {
       while (folded < nsub) fold(folded++);
@@ -968,8 +978,10 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 // conversion work the GEMM needs, and the fp32 -> fp16 hi / lo conversion is
 // what bounds this kernel.  Here the pair splits both operands instead: CTA r
 // converts dZ columns (h) [128r, 128r + 128) and Y columns (c) [128r, 128r +
-// 128) of every 16-row stage; the even CTA issues one M = 256 (h), N = 256 (c)
-// pair MMA per product that reads the A half and the B half of each CTA from
+// 128) of every BK-row stage (32 by default: a stage is one synchronisation
+// chain of the converters, and the chain, not the bandwidth, set the 16-row
+// kernel's pace); the even CTA issues BK / 16 M = 256 (h), N = 256 (c) K = 16
+// pair MMAs per product that read the A half and the B half of each CTA from
 // the same shared-memory offsets; CTA r's TMEM accumulates D[h][c] for its 128
 // h rows and all 256 c columns (256 fp32 columns, double-buffered).
 // Synchronisation: the MMA commits multicast to both CTAs' empty / tfull
@@ -980,30 +992,42 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 #ifndef MARS_PAIR_STAGES
 #define MARS_PAIR_STAGES 6
 #endif
-constexpr int kPairStages = MARS_PAIR_STAGES;
+#ifndef MARS_DWP_BK
+#define MARS_DWP_BK 32        // rows per pair stage (BK / 16 MMA K-steps per stage)
+#endif
+#ifndef MARS_DWP_NG
+#define MARS_DWP_NG 1         // converter groups working on alternate stages
+#endif
 
+template <int BK>
 struct H3PairCfg {
-  static constexpr int ATOM = 64 * kDwBK * 2;          // fp16 MN atom column: 64 cols x 16 rows
-  static constexpr int BOX32 = 32 * kDwBK * 4;         // one 32-column fp32 block: 16 rows x 128 B
+  static constexpr int ATOM = 64 * BK * 2;             // fp16 MN atom column: 64 cols x BK rows
+  static constexpr int BOX32 = 32 * BK * 4;            // one 32-column fp32 block: BK rows x 128 B
   static constexpr int HALF = 128;                     // columns of each operand per CTA
-  static constexpr int A32 = (HALF / 32) * BOX32;      // 8 KB
+  static constexpr int A32 = (HALF / 32) * BOX32;
   static constexpr int B32 = (HALF / 32) * BOX32;
-  static constexpr int A16 = (HALF / 64) * ATOM;       // 4 KB (hi; lo follows)
+  static constexpr int A16 = (HALF / 64) * ATOM;       // hi; lo follows
   static constexpr int B16 = (HALF / 64) * ATOM;
-  static constexpr int STAGE = A32 + B32 + 2 * A16 + 2 * B16;   // 32 KB
-  static constexpr int SMEM = kPairStages * STAGE + 1024 + 512;
+  static constexpr int STAGE = A32 + B32 + 2 * A16 + 2 * B16;   // 2 KB per row
+  static constexpr int S = BK == 16 ? MARS_PAIR_STAGES : (200 * 1024) / STAGE;
+  static constexpr int SMEM = S * STAGE + 1024 + 512;
+  static constexpr int SUB = 128 / BK;                 // stages per 128-row TMEM work run
   static constexpr uint32_t TMEM_COLS = 512;           // 2 buffers x 256 fp32 columns
   static constexpr int MC = 128;                       // columns per folding thread
 };
 
+template <int BK, int NG>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1)
 k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
                const float* __restrict__ rs_dz, const float* __restrict__ rs_y,
                float* __restrict__ part, int32_t R, int32_t rows_per_chunk) {
-  using Cfg = H3PairCfg;
-  constexpr int S = kPairStages;
+  using Cfg = H3PairCfg<BK>;
+  constexpr int S = Cfg::S;
+  constexpr int SUB = Cfg::SUB;
   constexpr int MC = Cfg::MC;
   constexpr int CIN = 256, HH = 256;
+  constexpr int GW = 10 / NG;                            // converter warps per group
+  static_assert(10 % NG == 0 && SUB >= NG, "converter groups");
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
@@ -1020,8 +1044,8 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
   const int chunk = blockIdx.x >> 1;
   const int32_t r0 = chunk * rows_per_chunk;
   const int32_t r1 = min(R, r0 + rows_per_chunk);
-  const int nk = r1 > r0 ? (r1 - r0 + kDwBK - 1) / kDwBK : 0;
-  const int nsub = (nk + kDwSub - 1) / kDwSub;
+  const int nk = r1 > r0 ? (r1 - r0 + BK - 1) / BK : 0;
+  const int nsub = (nk + SUB - 1) / SUB;
   auto stA32 = [&](int s) { return smem + s * Cfg::STAGE; };
   auto stB32 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32; };
   auto stA16 = [&](int s) { return smem + s * Cfg::STAGE + Cfg::A32 + Cfg::B32; };  // hi, lo
@@ -1030,7 +1054,7 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&conv[s], 11);         // 10 local converter warps + 1 from the odd CTA
+      mbar_init(&conv[s], GW + 1);     // the group's local converter warps + 1 from the odd CTA
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -1054,7 +1078,7 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
       for (int kb = 0; kb < nk; ++kb) {
         mbar_wait(&empty[s], ph ^ 1);
         mbar_expect_tx(&full[s], Cfg::A32 + Cfg::B32);
-        const int32_t row = r0 + kb * kDwBK;
+        const int32_t row = r0 + kb * BK;
         tma_load_3d(stA32(s), &tmDZ, 0, row, (int)rank * (Cfg::HALF / 32), &full[s]);
         tma_load_3d(stB32(s), &tmY, 0, row, (int)rank * (Cfg::HALF / 32), &full[s]);
         if (++s == S) { s = 0; ph ^= 1; }
@@ -1070,20 +1094,23 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
         mbar_wait_cluster(&tempty[buf], ((sub >> 1) & 1) ^ 1);
         tc_fence_after();
         const uint32_t twork = tbase + buf * CIN;
-        const int kb1 = min(nk, (sub + 1) * kDwSub);
-        for (int kb = sub * kDwSub; kb < kb1; ++kb) {
+        const int kb1 = min(nk, (sub + 1) * SUB);
+        for (int kb = sub * SUB; kb < kb1; ++kb) {
           mbar_wait_cluster(&conv[s], ph);
           tc_fence_after();
-          const uint32_t a = smem_u32(stA16(s)), al = a + Cfg::A16;
-          const uint32_t b = smem_u32(stB16(s)), bl = b + Cfg::B16;
-          const uint64_t ah = sdesc_sw128(a, Cfg::ATOM, 1024);
-          const uint64_t alo = sdesc_sw128(al, Cfg::ATOM, 1024);
-          const uint64_t bh = sdesc_sw128(b, Cfg::ATOM, 1024);
-          const uint64_t blo = sdesc_sw128(bl, Cfg::ATOM, 1024);
-          const uint32_t first = kb == sub * kDwSub ? 0u : 1u;
-          mma_f16_pair(twork, ah, bh, idesc, first);
-          mma_f16_pair(twork, ah, blo, idesc, 1);
-          mma_f16_pair(twork, alo, bh, idesc, 1);
+#pragma unroll
+          for (int j = 0; j < BK / 16; ++j) {                // K = 16 steps: 16 rows = 2 KB of an atom column
+            const uint32_t a = smem_u32(stA16(s)) + j * 2048, al = a + Cfg::A16;
+            const uint32_t b = smem_u32(stB16(s)) + j * 2048, bl = b + Cfg::B16;
+            const uint64_t ah = sdesc_sw128(a, Cfg::ATOM, 1024);
+            const uint64_t alo = sdesc_sw128(al, Cfg::ATOM, 1024);
+            const uint64_t bh = sdesc_sw128(b, Cfg::ATOM, 1024);
+            const uint64_t blo = sdesc_sw128(bl, Cfg::ATOM, 1024);
+            const uint32_t first = (kb == sub * SUB && j == 0) ? 0u : 1u;
+            mma_f16_pair(twork, ah, bh, idesc, first);
+            mma_f16_pair(twork, ah, blo, idesc, 1);
+            mma_f16_pair(twork, alo, bh, idesc, 1);
+          }
           mma_commit_pair(&empty[s], 0x3);
           if (++s == S) { s = 0; ph ^= 1; }
         }
@@ -1147,58 +1174,68 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
         if (threadIdx.x == 4 * 32) mbar_arrive_cluster(tempty0 + buf * 8);
       }
     };
-    constexpr int NTA = kDwBK * Cfg::HALF / 8;          // 8-column tasks of dZ per stage
+    // converter group: warps 2 + GW g .. 2 + GW g + GW - 1 convert stages kb = g (mod NG)
+    const int grp = (warp - 2) / GW;
+    const int gt = ct - grp * GW * 32;                   // thread index within the group
+    constexpr int GT = GW * 32;
+    constexpr int NTA = BK * Cfg::HALF / 8;              // 8-column tasks of dZ per stage
     constexpr int NTT = 2 * NTA;
-    constexpr int MAXT = (NTT + NT - 1) / NT;             // tasks per thread (2)
+    constexpr int MAXT = (NTT + GT - 1) / GT;            // tasks per thread
     // a thread's tasks are the same in every stage: their offsets from the
     // stage base (swizzled source chunks, destination chunk) are computed once
     // (the second 16-byte chunk of a task is the first's chunk index ^ 1: w0 is even)
     uint32_t so0[MAXT], dof[MAXT];
     int ntask = 0;
 #pragma unroll
-    for (int q = 0; q < MAXT; ++q) {
-      const int i = ct + q * NT;
-      so0[q] = dof[q] = 0;
+    for (int t = 0; t < MAXT; ++t) {
+      const int i = gt + t * GT;
+      so0[t] = dof[t] = 0;
       if (i < NTT) {
         const bool isA = i < NTA;
         const int ii = isA ? i : i - NTA;
-        const int r = ii % kDwBK, c0 = (ii / kDwBK) * 8;
+        const int r = ii % BK, c0 = (ii / BK) * 8;
         const uint32_t sb = (isA ? 0u : (uint32_t)Cfg::A32) + (c0 / 32) * Cfg::BOX32 + r * 128;
         const int w0 = (c0 % 32) / 4;
-        so0[q] = sb + ((w0 ^ (r & 7)) << 4);
-        dof[q] = Cfg::A32 + Cfg::B32 + (isA ? 0u : 2u * Cfg::A16) + (c0 / 64) * Cfg::ATOM +
+        so0[t] = sb + ((w0 ^ (r & 7)) << 4);
+        dof[t] = Cfg::A32 + Cfg::B32 + (isA ? 0u : 2u * Cfg::A16) + (c0 / 64) * Cfg::ATOM +
                  r * 128 + ((((c0 % 64) / 8) ^ (r & 7)) << 4);
-        ntask = q + 1;
+        ntask = t + 1;
       }
     }
-    int s = 0;
+    int s = grp;
     uint32_t ph = 0;
-    for (int kb = 0; kb < nk; ++kb) {
+    for (int kb = grp; kb < nk; kb += NG) {
       mbar_wait(&full[s], ph);
       uint8_t* stage = smem + s * Cfg::STAGE;
 #pragma unroll
-      for (int q = 0; q < MAXT; ++q) {
-        if (q >= ntask) break;
-        const float4 v0 = *reinterpret_cast<const float4*>(stage + so0[q]);
-        const float4 v1 = *reinterpret_cast<const float4*>(stage + (so0[q] ^ 16u));
-        const float sc = so0[q] < (uint32_t)Cfg::A32 ? sz : sy;
+      for (int t = 0; t < MAXT; ++t) {
+        if (t >= ntask) break;
+        const float4 v0 = *reinterpret_cast<const float4*>(stage + so0[t]);
+        const float4 v1 = *reinterpret_cast<const float4*>(stage + (so0[t] ^ 16u));
+        const float sc = so0[t] < (uint32_t)Cfg::A32 ? sz : sy;
         const float x[8] = {v0.x * sc, v0.y * sc, v0.z * sc, v0.w * sc,
                             v1.x * sc, v1.y * sc, v1.z * sc, v1.w * sc};
         uint4 hv, lv;
         split_h8(x, hv, lv);
-        *reinterpret_cast<uint4*>(stage + dof[q]) = hv;
-        *reinterpret_cast<uint4*>(stage + dof[q] + Cfg::A16) = lv;      // A16 == B16
+        *reinterpret_cast<uint4*>(stage + dof[t]) = hv;
+        *reinterpret_cast<uint4*>(stage + dof[t] + Cfg::A16) = lv;      // A16 == B16
       }
       fence_proxy_async_smem();
       if (rank == 0) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&conv[s]);
       } else {
-        dwconv_bar();                                        // the 10 converter warps
-        if (threadIdx.x == 2 * 32) mbar_arrive_cluster(conv0 + s * 8);
+        if (NG == 1) {
+          dwconv_bar();                                      // the 10 converter warps
+        } else {
+          asm volatile("bar.sync %0, %1;" ::"r"(4 + grp), "r"(GT) : "memory");
+        }
+        if (gt == 0) mbar_arrive_cluster(conv0 + s * 8);
       }
-      if (++s == S) { s = 0; ph ^= 1; }
-      if (folder && (kb % kDwSub) == kDwSub / 2 && kb / kDwSub >= 1) fold(folded++);
+      s += NG;
+      if (s >= S) { s -= S; ph ^= 1; }
+      // fold run j once the conversion has passed the middle of run j + 1
+      while (folder && folded < nsub && kb >= (folded + 1) * SUB + SUB / 2) fold(folded++);
     }
     if (folder) {
       while (folded < nsub) fold(folded++);
@@ -1219,6 +1256,9 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
     tmem_dealloc_pair(tbase, Cfg::TMEM_COLS);
   }
 }
+
+constexpr int kDwpBK = MARS_DWP_BK;
+#define K_DW_PAIR k_tc3h_dw_pair<MARS_DWP_BK, MARS_DWP_NG>
 
 __global__ void k_dw3h_reduce(const float* __restrict__ part, int nchunk, int CIN, int H,
                               float* __restrict__ dW) {
@@ -1249,12 +1289,12 @@ cudaError_t dw3h_c(const float* Y, const float* rs_y, const float* dZ, const flo
 int dw_pair_clusters() {
   static int n = 0;
   if (!n) {
-    cudaFuncSetAttribute(k_tc3h_dw_pair, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         H3PairCfg::SMEM);
+    cudaFuncSetAttribute(K_DW_PAIR, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         H3PairCfg<kDwpBK>::SMEM);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(2 * 74, 1, 1);
     cfg.blockDim = dim3(384, 1, 1);
-    cfg.dynamicSmemBytes = H3PairCfg::SMEM;
+    cfg.dynamicSmemBytes = H3PairCfg<kDwpBK>::SMEM;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
     at[0].val.clusterDim.x = 2;
@@ -1263,7 +1303,7 @@ int dw_pair_clusters() {
     cfg.attrs = at;
     cfg.numAttrs = 1;
     int c = 0;
-    if (cudaOccupancyMaxActiveClusters(&c, k_tc3h_dw_pair, &cfg) != cudaSuccess || c < 1) {
+    if (cudaOccupancyMaxActiveClusters(&c, K_DW_PAIR, &cfg) != cudaSuccess || c < 1) {
       cudaGetLastError();
       c = tc_num_sms() / 2;
     }
@@ -1275,19 +1315,19 @@ int dw_pair_clusters() {
 
 cudaError_t dw3h_pair(const float* Y, const float* rs_y, const float* dZ, const float* rs_dz,
                       float* part, int nchunk, int64_t R, int rows, cudaStream_t s) {
-  using Cfg = H3PairCfg;
+  using Cfg = H3PairCfg<kDwpBK>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_tc3h_dw_pair, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(K_DW_PAIR, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          Cfg::SMEM);
     if (e != cudaSuccess) return e;
     attr = true;
   }
   CUtensorMap tdz, ty;
-  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, 256, kDwBK, Cfg::HALF / 32) ||
-      !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, 256, kDwBK, Cfg::HALF / 32))
+  if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, 256, kDwpBK, Cfg::HALF / 32) ||
+      !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, 256, kDwpBK, Cfg::HALF / 32))
     return cudaErrorInvalidValue;
-  k_tc3h_dw_pair<<<2 * nchunk, 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part, (int32_t)R, rows);
+  K_DW_PAIR<<<2 * nchunk, 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part, (int32_t)R, rows);
   return cudaGetLastError();
 }
 
@@ -1350,7 +1390,7 @@ cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, con
     // needs both SMs of a TPC free; not every SM can be paired)
     nchunk = std::min(tc_dw_chunks(R, CIN), dw_pair_clusters());
     rows = (int)((R + nchunk - 1) / nchunk);
-    rows = (rows + kDwBK - 1) / kDwBK * kDwBK;
+    rows = (rows + kDwpBK - 1) / kDwpBK * kDwpBK;
     nchunk = (int)((R + rows - 1) / rows);
     e = dw3h_pair(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, s);
     if (e != cudaSuccess) return e;

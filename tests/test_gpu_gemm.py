@@ -26,7 +26,7 @@ def test_rows(impl, M, N, K):
 
 @pytest.mark.parametrize("impl", ["auto", "simt"])
 @pytest.mark.parametrize("H", [256, 128])
-@pytest.mark.parametrize("M,K", [(16, 64), (5000, 256), (40001, 64), (123457, 256), (3001, 128)])
+@pytest.mark.parametrize("M,K", [(16, 64), (16, 256), (33, 256), (5000, 256), (40001, 64), (123457, 256), (3001, 128)])
 def test_dw(impl, H, M, K):
     rng = np.random.default_rng(M + K + H)
     A = rng.standard_normal((M, K)).astype(np.float32)
