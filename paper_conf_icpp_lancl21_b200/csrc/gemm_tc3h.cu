@@ -310,17 +310,21 @@ k_tc3h_rows(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUt
 #ifndef MARS_RP_SLABS
 #define MARS_RP_SLABS 1
 #endif
-constexpr int kRpStages = MARS_RP_STAGES;
+#ifndef MARS_RP_NARROW
+#define MARS_RP_NARROW 1      // K <= 64: 4 stages, 4 epilogue slabs per warp (output-bound launches)
+#endif
+template <int SS, int NS>
 struct H3RowsPairCfg {
   static constexpr int N = 256, NHALF = 128;
   static constexpr int A_BYTES = kBM * kBK * 4;       // fp32 staging, later hi | lo (8 KB each)
   static constexpr int B_BYTES = NHALF * kBK * 2;     // one fp16 half tile (8 KB)
   static constexpr int STAGE = A_BYTES + 2 * B_BYTES; // 32 KB
   static constexpr int SLAB = 32 * 32 * 4;
-  static constexpr int NSLAB = MARS_RP_SLABS;
+  static constexpr int S = SS;
+  static constexpr int NSLAB = NS;
   static constexpr int STAGING = 4 * NSLAB * SLAB;    // slabs per epilogue warp
   static constexpr int SCALES = kScaleSlots * kBM * 4;
-  static constexpr int SMEM = kRpStages * STAGE + STAGING + SCALES + 1024 + 512;
+  static constexpr int SMEM = SS * STAGE + STAGING + SCALES + 1024 + 512;
   static constexpr uint32_t TMEM_COLS = 512;
 };
 
@@ -328,13 +332,13 @@ __device__ __forceinline__ void rp_epi_bar() {     // the 4 epilogue warps
   asm volatile("bar.sync 2, 128;" ::: "memory");
 }
 
+template <class Cfg>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 k_tc3h_rows_pair(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmBhi,
                  const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmC,
                  const float* __restrict__ rs, const float* __restrict__ inv_tb, int32_t M,
                  int32_t K) {
-  using Cfg = H3RowsPairCfg;
-  constexpr int S = kRpStages, N = Cfg::N;
+  constexpr int S = Cfg::S, N = Cfg::N;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint8_t* staging = smem + S * Cfg::STAGE;
@@ -509,11 +513,8 @@ k_tc3h_rows_pair(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
       for (int c0 = 0; c0 < N; c0 += 32, ++nslab) {
         uint32_t r[32];
         tmem_ld32(tbase + ((uint32_t)(q * 32) << 16) + acc * N + c0, r);
-        uint8_t* slab = slab0 + (Cfg::NSLAB == 2 ? (nslab & 1) * Cfg::SLAB : 0);
-        if (lane == 0) {                      // the store that last read this slab is done
-          if (Cfg::NSLAB == 2) bulk_wait_read<1>();
-          else bulk_wait_read<0>();
-        }
+        uint8_t* slab = slab0 + (nslab % Cfg::NSLAB) * Cfg::SLAB;
+        if (lane == 0) bulk_wait_read<Cfg::NSLAB - 1>();   // the store that last read this slab is done
         __syncwarp();
         tmem_wait_ld();
 #pragma unroll
@@ -550,15 +551,19 @@ k_tc3h_rows_pair(const __grid_constant__ CUtensorMap tmA, const __grid_constant_
   }
 }
 
-int rows_pair_clusters() {
+using RpWide = H3RowsPairCfg<MARS_RP_STAGES, MARS_RP_SLABS>;
+using RpNarrow = H3RowsPairCfg<4, 4>;
+
+template <class Cfg>
+int rows_pair_clusters_t() {
   static int n = 0;
   if (!n) {
-    cudaFuncSetAttribute(k_tc3h_rows_pair, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         H3RowsPairCfg::SMEM);
+    cudaFuncSetAttribute(k_tc3h_rows_pair<Cfg>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         Cfg::SMEM);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(2 * 74, 1, 1);
     cfg.blockDim = dim3(kThreads, 1, 1);
-    cfg.dynamicSmemBytes = H3RowsPairCfg::SMEM;
+    cfg.dynamicSmemBytes = Cfg::SMEM;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
     at[0].val.clusterDim.x = 2;
@@ -567,7 +572,7 @@ int rows_pair_clusters() {
     cfg.attrs = at;
     cfg.numAttrs = 1;
     int c = 0;
-    if (cudaOccupancyMaxActiveClusters(&c, k_tc3h_rows_pair, &cfg) != cudaSuccess || c < 1) {
+    if (cudaOccupancyMaxActiveClusters(&c, k_tc3h_rows_pair<Cfg>, &cfg) != cudaSuccess || c < 1) {
       cudaGetLastError();
       c = tc_num_sms() / 2;
     }
@@ -576,12 +581,12 @@ int rows_pair_clusters() {
   return n;
 }
 
-cudaError_t rows3h_pair(const float* A, const float* rs, const __half* Bhi, const __half* Blo,
-                        const float* inv_tb, float* C, int64_t M, int K, cudaStream_t s) {
-  using Cfg = H3RowsPairCfg;
+template <class Cfg>
+cudaError_t rows3h_pair_t(const float* A, const float* rs, const __half* Bhi, const __half* Blo,
+                          const float* inv_tb, float* C, int64_t M, int K, cudaStream_t s) {
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(k_tc3h_rows_pair,
+    cudaError_t e = cudaFuncSetAttribute(k_tc3h_rows_pair<Cfg>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
     if (e != cudaSuccess) return e;
     attr = true;
@@ -598,9 +603,18 @@ cudaError_t rows3h_pair(const float* A, const float* rs, const __half* Bhi, cons
     return cudaErrorInvalidValue;
   const int ntiles = (int)((M + kBM - 1) / kBM);
   const int npair = (ntiles + 1) / 2;
-  const int nclu = std::min(npair, rows_pair_clusters());
-  k_tc3h_rows_pair<<<2 * nclu, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, tc, rs, inv_tb, (int32_t)M, K);
+  const int nclu = std::min(npair, rows_pair_clusters_t<Cfg>());
+  k_tc3h_rows_pair<Cfg><<<2 * nclu, kThreads, Cfg::SMEM, s>>>(ta, tbh, tbl, tc, rs, inv_tb,
+                                                               (int32_t)M, K);
   return cudaGetLastError();
+}
+
+// K <= 64 launches write four times the bytes they read: the epilogue's slab
+// round trips bound them, so they run with 4 slabs per epilogue warp.
+cudaError_t rows3h_pair(const float* A, const float* rs, const __half* Bhi, const __half* Blo,
+                        const float* inv_tb, float* C, int64_t M, int K, cudaStream_t s) {
+  if (MARS_RP_NARROW && K <= 64) return rows3h_pair_t<RpNarrow>(A, rs, Bhi, Blo, inv_tb, C, M, K, s);
+  return rows3h_pair_t<RpWide>(A, rs, Bhi, Blo, inv_tb, C, M, K, s);
 }
 
 // ---------------------------------------------------------------- row scales
