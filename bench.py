@@ -460,14 +460,21 @@ def run_mine(args):
         t0 = time.perf_counter()
         cur, nxt = ga, gb
         cur.reload(pinned)
+        losses, prev = [], None
         for k in range(ke):
             m2.step(cur, 1 + k, base, B)
+            tk = m2.enqueue_loss()                   # D2H of step k's loss, asynchronous
             if k + 1 < ke:
                 nxt.reload(pinned)
-            loss_k, _ = m2.read_step(want_grads=False)
+            if prev is not None:                     # the host reads step k-1's loss while
+                losses.append(m2.wait_loss(prev))    # step k runs (one-step logging lag)
+            prev = tk
             cur, nxt = nxt, cur
+        losses.append(m2.wait_loss(prev))
         torch.cuda.synchronize()
         dt = time.perf_counter() - t0
+        if len(losses) != ke or not all(np.isfinite(losses)):
+            raise RuntimeError("e2e: a step's loss was not read back or is not finite")
         m2.free()
         ga.free()
         gb.free()
@@ -476,7 +483,9 @@ def run_mine(args):
                "note": "per step: mars_graph_reload of a double-buffered graph handle (H2D from "
                        "pinned host memory + CSR build on libmars's loader stream, overlapping "
                        "the previous step's compute) + mars_dgi_step (captured graph replay) + "
-                       "loss D2H (mars_dgi_read_step); wall clock, rank-local (no allreduce)"}
+                       "loss D2H (mars_dgi_enqueue_loss after the step; the host reads it with "
+                       "mars_dgi_wait_loss while the next step runs, every step's loss checked "
+                       "finite); wall clock, rank-local (no allreduce)"}
 
     # the bf16 path (MARS_BF16, 2e-2 parity bar) on the same workload, same timing
     b16 = None

@@ -479,6 +479,19 @@ MARS_API mars_status mars_ppo_iteration_joint(mars_ppo* o, const mars_graph* g, 
  * row-sharded model, ECUDA if a cross-shard barrier timed out. */
 MARS_API mars_status mars_dgi_read_step(mars_dgi* m, float* loss, float* grads);
 
+/* Asynchronous loss read-back for a training loop that reads every step's
+ * loss without stalling the device between steps (a10's scalar, the value
+ * mars_dgi_read_step returns).  mars_dgi_enqueue_loss enqueues, on the
+ * library stream after everything enqueued so far (normally the step just
+ * launched), a device-to-host copy of the most recent step's loss into a
+ * page-locked slot owned by the model, and returns a ticket (0, 1, 2, ...).
+ * mars_dgi_wait_loss blocks until that copy has landed and returns the loss;
+ * MARS_ENUMERIC if a step up to that one skipped its Adam update (the check
+ * mars_dgi_read_step makes).  The last 16 tickets are valid (EINVAL for
+ * older ones); enqueueing a 17th waits for the oldest slot's copy. */
+MARS_API mars_status mars_dgi_enqueue_loss(mars_dgi* m, int64_t* ticket);
+MARS_API mars_status mars_dgi_wait_loss(mars_dgi* m, int64_t ticket, float* loss);
+
 /* ------------------------------------------------------------------------ */
 /* Row-sharded single graph: one op graph too large for   */
 /* one GPU (config 5: ~1M ops) split into P <= 8 contiguous row blocks, one   */

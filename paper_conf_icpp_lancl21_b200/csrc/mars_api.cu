@@ -406,6 +406,16 @@ struct mars_dgi {
   StepParams* h_sp = nullptr;       // pinned ring
   cudaEvent_t* sp_ev = nullptr;
   int sp_ring = 32, sp_next = 0;
+  // asynchronous loss read-back (mars_dgi_enqueue_loss / mars_dgi_wait_loss):
+  // pinned {loss, skipped count} slots, one event each, tickets modulo the ring
+  struct LossSlot {
+    float loss;
+    int32_t skipped;
+  };
+  static constexpr int kLossRing = 16;
+  LossSlot* loss_ring = nullptr;
+  cudaEvent_t loss_ev[kLossRing] = {};
+  int64_t loss_next = 0;
   Workspace ws;
   const mars_graph* ws_graph = nullptr;
   mars_contrastive ct{1, MARS_CORRUPT_PERMUTE, 0.f, MARS_READOUT_SIGMOID_MEAN, MARS_AGG_GCN,
@@ -527,6 +537,9 @@ struct mars_dgi {
       delete[] sp_ev;
     }
     if (h_sp) cudaFreeHost(h_sp);
+    for (cudaEvent_t e : loss_ev)
+      if (e) cudaEventDestroy(e);
+    if (loss_ring) cudaFreeHost(loss_ring);
     if (comm && g_nccl.CommDestroy) g_nccl.CommDestroy(comm);
     if (own_stream) cudaStreamDestroy(own_stream);
   }
@@ -3014,6 +3027,40 @@ extern "C" mars_status mars_dgi_read_step(mars_dgi* m, float* loss, float* grads
   if (derr) return fail(MARS_ECUDA, "data-parallel barrier timed out (a peer rank did not step)");
   if (loss) *loss = l;
   return check_skipped(m, skipped);
+}
+
+extern "C" mars_status mars_dgi_enqueue_loss(mars_dgi* m, int64_t* ticket) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (!ticket) return fail(MARS_EINVAL, "ticket is NULL");
+  CK(cudaSetDevice(m->cfg.device));
+  if (!m->loss_ring) {
+    CK(cudaMallocHost(&m->loss_ring, sizeof(mars_dgi::LossSlot) * mars_dgi::kLossRing));
+    for (cudaEvent_t& e : m->loss_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  const int slot = (int)(m->loss_next % mars_dgi::kLossRing);
+  // the slot's previous copy must have landed before it is overwritten
+  CK(cudaEventSynchronize(m->loss_ev[slot]));
+  cudaStream_t s = m->stream;
+  mars_dgi::LossSlot* d = m->loss_ring + slot;
+  CK(cudaMemcpyAsync(&d->loss, m->grads_final() + m->P, sizeof(float), cudaMemcpyDeviceToHost, s));
+  CK(cudaMemcpyAsync(&d->skipped, &m->adam_st->skipped, sizeof(int32_t), cudaMemcpyDeviceToHost,
+                     s));
+  CK(cudaEventRecord(m->loss_ev[slot], s));
+  *ticket = m->loss_next++;
+  return MARS_OK;
+}
+
+extern "C" mars_status mars_dgi_wait_loss(mars_dgi* m, int64_t ticket, float* loss) {
+  if (mars_status st = check_dgi(m)) return st;
+  if (ticket < 0 || ticket >= m->loss_next || ticket < m->loss_next - mars_dgi::kLossRing)
+    return fail(MARS_EINVAL, "loss ticket %lld is not one of the last %d enqueued",
+                (long long)ticket, mars_dgi::kLossRing);
+  CK(cudaSetDevice(m->cfg.device));
+  const int slot = (int)(ticket % mars_dgi::kLossRing);
+  CK(cudaEventSynchronize(m->loss_ev[slot]));
+  const mars_dgi::LossSlot d = m->loss_ring[slot];
+  if (loss) *loss = d.loss;
+  return check_skipped(m, d.skipped);
 }
 
 // ---------------------------------------------------------------- placer (NEXT-2)

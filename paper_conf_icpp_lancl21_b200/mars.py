@@ -130,6 +130,8 @@ SIGNATURES = {
                                        ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
                                        ctypes.c_int32, ctypes.c_void_p]),
     "mars_dgi_read_step": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_enqueue_loss": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_void_p]),
+    "mars_dgi_wait_loss": (ctypes.c_int, [ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p]),
     "mars_graph_load_shard": (ctypes.c_int, [ctypes.POINTER(GraphDesc), ctypes.c_int32,
                                              ctypes.c_int32, ctypes.c_int32,
                                              ctypes.POINTER(ctypes.c_void_p)]),
@@ -538,6 +540,19 @@ class DGI:
         _check(lib().mars_dgi_read_step(self.handle, ctypes.byref(loss),
                                         None if grads is None else _ptr(grads)))
         return loss.value, grads
+
+    def enqueue_loss(self) -> int:
+        """mars_dgi_enqueue_loss: ticket of an asynchronous D2H copy of the
+        most recent step's loss (see mars.h)."""
+        t = ctypes.c_int64()
+        _check(lib().mars_dgi_enqueue_loss(self.handle, ctypes.byref(t)))
+        return t.value
+
+    def wait_loss(self, ticket: int) -> float:
+        """mars_dgi_wait_loss: the loss of an enqueued read-back (blocks)."""
+        loss = ctypes.c_float()
+        _check(lib().mars_dgi_wait_loss(self.handle, ctypes.c_int64(ticket), ctypes.byref(loss)))
+        return loss.value
 
     def last_launches(self) -> int:
         return int(lib().mars_dgi_last_launches(self.handle))

@@ -294,6 +294,41 @@ def test_nonfinite_step_skips_adam():
     assert m.get_state()[3] == 2
 
 
+def test_async_loss_readback():
+    """mars_dgi_enqueue_loss / mars_dgi_wait_loss: the losses read with a
+    one-step lag equal the synchronous per-step losses bitwise; tickets older
+    than the 16-slot ring are rejected; a skipped (non-finite) step is
+    reported by the wait like mars_dgi_read_step reports it."""
+    gs = [SG.tiny(0), SG.tiny(1)]
+    g = mars.graph_load(gs)
+    ref = mars.dgi_create(in_dim=16, hidden_dim=32, seed=5)
+    want = [ref.step(g, k, 0, want_loss=True)["loss"] for k in range(20)]
+    m = mars.dgi_create(in_dim=16, hidden_dim=32, seed=5)
+    got, tickets = [], []
+    for k in range(20):
+        m.step(g, k, 0)
+        tickets.append(m.enqueue_loss())
+        if k > 0:
+            got.append(m.wait_loss(tickets[k - 1]))
+    got.append(m.wait_loss(tickets[-1]))
+    assert tickets == list(range(20))
+    assert got == want
+    with pytest.raises(mars.MarsError) as e:
+        m.wait_loss(tickets[2])                       # recycled slot
+    assert e.value.status == mars.mars.MARS_EINVAL
+    with pytest.raises(mars.MarsError):
+        m.wait_loss(20)                               # not enqueued yet
+    p, mm, v, t = m.get_state()
+    bad = p.copy()
+    bad[0] = np.nan
+    m.set_state(bad, mm, v, t)
+    m.step(g, 20, 0)
+    tk = m.enqueue_loss()
+    with pytest.raises(mars.MarsError) as e:
+        m.wait_loss(tk)
+    assert e.value.status == mars.mars.MARS_ENUMERIC
+
+
 def test_two_models_share_a_graph_with_long_rows():
     """Two models stepping the same graph set concurrently on their own streams
     (the long-row segment scratch is per model): results equal the
