@@ -671,6 +671,51 @@ __global__ void k_split_w3h(const float* __restrict__ W, int CIN, int H,
   Bt_lo[(int64_t)h * CIN + c] = lo;
 }
 
+// All layers' weights in one launch (grid: kSplitBlocks x layers): every block
+// forms its layer's max |W| itself (at most 256 KB, read from L2), block 0
+// publishes {t, 1/t}, and each block splits its share of the entries --
+// the same values as k_wscale + k_split_w3h per layer, in one graph node
+// instead of six.
+constexpr int kSplitBlocks = 8;
+__global__ void __launch_bounds__(1024) k_split_w3h_all(const W3Split a) {
+  __shared__ float sh[32];
+  __shared__ float ts;
+  const int l = blockIdx.y;
+  const float* __restrict__ W = a.W[l];
+  const int CIN = a.cin[l], H = a.H, n = CIN * H;
+  float m = 0.f;
+  for (int e = threadIdx.x; e < n; e += 1024) m = fmaxf(m, fabsf(W[e]));
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(kFull, m, o));
+  if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = m;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    m = sh[threadIdx.x];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(kFull, m, o));
+    if (threadIdx.x == 0) {
+      const float t = pow2_scale(m);
+      ts = t;
+      if (blockIdx.x == 0) {
+        a.wsc[l][0] = t;
+        a.wsc[l][1] = 1.f / t;
+      }
+    }
+  }
+  __syncthreads();
+  const float t = ts;
+  for (int e = blockIdx.x * 1024 + threadIdx.x; e < n; e += kSplitBlocks * 1024) {
+    const int c = e / H, h = e % H;
+    const float x = W[e] * t;
+    const __half hi = __float2half_rn(x);
+    const __half lo = __float2half_rn(x - __half2float(hi));
+    static_cast<__half*>(a.b_hi[l])[e] = hi;
+    static_cast<__half*>(a.b_lo[l])[e] = lo;
+    static_cast<__half*>(a.bt_hi[l])[(int64_t)h * CIN + c] = hi;
+    static_cast<__half*>(a.bt_lo[l])[(int64_t)h * CIN + c] = lo;
+  }
+}
+
 template <int N>
 // N = the tile width (64, 128, 256); n = the actual output width (n <= N: the
 // weight rows beyond n are zero-filled by TMA and the store is clipped to n).
@@ -1356,6 +1401,13 @@ cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void*
   k_split_w3h<<<cdiv((int64_t)CIN * H, 256), 256, 0, s>>>(
       W, CIN, H, wsc, static_cast<__half*>(Bt_hi), static_cast<__half*>(Bt_lo),
       static_cast<__half*>(B_hi), static_cast<__half*>(B_lo));
+  return cudaGetLastError();
+}
+
+cudaError_t tc3h_split_weights_all(const W3Split& a, int nl, cudaStream_t s, int* launches) {
+  if (nl < 1 || nl > 3) return cudaErrorInvalidValue;
+  count_launch(launches);
+  k_split_w3h_all<<<dim3(kSplitBlocks, nl), 1024, 0, s>>>(a);
   return cudaGetLastError();
 }
 

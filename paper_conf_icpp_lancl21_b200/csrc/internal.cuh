@@ -204,6 +204,15 @@ bool tc_supported(int cin, int h);
 bool tc3h_supported(int cin, int h);   // the 3xFP16 fp32 path (also the tiny widths)
 size_t tc_dw_partial_floats(int64_t R, int CIN);
 // gemm_tc3h.cu: 3xFP16 row GEMMs with power-of-two scaling (fp32 path)
+// The same split for up to three layers in one launch (the DGI step's W1..W3).
+struct W3Split {
+  const float* W[3];
+  int cin[3];
+  int H;
+  float* wsc[3];
+  void *bt_hi[3], *bt_lo[3], *b_hi[3], *b_lo[3];   // fp16
+};
+cudaError_t tc3h_split_weights_all(const W3Split& a, int nl, cudaStream_t s, int* launches);
 cudaError_t tc3h_split_weights(const float* W, int CIN, int H, float* wsc, void* Bt_hi,
                                void* Bt_lo, void* B_hi, void* B_lo, cudaStream_t s,
                                int* launches);

@@ -1845,13 +1845,29 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   MARK(MARS_PH_PERM);
   const bool b16 = m->cfg.precision == MARS_BF16;        // bf16 storage + bf16 MMAs
   bool tc[3];
-  for (int l = 0; l < 3; ++l) {
-    int Cin = l == 0 ? F : H;
-    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(Cin, H);
-    if (b16) RET(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl));
-    else if (tc[l])
-      RET(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
-                             w.h3_w_hi[l], w.h3_w_lo[l], s, nl));
+  for (int l = 0; l < 3; ++l)
+    tc[l] = m->gemm_impl != MARS_GEMM_SIMT && tc3h_supported(l == 0 ? F : H, H);
+  if (!b16 && tc[0] && tc[1] && tc[2]) {                  // one launch for the three splits
+    W3Split a{};
+    a.H = H;
+    for (int l = 0; l < 3; ++l) {
+      a.W[l] = W[l];
+      a.cin[l] = l == 0 ? F : H;
+      a.wsc[l] = w.h3_wsc[l];
+      a.bt_hi[l] = w.h3_wt_hi[l];
+      a.bt_lo[l] = w.h3_wt_lo[l];
+      a.b_hi[l] = w.h3_w_hi[l];
+      a.b_lo[l] = w.h3_w_lo[l];
+    }
+    RET(tc3h_split_weights_all(a, 3, s, nl));
+  } else {
+    for (int l = 0; l < 3; ++l) {
+      int Cin = l == 0 ? F : H;
+      if (b16) RET(tc16_weights(W[l], Cin, H, w.w16t[l], w.w16[l], s, nl));
+      else if (tc[l])
+        RET(tc3h_split_weights(W[l], Cin, H, w.h3_wsc[l], w.h3_wt_hi[l], w.h3_wt_lo[l],
+                               w.h3_w_hi[l], w.h3_w_lo[l], s, nl));
+    }
   }
   MARK(MARS_PH_GEMM_FWD);
   const size_t es = b16 ? 2 : 4;                         // storage bytes per element

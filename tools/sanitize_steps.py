@@ -1,6 +1,7 @@
 """compute-sanitizer workload (tools/sanitize.sh): one eager step per case on
 small sets -- tiny (SIMT GEMMs), Inception x2 at H = 128 and one Inception
-graph at H = 256 (tcgen05 row / dW kernels, incl. the CTA-pair dW), both
+graph at H = 256 (tcgen05 row / dW kernels, incl. the CTA-pair dW), two GNMT
+graphs (R > 2 x 128 x #SM rows: the CTA-pair row GEMMs, both instantiations), both
 precisions, plus an encode and the featuriser; then the NEXT-4 variants
 (MARS_SAN_ONLY=default | variants selects one group).  Small so the
 instrumented run finishes in minutes."""
@@ -16,7 +17,8 @@ cases = [([SG.tiny(0), SG.tiny(1)], 16, 32, mars.MARS_FP32),
          ([SG.cached("inception", i) for i in range(2)], 64, 128, mars.MARS_FP32),
          ([SG.cached("inception", 0)], 64, 256, mars.MARS_FP32),
          ([SG.cached("inception", 0)], 64, 256, mars.MARS_BF16),
-         ([SG.cached("bert", 0)], 64, 256, mars.MARS_FP32)]          # long rows
+         ([SG.cached("bert", 0)], 64, 256, mars.MARS_FP32),          # long rows
+         ([SG.cached("gnmt", i) for i in range(2)], 64, 256, mars.MARS_FP32)]   # pair row GEMMs
 # NEXT-4 variants (c34-c38): shared positive with padding, masking, mean
 # readout, SAGE-GCN values, and the SAGE-mean encoder's redirected CSR
 variants = [([SG.tiny(0), SG.tiny(1)], 16, 32, mars.MARS_FP32, "gcn",
