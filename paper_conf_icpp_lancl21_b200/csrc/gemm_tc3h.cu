@@ -937,12 +937,12 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 #pragma unroll
       for (int h = 0; h < NH; ++h)
 #pragma unroll
-        for (int c0 = 0; c0 < MC; c0 += 32) {
-          uint32_t w[32];
-          tmem_ld32(twork + lane_off + h * CINT + c0, w);
+        for (int c0 = 0; c0 < MC; c0 += 16) {          // 16 columns at a time: register budget
+          uint32_t w[16];
+          tmem_ld16(twork + lane_off + h * CINT + c0, w);
           tmem_wait_ld();
 #pragma unroll
-          for (int j = 0; j < 32; ++j) master[h][c0 + j] += __uint_as_float(w[j]);
+          for (int j = 0; j < 16; ++j) master[h][c0 + j] += __uint_as_float(w[j]);
         }
       tc_fence_before();
       __syncwarp();
@@ -1057,6 +1057,19 @@ k_tc3h_dw(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUte
 #ifndef MARS_DWP_NG
 #define MARS_DWP_NG 1         // converter groups working on alternate stages
 #endif
+#ifndef MARS_DWP_RUN
+#define MARS_DWP_RUN 128      // rows per tensor-core accumulation run before the fp32 fold
+#endif
+
+#define MARS_DWP_WARPS 10     // TMA + MMA + 8 converter / folder warps
+constexpr int kDwpThreads = MARS_DWP_WARPS * 32;
+// one CTA per SM: warps are spread over the 4 SM sub-partitions, each with a
+// quarter of the register file (16384), so the busiest one bounds the count
+constexpr int kDwpRegs = (16384 / (32 * ((MARS_DWP_WARPS + 3) / 4))) / 8 * 8;
+template <int NCW>
+__device__ __forceinline__ void dwp_conv_bar() {    // the converter warps
+  asm volatile("bar.sync 2, %0;" ::"n"(NCW * 32) : "memory");
+}
 
 template <int BK>
 struct H3PairCfg {
@@ -1070,13 +1083,13 @@ struct H3PairCfg {
   static constexpr int STAGE = A32 + B32 + 2 * A16 + 2 * B16;   // 2 KB per row
   static constexpr int S = BK == 16 ? MARS_PAIR_STAGES : (200 * 1024) / STAGE;
   static constexpr int SMEM = S * STAGE + 1024 + 512;
-  static constexpr int SUB = 128 / BK;                 // stages per 128-row TMEM work run
+  static constexpr int SUB = MARS_DWP_RUN / BK;        // stages per TMEM work run (MARS_DWP_RUN rows)
   static constexpr uint32_t TMEM_COLS = 512;           // 2 buffers x 256 fp32 columns
   static constexpr int MC = 128;                       // columns per folding thread
 };
 
 template <int BK, int NG>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(384, 1)
+__global__ void __cluster_dims__(2, 1, 1) __maxnreg__(kDwpRegs)
 k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__ CUtensorMap tmY,
                const float* __restrict__ rs_dz, const float* __restrict__ rs_y,
                float* __restrict__ part, int32_t R, int32_t rows_per_chunk) {
@@ -1085,8 +1098,10 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
   constexpr int SUB = Cfg::SUB;
   constexpr int MC = Cfg::MC;
   constexpr int CIN = 256, HH = 256;
-  constexpr int GW = 10 / NG;                            // converter warps per group
-  static_assert(10 % NG == 0 && SUB >= NG, "converter groups");
+  constexpr int NCW = kDwpThreads / 32 - 2;              // converter (and folder) warps
+  constexpr int GW = NCW / NG;                           // converter warps per group
+  static_assert(NCW % NG == 0 && SUB >= NG, "converter groups");
+  static_assert(NCW == 8, "8 folder warps: 4 TMEM lane quadrants x 2 column halves");
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * Cfg::STAGE);
@@ -1096,7 +1111,7 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
   uint64_t* tfull = bars + 3 * S;        // [2]
   uint64_t* tempty = bars + 3 * S + 2;   // [2] even CTA: both CTAs' folders
   uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 3 * S + 4);
-  float* wmin = reinterpret_cast<float*>(bars + 3 * S + 6);   // [2][10] per-warp minima
+  float* wmin = reinterpret_cast<float*>(bars + 3 * S + 6);   // [2][NCW] per-warp minima
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_rank();
@@ -1118,7 +1133,7 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 9);        // 8 local folder warps + 1 from the odd CTA
+      mbar_init(&tempty[b], NCW + 1);  // the local folder warps + 1 from the odd CTA
     }
     fence_mbar_init();
     tma_prefetch(&tmDZ);
@@ -1176,10 +1191,10 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
         mma_commit_pair(&tfull[buf], 0x3);
       }
     }
-  } else {                         // ---- convert (warps 2..11); warps 4..11 also fold
-    const bool folder = warp >= 4;
+  } else {                         // ---- convert and fold (warps 2 .. 2 + NCW - 1)
+    constexpr bool folder = true;
     const int ct = (warp - 2) * 32 + lane;
-    constexpr int NT = 10 * 32;
+    constexpr int NT = NCW * 32;
     float mz = INFINITY, my = INFINITY;
     for (int32_t r = r0 + ct; r < r1; r += NT) {
       mz = fminf(mz, __ldg(rs_dz + r));
@@ -1192,20 +1207,20 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
     }
     if (lane == 0) {
       wmin[warp - 2] = mz;
-      wmin[10 + warp - 2] = my;
+      wmin[NCW + warp - 2] = my;
     }
-    dwconv_bar();
+    dwp_conv_bar<NCW>();
     float sz = INFINITY, sy = INFINITY;
 #pragma unroll
-    for (int k = 0; k < 10; ++k) {
+    for (int k = 0; k < NCW; ++k) {
       sz = fminf(sz, wmin[k]);
-      sy = fminf(sy, wmin[10 + k]);
+      sy = fminf(sy, wmin[NCW + k]);
     }
     if (!(sz < INFINITY)) sz = 1.f;          // empty chunk
     if (!(sy < INFINITY)) sy = 1.f;
     const uint32_t conv0 = mapa_u32(conv, 0), tempty0 = mapa_u32(tempty, 0);
 
-    const int q = warp & 3, ch = (warp - 4) >> 2;
+    const int q = warp & 3, ch = (warp - 2) >> 2;     // TMEM lane quadrant, column half
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     float master[MC];
 #pragma unroll
@@ -1217,20 +1232,20 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
       tc_fence_after();
       const uint32_t twork = tbase + buf * CIN + ch * MC;
 #pragma unroll
-      for (int c0 = 0; c0 < MC; c0 += 32) {
-        uint32_t w[32];
-        tmem_ld32(twork + lane_off + c0, w);
+      for (int c0 = 0; c0 < MC; c0 += 16) {            // 16 columns at a time: register budget
+        uint32_t w[16];
+        tmem_ld16(twork + lane_off + c0, w);
         tmem_wait_ld();
 #pragma unroll
-        for (int j = 0; j < 32; ++j) master[c0 + j] += __uint_as_float(w[j]);
+        for (int j = 0; j < 16; ++j) master[c0 + j] += __uint_as_float(w[j]);
       }
       tc_fence_before();
       if (rank == 0) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&tempty[buf]);
       } else {
-        asm volatile("bar.sync 3, 256;" ::: "memory");      // the 8 folder warps
-        if (threadIdx.x == 4 * 32) mbar_arrive_cluster(tempty0 + buf * 8);
+        asm volatile("bar.sync 3, %0;" ::"r"(NT) : "memory");   // the folder warps
+        if (threadIdx.x == 2 * 32) mbar_arrive_cluster(tempty0 + buf * 8);
       }
     };
     // converter group: warps 2 + GW g .. 2 + GW g + GW - 1 convert stages kb = g (mod NG)
@@ -1285,7 +1300,7 @@ k_tc3h_dw_pair(const __grid_constant__ CUtensorMap tmDZ, const __grid_constant__
         if (lane == 0) mbar_arrive(&conv[s]);
       } else {
         if (NG == 1) {
-          dwconv_bar();                                      // the 10 converter warps
+          dwp_conv_bar<NCW>();                               // the converter warps
         } else {
           asm volatile("bar.sync %0, %1;" ::"r"(4 + grp), "r"(GT) : "memory");
         }
@@ -1352,7 +1367,7 @@ int dw_pair_clusters() {
                          H3PairCfg<kDwpBK>::SMEM);
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(2 * 74, 1, 1);
-    cfg.blockDim = dim3(384, 1, 1);
+    cfg.blockDim = dim3(kDwpThreads, 1, 1);
     cfg.dynamicSmemBytes = H3PairCfg<kDwpBK>::SMEM;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
@@ -1386,7 +1401,7 @@ cudaError_t dw3h_pair(const float* Y, const float* rs_y, const float* dZ, const 
   if (!tc_tmap_blocks(&tdz, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, dZ, R, 256, kDwpBK, Cfg::HALF / 32) ||
       !tc_tmap_blocks(&ty, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, Y, R, 256, kDwpBK, Cfg::HALF / 32))
     return cudaErrorInvalidValue;
-  K_DW_PAIR<<<2 * nchunk, 384, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part, (int32_t)R, rows);
+  K_DW_PAIR<<<2 * nchunk, kDwpThreads, Cfg::SMEM, s>>>(tdz, ty, rs_dz, rs_y, part, (int32_t)R, rows);
   return cudaGetLastError();
 }
 
