@@ -36,6 +36,17 @@ constexpr int kSpmmThreads = 32;   // one warp per block: a slow (hub) row holds
 #define MARS_SPMM_KU 4
 #endif
 constexpr int kU = MARS_SPMM_KU;   // neighbours whose gathers are in flight together
+// The backward rows also stream their own Z rows (PReLU') and write dZ: with
+// 2 neighbours per gather batch (fp32) they fit the 64-register budget
+// without spilling, measured -8 % against 4 ((17)).
+#ifndef MARS_SPMM_KU_BWD
+#define MARS_SPMM_KU_BWD 2
+#endif
+#ifndef MARS_SPMM_KU_BWD16
+#define MARS_SPMM_KU_BWD16 4
+#endif
+template <typename T>
+constexpr int kUB = std::is_same<T, float>::value ? MARS_SPMM_KU_BWD : MARS_SPMM_KU_BWD16;
 
 // C in {16, 32, 64, 128, 256} (mars.h restricts F and H to these widths).
 #ifndef MARS_SPMM_LMAX_BF16
@@ -188,7 +199,7 @@ __device__ __forceinline__ void gather_batch(const Src& src, int t, int nvalid, 
 // broadcast by shuffles, then batches of kU neighbours; the last partial batch
 // is one padded batch (measured against a neighbour-at-a-time tail and
 // predicated tails).
-template <class S, bool BOTH, int ACT, bool PERM, typename T, class Src>
+template <class S, bool BOTH, int ACT, bool PERM, typename T, int KU = kU, class Src>
 __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __restrict__ colind,
                                            const float* __restrict__ vals,
                                            const int32_t* __restrict__ perm, int32_t rb,
@@ -204,8 +215,8 @@ __device__ __forceinline__ void row_gather(const Src& src, const int32_t* __rest
       cv = vals[k0 + sl];
       if (PERM && BOTH) cjn = perm[k0 + sl];   // colperm: pi[colind[k]], no dependent lookup
     }
-    for (int t = 0; t < cnt; t += kU)
-      gather_batch<S, kU, BOTH, ACT, PERM, T>(src, t, min(kU, cnt - t), cj, cv, cjn, gmask, sl,
+    for (int t = 0; t < cnt; t += KU)
+      gather_batch<S, KU, BOTH, ACT, PERM, T>(src, t, min(KU, cnt - t), cj, cv, cjn, gmask, sl,
                                               a, accp, accn);
   }
 }
@@ -327,10 +338,10 @@ __device__ __forceinline__ void bwd_row(int32_t i, int32_t long_min,
 #pragma unroll
     for (int e = 0; e < V; ++e) accp[q][e] = accn[q][e] = 0.f;
   if (SH)
-    row_gather<S, true, false, false, T>(PeerSrc<T, C>{pr}, colind, vals, nullptr, rb, re, gmask,
+    row_gather<S, true, false, false, T, kUB<T>>(PeerSrc<T, C>{pr}, colind, vals, nullptr, rb, re, gmask,
                                          sl, a, accp, accn);
   else
-    row_gather<S, true, false, false, T>(StackedSrc<T, C>{dY, Nt}, colind, vals, nullptr, rb, re,
+    row_gather<S, true, false, false, T, kUB<T>>(StackedSrc<T, C>{dY, Nt}, colind, vals, nullptr, rb, re,
                                          gmask, sl, a, accp, accn);
   float o[2][S::NT][V];
 #pragma unroll
