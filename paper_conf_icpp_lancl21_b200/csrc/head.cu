@@ -578,8 +578,8 @@ k_dz3(const T* __restrict__ Z3, const float* __restrict__ alpha,
         if (act && r + u < r1) StoreN<T, V>::store(dZ + (base + r + u) * H + (lane + q * LPR) * V, o);
       }
       if (rs) {                     // row scale of the stored dZ3 row (3xFP16 dY GEMM)
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(kFull, mx, o));
+        // |values| >= 0: the unsigned max of the bit patterns is the float max
+        mx = __uint_as_float(__reduce_max_sync(kFull, __float_as_uint(mx)));
         if (lane == 0 && r + u < r1) rs[base + r + u] = pow2_scale(mx);
       }
     }

@@ -35,6 +35,9 @@ constexpr int kSpmmThreads = 32;   // one warp per block: a slow (hub) row holds
 #ifndef MARS_SPMM_KU
 #define MARS_SPMM_KU 4
 #endif
+#ifndef MARS_SPMM_REDUX
+#define MARS_SPMM_REDUX 1           // row-scale maxima by redux.sync (whole-warp rows)
+#endif
 constexpr int kU = MARS_SPMM_KU;   // neighbours whose gathers are in flight together
 // The backward rows also stream their own Z rows (PReLU') and write dZ: with
 // 2 neighbours per gather batch (fp32) they fit the 64-register budget
@@ -231,8 +234,15 @@ __device__ __forceinline__ void row_scale_out(const float (&x)[S::NT][NV], unsig
   for (int q = 0; q < S::NT; ++q)
 #pragma unroll
     for (int e = 0; e < NV; ++e) m = fmaxf(m, fabsf(x[q][e]));
+  if constexpr (MARS_SPMM_REDUX && S::L == 32) {
+    // |x| >= 0: the unsigned maximum of the bit patterns is the float
+    // maximum -- one redux.sync over the warp (a NaN, whose bits exceed
+    // +inf's, gives the scale 1 in pow2_scale)
+    m = __uint_as_float(__reduce_max_sync(gmask, __float_as_uint(m)));
+  } else {
 #pragma unroll
-  for (int o = S::L / 2; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gmask, m, o));
+    for (int o = S::L / 2; o > 0; o >>= 1) m = fmaxf(m, __shfl_xor_sync(gmask, m, o));
+  }
   if (sl == 0) *dst = pow2_scale(m);
 }
 
