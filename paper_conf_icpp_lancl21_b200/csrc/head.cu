@@ -218,6 +218,9 @@ __device__ __forceinline__ double softplus_d(double x) {
 // the sigmoid / softplus of logit j in fp64 (parallel over lanes) and the
 // dl values are broadcast back.
 template <int NC, typename T>
+#ifndef MARS_SCORE_RS
+#define MARS_SCORE_RS 1      // logit warp sums as one reduce-scatter (k_score)
+#endif
 #ifndef MARS_SCORE_MINB
 #define MARS_SCORE_MINB 2
 #endif
@@ -283,11 +286,30 @@ k_score(const T* __restrict__ Z3, const float* __restrict__ alpha,
 #pragma unroll
         for (int e = 0; e < V; ++e) t = fmaf(prelu(x[e], a), v[q][e], t);
       }
-      l[j] = warp_sum(t);
+      l[j] = (MARS_SCORE_RS && 2 * NU == 8) ? t : warp_sum(t);
     }
     float mine = l[0];
+    if constexpr (MARS_SCORE_RS && 2 * NU == 8) {
+      // the 8 logits' warp sums as one reduce-scatter (9 shuffles instead of
+      // 40): halving exchanges over lane bits 4, 3, 2 leave lane L with a
+      // partial of logit 4 b4 + 2 b3 + b2, then bits 1, 0 finish it
+      const bool b4 = lane & 16, b3 = lane & 8, b2 = lane & 4;
+      float u4[4], u2[2];
 #pragma unroll
-    for (int j = 1; j < 2 * NU; ++j) mine = lane == j ? l[j] : mine;
+      for (int k = 0; k < 4; ++k)
+        u4[k] = (b4 ? l[k + 4] : l[k]) + __shfl_xor_sync(kFull, b4 ? l[k] : l[k + 4], 16);
+#pragma unroll
+      for (int k = 0; k < 2; ++k)
+        u2[k] = (b3 ? u4[k + 2] : u4[k]) + __shfl_xor_sync(kFull, b3 ? u4[k] : u4[k + 2], 8);
+      float u1 = (b2 ? u2[1] : u2[0]) + __shfl_xor_sync(kFull, b2 ? u2[0] : u2[1], 4);
+      u1 += __shfl_xor_sync(kFull, u1, 2);
+      u1 += __shfl_xor_sync(kFull, u1, 1);
+      const int src = ((lane & 4) << 2) | ((lane & 2) << 2) | ((lane & 1) << 2);   // logit lane & 7
+      mine = __shfl_sync(kFull, u1, src);
+    } else {
+#pragma unroll
+      for (int j = 1; j < 2 * NU; ++j) mine = lane == j ? l[j] : mine;
+    }
     float dmine = 0.f;
     if (lane < 2 * NU && i + (lane >> 1) < r1) {
       const double x = (double)mine;
