@@ -62,6 +62,8 @@ struct GraphDev {
   int32_t nbuckets;
   const int32_t* bucket_off; // [G+1]
   const int32_t* bucket_log2;// [G]
+  int32_t max_bucket_log2 = 0;  // host copy of max_g bucket_log2[g] (per-graph perm kernel)
+  int32_t max_graph_nodes = 0;  // host copy of max_g N_g
   const int32_t* gsize;      // [G] node count N_g of each graph (all shards of a row-sharded graph)
   const int64_t* pair_off;   // [G] pair index of graph g = pair_base + pair_off[g] (c15)
 };
@@ -151,6 +153,13 @@ struct PermWork {
 };
 cudaError_t launch_perm(const GraphDev& g, uint64_t seed, const StepParams* sp,
                         const PermWork& w, int32_t* perm_global, cudaStream_t s, int* launches);
+// launch_perm + launch_colperm over the same (unsharded) view in one launch of
+// one CTA per graph (buckets and members in shared memory); returns
+// cudaErrorNotSupported when a graph is too large for it (the caller then
+// runs the two launches above).
+cudaError_t launch_perm_graph(const GraphDev& g, uint64_t seed, const StepParams* sp,
+                              const PermWork& w, int32_t* perm_global, int32_t* colperm,
+                              cudaStream_t s, int* launches);
 
 // ---------------------------------------------------------------- spmm.cu
 // A row is long when its serial gather time would exceed about half the row

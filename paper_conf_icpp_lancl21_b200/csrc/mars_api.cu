@@ -330,6 +330,13 @@ static cudaError_t build_long_rows(mars_graph* gr, GraphDev& v, cudaStream_t s,
   return cudaStreamSynchronize(s);   // the host vectors go out of scope
 }
 
+#ifndef MARS_PERM_GRAPH
+#define MARS_PERM_GRAPH 1  // a4: one CTA per graph (launch_perm_graph)
+#endif
+#ifndef MARS_PERM_GRAPH_COLPERM
+#define MARS_PERM_GRAPH_COLPERM 0   // colperm inside that kernel (16 CTAs) or over the whole GPU
+#endif
+
 struct Workspace {
   int32_t Nt = 0, G = 0, nchunks = 0, nbuckets = 0, F = 0, H = 0;
   int32_t Nperm = 0;      // rows of the permutation (the whole graph when row-sharded)
@@ -804,6 +811,10 @@ extern "C" mars_status mars_graph_load(const mars_graph_desc* descs, int32_t G, 
   v.nbuckets = bucket_off[G];
   v.bucket_off = gr->bucket_off;
   v.bucket_log2 = gr->bucket_log2;
+  for (int g = 0; g < G; ++g) {
+    v.max_bucket_log2 = std::max(v.max_bucket_log2, bucket_log2[g]);
+    v.max_graph_nodes = std::max(v.max_graph_nodes, gr->h_node_off[g + 1] - gr->h_node_off[g]);
+  }
   v.gsize = gr->gsize;
   v.pair_off = gr->pair_off;
   CK(build_long_rows(gr, v, s));
@@ -1827,8 +1838,17 @@ static cudaError_t enqueue_step(mars_dgi* m, const mars_graph* gr, cudaStream_t 
   if (!mat) {
     // a4: corruption permutation (the X~ gather is fused into layer 1's SpMM);
     // a row-sharded graph permutes the whole graph on every shard
-    RET(launch_perm(gr->perm_view(), m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
-    RET(launch_colperm(g, w.perm, w.colperm, s, nl));
+    cudaError_t pe = cudaErrorNotSupported;
+    if (MARS_PERM_GRAPH && !shard && !gr->sharded)
+      pe = launch_perm_graph(g, m->cfg.seed, m->d_sp, w.pw, w.perm,
+                             MARS_PERM_GRAPH_COLPERM ? w.colperm : nullptr, s, nl);
+    if (pe == cudaErrorNotSupported) {
+      RET(launch_perm(gr->perm_view(), m->cfg.seed, m->d_sp, w.pw, w.perm, s, nl));
+      RET(launch_colperm(g, w.perm, w.colperm, s, nl));
+    } else {
+      RET(pe);
+      if (!MARS_PERM_GRAPH_COLPERM) RET(launch_colperm(g, w.perm, w.colperm, s, nl));
+    }
   } else {
     // K samples (c34): sample k of graph g is pair pair_off[g] K + k; the
     // corrupted layer-1 inputs are materialised block by block (c35)
