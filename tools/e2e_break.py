@@ -19,9 +19,11 @@ class P:
     pass
 
 
+WL = os.environ.get("MARS_AB_WORKLOAD", "gnmt")
+NG = 8 if WL == "bert" else 16
 gs = []
-for i in range(16):
-    g = SG.cached("gnmt", i)
+for i in range(NG):
+    g = SG.cached(WL, i)
     p = P()
     p.num_nodes = g.num_nodes
     p.indptr = torch.from_numpy(np.ascontiguousarray(g.indptr)).pin_memory().numpy()
@@ -29,12 +31,12 @@ for i in range(16):
     p.features = torch.from_numpy(np.ascontiguousarray(g.features)).pin_memory().numpy()
     gs.append(p)
 stream = torch.cuda.Stream()
-m = mars.dgi_create(in_dim=64, hidden_dim=256, seed=0)
+m = mars.dgi_create(in_dim=64, hidden_dim=128 if WL == "inception" else 256, seed=0)
 m.set_stream(stream.cuda_stream)
 ga = mars.graph_load(gs)
 gb = mars.graph_load(gs)
 for k in range(4):
-    m.step(ga if k % 2 == 0 else gb, 100 + k, 0, 16)
+    m.step(ga if k % 2 == 0 else gb, 100 + k, 0, NG)
 torch.cuda.synchronize()
 n = 40
 
@@ -46,7 +48,7 @@ def run(reload, read):
     if reload:
         cur.reload(gs)
     for k in range(n):
-        m.step(cur, 1 + k, 0, 16)
+        m.step(cur, 1 + k, 0, NG)
         if reload and k + 1 < n:
             nxt.reload(gs)
         if read:
