@@ -59,34 +59,65 @@ inline unsigned cdiv(int64_t a, int64_t b) { return (unsigned)((a + b - 1) / b);
 // dW[c][h] = Σ_k part[k][h·CIN + c] in fp64.  Block = 32 consecutive outputs ×
 // 8 k-groups (group j sums k = j, j+8, ...), the 8 group sums combined in order
 // j = 0..7; grid = ceil(H·CIN / 32) blocks of 256 threads.
+// kDwRedVec consecutive outputs per lane (16-byte loads: n = H * CIN is a
+// multiple of 4); per output the same fixed order as one output per lane.
+#ifndef MARS_DWRED_VEC
+#define MARS_DWRED_VEC 4
+#endif
+constexpr int kDwRedVec = MARS_DWRED_VEC;
+inline unsigned dw_reduce_blocks(int64_t n) { return (unsigned)((n + 32 * kDwRedVec - 1) / (32 * kDwRedVec)); }
 __device__ __forceinline__ void dw_reduce_body(const float* __restrict__ part, int nchunk, int CIN,
                                                int H, float* __restrict__ dW) {
-  __shared__ double sh[8][32];
+  constexpr int VV = kDwRedVec;
+  __shared__ double sh[8][32 * VV];
   const int lane = threadIdx.x & 31, j = threadIdx.x >> 5;
   const int64_t n = (int64_t)H * CIN;
-  const int64_t e = (int64_t)blockIdx.x * 32 + lane;     // e = h * CIN + c
-  double t = 0.0;
+  const int64_t e = ((int64_t)blockIdx.x * 32 + lane) * VV;   // e = h * CIN + c, VV consecutive
+  double t[VV];
+#pragma unroll
+  for (int v = 0; v < VV; ++v) t[v] = 0.0;
+  auto ld = [&](int k, float (&a)[VV]) {
+    if constexpr (VV == 4) {
+      const float4 x = *reinterpret_cast<const float4*>(part + (int64_t)k * n + e);
+      a[0] = x.x; a[1] = x.y; a[2] = x.z; a[3] = x.w;
+    } else {
+#pragma unroll
+      for (int v = 0; v < VV; ++v) a[v] = part[(int64_t)k * n + e + v];
+    }
+  };
   if (e < n) {
-    // loads issued four at a time, summed in the fixed order k = j, j+8, ...
+    // loads issued four chunks at a time, summed in the fixed order k = j, j+8, ...
     int k = j;
     for (; k + 24 < nchunk; k += 32) {
-      const float a0 = part[(int64_t)k * n + e], a1 = part[(int64_t)(k + 8) * n + e];
-      const float a2 = part[(int64_t)(k + 16) * n + e], a3 = part[(int64_t)(k + 24) * n + e];
-      t += (double)a0;
-      t += (double)a1;
-      t += (double)a2;
-      t += (double)a3;
+      float a0[VV], a1[VV], a2[VV], a3[VV];
+      ld(k, a0); ld(k + 8, a1); ld(k + 16, a2); ld(k + 24, a3);
+#pragma unroll
+      for (int v = 0; v < VV; ++v) {
+        t[v] += (double)a0[v];
+        t[v] += (double)a1[v];
+        t[v] += (double)a2[v];
+        t[v] += (double)a3[v];
+      }
     }
-    for (; k < nchunk; k += 8) t += (double)part[(int64_t)k * n + e];
+    for (; k < nchunk; k += 8) {
+      float a[VV];
+      ld(k, a);
+#pragma unroll
+      for (int v = 0; v < VV; ++v) t[v] += (double)a[v];
+    }
   }
-  sh[j][lane] = t;
+#pragma unroll
+  for (int v = 0; v < VV; ++v) sh[j][lane * VV + v] = t[v];
   __syncthreads();
   if (j == 0 && e < n) {
-    double s = 0.0;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) s += sh[q][lane];
-    const int h = (int)(e / CIN), c = (int)(e % CIN);
-    dW[(int64_t)c * H + h] = (float)s;
+    for (int v = 0; v < VV; ++v) {
+      double s = 0.0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) s += sh[q][lane * VV + v];
+      const int h = (int)((e + v) / CIN), c = (int)((e + v) % CIN);
+      dW[(int64_t)c * H + h] = (float)s;
+    }
   }
 }
 

@@ -454,7 +454,7 @@ cudaError_t tc16_gemm_dw(const void* Y, const void* dZ, float* dW, int64_t R, in
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
-  k_dw16_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
+  k_dw16_reduce<<<dw_reduce_blocks((int64_t)H * CIN), 256, 0, s>>>(part, nchunk, CIN, H, dW);
   return cudaGetLastError();
 }
 

@@ -1475,7 +1475,7 @@ cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, con
     nchunk = (int)((R + rows - 1) / rows);
     e = dw3h_pair(Y, rs_y, dZ, rs_dz, part, nchunk, R, rows, s);
     if (e != cudaSuccess) return e;
-    k_dw3h_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
+    k_dw3h_reduce<<<dw_reduce_blocks((int64_t)H * CIN), 256, 0, s>>>(part, nchunk, CIN, H, dW);
     return cudaGetLastError();
   }
   // H in {32, 64} runs the H = 128 tiles and C_in in {16, 32} the 64-column
@@ -1491,7 +1491,7 @@ cudaError_t tc3h_gemm_dw(const float* Y, const float* rs_y, const float* dZ, con
     default: return cudaErrorInvalidValue;
   }
   if (e != cudaSuccess) return e;
-  k_dw3h_reduce<<<cdiv((int64_t)H * CIN, 32), 256, 0, s>>>(part, nchunk, CIN, H, dW);
+  k_dw3h_reduce<<<dw_reduce_blocks((int64_t)H * CIN), 256, 0, s>>>(part, nchunk, CIN, H, dW);
   return cudaGetLastError();
 }
 
